@@ -1,0 +1,159 @@
+/*
+ * neo.h -- C-ABI of the B200-native CKKS Hybrid key-switching library (libneo.so).
+ *
+ * The operations follow the problem statement of "Neo: Towards Efficient Fully
+ * Homomorphic Encryption Acceleration using Tensor Core" (ISCA'25); citations are
+ * /root/reference/PAPER.md lines (L<n>) and the readings Z1-Z23 of SURVEY.md §8(c),
+ * restated in DESIGN.md.
+ *
+ * Conventions (all entry points):
+ *  - Residues are uint64 in [0, m) for the limb's modulus m (canonical).  Inputs that
+ *    are not canonical give unspecified (but memory-safe) outputs.
+ *  - Limb ids index the concatenated basis q_0..q_{num_q-1}, p_0..p_{num_p-1}.
+ *  - Polynomials are laid out [batch][limb][N] with the limb contiguous (D1, L280, L355).
+ *    Ciphertexts are [batch][2][level+1][N], NTT form, natural order (Z6).
+ *  - Tensor arguments are CUDA DEVICE pointers owned by the caller; the library never
+ *    frees them.  Host arrays (limb id lists, prime lists) are read before return.
+ *    Device buffers must be 16-byte aligned.
+ *  - `stream` is a cudaStream_t (NULL = legacy default stream).  Every compute call is
+ *    asynchronous on it: no host synchronisation and no device allocation inside the
+ *    hot-path calls (ntt, intt, bconv, tensor, automorphism, keyswitch, hmult, hrot,
+ *    rescale).  create/destroy calls may synchronise and allocate.
+ *  - No aliasing between inputs and outputs except where an entry point says "in place".
+ *  - Errors: arguments are validated before any launch; a non-OK status is returned and
+ *    a thread-local message is available from neo_last_error().  Launch failures return
+ *    NEO_ECUDA.  Nothing aborts or throws across the ABI.
+ *  - A context is immutable after creation and may be shared by threads.
+ */
+#ifndef NEO_H
+#define NEO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct neo_ctx neo_ctx;   /* parameters + device constant tables */
+typedef struct neo_evk neo_evk;   /* a device-resident evaluation (key-switching) key */
+typedef void* neo_stream_t;       /* cudaStream_t */
+
+typedef enum {
+    NEO_OK = 0,
+    NEO_EINVAL = 1,        /* bad argument (null pointer, level out of range, batch <= 0, ...) */
+    NEO_EUNSUPPORTED = 2,  /* valid request outside what this build implements (e.g. log_n) */
+    NEO_ENOMEM = 3,        /* device/host allocation failed in a create call */
+    NEO_ECUDA = 4,         /* a CUDA call or kernel launch failed */
+    NEO_ENCCL = 5,         /* reserved for the limb-sharded path */
+    NEO_ENOPRIME = 6       /* not enough word_bits-bit primes p = 1 mod 2N */
+} neo_status;
+
+/* Operation codes for neo_workspace_size. */
+enum { NEO_OP_KEYSWITCH = 0, NEO_OP_HMULT = 1, NEO_OP_HROT = 2, NEO_OP_RESCALE = 3 };
+
+/* Parameter description (Table 1, Table 4).
+ *  log_n      : log2 N; this build supports 12 and 16 (N = 2^12 tiny config, 2^16 Set-B).
+ *  num_q      : number of Q limbs (L+1; Set-B: 36, Z2).
+ *  num_p      : number of special limbs (K+1; Set-B: 12, Z3).
+ *  dnum       : digits; alpha = ceil(num_q/dnum) (L98); ceil(num_q/alpha) must equal dnum.
+ *  word_bits  : prime bit width; this build supports 36 (WordSize of Set-B, L510).
+ *  device     : CUDA device ordinal the tables live on.
+ *  q, p       : optional explicit primes (host arrays of num_q / num_p entries, each
+ *               = 1 mod 2N, word_bits wide); NULL selects rule Z4: k*2N+1 for k from
+ *               floor((2^W-1)/2N) downward, prime, first num_q are q, next num_p are p.
+ * psi is always the minimal primitive 2N-th root of each prime (Z5). */
+typedef struct {
+    int32_t log_n, num_q, num_p, dnum, word_bits, device;
+    const uint64_t* q;
+    const uint64_t* p;
+} neo_params_desc;
+
+/* Build the context: primes, psi, NTT twiddle tables, BConv tables for every
+ * (level, digit) of ModUp and every level of ModDown, P^-1 and q_l^-1 tables. */
+neo_status neo_params_create(const neo_params_desc* desc, neo_ctx** out);
+neo_status neo_params_destroy(neo_ctx* ctx);
+
+/* Copy the moduli and psi to host arrays (any may be NULL): q[num_q], p[num_p],
+ * psi[num_q+num_p] (psi indexed by limb id). */
+neo_status neo_params_query(const neo_ctx* ctx, uint64_t* q, uint64_t* p, uint64_t* psi);
+
+/* Bytes of device workspace `ws` the caller must pass to op (NEO_OP_*) at this level
+ * and batch; 0 on invalid arguments. */
+size_t neo_workspace_size(const neo_ctx* ctx, int32_t op, int32_t level, int32_t batch);
+
+/* Negacyclic NTT, IN PLACE, per limb (L438-450; definition a_hat[i] = a(psi^(2i+1)),
+ * natural order in and out, Z6).  poly is [batch][n_limbs][N]; row k is reduced mod the
+ * prime of limb id limb_ids[k] (host array), 1 <= n_limbs <= 160.  ws is a device scratch
+ * buffer of at least batch*n_limbs*N*8 bytes (the two passes run out of place). */
+neo_status neo_ntt(const neo_ctx* ctx, uint64_t* poly, const int32_t* limb_ids, int32_t n_limbs,
+                   int32_t batch, void* ws, size_t ws_bytes, neo_stream_t stream);
+/* Inverse of neo_ntt (includes the N^-1 scaling), IN PLACE; same arguments. */
+neo_status neo_intt(const neo_ctx* ctx, uint64_t* poly, const int32_t* limb_ids, int32_t n_limbs,
+                    int32_t batch, void* ws, size_t ws_bytes, neo_stream_t stream);
+
+/* Basis conversion, Algorithm 1 (L296-319), non-centred (Z7), coefficient form:
+ *   out[t] = sum_i [in_i * qhat_i^-1]_{q_i} * (qhat_i mod t) mod t,
+ *   qhat_i = prod_{i' != i} q_{i'} over the input limbs.
+ * in [batch][n_in][N] with limb ids in_ids (1 <= n_in <= 16, distinct);
+ * out [batch][n_out][N] with limb ids out_ids (1 <= n_out <= 64). */
+neo_status neo_bconv(const neo_ctx* ctx, const uint64_t* in, const int32_t* in_ids, int32_t n_in,
+                     uint64_t* out, const int32_t* out_ids, int32_t n_out, int32_t batch,
+                     neo_stream_t stream);
+
+/* HMULT tensor product (L132), NTT form: from ct_a, ct_b [batch][2][level+1][N] writes
+ * d [batch][3][level+1][N] with d0 = a0 b0, d1 = a0 b1 + a1 b0, d2 = a1 b1. */
+neo_status neo_tensor(const neo_ctx* ctx, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level,
+                      uint64_t* d, int32_t batch, neo_stream_t stream);
+
+/* Galois automorphism X -> X^g (AUTO, L268-270) in the NTT domain:
+ *   out[i] = in[(g*i + (g-1)/2) mod N]   per limb; in/out [batch][n_limbs][N].
+ * galois_elt must be odd and < 2N. */
+neo_status neo_automorphism(const neo_ctx* ctx, const uint64_t* in, int32_t n_limbs,
+                            uint32_t galois_elt, uint64_t* out, int32_t batch, neo_stream_t stream);
+
+/* Evaluation key (L184; gadget Z8): evk is a DEVICE array [dnum][2][num_q+num_p][N] in NTT
+ * form, evk[j][0] = b_j, evk[j][1] = a_j.  The library copies it (it may be freed after
+ * return).  Synchronises the current device. */
+neo_status neo_evk_create(const neo_ctx* ctx, const uint64_t* evk, neo_evk** out);
+neo_status neo_evk_destroy(neo_evk* evk);
+
+/* Hybrid key-switch (Table 2, Eq. 2, Fig. 5) at `level`:
+ *   INTT -> ModUp BConv (per digit) -> NTT -> KeyIP -> INTT(P part) -> ModDown BConv
+ *   -> NTT -> (acc - conv) * P^-1.
+ * d [batch][level+1][N] NTT form; out0, out1 [batch][level+1][N] NTT form with
+ * out0 + out1 s ~= d s' for the key's (s, s').  All batch entries use the same key (Z21).
+ * ws: device workspace of at least neo_workspace_size(ctx, NEO_OP_KEYSWITCH, level, batch). */
+neo_status neo_keyswitch(const neo_ctx* ctx, const neo_evk* evk, const uint64_t* d, int32_t level,
+                         uint64_t* out0, uint64_t* out1, int32_t batch, void* ws, size_t ws_bytes,
+                         neo_stream_t stream);
+
+/* HMULT (L132) = tensor + relinearise (KS of d2 with the relinearisation key) + add to
+ * (d0, d1).  No rescale (Z22).  ct_a, ct_b, ct_out: [batch][2][level+1][N]. */
+neo_status neo_hmult(const neo_ctx* ctx, const neo_evk* relin, const uint64_t* ct_a,
+                     const uint64_t* ct_b, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
+                     size_t ws_bytes, neo_stream_t stream);
+
+/* HROTATE (L136): (sigma_g(c0) + k0, k1) with (k0, k1) = KS(sigma_g(c1)) under rotkey
+ * = KSGen(s, sigma_g(s)) (L184).  galois_elt = 5^r mod 2N rotates slots left by r (Z11). */
+neo_status neo_hrot(const neo_ctx* ctx, const neo_evk* rotkey, uint32_t galois_elt,
+                    const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
+                    size_t ws_bytes, neo_stream_t stream);
+
+/* Rescale (L137), floor reading (Z10): ct_in [batch][2][level+1][N] -> ct_out
+ * [batch][2][level][N], c'_i = (c_i - NTT_i([INTT_l(c_l)] mod q_i)) * q_l^-1 mod q_i.
+ * level >= 1. */
+neo_status neo_rescale(const neo_ctx* ctx, const uint64_t* ct_in, int32_t level, uint64_t* ct_out,
+                       int32_t batch, void* ws, size_t ws_bytes, neo_stream_t stream);
+
+/* Thread-local message describing the last non-OK status returned on this thread. */
+const char* neo_last_error(void);
+
+/* Number of kernels the last hot-path call on this thread launched (for bench.py's
+ * gpu_launches accounting). */
+int32_t neo_last_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NEO_H */

@@ -1,0 +1,520 @@
+// abi.cpp -- the extern "C" entry points of libneo.so (include/neo.h) and the key-switch
+// orchestrator (Fig. 5: INTT -> ModUp -> NTT -> KeyIP -> INTT -> ModDown -> NTT).
+#include <algorithm>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "context.h"
+#include "kernels.h"
+#include "ntt.h"
+
+namespace neo {
+neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err);
+}
+using namespace neo;
+
+static thread_local std::string g_err;
+static thread_local int g_launches = 0;
+
+#define FAIL(code, msg)      \
+    do {                     \
+        g_err = (msg);       \
+        return (code);       \
+    } while (0)
+#define CK(x)                                                               \
+    do {                                                                    \
+        cudaError_t e_ = (x);                                               \
+        if (e_ != cudaSuccess) {                                            \
+            g_err = std::string("CUDA error: ") + cudaGetErrorString(e_);   \
+            return NEO_ECUDA;                                               \
+        }                                                                   \
+    } while (0)
+
+static inline cudaStream_t S(neo_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
+
+// ------------------------------------------------------------------ NTT over a row set
+// rows k < n of batch entry b: src + b*src_bs + src_off[k]*N  ->  dst + b*dst_bs + dst_off[k]*N
+static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long src_bs, const int* src_off,
+                           u64* dst, long long dst_bs, const int* dst_off, const int* prime, int n, u64* tmp,
+                           int batch, cudaStream_t st) {
+    if (n <= 0) return NEO_OK;
+    if (n > NEO_MAX_ROWS) FAIL(NEO_EUNSUPPORTED, "too many limb rows in one transform");
+    RowSet a, b;
+    const long long N = c->N;
+    a.n = b.n = n;
+    // first pass: src -> tmp ; second pass: tmp -> dst
+    a.src = src; a.src_bstride = src_bs;
+    a.dst = tmp; a.dst_bstride = (long long)n * N;
+    b.src = tmp; b.src_bstride = (long long)n * N;
+    b.dst = dst; b.dst_bstride = dst_bs;
+    for (int k = 0; k < n; ++k) {
+        a.src_off[k] = src_off[k]; a.dst_off[k] = k; a.prime[k] = (short)prime[k];
+        b.src_off[k] = k; b.dst_off[k] = dst_off[k]; b.prime[k] = (short)prime[k];
+    }
+    // forward: column pass then row pass; inverse: row pass then column pass
+    CK(ntt_pass(fwd, a, c->ntt, batch, fwd, st));
+    CK(ntt_pass(!fwd, b, c->ntt, batch, fwd, st));
+    g_launches += 2;
+    return NEO_OK;
+}
+
+// ------------------------------------------------------------------ workspace layout
+struct KsLayout {
+    size_t y, up, acc, conv, pc, tmp, extra, total;   // u64 offsets
+};
+
+static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
+    const size_t N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p;
+    KsLayout L;
+    size_t o = 0;
+    L.y = o; o += B * Lq * N;
+    L.up = o; o += B * beta * E * N;
+    L.acc = o; o += B * 2 * E * N;
+    L.conv = o; o += B * 2 * Lq * N;
+    L.pc = o; o += B * 2 * P * N;
+    L.tmp = o; o += B * std::max(std::max(beta * E, 2 * Lq), 2 * P) * N;
+    L.extra = o;
+    if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
+    if (op == NEO_OP_HROT) o += B * 2 * Lq * N;
+    L.total = o;
+    return L;
+}
+
+static size_t rescale_ws(const neo_ctx* c, int l, int B) {
+    const size_t N = c->N;
+    return (size_t)2 * B * N + (size_t)2 * B * l * N + (size_t)2 * B * std::max(l, 1) * N;
+}
+
+// ------------------------------------------------------------------ key-switch core
+static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
+                          u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
+                          const u64* add0, const u64* add1, long long add_bs, cudaStream_t st) {
+    const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p;
+    u64 *y = ws + Ly.y, *up = ws + Ly.up, *acc = ws + Ly.acc, *conv = ws + Ly.conv, *pc = ws + Ly.pc,
+        *tmp = ws + Ly.tmp;
+    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    neo_status s;
+
+    // a3: INTT of d (l+1 limbs) -> y (coefficient form)
+    for (int i = 0; i < Lq; ++i) { so[i] = i; dof[i] = i; pr[i] = i; }
+    if ((s = ntt_rows(c, false, d, d_bs, so, y, (long long)Lq * N, dof, pr, Lq, tmp, B, st))) return s;
+
+    // a4: ModUp BConv, one launch per digit: y[D_j] -> up[j][targets]
+    for (int j = 0; j < beta; ++j) {
+        const BConvTab& T = c->modup[l][j];
+        const std::vector<int>& dj = c->digits[l][j];
+        BConvIO io;
+        io.in = y; io.out = up;
+        io.in_bstride = (long long)Lq * N;
+        io.out_bstride = (long long)beta * E * N;
+        for (int i = 0; i < T.n_in; ++i) io.in_off[i] = dj[i];
+        int o = 0;
+        for (int pos = 0; pos < E; ++pos) {
+            int id = c->ext_id(l, pos);
+            if (std::find(dj.begin(), dj.end(), id) != dj.end()) continue;
+            io.out_off[o++] = j * E + pos;
+        }
+        CK(launch_bconv(T, io, N, B, st));
+        ++g_launches;
+    }
+
+    // a5: NTT of every ModUp output row
+    int n = 0;
+    for (int j = 0; j < beta; ++j) {
+        const std::vector<int>& dj = c->digits[l][j];
+        for (int pos = 0; pos < E; ++pos) {
+            int id = c->ext_id(l, pos);
+            if (std::find(dj.begin(), dj.end(), id) != dj.end()) continue;
+            so[n] = dof[n] = j * E + pos;
+            pr[n] = id;
+            ++n;
+        }
+    }
+    if ((s = ntt_rows(c, true, up, (long long)beta * E * N, so, up, (long long)beta * E * N, dof, pr, n, tmp, B, st)))
+        return s;
+
+    // a6: KeyIP over all E limbs of PQ_l
+    {
+        KeyIPArgs A;
+        A.d = d; A.up = up; A.evk = k->d; A.acc = acc; A.mods = c->d_mods;
+        A.d_bstride = d_bs;
+        A.up_bstride = (long long)beta * E * N;
+        A.acc_bstride = (long long)2 * E * N;
+        A.acc_cstride = (long long)E * N;
+        A.N = N; A.beta = beta; A.evk_limbs = c->num_q + c->num_p;
+        for (int pos = 0; pos < E; ++pos) {
+            int id = c->ext_id(l, pos);
+            A.limb[pos] = id;
+            for (int j = 0; j < beta; ++j) {
+                const std::vector<int>& dj = c->digits[l][j];
+                bool own = std::find(dj.begin(), dj.end(), id) != dj.end();
+                A.src_kind[j][pos] = own ? 0 : 1;
+                A.src_off[j][pos] = own ? id : j * E + pos;
+            }
+        }
+        CK(launch_keyip(A, E, B, st));
+        ++g_launches;
+    }
+
+    // a7: INTT of the P part of acc_0, acc_1 -> pc [2B][P][N]
+    for (int k2 = 0; k2 < P; ++k2) { so[k2] = Lq + k2; dof[k2] = k2; pr[k2] = c->num_q + k2; }
+    if ((s = ntt_rows(c, false, acc, (long long)E * N, so, pc, (long long)P * N, dof, pr, P, tmp, 2 * B, st)))
+        return s;
+
+    // a8: ModDown BConv P -> q_0..q_l, batch 2B
+    {
+        const BConvTab& T = c->moddown[l];
+        BConvIO io;
+        io.in = pc; io.out = conv;
+        io.in_bstride = (long long)P * N;
+        io.out_bstride = (long long)Lq * N;
+        for (int i = 0; i < P; ++i) io.in_off[i] = i;
+        for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
+        CK(launch_bconv(T, io, N, 2 * B, st));
+        ++g_launches;
+    }
+
+    // a9: NTT of conv (in place through tmp)
+    for (int i = 0; i < Lq; ++i) { so[i] = dof[i] = i; pr[i] = i; }
+    if ((s = ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st)))
+        return s;
+
+    // a10: combine
+    {
+        CombineArgs A;
+        A.acc = acc; A.conv = conv; A.add0 = add0; A.add1 = add1; A.out0 = out0; A.out1 = out1;
+        A.mods = c->d_mods;
+        A.acc_bstride = (long long)2 * E * N;
+        A.acc_cstride = (long long)E * N;
+        A.conv_stride = (long long)Lq * N;
+        A.add_bstride = add_bs;
+        A.out_bstride = out_bs;
+        A.N = N;
+        for (int i = 0; i < Lq; ++i) A.pinv[i] = c->pinv[i];
+        CK(launch_combine(A, Lq, B, st));
+        ++g_launches;
+    }
+    return NEO_OK;
+}
+
+// ------------------------------------------------------------------ validation helpers
+static neo_status check_ctx(const neo_ctx* c) {
+    if (!c) FAIL(NEO_EINVAL, "null context");
+    return NEO_OK;
+}
+static neo_status check_level(const neo_ctx* c, int level, int batch) {
+    if (level < 0 || level >= c->num_q) FAIL(NEO_EINVAL, "level out of range");
+    if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
+    return NEO_OK;
+}
+static neo_status check_ws(const neo_ctx* c, int op, int level, int batch, const void* ws, size_t bytes) {
+    size_t need = neo_workspace_size(c, op, level, batch);
+    if (!ws || bytes < need) FAIL(NEO_EINVAL, "workspace missing or too small (see neo_workspace_size)");
+    if (reinterpret_cast<uintptr_t>(ws) % 16) FAIL(NEO_EINVAL, "workspace must be 16-byte aligned");
+    return NEO_OK;
+}
+static neo_status check_ptr(const void* p, const char* what) {
+    if (!p) FAIL(NEO_EINVAL, std::string("null pointer: ") + what);
+    if (reinterpret_cast<uintptr_t>(p) % 16) FAIL(NEO_EINVAL, std::string("pointer not 16-byte aligned: ") + what);
+    return NEO_OK;
+}
+#define TRY(x)                      \
+    do {                            \
+        neo_status s_ = (x);        \
+        if (s_ != NEO_OK) return s_; \
+    } while (0)
+
+// ------------------------------------------------------------------ C ABI
+extern "C" {
+
+const char* neo_last_error(void) { return g_err.c_str(); }
+int32_t neo_last_launch_count(void) { return g_launches; }
+
+neo_status neo_params_create(const neo_params_desc* desc, neo_ctx** out) {
+    if (!desc || !out) FAIL(NEO_EINVAL, "null argument");
+    *out = nullptr;
+    if (desc->log_n != 12 && desc->log_n != 16) FAIL(NEO_EUNSUPPORTED, "log_n must be 12 or 16 in this build");
+    if (desc->word_bits != 36) FAIL(NEO_EUNSUPPORTED, "word_bits must be 36 in this build");
+    if (desc->num_q < 1 || desc->num_p < 1 || desc->dnum < 1 || desc->dnum > desc->num_q)
+        FAIL(NEO_EINVAL, "need num_q >= 1, num_p >= 1, 1 <= dnum <= num_q");
+    if (desc->num_q + desc->num_p > KS_MAX_EXT) FAIL(NEO_EUNSUPPORTED, "num_q + num_p must be <= 64");
+    if (desc->num_p > BC_MAX_IN) FAIL(NEO_EUNSUPPORTED, "num_p must be <= 16");
+    int alpha = (desc->num_q + desc->dnum - 1) / desc->dnum;
+    if ((desc->num_q + alpha - 1) / alpha != desc->dnum) FAIL(NEO_EINVAL, "every digit must be non-empty");
+    if (alpha > BC_MAX_IN) FAIL(NEO_EUNSUPPORTED, "alpha must be <= 16");
+    if (desc->dnum > KS_MAX_BETA) FAIL(NEO_EUNSUPPORTED, "dnum must be <= 8");
+    if ((desc->q == nullptr) != (desc->p == nullptr)) FAIL(NEO_EINVAL, "give both q and p or neither");
+    neo_ctx* c = new (std::nothrow) neo_ctx();
+    if (!c) FAIL(NEO_ENOMEM, "host allocation failed");
+    std::string err;
+    neo_status s;
+    try {
+        s = build_context(c, desc, err);
+    } catch (...) {
+        s = NEO_ENOMEM;
+        err = "exception while building the context";
+    }
+    if (s != NEO_OK) {
+        neo_params_destroy(c);
+        FAIL(s, err);
+    }
+    *out = c;
+    return NEO_OK;
+}
+
+neo_status neo_params_destroy(neo_ctx* c) {
+    if (!c) return NEO_OK;
+    if (c->d_tab) cudaFree(c->d_tab);
+    if (c->d_mods) cudaFree(c->d_mods);
+    delete c;
+    return NEO_OK;
+}
+
+neo_status neo_params_query(const neo_ctx* c, uint64_t* q, uint64_t* p, uint64_t* psi) {
+    TRY(check_ctx(c));
+    if (q) std::copy(c->mod.begin(), c->mod.begin() + c->num_q, q);
+    if (p) std::copy(c->mod.begin() + c->num_q, c->mod.end(), p);
+    if (psi) std::copy(c->psi.begin(), c->psi.end(), psi);
+    return NEO_OK;
+}
+
+size_t neo_workspace_size(const neo_ctx* c, int32_t op, int32_t level, int32_t batch) {
+    if (!c || batch <= 0 || level < 0 || level >= c->num_q) return 0;
+    switch (op) {
+        case NEO_OP_KEYSWITCH:
+        case NEO_OP_HMULT:
+        case NEO_OP_HROT: return ks_layout(c, level, batch, op).total * sizeof(u64);
+        case NEO_OP_RESCALE: return level >= 1 ? rescale_ws(c, level, batch) * sizeof(u64) : 0;
+        default: return 0;
+    }
+}
+
+static neo_status ntt_api(const neo_ctx* c, bool fwd, uint64_t* poly, const int32_t* ids, int32_t n, int32_t batch,
+                          void* ws, size_t ws_bytes, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_ptr(poly, "poly"));
+    if (!ids || n <= 0 || n > NEO_MAX_ROWS) FAIL(NEO_EINVAL, "need 1 <= n_limbs <= 160 limb ids");
+    if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
+    for (int k = 0; k < n; ++k)
+        if (ids[k] < 0 || ids[k] >= c->num_q + c->num_p) FAIL(NEO_EINVAL, "unknown limb id");
+    size_t need = (size_t)batch * n * c->N * sizeof(u64);
+    if (!ws || ws_bytes < need) FAIL(NEO_EINVAL, "ntt workspace must hold batch*n_limbs*N words");
+    int off[NEO_MAX_ROWS];
+    for (int k = 0; k < n; ++k) off[k] = k;
+    long long bs = (long long)n * c->N;
+    return ntt_rows(c, fwd, poly, bs, off, poly, bs, off, ids, n, static_cast<u64*>(ws), batch, S(st));
+}
+
+neo_status neo_ntt(const neo_ctx* c, uint64_t* poly, const int32_t* ids, int32_t n, int32_t batch, void* ws,
+                      size_t ws_bytes, neo_stream_t st) {
+    return ntt_api(c, true, poly, ids, n, batch, ws, ws_bytes, st);
+}
+neo_status neo_intt(const neo_ctx* c, uint64_t* poly, const int32_t* ids, int32_t n, int32_t batch, void* ws,
+                       size_t ws_bytes, neo_stream_t st) {
+    return ntt_api(c, false, poly, ids, n, batch, ws, ws_bytes, st);
+}
+
+neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids, int32_t n_in, uint64_t* out,
+                     const int32_t* out_ids, int32_t n_out, int32_t batch, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_ptr(in, "in"));
+    TRY(check_ptr(out, "out"));
+    if (!in_ids || !out_ids || n_in < 1 || n_in > BC_MAX_IN || n_out < 1 || n_out > BC_MAX_OUT)
+        FAIL(NEO_EINVAL, "need 1 <= n_in <= 16 and 1 <= n_out <= 64");
+    if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
+    const int nl = c->num_q + c->num_p;
+    for (int i = 0; i < n_in; ++i) {
+        if (in_ids[i] < 0 || in_ids[i] >= nl) FAIL(NEO_EINVAL, "unknown input limb id");
+        for (int k = 0; k < i; ++k)
+            if (in_ids[k] == in_ids[i]) FAIL(NEO_EINVAL, "input limb ids must be distinct");
+    }
+    for (int j = 0; j < n_out; ++j)
+        if (out_ids[j] < 0 || out_ids[j] >= nl) FAIL(NEO_EINVAL, "unknown output limb id");
+    // constants of Algorithm 1 for this (in, out) pair, passed by value (no allocation)
+    BConvTab T;
+    std::memset(&T, 0, sizeof(T));
+    T.n_in = n_in;
+    T.n_out = n_out;
+    auto mulm = [](u64 a, u64 b, u64 m) { return (u64)((u128)a * b % m); };
+    auto powm = [&](u64 a, u64 e, u64 m) {
+        u64 r = 1;
+        for (a %= m; e; e >>= 1, a = mulm(a, a, m))
+            if (e & 1) r = mulm(r, a, m);
+        return r;
+    };
+    for (int i = 0; i < n_in; ++i) {
+        u64 qi = c->mod[in_ids[i]], qh = 1;
+        for (int k = 0; k < n_in; ++k)
+            if (k != i) qh = mulm(qh, c->mod[in_ids[k]] % qi, qi);
+        u64 inv = powm(qh, qi - 2, qi);
+        T.qin[i] = qi;
+        T.qhat_inv[i] = TW{inv, (u64)(((u128)inv << 64) / qi)};
+    }
+    for (int j = 0; j < n_out; ++j) {
+        u64 t = c->mod[out_ids[j]];
+        T.tmod[j] = ModQ{t, (u64)(((u128)1 << 98) / t)};
+        for (int i = 0; i < n_in; ++i) {
+            u64 f = 1;
+            for (int k = 0; k < n_in; ++k)
+                if (k != i) f = mulm(f, c->mod[in_ids[k]] % t, t);
+            T.f_lo[i][j] = (unsigned)(f & 0x3FFFF);
+            T.f_hi[i][j] = (unsigned)(f >> 18);
+        }
+    }
+    BConvIO io;
+    io.in = in; io.out = out;
+    io.in_bstride = (long long)n_in * c->N;
+    io.out_bstride = (long long)n_out * c->N;
+    for (int i = 0; i < n_in; ++i) io.in_off[i] = i;
+    for (int j = 0; j < n_out; ++j) io.out_off[j] = j;
+    CK(launch_bconv(T, io, c->N, batch, S(st)));
+    g_launches = 1;
+    return NEO_OK;
+}
+
+neo_status neo_tensor(const neo_ctx* c, const uint64_t* a, const uint64_t* b, int32_t level, uint64_t* d,
+                      int32_t batch, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(a, "ct_a"));
+    TRY(check_ptr(b, "ct_b"));
+    TRY(check_ptr(d, "d"));
+    CK(launch_tensor(a, b, d, c->d_mods, level + 1, c->N, batch, S(st)));
+    g_launches = 1;
+    return NEO_OK;
+}
+
+neo_status neo_automorphism(const neo_ctx* c, const uint64_t* in, int32_t n_limbs, uint32_t g, uint64_t* out,
+                            int32_t batch, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_ptr(in, "in"));
+    TRY(check_ptr(out, "out"));
+    if (n_limbs <= 0 || batch <= 0) FAIL(NEO_EINVAL, "n_limbs and batch must be positive");
+    if ((g & 1) == 0 || g >= 2u * (unsigned)c->N) FAIL(NEO_EINVAL, "galois element must be odd and < 2N");
+    CK(launch_automorph(in, out, g, c->N, n_limbs * batch, S(st)));
+    g_launches = 1;
+    return NEO_OK;
+}
+
+neo_status neo_evk_create(const neo_ctx* c, const uint64_t* evk, neo_evk** out) {
+    TRY(check_ctx(c));
+    if (!evk || !out) FAIL(NEO_EINVAL, "null argument");
+    *out = nullptr;
+    neo_evk* k = new (std::nothrow) neo_evk();
+    if (!k) FAIL(NEO_ENOMEM, "host allocation failed");
+    k->ctx = c;
+    size_t bytes = (size_t)c->dnum * 2 * (c->num_q + c->num_p) * c->N * sizeof(u64);
+    if (cudaMalloc(&k->d, bytes) != cudaSuccess) {
+        delete k;
+        FAIL(NEO_ENOMEM, "cudaMalloc of the evaluation key failed");
+    }
+    cudaError_t e = cudaMemcpy(k->d, evk, bytes, cudaMemcpyDeviceToDevice);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) {
+        cudaFree(k->d);
+        delete k;
+        FAIL(NEO_ECUDA, std::string("evk copy failed: ") + cudaGetErrorString(e));
+    }
+    *out = k;
+    return NEO_OK;
+}
+
+neo_status neo_evk_destroy(neo_evk* k) {
+    if (!k) return NEO_OK;
+    if (k->d) cudaFree(k->d);
+    delete k;
+    return NEO_OK;
+}
+
+neo_status neo_keyswitch(const neo_ctx* c, const neo_evk* k, const uint64_t* d, int32_t level, uint64_t* out0,
+                         uint64_t* out1, int32_t batch, void* ws, size_t ws_bytes, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    if (!k || k->ctx != c) FAIL(NEO_EINVAL, "evaluation key missing or from another context");
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(d, "d"));
+    TRY(check_ptr(out0, "out0"));
+    TRY(check_ptr(out1, "out1"));
+    TRY(check_ws(c, NEO_OP_KEYSWITCH, level, batch, ws, ws_bytes));
+    KsLayout Ly = ks_layout(c, level, batch, NEO_OP_KEYSWITCH);
+    const long long ls = (long long)(level + 1) * c->N;
+    return ks_core(c, k, d, ls, level, batch, static_cast<u64*>(ws), Ly, out0, out1, ls, nullptr, nullptr, 0, S(st));
+}
+
+neo_status neo_hmult(const neo_ctx* c, const neo_evk* relin, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level,
+                     uint64_t* ct_out, int32_t batch, void* ws, size_t ws_bytes, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    if (!relin || relin->ctx != c) FAIL(NEO_EINVAL, "relinearisation key missing or from another context");
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(ct_a, "ct_a"));
+    TRY(check_ptr(ct_b, "ct_b"));
+    TRY(check_ptr(ct_out, "ct_out"));
+    TRY(check_ws(c, NEO_OP_HMULT, level, batch, ws, ws_bytes));
+    KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HMULT);
+    u64* w = static_cast<u64*>(ws);
+    u64* dd = w + Ly.extra;
+    const long long ls = (long long)(level + 1) * c->N;
+    cudaStream_t s = S(st);
+    CK(launch_tensor(ct_a, ct_b, dd, c->d_mods, level + 1, c->N, batch, s));
+    g_launches = 1;
+    return ks_core(c, relin, dd + 2 * ls, 3 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, dd, dd + ls,
+                   3 * ls, s);
+}
+
+neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint64_t* ct_in, int32_t level,
+                    uint64_t* ct_out, int32_t batch, void* ws, size_t ws_bytes, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    if (!rk || rk->ctx != c) FAIL(NEO_EINVAL, "rotation key missing or from another context");
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(ct_in, "ct_in"));
+    TRY(check_ptr(ct_out, "ct_out"));
+    if ((g & 1) == 0 || g >= 2u * (unsigned)c->N) FAIL(NEO_EINVAL, "galois element must be odd and < 2N");
+    TRY(check_ws(c, NEO_OP_HROT, level, batch, ws, ws_bytes));
+    KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HROT);
+    u64* w = static_cast<u64*>(ws);
+    u64* sc = w + Ly.extra;
+    const long long ls = (long long)(level + 1) * c->N;
+    cudaStream_t s = S(st);
+    CK(launch_automorph(ct_in, sc, g, c->N, 2 * (level + 1) * batch, s));
+    g_launches = 1;
+    return ks_core(c, rk, sc + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, sc, nullptr, 2 * ls, s);
+}
+
+neo_status neo_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch,
+                       void* ws, size_t ws_bytes, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level, batch));
+    if (level < 1) FAIL(NEO_EINVAL, "rescale needs level >= 1");
+    TRY(check_ptr(ct_in, "ct_in"));
+    TRY(check_ptr(ct_out, "ct_out"));
+    TRY(check_ws(c, NEO_OP_RESCALE, level, batch, ws, ws_bytes));
+    const int N = c->N, l = level, B2 = 2 * batch;
+    u64* w = static_cast<u64*>(ws);
+    u64* last = w;
+    u64* r = last + (size_t)B2 * N;
+    u64* tmp = r + (size_t)B2 * l * N;
+    cudaStream_t s = S(st);
+    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    so[0] = l; dof[0] = 0; pr[0] = l;
+    TRY(ntt_rows(c, false, ct_in, (long long)(l + 1) * N, so, last, N, dof, pr, 1, tmp, B2, s));
+    CK(launch_modswitch(last, r, c->d_mods, l, N, B2, s));
+    ++g_launches;
+    for (int i = 0; i < l; ++i) { so[i] = dof[i] = i; pr[i] = i; }
+    TRY(ntt_rows(c, true, r, (long long)l * N, so, r, (long long)l * N, dof, pr, l, tmp, B2, s));
+    RescaleArgs A;
+    A.in = ct_in; A.r = r; A.out = ct_out; A.mods = c->d_mods; A.N = N; A.l = l;
+    for (int i = 0; i < l; ++i) A.qlinv[i] = c->ql_inv[l][i];
+    CK(launch_rescale_combine(A, B2, s));
+    ++g_launches;
+    return NEO_OK;
+}
+
+}  // extern "C"

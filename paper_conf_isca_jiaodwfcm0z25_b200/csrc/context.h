@@ -1,0 +1,66 @@
+// context.h -- host-side definition of neo_ctx / neo_evk and of the per-launch constant
+// blocks (passed by value as kernel parameters, so no hot-path H2D copies are needed).
+#pragma once
+#include <string>
+#include <vector>
+
+#include "common.cuh"
+#include "neo.h"
+#include "ntt.h"
+
+namespace neo {
+
+constexpr int BC_MAX_IN = 16;
+constexpr int BC_MAX_OUT = 64;
+
+// Constants of one basis conversion (Algorithm 1) from n_in to n_out limbs:
+//   y_i = [c_i * qhat_i^-1]_{q_i};  out_j = sum_i y_i * (qhat_i mod t_j) mod t_j.
+// f is stored as 18-bit halves so the CUDA-core kernel accumulates with 32x32->64 MADs.
+struct BConvTab {
+    int n_in, n_out;
+    u64 qin[BC_MAX_IN];
+    TW qhat_inv[BC_MAX_IN];
+    ModQ tmod[BC_MAX_OUT];
+    unsigned f_lo[BC_MAX_IN][BC_MAX_OUT];   // (qhat_i mod t_j) & (2^18 - 1)
+    unsigned f_hi[BC_MAX_IN][BC_MAX_OUT];   // (qhat_i mod t_j) >> 18
+};
+
+// Row addressing of a BConv launch: input row i of batch entry b at in + b*in_bstride +
+// in_off[i]*N, output row j at out + b*out_bstride + out_off[j]*N.
+struct BConvIO {
+    const u64* in;
+    u64* out;
+    long long in_bstride, out_bstride;
+    int in_off[BC_MAX_IN];
+    int out_off[BC_MAX_OUT];
+};
+
+}  // namespace neo
+
+struct neo_ctx {
+    int log_n, N, num_q, num_p, dnum, alpha, word_bits, device;
+    std::vector<u64> mod;                 // by limb id
+    std::vector<u64> psi;                 // by limb id
+    std::vector<ModQ> h_mods;
+    NttLayout L;
+    TW* d_tab = nullptr;                  // [limb id][L.total]
+    ModQ* d_mods = nullptr;
+    neo::NttArgs ntt;
+    // per level l (index l = 0..num_q-1)
+    std::vector<std::vector<neo::BConvTab>> modup;   // [l][digit j]
+    std::vector<std::vector<std::vector<int>>> digits;  // [l][j] -> limb ids
+    std::vector<neo::BConvTab> moddown;              // [l]: P limbs -> q_0..q_l
+    std::vector<TW> pinv;                            // [i] P^-1 mod q_i (Shoup)
+    std::vector<std::vector<TW>> ql_inv;             // [l][i] q_l^-1 mod q_i, i < l
+
+    int beta(int level) const { return (level + 1 + alpha - 1) / alpha; }
+    int ext(int level) const { return level + 1 + num_p; }          // limbs of PQ_l
+    int ext_id(int level, int pos) const {                           // position -> limb id
+        return pos <= level ? pos : num_q + (pos - level - 1);
+    }
+};
+
+struct neo_evk {
+    const neo_ctx* ctx;
+    u64* d = nullptr;                     // [dnum][2][num_q+num_p][N]
+};

@@ -1,0 +1,179 @@
+// kernels.cu -- BConv (CUDA-core), KeyIP, combine, tensor, automorphism and rescale helpers.
+#include "context.h"
+#include "kernels.h"
+
+namespace neo {
+
+// ------------------------------------------------------------------ BConv (Algorithm 1)
+// One thread per coefficient: y_i = [c_i qhat_i^-1]_{q_i} (Shoup), then every output
+// out_j = sum_i y_i f_ij mod t_j with y and f split in 18-bit halves so that each MAC is
+// four 32x32->64 IMADs into three 64-bit partial sums (12 inputs: < 2^41 each), followed
+// by one Barrett reduction of the < 2^77 total.  (L296-319.)
+__global__ void __launch_bounds__(256)
+k_bconv(BConvTab T, BConvIO io, int N) {
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int b = blockIdx.y;
+    if (n >= N) return;
+    unsigned ylo[BC_MAX_IN], yhi[BC_MAX_IN];
+    const u64* in = io.in + b * io.in_bstride + n;
+#pragma unroll
+    for (int i = 0; i < BC_MAX_IN; ++i) {
+        if (i < T.n_in) {
+            u64 c = in[(size_t)io.in_off[i] * N];
+            u64 y = shoup(c, T.qhat_inv[i], T.qin[i]);
+            ylo[i] = (unsigned)(y & 0x3FFFF);
+            yhi[i] = (unsigned)(y >> 18);
+        } else {
+            ylo[i] = yhi[i] = 0;
+        }
+    }
+    u64* out = io.out + b * io.out_bstride + n;
+    for (int j = 0; j < T.n_out; ++j) {
+        u64 A = 0, B = 0, C = 0;
+#pragma unroll
+        for (int i = 0; i < BC_MAX_IN; ++i) {
+            if (i < T.n_in) {
+                const unsigned flo = T.f_lo[i][j], fhi = T.f_hi[i][j];
+                A += (u64)ylo[i] * flo;
+                B += (u64)ylo[i] * fhi + (u64)yhi[i] * flo;
+                C += (u64)yhi[i] * fhi;
+            }
+        }
+        u64 t = A + (B << 18);                 // < 2^60
+        u64 lo = t + (C << 36);
+        u64 hi = (C >> 28) + (lo < t);
+        out[(size_t)io.out_off[j] * N] = barrett_reduce(hi, lo, T.tmod[j]);
+    }
+}
+
+// ------------------------------------------------------------------ KeyIP (Alg. 3)
+// acc_c[t] = sum_j dhat_j[t] * evk_{j,c}[t] mod t for c = 0, 1 (L359-382); the evk is
+// read once per launch and shared by the whole batch in L2 (Z21).
+__global__ void __launch_bounds__(256)
+k_keyip(KeyIPArgs A) {
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int t = blockIdx.y, b = blockIdx.z;
+    if (n >= A.N) return;
+    const ModQ m = A.mods[A.limb[t]];
+    u64 h0 = 0, l0 = 0, h1 = 0, l1 = 0;
+    for (int j = 0; j < A.beta; ++j) {
+        const int so = A.src_off[j][t];
+        const u64* src = (A.src_kind[j][t] ? A.up + b * A.up_bstride : A.d + b * A.d_bstride);
+        const u64 x = src[(size_t)so * A.N + n];
+        const u64* e = A.evk + ((size_t)(2 * j) * A.evk_limbs + A.limb[t]) * A.N + n;
+        mac128(h0, l0, x, e[0]);
+        mac128(h1, l1, x, e[(size_t)A.evk_limbs * A.N]);
+    }
+    u64* acc = A.acc + b * A.acc_bstride + (size_t)t * A.N + n;
+    acc[0] = barrett_reduce(h0, l0, m);
+    acc[(size_t)A.acc_cstride] = barrett_reduce(h1, l1, m);
+}
+
+// ------------------------------------------------------------------ combine (ModDown tail)
+// out_c[i] = (acc_c[i] - conv_c[i]) * P^-1 mod q_i  (+ add_c[i]); Fig. 5, Z9.
+__global__ void __launch_bounds__(256)
+k_combine(CombineArgs A) {
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int i = blockIdx.y, bc = blockIdx.z, b = bc >> 1, c = bc & 1;
+    if (n >= A.N) return;
+    const u64 q = A.mods[i].q;
+    const size_t row = (size_t)i * A.N + n;
+    u64 a = A.acc[b * A.acc_bstride + c * A.acc_cstride + row];
+    u64 v = A.conv[(size_t)bc * A.conv_stride + row];
+    u64 r = shoup(sub_mod(a, v, q), A.pinv[i], q);
+    const u64* add = c ? A.add1 : A.add0;
+    if (add) r = add_mod(r, add[b * A.add_bstride + row], q);
+    u64* out = c ? A.out1 : A.out0;
+    out[b * A.out_bstride + row] = r;
+}
+
+// ------------------------------------------------------------------ tensor (HMULT, L132)
+__global__ void __launch_bounds__(256)
+k_tensor(const u64* __restrict__ cta, const u64* __restrict__ ctb, u64* __restrict__ d,
+         const ModQ* __restrict__ mods, int limbs, int N) {
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int i = blockIdx.y, b = blockIdx.z;
+    if (n >= N) return;
+    const ModQ m = mods[i];
+    const size_t cs = (size_t)limbs * N;             // component stride
+    const size_t base = (size_t)b * 2 * cs + (size_t)i * N + n;
+    const u64 a0 = cta[base], a1 = cta[base + cs], b0 = ctb[base], b1 = ctb[base + cs];
+    const size_t ob = (size_t)b * 3 * cs + (size_t)i * N + n;
+    d[ob] = mul_mod(a0, b0, m);
+    u64 h = 0, l = 0;
+    mac128(h, l, a0, b1);
+    mac128(h, l, a1, b0);
+    d[ob + cs] = barrett_reduce(h, l, m);
+    d[ob + 2 * cs] = mul_mod(a1, b1, m);
+}
+
+// ------------------------------------------------------------------ automorphism (AUTO)
+// out[i] = in[(g i + (g-1)/2) mod N]: X -> X^g in the natural-order NTT domain.
+__global__ void __launch_bounds__(256)
+k_automorph(const u64* __restrict__ in, u64* __restrict__ out, unsigned g, int N) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    const size_t row = (size_t)blockIdx.y * N;
+    if (i >= N) return;
+    const unsigned src = (unsigned)(((unsigned long long)g * i + (g - 1) / 2) & (N - 1));
+    out[row + i] = in[row + src];
+}
+
+// ------------------------------------------------------------------ rescale helpers (L137)
+// r[bc][i] = last[bc] mod q_i for i < l  (last < q_l < 2 q_i for equal-width primes)
+__global__ void __launch_bounds__(256)
+k_modswitch(const u64* __restrict__ last, u64* __restrict__ r, const ModQ* __restrict__ mods, int l, int N) {
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int i = blockIdx.y, bc = blockIdx.z;
+    if (n >= N) return;
+    const u64 q = mods[i].q;
+    u64 v = last[(size_t)bc * N + n];
+    v = v >= q ? v - q : v;
+    r[((size_t)bc * l + i) * N + n] = v;
+}
+
+// out[bc][i] = (in[bc][i] - r[bc][i]) * q_l^-1 mod q_i, in has l+1 limbs, out has l.
+__global__ void __launch_bounds__(256)
+k_rescale_combine(RescaleArgs A) {
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int i = blockIdx.y, bc = blockIdx.z;
+    if (n >= A.N) return;
+    const u64 q = A.mods[i].q;
+    u64 x = A.in[((size_t)bc * (A.l + 1) + i) * A.N + n];
+    u64 v = A.r[((size_t)bc * A.l + i) * A.N + n];
+    A.out[((size_t)bc * A.l + i) * A.N + n] = shoup(sub_mod(x, v, q), A.qlinv[i], q);
+}
+
+// ------------------------------------------------------------------ launchers
+static inline dim3 g1(int N) { return dim3((N + 255) / 256); }
+
+cudaError_t launch_bconv(const BConvTab& T, const BConvIO& io, int N, int batch, cudaStream_t st) {
+    k_bconv<<<dim3((N + 255) / 256, batch), 256, 0, st>>>(T, io, N);
+    return cudaGetLastError();
+}
+cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t st) {
+    k_keyip<<<dim3((A.N + 255) / 256, limbs, batch), 256, 0, st>>>(A);
+    return cudaGetLastError();
+}
+cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStream_t st) {
+    k_combine<<<dim3((A.N + 255) / 256, limbs, 2 * batch), 256, 0, st>>>(A);
+    return cudaGetLastError();
+}
+cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, int limbs, int N, int batch,
+                          cudaStream_t st) {
+    k_tensor<<<dim3(g1(N).x, limbs, batch), 256, 0, st>>>(a, b, d, mods, limbs, N);
+    return cudaGetLastError();
+}
+cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st) {
+    k_automorph<<<dim3(g1(N).x, rows), 256, 0, st>>>(in, out, g, N);
+    return cudaGetLastError();
+}
+cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st) {
+    k_modswitch<<<dim3(g1(N).x, l, bc), 256, 0, st>>>(last, r, mods, l, N);
+    return cudaGetLastError();
+}
+cudaError_t launch_rescale_combine(const RescaleArgs& A, int bc, cudaStream_t st) {
+    k_rescale_combine<<<dim3(g1(A.N).x, A.l, bc), 256, 0, st>>>(A);
+    return cudaGetLastError();
+}
+
+}  // namespace neo

@@ -1,0 +1,54 @@
+// kernels.h -- argument blocks and launchers of the streaming kernels (kernels.cu).
+#pragma once
+#include "context.h"
+
+namespace neo {
+
+constexpr int KS_MAX_EXT = 64;
+constexpr int KS_MAX_BETA = 8;
+
+struct KeyIPArgs {
+    const u64* d;          // KS input [B][l+1][N] (NTT form)
+    const u64* up;         // ModUp outputs after NTT [B][beta][E][N]
+    const u64* evk;        // [dnum][2][evk_limbs][N]
+    u64* acc;              // [B][2][E][N]
+    const ModQ* mods;
+    long long d_bstride, up_bstride, acc_bstride, acc_cstride;
+    int N, beta, evk_limbs;
+    int limb[KS_MAX_EXT];                    // position -> limb id
+    unsigned char src_kind[KS_MAX_BETA][KS_MAX_EXT];   // 0: d, 1: up
+    int src_off[KS_MAX_BETA][KS_MAX_EXT];    // row (in N units) inside the chosen buffer
+};
+
+struct CombineArgs {
+    const u64* acc;        // [B][2][E][N]; Q limbs are positions 0..l
+    const u64* conv;       // [2B][l+1][N]
+    const u64* add0;       // optional [B][..][N] addend of component 0 (nullptr: none)
+    const u64* add1;
+    u64* out0;
+    u64* out1;
+    const ModQ* mods;
+    long long acc_bstride, acc_cstride, conv_stride, add_bstride, out_bstride;
+    int N;
+    TW pinv[64];
+};
+
+struct RescaleArgs {
+    const u64* in;         // [2B][l+1][N]
+    const u64* r;          // [2B][l][N]
+    u64* out;              // [2B][l][N]
+    const ModQ* mods;
+    int N, l;
+    TW qlinv[64];
+};
+
+cudaError_t launch_bconv(const BConvTab& T, const BConvIO& io, int N, int batch, cudaStream_t st);
+cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t st);
+cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStream_t st);
+cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, int limbs, int N, int batch,
+                          cudaStream_t st);
+cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st);
+cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st);
+cudaError_t launch_rescale_combine(const RescaleArgs& A, int bc, cudaStream_t st);
+
+}  // namespace neo

@@ -1,0 +1,246 @@
+// params.cpp -- host generation of the RNS parameters and device constant tables.
+//
+// Primes (rule Z4): q = k*2N + 1 for k from floor((2^W - 1)/2N) downward, W-bit, prime
+// (deterministic Miller-Rabin); the first num_q are q_0.., the next num_p are p_0...
+// psi (rule Z5): the minimal primitive 2N-th root of unity.
+// Tables: NTT twiddles (ntt_tables.h), BConv constants per (level, digit) for ModUp
+// (Eq. 2) and per level for ModDown (Table 2), P^-1 mod q_i, q_l^-1 mod q_i.
+#include <algorithm>
+#include <cstring>
+#include <stdexcept>
+
+#include "context.h"
+
+namespace neo {
+
+static inline u64 mulm(u64 a, u64 b, u64 m) { return (u64)((u128)a * b % m); }
+static u64 powm(u64 a, u64 e, u64 m) {
+    u64 r = 1 % m;
+    a %= m;
+    for (; e; e >>= 1, a = mulm(a, a, m))
+        if (e & 1) r = mulm(r, a, m);
+    return r;
+}
+static u64 invm(u64 a, u64 m) { return powm(a, m - 2, m); }   // m prime
+
+static bool is_prime_u64(u64 n) {
+    static const u64 bases[] = {2, 3, 5, 7, 11, 13, 17, 19, 23, 29, 31, 37};
+    if (n < 2) return false;
+    for (u64 b : bases)
+        if (n % b == 0) return n == b;
+    u64 d = n - 1;
+    int s = 0;
+    while (!(d & 1)) { d >>= 1; ++s; }
+    for (u64 b : bases) {
+        u64 x = powm(b, d, n);
+        if (x == 1 || x == n - 1) continue;
+        bool comp = true;
+        for (int r = 1; r < s; ++r) {
+            x = mulm(x, x, n);
+            if (x == n - 1) { comp = false; break; }
+        }
+        if (comp) return false;
+    }
+    return true;
+}
+
+std::vector<u64> gen_primes(int log_n, int bits, int count) {
+    u64 two_n = 2ull << log_n;
+    u64 k = ((1ull << bits) - 1) / two_n;
+    std::vector<u64> out;
+    while ((int)out.size() < count) {
+        if (k == 0) break;
+        u64 q = k * two_n + 1;
+        if ((q >> (bits - 1)) != 1) break;        // fell below W bits
+        if (is_prime_u64(q)) out.push_back(q);
+        --k;
+    }
+    return out;
+}
+
+u64 min_psi(u64 q, u64 n) {
+    u64 e = (q - 1) / (2 * n);
+    u64 psi0 = 0;
+    for (u64 x = 2;; ++x) {
+        psi0 = powm(x, e, q);
+        if (powm(psi0, n, q) == q - 1) break;
+    }
+    u64 best = psi0, cur = psi0, sq = mulm(psi0, psi0, q);
+    for (u64 i = 1; i < n; ++i) {
+        cur = mulm(cur, sq, q);
+        best = std::min(best, cur);
+    }
+    return best;
+}
+
+static TW mk_tw(u64 w, u64 q) { return TW{w, (u64)(((u128)w << 64) / q)}; }
+
+static int brev(int x, int R) {
+    int lg = 0;
+    while ((1 << lg) < R) ++lg;
+    int y = 0;
+    for (int b = 0; b < lg; ++b) y |= ((x >> b) & 1) << (lg - 1 - b);
+    return y;
+}
+
+// Fill one prime's twiddle block (formulas documented in ntt_tables.h).
+static void fill_ntt_block(TW* t, const NttLayout& L, u64 q, u64 psi, int N) {
+    const int R = L.R, N1 = L.N1, N2 = L.N2;
+    const u64 ipsi = invm(psi, q);
+    auto P = [&](u64 base, long long e) { return powm(base, (u64)e, q); };
+    const u64 psi1 = P(psi, N2), ipsi1 = P(ipsi, N2);
+    const u64 rho = P(psi1, R), irho = P(ipsi1, R);
+    const u64 om1 = P(psi1, 2 * R), iom1 = P(ipsi1, 2 * R);
+    const u64 om2 = P(psi, 2 * N1), iom2 = P(ipsi, 2 * N1);
+    const u64 om2R = P(om2, R), iom2R = P(iom2, R);
+    const u64 ninv = invm((u64)N % q, q);
+    for (int k = 0; k < R; ++k) {
+        t[L.colf_neg + k] = mk_tw(P(rho, brev(k, R)), q);
+        t[L.coli_neg + k] = mk_tw(P(irho, brev(k, R)), q);
+    }
+    for (int r = 0; r < R; ++r)
+        for (int x = 0; x < R; ++x) {
+            t[L.colf_tw1 + r * R + x] = mk_tw(P(psi1, (long long)(2 * x + 1) * r), q);
+            t[L.coli_tw1 + r * R + x] = mk_tw(P(ipsi1, (long long)(2 * r + 1) * x), q);
+            t[L.rowf_tw2 + r * R + x] = mk_tw(P(om2, (long long)x * r), q);
+            t[L.rowi_tw2 + r * R + x] = mk_tw(P(iom2, (long long)x * r), q);
+        }
+    for (int j = 0; j < R / 2; ++j) {
+        t[L.colf_cyc + j] = mk_tw(P(om1, j), q);
+        t[L.coli_cyc + j] = mk_tw(P(iom1, j), q);
+        t[L.rowf_cyc + j] = mk_tw(P(om2R, j), q);
+        t[L.rowi_cyc + j] = mk_tw(P(iom2R, j), q);
+    }
+    const u64 two_n = 2ull * N;
+    for (int n2 = 0; n2 < N2; ++n2)
+        for (int r = 0; r < R; ++r) {
+            u64 ea = ((u64)(2 * r + 1) * n2) % two_n;
+            u64 eb = ((u64)2 * R * r * n2) % two_n;          // here r plays ib
+            t[L.outf_a + n2 * R + r] = mk_tw(P(psi, ea), q);
+            t[L.outf_b + n2 * R + r] = mk_tw(P(psi, eb), q);
+            t[L.outi_a + n2 * R + r] = mk_tw(mulm(ninv, P(ipsi, ea), q), q);
+            t[L.outi_b + n2 * R + r] = mk_tw(P(ipsi, eb), q);
+        }
+}
+
+static ModQ mk_mod(u64 q) {
+    ModQ m;
+    m.q = q;
+    m.mu = (u64)(((u128)1 << 98) / q);
+    return m;
+}
+
+// Algorithm 1 constants for src -> dst limb ids.
+static BConvTab make_bconv(const neo_ctx* c, const std::vector<int>& src, const std::vector<int>& dst) {
+    BConvTab b;
+    std::memset(&b, 0, sizeof(b));
+    b.n_in = (int)src.size();
+    b.n_out = (int)dst.size();
+    for (int i = 0; i < b.n_in; ++i) {
+        u64 qi = c->mod[src[i]];
+        b.qin[i] = qi;
+        u64 qh = 1;                                          // qhat_i mod q_i
+        for (int k = 0; k < b.n_in; ++k)
+            if (k != i) qh = mulm(qh, c->mod[src[k]] % qi, qi);
+        b.qhat_inv[i] = mk_tw(invm(qh, qi), qi);
+    }
+    for (int j = 0; j < b.n_out; ++j) {
+        u64 t = c->mod[dst[j]];
+        b.tmod[j] = mk_mod(t);
+        for (int i = 0; i < b.n_in; ++i) {
+            u64 f = 1;                                       // qhat_i mod t
+            for (int k = 0; k < b.n_in; ++k)
+                if (k != i) f = mulm(f, c->mod[src[k]] % t, t);
+            b.f_lo[i][j] = (unsigned)(f & 0x3FFFF);
+            b.f_hi[i][j] = (unsigned)(f >> 18);
+        }
+    }
+    return b;
+}
+
+// Build everything; throws std::runtime_error / returns status through abi.cpp.
+neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err) {
+    c->log_n = d->log_n;
+    c->N = 1 << d->log_n;
+    c->num_q = d->num_q;
+    c->num_p = d->num_p;
+    c->dnum = d->dnum;
+    c->word_bits = d->word_bits;
+    c->device = d->device;
+    c->alpha = (c->num_q + c->dnum - 1) / c->dnum;
+    const int nl = c->num_q + c->num_p;
+    if (d->q && d->p) {
+        c->mod.assign(d->q, d->q + c->num_q);
+        c->mod.insert(c->mod.end(), d->p, d->p + c->num_p);
+        for (u64 m : c->mod)
+            if (m % (2ull * c->N) != 1 || (m >> (c->word_bits - 1)) != 1 || !is_prime_u64(m)) {
+                err = "explicit prime is not a word_bits-bit prime = 1 mod 2N";
+                return NEO_EINVAL;
+            }
+    } else {
+        c->mod = gen_primes(c->log_n, c->word_bits, nl);
+        if ((int)c->mod.size() != nl) { err = "not enough NTT-friendly primes"; return NEO_ENOPRIME; }
+    }
+    c->psi.resize(nl);
+    c->h_mods.resize(nl);
+    for (int i = 0; i < nl; ++i) {
+        c->psi[i] = min_psi(c->mod[i], (u64)c->N);
+        c->h_mods[i] = mk_mod(c->mod[i]);
+    }
+    c->L = make_ntt_layout(c->log_n);
+
+    // ---- device tables
+    std::vector<TW> tab((size_t)nl * c->L.total);
+    for (int i = 0; i < nl; ++i) fill_ntt_block(&tab[(size_t)i * c->L.total], c->L, c->mod[i], c->psi[i], c->N);
+    if (cudaSetDevice(c->device) != cudaSuccess) { err = "cudaSetDevice failed"; return NEO_ECUDA; }
+    if (cudaMalloc(&c->d_tab, tab.size() * sizeof(TW)) != cudaSuccess ||
+        cudaMalloc(&c->d_mods, nl * sizeof(ModQ)) != cudaSuccess) {
+        err = "cudaMalloc of constant tables failed";
+        return NEO_ENOMEM;
+    }
+    if (cudaMemcpy(c->d_tab, tab.data(), tab.size() * sizeof(TW), cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(c->d_mods, c->h_mods.data(), nl * sizeof(ModQ), cudaMemcpyHostToDevice) != cudaSuccess) {
+        err = "cudaMemcpy of constant tables failed";
+        return NEO_ECUDA;
+    }
+    c->ntt.tab = c->d_tab;
+    c->ntt.tab_stride = c->L.total;
+    c->ntt.mods = c->d_mods;
+    c->ntt.N = c->N;
+    c->ntt.N1 = c->L.N1;
+    c->ntt.N2 = c->L.N2;
+    c->ntt.L = c->L;
+
+    // ---- BConv / ModDown / rescale constants per level
+    std::vector<int> pids;
+    for (int k = 0; k < c->num_p; ++k) pids.push_back(c->num_q + k);
+    c->modup.resize(c->num_q);
+    c->digits.resize(c->num_q);
+    c->moddown.resize(c->num_q);
+    c->ql_inv.resize(c->num_q);
+    for (int l = 0; l < c->num_q; ++l) {
+        std::vector<int> qids;
+        for (int i = 0; i <= l; ++i) qids.push_back(i);
+        for (int j = 0; j < c->beta(l); ++j) {
+            std::vector<int> dj, tg;
+            for (int i = j * c->alpha; i < std::min((j + 1) * c->alpha, l + 1); ++i) dj.push_back(i);
+            for (int pos = 0; pos < c->ext(l); ++pos) {
+                int id = c->ext_id(l, pos);
+                if (std::find(dj.begin(), dj.end(), id) == dj.end()) tg.push_back(id);
+            }
+            c->digits[l].push_back(dj);
+            c->modup[l].push_back(make_bconv(c, dj, tg));
+        }
+        c->moddown[l] = make_bconv(c, pids, qids);
+        for (int i = 0; i < l; ++i) c->ql_inv[l].push_back(mk_tw(invm(c->mod[l] % c->mod[i], c->mod[i]), c->mod[i]));
+    }
+    c->pinv.resize(c->num_q);
+    for (int i = 0; i < c->num_q; ++i) {
+        u64 P = 1;
+        for (int k = 0; k < c->num_p; ++k) P = mulm(P, c->mod[c->num_q + k] % c->mod[i], c->mod[i]);
+        c->pinv[i] = mk_tw(invm(P, c->mod[i]), c->mod[i]);
+    }
+    return NEO_OK;
+}
+
+}  // namespace neo

@@ -1,0 +1,214 @@
+"""Thin ctypes binding of libneo.so (include/neo.h).  Argument marshalling only: every step
+of the key-switching path runs in the library's CUDA kernels.  There is no fallback -- if
+libneo.so is missing or a call fails, this module raises.
+
+Tensors are torch.uint64 CUDA tensors (device memory and streams come from PyTorch); the
+functions carry the C names of neo.h and take the same arguments, with (pointer, size)
+pairs replaced by tensors.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libneo.so")
+
+NEO_OP_KEYSWITCH, NEO_OP_HMULT, NEO_OP_HROT, NEO_OP_RESCALE = 0, 1, 2, 3
+_STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM", 4: "NEO_ECUDA",
+           5: "NEO_ENCCL", 6: "NEO_ENOPRIME"}
+
+EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_workspace_size",
+            "neo_ntt", "neo_intt", "neo_bconv", "neo_tensor", "neo_automorphism", "neo_evk_create",
+            "neo_evk_destroy", "neo_keyswitch", "neo_hmult", "neo_hrot", "neo_rescale",
+            "neo_last_error", "neo_last_launch_count")
+
+
+class NeoError(RuntimeError):
+    def __init__(self, status: int, where: str, msg: str):
+        super().__init__(f"{where}: {_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class ParamsDesc(ctypes.Structure):
+    _fields_ = [("log_n", ctypes.c_int32), ("num_q", ctypes.c_int32), ("num_p", ctypes.c_int32),
+                ("dnum", ctypes.c_int32), ("word_bits", ctypes.c_int32), ("device", ctypes.c_int32),
+                ("q", ctypes.POINTER(ctypes.c_uint64)), ("p", ctypes.POINTER(ctypes.c_uint64))]
+
+
+_lib = None
+_vp, _i32, _u32, _sz = ctypes.c_void_p, ctypes.c_int32, ctypes.c_uint32, ctypes.c_size_t
+_i32p = ctypes.POINTER(ctypes.c_int32)
+_u64p = ctypes.POINTER(ctypes.c_uint64)
+
+
+def lib() -> ctypes.CDLL:
+    """Load libneo.so (built by paper_conf_isca_jiaodwfcm0z25_b200.build); raise if absent."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is not built (run python -m paper_conf_isca_jiaodwfcm0z25_b200.build)")
+        L = ctypes.CDLL(LIB_PATH)
+        sig = {
+            "neo_params_create": [ctypes.POINTER(ParamsDesc), ctypes.POINTER(_vp)],
+            "neo_params_destroy": [_vp],
+            "neo_params_query": [_vp, _u64p, _u64p, _u64p],
+            "neo_ntt": [_vp, _vp, _i32p, _i32, _i32, _vp, _sz, _vp],
+            "neo_intt": [_vp, _vp, _i32p, _i32, _i32, _vp, _sz, _vp],
+            "neo_bconv": [_vp, _vp, _i32p, _i32, _vp, _i32p, _i32, _i32, _vp],
+            "neo_tensor": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
+            "neo_automorphism": [_vp, _vp, _i32, _u32, _vp, _i32, _vp],
+            "neo_evk_create": [_vp, _vp, ctypes.POINTER(_vp)],
+            "neo_evk_destroy": [_vp],
+            "neo_keyswitch": [_vp, _vp, _vp, _i32, _vp, _vp, _i32, _vp, _sz, _vp],
+            "neo_hmult": [_vp, _vp, _vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+            "neo_hrot": [_vp, _vp, _u32, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+            "neo_rescale": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+        }
+        for name, args in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = ctypes.c_int
+        L.neo_workspace_size.argtypes = [_vp, _i32, _i32, _i32]
+        L.neo_workspace_size.restype = _sz
+        L.neo_last_error.restype = ctypes.c_char_p
+        L.neo_last_error.argtypes = []
+        L.neo_last_launch_count.restype = _i32
+        L.neo_last_launch_count.argtypes = []
+        _lib = L
+    return _lib
+
+
+def _check(status: int, where: str):
+    if status != 0:
+        raise NeoError(status, where, lib().neo_last_error().decode())
+
+
+def _ptr(t: torch.Tensor | None):
+    if t is None:
+        return None
+    if t.dtype != torch.uint64 or not t.is_cuda or not t.is_contiguous():
+        raise TypeError("expected a contiguous torch.uint64 CUDA tensor")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(stream) -> ctypes.c_void_p:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _ids(ids) -> ctypes.Array:
+    ids = [int(i) for i in ids]
+    return (ctypes.c_int32 * len(ids))(*ids)
+
+
+def last_launch_count() -> int:
+    return int(lib().neo_last_launch_count())
+
+
+class Context:
+    """neo_params_create / neo_params_destroy; q, p, psi from neo_params_query."""
+
+    def __init__(self, log_n: int, num_q: int, num_p: int, dnum: int, word_bits: int = 36, device: int = 0):
+        self.log_n, self.num_q, self.num_p, self.dnum = log_n, num_q, num_p, dnum
+        self.N = 1 << log_n
+        self.alpha = -(-num_q // dnum)
+        d = ParamsDesc(log_n, num_q, num_p, dnum, word_bits, device, None, None)
+        h = ctypes.c_void_p()
+        _check(lib().neo_params_create(ctypes.byref(d), ctypes.byref(h)), "neo_params_create")
+        self.handle = h
+        q = (ctypes.c_uint64 * num_q)()
+        p = (ctypes.c_uint64 * num_p)()
+        psi = (ctypes.c_uint64 * (num_q + num_p))()
+        _check(lib().neo_params_query(h, q, p, psi), "neo_params_query")
+        self.q, self.p, self.psi = list(q), list(p), list(psi)
+        self.moduli = self.q + self.p
+
+    def close(self):
+        if self.handle:
+            lib().neo_params_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def workspace_size(self, op: int, level: int, batch: int) -> int:
+        return int(lib().neo_workspace_size(self.handle, op, level, batch))
+
+    def workspace(self, op: int, level: int, batch: int, device="cuda") -> torch.Tensor:
+        n = self.workspace_size(op, level, batch)
+        if n == 0:
+            raise NeoError(1, "neo_workspace_size", "invalid op/level/batch")
+        return torch.empty(n // 8, dtype=torch.uint64, device=device)
+
+
+class EvalKey:
+    """neo_evk_create / neo_evk_destroy (device copy of [dnum][2][num_q+num_p][N])."""
+
+    def __init__(self, ctx: Context, evk: torch.Tensor):
+        self.ctx = ctx
+        h = ctypes.c_void_p()
+        _check(lib().neo_evk_create(ctx.handle, _ptr(evk), ctypes.byref(h)), "neo_evk_create")
+        self.handle = h
+
+    def close(self):
+        if self.handle:
+            lib().neo_evk_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def neo_ntt(ctx: Context, poly: torch.Tensor, limb_ids, batch: int, ws: torch.Tensor, stream=None):
+    _check(lib().neo_ntt(ctx.handle, _ptr(poly), _ids(limb_ids), len(limb_ids), batch, _ptr(ws),
+                         ws.numel() * 8, _stream(stream)), "neo_ntt")
+
+
+def neo_intt(ctx: Context, poly: torch.Tensor, limb_ids, batch: int, ws: torch.Tensor, stream=None):
+    _check(lib().neo_intt(ctx.handle, _ptr(poly), _ids(limb_ids), len(limb_ids), batch, _ptr(ws),
+                          ws.numel() * 8, _stream(stream)), "neo_intt")
+
+
+def neo_bconv(ctx: Context, inp: torch.Tensor, in_ids, out: torch.Tensor, out_ids, batch: int, stream=None):
+    _check(lib().neo_bconv(ctx.handle, _ptr(inp), _ids(in_ids), len(in_ids), _ptr(out), _ids(out_ids),
+                           len(out_ids), batch, _stream(stream)), "neo_bconv")
+
+
+def neo_tensor(ctx: Context, ct_a, ct_b, level: int, d, batch: int, stream=None):
+    _check(lib().neo_tensor(ctx.handle, _ptr(ct_a), _ptr(ct_b), level, _ptr(d), batch, _stream(stream)),
+           "neo_tensor")
+
+
+def neo_automorphism(ctx: Context, inp, n_limbs: int, galois_elt: int, out, batch: int, stream=None):
+    _check(lib().neo_automorphism(ctx.handle, _ptr(inp), n_limbs, galois_elt, _ptr(out), batch,
+                                  _stream(stream)), "neo_automorphism")
+
+
+def neo_keyswitch(ctx: Context, evk: EvalKey, d, level: int, out0, out1, batch: int, ws, stream=None):
+    _check(lib().neo_keyswitch(ctx.handle, evk.handle, _ptr(d), level, _ptr(out0), _ptr(out1), batch,
+                               _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_keyswitch")
+
+
+def neo_hmult(ctx: Context, relin: EvalKey, ct_a, ct_b, level: int, ct_out, batch: int, ws, stream=None):
+    _check(lib().neo_hmult(ctx.handle, relin.handle, _ptr(ct_a), _ptr(ct_b), level, _ptr(ct_out), batch,
+                           _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_hmult")
+
+
+def neo_hrot(ctx: Context, rotkey: EvalKey, galois_elt: int, ct_in, level: int, ct_out, batch: int, ws,
+             stream=None):
+    _check(lib().neo_hrot(ctx.handle, rotkey.handle, galois_elt, _ptr(ct_in), level, _ptr(ct_out), batch,
+                          _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_hrot")
+
+
+def neo_rescale(ctx: Context, ct_in, level: int, ct_out, batch: int, ws, stream=None):
+    _check(lib().neo_rescale(ctx.handle, _ptr(ct_in), level, _ptr(ct_out), batch, _ptr(ws), ws.numel() * 8,
+                             _stream(stream)), "neo_rescale")

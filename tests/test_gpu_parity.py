@@ -1,0 +1,235 @@
+"""GPU parity: every stage of the CUDA path (through the C-ABI) against the CPU oracle,
+element by element and bit-exact on every residue (integer work: SURVEY §8(c) Z23).
+
+Inputs are seeded (synth); expected values come only from oracle/.  Sizes: the tiny config
+(N=2^12) with ragged shapes and batches, and Set-B (N=2^16, 36+12 limbs, dnum=3) in the
+launch configuration bench.py times."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import ckks
+
+pytestmark = pytest.mark.gpu
+
+neo = pytest.importorskip("paper_conf_isca_jiaodwfcm0z25_b200.neo")
+
+_CTX = {}
+_PRM = {}
+
+
+def ctx_of(name):
+    if name not in _CTX:
+        prm = {"tiny": ckks.tiny, "tiny3": ckks.tiny_dnum3, "setb": ckks.set_b}[name]()
+        _PRM[name] = prm
+        _CTX[name] = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+    return _CTX[name], _PRM[name]
+
+
+def dev(a: np.ndarray) -> torch.Tensor:
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint64)).cuda()
+
+
+def host(t: torch.Tensor) -> np.ndarray:
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+def rand_poly(prm, ids, seed):
+    return synth.uniform_residues(seed, [prm.moduli[i] for i in ids], prm.N)
+
+
+def rand_ct(prm, level, seed):
+    ids = list(range(level + 1))
+    return np.stack([rand_poly(prm, ids, seed), rand_poly(prm, ids, seed + 1)])
+
+
+def rand_evk(prm, seed):
+    ids = list(range(prm.num_q + prm.num_p))
+    return np.stack([np.stack([rand_poly(prm, ids, seed + 2 * j + c) for c in range(2)])
+                     for j in range(prm.dnum)])
+
+
+@pytest.mark.parametrize("name", ["tiny", "tiny3", "setb"])
+def test_params_match_oracle(name):
+    ctx, prm = ctx_of(name)
+    assert ctx.q == prm.q and ctx.p == prm.p and ctx.psi == prm.psi
+
+
+@pytest.mark.parametrize("name,batch", [("tiny", 3), ("setb", 1)])
+def test_ntt_intt(name, batch):
+    ctx, prm = ctx_of(name)
+    ids = list(range(prm.num_q + prm.num_p))
+    x = np.stack([rand_poly(prm, ids, 100 + b) for b in range(batch)])
+    t = dev(x)
+    ws = torch.empty(t.numel(), dtype=torch.uint64, device="cuda")
+    neo.neo_ntt(ctx, t, ids, batch, ws)
+    got = host(t)
+    for b in range(batch):
+        assert np.array_equal(got[b], ckks.ntt(prm, x[b], ids))
+    neo.neo_intt(ctx, t, ids, batch, ws)
+    assert np.array_equal(host(t), x)
+
+
+def test_intt_matches_oracle_ragged_ids():
+    ctx, prm = ctx_of("tiny")
+    ids = [3, 0, 2]                      # arbitrary order, P limb first
+    x = rand_poly(prm, ids, 7)[None]
+    t = dev(x)
+    ws = torch.empty_like(t)
+    neo.neo_intt(ctx, t, ids, 1, ws)
+    assert np.array_equal(host(t)[0], ckks.intt(prm, x[0], ids))
+
+
+@pytest.mark.parametrize("name,src,dst,batch", [
+    ("tiny", [0, 1, 2], [3], 2),                          # ModUp of the whole digit (dnum = 1)
+    ("tiny", [3], [0, 1, 2], 1),                          # ModDown shape
+    ("setb", list(range(12)), list(range(12, 48)), 1),    # Set-B ModUp digit 0
+    ("setb", list(range(36, 48)), list(range(36)), 2),    # Set-B ModDown
+    ("setb", [5, 17, 40, 2, 33], [0, 47, 9, 21, 3, 11, 30], 1),   # ragged
+])
+def test_bconv(name, src, dst, batch):
+    ctx, prm = ctx_of(name)
+    x = np.stack([rand_poly(prm, src, 200 + b) for b in range(batch)])
+    out = torch.empty((batch, len(dst), prm.N), dtype=torch.uint64, device="cuda")
+    neo.neo_bconv(ctx, dev(x), src, out, dst, batch)
+    got = host(out)
+    for b in range(batch):
+        assert np.array_equal(got[b], ckks.bconv(prm, x[b], src, dst))
+
+
+@pytest.mark.parametrize("name,level,batch", [("tiny", 2, 2), ("setb", 35, 1)])
+def test_tensor(name, level, batch):
+    ctx, prm = ctx_of(name)
+    a = np.stack([rand_ct(prm, level, 300 + 4 * b) for b in range(batch)])
+    b_ = np.stack([rand_ct(prm, level, 302 + 4 * b) for b in range(batch)])
+    d = torch.empty((batch, 3, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+    neo.neo_tensor(ctx, dev(a), dev(b_), level, d, batch)
+    got = host(d)
+    for bb in range(batch):
+        want = ckks.tensor(prm, a[bb], b_[bb], level)
+        for k in range(3):
+            assert np.array_equal(got[bb, k], want[k])
+
+
+@pytest.mark.parametrize("g", [5, 25, 8191, 3])
+def test_automorphism(g):
+    ctx, prm = ctx_of("tiny")
+    x = np.stack([rand_poly(prm, [0, 1, 2, 3], 400 + b) for b in range(2)])
+    out = torch.empty_like(dev(x))
+    neo.neo_automorphism(ctx, dev(x), 4, g, out, 2)
+    assert np.array_equal(host(out), ckks.automorphism_ntt(x, g))
+
+
+def _ks(name, level, batch, seed):
+    ctx, prm = ctx_of(name)
+    evk_np = rand_evk(prm, seed)
+    evk = neo.EvalKey(ctx, dev(evk_np))
+    d = np.stack([rand_poly(prm, list(range(level + 1)), seed + 50 + b) for b in range(batch)])
+    o0 = torch.empty((batch, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+    o1 = torch.empty_like(o0)
+    ws = ctx.workspace(neo.NEO_OP_KEYSWITCH, level, batch)
+    neo.neo_keyswitch(ctx, evk, dev(d), level, o0, o1, batch, ws)
+    g0, g1 = host(o0), host(o1)
+    for b in range(batch):
+        k0, k1 = ckks.keyswitch(prm, d[b], level, evk_np)
+        assert np.array_equal(g0[b], k0)
+        assert np.array_equal(g1[b], k1)
+
+
+@pytest.mark.parametrize("name,level,batch", [
+    ("tiny", 2, 2), ("tiny", 0, 1), ("tiny3", 2, 1), ("tiny3", 1, 3),
+])
+def test_keyswitch_tiny(name, level, batch):
+    _ks(name, level, batch, 500 + level)
+
+
+@pytest.mark.parametrize("level", [35, 13, 0])
+def test_keyswitch_setb(level):
+    """Set-B: full level (3 full digits), a partial last digit (l = 13), and level 0."""
+    _ks("setb", level, 1, 600 + level)
+
+
+def test_keyswitch_setb_batch2():
+    _ks("setb", 35, 2, 700)
+
+
+@pytest.mark.parametrize("name,level,batch", [("tiny", 2, 2), ("setb", 35, 1)])
+def test_hmult(name, level, batch):
+    ctx, prm = ctx_of(name)
+    evk_np = rand_evk(prm, 800)
+    relin = neo.EvalKey(ctx, dev(evk_np))
+    a = np.stack([rand_ct(prm, level, 810 + 4 * b) for b in range(batch)])
+    b_ = np.stack([rand_ct(prm, level, 812 + 4 * b) for b in range(batch)])
+    out = torch.empty((batch, 2, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+    ws = ctx.workspace(neo.NEO_OP_HMULT, level, batch)
+    neo.neo_hmult(ctx, relin, dev(a), dev(b_), level, out, batch, ws)
+    got = host(out)
+    for bb in range(batch):
+        assert np.array_equal(got[bb], ckks.hmult(prm, a[bb], b_[bb], level, evk_np))
+
+
+@pytest.mark.parametrize("name,level,batch,r", [("tiny", 2, 2, 1), ("setb", 35, 1, 1), ("setb", 20, 1, 7)])
+def test_hrot(name, level, batch, r):
+    ctx, prm = ctx_of(name)
+    g = pow(5, r, 2 * prm.N)
+    evk_np = rand_evk(prm, 900)
+    rk = neo.EvalKey(ctx, dev(evk_np))
+    ct = np.stack([rand_ct(prm, level, 910 + 2 * b) for b in range(batch)])
+    out = torch.empty((batch, 2, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+    ws = ctx.workspace(neo.NEO_OP_HROT, level, batch)
+    neo.neo_hrot(ctx, rk, g, dev(ct), level, out, batch, ws)
+    got = host(out)
+    for bb in range(batch):
+        assert np.array_equal(got[bb], ckks.hrot(prm, ct[bb], g, level, evk_np))
+
+
+@pytest.mark.parametrize("name,level,batch", [("tiny", 2, 2), ("tiny", 1, 1), ("setb", 35, 1)])
+def test_rescale(name, level, batch):
+    ctx, prm = ctx_of(name)
+    ct = np.stack([rand_ct(prm, level, 1000 + 2 * b) for b in range(batch)])
+    out = torch.empty((batch, 2, level, prm.N), dtype=torch.uint64, device="cuda")
+    ws = ctx.workspace(neo.NEO_OP_RESCALE, level, batch)
+    neo.neo_rescale(ctx, dev(ct), level, out, batch, ws)
+    got = host(out)
+    for bb in range(batch):
+        assert np.array_equal(got[bb], ckks.rescale(prm, ct[bb], level))
+
+
+def test_hmult_rescale_decrypts():
+    """Real encryptions (tiny, dnum=3): GPU HMULT + Rescale decodes to z_a z_b within 1e-6
+    at Delta = 2^40 and equals the oracle bit for bit."""
+    ctx, prm = ctx_of("tiny3")
+    delta = 2.0 ** 40
+    s = ckks.secret(prm, 11, 192)
+    za, zb = synth.complex_slots(101, prm.N // 2), synth.complex_slots(102, prm.N // 2)
+    cta = ckks.encrypt(prm, ckks.encode(prm.N, za, delta), s, 2, 201)
+    ctb = ckks.encrypt(prm, ckks.encode(prm.N, zb, delta), s, 2, 202)
+    relin_np = ckks.relin_key(prm, s, 301)
+    relin = neo.EvalKey(ctx, dev(relin_np))
+    out = torch.empty((1, 2, 3, prm.N), dtype=torch.uint64, device="cuda")
+    neo.neo_hmult(ctx, relin, dev(cta[None]), dev(ctb[None]), 2, out, 1, ctx.workspace(neo.NEO_OP_HMULT, 2, 1))
+    res = torch.empty((1, 2, 2, prm.N), dtype=torch.uint64, device="cuda")
+    neo.neo_rescale(ctx, out, 2, res, 1, ctx.workspace(neo.NEO_OP_RESCALE, 2, 1))
+    got = host(res)[0]
+    want = ckks.rescale(prm, ckks.hmult(prm, cta, ctb, 2, relin_np), 2)
+    assert np.array_equal(got, want)
+    m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, got, s, 1), [0, 1])
+    z = ckks.decode(prm.N, m, delta * delta / prm.q[2])
+    assert np.max(np.abs(z - za * zb)) < 1e-6
+
+
+def test_invalid_arguments_fail_loudly():
+    ctx, prm = ctx_of("tiny")
+    t = torch.zeros((1, 3, prm.N), dtype=torch.uint64, device="cuda")
+    ws = torch.empty_like(t)
+    with pytest.raises(neo.NeoError):
+        neo.neo_ntt(ctx, t, [0, 1, 99], 1, ws)
+    with pytest.raises(neo.NeoError):
+        neo.neo_automorphism(ctx, t, 3, 4, t.clone(), 1)        # even Galois element
+    evk = neo.EvalKey(ctx, dev(rand_evk(prm, 1)))
+    with pytest.raises(neo.NeoError):
+        neo.neo_keyswitch(ctx, evk, t, 5, t, t, 1, ws)          # level out of range
+    with pytest.raises(neo.NeoError):
+        neo.neo_keyswitch(ctx, evk, t[:, :3], 2, t.clone(), t.clone(), 1, ws)   # workspace too small
