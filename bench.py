@@ -1,0 +1,388 @@
+#!/usr/bin/env python
+"""bench.py -- throughput of Neo's Hybrid key-switching hot path on B200.
+
+Workload (BASELINE.json configs[1], Set-B of Table 4): N = 2^16, 36 Q limbs + 12 P
+limbs of 36 bits, dnum = 3, level l = 35.  One STEP is one pass over every row of
+SURVEY §8(a) for one batch of B ciphertexts per GPU:
+    HMULT(ct_a, ct_b)  [tensor + KS(d2) + combine]  ->  Rescale          (a1, a3-a11)
+    HROTATE(ct_c, g = 5)  [automorphism + KS + combine]                   (a2, a3-a10)
+i.e. 2*B key-switches per step per GPU.  value = key-switches/s over all ranks (weak
+scaling: every rank does its own B ciphertexts; data-parallel, no collective on the data
+path).  Inputs are synthetic uniform residues (timing is data-independent; parity is
+tested in tests/), resident in HBM, rotating over 2 input slots (216 MB at B=1) so that
+inputs + the two 151 MB keys exceed the 126 MB L2.
+
+`--impl reference` times the CPU oracle (oracle/, the reference arm of this tier) on the
+same workload: each step is one Set-B key-switch on the host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "key-switch ops/s (HMult, HRot) at N=2^16 on 1/2/4/8 B200"
+UNIT = "KS/s"
+LOG_N, NUM_Q, NUM_P, DNUM, LEVEL = 16, 36, 12, 3, 35
+HBM_FALLBACK = 6650.0   # GB/s, /opt/skills/guides/B200_PROFILING.md fallback
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=300)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--batch", type=int, default=1, help="ciphertexts per GPU per step")
+    ap.add_argument("--impl", choices=["neo", "reference"], default="neo")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    return ap.parse_args()
+
+
+def workload_config(batch: int, world: int) -> dict:
+    return {"workload": "setB_hmult_rescale_hrot", "N": 1 << LOG_N, "num_q": NUM_Q, "num_p": NUM_P,
+            "dnum": DNUM, "level": LEVEL, "word_bits": 36, "batch_per_gpu": batch,
+            "global_batch": batch * world, "ks_per_step_per_gpu": 2 * batch,
+            "parallelism": f"dp{world}",
+            "l2": "inputs rotate over 2 slots (3 ciphertexts each) + 2 x 151 MB keys > 126 MB L2"}
+
+
+# ----------------------------------------------------------------------------- inputs
+
+def rand_limbs(moduli, seed, n):
+    import synth
+    return synth.uniform_residues(seed, moduli, n)
+
+
+def rand_ct(moduli_q, seed, N, batch):
+    return np.stack([np.stack([rand_limbs(moduli_q, seed + 7 * b + c, N) for c in range(2)])
+                     for b in range(batch)])
+
+
+def rand_evk(moduli, seed, N):
+    return np.stack([np.stack([rand_limbs(moduli, seed + 2 * j + c, N) for c in range(2)])
+                     for j in range(DNUM)])
+
+
+# ----------------------------------------------------------------------------- clocks
+
+class ClockSampler:
+    """nvidia-smi sampling (B200_PROFILING.md clocks line) during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.15)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self) -> dict:
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for k, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(k)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- byte model
+
+def bytes_model(batch: int, l: int = LEVEL) -> dict:
+    """Algorithmic HBM bytes per step, per kernel kind (SURVEY §8(d) per-limb figures x the
+    limbs each launch processes; limb = N words of 8 bytes)."""
+    limb = (1 << LOG_N) * 8
+    Lq, P, beta, alpha = l + 1, NUM_P, -(-(l + 1) // 12), 12
+    E = Lq + P
+    ks_ntt = Lq + (beta * E - Lq) + 2 * P + 2 * Lq             # limb transforms per KS
+    resc_ntt = 2 + 2 * l
+    ntt_limbs = batch * (2 * ks_ntt + resc_ntt)                  # per step
+    per_pass = 2 * limb                                          # read + write one limb
+    bconv = batch * 2 * ((beta * alpha + beta * (E - alpha)) + (2 * P + 2 * Lq)) * limb
+    keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E) * limb   # dhat + out per ct, evk once
+    combine = batch * ((2 * Lq * 3 + 2 * Lq) + (2 * Lq * 2 + Lq + 2 * Lq)) * limb
+    tensor = batch * 7 * Lq * limb
+    auto = batch * 4 * Lq * limb
+    modsw = batch * (2 + 2 * l) * limb
+    rcomb = batch * 6 * l * limb
+    return {"ntt_col": ntt_limbs * per_pass, "ntt_row": ntt_limbs * per_pass, "bconv": bconv,
+            "keyip": keyip, "combine": combine, "tensor": tensor, "automorphism": auto,
+            "rescale_modswitch": modsw, "rescale_combine": rcomb}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return HBM_FALLBACK, "fallback (B200_PROFILING.md)"
+
+
+def load_traffic(kind: str):
+    """dram bytes per launch of `kind` from the committed ncu --set full summary, or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(kind)
+    except Exception:
+        return None
+
+
+# ----------------------------------------------------------------------------- CPU oracle
+
+def oracle_keyswitch_rate(d, evk, budget_s=12.0, min_reps=1):
+    """Time the CPU oracle (oracle/ckks.py fast mode) on Set-B key-switches."""
+    from oracle import _core, ckks
+    prm = ckks.set_b()
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        ckks.keyswitch(prm, d, LEVEL, evk)
+        reps += 1
+        el = time.perf_counter() - t0
+        if reps >= min_reps and el >= budget_s:
+            break
+        if reps >= min_reps and el / reps * (reps + 1) > budget_s * 1.5:
+            break
+    return reps / el, reps, el, _core.lib().or_num_threads()
+
+
+# ----------------------------------------------------------------------------- reference arm
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import _core, ckks
+    prm = ckks.set_b()
+    N = prm.N
+    d = rand_limbs(prm.q, 0x4E454F, N)
+    evk = rand_evk(prm.moduli, 0x4E454F + 100, N)
+    for _ in range(args.warmup):
+        ckks.keyswitch(prm, d, LEVEL, evk)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        ckks.keyswitch(prm, d, LEVEL, evk)
+    el = time.perf_counter() - t0
+    v = args.steps / el
+    cores = _core.lib().or_num_threads()
+    line = {"metric": METRIC, "value": v, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * el / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic", "config": dict(workload_config(1, 1), workload="setB_keyswitch"),
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": "each step = one Set-B key-switch (l=35, B=1) by the CPU oracle"},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- neo arm
+
+def run_neo(args):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_isca_jiaodwfcm0z25_b200 import neo
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    B = args.batch
+    ctx = neo.Context(LOG_N, NUM_Q, NUM_P, DNUM, device=local)
+    N, Lq = ctx.N, LEVEL + 1
+    seed = 0x4E454F + 1000 * rank
+    relin_np = rand_evk(ctx.moduli, seed + 100, N)
+    rot_np = rand_evk(ctx.moduli, seed + 200, N)
+    relin = neo.EvalKey(ctx, torch.from_numpy(relin_np).cuda())
+    rot = neo.EvalKey(ctx, torch.from_numpy(rot_np).cuda())
+    qmods = ctx.q[:Lq]
+    SLOTS = 2
+    host_in = [[rand_ct(qmods, seed + 10 * s + k, N, B) for k in range(3)] for s in range(SLOTS)]
+    dev_in = [[torch.from_numpy(x).cuda() for x in slot] for slot in host_in]
+    hm_out = torch.empty((B, 2, Lq, N), dtype=torch.uint64, device="cuda")
+    rs_out = torch.empty((B, 2, LEVEL, N), dtype=torch.uint64, device="cuda")
+    hr_out = torch.empty((B, 2, Lq, N), dtype=torch.uint64, device="cuda")
+    ws_n = max(ctx.workspace_size(neo.NEO_OP_HMULT, LEVEL, B), ctx.workspace_size(neo.NEO_OP_HROT, LEVEL, B),
+               ctx.workspace_size(neo.NEO_OP_RESCALE, LEVEL, B))
+    ws = torch.empty(ws_n // 8, dtype=torch.uint64, device="cuda")
+    g = 5                                   # 5^1 mod 2N: rotate slots left by one
+
+    launches = [0]
+
+    def step(s, a=None, b=None, c=None):
+        a = dev_in[s][0] if a is None else a
+        b = dev_in[s][1] if b is None else b
+        c = dev_in[s][2] if c is None else c
+        neo.neo_hmult(ctx, relin, a, b, LEVEL, hm_out, B, ws)
+        n = neo.last_launch_count()
+        neo.neo_rescale(ctx, hm_out, LEVEL, rs_out, B, ws)
+        n += neo.last_launch_count()
+        neo.neo_hrot(ctx, rot, g, c, LEVEL, hr_out, B, ws)
+        n += neo.last_launch_count()
+        launches[0] += n
+
+    # warm-up (untimed)
+    for w in range(max(args.warmup, 1)):
+        step(w % SLOTS)
+    torch.cuda.synchronize()
+    barrier()
+    torch.cuda.synchronize()
+
+    # timed region: device time with CUDA events on the launching stream
+    launches[0] = 0
+    neo.neo_profile_enable(True)
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        t_start.record()
+        for k in range(args.steps):
+            step(k % SLOTS)
+        t_end.record()
+        torch.cuda.synchronize()
+    barrier()
+    torch.cuda.synchronize()
+    ms = t_start.elapsed_time(t_end)
+    prof = neo.neo_profile_read()
+    neo.neo_profile_enable(False)
+    gpu_launches = launches[0]
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    ms_step = ms / args.steps
+    value = 2 * B * world / (ms_step / 1e3)
+
+    # roofline of the dominant kernel kind
+    peak, peak_src = load_peaks()
+    bm = bytes_model(B)
+    step_ms = {k: v[0] / args.steps for k, v in prof.items()}
+    dom = max(step_ms, key=lambda k: step_ms[k])
+    n_launch_dom = prof[dom][1] / args.steps
+    achieved = bm[dom] / (step_ms[dom] / 1e3) / 1e9 if step_ms[dom] > 0 else None
+    traffic = load_traffic(dom)
+    breakdown = {k: {"ms_per_step": round(step_ms[k], 5), "launches_per_step": prof[k][1] / args.steps,
+                     "share": round(step_ms[k] / ms_step, 4) if ms_step > 0 else None,
+                     "algo_GBps": round(bm[k] / (step_ms[k] / 1e3) / 1e9, 1) if step_ms[k] > 0 else None,
+                     "frac_hbm": round(bm[k] / (step_ms[k] / 1e3) / 1e9 / peak, 4) if step_ms[k] > 0 else None}
+                 for k in step_ms}
+
+    # end-to-end through the public API with pinned host buffers
+    e2e = None
+    if not args.no_e2e:
+        pinned = [[torch.from_numpy(x).pin_memory() for x in slot] for slot in host_in]
+        host_rs = torch.empty(rs_out.shape, dtype=torch.uint64).pin_memory()
+        host_hr = torch.empty(hr_out.shape, dtype=torch.uint64).pin_memory()
+        stage = [torch.empty_like(x) for x in dev_in[0]]
+        k_e2e = max(3, min(args.steps, 50))
+        for w in range(2):
+            for i in range(3):
+                stage[i].copy_(pinned[w % SLOTS][i], non_blocking=True)
+            step(0, *stage)
+        torch.cuda.synchronize()
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for k in range(k_e2e):
+            for i in range(3):
+                stage[i].copy_(pinned[k % SLOTS][i], non_blocking=True)
+            step(0, *stage)
+            host_rs.copy_(rs_out, non_blocking=True)
+            host_hr.copy_(hr_out, non_blocking=True)
+        e1.record()
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1)
+        if world > 1:
+            t = torch.tensor([ems], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        h2d = sum(x.numel() * 8 for x in dev_in[0])
+        d2h = (rs_out.numel() + hr_out.numel()) * 8
+        e2e = {"value": 2 * B * world / (ems / k_e2e / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "steps": k_e2e, "ms_per_step": ems / k_e2e}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        d0 = host_in[0][2][0, 1]                                  # c1 of one ciphertext: [36][N]
+        rate, reps, el, cores = oracle_keyswitch_rate(d0, rot_np)
+        cpu = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"{reps} Set-B key-switch(es) (l=35, B=1) by the CPU oracle in {el:.1f} s"}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "u64", "data": "synthetic (uniform residues, random keys)",
+                "config": workload_config(B, world),
+                "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
+                             "peak_source": peak_src, "unit": "GB/s",
+                             "frac": achieved / peak if achieved else None, "traffic": traffic,
+                             "launches_per_step": n_launch_dom,
+                             "algo_bytes_per_step": bm[dom]},
+                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
+                "clocks": clk.summary(), "breakdown": breakdown}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_neo(args)
+
+
+if __name__ == "__main__":
+    main()

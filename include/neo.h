@@ -153,6 +153,17 @@ const char* neo_last_error(void);
  * gpu_launches accounting). */
 int32_t neo_last_launch_count(void);
 
+/* Diagnostics: when enabled (on != 0), every kernel launched by this thread is bracketed
+ * by a pair of CUDA events on its stream; enabling or disabling clears the records.
+ * neo_profile_read synchronises on the recorded events and returns the summed device
+ * time (ms) and launch count of one kernel kind:
+ *   0 NTT column pass, 1 NTT row pass, 2 BConv, 3 KeyIP, 4 combine (ModDown tail),
+ *   5 tensor, 6 automorphism, 7 rescale mod-switch, 8 rescale combine. */
+enum { NEO_PK_NTT_COL = 0, NEO_PK_NTT_ROW, NEO_PK_BCONV, NEO_PK_KEYIP, NEO_PK_COMBINE,
+       NEO_PK_TENSOR, NEO_PK_AUTO, NEO_PK_MODSW, NEO_PK_RESCALE, NEO_PK_COUNT };
+neo_status neo_profile_enable(int32_t on);
+neo_status neo_profile_read(int32_t kind, double* total_ms, int32_t* launches);
+
 #ifdef __cplusplus
 }
 #endif

@@ -33,6 +33,41 @@ static thread_local int g_launches = 0;
 
 static inline cudaStream_t S(neo_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
 
+// ------------------------------------------------------------------ launch profiling
+// Optional CUDA-event pairs around every launch (neo_profile_enable), read back per
+// kernel kind by neo_profile_read; used by bench.py to time kernels inside its timed region.
+enum { PK_NTT_COL = 0, PK_NTT_ROW, PK_BCONV, PK_KEYIP, PK_COMBINE, PK_TENSOR, PK_AUTO, PK_MODSW,
+       PK_RESCALE, PK_COUNT };
+struct ProfRec { int kind; cudaEvent_t a, b; };
+static thread_local bool g_prof = false;
+static thread_local std::vector<ProfRec> g_recs;
+static thread_local std::vector<cudaEvent_t> g_pool;
+static thread_local size_t g_pool_used = 0;
+
+static cudaEvent_t prof_event() {
+    if (g_pool_used == g_pool.size()) {
+        cudaEvent_t e;
+        cudaEventCreate(&e);
+        g_pool.push_back(e);
+    }
+    return g_pool[g_pool_used++];
+}
+struct ProfScope {
+    int kind; cudaStream_t st; cudaEvent_t a = nullptr;
+    ProfScope(int k, cudaStream_t s) : kind(k), st(s) {
+        if (g_prof) { a = prof_event(); cudaEventRecord(a, st); }
+    }
+    ~ProfScope() {
+        if (a) { cudaEvent_t b = prof_event(); cudaEventRecord(b, st); g_recs.push_back({kind, a, b}); }
+        ++g_launches;
+    }
+};
+#define LAUNCH(kind, st, expr)          \
+    do {                                \
+        ProfScope ps_((kind), (st));    \
+        CK(expr);                       \
+    } while (0)
+
 // ------------------------------------------------------------------ NTT over a row set
 // rows k < n of batch entry b: src + b*src_bs + src_off[k]*N  ->  dst + b*dst_bs + dst_off[k]*N
 static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long src_bs, const int* src_off,
@@ -53,9 +88,8 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
         b.src_off[k] = k; b.dst_off[k] = dst_off[k]; b.prime[k] = (short)prime[k];
     }
     // forward: column pass then row pass; inverse: row pass then column pass
-    CK(ntt_pass(fwd, a, c->ntt, batch, fwd, st));
-    CK(ntt_pass(!fwd, b, c->ntt, batch, fwd, st));
-    g_launches += 2;
+    LAUNCH(fwd ? PK_NTT_COL : PK_NTT_ROW, st, ntt_pass(fwd, a, c->ntt, batch, fwd, st));
+    LAUNCH(fwd ? PK_NTT_ROW : PK_NTT_COL, st, ntt_pass(!fwd, b, c->ntt, batch, fwd, st));
     return NEO_OK;
 }
 
@@ -115,8 +149,7 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
             if (std::find(dj.begin(), dj.end(), id) != dj.end()) continue;
             io.out_off[o++] = j * E + pos;
         }
-        CK(launch_bconv(T, io, N, B, st));
-        ++g_launches;
+        LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, B, st));
     }
 
     // a5: NTT of every ModUp output row
@@ -153,8 +186,7 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
                 A.src_off[j][pos] = own ? id : j * E + pos;
             }
         }
-        CK(launch_keyip(A, E, B, st));
-        ++g_launches;
+        LAUNCH(PK_KEYIP, st, launch_keyip(A, E, B, st));
     }
 
     // a7: INTT of the P part of acc_0, acc_1 -> pc [2B][P][N]
@@ -171,8 +203,7 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
         io.out_bstride = (long long)Lq * N;
         for (int i = 0; i < P; ++i) io.in_off[i] = i;
         for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
-        CK(launch_bconv(T, io, N, 2 * B, st));
-        ++g_launches;
+        LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, 2 * B, st));
     }
 
     // a9: NTT of conv (in place through tmp)
@@ -192,8 +223,7 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
         A.out_bstride = out_bs;
         A.N = N;
         for (int i = 0; i < Lq; ++i) A.pinv[i] = c->pinv[i];
-        CK(launch_combine(A, Lq, B, st));
-        ++g_launches;
+        LAUNCH(PK_COMBINE, st, launch_combine(A, Lq, B, st));
     }
     return NEO_OK;
 }
@@ -229,6 +259,30 @@ static neo_status check_ptr(const void* p, const char* what) {
 extern "C" {
 
 const char* neo_last_error(void) { return g_err.c_str(); }
+
+neo_status neo_profile_enable(int32_t on) {
+    g_recs.clear();
+    g_pool_used = 0;
+    g_prof = on != 0;
+    return NEO_OK;
+}
+
+neo_status neo_profile_read(int32_t kind, double* total_ms, int32_t* launches) {
+    if (kind < 0 || kind >= PK_COUNT || !total_ms || !launches) FAIL(NEO_EINVAL, "bad profile kind or null output");
+    double t = 0;
+    int n = 0;
+    for (const ProfRec& r : g_recs) {
+        if (r.kind != kind) continue;
+        CK(cudaEventSynchronize(r.b));
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, r.a, r.b));
+        t += ms;
+        ++n;
+    }
+    *total_ms = t;
+    *launches = n;
+    return NEO_OK;
+}
 int32_t neo_last_launch_count(void) { return g_launches; }
 
 neo_status neo_params_create(const neo_params_desc* desc, neo_ctx** out) {
@@ -355,7 +409,7 @@ neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids
     }
     for (int j = 0; j < n_out; ++j) {
         u64 t = c->mod[out_ids[j]];
-        T.tmod[j] = ModQ{t, (u64)(((u128)1 << 98) / t)};
+        T.tmod[j] = ModQ{t, (u64)(((u128)1 << 98) / t), (double)t, 1.0 / (double)t};
         for (int i = 0; i < n_in; ++i) {
             u64 f = 1;
             for (int k = 0; k < n_in; ++k)
@@ -370,8 +424,7 @@ neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids
     io.out_bstride = (long long)n_out * c->N;
     for (int i = 0; i < n_in; ++i) io.in_off[i] = i;
     for (int j = 0; j < n_out; ++j) io.out_off[j] = j;
-    CK(launch_bconv(T, io, c->N, batch, S(st)));
-    g_launches = 1;
+    LAUNCH(PK_BCONV, S(st), launch_bconv(T, io, c->N, batch, S(st)));
     return NEO_OK;
 }
 
@@ -383,8 +436,7 @@ neo_status neo_tensor(const neo_ctx* c, const uint64_t* a, const uint64_t* b, in
     TRY(check_ptr(a, "ct_a"));
     TRY(check_ptr(b, "ct_b"));
     TRY(check_ptr(d, "d"));
-    CK(launch_tensor(a, b, d, c->d_mods, level + 1, c->N, batch, S(st)));
-    g_launches = 1;
+    LAUNCH(PK_TENSOR, S(st), launch_tensor(a, b, d, c->d_mods, level + 1, c->N, batch, S(st)));
     return NEO_OK;
 }
 
@@ -396,8 +448,7 @@ neo_status neo_automorphism(const neo_ctx* c, const uint64_t* in, int32_t n_limb
     TRY(check_ptr(out, "out"));
     if (n_limbs <= 0 || batch <= 0) FAIL(NEO_EINVAL, "n_limbs and batch must be positive");
     if ((g & 1) == 0 || g >= 2u * (unsigned)c->N) FAIL(NEO_EINVAL, "galois element must be odd and < 2N");
-    CK(launch_automorph(in, out, g, c->N, n_limbs * batch, S(st)));
-    g_launches = 1;
+    LAUNCH(PK_AUTO, S(st), launch_automorph(in, out, g, c->N, n_limbs * batch, S(st)));
     return NEO_OK;
 }
 
@@ -461,8 +512,7 @@ neo_status neo_hmult(const neo_ctx* c, const neo_evk* relin, const uint64_t* ct_
     u64* dd = w + Ly.extra;
     const long long ls = (long long)(level + 1) * c->N;
     cudaStream_t s = S(st);
-    CK(launch_tensor(ct_a, ct_b, dd, c->d_mods, level + 1, c->N, batch, s));
-    g_launches = 1;
+    LAUNCH(PK_TENSOR, s, launch_tensor(ct_a, ct_b, dd, c->d_mods, level + 1, c->N, batch, s));
     return ks_core(c, relin, dd + 2 * ls, 3 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, dd, dd + ls,
                    3 * ls, s);
 }
@@ -482,8 +532,7 @@ neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint6
     u64* sc = w + Ly.extra;
     const long long ls = (long long)(level + 1) * c->N;
     cudaStream_t s = S(st);
-    CK(launch_automorph(ct_in, sc, g, c->N, 2 * (level + 1) * batch, s));
-    g_launches = 1;
+    LAUNCH(PK_AUTO, s, launch_automorph(ct_in, sc, g, c->N, 2 * (level + 1) * batch, s));
     return ks_core(c, rk, sc + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, sc, nullptr, 2 * ls, s);
 }
 
@@ -505,15 +554,13 @@ neo_status neo_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, u
     int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
     so[0] = l; dof[0] = 0; pr[0] = l;
     TRY(ntt_rows(c, false, ct_in, (long long)(l + 1) * N, so, last, N, dof, pr, 1, tmp, B2, s));
-    CK(launch_modswitch(last, r, c->d_mods, l, N, B2, s));
-    ++g_launches;
+    LAUNCH(PK_MODSW, s, launch_modswitch(last, r, c->d_mods, l, N, B2, s));
     for (int i = 0; i < l; ++i) { so[i] = dof[i] = i; pr[i] = i; }
     TRY(ntt_rows(c, true, r, (long long)l * N, so, r, (long long)l * N, dof, pr, l, tmp, B2, s));
     RescaleArgs A;
     A.in = ct_in; A.r = r; A.out = ct_out; A.mods = c->d_mods; A.N = N; A.l = l;
     for (int i = 0; i < l; ++i) A.qlinv[i] = c->ql_inv[l][i];
-    CK(launch_rescale_combine(A, B2, s));
-    ++g_launches;
+    LAUNCH(PK_RESCALE, s, launch_rescale_combine(A, B2, s));
     return NEO_OK;
 }
 

@@ -20,6 +20,7 @@ struct TW {   // a constant with its Shoup companion
 struct ModQ {  // per-limb modulus constants
     u64 q;
     u64 mu;    // floor(2^98 / q)
+    double qd, qinv;   // q and fl(1/q)
 };
 
 #define NEO_DEV __device__ __forceinline__
@@ -49,6 +50,44 @@ NEO_DEV u64 barrett_reduce(u64 hi, u64 lo, ModQ m) {
 NEO_DEV u64 mul_mod(u64 a, u64 b, ModQ m) {     // a, b < 2^62 with a*b < 2^98
     return barrett_reduce(__umul64hi(a, b), a * b, m);
 }
+// ---------------------------------------------------------------------------
+// FP64 residue arithmetic.  A residue (or a lazy, signed representative of one) is held
+// exactly in a double while |x| < 2^50.  Multiplication by a constant w < q uses the pair
+// (w, wq = fl(w/q)):  h = fl(a w), l = a w - h (exact, FMA), qf = round(a wq) (magic-number
+// rounding), r = (h - qf q) + l.  For integral |a| < 2^45 every step is exact except the
+// quotient estimate, |qf - a w / q| <= 0.625, so r == a w (mod q) with |r| <= 0.625 q.
+// (DESIGN.md "FP64 residue arithmetic".)  sm_100a issues 63 DFMA/clk/SM vs ~2.2 64-bit
+// integer Shoup butterflies/clk/SM (tools/microbench/pipes.cu), hence FP64.
+struct TWD {   // constant w < q and fl(w / q)
+    double w, wq;
+};
+constexpr double kMagic = 6755399441055744.0;      // 1.5 * 2^52: fma(x, y, M) - M = round(x y)
+constexpr double kTwo52 = 4503599627370496.0;
+
+NEO_DEV double u2d(u64 x) {                         // exact for x < 2^52
+    return __dadd_rn(__longlong_as_double((long long)(x | 0x4330000000000000ull)), -kTwo52);
+}
+NEO_DEV u64 d2u(double r) {                         // 0 <= r < 2^52, integral
+    return (u64)__double_as_longlong(__dadd_rn(r, kTwo52)) - 0x4330000000000000ull;
+}
+NEO_DEV double mulc(double a, TWD t, double q) {    // a * w mod q, |result| <= 0.625 q
+    const double h = __dmul_rn(a, t.w);
+    const double l = __fma_rn(a, t.w, -h);
+    const double qf = __dadd_rn(__fma_rn(a, t.wq, kMagic), -kMagic);
+    return __dadd_rn(__fma_rn(-qf, q, h), l);
+}
+NEO_DEV double mulv(double a, double b, double q, double qinv) {   // a * b mod q, |a|,|b| < 2^37
+    const double h = __dmul_rn(a, b);
+    const double l = __fma_rn(a, b, -h);
+    const double qf = __dadd_rn(__fma_rn(h, qinv, kMagic), -kMagic);
+    return __dadd_rn(__fma_rn(-qf, q, h), l);
+}
+NEO_DEV double canon(double x, double q, double qinv) {   // |x| < 2^50 integral -> [0, q)
+    const double qf = __dadd_rn(__fma_rn(x, qinv, kMagic), -kMagic);
+    const double r = __fma_rn(-qf, q, x);                   // exact, |r| <= q/2 + 1
+    return r < 0.0 ? __dadd_rn(r, q) : (r >= q ? __dadd_rn(r, -q) : r);
+}
+
 // 128-bit accumulator helpers
 NEO_DEV void mac128(u64& hi, u64& lo, u64 a, u64 b) {
     u64 l = a * b, h = __umul64hi(a, b);

@@ -43,7 +43,7 @@ struct neo_ctx {
     std::vector<u64> psi;                 // by limb id
     std::vector<ModQ> h_mods;
     NttLayout L;
-    TW* d_tab = nullptr;                  // [limb id][L.total]
+    TWD* d_tab = nullptr;                 // [limb id][L.total]
     ModQ* d_mods = nullptr;
     neo::NttArgs ntt;
     // per level l (index l = 0..num_q-1)

@@ -6,7 +6,7 @@
 namespace neo {
 
 struct NttArgs {
-    const TW* tab;        // device: [limb id][L.total] twiddle blocks
+    const TWD* tabd;      // device: [limb id][L.total] twiddle blocks (w, w/q) in FP64
     long long tab_stride; // = L.total
     const ModQ* mods;     // device: per limb id
     int N, N1, N2;

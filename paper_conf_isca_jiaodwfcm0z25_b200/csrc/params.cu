@@ -74,6 +74,7 @@ u64 min_psi(u64 q, u64 n) {
 }
 
 static TW mk_tw(u64 w, u64 q) { return TW{w, (u64)(((u128)w << 64) / q)}; }
+static TWD mk_twd(u64 w, u64 q) { return TWD{(double)w, (double)w / (double)q}; }   // both exact < 2^53
 
 static int brev(int x, int R) {
     int lg = 0;
@@ -84,7 +85,7 @@ static int brev(int x, int R) {
 }
 
 // Fill one prime's twiddle block (formulas documented in ntt_tables.h).
-static void fill_ntt_block(TW* t, const NttLayout& L, u64 q, u64 psi, int N) {
+static void fill_ntt_block(TWD* t, const NttLayout& L, u64 q, u64 psi, int N) {
     const int R = L.R, N1 = L.N1, N2 = L.N2;
     const u64 ipsi = invm(psi, q);
     auto P = [&](u64 base, long long e) { return powm(base, (u64)e, q); };
@@ -95,31 +96,31 @@ static void fill_ntt_block(TW* t, const NttLayout& L, u64 q, u64 psi, int N) {
     const u64 om2R = P(om2, R), iom2R = P(iom2, R);
     const u64 ninv = invm((u64)N % q, q);
     for (int k = 0; k < R; ++k) {
-        t[L.colf_neg + k] = mk_tw(P(rho, brev(k, R)), q);
-        t[L.coli_neg + k] = mk_tw(P(irho, brev(k, R)), q);
+        t[L.colf_neg + k] = mk_twd(P(rho, brev(k, R)), q);
+        t[L.coli_neg + k] = mk_twd(P(irho, brev(k, R)), q);
     }
     for (int r = 0; r < R; ++r)
         for (int x = 0; x < R; ++x) {
-            t[L.colf_tw1 + r * R + x] = mk_tw(P(psi1, (long long)(2 * x + 1) * r), q);
-            t[L.coli_tw1 + r * R + x] = mk_tw(P(ipsi1, (long long)(2 * r + 1) * x), q);
-            t[L.rowf_tw2 + r * R + x] = mk_tw(P(om2, (long long)x * r), q);
-            t[L.rowi_tw2 + r * R + x] = mk_tw(P(iom2, (long long)x * r), q);
+            t[L.colf_tw1 + r * R + x] = mk_twd(P(psi1, (long long)(2 * x + 1) * r), q);
+            t[L.coli_tw1 + r * R + x] = mk_twd(P(ipsi1, (long long)(2 * r + 1) * x), q);
+            t[L.rowf_tw2 + r * R + x] = mk_twd(P(om2, (long long)x * r), q);
+            t[L.rowi_tw2 + r * R + x] = mk_twd(P(iom2, (long long)x * r), q);
         }
     for (int j = 0; j < R / 2; ++j) {
-        t[L.colf_cyc + j] = mk_tw(P(om1, j), q);
-        t[L.coli_cyc + j] = mk_tw(P(iom1, j), q);
-        t[L.rowf_cyc + j] = mk_tw(P(om2R, j), q);
-        t[L.rowi_cyc + j] = mk_tw(P(iom2R, j), q);
+        t[L.colf_cyc + j] = mk_twd(P(om1, j), q);
+        t[L.coli_cyc + j] = mk_twd(P(iom1, j), q);
+        t[L.rowf_cyc + j] = mk_twd(P(om2R, j), q);
+        t[L.rowi_cyc + j] = mk_twd(P(iom2R, j), q);
     }
     const u64 two_n = 2ull * N;
     for (int n2 = 0; n2 < N2; ++n2)
         for (int r = 0; r < R; ++r) {
             u64 ea = ((u64)(2 * r + 1) * n2) % two_n;
             u64 eb = ((u64)2 * R * r * n2) % two_n;          // here r plays ib
-            t[L.outf_a + n2 * R + r] = mk_tw(P(psi, ea), q);
-            t[L.outf_b + n2 * R + r] = mk_tw(P(psi, eb), q);
-            t[L.outi_a + n2 * R + r] = mk_tw(mulm(ninv, P(ipsi, ea), q), q);
-            t[L.outi_b + n2 * R + r] = mk_tw(P(ipsi, eb), q);
+            t[L.outf_a + n2 * R + r] = mk_twd(P(psi, ea), q);
+            t[L.outf_b + n2 * R + r] = mk_twd(P(psi, eb), q);
+            t[L.outi_a + n2 * R + r] = mk_twd(mulm(ninv, P(ipsi, ea), q), q);
+            t[L.outi_b + n2 * R + r] = mk_twd(P(ipsi, eb), q);
         }
 }
 
@@ -127,6 +128,8 @@ static ModQ mk_mod(u64 q) {
     ModQ m;
     m.q = q;
     m.mu = (u64)(((u128)1 << 98) / q);
+    m.qd = (double)q;
+    m.qinv = 1.0 / (double)q;
     return m;
 }
 
@@ -190,20 +193,20 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
     c->L = make_ntt_layout(c->log_n);
 
     // ---- device tables
-    std::vector<TW> tab((size_t)nl * c->L.total);
+    std::vector<TWD> tab((size_t)nl * c->L.total);
     for (int i = 0; i < nl; ++i) fill_ntt_block(&tab[(size_t)i * c->L.total], c->L, c->mod[i], c->psi[i], c->N);
     if (cudaSetDevice(c->device) != cudaSuccess) { err = "cudaSetDevice failed"; return NEO_ECUDA; }
-    if (cudaMalloc(&c->d_tab, tab.size() * sizeof(TW)) != cudaSuccess ||
+    if (cudaMalloc(&c->d_tab, tab.size() * sizeof(TWD)) != cudaSuccess ||
         cudaMalloc(&c->d_mods, nl * sizeof(ModQ)) != cudaSuccess) {
         err = "cudaMalloc of constant tables failed";
         return NEO_ENOMEM;
     }
-    if (cudaMemcpy(c->d_tab, tab.data(), tab.size() * sizeof(TW), cudaMemcpyHostToDevice) != cudaSuccess ||
+    if (cudaMemcpy(c->d_tab, tab.data(), tab.size() * sizeof(TWD), cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemcpy(c->d_mods, c->h_mods.data(), nl * sizeof(ModQ), cudaMemcpyHostToDevice) != cudaSuccess) {
         err = "cudaMemcpy of constant tables failed";
         return NEO_ECUDA;
     }
-    c->ntt.tab = c->d_tab;
+    c->ntt.tabd = c->d_tab;
     c->ntt.tab_stride = c->L.total;
     c->ntt.mods = c->d_mods;
     c->ntt.N = c->N;

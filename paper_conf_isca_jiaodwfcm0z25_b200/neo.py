@@ -23,7 +23,9 @@ _STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM",
 EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_workspace_size",
             "neo_ntt", "neo_intt", "neo_bconv", "neo_tensor", "neo_automorphism", "neo_evk_create",
             "neo_evk_destroy", "neo_keyswitch", "neo_hmult", "neo_hrot", "neo_rescale",
-            "neo_last_error", "neo_last_launch_count")
+            "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read")
+PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
+                 "rescale_modswitch", "rescale_combine")
 
 
 class NeoError(RuntimeError):
@@ -77,6 +79,10 @@ def lib() -> ctypes.CDLL:
         L.neo_last_error.argtypes = []
         L.neo_last_launch_count.restype = _i32
         L.neo_last_launch_count.argtypes = []
+        L.neo_profile_enable.argtypes = [_i32]
+        L.neo_profile_enable.restype = ctypes.c_int
+        L.neo_profile_read.argtypes = [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int32)]
+        L.neo_profile_read.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -106,6 +112,20 @@ def _ids(ids) -> ctypes.Array:
 
 def last_launch_count() -> int:
     return int(lib().neo_last_launch_count())
+
+
+def neo_profile_enable(on: bool):
+    _check(lib().neo_profile_enable(1 if on else 0), "neo_profile_enable")
+
+
+def neo_profile_read() -> dict:
+    """{kind: (total_ms, launches)} for every kernel kind recorded since neo_profile_enable."""
+    out = {}
+    for k, name in enumerate(PROFILE_KINDS):
+        ms, n = ctypes.c_double(), ctypes.c_int32()
+        _check(lib().neo_profile_read(k, ctypes.byref(ms), ctypes.byref(n)), "neo_profile_read")
+        out[name] = (ms.value, n.value)
+    return out
 
 
 class Context:
