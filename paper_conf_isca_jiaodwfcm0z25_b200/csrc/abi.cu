@@ -5,6 +5,7 @@
 #include <new>
 #include <string>
 
+#include "bconv_tc.h"
 #include "context.h"
 #include "kernels.h"
 #include "ntt.h"
@@ -149,7 +150,11 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
             if (std::find(dj.begin(), dj.end(), id) != dj.end()) continue;
             io.out_off[o++] = j * E + pos;
         }
-        LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, B, st));
+        if (c->use_tc)
+            LAUNCH(PK_BCONV, st, launch_bconv_tc(c->modup_tc[l][j], io, c->d_bmat + c->modup_boff[l][j], nullptr, N, B,
+                                                 c->num_sms, st));
+        else
+            LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, B, st));
     }
 
     // a5: NTT of every ModUp output row
@@ -203,7 +208,11 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
         io.out_bstride = (long long)Lq * N;
         for (int i = 0; i < P; ++i) io.in_off[i] = i;
         for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
-        LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, 2 * B, st));
+        if (c->use_tc)
+            LAUNCH(PK_BCONV, st, launch_bconv_tc(c->moddown_tc[l], io, c->d_bmat + c->moddown_boff[l], nullptr, N,
+                                                 2 * B, c->num_sms, st));
+        else
+            LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, 2 * B, st));
     }
 
     // a9: NTT of conv (in place through tmp)
@@ -321,6 +330,7 @@ neo_status neo_params_destroy(neo_ctx* c) {
     if (!c) return NEO_OK;
     if (c->d_tab) cudaFree(c->d_tab);
     if (c->d_mods) cudaFree(c->d_mods);
+    if (c->d_bmat) cudaFree(c->d_bmat);
     delete c;
     return NEO_OK;
 }
@@ -424,7 +434,20 @@ neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids
     io.out_bstride = (long long)n_out * c->N;
     for (int i = 0; i < n_in; ++i) io.in_off[i] = i;
     for (int j = 0; j < n_out; ++j) io.out_off[j] = j;
-    LAUNCH(PK_BCONV, S(st), launch_bconv(T, io, c->N, batch, S(st)));
+    if (c->use_tc && n_in <= BCTC_MAX_IN && n_out <= BCTC_MAX_OUT) {
+        std::vector<u64> sm, tm;
+        for (int i = 0; i < n_in; ++i) sm.push_back(c->mod[in_ids[i]]);
+        for (int j = 0; j < n_out; ++j) tm.push_back(c->mod[out_ids[j]]);
+        BConvTC P;
+        std::vector<uint8_t> bm;
+        make_bconv_tc(sm, tm, P, bm);
+        static thread_local BMatParam bp;
+        std::memset(&bp, 0, sizeof(bp));
+        std::memcpy(&bp, bm.data(), bm.size());
+        LAUNCH(PK_BCONV, S(st), launch_bconv_tc(P, io, nullptr, &bp, c->N, batch, c->num_sms, S(st)));
+    } else {
+        LAUNCH(PK_BCONV, S(st), launch_bconv(T, io, c->N, batch, S(st)));
+    }
     return NEO_OK;
 }
 

@@ -35,6 +35,21 @@ struct BConvIO {
     int out_off[BC_MAX_OUT];
 };
 
+constexpr int BCTC_MAX_IN = 12;     // K = 5 * n_in <= 64
+constexpr int BCTC_MAX_OUT = 51;    // N = 5 * n_out <= 256
+
+struct BConvTC {
+    int n_in, n_out, ncols;         // ncols = MMA N = round_up(5 n_out, 16)
+    double qin[BCTC_MAX_IN], qinv_in[BCTC_MAX_IN];
+    TWD qhat_inv[BCTC_MAX_IN];      // [qhat_i^-1]_{q_i}
+    double t[BCTC_MAX_OUT], tinv[BCTC_MAX_OUT];
+    TWD c24[BCTC_MAX_OUT];          // 2^24 mod t
+};
+
+struct BMatParam {                   // B passed by value (generic neo_bconv, no device tables)
+    uint4 d[256 * 64 / 16];
+};
+
 }  // namespace neo
 
 struct neo_ctx {
@@ -51,6 +66,14 @@ struct neo_ctx {
     std::vector<std::vector<std::vector<int>>> digits;  // [l][j] -> limb ids
     std::vector<neo::BConvTab> moddown;              // [l]: P limbs -> q_0..q_l
     std::vector<TW> pinv;                            // [i] P^-1 mod q_i (Shoup)
+    // tensor-core BConv (bconv_tc.cu): constants and device byte matrices per (l, j) / l
+    std::vector<std::vector<neo::BConvTC>> modup_tc;
+    std::vector<neo::BConvTC> moddown_tc;
+    std::vector<std::vector<size_t>> modup_boff;     // byte offsets into d_bmat
+    std::vector<size_t> moddown_boff;
+    uint8_t* d_bmat = nullptr;
+    int num_sms = 148;
+    bool use_tc = true;                              // NEO_BCONV=cuda selects the CUDA-core control kernel
     std::vector<std::vector<TW>> ql_inv;             // [l][i] q_l^-1 mod q_i, i < l
 
     int beta(int level) const { return (level + 1 + alpha - 1) / alpha; }

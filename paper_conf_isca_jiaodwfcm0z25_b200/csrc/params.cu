@@ -9,6 +9,9 @@
 #include <cstring>
 #include <stdexcept>
 
+#include <cstdlib>
+
+#include "bconv_tc.h"
 #include "context.h"
 
 namespace neo {
@@ -161,6 +164,43 @@ static BConvTab make_bconv(const neo_ctx* c, const std::vector<int>& src, const 
     return b;
 }
 
+// Tensor-core BConv constants (bconv_tc.cu): B[n = 5t + b][k = 5i + a] =
+// byte_b((2^(8a) qhat_i) mod t) in the SWIZZLE_NONE K-major core-matrix layout.
+void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BConvTC& P, std::vector<uint8_t>& bmat) {
+    std::memset(&P, 0, sizeof(P));
+    P.n_in = (int)src.size();
+    P.n_out = (int)dst.size();
+    P.ncols = ((5 * P.n_out + 15) / 16) * 16;
+    bmat.assign((size_t)P.ncols * 64, 0);
+    for (int i = 0; i < P.n_in; ++i) {
+        u64 qi = src[i], qh = 1;
+        for (int k = 0; k < P.n_in; ++k)
+            if (k != i) qh = mulm(qh, src[k] % qi, qi);
+        P.qin[i] = (double)qi;
+        P.qinv_in[i] = 1.0 / (double)qi;
+        P.qhat_inv[i] = mk_twd(invm(qh, qi), qi);
+    }
+    for (int t = 0; t < P.n_out; ++t) {
+        u64 m = dst[t];
+        P.t[t] = (double)m;
+        P.tinv[t] = 1.0 / (double)m;
+        P.c24[t] = mk_twd((1ull << 24) % m, m);
+        for (int i = 0; i < P.n_in; ++i) {
+            u64 f = 1;                                          // qhat_i mod t
+            for (int k = 0; k < P.n_in; ++k)
+                if (k != i) f = mulm(f, src[k] % m, m);
+            for (int a = 0; a < 5; ++a) {
+                u64 v = mulm(f, (1ull << (8 * a)) % m, m);      // (2^(8a) qhat_i) mod t
+                for (int b = 0; b < 5; ++b) {
+                    int n = 5 * t + b, k = 5 * i + a;
+                    size_t off = (size_t)(n / 8) * 512 + (k / 16) * 128 + (n % 8) * 16 + (k % 16);
+                    bmat[off] = (uint8_t)((v >> (8 * b)) & 0xFF);
+                }
+            }
+        }
+    }
+}
+
 // Build everything; throws std::runtime_error / returns status through abi.cpp.
 neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err) {
     c->log_n = d->log_n;
@@ -236,6 +276,52 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
         }
         c->moddown[l] = make_bconv(c, pids, qids);
         for (int i = 0; i < l; ++i) c->ql_inv[l].push_back(mk_tw(invm(c->mod[l] % c->mod[i], c->mod[i]), c->mod[i]));
+    }
+    // tensor-core BConv tables (used when alpha <= 12 and every conversion has <= 51 targets)
+    {
+        const char* e = std::getenv("NEO_BCONV");
+        c->use_tc = !(e && std::string(e) == "cuda");
+        int dev_sms = 0;
+        cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
+        if (dev_sms > 0) c->num_sms = dev_sms;
+        std::vector<uint8_t> all, bm;
+        c->modup_tc.resize(c->num_q);
+        c->modup_boff.resize(c->num_q);
+        c->moddown_tc.resize(c->num_q);
+        c->moddown_boff.resize(c->num_q);
+        std::vector<u64> pm;
+        for (int k = 0; k < c->num_p; ++k) pm.push_back(c->mod[c->num_q + k]);
+        bool fits = c->alpha <= BCTC_MAX_IN && c->num_p <= BCTC_MAX_IN;
+        for (int l = 0; l < c->num_q && fits; ++l) {
+            std::vector<u64> qm(c->mod.begin(), c->mod.begin() + l + 1);
+            for (int j = 0; j < c->beta(l); ++j) {
+                std::vector<u64> sm, tm;
+                const std::vector<int>& dj = c->digits[l][j];
+                for (int id : dj) sm.push_back(c->mod[id]);
+                for (int pos = 0; pos < c->ext(l); ++pos) {
+                    int id = c->ext_id(l, pos);
+                    if (std::find(dj.begin(), dj.end(), id) == dj.end()) tm.push_back(c->mod[id]);
+                }
+                if ((int)tm.size() > BCTC_MAX_OUT) { fits = false; break; }
+                BConvTC P;
+                make_bconv_tc(sm, tm, P, bm);
+                c->modup_tc[l].push_back(P);
+                c->modup_boff[l].push_back(all.size());
+                all.insert(all.end(), bm.begin(), bm.end());
+            }
+            if ((int)qm.size() > BCTC_MAX_OUT) { fits = false; break; }
+            make_bconv_tc(pm, qm, c->moddown_tc[l], bm);
+            c->moddown_boff[l] = all.size();
+            all.insert(all.end(), bm.begin(), bm.end());
+        }
+        if (!fits) c->use_tc = false;
+        if (!all.empty()) {
+            if (cudaMalloc(&c->d_bmat, all.size()) != cudaSuccess) { err = "cudaMalloc of BConv tables failed"; return NEO_ENOMEM; }
+            if (cudaMemcpy(c->d_bmat, all.data(), all.size(), cudaMemcpyHostToDevice) != cudaSuccess) {
+                err = "cudaMemcpy of BConv tables failed";
+                return NEO_ECUDA;
+            }
+        }
     }
     c->pinv.resize(c->num_q);
     for (int i = 0; i < c->num_q; ++i) {
