@@ -10,16 +10,33 @@
 // butterfly costs 8 DFMA-pipe ops and the B200 FP64 pipe runs 63 ops/clk/SM.  Values stay
 // lazy (signed, |x| < 16q) inside a pass; the intermediate buffer between the two passes
 // holds those doubles; the ABI-facing side of each pass holds canonical uint64.
+//
+// Both passes are persistent kernels (2 CTAs/SM) that walk their tiles in limb-major order
+// through a two-stage cp.async pipeline: tile t+1 (data, per-prime twiddles, the outer
+// twist slice) streams into shared memory while tile t is transformed, so HBM traffic
+// overlaps the FP64 work.  Tile = 16 columns x N1 rows (column pass) or 16 rows x N2
+// (row pass) = 32 KB at N = 2^16; every global access is a full 128-byte segment.
+#include <cstdlib>
+
 #include "common.cuh"
-#include "ntt_tables.h"
 #include "ntt.h"
+#include "ntt_tables.h"
 
 namespace neo {
+
+// ------------------------------------------------------------------ cp.async
+NEO_DEV uint32_t s_u32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+NEO_DEV void cp16(void* s, const void* g) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s_u32(s)), "l"(g) : "memory");
+}
+NEO_DEV void cp_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+NEO_DEV void cp_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
 
 // ------------------------------------------------------------------ in-register transforms
 
 // Negacyclic R-point forward NTT (Cooley-Tukey, merged psi): natural in, bit-reversed out.
-// tab[k] = rho^bitrev(k) (k = 1..R-1), rho a primitive 2R-th root.  |out| <= |in| + R/2... see DESIGN.
+// tab[k] = rho^bitrev(k) (k = 1..R-1), rho a primitive 2R-th root.
 template <int R>
 NEO_DEV void neg_fwd(double (&a)[R], const TWD* tab, double q) {
     int t = R;
@@ -82,210 +99,302 @@ NEO_DEV void cyc_dif(double (&a)[R], const TWD* tab, double q) {
     }
 }
 
+// ------------------------------------------------------------------ tiling
+
+constexpr int kC = 16;   // columns per column-pass tile / rows per row-pass tile
+
+struct TileMap {        // rows (b, k) in limb-major order: consecutive tiles share a prime
+    int batch, tpr, total;
+    NEO_DEV void decode(int t, int& b, int& k, int& blk) const {
+        const int ri = t / tpr;
+        blk = t - ri * tpr;
+        k = ri / batch;
+        b = ri - k * batch;
+    }
+};
+
+// 16-byte chunk swizzle for [row][16 doubles] tiles read/written column-wise
+NEO_DEV int swz(int row, int col) { return row * 16 + ((((col >> 1) ^ (row & 7)) << 1) | (col & 1)); }
+
 // ------------------------------------------------------------------ column pass
 
-constexpr int kCols = 16;     // columns per CTA (column pass)
-constexpr int kRows = 16;     // rows per CTA (row pass)
-
 template <int R>
-struct ColSmem {
+struct ColCfg {
+    static constexpr int NT = kC * R;
     static constexpr int NS = R + R * R + R / 2;        // neg, tw1, cyc
-    static constexpr int NO = 2 * kCols * R;            // outer A, B for this CTA's columns
+    static constexpr int NO = 2 * kC * R;               // outer twist A, B for the tile's columns
     static constexpr int XP = R * R + 1;                // odd pitch: conflict-free exchange
-    static constexpr size_t bytes = (size_t)(NS + NO) * sizeof(TWD) + (size_t)kCols * XP * sizeof(double);
+    static constexpr int DATA = kC * XP;                // doubles (>= R*R*kC)
+    static constexpr size_t STAGE = (size_t)(NS + NO) * sizeof(TWD) + (size_t)DATA * 8;
 };
 
 // Forward: src = canonical u64 coefficients, dst = lazy doubles tmp[i1][n2].
 // Inverse: src = lazy doubles tmp[i1][n2], dst = canonical u64 coefficients.
-template <int R, bool FWD>
-__global__ void __launch_bounds__(kCols * R)
-k_ntt_col(RowSet rs, NttArgs a) {
-    using SM = ColSmem<R>;
-    constexpr int C = kCols;
+template <int R, bool FWD, int STAGES, int MINB>
+__global__ void __launch_bounds__(ColCfg<R>::NT, MINB)
+k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
+    using CF = ColCfg<R>;
+    constexpr int C = kC, NT = CF::NT;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    TWD* stab = reinterpret_cast<TWD*>(smem_raw);
-    TWD* sA = stab + SM::NS;
-    TWD* sB = sA + C * R;
-    double* sx = reinterpret_cast<double*>(sB + C * R);
-
-    const int k = blockIdx.y, b = blockIdx.z;
-    const int lid = rs.prime[k];
-    const ModQ mq = a.mods[lid];
-    const double q = mq.qd;
-    const TWD* ptab = a.tabd + (size_t)lid * a.tab_stride;
-    const u64* __restrict__ src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N;
-    u64* __restrict__ dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * a.N;
-    const int N2 = a.N2;
     const int tid = threadIdx.x, c = tid % C, r = tid / C;
-    const int col0 = blockIdx.x * C;
-    const int n2 = col0 + c;
+    const int N1 = a.N1, N2 = a.N2;
 
-    // element loads first (longest latency), then the constant tables
-    double x[R];
-    if (FWD) {
-#pragma unroll
-        for (int na = 0; na < R; ++na) x[na] = u2d(src[(size_t)(R * na + r) * N2 + n2]);
-    } else {
-        const double* s = reinterpret_cast<const double*>(src);
-#pragma unroll
-        for (int ib = 0; ib < R; ++ib) x[ib] = s[(size_t)(r + R * ib) * N2 + n2];
-    }
-    {
-        const int off = FWD ? a.L.colf_neg : a.L.coli_neg;         // neg, tw1, cyc contiguous
-        for (int e = tid; e < SM::NS; e += blockDim.x) stab[e] = ptab[off + e];
-        const int oa = (FWD ? a.L.outf_a : a.L.outi_a) + col0 * R;
-        const int ob = (FWD ? a.L.outf_b : a.L.outi_b) + col0 * R;
-        for (int e = tid; e < C * R; e += blockDim.x) {
-            sA[e] = ptab[oa + e];
-            sB[e] = ptab[ob + e];
+    auto stage_ptr = [&](int s) { return smem_raw + s * CF::STAGE; };
+    auto issue = [&](int t, int s) {
+        if (t < tm.total) {
+            int b, k, blk;
+            tm.decode(t, b, k, blk);
+            const int lid = rs.prime[k];
+            const TWD* ptab = a.tabd + (size_t)lid * a.tab_stride;
+            unsigned char* st = stage_ptr(s);
+            TWD* sT = reinterpret_cast<TWD*>(st);
+            double* sD = reinterpret_cast<double*>(st + (CF::NS + CF::NO) * sizeof(TWD));
+            const int col0 = blk * C;
+            const int off = FWD ? a.L.colf_neg : a.L.coli_neg;
+            for (int e = tid; e < CF::NS; e += NT) cp16(sT + e, ptab + off + e);
+            const int oa = (FWD ? a.L.outf_a : a.L.outi_a) + col0 * R;
+            const int ob = (FWD ? a.L.outf_b : a.L.outi_b) + col0 * R;
+            for (int e = tid; e < C * R; e += NT) {       // [c][x] in memory -> [x][c] in smem (no conflicts)
+                const int cc = e / R, xx = e % R;
+                cp16(sT + CF::NS + xx * C + cc, ptab + oa + e);
+                cp16(sT + CF::NS + C * R + xx * C + cc, ptab + ob + e);
+            }
+            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N + col0;
+            for (int e = tid; e < N1 * (C / 2); e += NT) {
+                const int row = e / (C / 2), part = e % (C / 2);
+                cp16(sD + row * C + 2 * part, src + (size_t)row * N2 + 2 * part);
+            }
         }
-    }
-    __syncthreads();
-    const TWD* NEG = stab;
-    const TWD* TW1 = stab + R;
-    const TWD* CYC = stab + R + R * R;
-    double* S = sx + c * SM::XP;
+        cp_commit();
+    };
 
-    if (FWD) {
-        neg_fwd<R>(x, NEG, q);
+    const int G = gridDim.x;
+    int t = blockIdx.x;
 #pragma unroll
-        for (int ia = 0; ia < R; ++ia) S[ia * R + r] = mulc(x[BitRev<R>::of(ia)], TW1[r * R + ia], q);
+    for (int s = 0; s < STAGES; ++s) issue(t + s * G, s);
+    for (int it = 0; t < tm.total; t += G, ++it) {
+        const int s = it % STAGES;
+        cp_wait<STAGES - 1>();
         __syncthreads();
+        int b, k, blk;
+        tm.decode(t, b, k, blk);
+        const int lid = rs.prime[k];
+        const ModQ mq = a.mods[lid];
+        const double q = mq.qd;
+        unsigned char* st = stage_ptr(s);
+        const TWD* NEG = reinterpret_cast<const TWD*>(st);
+        const TWD* TW1 = NEG + R;
+        const TWD* CYC = NEG + R + R * R;
+        const TWD* sA = NEG + CF::NS;
+        const TWD* sB = sA + C * R;
+        double* sD = reinterpret_cast<double*>(st + (CF::NS + CF::NO) * sizeof(TWD));
+        double* S = sD + c * CF::XP;
+        const int n2 = blk * C + c;
+        u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * a.N;
+        double x[R];
+        if (FWD) {
+            const u64* d64 = reinterpret_cast<const u64*>(sD);
 #pragma unroll
-        for (int nb = 0; nb < R; ++nb) x[nb] = S[r * R + nb];
-        cyc_dif<R>(x, CYC, q);
-        const TWD ta = sA[c * R + r];
-        double* d = reinterpret_cast<double*>(dst);
+            for (int na = 0; na < R; ++na) x[na] = u2d(d64[(R * na + r) * C + c]);
+            neg_fwd<R>(x, NEG, q);
+            __syncthreads();                               // tile consumed: exchange in place
 #pragma unroll
-        for (int ib = 0; ib < R; ++ib) {
-            const double v = mulc(mulc(x[BitRev<R>::of(ib)], ta, q), sB[c * R + ib], q);
-            d[(size_t)(r + R * ib) * N2 + n2] = v;
+            for (int ia = 0; ia < R; ++ia) S[ia * R + r] = mulc(x[BitRev<R>::of(ia)], TW1[r * R + ia], q);
+            __syncthreads();
+#pragma unroll
+            for (int nb = 0; nb < R; ++nb) x[nb] = S[r * R + nb];
+            cyc_dif<R>(x, CYC, q);
+            const TWD ta = sA[r * C + c];
+            double* dd = reinterpret_cast<double*>(dst);
+#pragma unroll
+            for (int ib = 0; ib < R; ++ib)
+                dd[(size_t)(r + R * ib) * N2 + n2] = mulc(mulc(x[BitRev<R>::of(ib)], ta, q), sB[ib * C + c], q);
+        } else {
+            const TWD ta = sA[r * C + c];
+#pragma unroll
+            for (int ib = 0; ib < R; ++ib) x[ib] = mulc(mulc(sD[(r + R * ib) * C + c], ta, q), sB[ib * C + c], q);
+            cyc_dif<R>(x, CYC, q);
+            __syncthreads();
+#pragma unroll
+            for (int nb = 0; nb < R; ++nb) S[nb * R + r] = mulc(x[BitRev<R>::of(nb)], TW1[r * R + nb], q);
+            __syncthreads();
+#pragma unroll
+            for (int j = 0; j < R; ++j) x[j] = S[r * R + BitRev<R>::of(j)];
+            neg_inv<R>(x, NEG, q);
+#pragma unroll
+            for (int na = 0; na < R; ++na) dst[(size_t)(R * na + r) * N2 + n2] = d2u(canon(x[na], q, mq.qinv));
         }
-    } else {
-        const TWD ta = sA[c * R + r];
-#pragma unroll
-        for (int ib = 0; ib < R; ++ib) x[ib] = mulc(mulc(x[ib], ta, q), sB[c * R + ib], q);
-        cyc_dif<R>(x, CYC, q);
-#pragma unroll
-        for (int nb = 0; nb < R; ++nb) S[nb * R + r] = mulc(x[BitRev<R>::of(nb)], TW1[r * R + nb], q);
-        __syncthreads();
-#pragma unroll
-        for (int j = 0; j < R; ++j) x[j] = S[r * R + BitRev<R>::of(j)];
-        neg_inv<R>(x, NEG, q);
-#pragma unroll
-        for (int na = 0; na < R; ++na) dst[(size_t)(R * na + r) * N2 + n2] = d2u(canon(x[na], q, mq.qinv));
+        __syncthreads();                                   // stage s free
+        issue(t + STAGES * G, s);
     }
+    cp_wait<0>();
 }
 
 // ------------------------------------------------------------------ row pass
 
 template <int R>
-struct RowSmem {
+struct RowCfg {
+    static constexpr int NT = kC * R;
     static constexpr int NS = R / 2 + R * R;            // cyc, tw2
-    static constexpr int XP = R * R + 1;
-    static constexpr int TP = kRows + 1;
-    static size_t bytes(int N2) {
-        size_t xb = (size_t)kRows * XP * sizeof(double), tb = (size_t)N2 * TP * sizeof(double);
-        return (size_t)NS * sizeof(TWD) + (xb > tb ? xb : tb);
-    }
+    static constexpr int EP = R + 1;                    // exchange: element (ia, nb) at ia + EP*nb
+    static constexpr int XP = R * EP + 1;               // per-row region, odd
+    static constexpr int N2 = R * R;
+    static constexpr int DATA = (kC * XP > N2 * kC) ? kC * XP : N2 * kC;
+    static constexpr size_t STAGE = (size_t)NS * sizeof(TWD) + (size_t)DATA * 8;
 };
 
 // Forward: src = lazy doubles tmp[i1][n2], dst = canonical u64 a_hat[i1 + N1 i2].
 // Inverse: src = canonical u64 a_hat, dst = lazy doubles tmp[i1][n2].
-template <int R, bool FWD>
-__global__ void __launch_bounds__(kRows * R)
-k_ntt_row(RowSet rs, NttArgs a) {
-    using SM = RowSmem<R>;
-    constexpr int RR = kRows;
-    constexpr int TP = SM::TP;
+template <int R, bool FWD, int STAGES, int MINB>
+__global__ void __launch_bounds__(RowCfg<R>::NT, MINB)
+k_ntt_row(RowSet rs, NttArgs a, TileMap tm) {
+    using CF = RowCfg<R>;
+    constexpr int RR = kC, NT = CF::NT, N2 = CF::N2;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    TWD* stab = reinterpret_cast<TWD*>(smem_raw);
-    double* sx = reinterpret_cast<double*>(stab + SM::NS);     // exchange, then transpose buffer
-
-    const int k = blockIdx.y, b = blockIdx.z;
-    const int lid = rs.prime[k];
-    const ModQ mq = a.mods[lid];
-    const double q = mq.qd;
-    const TWD* ptab = a.tabd + (size_t)lid * a.tab_stride;
-    const u64* __restrict__ src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N;
-    u64* __restrict__ dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * a.N;
-    const int N1 = a.N1, N2 = a.N2;
     const int tid = threadIdx.x, rho = tid / R, r = tid % R;
-    const int row0 = blockIdx.x * RR;
-    const int i1 = row0 + rho;
+    const int N1 = a.N1;
 
-    double x[R];
-    if (FWD) {
-        const double* s = reinterpret_cast<const double*>(src);
-#pragma unroll
-        for (int na = 0; na < R; ++na) x[na] = s[(size_t)i1 * N2 + R * na + r];
-    } else {
-        for (int e = tid; e < N2 * RR; e += blockDim.x) {
-            const int i2 = e / RR, rr = e % RR;
-            sx[i2 * TP + rr] = u2d(src[(size_t)row0 + rr + (size_t)N1 * i2]);
+    auto stage_ptr = [&](int s) { return smem_raw + s * CF::STAGE; };
+    auto issue = [&](int t, int s) {
+        if (t < tm.total) {
+            int b, k, blk;
+            tm.decode(t, b, k, blk);
+            const int lid = rs.prime[k];
+            const TWD* ptab = a.tabd + (size_t)lid * a.tab_stride;
+            unsigned char* st = stage_ptr(s);
+            TWD* sT = reinterpret_cast<TWD*>(st);
+            double* sD = reinterpret_cast<double*>(st + CF::NS * sizeof(TWD));
+            const int off = FWD ? a.L.rowf_cyc : a.L.rowi_cyc;   // cyc, then tw2 [r][x] -> [x][r]
+            for (int e = tid; e < CF::NS; e += NT) {
+                int d = e;
+                if (e >= R / 2) {
+                    const int f = e - R / 2;
+                    d = R / 2 + (f % R) * R + f / R;
+                }
+                cp16(sT + d, ptab + off + e);
+            }
+            const int row0 = blk * RR;
+            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N;
+            if (FWD) {   // 16 contiguous rows
+                const u64* g = src + (size_t)row0 * N2;
+                for (int e = tid; e < RR * N2 / 2; e += NT) cp16(sD + 2 * e, g + 2 * e);
+            } else {     // 128-byte segments a_hat[row0 .. row0+15 + N1 i2], swizzled
+                for (int e = tid; e < N2 * 8; e += NT) {
+                    const int i2 = e >> 3, p = e & 7;
+                    cp16(sD + i2 * 16 + ((p ^ (i2 & 7)) << 1), src + row0 + (size_t)N1 * i2 + 2 * p);
+                }
+            }
         }
-    }
-    {
-        const int off = FWD ? a.L.rowf_cyc : a.L.rowi_cyc;         // cyc, tw2 contiguous
-        for (int e = tid; e < SM::NS; e += blockDim.x) stab[e] = ptab[off + e];
-    }
-    __syncthreads();
-    const TWD* CYC = stab;
-    const TWD* TW2 = stab + R / 2;
-    double* S = sx + rho * SM::XP;
+        cp_commit();
+    };
 
-    if (FWD) {
-        cyc_dif<R>(x, CYC, q);
+    const int G = gridDim.x;
+    int t = blockIdx.x;
 #pragma unroll
-        for (int ia = 0; ia < R; ++ia) S[ia * R + r] = mulc(x[BitRev<R>::of(ia)], TW2[r * R + ia], q);
+    for (int s = 0; s < STAGES; ++s) issue(t + s * G, s);
+    for (int it = 0; t < tm.total; t += G, ++it) {
+        const int s = it % STAGES;
+        cp_wait<STAGES - 1>();
         __syncthreads();
+        int b, k, blk;
+        tm.decode(t, b, k, blk);
+        const int lid = rs.prime[k];
+        const ModQ mq = a.mods[lid];
+        const double q = mq.qd;
+        unsigned char* st = stage_ptr(s);
+        const TWD* CYC = reinterpret_cast<const TWD*>(st);
+        const TWD* TW2 = CYC + R / 2;
+        double* sD = reinterpret_cast<double*>(st + CF::NS * sizeof(TWD));
+        double* S = sD + rho * CF::XP;
+        const int row0 = blk * RR, i1 = row0 + rho;
+        u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * a.N;
+        double x[R];
+        if (FWD) {
 #pragma unroll
-        for (int nb = 0; nb < R; ++nb) x[nb] = S[r * R + nb];
-        cyc_dif<R>(x, CYC, q);
-        __syncthreads();
+            for (int na = 0; na < R; ++na) x[na] = sD[rho * N2 + R * na + r];
+            cyc_dif<R>(x, CYC, q);
+            __syncthreads();
 #pragma unroll
-        for (int ib = 0; ib < R; ++ib) sx[(r + R * ib) * TP + rho] = x[BitRev<R>::of(ib)];
-        __syncthreads();
-        for (int e = tid; e < N2 * RR; e += blockDim.x) {
-            const int i2 = e / RR, rr = e % RR;
-            dst[(size_t)row0 + rr + (size_t)N1 * i2] = d2u(canon(sx[i2 * TP + rr], q, mq.qinv));
+            for (int ia = 0; ia < R; ++ia) S[ia + CF::EP * r] = mulc(x[BitRev<R>::of(ia)], TW2[ia * R + r], q);
+            __syncthreads();
+#pragma unroll
+            for (int nb = 0; nb < R; ++nb) x[nb] = S[r + CF::EP * nb];
+            cyc_dif<R>(x, CYC, q);
+            __syncthreads();
+            u64* T = reinterpret_cast<u64*>(sD);
+#pragma unroll
+            for (int ib = 0; ib < R; ++ib) T[swz(r + R * ib, rho)] = d2u(canon(x[BitRev<R>::of(ib)], q, mq.qinv));
+            __syncthreads();
+            for (int e = tid; e < N2 * 8; e += NT) {
+                const int i2 = e >> 3, p = e & 7;
+                const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
+                *reinterpret_cast<uint4*>(dst + row0 + (size_t)N1 * i2 + 2 * p) = v;
+            }
+        } else {
+            const u64* T = reinterpret_cast<const u64*>(sD);
+#pragma unroll
+            for (int ib = 0; ib < R; ++ib) x[ib] = u2d(T[swz(r + R * ib, rho)]);
+            cyc_dif<R>(x, CYC, q);
+            __syncthreads();
+#pragma unroll
+            for (int nb = 0; nb < R; ++nb) S[r + CF::EP * nb] = mulc(x[BitRev<R>::of(nb)], TW2[nb * R + r], q);
+            __syncthreads();
+#pragma unroll
+            for (int ia = 0; ia < R; ++ia) x[ia] = S[ia + CF::EP * r];
+            cyc_dif<R>(x, CYC, q);
+            double* dd = reinterpret_cast<double*>(dst);
+#pragma unroll
+            for (int na = 0; na < R; ++na) dd[(size_t)i1 * N2 + R * na + r] = x[BitRev<R>::of(na)];
         }
-    } else {
-#pragma unroll
-        for (int ib = 0; ib < R; ++ib) x[ib] = sx[(r + R * ib) * TP + rho];
-        cyc_dif<R>(x, CYC, q);
         __syncthreads();
-#pragma unroll
-        for (int nb = 0; nb < R; ++nb) S[nb * R + r] = mulc(x[BitRev<R>::of(nb)], TW2[r * R + nb], q);
-        __syncthreads();
-#pragma unroll
-        for (int ia = 0; ia < R; ++ia) x[ia] = S[r * R + ia];
-        cyc_dif<R>(x, CYC, q);
-        double* d = reinterpret_cast<double*>(dst);
-#pragma unroll
-        for (int na = 0; na < R; ++na) d[(size_t)i1 * N2 + R * na + r] = x[BitRev<R>::of(na)];
+        issue(t + STAGES * G, s);
     }
+    cp_wait<0>();
 }
 
 // ------------------------------------------------------------------ launchers
 
-template <int R, bool FWD>
-static cudaError_t launch_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st) {
+// Pipeline depth / occupancy variant: 0 = 2 stages x 2 CTAs/SM (default), 1 = 1 stage x 3,
+// 2 = 1 stage x 4 (selected by NEO_NTT_CFG for experiments; recorded in DESIGN.md).
+static int ntt_cfg() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = std::getenv("NEO_NTT_CFG");
+        v = e ? std::atoi(e) : 0;
+        if (v < 0 || v > 2) v = 0;
+    }
+    return v;
+}
+
+template <int R, bool FWD, int STAGES, int MINB>
+static cudaError_t launch_cfg(bool col, const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st) {
     static bool init = false;
-    const size_t smc = ColSmem<R>::bytes, smr = RowSmem<R>::bytes(a.N2);
+    const size_t smc = STAGES * ColCfg<R>::STAGE, smr = STAGES * RowCfg<R>::STAGE;
     if (!init) {
-        cudaFuncSetAttribute(k_ntt_col<R, FWD>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc);
-        cudaFuncSetAttribute(k_ntt_row<R, FWD>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024);
+        cudaFuncSetAttribute(k_ntt_col<R, FWD, STAGES, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc);
+        cudaFuncSetAttribute(k_ntt_row<R, FWD, STAGES, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smr);
         init = true;
     }
-    if (col) {
-        dim3 grid(a.N2 / kCols, rs.n, batch);
-        k_ntt_col<R, FWD><<<grid, kCols * R, smc, st>>>(rs, a);
-    } else {
-        dim3 grid(a.N1 / kRows, rs.n, batch);
-        k_ntt_row<R, FWD><<<grid, kRows * R, smr, st>>>(rs, a);
-    }
+    TileMap tm;
+    tm.batch = batch;
+    tm.tpr = col ? a.N2 / kC : a.N1 / kC;
+    tm.total = tm.tpr * rs.n * batch;
+    int grid = MINB * a.num_sms;
+    if (grid > tm.total) grid = tm.total;
+    if (col)
+        k_ntt_col<R, FWD, STAGES, MINB><<<grid, ColCfg<R>::NT, smc, st>>>(rs, a, tm);
+    else
+        k_ntt_row<R, FWD, STAGES, MINB><<<grid, RowCfg<R>::NT, smr, st>>>(rs, a, tm);
     return cudaGetLastError();
+}
+
+template <int R, bool FWD>
+static cudaError_t launch_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st) {
+    switch (ntt_cfg()) {
+        case 1: return launch_cfg<R, FWD, 1, 3>(col, rs, a, batch, st);
+        case 2: return launch_cfg<R, FWD, 1, 4>(col, rs, a, batch, st);
+        default: return launch_cfg<R, FWD, 2, 2>(col, rs, a, batch, st);
+    }
 }
 
 cudaError_t ntt_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, bool fwd, cudaStream_t st) {

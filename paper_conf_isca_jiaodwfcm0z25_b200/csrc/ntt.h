@@ -10,6 +10,7 @@ struct NttArgs {
     long long tab_stride; // = L.total
     const ModQ* mods;     // device: per limb id
     int N, N1, N2;
+    int num_sms;          // persistent grid = 2 CTAs per SM
     NttLayout L;
 };
 

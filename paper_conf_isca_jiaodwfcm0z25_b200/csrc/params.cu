@@ -253,6 +253,12 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
     c->ntt.N1 = c->L.N1;
     c->ntt.N2 = c->L.N2;
     c->ntt.L = c->L;
+    {
+        int dev_sms = 0;
+        cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
+        c->num_sms = dev_sms > 0 ? dev_sms : 148;
+    }
+    c->ntt.num_sms = c->num_sms;
 
     // ---- BConv / ModDown / rescale constants per level
     std::vector<int> pids;
@@ -281,9 +287,6 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
     {
         const char* e = std::getenv("NEO_BCONV");
         c->use_tc = !(e && std::string(e) == "cuda");
-        int dev_sms = 0;
-        cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
-        if (dev_sms > 0) c->num_sms = dev_sms;
         std::vector<uint8_t> all, bm;
         c->modup_tc.resize(c->num_q);
         c->modup_boff.resize(c->num_q);
