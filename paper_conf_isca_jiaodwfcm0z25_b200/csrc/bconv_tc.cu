@@ -22,131 +22,211 @@
 namespace neo {
 
 constexpr int kTileM = 128;
-constexpr int kTmemCols = 256;
+constexpr int kStages = 2;                         // A-tile stages and TMEM accumulators
+constexpr int kInStages = 4;                       // TMA input stages (12 KB each)
+constexpr int kAccCols = 256;                      // TMEM columns per accumulator (N <= 256)
+constexpr int kEpiWarps = 8;                       // two per TMEM lane quarter (target halves)
+constexpr int kThreads = (4 + kEpiWarps + 1) * 32; // producers, epilogue, MMA
+constexpr size_t kInBytes = (size_t)BCTC_MAX_IN * kTileM * 8;
+constexpr size_t kSmemBytes = kStages * kTileM * 64 + 256 * 64 + kInStages * kInBytes;   // 96 KB
+constexpr size_t kSmemAlloc = 140 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
+static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocation");
 
+// Warp-specialised pipeline (one persistent CTA per SM):
+//   TMA (producer warp 0, lane 0): 1-D bulk copies of the n_in input rows of tile i+3
+//                          (1 KB each) into input stage (i+3) % 4
+//   producers (warps 0-3): y = [c qhat^-1] of one coefficient, split into bytes, write the
+//                          A row of stage s, arrive full_a[s]
+//   MMA (last warp, lane 0): wait full_a[s], tmem_empty[s]; two K=32 MMAs into accumulator
+//                          s; commit -> empty_a[s], tmem_full[s]
+//   epilogue (8 warps):    wait tmem_full[s], tcgen05.ld, combine the 5 byte-planes,
+//                          reduce mod t, store; arrive tmem_empty[s]
+// so HBM reads run 3 tiles ahead, and the MMA of tile i overlaps the epilogue of i-1.
 template <class LoadB>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC& P, const BConvIO& io, LoadB loadB, int N,
                                               int tiles_per_entry, int total_tiles) {
     extern __shared__ __align__(1024) uint8_t smem[];
-    uint8_t* sA = smem;                     // 128 rows x 64 B
-    uint8_t* sB = smem + kTileM * 64;       // ncols rows x 64 B
-    __shared__ uint64_t mbar;
+    uint8_t* sA = smem;                                 // kStages x (128 rows x 64 B)
+    uint8_t* sB = smem + kStages * kTileM * 64;         // ncols rows x 64 B
+    u64* sIn = reinterpret_cast<u64*>(sB + 256 * 64);   // kInStages x [n_in][128]
+    __shared__ uint64_t full_a[kStages], empty_a[kStages], tfull[kStages], tempty[kStages];
+    __shared__ uint64_t in_full[kInStages], in_empty[kInStages];
     __shared__ uint32_t tmem_base;
 
-    const int tid = threadIdx.x, warp = tid >> 5;
-    if (warp == 0) tc::tmem_alloc(&tmem_base, kTmemCols);
-    if (tid == 0) tc::mbar_init(&mbar, 1);
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int G = gridDim.x;
+    if (warp == 0) tc::tmem_alloc(&tmem_base, kStages * kAccCols);
+    if (tid == 0) {
+        for (int s = 0; s < kStages; ++s) {
+            tc::mbar_init(&full_a[s], kTileM);
+            tc::mbar_init(&empty_a[s], 1);
+            tc::mbar_init(&tfull[s], 1);
+            tc::mbar_init(&tempty[s], kEpiWarps * 32);
+        }
+        for (int s = 0; s < kInStages; ++s) {
+            tc::mbar_init(&in_full[s], 1);
+            tc::mbar_init(&in_empty[s], kTileM);
+        }
+    }
     {
-        uint4* s = reinterpret_cast<uint4*>(sB);
-        for (int e = tid; e < P.ncols * 4; e += kTileM) s[e] = loadB(e);
+        uint4* s4 = reinterpret_cast<uint4*>(sB);
+        for (int e = tid; e < P.ncols * 4; e += kThreads) s4[e] = loadB(e);
     }
     tc::fence_proxy_async();
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
     const uint32_t tmem = tmem_base;
-    const uint32_t idesc = tc::idesc_u8(kTileM, P.ncols);
-    const uint32_t aaddr = tc::smem_u32(sA), baddr = tc::smem_u32(sB);
-    // row m of A at (m/8)*512 + (m%8)*16, K chunk c (16 bytes) at + c*128
-    uint8_t* arow = sA + (tid >> 3) * 512 + (tid & 7) * 16;
-    uint32_t phase = 0;
+    const uint32_t in_bytes = (uint32_t)P.n_in * kTileM * 8;
 
-    for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+    // TMA issue of tile index i (i-th tile of this CTA) into input stage i % kInStages
+    auto tma_issue = [&](int i) {
+        const int tile = blockIdx.x + i * G;
+        if (tile >= total_tiles) return;
+        const int s = i % kInStages, k = i / kInStages;
+        tc::mbar_wait(&in_empty[s], (k & 1) ^ 1);
         const int b = tile / tiles_per_entry;
-        const int m = (tile - b * tiles_per_entry) * kTileM + tid;
-        // ---- A row: bytes of y_i = [c_i qhat_i^-1]_{q_i}, y_i occupying bits [40 i, 40 i + 40)
-        uint32_t w[16];
+        const int m0 = (tile - b * tiles_per_entry) * kTileM;
+        const u64* in = io.in + b * io.in_bstride + m0;
+        u64* dst = sIn + (size_t)s * BCTC_MAX_IN * kTileM;
+        tc::mbar_arrive_tx(&in_full[s], in_bytes);
+        for (int j = 0; j < P.n_in; ++j) tc::bulk_g2s(dst + j * kTileM, in + (size_t)io.in_off[j] * N, kTileM * 8, &in_full[s]);
+    };
+
+    if (warp < 4) {
+        // ------------------------------------------------ producers (+ TMA issue on thread 0)
+        if (tid == 0)
+            for (int i = 0; i < kInStages - 1; ++i) tma_issue(i);
+        uint8_t* arow0 = sA + (tid >> 3) * 512 + (tid & 7) * 16;   // row tid of stage 0
+        int i = 0;
+        for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
+            if (tid == 0) tma_issue(i + kInStages - 1);
+            const int si = i % kInStages, ki = i / kInStages;
+            tc::mbar_wait(&in_full[si], ki & 1);
+            const u64* src = sIn + (size_t)si * BCTC_MAX_IN * kTileM + tid;
+            u64 c[BCTC_MAX_IN];
 #pragma unroll
-        for (int k = 0; k < 16; ++k) w[k] = 0;
-        const u64* in = io.in + b * io.in_bstride + m;
+            for (int j = 0; j < BCTC_MAX_IN; ++j) c[j] = (j < P.n_in) ? src[j * kTileM] : 0;
+            tc::mbar_arrive(&in_empty[si]);
+            uint32_t w[16];
 #pragma unroll
-        for (int i = 0; i < 12; ++i) {
-            if (i < P.n_in) {
-                const double q = P.qin[i];
-                const double c = u2d(in[(size_t)io.in_off[i] * N]);
-                const u64 y = d2u(canon(mulc(c, P.qhat_inv[i], q), q, P.qinv_in[i]));
-                const int bit = 40 * i, wi = bit >> 5, sh = bit & 31;
-                w[wi] |= (uint32_t)(y << sh);
-                w[wi + 1] |= (uint32_t)(y >> (32 - sh));
-                if (sh > 24) w[wi + 2] |= (uint32_t)(y >> (64 - sh));
-            }
-        }
+            for (int kk = 0; kk < 16; ++kk) w[kk] = 0;
 #pragma unroll
-        for (int c = 0; c < 4; ++c)
-            *reinterpret_cast<uint4*>(arow + c * 128) = make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]);
-        tc::fence_proxy_async();
-        __syncthreads();
-        // ---- one thread issues the GEMM: K = 64 as two K = 32 steps (LBO = 128, SBO = 512)
-        if (tid == 0) {
-            tc::fence_after();
-            tc::mma_u8(tmem, tc::sdesc(aaddr, 128, 512), tc::sdesc(baddr, 128, 512), idesc, 0);
-            tc::mma_u8(tmem, tc::sdesc(aaddr + 256, 128, 512), tc::sdesc(baddr + 256, 128, 512), idesc, 1);
-            tc::commit(&mbar);
-        }
-        tc::mbar_wait(&mbar, phase);
-        phase ^= 1;
-        tc::fence_after();
-        // ---- epilogue: lane (warp*32 + lane) = row m; columns 5t..5t+4 hold D_0..D_4 of target t
-        const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
-        u64* outb = io.out + b * io.out_bstride + m;
-        for (int g = 0; g < P.n_out; g += 8) {
-            uint32_t v[40];
-#pragma unroll
-            for (int s = 0; s < 5; ++s) {
-                uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * s]);
-                tc::tmem_ld8(trow + (uint32_t)(5 * g + 8 * s), vv);
-            }
-            tc::tmem_wait_ld();
-#pragma unroll
-            for (int u = 0; u < 8; ++u) {
-                const int t = g + u;
-                if (t < P.n_out) {
-                    const uint32_t* D = &v[5 * u];
-                    const u64 lo = (u64)D[0] + ((u64)D[1] << 8) + ((u64)D[2] << 16);     // < 2^39
-                    const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
-                    const double tq = P.t[t];
-                    const double r = __dadd_rn(u2d(lo), mulc(u2d(hi), P.c24[t], tq));   // == V (mod t)
-                    outb[(size_t)io.out_off[t] * N] = d2u(canon(r, tq, P.tinv[t]));
+            for (int j = 0; j < BCTC_MAX_IN; ++j) {
+                if (j < P.n_in) {
+                    const double q = P.qin[j];
+                    const u64 y = d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
+                    const int bit = 40 * j, wi = bit >> 5, sh = bit & 31;
+                    w[wi] |= (uint32_t)(y << sh);
+                    w[wi + 1] |= (uint32_t)(y >> (32 - sh));
+                    if (sh > 24) w[wi + 2] |= (uint32_t)(y >> (64 - sh));
                 }
             }
+            const int s = i % kStages, k = i / kStages;
+            tc::mbar_wait(&empty_a[s], (k & 1) ^ 1);
+            uint8_t* arow = arow0 + s * (kTileM * 64);
+#pragma unroll
+            for (int cc = 0; cc < 4; ++cc)
+                *reinterpret_cast<uint4*>(arow + cc * 128) =
+                    make_uint4(w[4 * cc], w[4 * cc + 1], w[4 * cc + 2], w[4 * cc + 3]);
+            tc::fence_proxy_async();
+            tc::mbar_arrive(&full_a[s]);
         }
-        tc::fence_before();
-        __syncthreads();
+    } else if (warp < 4 + kEpiWarps) {
+        // ------------------------------------------------ epilogue
+        const int ew = warp - 4, quarter = ew & 3, half = ew >> 2;
+        const int et = quarter * 32 + lane;                  // TMEM lane = A row = coefficient
+        int i = 0;
+        for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
+            const int s = i % kStages, k = i / kStages;
+            const int b = tile / tiles_per_entry;
+            const int m = (tile - b * tiles_per_entry) * kTileM + et;
+            tc::mbar_wait(&tfull[s], k & 1);
+            tc::fence_after();
+            const uint32_t trow = tmem + (uint32_t)(s * kAccCols) + ((uint32_t)(quarter * 32) << 16);
+            u64* outb = io.out + b * io.out_bstride + m;
+            for (int g = 8 * half; g < P.n_out; g += 16) {
+                uint32_t v[40];
+#pragma unroll
+                for (int q5 = 0; q5 < 5; ++q5) {
+                    uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * q5]);
+                    tc::tmem_ld8(trow + (uint32_t)(5 * g + 8 * q5), vv);
+                }
+                tc::tmem_wait_ld();
+#pragma unroll
+                for (int u = 0; u < 8; ++u) {
+                    const int t = g + u;
+                    if (t < P.n_out) {
+                        const uint32_t* D = &v[5 * u];
+                        const u64 lo = (u64)D[0] + ((u64)D[1] << 8) + ((u64)D[2] << 16);     // < 2^39
+                        const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
+                        const double tq = P.t[t];
+                        const double r = __dadd_rn(u2d(lo), mulc(u2d(hi), P.c24[t], tq));   // == V (mod t)
+                        outb[(size_t)io.out_off[t] * N] = d2u(canon(r, tq, P.tinv[t]));
+                    }
+                }
+            }
+            tc::fence_before();
+            tc::mbar_arrive(&tempty[s]);
+        }
+    } else {
+        // ------------------------------------------------ MMA issuer
+        if (lane == 0) {
+            const uint32_t idesc = tc::idesc_u8(kTileM, P.ncols);
+            const uint32_t aaddr = tc::smem_u32(sA), baddr = tc::smem_u32(sB);
+            int i = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
+                const int s = i % kStages, k = i / kStages;
+                tc::mbar_wait(&full_a[s], k & 1);
+                tc::mbar_wait(&tempty[s], (k & 1) ^ 1);
+                tc::fence_after();
+                const uint32_t acc = tmem + (uint32_t)(s * kAccCols);
+                const uint32_t as = aaddr + s * (kTileM * 64);
+                // K = 64 as two K = 32 steps (LBO = 128 B between K chunks, SBO = 512 B between row groups)
+                tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(baddr, 128, 512), idesc, 0);
+                tc::mma_u8(acc, tc::sdesc(as + 256, 128, 512), tc::sdesc(baddr + 256, 128, 512), idesc, 1);
+                tc::commit(&empty_a[s]);
+                tc::commit(&tfull[s]);
+            }
+        }
+        __syncwarp();
     }
-    if (warp == 0) tc::tmem_dealloc(tmem, kTmemCols);
+    tc::fence_before();
+    __syncthreads();
+    if (warp == 0) tc::tmem_dealloc(tmem, kStages * kAccCols);
 }
 
-__global__ void __launch_bounds__(kTileM, 1)
+__global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_g(const __grid_constant__ BConvTC P, const __grid_constant__ BConvIO io, const uint4* __restrict__ bmat,
              int N, int tiles_per_entry, int total_tiles) {
     bconv_tc_body(P, io, [&](int e) { return bmat[e]; }, N, tiles_per_entry, total_tiles);
 }
 
-__global__ void __launch_bounds__(kTileM, 1)
+__global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_p(const __grid_constant__ BConvTC P, const __grid_constant__ BConvIO io,
              const __grid_constant__ BMatParam B, int N, int tiles_per_entry, int total_tiles) {
     bconv_tc_body(P, io, [&](int e) { return B.d[e]; }, N, tiles_per_entry, total_tiles);
 }
 
-size_t bconv_tc_smem(int ncols) { return (size_t)kTileM * 64 + (size_t)ncols * 64; }
+size_t bconv_tc_smem(int) { return kSmemAlloc; }
 
 cudaError_t launch_bconv_tc(const BConvTC& P, const BConvIO& io, const uint8_t* bmat, const BMatParam* bp, int N,
                             int batch, int num_sms, cudaStream_t st) {
     static bool init = false;
     if (!init) {
-        cudaFuncSetAttribute(k_bconv_tc_g, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
-        cudaFuncSetAttribute(k_bconv_tc_p, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+        cudaFuncSetAttribute(k_bconv_tc_g, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
+        cudaFuncSetAttribute(k_bconv_tc_p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         init = true;
     }
     const int tiles_per_entry = N / kTileM;
     const int total = tiles_per_entry * batch;
-    int grid = num_sms * 2;
+    int grid = num_sms;
     if (grid > total) grid = total;
     if (bp)
-        k_bconv_tc_p<<<grid, kTileM, bconv_tc_smem(P.ncols), st>>>(P, io, *bp, N, tiles_per_entry, total);
+        k_bconv_tc_p<<<grid, kThreads, kSmemAlloc, st>>>(P, io, *bp, N, tiles_per_entry, total);
     else
-        k_bconv_tc_g<<<grid, kTileM, bconv_tc_smem(P.ncols), st>>>(P, io, reinterpret_cast<const uint4*>(bmat), N,
-                                                                   tiles_per_entry, total);
+        k_bconv_tc_g<<<grid, kThreads, kSmemAlloc, st>>>(P, io, reinterpret_cast<const uint4*>(bmat), N,
+                                                         tiles_per_entry, total);
     return cudaGetLastError();
 }
 

@@ -354,14 +354,15 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm) {
 
 // ------------------------------------------------------------------ launchers
 
-// Pipeline depth / occupancy variant: 0 = 2 stages x 2 CTAs/SM (default), 1 = 1 stage x 3,
-// 2 = 1 stage x 4 (selected by NEO_NTT_CFG for experiments; recorded in DESIGN.md).
+// Pipeline depth / occupancy variant: 0 = 2 stages x 2 CTAs/SM, 1 = 1 stage x 3,
+// 2 = 1 stage x 4 CTAs/SM (default: fastest on B200, bench of 2026-10-17 in DESIGN.md);
+// NEO_NTT_CFG overrides for experiments.
 static int ntt_cfg() {
     static int v = -1;
     if (v < 0) {
         const char* e = std::getenv("NEO_NTT_CFG");
-        v = e ? std::atoi(e) : 0;
-        if (v < 0 || v > 2) v = 0;
+        v = e ? std::atoi(e) : 2;
+        if (v < 0 || v > 2) v = 2;
     }
     return v;
 }
@@ -392,8 +393,8 @@ template <int R, bool FWD>
 static cudaError_t launch_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st) {
     switch (ntt_cfg()) {
         case 1: return launch_cfg<R, FWD, 1, 3>(col, rs, a, batch, st);
-        case 2: return launch_cfg<R, FWD, 1, 4>(col, rs, a, batch, st);
-        default: return launch_cfg<R, FWD, 2, 2>(col, rs, a, batch, st);
+        case 0: return launch_cfg<R, FWD, 2, 2>(col, rs, a, batch, st);
+        default: return launch_cfg<R, FWD, 1, 4>(col, rs, a, batch, st);
     }
 }
 
