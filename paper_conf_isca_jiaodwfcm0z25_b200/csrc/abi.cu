@@ -135,26 +135,37 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
     for (int i = 0; i < Lq; ++i) { so[i] = i; dof[i] = i; pr[i] = i; }
     if ((s = ntt_rows(c, false, d, d_bs, so, y, (long long)Lq * N, dof, pr, Lq, tmp, B, st))) return s;
 
-    // a4: ModUp BConv, one launch per digit: y[D_j] -> up[j][targets]
-    for (int j = 0; j < beta; ++j) {
-        const BConvTab& T = c->modup[l][j];
-        const std::vector<int>& dj = c->digits[l][j];
-        BConvIO io;
-        io.in = y; io.out = up;
-        io.in_bstride = (long long)Lq * N;
-        io.out_bstride = (long long)beta * E * N;
-        for (int i = 0; i < T.n_in; ++i) io.in_off[i] = dj[i];
-        int o = 0;
-        for (int pos = 0; pos < E; ++pos) {
-            int id = c->ext_id(l, pos);
-            if (std::find(dj.begin(), dj.end(), id) != dj.end()) continue;
-            io.out_off[o++] = j * E + pos;
+    // a4: ModUp BConv of all beta digits: y[D_j] -> up[j][targets]  (one launch on tensor cores)
+    {
+        BConvMulti M;
+        M.njobs = 0;
+        for (int j = 0; j < beta; ++j) {
+            const BConvTab& T = c->modup[l][j];
+            const std::vector<int>& dj = c->digits[l][j];
+            BConvIO io;
+            io.in = y; io.out = up;
+            io.in_bstride = (long long)Lq * N;
+            io.out_bstride = (long long)beta * E * N;
+            for (int i = 0; i < T.n_in; ++i) io.in_off[i] = dj[i];
+            int o = 0;
+            for (int pos = 0; pos < E; ++pos) {
+                int id = c->ext_id(l, pos);
+                if (std::find(dj.begin(), dj.end(), id) != dj.end()) continue;
+                io.out_off[o++] = j * E + pos;
+            }
+            if (c->use_tc) {
+                M.P[M.njobs] = c->modup_tc[l][j];
+                M.io[M.njobs] = io;
+                M.bmat[M.njobs] = c->d_bmat + c->modup_boff[l][j];
+                if (++M.njobs == 4) {                      // at most 4 conversions per launch
+                    LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, B, c->num_sms, st));
+                    M.njobs = 0;
+                }
+            } else {
+                LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, B, st));
+            }
         }
-        if (c->use_tc)
-            LAUNCH(PK_BCONV, st, launch_bconv_tc(c->modup_tc[l][j], io, c->d_bmat + c->modup_boff[l][j], nullptr, N, B,
-                                                 c->num_sms, st));
-        else
-            LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, B, st));
+        if (M.njobs) LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, B, c->num_sms, st));
     }
 
     // a5: NTT of every ModUp output row
@@ -208,10 +219,14 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
         io.out_bstride = (long long)Lq * N;
         for (int i = 0; i < P; ++i) io.in_off[i] = i;
         for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
-        if (c->use_tc)
-            LAUNCH(PK_BCONV, st, launch_bconv_tc(c->moddown_tc[l], io, c->d_bmat + c->moddown_boff[l], nullptr, N,
-                                                 2 * B, c->num_sms, st));
-        else
+        if (c->use_tc) {
+            BConvMulti M;
+            M.njobs = 1;
+            M.P[0] = c->moddown_tc[l];
+            M.io[0] = io;
+            M.bmat[0] = c->d_bmat + c->moddown_boff[l];
+            LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, 2 * B, c->num_sms, st));
+        } else
             LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, 2 * B, st));
     }
 
@@ -444,7 +459,7 @@ neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids
         static thread_local BMatParam bp;
         std::memset(&bp, 0, sizeof(bp));
         std::memcpy(&bp, bm.data(), bm.size());
-        LAUNCH(PK_BCONV, S(st), launch_bconv_tc(P, io, nullptr, &bp, c->N, batch, c->num_sms, S(st)));
+        LAUNCH(PK_BCONV, S(st), launch_bconv_tc_param(P, io, bp, c->N, batch, c->num_sms, S(st)));
     } else {
         LAUNCH(PK_BCONV, S(st), launch_bconv(T, io, c->N, batch, S(st)));
     }

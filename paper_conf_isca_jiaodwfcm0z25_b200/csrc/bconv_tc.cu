@@ -25,11 +25,12 @@ constexpr int kTileM = 128;
 constexpr int kStages = 2;                         // A-tile stages and TMEM accumulators
 constexpr int kInStages = 4;                       // TMA input stages (12 KB each)
 constexpr int kAccCols = 256;                      // TMEM columns per accumulator (N <= 256)
-constexpr int kEpiWarps = 8;                       // two per TMEM lane quarter (target halves)
+constexpr int kEpiWarps = 16;                      // four per TMEM lane quarter (target quarters)
 constexpr int kThreads = (4 + kEpiWarps + 1) * 32; // producers, epilogue, MMA
 constexpr size_t kInBytes = (size_t)BCTC_MAX_IN * kTileM * 8;
-constexpr size_t kSmemBytes = kStages * kTileM * 64 + 256 * 64 + kInStages * kInBytes;   // 96 KB
-constexpr size_t kSmemAlloc = 140 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
+constexpr int kMaxJobs = 4;                        // conversions fused into one launch (ModUp digits)
+constexpr size_t kSmemBytes = kStages * kTileM * 64 + kMaxJobs * 256 * 64 + kInStages * kInBytes;  // 128 KB
+constexpr size_t kSmemAlloc = 160 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
 static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocation");
 
 // Warp-specialised pipeline (one persistent CTA per SM):
@@ -43,12 +44,21 @@ static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocati
 //                          reduce mod t, store; arrive tmem_empty[s]
 // so HBM reads run 3 tiles ahead, and the MMA of tile i overlaps the epilogue of i-1.
 template <class LoadB>
-__device__ __forceinline__ void bconv_tc_body(const BConvTC& P, const BConvIO& io, LoadB loadB, int N,
-                                              int tiles_per_entry, int total_tiles) {
+__device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
+                                              int tiles_per_entry, int batch) {
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t* sA = smem;                                 // kStages x (128 rows x 64 B)
-    uint8_t* sB = smem + kStages * kTileM * 64;         // ncols rows x 64 B
-    u64* sIn = reinterpret_cast<u64*>(sB + 256 * 64);   // kInStages x [n_in][128]
+    uint8_t* sB0 = smem + kStages * kTileM * 64;        // kMaxJobs x (ncols rows x 64 B)
+    u64* sIn = reinterpret_cast<u64*>(sB0 + kMaxJobs * 256 * 64);   // kInStages x [n_in][128]
+    const int tiles_per_job = tiles_per_entry * batch;
+    const int total_tiles = tiles_per_job * njobs;
+    // tile -> (job, batch entry, first coefficient)
+    auto decode = [&](int tile, int& j, int& b, int& m0) {
+        j = tile / tiles_per_job;
+        const int r = tile - j * tiles_per_job;
+        b = r / tiles_per_entry;
+        m0 = (r - b * tiles_per_entry) * kTileM;
+    };
     __shared__ uint64_t full_a[kStages], empty_a[kStages], tfull[kStages], tempty[kStages];
     __shared__ uint64_t in_full[kInStages], in_empty[kInStages];
     __shared__ uint32_t tmem_base;
@@ -68,16 +78,15 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC& P, const BConvIO& i
             tc::mbar_init(&in_empty[s], kTileM);
         }
     }
-    {
-        uint4* s4 = reinterpret_cast<uint4*>(sB);
-        for (int e = tid; e < P.ncols * 4; e += kThreads) s4[e] = loadB(e);
+    for (int j = 0; j < njobs; ++j) {
+        uint4* s4 = reinterpret_cast<uint4*>(sB0 + j * 256 * 64);
+        for (int e = tid; e < PJ[j].ncols * 4; e += kThreads) s4[e] = loadB(j, e);
     }
     tc::fence_proxy_async();
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
     const uint32_t tmem = tmem_base;
-    const uint32_t in_bytes = (uint32_t)P.n_in * kTileM * 8;
 
     // TMA issue of tile index i (i-th tile of this CTA) into input stage i % kInStages
     auto tma_issue = [&](int i) {
@@ -85,8 +94,11 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC& P, const BConvIO& i
         if (tile >= total_tiles) return;
         const int s = i % kInStages, k = i / kInStages;
         tc::mbar_wait(&in_empty[s], (k & 1) ^ 1);
-        const int b = tile / tiles_per_entry;
-        const int m0 = (tile - b * tiles_per_entry) * kTileM;
+        int jb, b, m0;
+        decode(tile, jb, b, m0);
+        const BConvTC& P = PJ[jb];
+        const BConvIO& io = IOJ[jb];
+        const uint32_t in_bytes = (uint32_t)P.n_in * kTileM * 8;
         const u64* in = io.in + b * io.in_bstride + m0;
         u64* dst = sIn + (size_t)s * BCTC_MAX_IN * kTileM;
         tc::mbar_arrive_tx(&in_full[s], in_bytes);
@@ -101,6 +113,9 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC& P, const BConvIO& i
         int i = 0;
         for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
             if (tid == 0) tma_issue(i + kInStages - 1);
+            int jb, b, m0;
+            decode(tile, jb, b, m0);
+            const BConvTC& P = PJ[jb];
             const int si = i % kInStages, ki = i / kInStages;
             tc::mbar_wait(&in_full[si], ki & 1);
             const u64* src = sIn + (size_t)si * BCTC_MAX_IN * kTileM + tid;
@@ -134,18 +149,21 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC& P, const BConvIO& i
         }
     } else if (warp < 4 + kEpiWarps) {
         // ------------------------------------------------ epilogue
-        const int ew = warp - 4, quarter = ew & 3, half = ew >> 2;
+        const int ew = warp - 4, quarter = ew & 3, part = ew >> 2;
         const int et = quarter * 32 + lane;                  // TMEM lane = A row = coefficient
         int i = 0;
         for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
             const int s = i % kStages, k = i / kStages;
-            const int b = tile / tiles_per_entry;
-            const int m = (tile - b * tiles_per_entry) * kTileM + et;
+            int jb, b, m0;
+            decode(tile, jb, b, m0);
+            const BConvTC& P = PJ[jb];
+            const BConvIO& io = IOJ[jb];
+            const int m = m0 + et;
             tc::mbar_wait(&tfull[s], k & 1);
             tc::fence_after();
             const uint32_t trow = tmem + (uint32_t)(s * kAccCols) + ((uint32_t)(quarter * 32) << 16);
             u64* outb = io.out + b * io.out_bstride + m;
-            for (int g = 8 * half; g < P.n_out; g += 16) {
+            for (int g = 8 * part; g < P.n_out; g += 8 * (kEpiWarps / 4)) {
                 uint32_t v[40];
 #pragma unroll
                 for (int q5 = 0; q5 < 5; ++q5) {
@@ -172,11 +190,14 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC& P, const BConvIO& i
     } else {
         // ------------------------------------------------ MMA issuer
         if (lane == 0) {
-            const uint32_t idesc = tc::idesc_u8(kTileM, P.ncols);
-            const uint32_t aaddr = tc::smem_u32(sA), baddr = tc::smem_u32(sB);
+            const uint32_t aaddr = tc::smem_u32(sA);
             int i = 0;
             for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
                 const int s = i % kStages, k = i / kStages;
+                int jb, b, m0;
+                decode(tile, jb, b, m0);
+                const uint32_t idesc = tc::idesc_u8(kTileM, PJ[jb].ncols);
+                const uint32_t baddr = tc::smem_u32(sB0 + jb * 256 * 64);
                 tc::mbar_wait(&full_a[s], k & 1);
                 tc::mbar_wait(&tempty[s], (k & 1) ^ 1);
                 tc::fence_after();
@@ -197,36 +218,44 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC& P, const BConvIO& i
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
-k_bconv_tc_g(const __grid_constant__ BConvTC P, const __grid_constant__ BConvIO io, const uint4* __restrict__ bmat,
-             int N, int tiles_per_entry, int total_tiles) {
-    bconv_tc_body(P, io, [&](int e) { return bmat[e]; }, N, tiles_per_entry, total_tiles);
+k_bconv_tc_g(const __grid_constant__ BConvMulti M, int N, int tiles_per_entry, int batch) {
+    bconv_tc_body(M.P, M.io, M.njobs, [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; }, N,
+                  tiles_per_entry, batch);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_p(const __grid_constant__ BConvTC P, const __grid_constant__ BConvIO io,
-             const __grid_constant__ BMatParam B, int N, int tiles_per_entry, int total_tiles) {
-    bconv_tc_body(P, io, [&](int e) { return B.d[e]; }, N, tiles_per_entry, total_tiles);
+             const __grid_constant__ BMatParam B, int N, int tiles_per_entry, int batch) {
+    bconv_tc_body(&P, &io, 1, [&](int, int e) { return B.d[e]; }, N, tiles_per_entry, batch);
 }
 
 size_t bconv_tc_smem(int) { return kSmemAlloc; }
 
-cudaError_t launch_bconv_tc(const BConvTC& P, const BConvIO& io, const uint8_t* bmat, const BMatParam* bp, int N,
-                            int batch, int num_sms, cudaStream_t st) {
+static void bconv_tc_init() {
     static bool init = false;
     if (!init) {
         cudaFuncSetAttribute(k_bconv_tc_g, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         cudaFuncSetAttribute(k_bconv_tc_p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         init = true;
     }
+}
+
+cudaError_t launch_bconv_tc(const BConvMulti& M, int N, int batch, int num_sms, cudaStream_t st) {
+    bconv_tc_init();
+    const int tiles_per_entry = N / kTileM;
+    const int total = tiles_per_entry * batch * M.njobs;
+    const int grid = num_sms < total ? num_sms : total;
+    k_bconv_tc_g<<<grid, kThreads, kSmemAlloc, st>>>(M, N, tiles_per_entry, batch);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bconv_tc_param(const BConvTC& P, const BConvIO& io, const BMatParam& bp, int N, int batch,
+                                  int num_sms, cudaStream_t st) {
+    bconv_tc_init();
     const int tiles_per_entry = N / kTileM;
     const int total = tiles_per_entry * batch;
-    int grid = num_sms;
-    if (grid > total) grid = total;
-    if (bp)
-        k_bconv_tc_p<<<grid, kThreads, kSmemAlloc, st>>>(P, io, *bp, N, tiles_per_entry, total);
-    else
-        k_bconv_tc_g<<<grid, kThreads, kSmemAlloc, st>>>(P, io, reinterpret_cast<const uint4*>(bmat), N,
-                                                         tiles_per_entry, total);
+    const int grid = num_sms < total ? num_sms : total;
+    k_bconv_tc_p<<<grid, kThreads, kSmemAlloc, st>>>(P, io, bp, N, tiles_per_entry, batch);
     return cudaGetLastError();
 }
 

@@ -13,8 +13,18 @@ void make_bconv_tc(const std::vector<u64>& src_mod, const std::vector<u64>& dst_
                    std::vector<uint8_t>& bmat);
 
 size_t bconv_tc_smem(int ncols);
-// B from device memory (bmat) or by value (bp != nullptr).
-cudaError_t launch_bconv_tc(const BConvTC& P, const BConvIO& io, const uint8_t* bmat, const BMatParam* bp, int N,
-                            int batch, int num_sms, cudaStream_t st);
+
+// Up to 4 conversions with the same input/output batch geometry in one launch (e.g. the
+// beta ModUp digits); B matrices from device memory.
+struct BConvMulti {
+    int njobs;
+    BConvTC P[4];
+    BConvIO io[4];
+    const uint8_t* bmat[4];
+};
+cudaError_t launch_bconv_tc(const BConvMulti& M, int N, int batch, int num_sms, cudaStream_t st);
+// One conversion with B passed by value (generic neo_bconv).
+cudaError_t launch_bconv_tc_param(const BConvTC& P, const BConvIO& io, const BMatParam& bp, int N, int batch,
+                                  int num_sms, cudaStream_t st);
 
 }  // namespace neo
