@@ -140,6 +140,22 @@ neo_status neo_hrot(const neo_ctx* ctx, const neo_evk* rotkey, uint32_t galois_e
                     const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
                     size_t ws_bytes, neo_stream_t stream);
 
+/* Building blocks of the limb-sharded key-switch (each rank owns a subset of
+ * the limbs of PQ_l and calls these on its own limbs between NCCL all-gathers):
+ *
+ * KeyIP (Alg. 3) on an arbitrary limb subset:
+ *   acc[b][c][t] = sum_{j<beta} dhat[b][j][t] * evk_{j,c}[limb_ids[t]]  mod q_{limb_ids[t]}
+ * dhat [batch][beta][n][N] NTT form, acc [batch][2][n][N]; 1 <= n <= 64, 1 <= beta <= dnum. */
+neo_status neo_keyip(const neo_ctx* ctx, const neo_evk* evk, const uint64_t* dhat, const int32_t* limb_ids,
+                     int32_t n_limbs, int32_t beta, uint64_t* acc, int32_t batch, neo_stream_t stream);
+
+/* ModDown tail (Table 2, Z9) on Q limbs q_ids[0..n):
+ *   out[b][c][i] = (acc[b][c][i] - conv[b][c][i]) * P^-1  mod q_{q_ids[i]}
+ * acc, conv, out [batch][2][n][N] NTT form. */
+neo_status neo_moddown_combine(const neo_ctx* ctx, const uint64_t* acc, const uint64_t* conv,
+                               const int32_t* q_ids, int32_t n, uint64_t* out, int32_t batch,
+                               neo_stream_t stream);
+
 /* Rescale (L137), floor reading (Z10): ct_in [batch][2][level+1][N] -> ct_out
  * [batch][2][level][N], c'_i = (c_i - NTT_i([INTT_l(c_l)] mod q_i)) * q_l^-1 mod q_i.
  * level >= 1. */

@@ -246,7 +246,7 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
         A.add_bstride = add_bs;
         A.out_bstride = out_bs;
         A.N = N;
-        for (int i = 0; i < Lq; ++i) A.pinv[i] = c->pinv[i];
+        for (int i = 0; i < Lq; ++i) { A.pinv[i] = c->pinv[i]; A.limb[i] = i; }
         LAUNCH(PK_COMBINE, st, launch_combine(A, Lq, B, st));
     }
     return NEO_OK;
@@ -572,6 +572,58 @@ neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint6
     cudaStream_t s = S(st);
     LAUNCH(PK_AUTO, s, launch_automorph(ct_in, sc, g, c->N, 2 * (level + 1) * batch, s));
     return ks_core(c, rk, sc + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, sc, nullptr, 2 * ls, s);
+}
+
+neo_status neo_keyip(const neo_ctx* c, const neo_evk* k, const uint64_t* dhat, const int32_t* limb_ids, int32_t n,
+                     int32_t beta, uint64_t* acc, int32_t batch, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    if (!k || k->ctx != c) FAIL(NEO_EINVAL, "evaluation key missing or from another context");
+    TRY(check_ptr(dhat, "dhat"));
+    TRY(check_ptr(acc, "acc"));
+    if (!limb_ids || n < 1 || n > KS_MAX_EXT) FAIL(NEO_EINVAL, "need 1 <= n_limbs <= 64 limb ids");
+    if (beta < 1 || beta > c->dnum) FAIL(NEO_EINVAL, "beta must be in [1, dnum]");
+    if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
+    KeyIPArgs A;
+    A.d = dhat; A.up = dhat; A.evk = k->d; A.acc = acc; A.mods = c->d_mods;
+    A.d_bstride = A.up_bstride = (long long)beta * n * c->N;
+    A.acc_bstride = (long long)2 * n * c->N;
+    A.acc_cstride = (long long)n * c->N;
+    A.N = c->N; A.beta = beta; A.evk_limbs = c->num_q + c->num_p;
+    for (int t = 0; t < n; ++t) {
+        if (limb_ids[t] < 0 || limb_ids[t] >= c->num_q + c->num_p) FAIL(NEO_EINVAL, "unknown limb id");
+        A.limb[t] = limb_ids[t];
+        for (int j = 0; j < beta; ++j) { A.src_kind[j][t] = 1; A.src_off[j][t] = j * n + t; }
+    }
+    LAUNCH(PK_KEYIP, S(st), launch_keyip(A, n, batch, S(st)));
+    return NEO_OK;
+}
+
+neo_status neo_moddown_combine(const neo_ctx* c, const uint64_t* acc, const uint64_t* conv, const int32_t* q_ids,
+                               int32_t n, uint64_t* out, int32_t batch, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_ptr(acc, "acc"));
+    TRY(check_ptr(conv, "conv"));
+    TRY(check_ptr(out, "out"));
+    if (!q_ids || n < 1 || n > 64) FAIL(NEO_EINVAL, "need 1 <= n <= 64 Q limb ids");
+    if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
+    CombineArgs A;
+    A.acc = acc; A.conv = conv; A.add0 = nullptr; A.add1 = nullptr; A.out0 = out; A.out1 = out + (size_t)n * c->N;
+    A.mods = c->d_mods;
+    A.acc_bstride = (long long)2 * n * c->N;
+    A.acc_cstride = (long long)n * c->N;
+    A.conv_stride = (long long)n * c->N;
+    A.add_bstride = 0;
+    A.out_bstride = (long long)2 * n * c->N;
+    A.N = c->N;
+    for (int i = 0; i < n; ++i) {
+        if (q_ids[i] < 0 || q_ids[i] >= c->num_q) FAIL(NEO_EINVAL, "q_ids must be Q limbs");
+        A.pinv[i] = c->pinv[q_ids[i]];
+        A.limb[i] = q_ids[i];
+    }
+    LAUNCH(PK_COMBINE, S(st), launch_combine(A, n, batch, S(st)));
+    return NEO_OK;
 }
 
 neo_status neo_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch,

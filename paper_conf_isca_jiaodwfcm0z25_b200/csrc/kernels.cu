@@ -76,7 +76,7 @@ k_combine(CombineArgs A) {
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
     const int i = blockIdx.y, bc = blockIdx.z, b = bc >> 1, c = bc & 1;
     if (n >= A.N) return;
-    const u64 q = A.mods[i].q;
+    const u64 q = A.mods[A.limb[i]].q;
     const size_t row = (size_t)i * A.N + n;
     u64 a = A.acc[b * A.acc_bstride + c * A.acc_cstride + row];
     u64 v = A.conv[(size_t)bc * A.conv_stride + row];

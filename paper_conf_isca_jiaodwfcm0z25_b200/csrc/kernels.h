@@ -30,7 +30,8 @@ struct CombineArgs {
     const ModQ* mods;
     long long acc_bstride, acc_cstride, conv_stride, add_bstride, out_bstride;
     int N;
-    TW pinv[64];
+    TW pinv[64];           // per position
+    int limb[64];          // position -> limb id (modulus)
 };
 
 struct RescaleArgs {

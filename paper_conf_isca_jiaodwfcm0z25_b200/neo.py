@@ -23,6 +23,7 @@ _STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM",
 EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_workspace_size",
             "neo_ntt", "neo_intt", "neo_bconv", "neo_tensor", "neo_automorphism", "neo_evk_create",
             "neo_evk_destroy", "neo_keyswitch", "neo_hmult", "neo_hrot", "neo_rescale",
+            "neo_keyip", "neo_moddown_combine",
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine")
@@ -68,6 +69,8 @@ def lib() -> ctypes.CDLL:
             "neo_hmult": [_vp, _vp, _vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_hrot": [_vp, _vp, _u32, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_rescale": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+            "neo_keyip": [_vp, _vp, _vp, _i32p, _i32, _i32, _vp, _i32, _vp],
+            "neo_moddown_combine": [_vp, _vp, _vp, _i32p, _i32, _vp, _i32, _vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -232,3 +235,13 @@ def neo_hrot(ctx: Context, rotkey: EvalKey, galois_elt: int, ct_in, level: int, 
 def neo_rescale(ctx: Context, ct_in, level: int, ct_out, batch: int, ws, stream=None):
     _check(lib().neo_rescale(ctx.handle, _ptr(ct_in), level, _ptr(ct_out), batch, _ptr(ws), ws.numel() * 8,
                              _stream(stream)), "neo_rescale")
+
+
+def neo_keyip(ctx: Context, evk: EvalKey, dhat, limb_ids, beta: int, acc, batch: int, stream=None):
+    _check(lib().neo_keyip(ctx.handle, evk.handle, _ptr(dhat), _ids(limb_ids), len(limb_ids), beta, _ptr(acc),
+                           batch, _stream(stream)), "neo_keyip")
+
+
+def neo_moddown_combine(ctx: Context, acc, conv, q_ids, out, batch: int, stream=None):
+    _check(lib().neo_moddown_combine(ctx.handle, _ptr(acc), _ptr(conv), _ids(q_ids), len(q_ids), _ptr(out), batch,
+                                     _stream(stream)), "neo_moddown_combine")

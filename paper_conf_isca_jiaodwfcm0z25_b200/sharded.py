@@ -1,0 +1,199 @@
+"""Multi-GPU key-switching: one process per GPU, torch.distributed plumbing.
+
+* Data parallel (independent ciphertexts, P1): `dp_slice` partitions a batch; every rank
+  runs the single-GPU C-ABI path on its slice and no collective touches the data.
+  bench.py uses this for `--gpus N` (weak scaling).
+* Limb-sharded key-switch (P2): one key-switch at level l is split by RNS limb.  Each rank
+  owns a contiguous block of the Q limbs and of the P limbs of PQ_l.  NTT, KeyIP and the
+  ModDown tail are limb-local; only BConv needs other limbs, so the path has exactly two
+  exchange steps, both all-gathers of coefficient-form limbs:
+      INTT(own Q) -> ALL-GATHER Q -> ModUp BConv (own targets) -> NTT -> KeyIP (own limbs)
+      -> INTT(own P) -> ALL-GATHER P -> ModDown BConv (own Q) -> NTT -> (acc - conv) P^-1
+  (Table 2, Fig. 5).  The output stays sharded by Q limb.
+
+The orchestration below is host logic only.  Every arithmetic step goes through an `ops`
+backend: `NeoOps` runs the CUDA library through its C-ABI on the rank's GPU and gathers
+over NCCL.  The CPU tests run the same orchestration with a test-only backend built on the
+oracle over gloo (tests/test_dist_gloo.py).
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+
+def dp_slice(total: int, world: int, rank: int) -> tuple[int, int]:
+    """Contiguous, balanced slice [start, start+count) of `total` items for `rank`."""
+    base, extra = divmod(total, world)
+    start = rank * base + min(rank, extra)
+    return start, base + (1 if rank < extra else 0)
+
+
+def limb_blocks(ids: list[int], world: int) -> list[list[int]]:
+    """Split a limb-id list into `world` contiguous, balanced blocks (some may be empty)."""
+    out = []
+    for r in range(world):
+        s, n = dp_slice(len(ids), world, r)
+        out.append(ids[s:s + n])
+    return out
+
+
+def max_over_ranks(value: float, group=None) -> float:
+    """Max of a host float over all ranks (timing is reported as the slowest rank)."""
+    if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
+        return float(value)
+    backend = dist.get_backend(group)
+    dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else torch.device("cpu")
+    t = torch.tensor([float(value)], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return float(t.item())
+
+
+class ShardPlan:
+    """Limb ownership for a key-switch at `level` (digits of Z8: D_j = [j alpha, ...))."""
+
+    def __init__(self, level: int, num_q: int, num_p: int, alpha: int, world: int, rank: int):
+        self.level, self.num_q, self.num_p, self.alpha = level, num_q, num_p, alpha
+        self.world, self.rank = world, rank
+        self.q_ids = list(range(level + 1))
+        self.p_ids = list(range(num_q, num_q + num_p))
+        self.q_blocks = limb_blocks(self.q_ids, world)
+        self.p_blocks = limb_blocks(self.p_ids, world)
+        self.my_q = self.q_blocks[rank]
+        self.my_p = self.p_blocks[rank]
+        self.mine = self.my_q + self.my_p                 # this rank's limbs of PQ_l
+        beta = -(-(level + 1) // alpha)
+        self.digits = [list(range(j * alpha, min((j + 1) * alpha, level + 1))) for j in range(beta)]
+        self.beta = beta
+
+
+def limb_sharded_keyswitch(ops, plan: ShardPlan, d_local, evk):
+    """One key-switch of the rank's Q limbs `d_local` [B][len(my_q)][N] (NTT form).
+
+    Returns (k0, k1) restricted to this rank's Q limbs, each [B][len(my_q)][N].
+    """
+    P = plan
+    # a3: INTT of the rank's Q limbs, then exchange #1: every rank gets all Q limbs
+    y_local = ops.intt(d_local, P.my_q)
+    y_all = ops.allgather(y_local, [len(b) for b in P.q_blocks])          # [B][l+1][N]
+    # a4/a5: ModUp of every digit onto this rank's own target limbs, then NTT
+    if not P.my_q:
+        raise ValueError("limb-sharded key-switch needs world <= level + 1 (every rank owns a Q limb)")
+    dhat_rows = []                                                          # per digit: [B][n_mine][N]
+    for dj in P.digits:
+        targets = [t for t in P.mine if t not in dj]
+        up = ops.ntt(ops.bconv(ops.take(y_all, dj), dj, targets), targets) if targets else None
+        rows = []
+        for t in P.mine:
+            if t in dj:
+                rows.append(ops.take(d_local, [P.my_q.index(t)]))           # digit's own limb: d_t
+            else:
+                rows.append(ops.take(up, [targets.index(t)]))
+        dhat_rows.append(ops.cat(rows, axis=1))
+    acc = ops.keyip(ops.stack(dhat_rows, axis=1), P.mine, P.beta, evk)       # a6 -> [B][2][n_mine][N]
+    # a7: INTT of the rank's P limbs of acc, exchange #2: every rank gets all P limbs
+    p_pos = [P.mine.index(t) for t in P.my_p]
+    acc_p_local = ops.intt2(ops.take2(acc, p_pos), P.my_p) if p_pos else ops.empty2(acc, 0)
+    acc_p_all = ops.allgather2(acc_p_local, [len(b) for b in P.p_blocks])  # [B][2][num_p][N]
+    # a8/a9: ModDown BConv onto the rank's Q limbs, NTT, a10: combine
+    conv = ops.ntt2(ops.bconv2(acc_p_all, P.p_ids, P.my_q), P.my_q)
+    q_pos = [P.mine.index(t) for t in P.my_q]
+    out = ops.moddown_combine(ops.take2(acc, q_pos), conv, P.my_q)          # [B][2][n_q][N]
+    return ops.component(out, 0), ops.component(out, 1)
+
+
+class NeoOps:
+    """The CUDA library (C-ABI) as the backend of `limb_sharded_keyswitch`, NCCL gathers."""
+
+    def __init__(self, ctx, group=None, stream=None):
+        from . import neo
+        self.neo, self.ctx, self.group, self.stream = neo, ctx, group, stream
+
+    # ---- tensor plumbing (torch.uint64 CUDA tensors)
+    @staticmethod
+    def take(x, idx):
+        return x[:, idx].contiguous()
+
+    @staticmethod
+    def take2(x, idx):
+        return x[:, :, idx].contiguous()
+
+    @staticmethod
+    def cat(xs, axis):
+        return torch.cat(xs, dim=axis).contiguous()
+
+    @staticmethod
+    def stack(xs, axis):
+        return torch.stack(xs, dim=axis).contiguous()
+
+    @staticmethod
+    def component(x, c):
+        return x[:, c].contiguous()
+
+    @staticmethod
+    def empty2(like, n):
+        return torch.empty((like.shape[0], 2, n, like.shape[-1]), dtype=torch.uint64, device=like.device)
+
+    def _gather(self, x, sizes, dim):
+        world = len(sizes)
+        if world == 1:
+            return x
+        m = max(sizes)
+        shape = list(x.shape)
+        shape[dim] = m
+        pad = torch.zeros(shape, dtype=torch.uint64, device=x.device)
+        pad.narrow(dim, 0, x.shape[dim]).copy_(x)
+        if dist.get_backend(self.group) == "nccl":            # device-to-device over NVLink
+            parts = [torch.empty_like(pad) for _ in range(world)]
+            dist.all_gather([p.view(torch.int64) for p in parts], pad.view(torch.int64), group=self.group)
+        else:                                                  # gloo (tests: several ranks on one GPU)
+            host = pad.cpu()
+            parts = [torch.empty_like(host) for _ in range(world)]
+            dist.all_gather([p.view(torch.int64) for p in parts], host.view(torch.int64), group=self.group)
+            parts = [p.to(x.device) for p in parts]
+        return torch.cat([p.narrow(dim, 0, n) for p, n in zip(parts, sizes)], dim=dim).contiguous()
+
+    def allgather(self, x, sizes):
+        return self._gather(x, sizes, 1)
+
+    def allgather2(self, x, sizes):
+        return self._gather(x, sizes, 2)
+
+    # ---- arithmetic through the C-ABI
+    def intt(self, x, ids):
+        y = x.clone()
+        self.neo.neo_intt(self.ctx, y, ids, y.shape[0], torch.empty_like(y), self.stream)
+        return y
+
+    def ntt(self, x, ids):
+        y = x.clone()
+        self.neo.neo_ntt(self.ctx, y, ids, y.shape[0], torch.empty_like(y), self.stream)
+        return y
+
+    def intt2(self, x, ids):
+        B = x.shape[0]
+        return self.intt(x.reshape(2 * B, len(ids), -1), ids).reshape(x.shape)
+
+    def ntt2(self, x, ids):
+        B = x.shape[0]
+        return self.ntt(x.reshape(2 * B, len(ids), -1), ids).reshape(x.shape)
+
+    def bconv(self, x, src, dst):
+        out = torch.empty((x.shape[0], len(dst), x.shape[-1]), dtype=torch.uint64, device=x.device)
+        self.neo.neo_bconv(self.ctx, x, src, out, dst, x.shape[0], self.stream)
+        return out
+
+    def bconv2(self, x, src, dst):
+        B = x.shape[0]
+        return self.bconv(x.reshape(2 * B, len(src), -1), src, dst).reshape(B, 2, len(dst), -1)
+
+    def keyip(self, dhat, ids, beta, evk):
+        B = dhat.shape[0]
+        acc = torch.empty((B, 2, len(ids), dhat.shape[-1]), dtype=torch.uint64, device=dhat.device)
+        self.neo.neo_keyip(self.ctx, evk, dhat, ids, beta, acc, B, self.stream)
+        return acc
+
+    def moddown_combine(self, acc, conv, q_ids):
+        out = torch.empty_like(acc)
+        self.neo.neo_moddown_combine(self.ctx, acc, conv, q_ids, out, acc.shape[0], self.stream)
+        return out
