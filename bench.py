@@ -174,7 +174,10 @@ def load_traffic(kind: str):
     try:
         with open(p) as f:
             d = json.load(f)
-        return d.get(kind)
+        e = d.get(kind)
+        return None if e is None else {"bytes_per_launch": e["bytes_per_launch"],
+                                       "algo_bytes_per_launch": e["algo_bytes_per_launch"],
+                                       "launch": e["launch"], "source": "profiles/ncu_traffic.json (r01 ncu --set full)"}
     except Exception:
         return None
 

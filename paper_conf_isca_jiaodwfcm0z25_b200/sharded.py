@@ -109,26 +109,27 @@ class NeoOps:
         from . import neo
         self.neo, self.ctx, self.group, self.stream = neo, ctx, group, stream
 
-    # ---- tensor plumbing (torch.uint64 CUDA tensors)
+    # ---- tensor plumbing (torch.uint64 CUDA tensors, moved through int64 views because
+    #      torch implements few uint64 CUDA ops; the bits are unchanged)
     @staticmethod
     def take(x, idx):
-        return x[:, idx].contiguous()
+        return x.view(torch.int64)[:, idx].contiguous().view(torch.uint64)
 
     @staticmethod
     def take2(x, idx):
-        return x[:, :, idx].contiguous()
+        return x.view(torch.int64)[:, :, idx].contiguous().view(torch.uint64)
 
     @staticmethod
     def cat(xs, axis):
-        return torch.cat(xs, dim=axis).contiguous()
+        return torch.cat([x.view(torch.int64) for x in xs], dim=axis).contiguous().view(torch.uint64)
 
     @staticmethod
     def stack(xs, axis):
-        return torch.stack(xs, dim=axis).contiguous()
+        return torch.stack([x.view(torch.int64) for x in xs], dim=axis).contiguous().view(torch.uint64)
 
     @staticmethod
     def component(x, c):
-        return x[:, c].contiguous()
+        return x.view(torch.int64)[:, c].contiguous().view(torch.uint64)
 
     @staticmethod
     def empty2(like, n):
@@ -141,17 +142,17 @@ class NeoOps:
         m = max(sizes)
         shape = list(x.shape)
         shape[dim] = m
-        pad = torch.zeros(shape, dtype=torch.uint64, device=x.device)
-        pad.narrow(dim, 0, x.shape[dim]).copy_(x)
+        pad = torch.zeros(shape, dtype=torch.int64, device=x.device)
+        pad.narrow(dim, 0, x.shape[dim]).copy_(x.view(torch.int64))
         if dist.get_backend(self.group) == "nccl":            # device-to-device over NVLink
             parts = [torch.empty_like(pad) for _ in range(world)]
-            dist.all_gather([p.view(torch.int64) for p in parts], pad.view(torch.int64), group=self.group)
+            dist.all_gather(parts, pad, group=self.group)
         else:                                                  # gloo (tests: several ranks on one GPU)
             host = pad.cpu()
             parts = [torch.empty_like(host) for _ in range(world)]
-            dist.all_gather([p.view(torch.int64) for p in parts], host.view(torch.int64), group=self.group)
+            dist.all_gather(parts, host, group=self.group)
             parts = [p.to(x.device) for p in parts]
-        return torch.cat([p.narrow(dim, 0, n) for p, n in zip(parts, sizes)], dim=dim).contiguous()
+        return torch.cat([p.narrow(dim, 0, n) for p, n in zip(parts, sizes)], dim=dim).contiguous().view(torch.uint64)
 
     def allgather(self, x, sizes):
         return self._gather(x, sizes, 1)
@@ -161,12 +162,12 @@ class NeoOps:
 
     # ---- arithmetic through the C-ABI
     def intt(self, x, ids):
-        y = x.clone()
+        y = x.view(torch.int64).clone().view(torch.uint64)
         self.neo.neo_intt(self.ctx, y, ids, y.shape[0], torch.empty_like(y), self.stream)
         return y
 
     def ntt(self, x, ids):
-        y = x.clone()
+        y = x.view(torch.int64).clone().view(torch.uint64)
         self.neo.neo_ntt(self.ctx, y, ids, y.shape[0], torch.empty_like(y), self.stream)
         return y
 
