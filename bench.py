@@ -222,7 +222,7 @@ def run_reference(args):
     line = {"metric": METRIC, "value": v, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * el / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
-            "data": "synthetic", "config": dict(workload_config(1, 1), workload="setB_keyswitch"),
+            "data": "synthetic", "config": dict(workload_config(1, 1), workload="setB_keyswitch", ks_per_step_per_gpu=1),
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                              "sample": "each step = one Set-B key-switch (l=35, B=1) by the CPU oracle"},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}

@@ -15,6 +15,8 @@
 // shared memory in the SWIZZLE_NONE K-major layout, B (<= 16 KB) is loaded once per CTA,
 // the accumulator D lives in TMEM (256 columns) and is drained with tcgen05.ld.
 // D_b <= 60 * 255 * 255 < 2^22, so s32 accumulation is exact.
+#include <cstdlib>
+
 #include "bconv_tc.h"
 #include "common.cuh"
 #include "tc.cuh"
@@ -23,14 +25,15 @@ namespace neo {
 
 constexpr int kTileM = 128;
 constexpr int kStages = 2;                         // A-tile stages and TMEM accumulators
-constexpr int kInStages = 4;                       // TMA input stages (12 KB each)
+constexpr int kInStages = 8;                       // TMA input stages (12 KB each)
 constexpr int kAccCols = 256;                      // TMEM columns per accumulator (N <= 256)
-constexpr int kEpiWarps = 16;                      // four per TMEM lane quarter (target quarters)
+constexpr int kEpiParts = 5;                       // target groups of 8 split over 5 warp sets
+constexpr int kEpiWarps = 4 * kEpiParts;           // per TMEM lane quarter: one warp per part
 constexpr int kThreads = (4 + kEpiWarps + 1) * 32; // producers, epilogue, MMA
 constexpr size_t kInBytes = (size_t)BCTC_MAX_IN * kTileM * 8;
 constexpr int kMaxJobs = 4;                        // conversions fused into one launch (ModUp digits)
 constexpr size_t kSmemBytes = kStages * kTileM * 64 + kMaxJobs * 256 * 64 + kInStages * kInBytes;  // 128 KB
-constexpr size_t kSmemAlloc = 160 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
+constexpr size_t kSmemAlloc = 200 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
 static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocation");
 
 // Warp-specialised pipeline (one persistent CTA per SM):
@@ -45,7 +48,7 @@ static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocati
 // so HBM reads run 3 tiles ahead, and the MMA of tile i overlaps the epilogue of i-1.
 template <class LoadB>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
-                                              int tiles_per_entry, int batch) {
+                                              int tiles_per_entry, int batch, int exp) {
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t* sA = smem;                                 // kStages x (128 rows x 64 B)
     uint8_t* sB0 = smem + kStages * kTileM * 64;        // kMaxJobs x (ncols rows x 64 B)
@@ -68,14 +71,14 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     if (warp == 0) tc::tmem_alloc(&tmem_base, kStages * kAccCols);
     if (tid == 0) {
         for (int s = 0; s < kStages; ++s) {
-            tc::mbar_init(&full_a[s], kTileM);
+            tc::mbar_init(&full_a[s], 4);                  // one arrival per producer warp
             tc::mbar_init(&empty_a[s], 1);
             tc::mbar_init(&tfull[s], 1);
-            tc::mbar_init(&tempty[s], kEpiWarps * 32);
+            tc::mbar_init(&tempty[s], kEpiWarps);          // one arrival per epilogue warp
         }
         for (int s = 0; s < kInStages; ++s) {
             tc::mbar_init(&in_full[s], 1);
-            tc::mbar_init(&in_empty[s], kTileM);
+            tc::mbar_init(&in_empty[s], 4);
         }
     }
     for (int j = 0; j < njobs; ++j) {
@@ -91,7 +94,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     // TMA issue of tile index i (i-th tile of this CTA) into input stage i % kInStages
     auto tma_issue = [&](int i) {
         const int tile = blockIdx.x + i * G;
-        if (tile >= total_tiles) return;
+        if (tile >= total_tiles || (exp & 32)) return;
         const int s = i % kInStages, k = i / kInStages;
         tc::mbar_wait(&in_empty[s], (k & 1) ^ 1);
         int jb, b, m0;
@@ -117,12 +120,13 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             decode(tile, jb, b, m0);
             const BConvTC& P = PJ[jb];
             const int si = i % kInStages, ki = i / kInStages;
-            tc::mbar_wait(&in_full[si], ki & 1);
+            if (!(exp & 32)) tc::mbar_wait(&in_full[si], ki & 1);
             const u64* src = sIn + (size_t)si * BCTC_MAX_IN * kTileM + tid;
             u64 c[BCTC_MAX_IN];
 #pragma unroll
             for (int j = 0; j < BCTC_MAX_IN; ++j) c[j] = (j < P.n_in) ? src[j * kTileM] : 0;
-            tc::mbar_arrive(&in_empty[si]);
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&in_empty[si]);
             uint32_t w[16];
 #pragma unroll
             for (int kk = 0; kk < 16; ++kk) w[kk] = 0;
@@ -130,7 +134,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             for (int j = 0; j < BCTC_MAX_IN; ++j) {
                 if (j < P.n_in) {
                     const double q = P.qin[j];
-                    const u64 y = d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
+                    const u64 y = (exp & 2) ? c[j] : d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
                     const int bit = 40 * j, wi = bit >> 5, sh = bit & 31;
                     w[wi] |= (uint32_t)(y << sh);
                     w[wi + 1] |= (uint32_t)(y >> (32 - sh));
@@ -145,7 +149,8 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                 *reinterpret_cast<uint4*>(arow + cc * 128) =
                     make_uint4(w[4 * cc], w[4 * cc + 1], w[4 * cc + 2], w[4 * cc + 3]);
             tc::fence_proxy_async();
-            tc::mbar_arrive(&full_a[s]);
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&full_a[s]);
         }
     } else if (warp < 4 + kEpiWarps) {
         // ------------------------------------------------ epilogue
@@ -163,18 +168,25 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             tc::fence_after();
             const uint32_t trow = tmem + (uint32_t)(s * kAccCols) + ((uint32_t)(quarter * 32) << 16);
             u64* outb = io.out + b * io.out_bstride + m;
-            for (int g = 8 * part; g < P.n_out; g += 8 * (kEpiWarps / 4)) {
+            for (int g = 8 * part; g < P.n_out; g += 8 * kEpiParts) {
                 uint32_t v[40];
+                if (exp & 8) {
 #pragma unroll
-                for (int q5 = 0; q5 < 5; ++q5) {
-                    uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * q5]);
-                    tc::tmem_ld8(trow + (uint32_t)(5 * g + 8 * q5), vv);
+                    for (int q5 = 0; q5 < 40; ++q5) v[q5] = q5 + g;
+                } else {
+#pragma unroll
+                    for (int q5 = 0; q5 < 5; ++q5) {
+                        uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * q5]);
+                        tc::tmem_ld8(trow + (uint32_t)(5 * g + 8 * q5), vv);
+                    }
+                    tc::tmem_wait_ld();
                 }
-                tc::tmem_wait_ld();
 #pragma unroll
                 for (int u = 0; u < 8; ++u) {
                     const int t = g + u;
-                    if (t < P.n_out) {
+                    if (t < P.n_out && (exp & 1)) {
+                        if (!(exp & 4) || v[5 * u] == 0x12345u) outb[(size_t)io.out_off[t] * N] = v[5 * u] + v[5 * u + 4];
+                    } else if (t < P.n_out) {
                         const uint32_t* D = &v[5 * u];
                         const u64 lo = (u64)D[0] + ((u64)D[1] << 8) + ((u64)D[2] << 16);     // < 2^39
                         const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
@@ -185,7 +197,8 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                 }
             }
             tc::fence_before();
-            tc::mbar_arrive(&tempty[s]);
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&tempty[s]);
         }
     } else {
         // ------------------------------------------------ MMA issuer
@@ -204,8 +217,10 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                 const uint32_t acc = tmem + (uint32_t)(s * kAccCols);
                 const uint32_t as = aaddr + s * (kTileM * 64);
                 // K = 64 as two K = 32 steps (LBO = 128 B between K chunks, SBO = 512 B between row groups)
-                tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(baddr, 128, 512), idesc, 0);
-                tc::mma_u8(acc, tc::sdesc(as + 256, 128, 512), tc::sdesc(baddr + 256, 128, 512), idesc, 1);
+                if (!(exp & 16)) {
+                    tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(baddr, 128, 512), idesc, 0);
+                    tc::mma_u8(acc, tc::sdesc(as + 256, 128, 512), tc::sdesc(baddr + 256, 128, 512), idesc, 1);
+                }
                 tc::commit(&empty_a[s]);
                 tc::commit(&tfull[s]);
             }
@@ -218,15 +233,15 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
-k_bconv_tc_g(const __grid_constant__ BConvMulti M, int N, int tiles_per_entry, int batch) {
+k_bconv_tc_g(const __grid_constant__ BConvMulti M, int N, int tiles_per_entry, int batch, int exp) {
     bconv_tc_body(M.P, M.io, M.njobs, [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; }, N,
-                  tiles_per_entry, batch);
+                  tiles_per_entry, batch, exp);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_p(const __grid_constant__ BConvTC P, const __grid_constant__ BConvIO io,
              const __grid_constant__ BMatParam B, int N, int tiles_per_entry, int batch) {
-    bconv_tc_body(&P, &io, 1, [&](int, int e) { return B.d[e]; }, N, tiles_per_entry, batch);
+    bconv_tc_body(&P, &io, 1, [&](int, int e) { return B.d[e]; }, N, tiles_per_entry, batch, 0);
 }
 
 size_t bconv_tc_smem(int) { return kSmemAlloc; }
@@ -245,7 +260,8 @@ cudaError_t launch_bconv_tc(const BConvMulti& M, int N, int batch, int num_sms, 
     const int tiles_per_entry = N / kTileM;
     const int total = tiles_per_entry * batch * M.njobs;
     const int grid = num_sms < total ? num_sms : total;
-    k_bconv_tc_g<<<grid, kThreads, kSmemAlloc, st>>>(M, N, tiles_per_entry, batch);
+    static const int exp = [] { const char* e = std::getenv("NEO_BCONV_EXP"); return e ? std::atoi(e) : 0; }();
+    k_bconv_tc_g<<<grid, kThreads, kSmemAlloc, st>>>(M, N, tiles_per_entry, batch, exp);   // exp != 0: timing experiments only
     return cudaGetLastError();
 }
 
