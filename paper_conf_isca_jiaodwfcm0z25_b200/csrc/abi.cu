@@ -73,7 +73,7 @@ struct ProfScope {
 // rows k < n of batch entry b: src + b*src_bs + src_off[k]*N  ->  dst + b*dst_bs + dst_off[k]*N
 static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long src_bs, const int* src_off,
                            u64* dst, long long dst_bs, const int* dst_off, const int* prime, int n, u64* tmp,
-                           int batch, cudaStream_t st) {
+                           int batch, cudaStream_t st, const RowEpi* epi = nullptr) {
     if (n <= 0) return NEO_OK;
     if (n > NEO_MAX_ROWS) FAIL(NEO_EUNSUPPORTED, "too many limb rows in one transform");
     RowSet a, b;
@@ -90,7 +90,7 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
     }
     // forward: column pass then row pass; inverse: row pass then column pass
     LAUNCH(fwd ? PK_NTT_COL : PK_NTT_ROW, st, ntt_pass(fwd, a, c->ntt, batch, fwd, st));
-    LAUNCH(fwd ? PK_NTT_ROW : PK_NTT_COL, st, ntt_pass(!fwd, b, c->ntt, batch, fwd, st));
+    LAUNCH(fwd ? PK_NTT_ROW : PK_NTT_COL, st, ntt_pass(!fwd, b, c->ntt, batch, fwd, st, epi));
     return NEO_OK;
 }
 
@@ -230,24 +230,20 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
             LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, 2 * B, st));
     }
 
-    // a9: NTT of conv (in place through tmp)
+    // a9 + a10: NTT of conv, with the ModDown tail (acc - conv) * P^-1 (+ add) fused into the
+    // epilogue of the row pass (conv is never written back)
     for (int i = 0; i < Lq; ++i) { so[i] = dof[i] = i; pr[i] = i; }
-    if ((s = ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st)))
-        return s;
-
-    // a10: combine
     {
-        CombineArgs A;
-        A.acc = acc; A.conv = conv; A.add0 = add0; A.add1 = add1; A.out0 = out0; A.out1 = out1;
-        A.mods = c->d_mods;
-        A.acc_bstride = (long long)2 * E * N;
-        A.acc_cstride = (long long)E * N;
-        A.conv_stride = (long long)Lq * N;
-        A.add_bstride = add_bs;
-        A.out_bstride = out_bs;
-        A.N = N;
-        for (int i = 0; i < Lq; ++i) { A.pinv[i] = c->pinv[i]; A.limb[i] = i; }
-        LAUNCH(PK_COMBINE, st, launch_combine(A, Lq, B, st));
+        RowEpi ep;
+        ep.acc = acc;
+        ep.acc_b = (long long)2 * E * N;
+        ep.acc_c = (long long)E * N;
+        ep.add0 = add0; ep.add1 = add1; ep.add_b = add_bs;
+        ep.out0 = out0; ep.out1 = out1; ep.out_b = out_bs;
+        for (int i = 0; i < Lq; ++i) ep.pinv[i] = c->pinv[i];
+        if ((s = ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st,
+                          &ep)))
+            return s;
     }
     return NEO_OK;
 }

@@ -47,26 +47,50 @@ k_bconv(BConvTab T, BConvIO io, int N) {
 }
 
 // ------------------------------------------------------------------ KeyIP (Alg. 3)
-// acc_c[t] = sum_j dhat_j[t] * evk_{j,c}[t] mod t for c = 0, 1 (L359-382); the evk is
-// read once per launch and shared by the whole batch in L2 (Z21).
-__global__ void __launch_bounds__(256)
-k_keyip(KeyIPArgs A) {
-    const int n = blockIdx.x * blockDim.x + threadIdx.x;
-    const int t = blockIdx.y, b = blockIdx.z;
-    if (n >= A.N) return;
+// acc_c[t] = sum_j dhat_j[t] * evk_{j,c}[t] mod t for c = 0, 1 (L359-382).  One thread per
+// (limb, coefficient) holds its 2*beta key words in registers and walks the whole batch, so
+// the key is read from HBM once per launch however large the batch (Z21; the CUDA-core IP
+// mapping of L488 with the evaluation key reused across the batch).
+template <int BETA>
+__device__ __forceinline__ void keyip_body(const KeyIPArgs& A, int n, int t, int batch) {
+    static_assert(BETA >= 1 && BETA <= KS_MAX_BETA, "beta out of range");
     const ModQ m = A.mods[A.limb[t]];
-    u64 h0 = 0, l0 = 0, h1 = 0, l1 = 0;
-    for (int j = 0; j < A.beta; ++j) {
-        const int so = A.src_off[j][t];
-        const u64* src = (A.src_kind[j][t] ? A.up + b * A.up_bstride : A.d + b * A.d_bstride);
-        const u64 x = src[(size_t)so * A.N + n];
+    u64 e0[BETA], e1[BETA];
+    const u64* src[BETA];
+    long long sb[BETA];
+#pragma unroll
+    for (int j = 0; j < BETA; ++j) {
         const u64* e = A.evk + ((size_t)(2 * j) * A.evk_limbs + A.limb[t]) * A.N + n;
-        mac128(h0, l0, x, e[0]);
-        mac128(h1, l1, x, e[(size_t)A.evk_limbs * A.N]);
+        e0[j] = e[0];
+        e1[j] = e[(size_t)A.evk_limbs * A.N];
+        const bool up = A.src_kind[j][t];
+        src[j] = (up ? A.up : A.d) + (size_t)A.src_off[j][t] * A.N + n;
+        sb[j] = up ? A.up_bstride : A.d_bstride;
     }
-    u64* acc = A.acc + b * A.acc_bstride + (size_t)t * A.N + n;
-    acc[0] = barrett_reduce(h0, l0, m);
-    acc[(size_t)A.acc_cstride] = barrett_reduce(h1, l1, m);
+    u64* acc = A.acc + (size_t)t * A.N + n;
+    for (int b = 0; b < batch; ++b) {
+        u64 x[BETA];
+#pragma unroll
+        for (int j = 0; j < BETA; ++j) x[j] = src[j][b * sb[j]];
+        u64 h0 = 0, l0 = 0, h1 = 0, l1 = 0;
+#pragma unroll
+        for (int j = 0; j < BETA; ++j) {
+            mac128(h0, l0, x[j], e0[j]);
+            mac128(h1, l1, x[j], e1[j]);
+        }
+        u64* o = acc + b * A.acc_bstride;
+        o[0] = barrett_reduce(h0, l0, m);
+        o[(size_t)A.acc_cstride] = barrett_reduce(h1, l1, m);
+    }
+}
+
+template <int BETA>
+__global__ void __launch_bounds__(256)
+k_keyip(const __grid_constant__ KeyIPArgs A, int batch) {
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int t = blockIdx.y;
+    if (n >= A.N) return;
+    keyip_body<BETA>(A, n, t, batch);
 }
 
 // ------------------------------------------------------------------ combine (ModDown tail)
@@ -151,7 +175,17 @@ cudaError_t launch_bconv(const BConvTab& T, const BConvIO& io, int N, int batch,
     return cudaGetLastError();
 }
 cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t st) {
-    k_keyip<<<dim3((A.N + 255) / 256, limbs, batch), 256, 0, st>>>(A);
+    const dim3 g((A.N + 255) / 256, limbs);
+    switch (A.beta) {
+        case 1: k_keyip<1><<<g, 256, 0, st>>>(A, batch); break;
+        case 2: k_keyip<2><<<g, 256, 0, st>>>(A, batch); break;
+        case 3: k_keyip<3><<<g, 256, 0, st>>>(A, batch); break;
+        case 4: k_keyip<4><<<g, 256, 0, st>>>(A, batch); break;
+        case 5: k_keyip<5><<<g, 256, 0, st>>>(A, batch); break;
+        case 6: k_keyip<6><<<g, 256, 0, st>>>(A, batch); break;
+        case 7: k_keyip<7><<<g, 256, 0, st>>>(A, batch); break;
+        default: k_keyip<8><<<g, 256, 0, st>>>(A, batch); break;
+    }
     return cudaGetLastError();
 }
 cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStream_t st) {

@@ -245,9 +245,9 @@ struct RowCfg {
 
 // Forward: src = lazy doubles tmp[i1][n2], dst = canonical u64 a_hat[i1 + N1 i2].
 // Inverse: src = canonical u64 a_hat, dst = lazy doubles tmp[i1][n2].
-template <int R, bool FWD, int STAGES, int MINB>
+template <int R, bool FWD, int STAGES, int MINB, bool EPI>
 __global__ void __launch_bounds__(RowCfg<R>::NT, MINB)
-k_ntt_row(RowSet rs, NttArgs a, TileMap tm) {
+k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
     using CF = RowCfg<R>;
     constexpr int RR = kC, NT = CF::NT, N2 = CF::N2;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -325,10 +325,34 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm) {
 #pragma unroll
             for (int ib = 0; ib < R; ++ib) T[swz(r + R * ib, rho)] = d2u(canon(x[BitRev<R>::of(ib)], q, mq.qinv));
             __syncthreads();
-            for (int e = tid; e < N2 * 8; e += NT) {
-                const int i2 = e >> 3, p = e & 7;
-                const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
-                *reinterpret_cast<uint4*>(dst + row0 + (size_t)N1 * i2 + 2 * p) = v;
+            if (!EPI) {
+                for (int e = tid; e < N2 * 8; e += NT) {
+                    const int i2 = e >> 3, p = e & 7;
+                    const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
+                    *reinterpret_cast<uint4*>(dst + row0 + (size_t)N1 * i2 + 2 * p) = v;
+                }
+            } else {      // fused ModDown tail (a10): out = (acc - conv) P^-1 (+ add)
+                const int bb = b >> 1, cc = b & 1;
+                const u64 qq = mq.q;
+                const TW pinv = ep.pinv[k];
+                const u64* accr = ep.acc + bb * ep.acc_b + cc * ep.acc_c + (size_t)k * a.N;
+                const u64* addr = cc ? ep.add1 : ep.add0;
+                if (addr) addr += bb * ep.add_b + (size_t)k * a.N;
+                u64* outr = (cc ? ep.out1 : ep.out0) + bb * ep.out_b + (size_t)k * a.N;
+                for (int e = tid; e < N2 * 8; e += NT) {
+                    const int i2 = e >> 3, p = e & 7;
+                    const size_t pos = row0 + (size_t)N1 * i2 + 2 * p;
+                    const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
+                    const uint4 av = *reinterpret_cast<const uint4*>(accr + pos);
+                    u64 r0 = shoup(sub_mod(((u64)av.y << 32) | av.x, ((u64)v.y << 32) | v.x, qq), pinv, qq);
+                    u64 r1 = shoup(sub_mod(((u64)av.w << 32) | av.z, ((u64)v.w << 32) | v.z, qq), pinv, qq);
+                    if (addr) {
+                        const uint4 dv = *reinterpret_cast<const uint4*>(addr + pos);
+                        r0 = add_mod(r0, ((u64)dv.y << 32) | dv.x, qq);
+                        r1 = add_mod(r1, ((u64)dv.w << 32) | dv.z, qq);
+                    }
+                    *reinterpret_cast<uint4*>(outr + pos) = make_uint4((unsigned)r0, (unsigned)(r0 >> 32), (unsigned)r1, (unsigned)(r1 >> 32));
+                }
             }
         } else {
             const u64* T = reinterpret_cast<const u64*>(sD);
@@ -368,12 +392,16 @@ static int ntt_cfg() {
 }
 
 template <int R, bool FWD, int STAGES, int MINB>
-static cudaError_t launch_cfg(bool col, const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st) {
+static cudaError_t launch_cfg(bool col, const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st,
+                             const RowEpi* epi) {
     static bool init = false;
     const size_t smc = STAGES * ColCfg<R>::STAGE, smr = STAGES * RowCfg<R>::STAGE;
     if (!init) {
         cudaFuncSetAttribute(k_ntt_col<R, FWD, STAGES, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc);
-        cudaFuncSetAttribute(k_ntt_row<R, FWD, STAGES, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smr);
+        cudaFuncSetAttribute(k_ntt_row<R, FWD, STAGES, MINB, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)smr);
+        cudaFuncSetAttribute(k_ntt_row<R, FWD, STAGES, MINB, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)smr);
         init = true;
     }
     TileMap tm;
@@ -382,27 +410,34 @@ static cudaError_t launch_cfg(bool col, const RowSet& rs, const NttArgs& a, int 
     tm.total = tm.tpr * rs.n * batch;
     int grid = MINB * a.num_sms;
     if (grid > tm.total) grid = tm.total;
-    if (col)
+    if (col) {
         k_ntt_col<R, FWD, STAGES, MINB><<<grid, ColCfg<R>::NT, smc, st>>>(rs, a, tm);
-    else
-        k_ntt_row<R, FWD, STAGES, MINB><<<grid, RowCfg<R>::NT, smr, st>>>(rs, a, tm);
+    } else if (epi) {
+        if (!FWD) return cudaErrorInvalidValue;
+        k_ntt_row<R, FWD, STAGES, MINB, true><<<grid, RowCfg<R>::NT, smr, st>>>(rs, a, tm, *epi);
+    } else {
+        static const RowEpi none{};
+        k_ntt_row<R, FWD, STAGES, MINB, false><<<grid, RowCfg<R>::NT, smr, st>>>(rs, a, tm, none);
+    }
     return cudaGetLastError();
 }
 
 template <int R, bool FWD>
-static cudaError_t launch_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st) {
+static cudaError_t launch_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st,
+                               const RowEpi* epi) {
     switch (ntt_cfg()) {
-        case 1: return launch_cfg<R, FWD, 1, 3>(col, rs, a, batch, st);
-        case 0: return launch_cfg<R, FWD, 2, 2>(col, rs, a, batch, st);
-        default: return launch_cfg<R, FWD, 1, 4>(col, rs, a, batch, st);
+        case 1: return launch_cfg<R, FWD, 1, 3>(col, rs, a, batch, st, epi);
+        case 0: return launch_cfg<R, FWD, 2, 2>(col, rs, a, batch, st, epi);
+        default: return launch_cfg<R, FWD, 1, 4>(col, rs, a, batch, st, epi);
     }
 }
 
-cudaError_t ntt_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, bool fwd, cudaStream_t st) {
+cudaError_t ntt_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, bool fwd, cudaStream_t st,
+                     const RowEpi* epi) {
     if (rs.n == 0 || batch == 0) return cudaSuccess;
     switch (a.L.R) {
-        case 8: return fwd ? launch_pass<8, true>(col, rs, a, batch, st) : launch_pass<8, false>(col, rs, a, batch, st);
-        case 16: return fwd ? launch_pass<16, true>(col, rs, a, batch, st) : launch_pass<16, false>(col, rs, a, batch, st);
+        case 8: return fwd ? launch_pass<8, true>(col, rs, a, batch, st, epi) : launch_pass<8, false>(col, rs, a, batch, st, epi);
+        case 16: return fwd ? launch_pass<16, true>(col, rs, a, batch, st, epi) : launch_pass<16, false>(col, rs, a, batch, st, epi);
         default: return cudaErrorInvalidValue;
     }
 }

@@ -14,9 +14,25 @@ struct NttArgs {
     NttLayout L;
 };
 
+// Optional epilogue of the forward row pass for the ModDown NTT (a9 + a10 fused):
+// instead of storing conv = NTT(...) the pass stores, for batch index bc = 2b + c and row k,
+//   out_c[b][k] = (acc[b][c][k] - conv) * P^-1 mod q  (+ add_c[b][k])
+struct RowEpi {
+    const u64* acc;
+    long long acc_b, acc_c;
+    const u64* add0;
+    const u64* add1;
+    long long add_b;
+    u64* out0;
+    u64* out1;
+    long long out_b;
+    TW pinv[64];          // per row k
+};
+
 // One pass over batch x rs.n limb rows.  Forward NTT = column pass (src -> tmp) then row
 // pass (tmp -> dst); inverse = row pass then column pass.  src and dst of one pass must
 // not overlap.
-cudaError_t ntt_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, bool fwd, cudaStream_t st);
+cudaError_t ntt_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, bool fwd, cudaStream_t st,
+                     const RowEpi* epi = nullptr);
 
 }  // namespace neo
