@@ -10,10 +10,10 @@
 //   out_t[m]     = sum_b 2^(8b) D_b[m, t]  mod t                 (epilogue, FP64)
 //
 // so sum_b 2^(8b) D_b == sum_i y_i (qhat_i mod t) (mod t): Algorithm 1's result exactly.
-// GEMM shape per 128-coefficient tile: M = 128, K = 5*n_in <= 64 (two K=32 MMAs),
-// N = 5*n_out rounded up to 16 (<= 256).  A (8 KB) is produced by the CUDA cores into
-// shared memory in the SWIZZLE_NONE K-major layout, B (<= 16 KB) is loaded once per CTA,
-// the accumulator D lives in TMEM (256 columns) and is drained with tcgen05.ld.
+// GEMM shape per 128-coefficient tile: M = 128, K = 5*n_in <= 64 (two K=32 MMAs), and the
+// targets split into one or two jobs of N = 5*J <= 128 columns.  A (8 KB) is produced by the
+// CUDA cores into shared memory in the SWIZZLE_NONE K-major layout, B (<= 16 KB) is loaded
+// once per CTA, the accumulators live in TMEM (4 x 128 columns) and are drained with tcgen05.ld.
 // D_b <= 60 * 255 * 255 < 2^22, so s32 accumulation is exact.
 #include <cstdlib>
 
@@ -24,57 +24,60 @@
 namespace neo {
 
 constexpr int kTileM = 128;
-constexpr int kStages = 2;                         // A-tile stages and TMEM accumulators
-constexpr int kInStages = 8;                       // TMA input stages (12 KB each)
-constexpr int kAccCols = 256;                      // TMEM columns per accumulator (N <= 256)
-constexpr int kEpiParts = 5;                       // target groups of 8 split over 5 warp sets
-constexpr int kEpiWarps = 4 * kEpiParts;           // per TMEM lane quarter: one warp per part
+constexpr int kAStages = 4;                        // A-tile ring
+constexpr int kSlots = 4;                          // TMEM accumulator ring (4 x 128 columns)
+constexpr int kSlotCols = 128;                     // per half-tile job: N = 5 * J <= 128
+constexpr int kInStages = 8;                       // TMA input ring (12 KB each)
+constexpr int kEpiWarps = 4 * kSlots;              // one 4-warp set per TMEM slot
 constexpr int kThreads = (4 + kEpiWarps + 1) * 32; // producers, epilogue, MMA
 constexpr size_t kInBytes = (size_t)BCTC_MAX_IN * kTileM * 8;
 constexpr int kMaxJobs = 4;                        // conversions fused into one launch (ModUp digits)
-constexpr size_t kSmemBytes = kStages * kTileM * 64 + kMaxJobs * 256 * 64 + kInStages * kInBytes;  // 128 KB
+constexpr size_t kBBytes = 2 * kSlotCols * 64;     // two half-matrices per conversion
+constexpr size_t kSmemBytes = kAStages * kTileM * 64 + kMaxJobs * kBBytes + kInStages * kInBytes;   // 192 KB
 constexpr size_t kSmemAlloc = 200 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
 static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocation");
 
-// Warp-specialised pipeline (one persistent CTA per SM):
-//   TMA (producer warp 0, lane 0): 1-D bulk copies of the n_in input rows of tile i+3
-//                          (1 KB each) into input stage (i+3) % 4
-//   producers (warps 0-3): y = [c qhat^-1] of one coefficient, split into bytes, write the
-//                          A row of stage s, arrive full_a[s]
-//   MMA (last warp, lane 0): wait full_a[s], tmem_empty[s]; two K=32 MMAs into accumulator
-//                          s; commit -> empty_a[s], tmem_full[s]
-//   epilogue (8 warps):    wait tmem_full[s], tcgen05.ld, combine the 5 byte-planes,
-//                          reduce mod t, store; arrive tmem_empty[s]
-// so HBM reads run 3 tiles ahead, and the MMA of tile i overlaps the epilogue of i-1.
+// Warp-specialised pipeline, one persistent CTA per SM.  A tile (128 coefficients) is split
+// into `nhalf` jobs of J targets (N = 5J <= 128 columns) so that four accumulators fit in TMEM:
+//   TMA (warp 0, lane 0): 1-D bulk copies of the n_in input rows of tile i+7 (1 KB each)
+//   producers (warps 0-3): y = [c qhat^-1] of one coefficient, split into bytes, write the A
+//                          row of A-stage i % 4, arrive full_a
+//   MMA (last warp, lane 0): per job q: wait full_a / tmem_empty[q % 4]; two K = 32 MMAs
+//                          into slot q % 4; commit -> tmem_full; after the tile's jobs
+//                          commit -> empty_a
+//   epilogue (4 sets of 4 warps, set e owns TMEM slot e): tcgen05.ld, combine the 5
+//                          byte-planes, reduce mod t, store; arrive tmem_empty[e]
+// Ring depths 8 (input) / 4 (A) / 4 (TMEM) absorb the mbarrier and TMA round trips.
 template <class LoadB>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
                                               int tiles_per_entry, int batch, int exp) {
     extern __shared__ __align__(1024) uint8_t smem[];
-    uint8_t* sA = smem;                                 // kStages x (128 rows x 64 B)
-    uint8_t* sB0 = smem + kStages * kTileM * 64;        // kMaxJobs x (ncols rows x 64 B)
-    u64* sIn = reinterpret_cast<u64*>(sB0 + kMaxJobs * 256 * 64);   // kInStages x [n_in][128]
+    uint8_t* sA = smem;                                  // kAStages x (128 rows x 64 B)
+    uint8_t* sB0 = smem + kAStages * kTileM * 64;        // kMaxJobs x 2 halves x (128 rows x 64 B)
+    u64* sIn = reinterpret_cast<u64*>(sB0 + kMaxJobs * kBBytes);   // kInStages x [n_in][128]
     const int tiles_per_job = tiles_per_entry * batch;
     const int total_tiles = tiles_per_job * njobs;
-    // tile -> (job, batch entry, first coefficient)
-    auto decode = [&](int tile, int& j, int& b, int& m0) {
+    auto decode = [&](int tile, int& j, int& b, int& m0) {   // tile -> (conversion, batch entry, first coeff)
         j = tile / tiles_per_job;
         const int r = tile - j * tiles_per_job;
         b = r / tiles_per_entry;
         m0 = (r - b * tiles_per_entry) * kTileM;
     };
-    __shared__ uint64_t full_a[kStages], empty_a[kStages], tfull[kStages], tempty[kStages];
+    __shared__ uint64_t full_a[kAStages], empty_a[kAStages], tfull[kSlots], tempty[kSlots];
     __shared__ uint64_t in_full[kInStages], in_empty[kInStages];
     __shared__ uint32_t tmem_base;
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int G = gridDim.x;
-    if (warp == 0) tc::tmem_alloc(&tmem_base, kStages * kAccCols);
+    if (warp == 0) tc::tmem_alloc(&tmem_base, kSlots * kSlotCols);
     if (tid == 0) {
-        for (int s = 0; s < kStages; ++s) {
-            tc::mbar_init(&full_a[s], 4);                  // one arrival per producer warp
+        for (int s = 0; s < kAStages; ++s) {
+            tc::mbar_init(&full_a[s], 4);                // one arrival per producer warp
             tc::mbar_init(&empty_a[s], 1);
+        }
+        for (int s = 0; s < kSlots; ++s) {
             tc::mbar_init(&tfull[s], 1);
-            tc::mbar_init(&tempty[s], kEpiWarps);          // one arrival per epilogue warp
+            tc::mbar_init(&tempty[s], 4);                // one arrival per warp of the set
         }
         for (int s = 0; s < kInStages; ++s) {
             tc::mbar_init(&in_full[s], 1);
@@ -82,29 +85,29 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         }
     }
     for (int j = 0; j < njobs; ++j) {
-        uint4* s4 = reinterpret_cast<uint4*>(sB0 + j * 256 * 64);
-        for (int e = tid; e < PJ[j].ncols * 4; e += kThreads) s4[e] = loadB(j, e);
+        uint4* s4 = reinterpret_cast<uint4*>(sB0 + j * kBBytes);
+        const int n16 = PJ[j].nhalf * kSlotCols * 4;    // 16-byte chunks (halves padded to 128 rows)
+        for (int e = tid; e < n16; e += kThreads) s4[e] = loadB(j, e);
     }
     tc::fence_proxy_async();
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
     const uint32_t tmem = tmem_base;
+    const int total_run = (exp & 256) ? 0 : total_tiles;      // exp 256: setup/teardown only
 
-    // TMA issue of tile index i (i-th tile of this CTA) into input stage i % kInStages
     auto tma_issue = [&](int i) {
         const int tile = blockIdx.x + i * G;
-        if (tile >= total_tiles || (exp & 32)) return;
+        if (tile >= total_run || (exp & 32)) return;
         const int s = i % kInStages, k = i / kInStages;
         tc::mbar_wait(&in_empty[s], (k & 1) ^ 1);
         int jb, b, m0;
         decode(tile, jb, b, m0);
         const BConvTC& P = PJ[jb];
         const BConvIO& io = IOJ[jb];
-        const uint32_t in_bytes = (uint32_t)P.n_in * kTileM * 8;
         const u64* in = io.in + b * io.in_bstride + m0;
         u64* dst = sIn + (size_t)s * BCTC_MAX_IN * kTileM;
-        tc::mbar_arrive_tx(&in_full[s], in_bytes);
+        tc::mbar_arrive_tx(&in_full[s], (uint32_t)P.n_in * kTileM * 8);
         for (int j = 0; j < P.n_in; ++j) tc::bulk_g2s(dst + j * kTileM, in + (size_t)io.in_off[j] * N, kTileM * 8, &in_full[s]);
     };
 
@@ -112,9 +115,9 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         // ------------------------------------------------ producers (+ TMA issue on thread 0)
         if (tid == 0)
             for (int i = 0; i < kInStages - 1; ++i) tma_issue(i);
-        uint8_t* arow0 = sA + (tid >> 3) * 512 + (tid & 7) * 16;   // row tid of stage 0
+        uint8_t* arow0 = sA + (tid >> 3) * 512 + (tid & 7) * 16;   // row tid of A-stage 0
         int i = 0;
-        for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
+        for (int tile = blockIdx.x; tile < total_run; tile += G, ++i) {
             if (tid == 0) tma_issue(i + kInStages - 1);
             int jb, b, m0;
             decode(tile, jb, b, m0);
@@ -141,95 +144,104 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                     if (sh > 24) w[wi + 2] |= (uint32_t)(y >> (64 - sh));
                 }
             }
-            const int s = i % kStages, k = i / kStages;
+            const int s = i % kAStages, k = i / kAStages;
             tc::mbar_wait(&empty_a[s], (k & 1) ^ 1);
             uint8_t* arow = arow0 + s * (kTileM * 64);
+            if (!(exp & 64)) {
 #pragma unroll
-            for (int cc = 0; cc < 4; ++cc)
-                *reinterpret_cast<uint4*>(arow + cc * 128) =
-                    make_uint4(w[4 * cc], w[4 * cc + 1], w[4 * cc + 2], w[4 * cc + 3]);
-            tc::fence_proxy_async();
+                for (int cc = 0; cc < 4; ++cc)
+                    *reinterpret_cast<uint4*>(arow + cc * 128) =
+                        make_uint4(w[4 * cc], w[4 * cc + 1], w[4 * cc + 2], w[4 * cc + 3]);
+                tc::fence_proxy_async();
+            }
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&full_a[s]);
         }
     } else if (warp < 4 + kEpiWarps) {
-        // ------------------------------------------------ epilogue
-        const int ew = warp - 4, quarter = ew & 3, part = ew >> 2;
+        // ------------------------------------------------ epilogue: set e owns TMEM slot e
+        const int ew = warp - 4, quarter = ew & 3, e = ew >> 2;
         const int et = quarter * 32 + lane;                  // TMEM lane = A row = coefficient
-        int i = 0;
-        for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
-            const int s = i % kStages, k = i / kStages;
+        const uint32_t trow = tmem + (uint32_t)(e * kSlotCols) + ((uint32_t)(quarter * 32) << 16);
+        int q = 0;                                           // job counter of this CTA
+        for (int tile = blockIdx.x; tile < total_run; tile += G) {
             int jb, b, m0;
             decode(tile, jb, b, m0);
             const BConvTC& P = PJ[jb];
-            const BConvIO& io = IOJ[jb];
-            const int m = m0 + et;
-            tc::mbar_wait(&tfull[s], k & 1);
-            tc::fence_after();
-            const uint32_t trow = tmem + (uint32_t)(s * kAccCols) + ((uint32_t)(quarter * 32) << 16);
-            u64* outb = io.out + b * io.out_bstride + m;
-            for (int g = 8 * part; g < P.n_out; g += 8 * kEpiParts) {
-                uint32_t v[40];
-                if (exp & 8) {
+            for (int h = 0; h < P.nhalf; ++h, ++q) {
+                if ((q % kSlots) != e) continue;
+                const int k = q / kSlots;
+                const BConvIO& io = IOJ[jb];
+                const int t0 = h * P.J, t1 = min(t0 + P.J, P.n_out);
+                tc::mbar_wait(&tfull[e], k & 1);
+                tc::fence_after();
+                u64* outb = io.out + b * io.out_bstride + m0 + et;
+                for (int g = t0; g < t1; g += 8) {
+                    uint32_t v[40];
+                    if (exp & 8) {
 #pragma unroll
-                    for (int q5 = 0; q5 < 40; ++q5) v[q5] = q5 + g;
-                } else {
+                        for (int x = 0; x < 40; ++x) v[x] = x + g;
+                    } else {
 #pragma unroll
-                    for (int q5 = 0; q5 < 5; ++q5) {
-                        uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * q5]);
-                        tc::tmem_ld8(trow + (uint32_t)(5 * g + 8 * q5), vv);
+                        for (int x = 0; x < 5; ++x) {
+                            uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * x]);
+                            tc::tmem_ld8(trow + (uint32_t)(5 * (g - t0) + 8 * x), vv);
+                        }
+                        tc::tmem_wait_ld();
                     }
-                    tc::tmem_wait_ld();
-                }
 #pragma unroll
-                for (int u = 0; u < 8; ++u) {
-                    const int t = g + u;
-                    if (t < P.n_out && (exp & 1)) {
-                        if (!(exp & 4) || v[5 * u] == 0x12345u) outb[(size_t)io.out_off[t] * N] = v[5 * u] + v[5 * u + 4];
-                    } else if (t < P.n_out) {
-                        const uint32_t* D = &v[5 * u];
-                        const u64 lo = (u64)D[0] + ((u64)D[1] << 8) + ((u64)D[2] << 16);     // < 2^39
-                        const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
-                        const double tq = P.t[t];
-                        const double r = __dadd_rn(u2d(lo), mulc(u2d(hi), P.c24[t], tq));   // == V (mod t)
-                        outb[(size_t)io.out_off[t] * N] = d2u(canon(r, tq, P.tinv[t]));
+                    for (int u = 0; u < 8; ++u) {
+                        const int t = g + u;
+                        if (t < t1 && (exp & 1)) {
+                            if (!(exp & 4) || v[5 * u] == 0x12345u) outb[(size_t)io.out_off[t] * N] = v[5 * u] + v[5 * u + 4];
+                        } else if (t < t1) {
+                            const uint32_t* D = &v[5 * u];
+                            const u64 lo = (u64)D[0] + ((u64)D[1] << 8) + ((u64)D[2] << 16);     // < 2^39
+                            const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
+                            const double tq = P.t[t];
+                            const double r = __dadd_rn(u2d(lo), mulc(u2d(hi), P.c24[t], tq));   // == V (mod t)
+                            outb[(size_t)io.out_off[t] * N] = d2u(canon(r, tq, P.tinv[t]));
+                        }
                     }
                 }
+                tc::fence_before();
+                __syncwarp();
+                if (lane == 0) tc::mbar_arrive(&tempty[e]);
             }
-            tc::fence_before();
-            __syncwarp();
-            if (lane == 0) tc::mbar_arrive(&tempty[s]);
         }
     } else {
         // ------------------------------------------------ MMA issuer
         if (lane == 0) {
             const uint32_t aaddr = tc::smem_u32(sA);
-            int i = 0;
-            for (int tile = blockIdx.x; tile < total_tiles; tile += G, ++i) {
-                const int s = i % kStages, k = i / kStages;
+            int i = 0, q = 0;
+            for (int tile = blockIdx.x; tile < total_run; tile += G, ++i) {
+                const int s = i % kAStages, k = i / kAStages;
                 int jb, b, m0;
                 decode(tile, jb, b, m0);
-                const uint32_t idesc = tc::idesc_u8(kTileM, PJ[jb].ncols);
-                const uint32_t baddr = tc::smem_u32(sB0 + jb * 256 * 64);
-                tc::mbar_wait(&full_a[s], k & 1);
-                tc::mbar_wait(&tempty[s], (k & 1) ^ 1);
-                tc::fence_after();
-                const uint32_t acc = tmem + (uint32_t)(s * kAccCols);
+                const BConvTC& P = PJ[jb];
+                const uint32_t idesc = tc::idesc_u8(kTileM, P.ncols);
                 const uint32_t as = aaddr + s * (kTileM * 64);
-                // K = 64 as two K = 32 steps (LBO = 128 B between K chunks, SBO = 512 B between row groups)
-                if (!(exp & 16)) {
-                    tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(baddr, 128, 512), idesc, 0);
-                    tc::mma_u8(acc, tc::sdesc(as + 256, 128, 512), tc::sdesc(baddr + 256, 128, 512), idesc, 1);
+                tc::mbar_wait(&full_a[s], k & 1);
+                for (int h = 0; h < P.nhalf; ++h, ++q) {
+                    const int slot = q % kSlots, kq = q / kSlots;
+                    tc::mbar_wait(&tempty[slot], (kq & 1) ^ 1);
+                    tc::fence_after();
+                    const uint32_t acc = tmem + (uint32_t)(slot * kSlotCols);
+                    const uint32_t bs = tc::smem_u32(sB0 + jb * kBBytes + h * (kSlotCols * 64));
+                    if (!(exp & 16)) {
+                        // K = 64 as two K = 32 steps (LBO = 128 B between K chunks, SBO = 512 B between row groups)
+                        tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(bs, 128, 512), idesc, 0);
+                        tc::mma_u8(acc, tc::sdesc(as + 256, 128, 512), tc::sdesc(bs + 256, 128, 512), idesc, 1);
+                    }
+                    tc::commit(&tfull[slot]);
                 }
                 tc::commit(&empty_a[s]);
-                tc::commit(&tfull[s]);
             }
         }
         __syncwarp();
     }
     tc::fence_before();
     __syncthreads();
-    if (warp == 0) tc::tmem_dealloc(tmem, kStages * kAccCols);
+    if (warp == 0) tc::tmem_dealloc(tmem, kSlots * kSlotCols);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)

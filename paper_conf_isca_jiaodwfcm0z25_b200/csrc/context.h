@@ -36,10 +36,12 @@ struct BConvIO {
 };
 
 constexpr int BCTC_MAX_IN = 12;     // K = 5 * n_in <= 64
-constexpr int BCTC_MAX_OUT = 51;    // N = 5 * n_out <= 256
+constexpr int BCTC_MAX_OUT = 50;    // two half-tile jobs of <= 25 targets (N = 5 J <= 128)
 
 struct BConvTC {
-    int n_in, n_out, ncols;         // ncols = MMA N = round_up(5 n_out, 16)
+    int n_in, n_out;
+    int nhalf, J;                   // targets split in nhalf jobs of J (last may be shorter)
+    int ncols;                      // MMA N per job = round_up(5 J, 16) <= 128
     double qin[BCTC_MAX_IN], qinv_in[BCTC_MAX_IN];
     TWD qhat_inv[BCTC_MAX_IN];      // [qhat_i^-1]_{q_i}
     double t[BCTC_MAX_OUT], tinv[BCTC_MAX_OUT];
@@ -47,7 +49,7 @@ struct BConvTC {
 };
 
 struct BMatParam {                   // B passed by value (generic neo_bconv, no device tables)
-    uint4 d[256 * 64 / 16];
+    uint4 d[2 * 128 * 64 / 16];      // two half-matrices of 128 rows x 64 B
 };
 
 }  // namespace neo

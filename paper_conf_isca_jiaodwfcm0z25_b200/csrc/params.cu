@@ -170,8 +170,10 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
     std::memset(&P, 0, sizeof(P));
     P.n_in = (int)src.size();
     P.n_out = (int)dst.size();
-    P.ncols = ((5 * P.n_out + 15) / 16) * 16;
-    bmat.assign((size_t)P.ncols * 64, 0);
+    P.nhalf = (5 * P.n_out > 128) ? 2 : 1;
+    P.J = (P.n_out + P.nhalf - 1) / P.nhalf;
+    P.ncols = ((5 * P.J + 15) / 16) * 16;
+    bmat.assign((size_t)P.nhalf * 128 * 64, 0);      // each half padded to 128 rows
     for (int i = 0; i < P.n_in; ++i) {
         u64 qi = src[i], qh = 1;
         for (int k = 0; k < P.n_in; ++k)
@@ -192,8 +194,8 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
             for (int a = 0; a < 5; ++a) {
                 u64 v = mulm(f, (1ull << (8 * a)) % m, m);      // (2^(8a) qhat_i) mod t
                 for (int b = 0; b < 5; ++b) {
-                    int n = 5 * t + b, k = 5 * i + a;
-                    size_t off = (size_t)(n / 8) * 512 + (k / 16) * 128 + (n % 8) * 16 + (k % 16);
+                    const int h = t / P.J, n = 5 * (t - h * P.J) + b, k = 5 * i + a;
+                    size_t off = (size_t)h * 128 * 64 + (size_t)(n / 8) * 512 + (k / 16) * 128 + (n % 8) * 16 + (k % 16);
                     bmat[off] = (uint8_t)((v >> (8 * b)) & 0xFF);
                 }
             }
