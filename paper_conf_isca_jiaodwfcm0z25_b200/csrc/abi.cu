@@ -71,14 +71,23 @@ struct ProfScope {
 
 // ------------------------------------------------------------------ NTT over a row set
 // rows k < n of batch entry b: src + b*src_bs + src_off[k]*N  ->  dst + b*dst_bs + dst_off[k]*N
+// in_lazy: (forward) src holds lazy doubles from the tensor-core BConv; scale: (inverse) per-row
+// constant folded into the column pass (Algorithm 2 line 1's [c qhat^-1] fused into the INTT).
 static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long src_bs, const int* src_off,
                            u64* dst, long long dst_bs, const int* dst_off, const int* prime, int n, u64* tmp,
-                           int batch, cudaStream_t st, const RowEpi* epi = nullptr) {
+                           int batch, cudaStream_t st, const RowEpi* epi = nullptr, bool in_lazy = false,
+                           const TWD* scale = nullptr) {
     if (n <= 0) return NEO_OK;
     if (n > NEO_MAX_ROWS) FAIL(NEO_EUNSUPPORTED, "too many limb rows in one transform");
     RowSet a, b;
     const long long N = c->N;
     a.n = b.n = n;
+    a.in_lazy = fwd && in_lazy;
+    a.has_scale = 0;
+    b.in_lazy = 0;
+    b.has_scale = (!fwd && scale) ? 1 : 0;
+    if (b.has_scale)
+        for (int k = 0; k < n; ++k) b.scale[k] = scale[k];
     // first pass: src -> tmp ; second pass: tmp -> dst
     a.src = src; a.src_bstride = src_bs;
     a.dst = tmp; a.dst_bstride = (long long)n * N;
@@ -131,14 +140,25 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
     int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
     neo_status s;
 
-    // a3: INTT of d (l+1 limbs) -> y (coefficient form)
+    // a3: INTT of d (l+1 limbs) -> y (coefficient form); on the tensor-core path the ModUp
+    // scaling y_i = [c_i qhat_i^-1]_{q_i} (Algorithm 2 line 1) is folded into the INTT
     for (int i = 0; i < Lq; ++i) { so[i] = i; dof[i] = i; pr[i] = i; }
-    if ((s = ntt_rows(c, false, d, d_bs, so, y, (long long)Lq * N, dof, pr, Lq, tmp, B, st))) return s;
+    {
+        TWD sc[NEO_MAX_ROWS];
+        if (c->use_tc)
+            for (int j = 0; j < beta; ++j)
+                for (size_t u = 0; u < c->digits[l][j].size(); ++u) sc[c->digits[l][j][u]] = c->modup_tc[l][j].qhat_inv[u];
+        if ((s = ntt_rows(c, false, d, d_bs, so, y, (long long)Lq * N, dof, pr, Lq, tmp, B, st, nullptr, false,
+                          c->use_tc ? sc : nullptr)))
+            return s;
+    }
 
     // a4: ModUp BConv of all beta digits: y[D_j] -> up[j][targets]  (one launch on tensor cores)
     {
         BConvMulti M;
         M.njobs = 0;
+        M.pre_scaled = 1;
+        M.lazy_out = 1;
         for (int j = 0; j < beta; ++j) {
             const BConvTab& T = c->modup[l][j];
             const std::vector<int>& dj = c->digits[l][j];
@@ -180,7 +200,8 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
             ++n;
         }
     }
-    if ((s = ntt_rows(c, true, up, (long long)beta * E * N, so, up, (long long)beta * E * N, dof, pr, n, tmp, B, st)))
+    if ((s = ntt_rows(c, true, up, (long long)beta * E * N, so, up, (long long)beta * E * N, dof, pr, n, tmp, B, st,
+                      nullptr, c->use_tc)))
         return s;
 
     // a6: KeyIP over all E limbs of PQ_l
@@ -205,9 +226,10 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
         LAUNCH(PK_KEYIP, st, launch_keyip(A, E, B, st));
     }
 
-    // a7: INTT of the P part of acc_0, acc_1 -> pc [2B][P][N]
+    // a7: INTT of the P part of acc_0, acc_1 -> pc [2B][P][N], with ModDown's [a_k Phat_k^-1] folded in
     for (int k2 = 0; k2 < P; ++k2) { so[k2] = Lq + k2; dof[k2] = k2; pr[k2] = c->num_q + k2; }
-    if ((s = ntt_rows(c, false, acc, (long long)E * N, so, pc, (long long)P * N, dof, pr, P, tmp, 2 * B, st)))
+    if ((s = ntt_rows(c, false, acc, (long long)E * N, so, pc, (long long)P * N, dof, pr, P, tmp, 2 * B, st, nullptr,
+                      false, c->use_tc ? c->moddown_tc[l].qhat_inv : nullptr)))
         return s;
 
     // a8: ModDown BConv P -> q_0..q_l, batch 2B
@@ -222,6 +244,8 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
         if (c->use_tc) {
             BConvMulti M;
             M.njobs = 1;
+            M.pre_scaled = 1;
+            M.lazy_out = 1;
             M.P[0] = c->moddown_tc[l];
             M.io[0] = io;
             M.bmat[0] = c->d_bmat + c->moddown_boff[l];
@@ -242,7 +266,7 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
         ep.out0 = out0; ep.out1 = out1; ep.out_b = out_bs;
         for (int i = 0; i < Lq; ++i) ep.pinv[i] = c->pinv[i];
         if ((s = ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st,
-                          &ep)))
+                          &ep, c->use_tc)))
             return s;
     }
     return NEO_OK;

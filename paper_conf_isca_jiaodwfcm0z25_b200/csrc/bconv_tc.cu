@@ -50,7 +50,7 @@ static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocati
 // Ring depths 8 (input) / 4 (A) / 4 (TMEM) absorb the mbarrier and TMA round trips.
 template <class LoadB>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
-                                              int tiles_per_entry, int batch, int exp) {
+                                              int tiles_per_entry, int batch, int exp, int pre_scaled, int lazy_out) {
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t* sA = smem;                                  // kAStages x (128 rows x 64 B)
     uint8_t* sB0 = smem + kAStages * kTileM * 64;        // kMaxJobs x 2 halves x (128 rows x 64 B)
@@ -137,7 +137,8 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             for (int j = 0; j < BCTC_MAX_IN; ++j) {
                 if (j < P.n_in) {
                     const double q = P.qin[j];
-                    const u64 y = (exp & 2) ? c[j] : d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
+                    const u64 y = (pre_scaled || (exp & 2)) ? c[j]
+                                                             : d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
                     const int bit = 40 * j, wi = bit >> 5, sh = bit & 31;
                     w[wi] |= (uint32_t)(y << sh);
                     w[wi + 1] |= (uint32_t)(y >> (32 - sh));
@@ -199,7 +200,8 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                             const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
                             const double tq = P.t[t];
                             const double r = __dadd_rn(u2d(lo), mulc(u2d(hi), P.c24[t], tq));   // == V (mod t)
-                            outb[(size_t)io.out_off[t] * N] = d2u(canon(r, tq, P.tinv[t]));
+                            outb[(size_t)io.out_off[t] * N] = lazy_out ? (u64)__double_as_longlong(r)
+                                                                       : d2u(canon(r, tq, P.tinv[t]));
                         }
                     }
                 }
@@ -247,13 +249,13 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
 __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_g(const __grid_constant__ BConvMulti M, int N, int tiles_per_entry, int batch, int exp) {
     bconv_tc_body(M.P, M.io, M.njobs, [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; }, N,
-                  tiles_per_entry, batch, exp);
+                  tiles_per_entry, batch, exp, M.pre_scaled, M.lazy_out);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_p(const __grid_constant__ BConvTC P, const __grid_constant__ BConvIO io,
              const __grid_constant__ BMatParam B, int N, int tiles_per_entry, int batch) {
-    bconv_tc_body(&P, &io, 1, [&](int, int e) { return B.d[e]; }, N, tiles_per_entry, batch, 0);
+    bconv_tc_body(&P, &io, 1, [&](int, int e) { return B.d[e]; }, N, tiles_per_entry, batch, 0, 0, 0);
 }
 
 size_t bconv_tc_smem(int) { return kSmemAlloc; }

@@ -18,6 +18,8 @@ size_t bconv_tc_smem(int ncols);
 // beta ModUp digits); B matrices from device memory.
 struct BConvMulti {
     int njobs;
+    int pre_scaled;      // inputs already hold y_i = [c_i qhat_i^-1]_{q_i} (scale folded into the INTT)
+    int lazy_out;        // write lazy doubles |x| < 2^40 for the next NTT instead of canonical u64
     BConvTC P[4];
     BConvIO io[4];
     const uint8_t* bmat[4];

@@ -106,9 +106,12 @@ struct RowSet {
     u64* dst;
     long long src_bstride, dst_bstride;   // elements between batch entries
     int n;                                 // rows per batch entry
+    int in_lazy;                           // forward column pass: src holds lazy doubles |x| < 2^40
+    int has_scale;                         // inverse column pass: multiply row k by scale[k]
     int src_off[NEO_MAX_ROWS];
     int dst_off[NEO_MAX_ROWS];
     short prime[NEO_MAX_ROWS];
+    TWD scale[NEO_MAX_ROWS];               // (w, w/q) per row
 };
 
 template <int R>

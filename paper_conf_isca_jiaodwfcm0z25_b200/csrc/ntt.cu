@@ -193,9 +193,14 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
         u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * a.N;
         double x[R];
         if (FWD) {
-            const u64* d64 = reinterpret_cast<const u64*>(sD);
+            if (rs.in_lazy) {                              // lazy doubles (BConv outputs), |x| < 2^40
 #pragma unroll
-            for (int na = 0; na < R; ++na) x[na] = u2d(d64[(R * na + r) * C + c]);
+                for (int na = 0; na < R; ++na) x[na] = sD[(R * na + r) * C + c];
+            } else {
+                const u64* d64 = reinterpret_cast<const u64*>(sD);
+#pragma unroll
+                for (int na = 0; na < R; ++na) x[na] = u2d(d64[(R * na + r) * C + c]);
+            }
             neg_fwd<R>(x, NEG, q);
             __syncthreads();                               // tile consumed: exchange in place
 #pragma unroll
@@ -210,7 +215,12 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
             for (int ib = 0; ib < R; ++ib)
                 dd[(size_t)(r + R * ib) * N2 + n2] = mulc(mulc(x[BitRev<R>::of(ib)], ta, q), sB[ib * C + c], q);
         } else {
-            const TWD ta = sA[r * C + c];
+            TWD ta = sA[r * C + c];
+            if (rs.has_scale) {                            // fold a per-row constant (e.g. qhat^-1) into the twist
+                double w = mulc(ta.w, rs.scale[k], q);
+                w = w < 0.0 ? __dadd_rn(w, q) : w;
+                ta = TWD{w, __dmul_rn(w, mq.qinv)};
+            }
 #pragma unroll
             for (int ib = 0; ib < R; ++ib) x[ib] = mulc(mulc(sD[(r + R * ib) * C + c], ta, q), sB[ib * C + c], q);
             cyc_dif<R>(x, CYC, q);
