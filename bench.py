@@ -137,25 +137,33 @@ class ClockSampler:
 # ----------------------------------------------------------------------------- byte model
 
 def bytes_model(batch: int, l: int = LEVEL) -> dict:
-    """Algorithmic HBM bytes per step, per kernel kind (SURVEY §8(d) per-limb figures x the
-    limbs each launch processes; limb = N words of 8 bytes)."""
+    """Algorithmic HBM bytes per step, per kernel kind: every limb a launch must read or write
+    once (limb = N words of 8 bytes; SURVEY §8(d) per-limb figures x the limbs each launch
+    processes).  Per KS with Lq = l+1 Q limbs, P special limbs, E = Lq + P:
+      INTT(d): col 2*Lq, row 2*Lq;  ModUp NTT: col 2*(beta*E - Lq), row 2*(beta*E - Lq);
+      INTT(acc_P): col 4P, row 4P;  NTT(conv) + fused ModDown tail: col 4*Lq,
+      row 2*Lq (intermediate) + 2*Lq (acc) + add limbs + 2*Lq (out);
+      BConv: ModUp Lq + (beta*E - Lq), ModDown 2P + 2*Lq;  KeyIP: beta*E + 2E per ciphertext,
+      2*beta*E key limbs once per launch.
+    Rescale: INTT of 2 limbs (col 4, row 4), NTT of 2l rows reading 2 unique limbs
+    (col 2 + 2l, row 2l + 2l (c_i) + 2l (out))."""
     limb = (1 << LOG_N) * 8
-    Lq, P, beta, alpha = l + 1, NUM_P, -(-(l + 1) // 12), 12
+    Lq, P = l + 1, NUM_P
+    beta = -(-Lq // 12)
     E = Lq + P
-    ks_ntt = Lq + (beta * E - Lq) + 2 * P + 2 * Lq             # limb transforms per KS
-    resc_ntt = 2 + 2 * l
-    ntt_limbs = batch * (2 * ks_ntt + resc_ntt)                  # per step
-    per_pass = 2 * limb                                          # read + write one limb
-    bconv = batch * 2 * ((beta * alpha + beta * (E - alpha)) + (2 * P + 2 * Lq)) * limb
-    keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E) * limb   # dhat + out per ct, evk once
-    combine = batch * ((2 * Lq * 3 + 2 * Lq) + (2 * Lq * 2 + Lq + 2 * Lq)) * limb
-    tensor = batch * 7 * Lq * limb
-    auto = batch * 4 * Lq * limb
-    modsw = batch * (2 + 2 * l) * limb
-    rcomb = batch * 6 * l * limb
-    return {"ntt_col": ntt_limbs * per_pass, "ntt_row": ntt_limbs * per_pass, "bconv": bconv,
-            "keyip": keyip, "combine": combine, "tensor": tensor, "automorphism": auto,
-            "rescale_modswitch": modsw, "rescale_combine": rcomb}
+    up = beta * E - Lq
+    ks_col = 2 * Lq + 2 * up + 4 * P + 4 * Lq
+    ks_row_base = 2 * Lq + 2 * up + 4 * P + 6 * Lq
+    add_hmult, add_hrot = 2 * Lq, Lq
+    ntt_col = batch * (2 * ks_col + 4 + 2 + 2 * l)
+    ntt_row = batch * (2 * ks_row_base + add_hmult + add_hrot + 4 + 6 * l)
+    bconv = batch * 2 * ((Lq + up) + (2 * P + 2 * Lq))
+    keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E)
+    tensor = batch * 7 * Lq
+    auto = batch * 4 * Lq
+    out = {"ntt_col": ntt_col, "ntt_row": ntt_row, "bconv": bconv, "keyip": keyip, "combine": 0,
+           "tensor": tensor, "automorphism": auto, "rescale_modswitch": 0, "rescale_combine": 0}
+    return {k: v * limb for k, v in out.items()}
 
 
 def load_peaks():
@@ -423,6 +431,11 @@ def run_neo(args):
                              "frac": achieved / peak if achieved else None, "traffic": traffic,
                              "launches_per_step": n_launch_dom,
                              "algo_bytes_per_step": bm[dom]},
+                "step_roofline": {"algo_bytes_per_step": sum(bm.values()),
+                                  "achieved": sum(bm.values()) / (ms_step / 1e3) / 1e9 / world * world,
+                                  "peak": peak, "unit": "GB/s",
+                                  "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
+                                  "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}

@@ -127,7 +127,7 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
 
 static size_t rescale_ws(const neo_ctx* c, int l, int B) {
     const size_t N = c->N;
-    return (size_t)2 * B * N + (size_t)2 * B * l * N + (size_t)2 * B * std::max(l, 1) * N;
+    return (size_t)2 * B * N + (size_t)2 * B * std::max(l, 1) * N;
 }
 
 // ------------------------------------------------------------------ key-switch core
@@ -657,20 +657,28 @@ neo_status neo_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, u
     TRY(check_ws(c, NEO_OP_RESCALE, level, batch, ws, ws_bytes));
     const int N = c->N, l = level, B2 = 2 * batch;
     u64* w = static_cast<u64*>(ws);
-    u64* last = w;
-    u64* r = last + (size_t)B2 * N;
-    u64* tmp = r + (size_t)B2 * l * N;
+    u64* last = w;                          // [2B][N]: INTT of c_l, canonical mod q_l
+    u64* tmp = last + (size_t)B2 * N;       // NTT intermediate
     cudaStream_t s = S(st);
     int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    // 1. coefficient form of the last limb of both components
     so[0] = l; dof[0] = 0; pr[0] = l;
     TRY(ntt_rows(c, false, ct_in, (long long)(l + 1) * N, so, last, N, dof, pr, 1, tmp, B2, s));
-    LAUNCH(PK_MODSW, s, launch_modswitch(last, r, c->d_mods, l, N, B2, s));
-    for (int i = 0; i < l; ++i) { so[i] = dof[i] = i; pr[i] = i; }
-    TRY(ntt_rows(c, true, r, (long long)l * N, so, r, (long long)l * N, dof, pr, l, tmp, B2, s));
-    RescaleArgs A;
-    A.in = ct_in; A.r = r; A.out = ct_out; A.mods = c->d_mods; A.N = N; A.l = l;
-    for (int i = 0; i < l; ++i) A.qlinv[i] = c->ql_inv[l][i];
-    LAUNCH(PK_RESCALE, s, launch_rescale_combine(A, B2, s));
+    // 2. NTT_i of ([c_l]_{q_l} mod q_i) for every i < l: every row reads the same coefficients
+    //    (< q_l < 2^36, a valid lazy representative mod q_i, so no mod-switch pass is needed),
+    //    and the row pass's epilogue writes (c_i - that) * q_l^-1 mod q_i directly (L137, Z10)
+    for (int i = 0; i < l; ++i) { so[i] = 0; dof[i] = i; pr[i] = i; }
+    RowEpi ep;
+    ep.acc = ct_in;
+    ep.acc_b = (long long)2 * (l + 1) * N;
+    ep.acc_c = (long long)(l + 1) * N;
+    ep.add0 = ep.add1 = nullptr;
+    ep.add_b = 0;
+    ep.out0 = ct_out;
+    ep.out1 = ct_out + (size_t)l * N;
+    ep.out_b = (long long)2 * l * N;
+    for (int i = 0; i < l; ++i) ep.pinv[i] = c->ql_inv[l][i];
+    TRY(ntt_rows(c, true, last, N, so, ct_out, (long long)l * N, dof, pr, l, tmp, B2, s, &ep));
     return NEO_OK;
 }
 
