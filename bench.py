@@ -432,7 +432,7 @@ def run_neo(args):
                              "launches_per_step": n_launch_dom,
                              "algo_bytes_per_step": bm[dom]},
                 "step_roofline": {"algo_bytes_per_step": sum(bm.values()),
-                                  "achieved": sum(bm.values()) / (ms_step / 1e3) / 1e9 / world * world,
+                                  "achieved": sum(bm.values()) / (ms_step / 1e3) / 1e9,
                                   "peak": peak, "unit": "GB/s",
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},

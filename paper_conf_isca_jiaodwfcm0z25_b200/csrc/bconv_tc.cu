@@ -93,6 +93,8 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
+    pdl_wait();            // B matrices / TMEM / barriers were set up while the predecessor drained
+    pdl_trigger();
     const uint32_t tmem = tmem_base;
     const int total_run = (exp & 256) ? 0 : total_tiles;      // exp 256: setup/teardown only
 
@@ -275,8 +277,8 @@ cudaError_t launch_bconv_tc(const BConvMulti& M, int N, int batch, int num_sms, 
     const int total = tiles_per_entry * batch * M.njobs;
     const int grid = num_sms < total ? num_sms : total;
     static const int exp = [] { const char* e = std::getenv("NEO_BCONV_EXP"); return e ? std::atoi(e) : 0; }();
-    k_bconv_tc_g<<<grid, kThreads, kSmemAlloc, st>>>(M, N, tiles_per_entry, batch, exp);   // exp != 0: timing experiments only
-    return cudaGetLastError();
+    // exp != 0: timing experiments only (NEO_BCONV_EXP)
+    return launch_k(k_bconv_tc_g, dim3(grid), dim3(kThreads), kSmemAlloc, st, M, N, tiles_per_entry, batch, exp);
 }
 
 cudaError_t launch_bconv_tc_param(const BConvTC& P, const BConvIO& io, const BMatParam& bp, int N, int batch,
@@ -285,8 +287,7 @@ cudaError_t launch_bconv_tc_param(const BConvTC& P, const BConvIO& io, const BMa
     const int tiles_per_entry = N / kTileM;
     const int total = tiles_per_entry * batch;
     const int grid = num_sms < total ? num_sms : total;
-    k_bconv_tc_p<<<grid, kThreads, kSmemAlloc, st>>>(P, io, bp, N, tiles_per_entry, batch);
-    return cudaGetLastError();
+    return launch_k(k_bconv_tc_p, dim3(grid), dim3(kThreads), kSmemAlloc, st, P, io, bp, N, tiles_per_entry, batch);
 }
 
 }  // namespace neo

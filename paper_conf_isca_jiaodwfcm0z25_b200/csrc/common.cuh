@@ -8,6 +8,7 @@
 //      mu = floor(2^98 / q);  qe = umulhi(X >> 34, mu)  in [X/q - 2, X/q]  => r in [0, 3q).
 #pragma once
 #include <cstdint>
+#include <utility>
 #include <cuda_runtime.h>
 
 typedef uint64_t u64;
@@ -93,6 +94,31 @@ NEO_DEV void mac128(u64& hi, u64& lo, u64 a, u64 b) {
     u64 l = a * b, h = __umul64hi(a, b);
     lo += l;
     hi += h + (lo < l);
+}
+
+// ---------------------------------------------------------------------------
+// Programmatic dependent launch (PDL): kernels are launched with programmatic stream
+// serialization so a kernel's launch and constant-table prologue overlap its predecessor's
+// tail; pdl_wait() must precede every access to data another kernel writes or reads.
+NEO_DEV void pdl_wait() { asm volatile("griddepcontrol.wait;\n" ::: "memory"); }
+NEO_DEV void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory"); }
+
+bool neo_pdl_enabled();   // NEO_PDL=1 enables (launch.cu); griddepcontrol.* are no-ops otherwise
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_k(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                            Args&&... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = neo_pdl_enabled() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
 }
 
 // ---------------------------------------------------------------------------

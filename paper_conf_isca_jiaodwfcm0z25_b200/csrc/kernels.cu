@@ -11,6 +11,7 @@ namespace neo {
 // by one Barrett reduction of the < 2^77 total.  (L296-319.)
 __global__ void __launch_bounds__(256)
 k_bconv(BConvTab T, BConvIO io, int N) {
+    pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
     const int b = blockIdx.y;
     if (n >= N) return;
@@ -87,6 +88,7 @@ __device__ __forceinline__ void keyip_body(const KeyIPArgs& A, int n, int t, int
 template <int BETA>
 __global__ void __launch_bounds__(256)
 k_keyip(const __grid_constant__ KeyIPArgs A, int batch) {
+    pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
     const int t = blockIdx.y;
     if (n >= A.N) return;
@@ -97,6 +99,7 @@ k_keyip(const __grid_constant__ KeyIPArgs A, int batch) {
 // out_c[i] = (acc_c[i] - conv_c[i]) * P^-1 mod q_i  (+ add_c[i]); Fig. 5, Z9.
 __global__ void __launch_bounds__(256)
 k_combine(CombineArgs A) {
+    pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
     const int i = blockIdx.y, bc = blockIdx.z, b = bc >> 1, c = bc & 1;
     if (n >= A.N) return;
@@ -115,6 +118,7 @@ k_combine(CombineArgs A) {
 __global__ void __launch_bounds__(256)
 k_tensor(const u64* __restrict__ cta, const u64* __restrict__ ctb, u64* __restrict__ d,
          const ModQ* __restrict__ mods, int limbs, int N) {
+    pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
     const int i = blockIdx.y, b = blockIdx.z;
     if (n >= N) return;
@@ -135,6 +139,7 @@ k_tensor(const u64* __restrict__ cta, const u64* __restrict__ ctb, u64* __restri
 // out[i] = in[(g i + (g-1)/2) mod N]: X -> X^g in the natural-order NTT domain.
 __global__ void __launch_bounds__(256)
 k_automorph(const u64* __restrict__ in, u64* __restrict__ out, unsigned g, int N) {
+    pdl_wait();
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     const size_t row = (size_t)blockIdx.y * N;
     if (i >= N) return;
@@ -146,6 +151,7 @@ k_automorph(const u64* __restrict__ in, u64* __restrict__ out, unsigned g, int N
 // r[bc][i] = last[bc] mod q_i for i < l  (last < q_l < 2 q_i for equal-width primes)
 __global__ void __launch_bounds__(256)
 k_modswitch(const u64* __restrict__ last, u64* __restrict__ r, const ModQ* __restrict__ mods, int l, int N) {
+    pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
     const int i = blockIdx.y, bc = blockIdx.z;
     if (n >= N) return;
@@ -158,6 +164,7 @@ k_modswitch(const u64* __restrict__ last, u64* __restrict__ r, const ModQ* __res
 // out[bc][i] = (in[bc][i] - r[bc][i]) * q_l^-1 mod q_i, in has l+1 limbs, out has l.
 __global__ void __launch_bounds__(256)
 k_rescale_combine(RescaleArgs A) {
+    pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
     const int i = blockIdx.y, bc = blockIdx.z;
     if (n >= A.N) return;
@@ -171,43 +178,36 @@ k_rescale_combine(RescaleArgs A) {
 static inline dim3 g1(int N) { return dim3((N + 255) / 256); }
 
 cudaError_t launch_bconv(const BConvTab& T, const BConvIO& io, int N, int batch, cudaStream_t st) {
-    k_bconv<<<dim3((N + 255) / 256, batch), 256, 0, st>>>(T, io, N);
-    return cudaGetLastError();
+    return launch_k(k_bconv, dim3((N + 255) / 256, batch), dim3(256), 0, st, T, io, N);
 }
 cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t st) {
     const dim3 g((A.N + 255) / 256, limbs);
     switch (A.beta) {
-        case 1: k_keyip<1><<<g, 256, 0, st>>>(A, batch); break;
-        case 2: k_keyip<2><<<g, 256, 0, st>>>(A, batch); break;
-        case 3: k_keyip<3><<<g, 256, 0, st>>>(A, batch); break;
-        case 4: k_keyip<4><<<g, 256, 0, st>>>(A, batch); break;
-        case 5: k_keyip<5><<<g, 256, 0, st>>>(A, batch); break;
-        case 6: k_keyip<6><<<g, 256, 0, st>>>(A, batch); break;
-        case 7: k_keyip<7><<<g, 256, 0, st>>>(A, batch); break;
-        default: k_keyip<8><<<g, 256, 0, st>>>(A, batch); break;
+        case 1: return launch_k(k_keyip<1>, g, dim3(256), 0, st, A, batch);
+        case 2: return launch_k(k_keyip<2>, g, dim3(256), 0, st, A, batch);
+        case 3: return launch_k(k_keyip<3>, g, dim3(256), 0, st, A, batch);
+        case 4: return launch_k(k_keyip<4>, g, dim3(256), 0, st, A, batch);
+        case 5: return launch_k(k_keyip<5>, g, dim3(256), 0, st, A, batch);
+        case 6: return launch_k(k_keyip<6>, g, dim3(256), 0, st, A, batch);
+        case 7: return launch_k(k_keyip<7>, g, dim3(256), 0, st, A, batch);
+        default: return launch_k(k_keyip<8>, g, dim3(256), 0, st, A, batch);
     }
-    return cudaGetLastError();
 }
 cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStream_t st) {
-    k_combine<<<dim3((A.N + 255) / 256, limbs, 2 * batch), 256, 0, st>>>(A);
-    return cudaGetLastError();
+    return launch_k(k_combine, dim3((A.N + 255) / 256, limbs, 2 * batch), dim3(256), 0, st, A);
 }
 cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, int limbs, int N, int batch,
                           cudaStream_t st) {
-    k_tensor<<<dim3(g1(N).x, limbs, batch), 256, 0, st>>>(a, b, d, mods, limbs, N);
-    return cudaGetLastError();
+    return launch_k(k_tensor, dim3(g1(N).x, limbs, batch), dim3(256), 0, st, a, b, d, mods, limbs, N);
 }
 cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st) {
-    k_automorph<<<dim3(g1(N).x, rows), 256, 0, st>>>(in, out, g, N);
-    return cudaGetLastError();
+    return launch_k(k_automorph, dim3(g1(N).x, rows), dim3(256), 0, st, in, out, g, N);
 }
 cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st) {
-    k_modswitch<<<dim3(g1(N).x, l, bc), 256, 0, st>>>(last, r, mods, l, N);
-    return cudaGetLastError();
+    return launch_k(k_modswitch, dim3(g1(N).x, l, bc), dim3(256), 0, st, last, r, mods, l, N);
 }
 cudaError_t launch_rescale_combine(const RescaleArgs& A, int bc, cudaStream_t st) {
-    k_rescale_combine<<<dim3(g1(A.N).x, A.l, bc), 256, 0, st>>>(A);
-    return cudaGetLastError();
+    return launch_k(k_rescale_combine, dim3(g1(A.N).x, A.l, bc), dim3(256), 0, st, A);
 }
 
 }  // namespace neo

@@ -170,6 +170,8 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
 
     const int G = gridDim.x;
     int t = blockIdx.x;
+    pdl_wait();            // predecessor's writes visible (and its reads done) before any access
+    pdl_trigger();         // persistent grid is fully resident: let the next kernel launch now
 #pragma unroll
     for (int s = 0; s < STAGES; ++s) issue(t + s * G, s);
     for (int it = 0; t < tm.total; t += G, ++it) {
@@ -300,6 +302,8 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
 
     const int G = gridDim.x;
     int t = blockIdx.x;
+    pdl_wait();            // predecessor's writes visible (and its reads done) before any access
+    pdl_trigger();         // persistent grid is fully resident: let the next kernel launch now
 #pragma unroll
     for (int s = 0; s < STAGES; ++s) issue(t + s * G, s);
     for (int it = 0; t < tm.total; t += G, ++it) {
@@ -421,13 +425,15 @@ static cudaError_t launch_cfg(bool col, const RowSet& rs, const NttArgs& a, int 
     int grid = MINB * a.num_sms;
     if (grid > tm.total) grid = tm.total;
     if (col) {
-        k_ntt_col<R, FWD, STAGES, MINB><<<grid, ColCfg<R>::NT, smc, st>>>(rs, a, tm);
+        return launch_k(k_ntt_col<R, FWD, STAGES, MINB>, dim3(grid), dim3(ColCfg<R>::NT), smc, st, rs, a, tm);
     } else if (epi) {
         if (!FWD) return cudaErrorInvalidValue;
-        k_ntt_row<R, FWD, STAGES, MINB, true><<<grid, RowCfg<R>::NT, smr, st>>>(rs, a, tm, *epi);
+        return launch_k(k_ntt_row<R, FWD, STAGES, MINB, true>, dim3(grid), dim3(RowCfg<R>::NT), smr, st, rs, a, tm,
+                        *epi);
     } else {
         static const RowEpi none{};
-        k_ntt_row<R, FWD, STAGES, MINB, false><<<grid, RowCfg<R>::NT, smr, st>>>(rs, a, tm, none);
+        return launch_k(k_ntt_row<R, FWD, STAGES, MINB, false>, dim3(grid), dim3(RowCfg<R>::NT), smr, st, rs, a, tm,
+                        none);
     }
     return cudaGetLastError();
 }
