@@ -158,7 +158,7 @@ def bytes_model(batch: int, l: int = LEVEL) -> dict:
     ntt_col = batch * (2 * ks_col + 4 + 2 + 2 * l)
     ntt_row = batch * (2 * ks_row_base + add_hmult + add_hrot + 4 + 6 * l)
     bconv = batch * 2 * ((Lq + up) + (2 * P + 2 * Lq))
-    keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E)
+    keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E * 5 / 8)          # key stored in 5 bytes per residue
     tensor = batch * 7 * Lq
     auto = batch * 4 * Lq
     out = {"ntt_col": ntt_col, "ntt_row": ntt_row, "bconv": bconv, "keyip": keyip, "combine": 0,

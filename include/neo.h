@@ -113,8 +113,9 @@ neo_status neo_automorphism(const neo_ctx* ctx, const uint64_t* in, int32_t n_li
                             uint32_t galois_elt, uint64_t* out, int32_t batch, neo_stream_t stream);
 
 /* Evaluation key (L184; gadget Z8): evk is a DEVICE array [dnum][2][num_q+num_p][N] in NTT
- * form, evk[j][0] = b_j, evk[j][1] = a_j.  The library copies it (it may be freed after
- * return).  Synchronises the current device. */
+ * form, evk[j][0] = b_j, evk[j][1] = a_j.  The library re-lays it out once into 5 bytes per
+ * residue (a 32-bit and an 8-bit plane: 94 MB instead of 151 MB at Set-B), so the caller may
+ * free its copy after return.  Synchronises the current device. */
 neo_status neo_evk_create(const neo_ctx* ctx, const uint64_t* evk, neo_evk** out);
 neo_status neo_evk_destroy(neo_evk* evk);
 

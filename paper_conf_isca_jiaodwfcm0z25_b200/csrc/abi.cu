@@ -207,7 +207,7 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
     // a6: KeyIP over all E limbs of PQ_l
     {
         KeyIPArgs A;
-        A.d = d; A.up = up; A.evk = k->d; A.acc = acc; A.mods = c->d_mods;
+        A.d = d; A.up = up; A.evk_lo = k->lo; A.evk_hi = k->hi; A.acc = acc; A.mods = c->d_mods;
         A.d_bstride = d_bs;
         A.up_bstride = (long long)beta * E * N;
         A.acc_bstride = (long long)2 * E * N;
@@ -517,17 +517,16 @@ neo_status neo_evk_create(const neo_ctx* c, const uint64_t* evk, neo_evk** out) 
     neo_evk* k = new (std::nothrow) neo_evk();
     if (!k) FAIL(NEO_ENOMEM, "host allocation failed");
     k->ctx = c;
-    size_t bytes = (size_t)c->dnum * 2 * (c->num_q + c->num_p) * c->N * sizeof(u64);
-    if (cudaMalloc(&k->d, bytes) != cudaSuccess) {
-        delete k;
+    const size_t n = (size_t)c->dnum * 2 * (c->num_q + c->num_p) * c->N;
+    if (cudaMalloc(&k->lo, n * sizeof(uint32_t)) != cudaSuccess || cudaMalloc(&k->hi, n) != cudaSuccess) {
+        neo_evk_destroy(k);
         FAIL(NEO_ENOMEM, "cudaMalloc of the evaluation key failed");
     }
-    cudaError_t e = cudaMemcpy(k->d, evk, bytes, cudaMemcpyDeviceToDevice);
+    cudaError_t e = launch_pack5(evk, k->lo, k->hi, n, nullptr);   // re-layout once: 5 bytes per residue
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
     if (e != cudaSuccess) {
-        cudaFree(k->d);
-        delete k;
-        FAIL(NEO_ECUDA, std::string("evk copy failed: ") + cudaGetErrorString(e));
+        neo_evk_destroy(k);
+        FAIL(NEO_ECUDA, std::string("evk re-layout failed: ") + cudaGetErrorString(e));
     }
     *out = k;
     return NEO_OK;
@@ -535,7 +534,8 @@ neo_status neo_evk_create(const neo_ctx* c, const uint64_t* evk, neo_evk** out) 
 
 neo_status neo_evk_destroy(neo_evk* k) {
     if (!k) return NEO_OK;
-    if (k->d) cudaFree(k->d);
+    if (k->lo) cudaFree(k->lo);
+    if (k->hi) cudaFree(k->hi);
     delete k;
     return NEO_OK;
 }
@@ -605,7 +605,7 @@ neo_status neo_keyip(const neo_ctx* c, const neo_evk* k, const uint64_t* dhat, c
     if (beta < 1 || beta > c->dnum) FAIL(NEO_EINVAL, "beta must be in [1, dnum]");
     if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
     KeyIPArgs A;
-    A.d = dhat; A.up = dhat; A.evk = k->d; A.acc = acc; A.mods = c->d_mods;
+    A.d = dhat; A.up = dhat; A.evk_lo = k->lo; A.evk_hi = k->hi; A.acc = acc; A.mods = c->d_mods;
     A.d_bstride = A.up_bstride = (long long)beta * n * c->N;
     A.acc_bstride = (long long)2 * n * c->N;
     A.acc_cstride = (long long)n * c->N;

@@ -87,5 +87,8 @@ struct neo_ctx {
 
 struct neo_evk {
     const neo_ctx* ctx;
-    u64* d = nullptr;                     // [dnum][2][num_q+num_p][N]
+    // 36-bit residues stored as 5 bytes (SURVEY §7 planar layout): low 32 bits and the top
+    // byte in two planes, each [dnum][2][num_q+num_p][N]; 94 MB instead of 151 MB at Set-B.
+    uint32_t* lo = nullptr;
+    uint8_t* hi = nullptr;
 };

@@ -61,9 +61,10 @@ __device__ __forceinline__ void keyip_body(const KeyIPArgs& A, int n, int t, int
     long long sb[BETA];
 #pragma unroll
     for (int j = 0; j < BETA; ++j) {
-        const u64* e = A.evk + ((size_t)(2 * j) * A.evk_limbs + A.limb[t]) * A.N + n;
-        e0[j] = e[0];
-        e1[j] = e[(size_t)A.evk_limbs * A.N];
+        const size_t o0 = ((size_t)(2 * j) * A.evk_limbs + A.limb[t]) * A.N + n;
+        const size_t o1 = o0 + (size_t)A.evk_limbs * A.N;
+        e0[j] = (u64)A.evk_lo[o0] | ((u64)A.evk_hi[o0] << 32);
+        e1[j] = (u64)A.evk_lo[o1] | ((u64)A.evk_hi[o1] << 32);
         const bool up = A.src_kind[j][t];
         src[j] = (up ? A.up : A.d) + (size_t)A.src_off[j][t] * A.N + n;
         sb[j] = up ? A.up_bstride : A.d_bstride;
@@ -174,7 +175,22 @@ k_rescale_combine(RescaleArgs A) {
     A.out[((size_t)bc * A.l + i) * A.N + n] = shoup(sub_mod(x, v, q), A.qlinv[i], q);
 }
 
+// ------------------------------------------------------------------ 5-byte key packing
+__global__ void __launch_bounds__(256)
+k_pack5(const u64* __restrict__ in, uint32_t* __restrict__ lo, uint8_t* __restrict__ hi, size_t n) {
+    pdl_wait();
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+        const u64 v = in[i];
+        lo[i] = (uint32_t)v;
+        hi[i] = (uint8_t)(v >> 32);
+    }
+}
+
 // ------------------------------------------------------------------ launchers
+cudaError_t launch_pack5(const u64* in, uint32_t* lo, uint8_t* hi, size_t n, cudaStream_t st) {
+    return launch_k(k_pack5, dim3(4096), dim3(256), 0, st, in, lo, hi, n);
+}
+
 static inline dim3 g1(int N) { return dim3((N + 255) / 256); }
 
 cudaError_t launch_bconv(const BConvTab& T, const BConvIO& io, int N, int batch, cudaStream_t st) {

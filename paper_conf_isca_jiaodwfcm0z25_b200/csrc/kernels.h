@@ -10,7 +10,8 @@ constexpr int KS_MAX_BETA = 8;
 struct KeyIPArgs {
     const u64* d;          // KS input [B][l+1][N] (NTT form)
     const u64* up;         // ModUp outputs after NTT [B][beta][E][N]
-    const u64* evk;        // [dnum][2][evk_limbs][N]
+    const uint32_t* evk_lo;   // [dnum][2][evk_limbs][N] low 32 bits of each key residue
+    const uint8_t* evk_hi;    // [dnum][2][evk_limbs][N] bits 32..39
     u64* acc;              // [B][2][E][N]
     const ModQ* mods;
     long long d_bstride, up_bstride, acc_bstride, acc_cstride;
@@ -51,5 +52,6 @@ cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, 
 cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st);
 cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st);
 cudaError_t launch_rescale_combine(const RescaleArgs& A, int bc, cudaStream_t st);
+cudaError_t launch_pack5(const u64* in, uint32_t* lo, uint8_t* hi, size_t n, cudaStream_t st);
 
 }  // namespace neo
