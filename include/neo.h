@@ -50,7 +50,7 @@ typedef enum {
 } neo_status;
 
 /* Operation codes for neo_workspace_size. */
-enum { NEO_OP_KEYSWITCH = 0, NEO_OP_HMULT = 1, NEO_OP_HROT = 2, NEO_OP_RESCALE = 3 };
+enum { NEO_OP_KEYSWITCH = 0, NEO_OP_HMULT = 1, NEO_OP_HROT = 2, NEO_OP_RESCALE = 3, NEO_OP_HROT_HOISTED = 4 };
 
 /* Parameter description (Table 1, Table 4).
  *  log_n      : log2 N; this build supports 12 and 16 (N = 2^12 tiny config, 2^16 Set-B).
@@ -140,6 +140,20 @@ neo_status neo_hmult(const neo_ctx* ctx, const neo_evk* relin, const uint64_t* c
 neo_status neo_hrot(const neo_ctx* ctx, const neo_evk* rotkey, uint32_t galois_elt,
                     const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
                     size_t ws_bytes, neo_stream_t stream);
+
+/* Hoisted rotations: n_rot rotations of the same ciphertexts share one
+ * ModUp of c1.  For rotation r with Galois element g_r the result is
+ *   sigma_{g_r}( c0 + k0', k1' ),   (k0', k1') = KeySwitch(c1) under sigma_{g_r}^{-1}(rotkey_r),
+ * which decrypts to the slot rotation like neo_hrot (it is a different, equally valid
+ * ciphertext: the automorphism is applied after ModDown instead of before ModUp).
+ * keys[r] must come from neo_evk_create_hoisted (which stores sigma_{g^-1}(evk) once).
+ * ct_in [batch][2][level+1][N]; ct_out [n_rot][batch][2][level+1][N];
+ * ws >= neo_workspace_size(ctx, NEO_OP_HROT_HOISTED, level, batch). */
+neo_status neo_evk_create_hoisted(const neo_ctx* ctx, const uint64_t* evk, uint32_t galois_elt,
+                                  neo_evk** out);
+neo_status neo_hrot_hoisted(const neo_ctx* ctx, const neo_evk* const* keys, int32_t n_rot,
+                            const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch,
+                            void* ws, size_t ws_bytes, neo_stream_t stream);
 
 /* Building blocks of the limb-sharded key-switch (each rank owns a subset of
  * the limbs of PQ_l and calls these on its own limbs between NCCL all-gathers):

@@ -366,6 +366,21 @@ def hrot(prm, ct, g, level, rotkey, mode="fast"):
     return np.stack([add(prm, c0, k0, ids), k1])
 
 
+def hrot_hoisted(prm, ct, gs, level, rotkeys, mode="fast"):
+    """Hoisted HROTATE: for each g, sigma_g(c0 + k0', k1') with
+    (k0', k1') = KeySwitch(c1) under the key sigma_{g^-1}(rotkey_g).  The key-switch input
+    c1 is the same for every g, so an implementation may run its ModUp once."""
+    out = []
+    ids = list(range(level + 1))
+    for g, key in zip(gs, rotkeys):
+        ginv = pow(g, -1, 2 * prm.N)
+        kp = automorphism_ntt(key, ginv)
+        k0, k1 = keyswitch(prm, ct[1], level, kp, mode)
+        pre = np.stack([add(prm, ct[0], k0, ids), k1])
+        out.append(automorphism_ntt(pre, g))
+    return np.stack(out)
+
+
 def rescale(prm, ct, level, mode="fast"):
     """Rescale (L137), floor reading Z10: c'_i = (c_i - ([c_l]_{q_l} mod q_i)) * q_l^-1 mod q_i."""
     ql = prm.moduli[level]

@@ -120,7 +120,7 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
     L.tmp = o; o += B * std::max(std::max(beta * E, 2 * Lq), 2 * P) * N;
     L.extra = o;
     if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
-    if (op == NEO_OP_HROT) o += B * 2 * Lq * N;
+    if (op == NEO_OP_HROT || op == NEO_OP_HROT_HOISTED) o += B * 2 * Lq * N;
     L.total = o;
     return L;
 }
@@ -131,12 +131,11 @@ static size_t rescale_ws(const neo_ctx* c, int l, int B) {
 }
 
 // ------------------------------------------------------------------ key-switch core
-static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
-                          u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
-                          const u64* add0, const u64* add1, long long add_bs, cudaStream_t st) {
-    const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p;
-    u64 *y = ws + Ly.y, *up = ws + Ly.up, *acc = ws + Ly.acc, *conv = ws + Ly.conv, *pc = ws + Ly.pc,
-        *tmp = ws + Ly.tmp;
+// a3-a5: ModUp of d (INTT, BConv of every digit onto PQ_l, NTT) into the workspace.
+static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l, int B, u64* ws, const KsLayout& Ly,
+                           cudaStream_t st) {
+    const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l);
+    u64 *y = ws + Ly.y, *up = ws + Ly.up, *tmp = ws + Ly.tmp;
     int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
     neo_status s;
 
@@ -204,6 +203,18 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
                       nullptr, c->use_tc)))
         return s;
 
+    return NEO_OK;
+}
+
+// a6-a10: KeyIP of the ModUp outputs (and d's own digit limbs) with key k, ModDown, combine.
+static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
+                            u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
+                            const u64* add0, const u64* add1, long long add_bs, cudaStream_t st) {
+    const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p;
+    u64 *up = ws + Ly.up, *acc = ws + Ly.acc, *conv = ws + Ly.conv, *pc = ws + Ly.pc, *tmp = ws + Ly.tmp;
+    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    neo_status s;
+
     // a6: KeyIP over all E limbs of PQ_l
     {
         KeyIPArgs A;
@@ -270,6 +281,14 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
             return s;
     }
     return NEO_OK;
+}
+
+static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
+                          u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
+                          const u64* add0, const u64* add1, long long add_bs, cudaStream_t st) {
+    neo_status s = ks_modup(c, d, d_bs, l, B, ws, Ly, st);
+    if (s) return s;
+    return ks_finish(c, k, d, d_bs, l, B, ws, Ly, out0, out1, out_bs, add0, add1, add_bs, st);
 }
 
 // ------------------------------------------------------------------ validation helpers
@@ -383,7 +402,8 @@ size_t neo_workspace_size(const neo_ctx* c, int32_t op, int32_t level, int32_t b
     switch (op) {
         case NEO_OP_KEYSWITCH:
         case NEO_OP_HMULT:
-        case NEO_OP_HROT: return ks_layout(c, level, batch, op).total * sizeof(u64);
+        case NEO_OP_HROT:
+        case NEO_OP_HROT_HOISTED: return ks_layout(c, level, batch, op).total * sizeof(u64);
         case NEO_OP_RESCALE: return level >= 1 ? rescale_ws(c, level, batch) * sizeof(u64) : 0;
         default: return 0;
     }
@@ -510,26 +530,48 @@ neo_status neo_automorphism(const neo_ctx* c, const uint64_t* in, int32_t n_limb
     return NEO_OK;
 }
 
-neo_status neo_evk_create(const neo_ctx* c, const uint64_t* evk, neo_evk** out) {
+static neo_status evk_create(const neo_ctx* c, const uint64_t* evk, uint32_t galois, neo_evk** out) {
     TRY(check_ctx(c));
     if (!evk || !out) FAIL(NEO_EINVAL, "null argument");
     *out = nullptr;
     neo_evk* k = new (std::nothrow) neo_evk();
     if (!k) FAIL(NEO_ENOMEM, "host allocation failed");
     k->ctx = c;
+    k->galois = galois;
     const size_t n = (size_t)c->dnum * 2 * (c->num_q + c->num_p) * c->N;
     if (cudaMalloc(&k->lo, n * sizeof(uint32_t)) != cudaSuccess || cudaMalloc(&k->hi, n) != cudaSuccess) {
         neo_evk_destroy(k);
         FAIL(NEO_ENOMEM, "cudaMalloc of the evaluation key failed");
     }
-    cudaError_t e = launch_pack5(evk, k->lo, k->hi, n, nullptr);   // re-layout once: 5 bytes per residue
+    cudaError_t e = cudaSuccess;
+    const u64* src = evk;
+    u64* perm = nullptr;
+    if (galois) {                          // sigma_{g^-1} of every key polynomial (NTT-domain gather)
+        const u64 two_n = 2ull * c->N;
+        u64 ginv = 1, b = galois, ex = c->N - 1;            // g^-1 = g^(N-1) mod 2N (odd g)
+        for (; ex; ex >>= 1, b = b * b % two_n)
+            if (ex & 1) ginv = ginv * b % two_n;
+        e = cudaMalloc(&perm, n * sizeof(u64));
+        if (e == cudaSuccess) e = launch_automorph(evk, perm, (unsigned)ginv, c->N, (int)(n / c->N), nullptr);
+        src = perm;
+    }
+    if (e == cudaSuccess) e = launch_pack5(src, k->lo, k->hi, n, nullptr);   // 5 bytes per residue
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    if (perm) cudaFree(perm);
     if (e != cudaSuccess) {
         neo_evk_destroy(k);
         FAIL(NEO_ECUDA, std::string("evk re-layout failed: ") + cudaGetErrorString(e));
     }
     *out = k;
     return NEO_OK;
+}
+
+neo_status neo_evk_create(const neo_ctx* c, const uint64_t* evk, neo_evk** out) { return evk_create(c, evk, 0, out); }
+
+neo_status neo_evk_create_hoisted(const neo_ctx* c, const uint64_t* evk, uint32_t galois_elt, neo_evk** out) {
+    TRY(check_ctx(c));
+    if ((galois_elt & 1) == 0 || galois_elt >= 2u * (unsigned)c->N) FAIL(NEO_EINVAL, "galois element must be odd and < 2N");
+    return evk_create(c, evk, galois_elt, out);
 }
 
 neo_status neo_evk_destroy(neo_evk* k) {
@@ -592,6 +634,35 @@ neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint6
     cudaStream_t s = S(st);
     LAUNCH(PK_AUTO, s, launch_automorph(ct_in, sc, g, c->N, 2 * (level + 1) * batch, s));
     return ks_core(c, rk, sc + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, sc, nullptr, 2 * ls, s);
+}
+
+neo_status neo_hrot_hoisted(const neo_ctx* c, const neo_evk* const* keys, int32_t n_rot, const uint64_t* ct_in,
+                            int32_t level, uint64_t* ct_out, int32_t batch, void* ws, size_t ws_bytes,
+                            neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(ct_in, "ct_in"));
+    TRY(check_ptr(ct_out, "ct_out"));
+    if (!keys || n_rot < 1) FAIL(NEO_EINVAL, "need n_rot >= 1 hoisted rotation keys");
+    for (int r = 0; r < n_rot; ++r)
+        if (!keys[r] || keys[r]->ctx != c || keys[r]->galois == 0)
+            FAIL(NEO_EINVAL, "keys must come from neo_evk_create_hoisted on this context");
+    TRY(check_ws(c, NEO_OP_HROT_HOISTED, level, batch, ws, ws_bytes));
+    KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HROT_HOISTED);
+    u64* w = static_cast<u64*>(ws);
+    u64* pre = w + Ly.extra;                                  // [B][2][l+1][N] before the automorphism
+    const long long ls = (long long)(level + 1) * c->N;
+    cudaStream_t s = S(st);
+    // one ModUp of c1 for all rotations (hoisting): sigma_g(KS'(c1)) with KS' under sigma_g^-1(key)
+    TRY(ks_modup(c, ct_in + ls, 2 * ls, level, batch, w, Ly, s));
+    for (int r = 0; r < n_rot; ++r) {
+        TRY(ks_finish(c, keys[r], ct_in + ls, 2 * ls, level, batch, w, Ly, pre, pre + ls, 2 * ls, ct_in, nullptr,
+                      2 * ls, s));
+        u64* dst = ct_out + (size_t)r * batch * 2 * ls;
+        LAUNCH(PK_AUTO, s, launch_automorph(pre, dst, keys[r]->galois, c->N, 2 * (level + 1) * batch, s));
+    }
+    return NEO_OK;
 }
 
 neo_status neo_keyip(const neo_ctx* c, const neo_evk* k, const uint64_t* dhat, const int32_t* limb_ids, int32_t n,

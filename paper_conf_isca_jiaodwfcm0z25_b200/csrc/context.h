@@ -91,4 +91,5 @@ struct neo_evk {
     // byte in two planes, each [dnum][2][num_q+num_p][N]; 94 MB instead of 151 MB at Set-B.
     uint32_t* lo = nullptr;
     uint8_t* hi = nullptr;
+    uint32_t galois = 0;                  // hoisted rotation keys: the key is stored as sigma_{g^-1}(evk_g)
 };

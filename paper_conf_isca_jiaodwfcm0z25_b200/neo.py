@@ -16,14 +16,14 @@ import torch
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libneo.so")
 
-NEO_OP_KEYSWITCH, NEO_OP_HMULT, NEO_OP_HROT, NEO_OP_RESCALE = 0, 1, 2, 3
+NEO_OP_KEYSWITCH, NEO_OP_HMULT, NEO_OP_HROT, NEO_OP_RESCALE, NEO_OP_HROT_HOISTED = 0, 1, 2, 3, 4
 _STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM", 4: "NEO_ECUDA",
            5: "NEO_ENCCL", 6: "NEO_ENOPRIME"}
 
 EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_workspace_size",
             "neo_ntt", "neo_intt", "neo_bconv", "neo_tensor", "neo_automorphism", "neo_evk_create",
             "neo_evk_destroy", "neo_keyswitch", "neo_hmult", "neo_hrot", "neo_rescale",
-            "neo_keyip", "neo_moddown_combine",
+            "neo_keyip", "neo_moddown_combine", "neo_evk_create_hoisted", "neo_hrot_hoisted",
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine")
@@ -70,6 +70,8 @@ def lib() -> ctypes.CDLL:
             "neo_hrot": [_vp, _vp, _u32, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_rescale": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_keyip": [_vp, _vp, _vp, _i32p, _i32, _i32, _vp, _i32, _vp],
+            "neo_evk_create_hoisted": [_vp, _vp, _u32, ctypes.POINTER(_vp)],
+            "neo_hrot_hoisted": [_vp, ctypes.POINTER(_vp), _i32, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_moddown_combine": [_vp, _vp, _vp, _i32p, _i32, _vp, _i32, _vp],
         }
         for name, args in sig.items():
@@ -171,12 +173,18 @@ class Context:
 
 
 class EvalKey:
-    """neo_evk_create / neo_evk_destroy (device copy of [dnum][2][num_q+num_p][N])."""
+    """neo_evk_create / neo_evk_destroy (device copy of [dnum][2][num_q+num_p][N]);
+    with hoisted_galois=g, neo_evk_create_hoisted (key for neo_hrot_hoisted)."""
 
-    def __init__(self, ctx: Context, evk: torch.Tensor):
+    def __init__(self, ctx: Context, evk: torch.Tensor, hoisted_galois: int | None = None):
         self.ctx = ctx
         h = ctypes.c_void_p()
-        _check(lib().neo_evk_create(ctx.handle, _ptr(evk), ctypes.byref(h)), "neo_evk_create")
+        if hoisted_galois is None:
+            _check(lib().neo_evk_create(ctx.handle, _ptr(evk), ctypes.byref(h)), "neo_evk_create")
+        else:
+            _check(lib().neo_evk_create_hoisted(ctx.handle, _ptr(evk), hoisted_galois, ctypes.byref(h)),
+                   "neo_evk_create_hoisted")
+        self.galois = hoisted_galois
         self.handle = h
 
     def close(self):
@@ -245,3 +253,9 @@ def neo_keyip(ctx: Context, evk: EvalKey, dhat, limb_ids, beta: int, acc, batch:
 def neo_moddown_combine(ctx: Context, acc, conv, q_ids, out, batch: int, stream=None):
     _check(lib().neo_moddown_combine(ctx.handle, _ptr(acc), _ptr(conv), _ids(q_ids), len(q_ids), _ptr(out), batch,
                                      _stream(stream)), "neo_moddown_combine")
+
+
+def neo_hrot_hoisted(ctx: Context, keys, ct_in, level: int, ct_out, batch: int, ws, stream=None):
+    arr = (ctypes.c_void_p * len(keys))(*[k.handle.value for k in keys])
+    _check(lib().neo_hrot_hoisted(ctx.handle, arr, len(keys), _ptr(ct_in), level, _ptr(ct_out), batch, _ptr(ws),
+                                  ws.numel() * 8, _stream(stream)), "neo_hrot_hoisted")

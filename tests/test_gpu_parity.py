@@ -233,3 +233,20 @@ def test_invalid_arguments_fail_loudly():
         neo.neo_keyswitch(ctx, evk, t, 5, t, t, 1, ws)          # level out of range
     with pytest.raises(neo.NeoError):
         neo.neo_keyswitch(ctx, evk, t[:, :3], 2, t.clone(), t.clone(), 1, ws)   # workspace too small
+
+
+@pytest.mark.parametrize("name,level,batch,rs", [("tiny", 2, 2, (1, 2, 7)), ("setb", 35, 1, (1, 4))])
+def test_hrot_hoisted(name, level, batch, rs):
+    ctx, prm = ctx_of(name)
+    gs = [pow(5, r, 2 * prm.N) for r in rs]
+    keys_np = [rand_evk(prm, 950 + 10 * r) for r in rs]
+    keys = [neo.EvalKey(ctx, dev(k), hoisted_galois=g) for k, g in zip(keys_np, gs)]
+    ct = np.stack([rand_ct(prm, level, 970 + 2 * b) for b in range(batch)])
+    out = torch.empty((len(rs), batch, 2, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+    ws = ctx.workspace(neo.NEO_OP_HROT_HOISTED, level, batch)
+    neo.neo_hrot_hoisted(ctx, keys, dev(ct), level, out, batch, ws)
+    got = host(out)
+    for bb in range(batch):
+        want = ckks.hrot_hoisted(prm, ct[bb], gs, level, keys_np)
+        for r in range(len(rs)):
+            assert np.array_equal(got[r, bb], want[r])

@@ -217,3 +217,15 @@ def test_set_b_keyswitch_exact_rounding_bound():
             want += v * d_coef[k - i] if k >= i else -v * d_coef[k - i + prm.N]
         got = ckks.crt_lift(prm, dec[:, k:k + 1], ids)[0]
         assert abs(_centered(got - want, M)) <= bound
+
+
+def test_hrot_hoisted_rotates_slots(enc_setup):
+    """Hoisted HROTATE (one ModUp, automorphism after ModDown) decodes to the rotations."""
+    prm, delta, s, za, zb, cta, ctb = enc_setup
+    rs = [1, 3]
+    gs = [pow(5, r, 2 * prm.N) for r in rs]
+    keys = [ckks.rot_key(prm, s, g, 600 + r) for g, r in zip(gs, rs)]
+    out = ckks.hrot_hoisted(prm, cta, gs, 2, keys)
+    for r, ct in zip(rs, out):
+        m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, ct, s, 2), [0, 1, 2])
+        assert np.max(np.abs(ckks.decode(prm.N, m, delta) - np.roll(za, -r))) < 1e-6
