@@ -46,6 +46,7 @@ def parse():
     ap.add_argument("--impl", choices=["neo", "reference"], default="neo")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-hoisted", action="store_true")
     ap.add_argument("--streams", type=int, default=2, choices=[1, 2],
                     help="2: HRot runs on a second CUDA stream, overlapping HMult+Rescale")
     ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
@@ -383,6 +384,32 @@ def run_neo(args):
                      "frac_hbm": round(bm[k] / (step_ms[k] / 1e3) / 1e9 / peak, 4) if step_ms[k] > 0 else None}
                  for k in step_ms}
 
+    # secondary: hoisted rotations (one ModUp shared by n_rot rotations of the same ciphertext)
+    hoisted = None
+    if not args.no_hoisted:
+        n_rot = 4
+        hk = []
+        for r in range(n_rot):
+            gr = pow(5, r + 1, 2 * N)
+            hk.append(neo.EvalKey(ctx, torch.from_numpy(rand_evk(ctx.moduli, seed + 300 + 7 * r, N)).cuda(),
+                                  hoisted_galois=gr))
+        hout = torch.empty((n_rot, B, 2, Lq, N), dtype=torch.uint64, device="cuda")
+        hws = ctx.workspace(neo.NEO_OP_HROT_HOISTED, LEVEL, B)
+        for w in range(3):
+            neo.neo_hrot_hoisted(ctx, hk, dev_in[w % SLOTS][2], LEVEL, hout, B, hws)
+        torch.cuda.synchronize()
+        h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        kh = max(3, min(args.steps, 100))
+        h0.record()
+        for k in range(kh):
+            neo.neo_hrot_hoisted(ctx, hk, dev_in[k % SLOTS][2], LEVEL, hout, B, hws)
+        h1.record()
+        torch.cuda.synchronize()
+        hms = h0.elapsed_time(h1) / kh
+        hoisted = {"n_rot": n_rot, "value": n_rot * B * world / (hms / 1e3), "unit": "rotations/s",
+                   "ms_per_call": hms, "note": "neo_hrot_hoisted, one stream, Set-B l=35"}
+        del hk
+
     # end-to-end through the public API with pinned host buffers: every step copies its three
     # input ciphertexts host->device and both results device->host.  Copies run on their own
     # streams, double-buffered, so the H2D of step k+1 and the D2H of step k-1 overlap the
@@ -464,7 +491,7 @@ def run_neo(args):
                                   "peak": peak, "unit": "GB/s",
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
-                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
+                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}
         print(json.dumps(line), flush=True)
