@@ -195,6 +195,14 @@ enum { NEO_PK_NTT_COL = 0, NEO_PK_NTT_ROW, NEO_PK_BCONV, NEO_PK_KEYIP, NEO_PK_CO
 neo_status neo_profile_enable(int32_t on);
 neo_status neo_profile_read(int32_t kind, double* total_ms, int32_t* launches);
 
+/* Diagnostics: when NEO_BCONV_DBG=1 is set in the environment before the first key-switch,
+ * the tensor-core BConv records per-role clock64 stamps of CTA 0 (tiles 0..61: producer
+ * start / A ready, MMA start / committed, epilogue start / end) and globaltimer stamps of the
+ * setup phase (row 63) of the last ModUp and ModDown launch.  neo_debug_bconv_trace
+ * synchronises the device and copies the 2 x 64 x 8 uint64 stamps (ModUp, then ModDown) to
+ * `host` (caller-owned, 8 KB).  Returns 1 if tracing is on, 0 if it is off (host untouched). */
+int32_t neo_debug_bconv_trace(unsigned long long* host);
+
 #ifdef __cplusplus
 }
 #endif

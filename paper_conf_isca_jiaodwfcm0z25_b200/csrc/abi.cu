@@ -1,6 +1,7 @@
 // abi.cpp -- the extern "C" entry points of libneo.so (include/neo.h) and the key-switch
 // orchestrator (Fig. 5: INTT -> ModUp -> NTT -> KeyIP -> INTT -> ModDown -> NTT).
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -33,6 +34,18 @@ static thread_local int g_launches = 0;
     } while (0)
 
 static inline cudaStream_t S(neo_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
+
+// BConv pipeline trace (debug only, NEO_BCONV_DBG=1): CTA 0's clock64 stamps of the last launch
+static unsigned long long* bconv_dbg() {
+    static unsigned long long* p = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        const char* e = std::getenv("NEO_BCONV_DBG");
+        if (e && e[0] == '1') cudaMalloc(&p, 2 * 64 * 8 * sizeof(unsigned long long));
+    }
+    return p;
+}
 
 // ------------------------------------------------------------------ launch profiling
 // Optional CUDA-event pairs around every launch (neo_profile_enable), read back per
@@ -155,6 +168,7 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
     // a4: ModUp BConv of all beta digits: y[D_j] -> up[j][targets]  (one launch on tensor cores)
     {
         BConvMulti M;
+        M.dbg = bconv_dbg();
         M.njobs = 0;
         M.pre_scaled = 1;
         M.lazy_out = 1;
@@ -254,6 +268,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
         if (c->use_tc) {
             BConvMulti M;
+            M.dbg = bconv_dbg() ? bconv_dbg() + 512 : nullptr;
             M.njobs = 1;
             M.pre_scaled = 1;
             M.lazy_out = 1;
@@ -322,6 +337,15 @@ static neo_status check_ptr(const void* p, const char* what) {
 extern "C" {
 
 const char* neo_last_error(void) { return g_err.c_str(); }
+
+// Debug: copy the BConv pipeline traces (ModUp, ModDown: 2 x 64 x 8 stamps) to host; 0 if tracing is off.
+int32_t neo_debug_bconv_trace(unsigned long long* host) {
+    unsigned long long* p = bconv_dbg();
+    if (!p || !host) return 0;
+    cudaDeviceSynchronize();
+    cudaMemcpy(host, p, 2 * 64 * 8 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+    return 1;
+}
 
 neo_status neo_profile_enable(int32_t on) {
     g_recs.clear();

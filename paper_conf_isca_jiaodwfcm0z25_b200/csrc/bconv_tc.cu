@@ -48,9 +48,16 @@ static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocati
 //   epilogue (4 sets of 4 warps, set e owns TMEM slot e): tcgen05.ld, combine the 5
 //                          byte-planes, reduce mod t, store; arrive tmem_empty[e]
 // Ring depths 8 (input) / 4 (A) / 4 (TMEM) absorb the mbarrier and TMA round trips.
-template <class LoadB>
+template <bool kPre, bool kLazy, class LoadB>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
-                                              int tiles_per_entry, int batch, int exp, int pre_scaled, int lazy_out) {
+                                              int tiles_per_entry, int batch, int exp,
+                                              const CUtensorMap* tmaps = nullptr, const int* use_tmap = nullptr,
+                                              unsigned long long* dbg = nullptr) {
+    // debug trace (CTA 0 only): [i][0] producer after in_full, [1] producer arrive full_a,
+    // [2] MMA after waits, [3] MMA committed, [4] epilogue(set 0/1..) start, [5] epilogue end
+    auto T = [&](int i, int ev) {
+        if (dbg && blockIdx.x == 0 && i < 62) dbg[i * 8 + ev] = clock64();
+    };
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t* sA = smem;                                  // kAStages x (128 rows x 64 B)
     uint8_t* sB0 = smem + kAStages * kTileM * 64;        // kMaxJobs x 2 halves x (128 rows x 64 B)
@@ -69,6 +76,15 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int G = gridDim.x;
+    auto GT = [&](int ev) {      // setup trace (row 63): globaltimer ns of CTA 0 / CTA G-1, thread 0
+        if (dbg && tid == 0 && (blockIdx.x == 0 || blockIdx.x == gridDim.x - 1)) {
+            unsigned long long t;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            dbg[63 * 8 + ev + (blockIdx.x ? 4 : 0)] = t;
+            if (!blockIdx.x) dbg[62 * 8 + ev] = clock64();
+        }
+    };
+    GT(0);
     if (warp == 0) tc::tmem_alloc(&tmem_base, kSlots * kSlotCols);
     if (tid == 0) {
         for (int s = 0; s < kAStages; ++s) {
@@ -93,8 +109,10 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
+    GT(1);
     pdl_wait();            // B matrices / TMEM / barriers were set up while the predecessor drained
     pdl_trigger();
+    GT(2);
     const uint32_t tmem = tmem_base;
     const int total_run = (exp & 256) ? 0 : total_tiles;      // exp 256: setup/teardown only
 
@@ -110,13 +128,20 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         const u64* in = io.in + b * io.in_bstride + m0;
         u64* dst = sIn + (size_t)s * BCTC_MAX_IN * kTileM;
         tc::mbar_arrive_tx(&in_full[s], (uint32_t)P.n_in * kTileM * 8);
-        for (int j = 0; j < P.n_in; ++j) tc::bulk_g2s(dst + j * kTileM, in + (size_t)io.in_off[j] * N, kTileM * 8, &in_full[s]);
+        if (use_tmap && use_tmap[jb])      // one instruction for the [n_in][128] box
+            tc::tensor_g2s_3d(dst, &tmaps[jb], m0, io.in_off[0], b, &in_full[s]);
+        else                               // each 1-D bulk copy costs ~170 issue cycles
+            for (int j = 0; j < P.n_in; ++j)
+                tc::bulk_g2s(dst + j * kTileM, in + (size_t)io.in_off[j] * N, kTileM * 8, &in_full[s]);
     };
 
     if (warp < 4) {
         // ------------------------------------------------ producers (+ TMA issue on thread 0)
         if (tid == 0)
-            for (int i = 0; i < kInStages - 1; ++i) tma_issue(i);
+            for (int i = 0; i < kInStages - 1; ++i) {
+                tma_issue(i);
+                if (dbg && blockIdx.x == 0 && i < 3) dbg[62 * 8 + 4 + i] = clock64();
+            }
         uint8_t* arow0 = sA + (tid >> 3) * 512 + (tid & 7) * 16;   // row tid of A-stage 0
         int i = 0;
         for (int tile = blockIdx.x; tile < total_run; tile += G, ++i) {
@@ -126,6 +151,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             const BConvTC& P = PJ[jb];
             const int si = i % kInStages, ki = i / kInStages;
             if (!(exp & 32)) tc::mbar_wait(&in_full[si], ki & 1);
+            if (tid == 0) T(i, 0);
             const u64* src = sIn + (size_t)si * BCTC_MAX_IN * kTileM + tid;
             u64 c[BCTC_MAX_IN];
 #pragma unroll
@@ -139,8 +165,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             for (int j = 0; j < BCTC_MAX_IN; ++j) {
                 if (j < P.n_in) {
                     const double q = P.qin[j];
-                    const u64 y = (pre_scaled || (exp & 2)) ? c[j]
-                                                             : d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
+                    const u64 y = kPre ? c[j] : d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
                     const int bit = 40 * j, wi = bit >> 5, sh = bit & 31;
                     w[wi] |= (uint32_t)(y << sh);
                     w[wi + 1] |= (uint32_t)(y >> (32 - sh));
@@ -150,15 +175,13 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             const int s = i % kAStages, k = i / kAStages;
             tc::mbar_wait(&empty_a[s], (k & 1) ^ 1);
             uint8_t* arow = arow0 + s * (kTileM * 64);
-            if (!(exp & 64)) {
 #pragma unroll
-                for (int cc = 0; cc < 4; ++cc)
-                    *reinterpret_cast<uint4*>(arow + cc * 128) =
-                        make_uint4(w[4 * cc], w[4 * cc + 1], w[4 * cc + 2], w[4 * cc + 3]);
-                tc::fence_proxy_async();
-            }
+            for (int cc = 0; cc < 4; ++cc)
+                *reinterpret_cast<uint4*>(arow + cc * 128) = make_uint4(w[4 * cc], w[4 * cc + 1], w[4 * cc + 2], w[4 * cc + 3]);
+            tc::fence_proxy_async();
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&full_a[s]);
+            if (tid == 0) T(i, 1);
         }
     } else if (warp < 4 + kEpiWarps) {
         // ------------------------------------------------ epilogue: set e owns TMEM slot e
@@ -176,40 +199,41 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                 const BConvIO& io = IOJ[jb];
                 const int t0 = h * P.J, t1 = min(t0 + P.J, P.n_out);
                 tc::mbar_wait(&tfull[e], k & 1);
+                if (lane == 0 && quarter == 0 && h == 0) T(q / P.nhalf, 4);
                 tc::fence_after();
                 u64* outb = io.out + b * io.out_bstride + m0 + et;
+                // 8 targets per group, branch-free so the 8 FP64 chains interleave; the ragged
+                // last group re-reads its last valid column and predicates the stores.
                 for (int g = t0; g < t1; g += 8) {
                     uint32_t v[40];
-                    if (exp & 8) {
 #pragma unroll
-                        for (int x = 0; x < 40; ++x) v[x] = x + g;
-                    } else {
+                    for (int x = 0; x < 5; ++x) {
+                        uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * x]);
+                        tc::tmem_ld8(trow + (uint32_t)(5 * (g - t0) + 8 * x), vv);
+                    }
+                    tc::tmem_wait_ld();
+                    double r[8];
 #pragma unroll
-                        for (int x = 0; x < 5; ++x) {
-                            uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * x]);
-                            tc::tmem_ld8(trow + (uint32_t)(5 * (g - t0) + 8 * x), vv);
-                        }
-                        tc::tmem_wait_ld();
+                    for (int u = 0; u < 8; ++u) {
+                        const int t = min(g + u, t1 - 1);
+                        const uint32_t* D = &v[5 * u];
+                        const u64 lo = (u64)D[0] + ((u64)D[1] << 8) + ((u64)D[2] << 16);     // < 2^39
+                        const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
+                        const double tq = P.t[t];
+                        r[u] = __dadd_rn(u2d(lo), mulc(u2d(hi), P.c24[t], tq));              // == V (mod t)
+                        if (!kLazy) r[u] = canon(r[u], tq, P.tinv[t]);
                     }
 #pragma unroll
                     for (int u = 0; u < 8; ++u) {
                         const int t = g + u;
-                        if (t < t1 && (exp & 1)) {
-                            if (!(exp & 4) || v[5 * u] == 0x12345u) outb[(size_t)io.out_off[t] * N] = v[5 * u] + v[5 * u + 4];
-                        } else if (t < t1) {
-                            const uint32_t* D = &v[5 * u];
-                            const u64 lo = (u64)D[0] + ((u64)D[1] << 8) + ((u64)D[2] << 16);     // < 2^39
-                            const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
-                            const double tq = P.t[t];
-                            const double r = __dadd_rn(u2d(lo), mulc(u2d(hi), P.c24[t], tq));   // == V (mod t)
-                            outb[(size_t)io.out_off[t] * N] = lazy_out ? (u64)__double_as_longlong(r)
-                                                                       : d2u(canon(r, tq, P.tinv[t]));
-                        }
+                        const u64 val = kLazy ? (u64)__double_as_longlong(r[u]) : d2u(r[u]);
+                        if (t < t1) outb[(size_t)io.out_off[t] * N] = val;
                     }
                 }
                 tc::fence_before();
                 __syncwarp();
                 if (lane == 0) tc::mbar_arrive(&tempty[e]);
+                if (lane == 0 && quarter == 0 && h == P.nhalf - 1) T(q / P.nhalf, 5);
             }
         }
     } else {
@@ -225,13 +249,14 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                 const uint32_t idesc = tc::idesc_u8(kTileM, P.ncols);
                 const uint32_t as = aaddr + s * (kTileM * 64);
                 tc::mbar_wait(&full_a[s], k & 1);
+                T(i, 2);
                 for (int h = 0; h < P.nhalf; ++h, ++q) {
                     const int slot = q % kSlots, kq = q / kSlots;
                     tc::mbar_wait(&tempty[slot], (kq & 1) ^ 1);
                     tc::fence_after();
                     const uint32_t acc = tmem + (uint32_t)(slot * kSlotCols);
                     const uint32_t bs = tc::smem_u32(sB0 + jb * kBBytes + h * (kSlotCols * 64));
-                    if (!(exp & 16)) {
+                    {
                         // K = 64 as two K = 32 steps (LBO = 128 B between K chunks, SBO = 512 B between row groups)
                         tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(bs, 128, 512), idesc, 0);
                         tc::mma_u8(acc, tc::sdesc(as + 256, 128, 512), tc::sdesc(bs + 256, 128, 512), idesc, 1);
@@ -239,6 +264,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                     tc::commit(&tfull[slot]);
                 }
                 tc::commit(&empty_a[s]);
+                T(i, 3);
             }
         }
         __syncwarp();
@@ -246,18 +272,21 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     tc::fence_before();
     __syncthreads();
     if (warp == 0) tc::tmem_dealloc(tmem, kSlots * kSlotCols);
+    GT(3);
 }
 
+template <bool kPre, bool kLazy>
 __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_g(const __grid_constant__ BConvMulti M, int N, int tiles_per_entry, int batch, int exp) {
-    bconv_tc_body(M.P, M.io, M.njobs, [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; }, N,
-                  tiles_per_entry, batch, exp, M.pre_scaled, M.lazy_out);
+    bconv_tc_body<kPre, kLazy>(M.P, M.io, M.njobs,
+                               [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; }, N,
+                               tiles_per_entry, batch, exp, M.tmap, M.use_tmap, M.dbg);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_p(const __grid_constant__ BConvTC P, const __grid_constant__ BConvIO io,
              const __grid_constant__ BMatParam B, int N, int tiles_per_entry, int batch) {
-    bconv_tc_body(&P, &io, 1, [&](int, int e) { return B.d[e]; }, N, tiles_per_entry, batch, 0, 0, 0);
+    bconv_tc_body<false, false>(&P, &io, 1, [&](int, int e) { return B.d[e]; }, N, tiles_per_entry, batch, 0);
 }
 
 size_t bconv_tc_smem(int) { return kSmemAlloc; }
@@ -265,20 +294,63 @@ size_t bconv_tc_smem(int) { return kSmemAlloc; }
 static void bconv_tc_init() {
     static bool init = false;
     if (!init) {
-        cudaFuncSetAttribute(k_bconv_tc_g, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
+        cudaFuncSetAttribute(k_bconv_tc_g<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
+        cudaFuncSetAttribute(k_bconv_tc_g<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
+        cudaFuncSetAttribute(k_bconv_tc_g<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
+        cudaFuncSetAttribute(k_bconv_tc_g<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         cudaFuncSetAttribute(k_bconv_tc_p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         init = true;
     }
 }
 
-cudaError_t launch_bconv_tc(const BConvMulti& M, int N, int batch, int num_sms, cudaStream_t st) {
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda link dependency)
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static EncodeTiledFn encode_tiled() {
+    static EncodeTiledFn fn = [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            p = nullptr;
+        return reinterpret_cast<EncodeTiledFn>(p);
+    }();
+    return fn;
+}
+
+// 3-D map over job j's input: dim0 = coefficient (N), dim1 = limb row, dim2 = batch entry;
+// box = one tile {128, n_in, 1}.  Needs the input rows of the job to be consecutive.
+static bool make_input_tmap(const BConvTC& P, const BConvIO& io, int N, int batch, CUtensorMap* map) {
+    EncodeTiledFn enc = encode_tiled();
+    if (!enc || P.n_in < 1) return false;
+    for (int i = 1; i < P.n_in; ++i)
+        if (io.in_off[i] != io.in_off[0] + i) return false;
+    const long long rows = io.in_off[0] + P.n_in;
+    if (batch > 1 && rows * N > io.in_bstride) return false;
+    if ((reinterpret_cast<uintptr_t>(io.in) & 15) != 0) return false;
+    const cuuint64_t dim[3] = {(cuuint64_t)N, (cuuint64_t)rows, (cuuint64_t)batch};
+    const cuuint64_t stride[2] = {(cuuint64_t)N * 8, (cuuint64_t)(batch > 1 ? io.in_bstride : rows * N) * 8};
+    const cuuint32_t box[3] = {(cuuint32_t)kTileM, (cuuint32_t)P.n_in, 1};
+    const cuuint32_t estr[3] = {1, 1, 1};
+    return enc(map, CU_TENSOR_MAP_DATA_TYPE_UINT64, 3, const_cast<u64*>(io.in), dim, stride, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+cudaError_t launch_bconv_tc(const BConvMulti& M0, int N, int batch, int num_sms, cudaStream_t st) {
     bconv_tc_init();
+    BConvMulti M = M0;
+    static const bool no_tmap = [] { const char* e = std::getenv("NEO_BCONV_TMAP"); return e && e[0] == '0'; }();
+    for (int j = 0; j < 4; ++j) M.use_tmap[j] = (j < M.njobs && !no_tmap) ? make_input_tmap(M.P[j], M.io[j], N, batch, &M.tmap[j]) : 0;
     const int tiles_per_entry = N / kTileM;
     const int total = tiles_per_entry * batch * M.njobs;
     const int grid = num_sms < total ? num_sms : total;
     static const int exp = [] { const char* e = std::getenv("NEO_BCONV_EXP"); return e ? std::atoi(e) : 0; }();
-    // exp != 0: timing experiments only (NEO_BCONV_EXP)
-    return launch_k(k_bconv_tc_g, dim3(grid), dim3(kThreads), kSmemAlloc, st, M, N, tiles_per_entry, batch, exp);
+    // exp != 0: timing experiments only (NEO_BCONV_EXP: 32 no TMA, 256 setup/teardown only)
+    auto k = M.pre_scaled ? (M.lazy_out ? k_bconv_tc_g<true, true> : k_bconv_tc_g<true, false>)
+                          : (M.lazy_out ? k_bconv_tc_g<false, true> : k_bconv_tc_g<false, false>);
+    return launch_k(k, dim3(grid), dim3(kThreads), kSmemAlloc, st, M, N, tiles_per_entry, batch, exp);
 }
 
 cudaError_t launch_bconv_tc_param(const BConvTC& P, const BConvIO& io, const BMatParam& bp, int N, int batch,

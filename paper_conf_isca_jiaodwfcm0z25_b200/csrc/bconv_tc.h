@@ -1,5 +1,7 @@
 // bconv_tc.h -- tensor-core BConv (bconv_tc.cu): constants and launcher.
 #pragma once
+#include <cuda.h>   // CUtensorMap (the type only; the encoder is fetched through the runtime)
+
 #include <vector>
 
 #include "common.cuh"
@@ -17,12 +19,15 @@ size_t bconv_tc_smem(int ncols);
 // Up to 4 conversions with the same input/output batch geometry in one launch (e.g. the
 // beta ModUp digits); B matrices from device memory.
 struct BConvMulti {
+    CUtensorMap tmap[4];     // filled by launch_bconv_tc: 3-D map {N, rows, batch} of job j's input
+    int use_tmap[4];         // 1: one tensor TMA per tile (inputs rows contiguous), 0: per-row bulk copies
     int njobs;
     int pre_scaled;      // inputs already hold y_i = [c_i qhat_i^-1]_{q_i} (scale folded into the INTT)
     int lazy_out;        // write lazy doubles |x| < 2^40 for the next NTT instead of canonical u64
     BConvTC P[4];
     BConvIO io[4];
     const uint8_t* bmat[4];
+    unsigned long long* dbg;   // optional clock64 trace of CTA 0 (NEO_BCONV_DBG): [tile][8]
 };
 cudaError_t launch_bconv_tc(const BConvMulti& M, int N, int batch, int num_sms, cudaStream_t st);
 // One conversion with B passed by value (generic neo_bconv).

@@ -85,8 +85,8 @@ NEO_DEV double mulv(double a, double b, double q, double qinv) {   // a * b mod 
 }
 NEO_DEV double canon(double x, double q, double qinv) {   // |x| < 2^50 integral -> [0, q)
     const double qf = __dadd_rn(__fma_rn(x, qinv, kMagic), -kMagic);
-    const double r = __fma_rn(-qf, q, x);                   // exact, |r| <= q/2 + 1
-    return r < 0.0 ? __dadd_rn(r, q) : (r >= q ? __dadd_rn(r, -q) : r);
+    const double r = __fma_rn(-qf, q, x);                   // exact, |r| <= q/2 + 1 < q
+    return __dadd_rn(r, r < 0.0 ? q : 0.0);                 // branch-free: selects, one DADD
 }
 
 // 128-bit accumulator helpers

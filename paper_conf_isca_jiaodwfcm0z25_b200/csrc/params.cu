@@ -171,7 +171,9 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
     P.n_in = (int)src.size();
     P.n_out = (int)dst.size();
     P.nhalf = (5 * P.n_out > 128) ? 2 : 1;
-    P.J = (P.n_out + P.nhalf - 1) / P.nhalf;
+    // the epilogue drains 8 targets per tcgen05.ld group: a first half of 24 targets has no
+    // ragged group (n_out <= 48; 25 + 25 for the largest bases)
+    P.J = P.nhalf == 1 ? P.n_out : (P.n_out <= 48 ? 24 : 25);
     P.ncols = ((5 * P.J + 15) / 16) * 16;
     bmat.assign((size_t)P.nhalf * 128 * 64, 0);      // each half padded to 128 rows
     for (int i = 0; i < P.n_in; ++i) {

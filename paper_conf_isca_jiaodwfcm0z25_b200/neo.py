@@ -24,7 +24,8 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_ntt", "neo_intt", "neo_bconv", "neo_tensor", "neo_automorphism", "neo_evk_create",
             "neo_evk_destroy", "neo_keyswitch", "neo_hmult", "neo_hrot", "neo_rescale",
             "neo_keyip", "neo_moddown_combine", "neo_evk_create_hoisted", "neo_hrot_hoisted",
-            "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read")
+            "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
+            "neo_debug_bconv_trace")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine")
 
@@ -88,6 +89,8 @@ def lib() -> ctypes.CDLL:
         L.neo_profile_enable.restype = ctypes.c_int
         L.neo_profile_read.argtypes = [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int32)]
         L.neo_profile_read.restype = ctypes.c_int
+        L.neo_debug_bconv_trace.argtypes = [ctypes.POINTER(ctypes.c_ulonglong)]
+        L.neo_debug_bconv_trace.restype = _i32
         _lib = L
     return _lib
 
@@ -131,6 +134,15 @@ def neo_profile_read() -> dict:
         _check(lib().neo_profile_read(k, ctypes.byref(ms), ctypes.byref(n)), "neo_profile_read")
         out[name] = (ms.value, n.value)
     return out
+
+
+def neo_debug_bconv_trace():
+    """The BConv pipeline trace (NEO_BCONV_DBG=1) as a [2][64][8] list (ModUp, ModDown), or None."""
+    buf = (ctypes.c_ulonglong * 1024)()
+    if not lib().neo_debug_bconv_trace(buf):
+        return None
+    v = list(buf)
+    return [[v[w * 512 + r * 8: w * 512 + r * 8 + 8] for r in range(64)] for w in range(2)]
 
 
 class Context:
