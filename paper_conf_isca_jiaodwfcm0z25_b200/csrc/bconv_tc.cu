@@ -10,10 +10,14 @@
 //   out_t[m]     = sum_b 2^(8b) D_b[m, t]  mod t                 (epilogue, FP64)
 //
 // so sum_b 2^(8b) D_b == sum_i y_i (qhat_i mod t) (mod t): Algorithm 1's result exactly.
+// All moduli are < 2^36, so the top bytes y^(4), C_4 are < 16: D_0..3 < 12 * 1035 * 255 < 2^22,
+// D_4 < 12 * 1035 * 15 < 2^18 and V = sum_b 2^(8b) D_b < 2^46.1 + 2^50 < 2^51 is an exact
+// double; the epilogue is one integer sum plus one FP64 Barrett step (4 FP64 ops).
 // GEMM shape per 128-coefficient tile: M = 128, K = 5*n_in <= 64 (two K=32 MMAs), and the
-// targets split into one or two jobs of N = 5*J <= 128 columns.  A (8 KB) is produced by the
-// CUDA cores into shared memory in the SWIZZLE_NONE K-major layout, B (<= 16 KB) is loaded
-// once per CTA, the accumulators live in TMEM (4 x 128 columns) and are drained with tcgen05.ld.
+// targets split into parts of J = 9 (45 columns, padded to 48), all parts of a tile in one
+// MMA of N = 48 * parts <= 240.  A (8 KB) is produced by the CUDA cores into shared memory in
+// the SWIZZLE_NONE K-major layout, B (<= 15 KB) is loaded once per CTA, the accumulators live
+// in TMEM (2 tile slots x 256 columns) and are drained with tcgen05.ld.
 // D_b <= 60 * 255 * 255 < 2^22, so s32 accumulation is exact.
 #include <cstdlib>
 
@@ -25,43 +29,72 @@ namespace neo {
 
 constexpr int kTileM = 128;
 constexpr int kAStages = 4;                        // A-tile ring
-constexpr int kSlots = 4;                          // TMEM accumulator ring (4 x 128 columns)
-constexpr int kSlotCols = 128;                     // per half-tile job: N = 5 * J <= 128
+constexpr int kSlots = 2;                          // TMEM accumulator ring: 2 tile slots x 256 columns
+constexpr int kSlotCols = 256;                     // a tile's parts at 48-column stride
+constexpr int kSets = 4;                           // epilogue sets of 4 warps: set e drains parts q = e (mod 4)
 constexpr int kInStages = 8;                       // TMA input ring (12 KB each)
-constexpr int kEpiWarps = 4 * kSlots;              // one 4-warp set per TMEM slot
-constexpr int kThreads = (4 + kEpiWarps + 1) * 32; // producers, epilogue, MMA
+constexpr int kEpiWarps = 4 * kSets;
+constexpr int kThreads = (4 + kEpiWarps + 2) * 32; // producers, epilogue, MMA, TMA
 constexpr size_t kInBytes = (size_t)BCTC_MAX_IN * kTileM * 8;
 constexpr int kMaxJobs = 4;                        // conversions fused into one launch (ModUp digits)
-constexpr size_t kBBytes = 2 * kSlotCols * 64;     // two half-matrices per conversion
-constexpr size_t kSmemBytes = kAStages * kTileM * 64 + kMaxJobs * kBBytes + kInStages * kInBytes;   // 192 KB
-constexpr size_t kSmemAlloc = 200 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
+constexpr size_t kPartBytes = (size_t)BCTC_PART_ROWS * 64;
+constexpr size_t kBBytes = BCTC_MAX_PARTS * kPartBytes;   // 15 KB per conversion
+struct JobH {                                      // per-conversion header, staged in smem
+    const u64* in;
+    u64* out;
+    long long in_bs, out_bs;
+    int n_in, n_out, nparts, J, ncols, in_off0, use_tmap, pad;
+};
+struct TgtC {                                      // per-target epilogue constants, staged in smem
+    double t, tinv;
+    long long offb;                                // out_off[t] * N * 8 (bytes)
+    long long pad;
+};
+constexpr int kTgtRow = (BCTC_MAX_PARTS * BCTC_PART_J + 7) / 8 * 8;   // padded: parts need no clamp
+constexpr int kMaxSched = 1024;                    // per-CTA tile schedule entries staged in smem
+constexpr size_t kTabBytes = kMaxJobs * (sizeof(JobH) + kTgtRow * sizeof(TgtC)) + kMaxSched * 4;
+constexpr size_t kSmemBytes = kAStages * kTileM * 64 + kMaxJobs * kBBytes + kInStages * kInBytes + kTabBytes;
+constexpr size_t kSmemAlloc = 214 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
 static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocation");
+static_assert(kSlots * kSlotCols == 512, "TMEM plan");
 
-// Warp-specialised pipeline, one persistent CTA per SM.  A tile (128 coefficients) is split
-// into `nhalf` jobs of J targets (N = 5J <= 128 columns) so that four accumulators fit in TMEM:
-//   TMA (warp 0, lane 0): 1-D bulk copies of the n_in input rows of tile i+7 (1 KB each)
-//   producers (warps 0-3): y = [c qhat^-1] of one coefficient, split into bytes, write the A
-//                          row of A-stage i % 4, arrive full_a
-//   MMA (last warp, lane 0): per job q: wait full_a / tmem_empty[q % 4]; two K = 32 MMAs
-//                          into slot q % 4; commit -> tmem_full; after the tile's jobs
-//                          commit -> empty_a
-//   epilogue (4 sets of 4 warps, set e owns TMEM slot e): tcgen05.ld, combine the 5
-//                          byte-planes, reduce mod t, store; arrive tmem_empty[e]
-// Ring depths 8 (input) / 4 (A) / 4 (TMEM) absorb the mbarrier and TMA round trips.
+// Warp-specialised pipeline, one persistent CTA per SM:
+//   TMA (warp 21, lane 0): one 3-D tensor copy of the [n_in][128] input box of tile i+7
+//   producers (warps 0-3): y = [c qhat^-1] of one coefficient (or the pre-scaled input),
+//                          split into bytes, write the A row of A-stage i % 4, arrive full_a
+//   MMA (warp 20, lane 0): per tile i: wait full_a / tmem_empty[i % 2]; two K = 32 MMAs of
+//                          N = 48 * parts into slot i % 2; commit -> tmem_full, commit -> empty_a
+//                          (a serial chain of high-latency tcgen05 / mbarrier ops: one MMA pair
+//                          per tile instead of one per part halves the thread's time per tile)
+//   epilogue (4 sets of 4 warps, set q % 4 drains the q-th part of the CTA): tcgen05.ld of its
+//                          32 TMEM lanes x 48 columns, V = sum_b 2^(8b) D_b, one FP64 Barrett
+//                          step, store; every warp arrives tmem_empty once per tile
+// A tile of 36 targets is 4 parts, one per set.  Per-job / per-target constants and the tile
+// schedule are staged in shared memory during setup (register-indexed reads of the large
+// parameter block miss the constant cache on the critical path).
 template <bool kPre, bool kLazy, class LoadB>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
                                               int tiles_per_entry, int batch, int exp,
                                               const CUtensorMap* tmaps = nullptr, const int* use_tmap = nullptr,
                                               unsigned long long* dbg = nullptr) {
-    // debug trace (CTA 0 only): [i][0] producer after in_full, [1] producer arrive full_a,
-    // [2] MMA after waits, [3] MMA committed, [4] epilogue(set 0/1..) start, [5] epilogue end
+    // NEO_BCONV_DBG trace of CTA 0: [i][0..3] producer in / A ready, MMA start / committed,
+    // [i][4..5] epilogue part 0 start / last part end; row 60: waiting cycles per barrier
+    unsigned long long wacc[6] = {0, 0, 0, 0, 0, 0};
+    auto WAIT = [&](uint64_t* bar, uint32_t ph, int k) {
+        const unsigned long long t0 = dbg ? clock64() : 0;
+        tc::mbar_wait(bar, ph);
+        if (dbg) wacc[k] += clock64() - t0;
+    };
     auto T = [&](int i, int ev) {
-        if (dbg && blockIdx.x == 0 && i < 62) dbg[i * 8 + ev] = clock64();
+        if (dbg && blockIdx.x == 0 && i < 60) dbg[i * 8 + ev] = clock64();
     };
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t* sA = smem;                                  // kAStages x (128 rows x 64 B)
-    uint8_t* sB0 = smem + kAStages * kTileM * 64;        // kMaxJobs x 2 halves x (128 rows x 64 B)
+    uint8_t* sB0 = smem + kAStages * kTileM * 64;        // kMaxJobs x parts x (48 rows x 64 B)
     u64* sIn = reinterpret_cast<u64*>(sB0 + kMaxJobs * kBBytes);   // kInStages x [n_in][128]
+    JobH* sJob = reinterpret_cast<JobH*>(sIn + kInStages * BCTC_MAX_IN * kTileM);    // [job]
+    TgtC* sTgt = reinterpret_cast<TgtC*>(sJob + kMaxJobs);                           // [job][target]
+    uint32_t* sSched = reinterpret_cast<uint32_t*>(sTgt + kMaxJobs * kTgtRow);       // [i] -> jb | b | m-tile
     const int tiles_per_job = tiles_per_entry * batch;
     const int total_tiles = tiles_per_job * njobs;
     auto decode = [&](int tile, int& j, int& b, int& m0) {   // tile -> (conversion, batch entry, first coeff)
@@ -70,21 +103,22 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         b = r / tiles_per_entry;
         m0 = (r - b * tiles_per_entry) * kTileM;
     };
+    auto tile_at = [&](int i, int& j, int& b, int& m0) {   // the CTA's i-th tile, blockIdx.x + i G
+        if (i < kMaxSched) {
+            const uint32_t w = sSched[i];
+            j = w >> 28;
+            b = (w >> 16) & 0xFFF;
+            m0 = (int)(w & 0xFFFF) * kTileM;
+        } else {
+            decode(blockIdx.x + i * gridDim.x, j, b, m0);
+        }
+    };
     __shared__ uint64_t full_a[kAStages], empty_a[kAStages], tfull[kSlots], tempty[kSlots];
     __shared__ uint64_t in_full[kInStages], in_empty[kInStages];
     __shared__ uint32_t tmem_base;
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int G = gridDim.x;
-    auto GT = [&](int ev) {      // setup trace (row 63): globaltimer ns of CTA 0 / CTA G-1, thread 0
-        if (dbg && tid == 0 && (blockIdx.x == 0 || blockIdx.x == gridDim.x - 1)) {
-            unsigned long long t;
-            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-            dbg[63 * 8 + ev + (blockIdx.x ? 4 : 0)] = t;
-            if (!blockIdx.x) dbg[62 * 8 + ev] = clock64();
-        }
-    };
-    GT(0);
     if (warp == 0) tc::tmem_alloc(&tmem_base, kSlots * kSlotCols);
     if (tid == 0) {
         for (int s = 0; s < kAStages; ++s) {
@@ -93,7 +127,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         }
         for (int s = 0; s < kSlots; ++s) {
             tc::mbar_init(&tfull[s], 1);
-            tc::mbar_init(&tempty[s], 4);                // one arrival per warp of the set
+            tc::mbar_init(&tempty[s], kEpiWarps);        // one arrival per epilogue warp
         }
         for (int s = 0; s < kInStages; ++s) {
             tc::mbar_init(&in_full[s], 1);
@@ -102,60 +136,48 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     }
     for (int j = 0; j < njobs; ++j) {
         uint4* s4 = reinterpret_cast<uint4*>(sB0 + j * kBBytes);
-        const int n16 = PJ[j].nhalf * kSlotCols * 4;    // 16-byte chunks (halves padded to 128 rows)
+        const int n16 = PJ[j].nparts * (int)(kPartBytes / 16);
         for (int e = tid; e < n16; e += kThreads) s4[e] = loadB(j, e);
+    }
+    if (tid < njobs) {
+        const BConvTC& P = PJ[tid];
+        const BConvIO& io = IOJ[tid];
+        sJob[tid] = JobH{io.in, io.out, io.in_bstride, io.out_bstride, P.n_in, P.n_out, P.nparts, P.J, P.ncols,
+                         io.in_off[0], use_tmap ? use_tmap[tid] : 0, 0};
+    }
+    for (int x = tid; x < kMaxSched && blockIdx.x + x * G < total_tiles; x += kThreads) {
+        int j, b, m0;
+        decode(blockIdx.x + x * G, j, b, m0);
+        sSched[x] = ((uint32_t)j << 28) | ((uint32_t)b << 16) | (uint32_t)(m0 / kTileM);
+    }
+    for (int x = tid; x < njobs * kTgtRow; x += kThreads) {
+        const int j = x / kTgtRow, t = min(x - j * kTgtRow, PJ[j].n_out - 1);   // pad: repeat the last target
+        sTgt[x] = TgtC{PJ[j].t[t], PJ[j].tinv[t], (long long)IOJ[j].out_off[t] * N * 8, 0};
     }
     tc::fence_proxy_async();
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
-    GT(1);
     pdl_wait();            // B matrices / TMEM / barriers were set up while the predecessor drained
     pdl_trigger();
-    GT(2);
     const uint32_t tmem = tmem_base;
     const int total_run = (exp & 256) ? 0 : total_tiles;      // exp 256: setup/teardown only
 
-    auto tma_issue = [&](int i) {
-        const int tile = blockIdx.x + i * G;
-        if (tile >= total_run || (exp & 32)) return;
-        const int s = i % kInStages, k = i / kInStages;
-        tc::mbar_wait(&in_empty[s], (k & 1) ^ 1);
-        int jb, b, m0;
-        decode(tile, jb, b, m0);
-        const BConvTC& P = PJ[jb];
-        const BConvIO& io = IOJ[jb];
-        const u64* in = io.in + b * io.in_bstride + m0;
-        u64* dst = sIn + (size_t)s * BCTC_MAX_IN * kTileM;
-        tc::mbar_arrive_tx(&in_full[s], (uint32_t)P.n_in * kTileM * 8);
-        if (use_tmap && use_tmap[jb])      // one instruction for the [n_in][128] box
-            tc::tensor_g2s_3d(dst, &tmaps[jb], m0, io.in_off[0], b, &in_full[s]);
-        else                               // each 1-D bulk copy costs ~170 issue cycles
-            for (int j = 0; j < P.n_in; ++j)
-                tc::bulk_g2s(dst + j * kTileM, in + (size_t)io.in_off[j] * N, kTileM * 8, &in_full[s]);
-    };
-
     if (warp < 4) {
-        // ------------------------------------------------ producers (+ TMA issue on thread 0)
-        if (tid == 0)
-            for (int i = 0; i < kInStages - 1; ++i) {
-                tma_issue(i);
-                if (dbg && blockIdx.x == 0 && i < 3) dbg[62 * 8 + 4 + i] = clock64();
-            }
+        // ------------------------------------------------ producers
         uint8_t* arow0 = sA + (tid >> 3) * 512 + (tid & 7) * 16;   // row tid of A-stage 0
         int i = 0;
         for (int tile = blockIdx.x; tile < total_run; tile += G, ++i) {
-            if (tid == 0) tma_issue(i + kInStages - 1);
             int jb, b, m0;
-            decode(tile, jb, b, m0);
-            const BConvTC& P = PJ[jb];
+            tile_at(i, jb, b, m0);
+            const int n_in = sJob[jb].n_in;
             const int si = i % kInStages, ki = i / kInStages;
-            if (!(exp & 32)) tc::mbar_wait(&in_full[si], ki & 1);
+            if (!(exp & 32)) WAIT(&in_full[si], ki & 1, 1);
             if (tid == 0) T(i, 0);
             const u64* src = sIn + (size_t)si * BCTC_MAX_IN * kTileM + tid;
             u64 c[BCTC_MAX_IN];
 #pragma unroll
-            for (int j = 0; j < BCTC_MAX_IN; ++j) c[j] = (j < P.n_in) ? src[j * kTileM] : 0;
+            for (int j = 0; j < BCTC_MAX_IN; ++j) c[j] = (j < n_in) ? src[j * kTileM] : 0;
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&in_empty[si]);
             uint32_t w[16];
@@ -163,9 +185,13 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             for (int kk = 0; kk < 16; ++kk) w[kk] = 0;
 #pragma unroll
             for (int j = 0; j < BCTC_MAX_IN; ++j) {
-                if (j < P.n_in) {
-                    const double q = P.qin[j];
-                    const u64 y = kPre ? c[j] : d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
+                if (j < n_in) {
+                    u64 y = c[j];
+                    if (!kPre) {
+                        const BConvTC& P = PJ[jb];
+                        const double q = P.qin[j];
+                        y = d2u(canon(mulc(u2d(c[j]), P.qhat_inv[j], q), q, P.qinv_in[j]));
+                    }
                     const int bit = 40 * j, wi = bit >> 5, sh = bit & 31;
                     w[wi] |= (uint32_t)(y << sh);
                     w[wi + 1] |= (uint32_t)(y >> (32 - sh));
@@ -173,7 +199,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                 }
             }
             const int s = i % kAStages, k = i / kAStages;
-            tc::mbar_wait(&empty_a[s], (k & 1) ^ 1);
+            WAIT(&empty_a[s], (k & 1) ^ 1, 2);
             uint8_t* arow = arow0 + s * (kTileM * 64);
 #pragma unroll
             for (int cc = 0; cc < 4; ++cc)
@@ -184,95 +210,130 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             if (tid == 0) T(i, 1);
         }
     } else if (warp < 4 + kEpiWarps) {
-        // ------------------------------------------------ epilogue: set e owns TMEM slot e
+        // ------------------------------------------------ epilogue: set e drains parts q = e (mod 4)
         const int ew = warp - 4, quarter = ew & 3, e = ew >> 2;
         const int et = quarter * 32 + lane;                  // TMEM lane = A row = coefficient
-        const uint32_t trow = tmem + (uint32_t)(e * kSlotCols) + ((uint32_t)(quarter * 32) << 16);
-        int q = 0;                                           // job counter of this CTA
-        for (int tile = blockIdx.x; tile < total_run; tile += G) {
+        int q = 0, i = 0;                                    // part counter, tile counter of this CTA
+        for (int tile = blockIdx.x; tile < total_run; tile += G, ++i) {
             int jb, b, m0;
-            decode(tile, jb, b, m0);
-            const BConvTC& P = PJ[jb];
-            for (int h = 0; h < P.nhalf; ++h, ++q) {
-                if ((q % kSlots) != e) continue;
-                const int k = q / kSlots;
-                const BConvIO& io = IOJ[jb];
-                const int t0 = h * P.J, t1 = min(t0 + P.J, P.n_out);
-                tc::mbar_wait(&tfull[e], k & 1);
-                if (lane == 0 && quarter == 0 && h == 0) T(q / P.nhalf, 4);
-                tc::fence_after();
-                u64* outb = io.out + b * io.out_bstride + m0 + et;
-                // 8 targets per group, branch-free so the 8 FP64 chains interleave; the ragged
-                // last group re-reads its last valid column and predicates the stores.
-                for (int g = t0; g < t1; g += 8) {
-                    uint32_t v[40];
-#pragma unroll
-                    for (int x = 0; x < 5; ++x) {
-                        uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * x]);
-                        tc::tmem_ld8(trow + (uint32_t)(5 * (g - t0) + 8 * x), vv);
-                    }
-                    tc::tmem_wait_ld();
-                    double r[8];
-#pragma unroll
-                    for (int u = 0; u < 8; ++u) {
-                        const int t = min(g + u, t1 - 1);
-                        const uint32_t* D = &v[5 * u];
-                        const u64 lo = (u64)D[0] + ((u64)D[1] << 8) + ((u64)D[2] << 16);     // < 2^39
-                        const u64 hi = (u64)D[3] + ((u64)D[4] << 8);                          // < 2^31
-                        const double tq = P.t[t];
-                        r[u] = __dadd_rn(u2d(lo), mulc(u2d(hi), P.c24[t], tq));              // == V (mod t)
-                        if (!kLazy) r[u] = canon(r[u], tq, P.tinv[t]);
-                    }
-#pragma unroll
-                    for (int u = 0; u < 8; ++u) {
-                        const int t = g + u;
-                        const u64 val = kLazy ? (u64)__double_as_longlong(r[u]) : d2u(r[u]);
-                        if (t < t1) outb[(size_t)io.out_off[t] * N] = val;
-                    }
-                }
+            tile_at(i, jb, b, m0);
+            const JobH& H = sJob[jb];
+            const int nparts = H.nparts;
+            const int slot = i % kSlots, k = i / kSlots;
+            const int p0 = (e - q) & (kSets - 1);            // my first part of this tile
+            q += nparts;
+            WAIT(&tfull[slot], k & 1, 3);                    // (every warp: orders its arrival below)
+            if (lane == 0 && quarter == 0 && e == 0) T(i, 4);
+            tc::fence_after();
+            char* outb = reinterpret_cast<char*>(H.out + b * H.out_bs + m0 + et);
+            if (p0 >= nparts) {
                 tc::fence_before();
                 __syncwarp();
-                if (lane == 0) tc::mbar_arrive(&tempty[e]);
-                if (lane == 0 && quarter == 0 && h == P.nhalf - 1) T(q / P.nhalf, 5);
+                if (lane == 0) tc::mbar_arrive(&tempty[slot]);
+                continue;
             }
+            for (int p = p0; p < nparts; p += kSets) {
+                const uint32_t trow = tmem + (uint32_t)(slot * kSlotCols + p * BCTC_PART_ROWS) + ((uint32_t)(quarter * 32) << 16);
+                const int t0 = p * H.J, nt = min(H.J, H.n_out - t0);
+                uint32_t v[48];
+#pragma unroll
+                for (int x = 0; x < 6; ++x) {
+                    uint32_t (&vv)[8] = *reinterpret_cast<uint32_t (*)[8]>(&v[8 * x]);
+                    tc::tmem_ld8(trow + (uint32_t)(8 * x), vv);
+                }
+                tc::tmem_wait_ld();
+                if (p + kSets >= nparts) {                   // my last part: the slot can be refilled
+                    tc::fence_before();
+                    __syncwarp();
+                    if (lane == 0) tc::mbar_arrive(&tempty[slot]);
+                }
+                const TgtC* tg = sTgt + jb * kTgtRow + t0;
+                // V = sum_b 2^(8b) D_b < 2^51 assembled directly as the bits of 2^52 + V:
+                // (D0 + 2^8 D1) + 2^16 D2 + 2^24 D3 as a 64-bit word, then D4 and the exponent of
+                // 2^52 added to the high word (no carry: hi + D4 < 2^20).
+#pragma unroll
+                for (int u = 0; u < BCTC_PART_J; ++u) {
+                    const TgtC& C = tg[u];
+                    const uint32_t* D = &v[5 * u];
+                    u64 w = (u64)(D[0] + (D[1] << 8)) + (u64)D[2] * 65536ull;
+                    w += (u64)D[3] * 16777216ull;
+                    const double Vd = __dadd_rn(__hiloint2double((int)((uint32_t)(w >> 32) + D[4] + 0x43300000u),
+                                                                 (int)(uint32_t)w), -kTwo52);
+                    const double qf = __dadd_rn(__fma_rn(Vd, C.tinv, kMagic), -kMagic);
+                    double r = __fma_rn(-qf, C.t, Vd);                 // V mod t, |r| <= t/2 + 1 (exact)
+                    if (!kLazy) r = __dadd_rn(r, r < 0.0 ? C.t : 0.0);
+                    const u64 val = kLazy ? (u64)__double_as_longlong(r) : d2u(r);
+                    const uint32_t ok = u < nt;
+                    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.u64 [%0], %1;\n\t}"
+                                 :: "l"(outb + C.offb), "l"(val), "r"(ok) : "memory");
+                }
+            }
+            if (lane == 0 && quarter == 0 && e == 0) T(i, 5);
         }
-    } else {
+    } else if (warp == 4 + kEpiWarps) {
         // ------------------------------------------------ MMA issuer
         if (lane == 0) {
             const uint32_t aaddr = tc::smem_u32(sA);
-            int i = 0, q = 0;
+            int i = 0;
             for (int tile = blockIdx.x; tile < total_run; tile += G, ++i) {
                 const int s = i % kAStages, k = i / kAStages;
                 int jb, b, m0;
-                decode(tile, jb, b, m0);
-                const BConvTC& P = PJ[jb];
-                const uint32_t idesc = tc::idesc_u8(kTileM, P.ncols);
+                tile_at(i, jb, b, m0);
+                const JobH& H = sJob[jb];
+                const uint32_t idesc = tc::idesc_u8(kTileM, H.nparts * BCTC_PART_ROWS);
                 const uint32_t as = aaddr + s * (kTileM * 64);
-                tc::mbar_wait(&full_a[s], k & 1);
+                const int slot = i % kSlots, kq = i / kSlots;
+                WAIT(&full_a[s], k & 1, 4);
                 T(i, 2);
-                for (int h = 0; h < P.nhalf; ++h, ++q) {
-                    const int slot = q % kSlots, kq = q / kSlots;
-                    tc::mbar_wait(&tempty[slot], (kq & 1) ^ 1);
-                    tc::fence_after();
-                    const uint32_t acc = tmem + (uint32_t)(slot * kSlotCols);
-                    const uint32_t bs = tc::smem_u32(sB0 + jb * kBBytes + h * (kSlotCols * 64));
-                    {
-                        // K = 64 as two K = 32 steps (LBO = 128 B between K chunks, SBO = 512 B between row groups)
-                        tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(bs, 128, 512), idesc, 0);
-                        tc::mma_u8(acc, tc::sdesc(as + 256, 128, 512), tc::sdesc(bs + 256, 128, 512), idesc, 1);
-                    }
-                    tc::commit(&tfull[slot]);
+                WAIT(&tempty[slot], (kq & 1) ^ 1, 5);
+                tc::fence_after();
+                const uint32_t acc = tmem + (uint32_t)(slot * kSlotCols);
+                const uint32_t bs = tc::smem_u32(sB0 + jb * kBBytes);
+                if (!(exp & 16)) {
+                    // K = 64 as two K = 32 steps (LBO = 128 B between K chunks, SBO = 512 B between row groups)
+                    tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(bs, 128, 512), idesc, 0);
+                    tc::mma_u8(acc, tc::sdesc(as + 256, 128, 512), tc::sdesc(bs + 256, 128, 512), idesc, 1);
                 }
+                tc::commit(&tfull[slot]);
                 tc::commit(&empty_a[s]);
                 T(i, 3);
             }
         }
         __syncwarp();
+    } else {
+        // ------------------------------------------------ TMA issuer (input ring, 7 tiles ahead)
+        if (lane == 0) {
+            int i = 0;
+            for (int tile = blockIdx.x; tile < total_run && !(exp & 32); tile += G, ++i) {
+                const int s = i % kInStages, k = i / kInStages;
+                WAIT(&in_empty[s], (k & 1) ^ 1, 0);
+                int jb, b, m0;
+                tile_at(i, jb, b, m0);
+                const JobH& H = sJob[jb];
+                u64* dst = sIn + (size_t)s * BCTC_MAX_IN * kTileM;
+                tc::mbar_arrive_tx(&in_full[s], (uint32_t)H.n_in * kTileM * 8);
+                if (H.use_tmap) {                  // one instruction for the [n_in][128] box
+                    tc::tensor_g2s_3d(dst, &tmaps[jb], m0, H.in_off0, b, &in_full[s]);
+                } else {                           // each 1-D bulk copy costs ~170 issue cycles
+                    const u64* in = H.in + b * H.in_bs + m0;
+                    for (int j = 0; j < H.n_in; ++j)
+                        tc::bulk_g2s(dst + j * kTileM, in + (size_t)IOJ[jb].in_off[j] * N, kTileM * 8, &in_full[s]);
+                }
+            }
+        }
+        __syncwarp();
+    }
+    if (dbg && blockIdx.x == 0) {      // waiting cycles: TMA, producer tid 0, epilogue set 0, MMA
+        if (warp == 5 + kEpiWarps && lane == 0) dbg[60 * 8 + 0] = wacc[0];
+        if (tid == 0) { dbg[60 * 8 + 1] = wacc[1]; dbg[60 * 8 + 2] = wacc[2]; }
+        if (warp == 4 && lane == 0) dbg[60 * 8 + 3] = wacc[3];
+        if (warp == 4 + kEpiWarps && lane == 0) { dbg[60 * 8 + 4] = wacc[4]; dbg[60 * 8 + 5] = wacc[5]; }
+        if (warp == 4 && lane == 0) dbg[60 * 8 + 6] = clock64();
+        if (tid == 0) dbg[60 * 8 + 7] = clock64();
     }
     tc::fence_before();
     __syncthreads();
     if (warp == 0) tc::tmem_dealloc(tmem, kSlots * kSlotCols);
-    GT(3);
 }
 
 template <bool kPre, bool kLazy>

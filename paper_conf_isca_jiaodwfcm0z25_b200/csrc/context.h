@@ -36,20 +36,22 @@ struct BConvIO {
 };
 
 constexpr int BCTC_MAX_IN = 12;     // K = 5 * n_in <= 64
-constexpr int BCTC_MAX_OUT = 50;    // two half-tile jobs of <= 25 targets (N = 5 J <= 128)
+constexpr int BCTC_MAX_OUT = 45;    // targets per conversion (5 parts of 9: one MMA of N = 240)
+constexpr int BCTC_PART_J = 9;      // targets per TMEM job (N = 5 J = 45 -> 48 columns)
+constexpr int BCTC_PART_ROWS = 48;  // B rows per part (padded to the MMA N)
+constexpr int BCTC_MAX_PARTS = (BCTC_MAX_OUT + BCTC_PART_J - 1) / BCTC_PART_J;   // 6
 
 struct BConvTC {
     int n_in, n_out;
-    int nhalf, J;                   // targets split in nhalf jobs of J (last may be shorter)
-    int ncols;                      // MMA N per job = round_up(5 J, 16) <= 128
+    int nparts, J;                  // targets split in nparts jobs of J (last may be shorter)
+    int ncols;                      // MMA N per job = round_up(5 J, 16) <= 48
     double qin[BCTC_MAX_IN], qinv_in[BCTC_MAX_IN];
     TWD qhat_inv[BCTC_MAX_IN];      // [qhat_i^-1]_{q_i}
     double t[BCTC_MAX_OUT], tinv[BCTC_MAX_OUT];
-    TWD c24[BCTC_MAX_OUT];          // 2^24 mod t
 };
 
 struct BMatParam {                   // B passed by value (generic neo_bconv, no device tables)
-    uint4 d[2 * 128 * 64 / 16];      // two half-matrices of 128 rows x 64 B
+    uint4 d[BCTC_MAX_PARTS * BCTC_PART_ROWS * 64 / 16];   // parts of 48 rows x 64 B
 };
 
 }  // namespace neo

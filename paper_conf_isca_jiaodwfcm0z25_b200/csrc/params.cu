@@ -170,12 +170,12 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
     std::memset(&P, 0, sizeof(P));
     P.n_in = (int)src.size();
     P.n_out = (int)dst.size();
-    P.nhalf = (5 * P.n_out > 128) ? 2 : 1;
-    // the epilogue drains 8 targets per tcgen05.ld group: a first half of 24 targets has no
-    // ragged group (n_out <= 48; 25 + 25 for the largest bases)
-    P.J = P.nhalf == 1 ? P.n_out : (P.n_out <= 48 ? 24 : 25);
+    // targets in parts of J = 9 (45 MMA columns, padded to 48): one TMEM job and one
+    // tcgen05.ld batch per part in the epilogue
+    P.J = std::min(P.n_out, BCTC_PART_J);
+    P.nparts = (P.n_out + P.J - 1) / P.J;
     P.ncols = ((5 * P.J + 15) / 16) * 16;
-    bmat.assign((size_t)P.nhalf * 128 * 64, 0);      // each half padded to 128 rows
+    bmat.assign((size_t)P.nparts * BCTC_PART_ROWS * 64, 0);
     for (int i = 0; i < P.n_in; ++i) {
         u64 qi = src[i], qh = 1;
         for (int k = 0; k < P.n_in; ++k)
@@ -188,7 +188,6 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
         u64 m = dst[t];
         P.t[t] = (double)m;
         P.tinv[t] = 1.0 / (double)m;
-        P.c24[t] = mk_twd((1ull << 24) % m, m);
         for (int i = 0; i < P.n_in; ++i) {
             u64 f = 1;                                          // qhat_i mod t
             for (int k = 0; k < P.n_in; ++k)
@@ -197,7 +196,8 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
                 u64 v = mulm(f, (1ull << (8 * a)) % m, m);      // (2^(8a) qhat_i) mod t
                 for (int b = 0; b < 5; ++b) {
                     const int h = t / P.J, n = 5 * (t - h * P.J) + b, k = 5 * i + a;
-                    size_t off = (size_t)h * 128 * 64 + (size_t)(n / 8) * 512 + (k / 16) * 128 + (n % 8) * 16 + (k % 16);
+                    size_t off = (size_t)h * BCTC_PART_ROWS * 64 + (size_t)(n / 8) * 512 + (k / 16) * 128 +
+                                 (n % 8) * 16 + (k % 16);
                     bmat[off] = (uint8_t)((v >> (8 * b)) & 0xFF);
                 }
             }
@@ -291,6 +291,9 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
     {
         const char* e = std::getenv("NEO_BCONV");
         c->use_tc = !(e && std::string(e) == "cuda");
+        // the epilogue's exact FP64 sum of the byte planes needs every modulus < 2^36 (bconv_tc.cu)
+        for (int k = 0; k < c->num_q + c->num_p; ++k)
+            if (c->mod[k] >> 36) c->use_tc = false;
         std::vector<uint8_t> all, bm;
         c->modup_tc.resize(c->num_q);
         c->modup_boff.resize(c->num_q);

@@ -87,12 +87,25 @@ __device__ __forceinline__ void tensor_g2s_3d(void* dst, const void* tmap, int c
     asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];\n"
                  ::"r"(smem_u32(dst)), "l"(tmap), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(mbar)) : "memory");
 }
+__device__ __forceinline__ bool mbar_try(uint64_t* mbar, uint32_t phase) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, P1;\n\t}\n" : "=r"(ok) : "r"(smem_u32(mbar)), "r"(phase) : "memory");
+    return ok != 0;
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* mbar, uint32_t phase) {
     asm volatile(
         "{\n\t.reg .pred P1;\n"
         "WAIT_%=:\n\t"
         "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
         "@!P1 bra WAIT_%=;\n\t}\n" ::"r"(smem_u32(mbar)), "r"(phase) : "memory");
+}
+// as mbar_wait, backing off with nanosleep between polls (roles that wait long: keeps the
+// polling traffic off the shared-memory pipe the working warps need)
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* mbar, uint32_t phase, uint32_t ns) {
+    while (!mbar_try(mbar, phase)) __nanosleep(ns);
 }
 
 }  // namespace tc
