@@ -30,6 +30,7 @@ NEO_DEV void cp16(void* s, const void* g) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s_u32(s)), "l"(g) : "memory");
 }
 NEO_DEV void cp_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+NEO_DEV void pf_l2(const void* g) { asm volatile("prefetch.global.L2 [%0];\n" ::"l"(g)); }
 template <int N>
 NEO_DEV void cp_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
 
@@ -168,6 +169,17 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
         cp_commit();
     };
 
+    // single-stage configurations: pull the CTA's next tile into L2 while this one is
+    // transformed, so its cp.async sees L2 rather than HBM latency (one 128-B line per row)
+    auto prefetch = [&](int t) {
+        if (STAGES == 1 && t < tm.total) {
+            int b, k, blk;
+            tm.decode(t, b, k, blk);
+            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N + blk * C;
+            for (int row = tid; row < N1; row += NT) pf_l2(src + (size_t)row * N2);
+        }
+    };
+
     const int G = gridDim.x;
     int t = blockIdx.x;
     pdl_wait();            // predecessor's writes visible (and its reads done) before any access
@@ -176,6 +188,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
     for (int s = 0; s < STAGES; ++s) issue(t + s * G, s);
     for (int it = 0; t < tm.total; t += G, ++it) {
         const int s = it % STAGES;
+        prefetch(t + G);
         cp_wait<STAGES - 1>();
         __syncthreads();
         int b, k, blk;
@@ -300,6 +313,30 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
         cp_commit();
     };
 
+    // L2 prefetch of the CTA's next tile (single-stage configurations) and of the fused
+    // ModDown tail's acc / add rows of this tile (consumed only after the transform)
+    auto prefetch = [&](int t, bool epi_rows) {
+        if (t >= tm.total) return;
+        int b, k, blk;
+        tm.decode(t, b, k, blk);
+        const int row0 = blk * RR;
+        if (epi_rows) {
+            const int bb = b >> 1, cc = b & 1;
+            const u64* accr = ep.acc + bb * ep.acc_b + cc * ep.acc_c + (size_t)k * a.N + row0;
+            const u64* addr = cc ? ep.add1 : ep.add0;
+            for (int i2 = tid; i2 < N2; i2 += NT) {
+                pf_l2(accr + (size_t)N1 * i2);
+                if (addr) pf_l2(addr + bb * ep.add_b + (size_t)k * a.N + row0 + (size_t)N1 * i2);
+            }
+        } else if (STAGES == 1) {
+            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N;
+            if (FWD)
+                for (int e = tid; e < RR * N2 / 16; e += NT) pf_l2(src + (size_t)row0 * N2 + 16 * e);
+            else
+                for (int i2 = tid; i2 < N2; i2 += NT) pf_l2(src + row0 + (size_t)N1 * i2);
+        }
+    };
+
     const int G = gridDim.x;
     int t = blockIdx.x;
     pdl_wait();            // predecessor's writes visible (and its reads done) before any access
@@ -308,6 +345,8 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
     for (int s = 0; s < STAGES; ++s) issue(t + s * G, s);
     for (int it = 0; t < tm.total; t += G, ++it) {
         const int s = it % STAGES;
+        if (EPI) prefetch(t, true);
+        prefetch(t + G, false);
         cp_wait<STAGES - 1>();
         __syncthreads();
         int b, k, blk;

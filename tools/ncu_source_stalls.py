@@ -1,6 +1,6 @@
 """Per-instruction stall breakdown of an ncu report (--page source, SASS view).
 
-usage: python tools/ncu_source_stalls.py report.ncu-rep [kernel-regex] [top]"""
+usage: python tools/ncu_source_stalls.py report.ncu-rep [kernel-regex] [top] [launch-index]"""
 import csv
 import io
 import subprocess
@@ -13,8 +13,18 @@ cmd = ["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"]
 if kre:
     cmd += ["-k", "regex:" + kre]
 rows = list(csv.reader(io.StringIO(subprocess.run(cmd, capture_output=True, text=True).stdout)))
-h = rows[1]
-data = [r for r in rows[2:] if len(r) == len(h)]
+blocks, cur = [], None
+for r in rows:
+    if r and r[0] == "Kernel Name":
+        cur = {"name": r[1], "rows": []}
+        blocks.append(cur)
+    elif cur is not None:
+        cur["rows"].append(r)
+which = int(sys.argv[4]) if len(sys.argv) > 4 else 0
+blk = blocks[which]
+print(blk["name"], f"({len(blocks)} kernels in report)")
+h = blk["rows"][0]
+data = [r for r in blk["rows"][1:] if len(r) == len(h)]
 ia, isrc, ie = h.index("Address"), h.index("Source"), h.index("Instructions Executed")
 iss = h.index("Warp Stall Sampling (All Samples)")
 cols = [c for c in h if c.startswith("stall_") and "Not Issued" not in c]
