@@ -5,8 +5,8 @@ timeout 300 python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 |
 timeout 900 python bench.py > gpurun_out/bench_full.json 2> gpurun_out/bench_full.err; tail -3 gpurun_out/bench_full.err
 cat gpurun_out/bench_full.json
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
-    python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --graph 0 --streams 1 > /dev/null 2>&1
+    python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-hoisted --graph 0 --streams 1 > /dev/null 2>&1
 wc -l gpurun_out/launches.csv
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_ntt_col|k_ntt_row|k_bconv_tc|k_keyip" -s 40 -c 8 \
-    -o gpurun_out/prof_top python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --graph 0 --streams 1 > gpurun_out/ncu_top.log 2>&1
+    -o gpurun_out/prof_top python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-hoisted --graph 0 --streams 1 > gpurun_out/ncu_top.log 2>&1
 tail -2 gpurun_out/ncu_top.log
