@@ -18,6 +18,8 @@ silent/garbled passages are SURVEY.md §8(c) Z1-Z23, listed in DESIGN.md):
 * HMULT         -- L132: d0 = a0 b0, d1 = a0 b1 + a1 b0, d2 = a1 b1; KS(d2) added to d0, d1
 * HROTATE       -- L136, L184: automorphism then KS with the rotation key (Z11)
 * Rescale       -- L137: divide by the last prime, floor rounding (Z10)
+* Double Rescale-- L138, L151: divide by the last two primes, floor (reading "DS")
+* PMULT / HADD / PADD -- L133-135: element-wise products and sums in the NTT domain
 * encode/decode, keygen, encrypt/decrypt -- L121-130 with the standard sign (Z1),
                    gadget of Z8, distributions of Z12 (host-only, never on the GPU path)
 
@@ -396,6 +398,48 @@ def rescale(prm, ct, level, mode="fast"):
     return np.stack(out)
 
 
+def double_rescale(prm, ct, level, mode="fast"):
+    """Double Rescale (DS, L138, L151): divide by the last TWO primes and drop two levels.
+    Reading ("DS"): floor rounding like Rescale (Z10), c' = floor(x / (q_{l-1} q_l)),
+    the "noise reduction limb" being r = x mod q_{l-1} q_l recovered exactly from the last two
+    limbs (Garner):  r = r_l + q_l * [(r_{l-1} - r_l) q_l^-1]_{q_{l-1}},  then
+    c'_i = (c_i - [r]_{q_i}) * (q_{l-1} q_l)^-1 mod q_i  for i < l-1."""
+    ql, qm = prm.moduli[level], prm.moduli[level - 1]
+    ids = list(range(level - 1))
+    ql_inv_m = pow(ql % qm, -1, qm)
+    out = []
+    for c in range(ct.shape[0]):
+        r_m, r_l = intt(prm, ct[c][level - 1:level + 1], [level - 1, level], mode)   # coeff form
+        g = scalar_mul(prm, sub(prm, r_m[None], (r_l % np.uint64(qm))[None], [level - 1]), [ql_inv_m],
+                       [level - 1])[0]                                           # in [0, q_{l-1})
+        red = np.stack([r_l % np.uint64(prm.moduli[i]) for i in ids])
+        red = add(prm, red, scalar_mul(prm, np.stack([g % np.uint64(prm.moduli[i]) for i in ids]),
+                                       [ql % prm.moduli[i] for i in ids], ids), ids)  # [r]_{q_i}
+        red_ntt = ntt(prm, red, ids, mode)
+        diff = sub(prm, ct[c][:level - 1], red_ntt, ids)
+        out.append(scalar_mul(prm, diff, [pow(ql * qm % prm.moduli[i], -1, prm.moduli[i]) for i in ids], ids))
+    return np.stack(out)
+
+
+def pmult(prm, ct, pt, level):
+    """PMULT (L133): plaintext m (NTT form, [level+1][N]) times ciphertext: (c0 m, c1 m)."""
+    ids = list(range(level + 1))
+    return np.stack([mul(prm, ct[0], pt, ids), mul(prm, ct[1], pt, ids)])
+
+
+def hadd(prm, ct_a, ct_b, level):
+    """HADD (L134): (a0 + b0, a1 + b1)."""
+    ids = list(range(level + 1))
+    return np.stack([add(prm, ct_a[0], ct_b[0], ids), add(prm, ct_a[1], ct_b[1], ids)])
+
+
+def padd(prm, ct, pt, level):
+    """PADD (L135): (c0 + m, c1) -- m joins c0, the component decryption does not multiply by
+    s (Z1: decrypt = c0 + c1 s)."""
+    ids = list(range(level + 1))
+    return np.stack([add(prm, ct[0], pt, ids), np.array(ct[1], copy=True)])
+
+
 # --------------------------------------------------------------------------- keys, enc/dec
 
 def secret(prm: Params, seed: int, h: int = 192) -> np.ndarray:
@@ -466,7 +510,8 @@ def encrypt(prm: Params, m: np.ndarray, s: np.ndarray, level: int, seed: int, mo
     ids = list(range(level + 1))
     a = synth.uniform_residues(synth.derive(seed, 0xA), [prm.moduli[i] for i in ids], prm.N)
     e = synth.rounded_gaussian(synth.derive(seed, 0xE), prm.N)
-    me = np.asarray(m, dtype=np.int64) + e
+    m = np.asarray(m)
+    me = (m + e.astype(object)) if m.dtype == object else m.astype(np.int64) + e   # object: |m| >= 2^63
     me_ntt = ntt(prm, reduce_signed(prm, me, ids), ids, mode)
     s_ntt = ntt(prm, reduce_signed(prm, s, ids), ids, mode)
     c0 = sub(prm, me_ntt, mul(prm, a, s_ntt, ids), ids)

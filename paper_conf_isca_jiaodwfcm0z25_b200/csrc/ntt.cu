@@ -106,10 +106,12 @@ constexpr int kC = 16;   // columns per column-pass tile / rows per row-pass til
 
 struct TileMap {        // rows (b, k) in limb-major order: consecutive tiles share a prime
     int batch, tpr, total;
+    int tpr_log;            // tpr = 2^tpr_log
+    unsigned bmagic;        // floor(2^32 / batch) + 1 (batch > 1): exact for ri * batch < 2^32
     NEO_DEV void decode(int t, int& b, int& k, int& blk) const {
-        const int ri = t / tpr;
-        blk = t - ri * tpr;
-        k = ri / batch;
+        const int ri = t >> tpr_log;
+        blk = t & (tpr - 1);
+        k = (batch == 1) ? ri : (int)__umulhi((unsigned)ri, bmagic);
         b = ri - k * batch;
     }
 };
@@ -193,11 +195,9 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
         __syncthreads();
         int b, k, blk;
         tm.decode(t, b, k, blk);
-        const int lid = rs.prime[k];
-        const ModQ mq = a.mods[lid];
-        const double q = mq.qd;
         unsigned char* st = stage_ptr(s);
         const TWD* NEG = reinterpret_cast<const TWD*>(st);
+        const double q = NEG[0].w, qinv = NEG[0].wq;      // entry 0 of the table holds (q, 1/q)
         const TWD* TW1 = NEG + R;
         const TWD* CYC = NEG + R + R * R;
         const TWD* sA = NEG + CF::NS;
@@ -234,7 +234,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
             if (rs.has_scale) {                            // fold a per-row constant (e.g. qhat^-1) into the twist
                 double w = mulc(ta.w, rs.scale[k], q);
                 w = w < 0.0 ? __dadd_rn(w, q) : w;
-                ta = TWD{w, __dmul_rn(w, mq.qinv)};
+                ta = TWD{w, __dmul_rn(w, qinv)};
             }
 #pragma unroll
             for (int ib = 0; ib < R; ++ib) x[ib] = mulc(mulc(sD[(r + R * ib) * C + c], ta, q), sB[ib * C + c], q);
@@ -247,7 +247,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
             for (int j = 0; j < R; ++j) x[j] = S[r * R + BitRev<R>::of(j)];
             neg_inv<R>(x, NEG, q);
 #pragma unroll
-            for (int na = 0; na < R; ++na) dst[(size_t)(R * na + r) * N2 + n2] = d2u(canon(x[na], q, mq.qinv));
+            for (int na = 0; na < R; ++na) dst[(size_t)(R * na + r) * N2 + n2] = d2u(canon(x[na], q, qinv));
         }
         __syncthreads();                                   // stage s free
         issue(t + STAGES * G, s);
@@ -351,11 +351,9 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
         __syncthreads();
         int b, k, blk;
         tm.decode(t, b, k, blk);
-        const int lid = rs.prime[k];
-        const ModQ mq = a.mods[lid];
-        const double q = mq.qd;
         unsigned char* st = stage_ptr(s);
         const TWD* CYC = reinterpret_cast<const TWD*>(st);
+        const double q = CYC[0].w, qinv = CYC[0].wq;      // entry 0 of the table holds (q, 1/q)
         const TWD* TW2 = CYC + R / 2;
         double* sD = reinterpret_cast<double*>(st + CF::NS * sizeof(TWD));
         double* S = sD + rho * CF::XP;
@@ -376,7 +374,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
             __syncthreads();
             u64* T = reinterpret_cast<u64*>(sD);
 #pragma unroll
-            for (int ib = 0; ib < R; ++ib) T[swz(r + R * ib, rho)] = d2u(canon(x[BitRev<R>::of(ib)], q, mq.qinv));
+            for (int ib = 0; ib < R; ++ib) T[swz(r + R * ib, rho)] = d2u(canon(x[BitRev<R>::of(ib)], q, qinv));
             __syncthreads();
             if (!EPI) {
                 for (int e = tid; e < N2 * 8; e += NT) {
@@ -386,7 +384,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                 }
             } else {      // fused ModDown tail (a10): out = (acc - conv) P^-1 (+ add)
                 const int bb = b >> 1, cc = b & 1;
-                const u64 qq = mq.q;
+                const u64 qq = d2u(q);
                 const TW pinv = ep.pinv[k];
                 const u64* accr = ep.acc + bb * ep.acc_b + cc * ep.acc_c + (size_t)k * a.N;
                 const u64* addr = cc ? ep.add1 : ep.add0;
@@ -460,6 +458,9 @@ static cudaError_t launch_cfg(bool col, const RowSet& rs, const NttArgs& a, int 
     TileMap tm;
     tm.batch = batch;
     tm.tpr = col ? a.N2 / kC : a.N1 / kC;
+    tm.tpr_log = 0;
+    while ((1 << tm.tpr_log) < tm.tpr) ++tm.tpr_log;
+    tm.bmagic = batch > 1 ? (unsigned)((1ull << 32) / (unsigned)batch + 1) : 0u;
     tm.total = tm.tpr * rs.n * batch;
     int grid = MINB * a.num_sms;
     if (grid > tm.total) grid = tm.total;

@@ -8,7 +8,8 @@
 //   pass 2 (row kernel)   : cyclic N2-point DFT over n2 with omega2 = psi^(2 N1),
 //                           written to a_hat[i1 + N1*i2]
 // and each N1/N2-point transform is itself R x R in registers with a shared-memory
-// exchange.  Every table entry is a TW {w, floor(w 2^64 / q)} pair.
+// exchange.  Every table entry is a TWD {w, fl(w / q)} pair; entry 0 of the four
+// neg / cyc tables (the unit twiddle, never multiplied by) holds {q, fl(1 / q)} instead.
 #pragma once
 
 struct NttLayout {

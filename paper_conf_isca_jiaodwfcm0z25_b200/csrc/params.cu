@@ -115,6 +115,10 @@ static void fill_ntt_block(TWD* t, const NttLayout& L, u64 q, u64 psi, int N) {
         t[L.rowf_cyc + j] = mk_twd(P(om2R, j), q);
         t[L.rowi_cyc + j] = mk_twd(P(iom2R, j), q);
     }
+    // entry 0 of the negacyclic and cyclic tables (the unit twiddle, never read as one) carries
+    // (q, fl(1/q)) for the kernels that stage these tables in shared memory
+    const TWD qq{(double)q, 1.0 / (double)q};
+    t[L.colf_neg] = t[L.coli_neg] = t[L.rowf_cyc] = t[L.rowi_cyc] = qq;
     const u64 two_n = 2ull * N;
     for (int n2 = 0; n2 < N2; ++n2)
         for (int r = 0; r < R; ++r) {
