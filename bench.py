@@ -163,7 +163,7 @@ def bytes_model(batch: int, l: int = LEVEL) -> dict:
     tensor = batch * 7 * Lq
     auto = batch * 4 * Lq
     out = {"ntt_col": ntt_col, "ntt_row": ntt_row, "bconv": bconv, "keyip": keyip, "combine": 0,
-           "tensor": tensor, "automorphism": auto, "rescale_modswitch": 0, "rescale_combine": 0}
+           "tensor": tensor, "automorphism": auto, "rescale_modswitch": 0, "rescale_combine": 0, "elementwise": 0}
     return {k: v * limb for k, v in out.items()}
 
 

@@ -50,7 +50,8 @@ typedef enum {
 } neo_status;
 
 /* Operation codes for neo_workspace_size. */
-enum { NEO_OP_KEYSWITCH = 0, NEO_OP_HMULT = 1, NEO_OP_HROT = 2, NEO_OP_RESCALE = 3, NEO_OP_HROT_HOISTED = 4 };
+enum { NEO_OP_KEYSWITCH = 0, NEO_OP_HMULT = 1, NEO_OP_HROT = 2, NEO_OP_RESCALE = 3, NEO_OP_HROT_HOISTED = 4,
+       NEO_OP_DOUBLE_RESCALE = 5 };
 
 /* Parameter description (Table 1, Table 4).
  *  log_n      : log2 N; this build supports 12 and 16 (N = 2^12 tiny config, 2^16 Set-B).
@@ -177,6 +178,27 @@ neo_status neo_moddown_combine(const neo_ctx* ctx, const uint64_t* acc, const ui
 neo_status neo_rescale(const neo_ctx* ctx, const uint64_t* ct_in, int32_t level, uint64_t* ct_out,
                        int32_t batch, void* ws, size_t ws_bytes, neo_stream_t stream);
 
+/* Double Rescale (DS, L138 and L151: "requires the last two levels of limbs to generate noise
+ * reduction limbs ... consumes two ciphertext levels").  Reading: floor
+ * division by q_{l-1} q_l, i.e. bit-identical to two successive neo_rescale calls:
+ *   r = x mod q_{l-1} q_l  (exact, Garner on the last two limbs),
+ *   c'_i = (c_i - [r]_{q_i}) * (q_{l-1} q_l)^-1 mod q_i,  i < l - 1.
+ * ct_in [batch][2][level+1][N] -> ct_out [batch][2][level-1][N]; level >= 2;
+ * ws >= neo_workspace_size(ctx, NEO_OP_DOUBLE_RESCALE, level, batch). */
+neo_status neo_double_rescale(const neo_ctx* ctx, const uint64_t* ct_in, int32_t level, uint64_t* ct_out,
+                              int32_t batch, void* ws, size_t ws_bytes, neo_stream_t stream);
+
+/* Element-wise ciphertext operations without key-switching (L133-135), NTT form, one launch
+ * each, no workspace.  ct_* are [batch][2][level+1][N]; pt is a plaintext polynomial
+ * [batch][level+1][N] (one per ciphertext).  ct_out may alias ct_in / ct_a (same position).
+ *   PMULT: (c0 * m, c1 * m);   HADD: (a0 + b0, a1 + b1);   PADD: (c0 + m, c1)  (Z1 sign). */
+neo_status neo_pmult(const neo_ctx* ctx, const uint64_t* ct_in, const uint64_t* pt, int32_t level,
+                     uint64_t* ct_out, int32_t batch, neo_stream_t stream);
+neo_status neo_hadd(const neo_ctx* ctx, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level,
+                    uint64_t* ct_out, int32_t batch, neo_stream_t stream);
+neo_status neo_padd(const neo_ctx* ctx, const uint64_t* ct_in, const uint64_t* pt, int32_t level,
+                    uint64_t* ct_out, int32_t batch, neo_stream_t stream);
+
 /* Thread-local message describing the last non-OK status returned on this thread. */
 const char* neo_last_error(void);
 
@@ -189,9 +211,10 @@ int32_t neo_last_launch_count(void);
  * neo_profile_read synchronises on the recorded events and returns the summed device
  * time (ms) and launch count of one kernel kind:
  *   0 NTT column pass, 1 NTT row pass, 2 BConv, 3 KeyIP, 4 combine (ModDown tail),
- *   5 tensor, 6 automorphism, 7 rescale mod-switch, 8 rescale combine. */
+ *   5 tensor, 6 automorphism, 7 mod-switch (Double Rescale's noise-reduction limbs),
+ *   8 rescale combine, 9 element-wise (PMULT / HADD / PADD). */
 enum { NEO_PK_NTT_COL = 0, NEO_PK_NTT_ROW, NEO_PK_BCONV, NEO_PK_KEYIP, NEO_PK_COMBINE,
-       NEO_PK_TENSOR, NEO_PK_AUTO, NEO_PK_MODSW, NEO_PK_RESCALE, NEO_PK_COUNT };
+       NEO_PK_TENSOR, NEO_PK_AUTO, NEO_PK_MODSW, NEO_PK_RESCALE, NEO_PK_EW, NEO_PK_COUNT };
 neo_status neo_profile_enable(int32_t on);
 neo_status neo_profile_read(int32_t kind, double* total_ms, int32_t* launches);
 

@@ -51,7 +51,7 @@ static unsigned long long* bconv_dbg() {
 // Optional CUDA-event pairs around every launch (neo_profile_enable), read back per
 // kernel kind by neo_profile_read; used by bench.py to time kernels inside its timed region.
 enum { PK_NTT_COL = 0, PK_NTT_ROW, PK_BCONV, PK_KEYIP, PK_COMBINE, PK_TENSOR, PK_AUTO, PK_MODSW,
-       PK_RESCALE, PK_COUNT };
+       PK_RESCALE, PK_EW, PK_COUNT };
 struct ProfRec { int kind; cudaEvent_t a, b; };
 static thread_local bool g_prof = false;
 static thread_local std::vector<ProfRec> g_recs;
@@ -141,6 +141,12 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
 static size_t rescale_ws(const neo_ctx* c, int l, int B) {
     const size_t N = c->N;
     return (size_t)2 * B * N + (size_t)2 * B * std::max(l, 1) * N;
+}
+
+// Double Rescale: last2 [2B][2][N], corr [2B][l-1][N], NTT intermediate [2B][max(l-1, 2)][N]
+static size_t ds_ws(const neo_ctx* c, int l, int B) {
+    const size_t N = c->N;
+    return (size_t)4 * B * N + (size_t)2 * B * (l - 1) * N + (size_t)2 * B * std::max(l - 1, 2) * N;
 }
 
 // ------------------------------------------------------------------ key-switch core
@@ -429,6 +435,7 @@ size_t neo_workspace_size(const neo_ctx* c, int32_t op, int32_t level, int32_t b
         case NEO_OP_HROT:
         case NEO_OP_HROT_HOISTED: return ks_layout(c, level, batch, op).total * sizeof(u64);
         case NEO_OP_RESCALE: return level >= 1 ? rescale_ws(c, level, batch) * sizeof(u64) : 0;
+        case NEO_OP_DOUBLE_RESCALE: return level >= 2 ? ds_ws(c, level, batch) * sizeof(u64) : 0;
         default: return 0;
     }
 }
@@ -774,6 +781,76 @@ neo_status neo_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, u
     ep.out_b = (long long)2 * l * N;
     for (int i = 0; i < l; ++i) ep.pinv[i] = c->ql_inv[l][i];
     TRY(ntt_rows(c, true, last, N, so, ct_out, (long long)l * N, dof, pr, l, tmp, B2, s, &ep));
+    return NEO_OK;
+}
+
+static neo_status ew_api(const neo_ctx* c, int op, const uint64_t* a, const uint64_t* b, int32_t level, uint64_t* out,
+                         int32_t batch, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(a, "ct_in"));
+    TRY(check_ptr(b, op == EW_HADD ? "ct_b" : "pt"));
+    TRY(check_ptr(out, "ct_out"));
+    EwArgs A;
+    A.a = a; A.b = b; A.out = out; A.mods = c->d_mods;
+    A.N = c->N; A.limbs = level + 1; A.op = op;
+    LAUNCH(PK_EW, S(st), launch_ew(A, batch, S(st)));
+    return NEO_OK;
+}
+
+neo_status neo_pmult(const neo_ctx* c, const uint64_t* ct_in, const uint64_t* pt, int32_t level, uint64_t* ct_out,
+                     int32_t batch, neo_stream_t st) {
+    return ew_api(c, EW_PMULT, ct_in, pt, level, ct_out, batch, st);
+}
+neo_status neo_hadd(const neo_ctx* c, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level, uint64_t* ct_out,
+                    int32_t batch, neo_stream_t st) {
+    return ew_api(c, EW_HADD, ct_a, ct_b, level, ct_out, batch, st);
+}
+neo_status neo_padd(const neo_ctx* c, const uint64_t* ct_in, const uint64_t* pt, int32_t level, uint64_t* ct_out,
+                    int32_t batch, neo_stream_t st) {
+    return ew_api(c, EW_PADD, ct_in, pt, level, ct_out, batch, st);
+}
+
+neo_status neo_double_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, uint64_t* ct_out,
+                              int32_t batch, void* ws, size_t ws_bytes, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level, batch));
+    if (level < 2) FAIL(NEO_EINVAL, "double rescale needs level >= 2");
+    TRY(check_ptr(ct_in, "ct_in"));
+    TRY(check_ptr(ct_out, "ct_out"));
+    TRY(check_ws(c, NEO_OP_DOUBLE_RESCALE, level, batch, ws, ws_bytes));
+    const int N = c->N, l = level, B2 = 2 * batch;
+    u64* w = static_cast<u64*>(ws);
+    u64* last2 = w;                                   // [2B][2][N] coefficient form of c_{l-1}, c_l
+    u64* corr = last2 + (size_t)B2 * 2 * N;           // [2B][l-1][N]
+    u64* tmp = corr + (size_t)B2 * (l - 1) * N;       // NTT intermediate
+    cudaStream_t s = S(st);
+    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    // 1. coefficient form of the last two limbs of both components
+    for (int k = 0; k < 2; ++k) { so[k] = l - 1 + k; dof[k] = k; pr[k] = l - 1 + k; }
+    TRY(ntt_rows(c, false, ct_in, (long long)(l + 1) * N, so, last2, 2LL * N, dof, pr, 2, tmp, B2, s));
+    // 2. the noise-reduction limbs [x mod q_{l-1} q_l]_{q_i}, i < l - 1 (Garner, exact)
+    DsArgs D;
+    D.last2 = last2; D.corr = corr; D.mods = c->d_mods; D.N = N; D.l = l;
+    D.qlinv_m = c->ds_qlinv_m[l];
+    for (int i = 0; i + 1 < l; ++i) D.ql[i] = c->ds_ql[l][i];
+    LAUNCH(PK_MODSW, s, launch_ds_corr(D, B2, s));
+    // 3. NTT of them; the row pass's epilogue writes (c_i - corr_i) (q_{l-1} q_l)^-1 mod q_i
+    for (int i = 0; i + 1 < l; ++i) { so[i] = dof[i] = pr[i] = i; }
+    RowEpi ep;
+    ep.acc = ct_in;
+    ep.acc_b = (long long)2 * (l + 1) * N;
+    ep.acc_c = (long long)(l + 1) * N;
+    ep.add0 = ep.add1 = nullptr;
+    ep.add_b = 0;
+    ep.out0 = ct_out;
+    ep.out1 = ct_out + (size_t)(l - 1) * N;
+    ep.out_b = (long long)2 * (l - 1) * N;
+    for (int i = 0; i + 1 < l; ++i) ep.pinv[i] = c->ds_inv[l][i];
+    TRY(ntt_rows(c, true, corr, (long long)(l - 1) * N, so, ct_out, (long long)(l - 1) * N, dof, pr, l - 1, tmp, B2,
+                 s, &ep));
     return NEO_OK;
 }
 

@@ -79,6 +79,10 @@ struct neo_ctx {
     int num_sms = 148;
     bool use_tc = true;                              // NEO_BCONV=cuda selects the CUDA-core control kernel
     std::vector<std::vector<TW>> ql_inv;             // [l][i] q_l^-1 mod q_i, i < l
+    // Double Rescale at level l >= 2 (i < l - 1): (q_{l-1} q_l)^-1 mod q_i and q_l mod q_i;
+    // ds_qlinv_m[l] = q_l^-1 mod q_{l-1}
+    std::vector<std::vector<TW>> ds_inv, ds_ql;
+    std::vector<TW> ds_qlinv_m;
 
     int beta(int level) const { return (level + 1 + alpha - 1) / alpha; }
     int ext(int level) const { return level + 1 + num_p; }          // limbs of PQ_l

@@ -175,6 +175,63 @@ k_rescale_combine(RescaleArgs A) {
     A.out[((size_t)bc * A.l + i) * A.N + n] = shoup(sub_mod(x, v, q), A.qlinv[i], q);
 }
 
+// ------------------------------------------------------------------ PMULT / HADD / PADD
+// L133-135, two coefficients per thread (16-byte accesses):
+//   PMULT (c0 m, c1 m);  HADD (a0 + b0, a1 + b1);  PADD (c0 + m, c1)   (Z1: m joins c0)
+__global__ void __launch_bounds__(256)
+k_ew(const __grid_constant__ EwArgs A) {
+    pdl_wait();
+    const int n = 2 * (blockIdx.x * blockDim.x + threadIdx.x);
+    const int i = blockIdx.y, b = blockIdx.z;
+    if (n >= A.N) return;
+    const ModQ m = A.mods[i];
+    const size_t cs = (size_t)A.limbs * A.N;
+    const size_t ct = (size_t)b * 2 * cs + (size_t)i * A.N + n;
+    const size_t pt = (size_t)b * cs + (size_t)i * A.N + n;
+    const ulonglong2 x0 = *reinterpret_cast<const ulonglong2*>(A.a + ct);
+    const ulonglong2 x1 = *reinterpret_cast<const ulonglong2*>(A.a + ct + cs);
+    ulonglong2 y0, y1;
+    if (A.op == EW_HADD) {
+        const ulonglong2 b0 = *reinterpret_cast<const ulonglong2*>(A.b + ct);
+        const ulonglong2 b1 = *reinterpret_cast<const ulonglong2*>(A.b + ct + cs);
+        y0 = make_ulonglong2(add_mod(x0.x, b0.x, m.q), add_mod(x0.y, b0.y, m.q));
+        y1 = make_ulonglong2(add_mod(x1.x, b1.x, m.q), add_mod(x1.y, b1.y, m.q));
+    } else {
+        const ulonglong2 p = *reinterpret_cast<const ulonglong2*>(A.b + pt);
+        if (A.op == EW_PMULT) {
+            y0 = make_ulonglong2(mul_mod(x0.x, p.x, m), mul_mod(x0.y, p.y, m));
+            y1 = make_ulonglong2(mul_mod(x1.x, p.x, m), mul_mod(x1.y, p.y, m));
+        } else {
+            y0 = make_ulonglong2(add_mod(x0.x, p.x, m.q), add_mod(x0.y, p.y, m.q));
+            y1 = x1;
+        }
+    }
+    *reinterpret_cast<ulonglong2*>(A.out + ct) = y0;
+    *reinterpret_cast<ulonglong2*>(A.out + ct + cs) = y1;
+}
+
+// ------------------------------------------------------------------ Double Rescale (L138, L151)
+// Garner: r = r_l + q_l g, g = [(r_{l-1} - r_l) q_l^-1]_{q_{l-1}}, is x mod q_{l-1} q_l exactly
+// (0 <= r < q_{l-1} q_l); corr_i = [r]_{q_i} = r_l + [q_l]_{q_i} g mod q_i.
+__global__ void __launch_bounds__(256)
+k_ds_corr(const __grid_constant__ DsArgs A) {
+    pdl_wait();
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int bc = blockIdx.y;
+    if (n >= A.N) return;
+    const u64 qm = A.mods[A.l - 1].q;
+    const u64 rm = A.last2[(size_t)bc * 2 * A.N + n];
+    const u64 rl = A.last2[((size_t)bc * 2 + 1) * A.N + n];
+    const u64 rlm = rl >= qm ? rl - qm : rl;                     // r_l < q_l < 2^36 <= 2 q_{l-1}
+    const u64 g = shoup(sub_mod(rm, rlm, qm), A.qlinv_m, qm);
+    u64* out = A.corr + (size_t)bc * (A.l - 1) * A.N + n;
+    for (int i = 0; i + 1 < A.l; ++i) {
+        const u64 qi = A.mods[i].q;
+        const u64 rli = rl >= qi ? rl - qi : rl;
+        out[(size_t)i * A.N] = add_mod(rli, shoup(g, A.ql[i], qi), qi);
+    }
+}
+
 // ------------------------------------------------------------------ 5-byte key packing
 __global__ void __launch_bounds__(256)
 k_pack5(const u64* __restrict__ in, uint32_t* __restrict__ lo, uint8_t* __restrict__ hi, size_t n) {
@@ -187,6 +244,12 @@ k_pack5(const u64* __restrict__ in, uint32_t* __restrict__ lo, uint8_t* __restri
 }
 
 // ------------------------------------------------------------------ launchers
+cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st) {
+    return launch_k(k_ew, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);
+}
+cudaError_t launch_ds_corr(const DsArgs& A, int bc, cudaStream_t st) {
+    return launch_k(k_ds_corr, dim3((A.N + 255) / 256, bc), dim3(256), 0, st, A);
+}
 cudaError_t launch_pack5(const u64* in, uint32_t* lo, uint8_t* hi, size_t n, cudaStream_t st) {
     return launch_k(k_pack5, dim3(4096), dim3(256), 0, st, in, lo, hi, n);
 }

@@ -44,6 +44,30 @@ struct RescaleArgs {
     TW qlinv[64];
 };
 
+// Element-wise ciphertext ops (L133-135) on [batch][2][limbs][N] ciphertexts and
+// [batch][limbs][N] plaintexts, NTT form.
+enum EwOp { EW_PMULT = 0, EW_HADD = 1, EW_PADD = 2 };
+struct EwArgs {
+    const u64* a;          // ct [B][2][limbs][N]
+    const u64* b;          // ct (HADD) or plaintext [B][limbs][N]
+    u64* out;              // ct [B][2][limbs][N]
+    const ModQ* mods;
+    int N, limbs, op;
+};
+
+// Double Rescale step 2: from the coefficient form of the last two limbs r[bc][2][N]
+// (mod q_{l-1}, mod q_l) writes corr[bc][i][N] = [x mod q_{l-1} q_l]_{q_i} for i < l - 1.
+struct DsArgs {
+    const u64* last2;      // [2B][2][N]
+    u64* corr;             // [2B][l-1][N]
+    const ModQ* mods;
+    int N, l;
+    TW qlinv_m;            // q_l^-1 mod q_{l-1}
+    TW ql[64];             // q_l mod q_i
+};
+
+cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st);
+cudaError_t launch_ds_corr(const DsArgs& A, int bc, cudaStream_t st);
 cudaError_t launch_bconv(const BConvTab& T, const BConvIO& io, int N, int batch, cudaStream_t st);
 cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t st);
 cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStream_t st);

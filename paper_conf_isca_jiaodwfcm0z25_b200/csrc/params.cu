@@ -291,6 +291,18 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
         c->moddown[l] = make_bconv(c, pids, qids);
         for (int i = 0; i < l; ++i) c->ql_inv[l].push_back(mk_tw(invm(c->mod[l] % c->mod[i], c->mod[i]), c->mod[i]));
     }
+    c->ds_inv.assign(c->num_q, {});
+    c->ds_ql.assign(c->num_q, {});
+    c->ds_qlinv_m.assign(c->num_q, TW{0, 0});
+    for (int l = 2; l < c->num_q; ++l) {
+        const u64 ql = c->mod[l], qm = c->mod[l - 1];
+        c->ds_qlinv_m[l] = mk_tw(invm(ql % qm, qm), qm);
+        for (int i = 0; i + 1 < l; ++i) {
+            const u64 qi = c->mod[i];
+            c->ds_inv[l].push_back(mk_tw(invm(mulm(ql % qi, qm % qi, qi), qi), qi));
+            c->ds_ql[l].push_back(mk_tw(ql % qi, qi));
+        }
+    }
     // tensor-core BConv tables (used when alpha <= 12 and every conversion has <= 51 targets)
     {
         const char* e = std::getenv("NEO_BCONV");

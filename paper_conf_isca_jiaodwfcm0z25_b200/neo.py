@@ -17,6 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libneo.so")
 
 NEO_OP_KEYSWITCH, NEO_OP_HMULT, NEO_OP_HROT, NEO_OP_RESCALE, NEO_OP_HROT_HOISTED = 0, 1, 2, 3, 4
+NEO_OP_DOUBLE_RESCALE = 5
 _STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM", 4: "NEO_ECUDA",
            5: "NEO_ENCCL", 6: "NEO_ENOPRIME"}
 
@@ -25,9 +26,9 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_evk_destroy", "neo_keyswitch", "neo_hmult", "neo_hrot", "neo_rescale",
             "neo_keyip", "neo_moddown_combine", "neo_evk_create_hoisted", "neo_hrot_hoisted",
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
-            "neo_debug_bconv_trace")
+            "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
-                 "rescale_modswitch", "rescale_combine")
+                 "rescale_modswitch", "rescale_combine", "elementwise")
 
 
 class NeoError(RuntimeError):
@@ -74,8 +75,14 @@ def lib() -> ctypes.CDLL:
             "neo_evk_create_hoisted": [_vp, _vp, _u32, ctypes.POINTER(_vp)],
             "neo_hrot_hoisted": [_vp, ctypes.POINTER(_vp), _i32, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_moddown_combine": [_vp, _vp, _vp, _i32p, _i32, _vp, _i32, _vp],
+            "neo_double_rescale": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+            "neo_pmult": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
+            "neo_hadd": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
+            "neo_padd": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
         }
         for name, args in sig.items():
+            if not hasattr(L, name):        # an older build (A/B runs); tests/test_abi.py requires every symbol
+                continue
             f = getattr(L, name)
             f.argtypes = args
             f.restype = ctypes.c_int
@@ -255,6 +262,26 @@ def neo_hrot(ctx: Context, rotkey: EvalKey, galois_elt: int, ct_in, level: int, 
 def neo_rescale(ctx: Context, ct_in, level: int, ct_out, batch: int, ws, stream=None):
     _check(lib().neo_rescale(ctx.handle, _ptr(ct_in), level, _ptr(ct_out), batch, _ptr(ws), ws.numel() * 8,
                              _stream(stream)), "neo_rescale")
+
+
+def neo_double_rescale(ctx: Context, ct_in, level: int, ct_out, batch: int, ws, stream=None):
+    _check(lib().neo_double_rescale(ctx.handle, _ptr(ct_in), level, _ptr(ct_out), batch, _ptr(ws),
+                                    ws.numel() * 8, _stream(stream)), "neo_double_rescale")
+
+
+def neo_pmult(ctx: Context, ct_in, pt, level: int, ct_out, batch: int, stream=None):
+    _check(lib().neo_pmult(ctx.handle, _ptr(ct_in), _ptr(pt), level, _ptr(ct_out), batch, _stream(stream)),
+           "neo_pmult")
+
+
+def neo_hadd(ctx: Context, ct_a, ct_b, level: int, ct_out, batch: int, stream=None):
+    _check(lib().neo_hadd(ctx.handle, _ptr(ct_a), _ptr(ct_b), level, _ptr(ct_out), batch, _stream(stream)),
+           "neo_hadd")
+
+
+def neo_padd(ctx: Context, ct_in, pt, level: int, ct_out, batch: int, stream=None):
+    _check(lib().neo_padd(ctx.handle, _ptr(ct_in), _ptr(pt), level, _ptr(ct_out), batch, _stream(stream)),
+           "neo_padd")
 
 
 def neo_keyip(ctx: Context, evk: EvalKey, dhat, limb_ids, beta: int, acc, batch: int, stream=None):
