@@ -161,7 +161,7 @@ def bytes_model(batch: int, l: int = LEVEL) -> dict:
     bconv = batch * 2 * ((Lq + up) + (2 * P + 2 * Lq))
     keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E * 5 / 8)          # key stored in 5 bytes per residue
     tensor = batch * 7 * Lq
-    auto = batch * 4 * Lq
+    auto = 0                     # AUTO is fused into the HRot INTT, KeyIP and ModDown-tail reads
     out = {"ntt_col": ntt_col, "ntt_row": ntt_row, "bconv": bconv, "keyip": keyip, "combine": 0,
            "tensor": tensor, "automorphism": auto, "rescale_modswitch": 0, "rescale_combine": 0, "elementwise": 0}
     return {k: v * limb for k, v in out.items()}

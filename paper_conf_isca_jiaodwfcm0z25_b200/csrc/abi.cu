@@ -89,7 +89,7 @@ struct ProfScope {
 static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long src_bs, const int* src_off,
                            u64* dst, long long dst_bs, const int* dst_off, const int* prime, int n, u64* tmp,
                            int batch, cudaStream_t st, const RowEpi* epi = nullptr, bool in_lazy = false,
-                           const TWD* scale = nullptr) {
+                           const TWD* scale = nullptr, unsigned galois = 0) {
     if (n <= 0) return NEO_OK;
     if (n > NEO_MAX_ROWS) FAIL(NEO_EUNSUPPORTED, "too many limb rows in one transform");
     RowSet a, b;
@@ -99,6 +99,15 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
     a.has_scale = 0;
     b.in_lazy = 0;
     b.has_scale = (!fwd && scale) ? 1 : 0;
+    // inverse transform of sigma_g(src): the automorphism is folded into the first (row) pass
+    a.galois = b.galois = 0;
+    a.galois_inv_n1 = b.galois_inv_n1 = 0;
+    if (galois && !fwd) {
+        a.galois = galois;
+        unsigned gi = galois;                 // g^-1 mod 2^32 by Newton: g g = 1 mod 8 and every
+        for (int it = 0; it < 4; ++it) gi *= 2u - galois * gi;   // x <- x (2 - g x) doubles the bits
+        a.galois_inv_n1 = gi & (unsigned)(c->ntt.N1 - 1);
+    }
     if (b.has_scale)
         for (int k = 0; k < n; ++k) b.scale[k] = scale[k];
     // first pass: src -> tmp ; second pass: tmp -> dst
@@ -152,7 +161,7 @@ static size_t ds_ws(const neo_ctx* c, int l, int B) {
 // ------------------------------------------------------------------ key-switch core
 // a3-a5: ModUp of d (INTT, BConv of every digit onto PQ_l, NTT) into the workspace.
 static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l, int B, u64* ws, const KsLayout& Ly,
-                           cudaStream_t st) {
+                           cudaStream_t st, unsigned galois = 0) {
     const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l);
     u64 *y = ws + Ly.y, *up = ws + Ly.up, *tmp = ws + Ly.tmp;
     int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
@@ -167,7 +176,7 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
             for (int j = 0; j < beta; ++j)
                 for (size_t u = 0; u < c->digits[l][j].size(); ++u) sc[c->digits[l][j][u]] = c->modup_tc[l][j].qhat_inv[u];
         if ((s = ntt_rows(c, false, d, d_bs, so, y, (long long)Lq * N, dof, pr, Lq, tmp, B, st, nullptr, false,
-                          c->use_tc ? sc : nullptr)))
+                          c->use_tc ? sc : nullptr, galois)))
             return s;
     }
 
@@ -229,7 +238,8 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
 // a6-a10: KeyIP of the ModUp outputs (and d's own digit limbs) with key k, ModDown, combine.
 static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
                             u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
-                            const u64* add0, const u64* add1, long long add_bs, cudaStream_t st) {
+                            const u64* add0, const u64* add1, long long add_bs, cudaStream_t st,
+                            unsigned galois = 0) {
     const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p;
     u64 *up = ws + Ly.up, *acc = ws + Ly.acc, *conv = ws + Ly.conv, *pc = ws + Ly.pc, *tmp = ws + Ly.tmp;
     int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
@@ -244,6 +254,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         A.acc_bstride = (long long)2 * E * N;
         A.acc_cstride = (long long)E * N;
         A.N = N; A.beta = beta; A.evk_limbs = c->num_q + c->num_p;
+        A.galois = galois;                     // d's own digit limbs are read as sigma_g(d)
         for (int pos = 0; pos < E; ++pos) {
             int id = c->ext_id(l, pos);
             A.limb[pos] = id;
@@ -296,6 +307,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         ep.acc_c = (long long)E * N;
         ep.add0 = add0; ep.add1 = add1; ep.add_b = add_bs;
         ep.out0 = out0; ep.out1 = out1; ep.out_b = out_bs;
+        ep.add_galois = galois;                // add0 is gathered through sigma_g
         for (int i = 0; i < Lq; ++i) ep.pinv[i] = c->pinv[i];
         if ((s = ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st,
                           &ep, c->use_tc)))
@@ -306,10 +318,11 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
 
 static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
                           u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
-                          const u64* add0, const u64* add1, long long add_bs, cudaStream_t st) {
-    neo_status s = ks_modup(c, d, d_bs, l, B, ws, Ly, st);
+                          const u64* add0, const u64* add1, long long add_bs, cudaStream_t st,
+                          unsigned galois = 0) {
+    neo_status s = ks_modup(c, d, d_bs, l, B, ws, Ly, st, galois);
     if (s) return s;
-    return ks_finish(c, k, d, d_bs, l, B, ws, Ly, out0, out1, out_bs, add0, add1, add_bs, st);
+    return ks_finish(c, k, d, d_bs, l, B, ws, Ly, out0, out1, out_bs, add0, add1, add_bs, st, galois);
 }
 
 // ------------------------------------------------------------------ validation helpers
@@ -660,11 +673,12 @@ neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint6
     TRY(check_ws(c, NEO_OP_HROT, level, batch, ws, ws_bytes));
     KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HROT);
     u64* w = static_cast<u64*>(ws);
-    u64* sc = w + Ly.extra;
     const long long ls = (long long)(level + 1) * c->N;
     cudaStream_t s = S(st);
-    LAUNCH(PK_AUTO, s, launch_automorph(ct_in, sc, g, c->N, 2 * (level + 1) * batch, s));
-    return ks_core(c, rk, sc + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, sc, nullptr, 2 * ls, s);
+    // AUTO fused into its consumers: the INTT's row pass and KeyIP read
+    // sigma_g(c1), the ModDown tail reads sigma_g(c0), each through the index map
+    return ks_core(c, rk, ct_in + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, ct_in, nullptr,
+                   2 * ls, s, g);
 }
 
 neo_status neo_hrot_hoisted(const neo_ctx* c, const neo_evk* const* keys, int32_t n_rot, const uint64_t* ct_in,
@@ -707,6 +721,7 @@ neo_status neo_keyip(const neo_ctx* c, const neo_evk* k, const uint64_t* dhat, c
     if (beta < 1 || beta > c->dnum) FAIL(NEO_EINVAL, "beta must be in [1, dnum]");
     if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
     KeyIPArgs A;
+    A.galois = 0;
     A.d = dhat; A.up = dhat; A.evk_lo = k->lo; A.evk_hi = k->hi; A.acc = acc; A.mods = c->d_mods;
     A.d_bstride = A.up_bstride = (long long)beta * n * c->N;
     A.acc_bstride = (long long)2 * n * c->N;
@@ -776,6 +791,7 @@ neo_status neo_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, u
     ep.acc_c = (long long)(l + 1) * N;
     ep.add0 = ep.add1 = nullptr;
     ep.add_b = 0;
+    ep.add_galois = 0;
     ep.out0 = ct_out;
     ep.out1 = ct_out + (size_t)l * N;
     ep.out_b = (long long)2 * l * N;
@@ -845,6 +861,7 @@ neo_status neo_double_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t l
     ep.acc_c = (long long)(l + 1) * N;
     ep.add0 = ep.add1 = nullptr;
     ep.add_b = 0;
+    ep.add_galois = 0;
     ep.out0 = ct_out;
     ep.out1 = ct_out + (size_t)(l - 1) * N;
     ep.out_b = (long long)2 * (l - 1) * N;

@@ -134,6 +134,8 @@ struct RowSet {
     int n;                                 // rows per batch entry
     int in_lazy;                           // forward column pass: src holds lazy doubles |x| < 2^40
     int has_scale;                         // inverse column pass: multiply row k by scale[k]
+    unsigned galois;                       // inverse row pass: read sigma_g(src) (X -> X^g, NTT domain); 0 = none
+    unsigned galois_inv_n1;                //   g^-1 mod N1
     int src_off[NEO_MAX_ROWS];
     int dst_off[NEO_MAX_ROWS];
     short prime[NEO_MAX_ROWS];

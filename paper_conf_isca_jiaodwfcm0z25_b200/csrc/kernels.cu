@@ -66,7 +66,9 @@ __device__ __forceinline__ void keyip_body(const KeyIPArgs& A, int n, int t, int
         e0[j] = (u64)A.evk_lo[o0] | ((u64)A.evk_hi[o0] << 32);
         e1[j] = (u64)A.evk_lo[o1] | ((u64)A.evk_hi[o1] << 32);
         const bool up = A.src_kind[j][t];
-        src[j] = (up ? A.up : A.d) + (size_t)A.src_off[j][t] * A.N + n;
+        const unsigned nn = (up || !A.galois) ? (unsigned)n      // sigma_g gather (fused HROTATE AUTO)
+                            : (unsigned)(((unsigned long long)A.galois * n + (A.galois - 1) / 2) & (A.N - 1));
+        src[j] = (up ? A.up : A.d) + (size_t)A.src_off[j][t] * A.N + nn;
         sb[j] = up ? A.up_bstride : A.d_bstride;
     }
     u64* acc = A.acc + (size_t)t * A.N + n;

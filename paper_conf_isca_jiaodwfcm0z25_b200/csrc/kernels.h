@@ -16,6 +16,7 @@ struct KeyIPArgs {
     const ModQ* mods;
     long long d_bstride, up_bstride, acc_bstride, acc_cstride;
     int N, beta, evk_limbs;
+    unsigned galois;                         // != 0: rows of kind 0 (d) are read as sigma_g(d)
     int limb[KS_MAX_EXT];                    // position -> limb id
     unsigned char src_kind[KS_MAX_BETA][KS_MAX_EXT];   // 0: d, 1: up
     int src_off[KS_MAX_BETA][KS_MAX_EXT];    // row (in N units) inside the chosen buffer

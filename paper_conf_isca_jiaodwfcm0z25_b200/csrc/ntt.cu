@@ -326,7 +326,8 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
             const u64* addr = cc ? ep.add1 : ep.add0;
             for (int i2 = tid; i2 < N2; i2 += NT) {
                 pf_l2(accr + (size_t)N1 * i2);
-                if (addr) pf_l2(addr + bb * ep.add_b + (size_t)k * a.N + row0 + (size_t)N1 * i2);
+                if (addr && !(cc == 0 && ep.add_galois))
+                    pf_l2(addr + bb * ep.add_b + (size_t)k * a.N + row0 + (size_t)N1 * i2);
             }
         } else if (STAGES == 1) {
             const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N;
@@ -398,17 +399,39 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                     u64 r0 = shoup(sub_mod(((u64)av.y << 32) | av.x, ((u64)v.y << 32) | v.x, qq), pinv, qq);
                     u64 r1 = shoup(sub_mod(((u64)av.w << 32) | av.z, ((u64)v.w << 32) | v.z, qq), pinv, qq);
                     if (addr) {
-                        const uint4 dv = *reinterpret_cast<const uint4*>(addr + pos);
-                        r0 = add_mod(r0, ((u64)dv.y << 32) | dv.x, qq);
-                        r1 = add_mod(r1, ((u64)dv.w << 32) | dv.z, qq);
+                        if (cc == 0 && ep.add_galois) {        // sigma_g(c0) of HROTATE, gathered
+                            const unsigned gg = ep.add_galois, msk = (unsigned)a.N - 1;
+                            const unsigned s0 = (unsigned)(((unsigned long long)gg * pos + (gg - 1) / 2) & msk);
+                            r0 = add_mod(r0, addr[s0], qq);
+                            r1 = add_mod(r1, addr[(s0 + gg) & msk], qq);
+                        } else {
+                            const uint4 dv = *reinterpret_cast<const uint4*>(addr + pos);
+                            r0 = add_mod(r0, ((u64)dv.y << 32) | dv.x, qq);
+                            r1 = add_mod(r1, ((u64)dv.w << 32) | dv.z, qq);
+                        }
                     }
                     *reinterpret_cast<uint4*>(outr + pos) = make_uint4((unsigned)r0, (unsigned)(r0 >> 32), (unsigned)r1, (unsigned)(r1 >> 32));
                 }
             }
         } else {
             const u64* T = reinterpret_cast<const u64*>(sD);
+            int i1o = i1;                                  // row of tmp this thread's row lands in
+            if (rs.galois) {
+                // fused automorphism X -> X^g (HROTATE): output index i1o + N1 i2 reads source
+                // index pi = g (i1o + N1 i2) + (g-1)/2 mod N = i1 + N1 ((kk + g i2) mod N2), with
+                // i1 = (g i1o + (g-1)/2) mod N1 the source row this tile holds and kk = floor(s / N1)
+                const unsigned g = rs.galois, cst = (g - 1) / 2;
+                const unsigned ginv = rs.galois_inv_n1;
+                i1o = (int)((ginv * (unsigned)(i1 + N1 - (int)(cst & (unsigned)(N1 - 1)))) & (unsigned)(N1 - 1));
+                const unsigned s0 = (unsigned)(((unsigned long long)g * (unsigned)i1o + cst) & (unsigned long long)(a.N - 1));
+                const unsigned kk = s0 / (unsigned)N1;
 #pragma unroll
-            for (int ib = 0; ib < R; ++ib) x[ib] = u2d(T[swz(r + R * ib, rho)]);
+                for (int ib = 0; ib < R; ++ib)
+                    x[ib] = u2d(T[swz((int)((kk + g * (unsigned)(r + R * ib)) & (unsigned)(N2 - 1)), rho)]);
+            } else {
+#pragma unroll
+                for (int ib = 0; ib < R; ++ib) x[ib] = u2d(T[swz(r + R * ib, rho)]);
+            }
             cyc_dif<R>(x, CYC, q);
             __syncthreads();
 #pragma unroll
@@ -419,7 +442,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
             cyc_dif<R>(x, CYC, q);
             double* dd = reinterpret_cast<double*>(dst);
 #pragma unroll
-            for (int na = 0; na < R; ++na) dd[(size_t)i1 * N2 + R * na + r] = x[BitRev<R>::of(na)];
+            for (int na = 0; na < R; ++na) dd[(size_t)i1o * N2 + R * na + r] = x[BitRev<R>::of(na)];
         }
         __syncthreads();
         issue(t + STAGES * G, s);

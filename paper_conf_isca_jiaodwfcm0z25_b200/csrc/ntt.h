@@ -26,6 +26,7 @@ struct RowEpi {
     u64* out0;
     u64* out1;
     long long out_b;
+    unsigned add_galois;  // != 0: the addend of component 0 is sigma_g(add0), gathered on the fly
     TW pinv[64];          // per row k
 };
 
