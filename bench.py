@@ -47,6 +47,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-hoisted", action="store_true")
+    ap.add_argument("--batch-hrot", type=int, default=256,
+                    help="BASELINE configs[2]: this many independent HRot key-switches (one shared key) "
+                         "split data-parallel over the ranks, plus a batch sweep up to it (0 = skip)")
     ap.add_argument("--streams", type=int, default=2, choices=[1, 2],
                     help="2: HRot runs on a second CUDA stream, overlapping HMult+Rescale")
     ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
@@ -161,7 +164,7 @@ def bytes_model(batch: int, l: int = LEVEL) -> dict:
     bconv = batch * 2 * ((Lq + up) + (2 * P + 2 * Lq))
     keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E * 5 / 8)          # key stored in 5 bytes per residue
     tensor = batch * 7 * Lq
-    auto = 0                     # AUTO is fused into the HRot INTT, KeyIP and ModDown-tail reads
+    auto = batch * 2 * Lq         # AUTO of c0 only (c1 is read through the index map by the INTT and KeyIP)
     out = {"ntt_col": ntt_col, "ntt_row": ntt_row, "bconv": bconv, "keyip": keyip, "combine": 0,
            "tensor": tensor, "automorphism": auto, "rescale_modswitch": 0, "rescale_combine": 0, "elementwise": 0}
     return {k: v * limb for k, v in out.items()}
@@ -410,6 +413,50 @@ def run_neo(args):
                    "ms_per_call": hms, "note": "neo_hrot_hoisted, one stream, Set-B l=35"}
         del hk
 
+    # BASELINE configs[2]: a batch of `batch_hrot` independent HRot(g=5)
+    # key-switches sharing one rotation key, split data-parallel over the ranks (weak per-rank
+    # shard, no collective), plus the Fig. 17 analogue: the same call at smaller batches.
+    # Timing is data-independent; inputs are uniform residues < 2^35 (< every 36-bit q), made
+    # on the device.
+    batch_block = None
+    if args.batch_hrot > 0:
+        Bg = args.batch_hrot
+        Bl = max(1, Bg // world)
+        gen = torch.Generator(device="cuda")
+        gen.manual_seed(seed + 77)
+        big_in = torch.randint(0, 1 << 35, (Bl, 2, Lq, N), dtype=torch.int64, device="cuda",
+                               generator=gen).view(torch.uint64)
+        big_out = torch.empty_like(big_in)
+        big_ws = torch.empty(ctx.workspace_size(neo.NEO_OP_HROT, LEVEL, Bl) // 8, dtype=torch.uint64, device="cuda")
+        sweep = []
+        sizes = sorted({b for b in (8, 16, 32, 64, 128) if b < Bl} | {Bl})
+        for bs in sizes:
+            neo.neo_hrot(ctx, rot, g, big_in[:bs], LEVEL, big_out[:bs], bs, big_ws)          # warm-up
+            torch.cuda.synchronize()
+            barrier()
+            reps = 3
+            b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            b0.record()
+            for _ in range(reps):
+                neo.neo_hrot(ctx, rot, g, big_in[:bs], LEVEL, big_out[:bs], bs, big_ws)
+            b1.record()
+            torch.cuda.synchronize()
+            bms = b0.elapsed_time(b1) / reps
+            if world > 1:
+                t = torch.tensor([bms], dtype=torch.float64, device="cuda")
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                bms = float(t.item())
+            sweep.append({"batch_per_gpu": bs, "ms_per_call": round(bms, 4),
+                          "value": bs * world / (bms / 1e3)})
+        last = sweep[-1]
+        batch_block = {"config": "BASELINE configs[2]: N=2^16, L=35, dnum=3, batch of independent HRot "
+                                 "key-switches (one shared key), data-parallel over the GPUs",
+                       "global_batch": Bl * world, "batch_per_gpu": Bl, "value": last["value"], "unit": "HRot/s",
+                       "ms_per_call": last["ms_per_call"], "sweep": sweep,
+                       "timing": "CUDA events around 3 neo_hrot calls per size after 1 warm-up, max over ranks"}
+        del big_in, big_out, big_ws
+        torch.cuda.empty_cache()
+
     # end-to-end through the public API with pinned host buffers: every step copies its three
     # input ciphertexts host->device and both results device->host.  Copies run on their own
     # streams, double-buffered, so the H2D of step k+1 and the D2H of step k-1 overlap the
@@ -492,6 +539,7 @@ def run_neo(args):
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted,
+                "batch_hrot": batch_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}
         print(json.dumps(line), flush=True)

@@ -142,7 +142,8 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
     L.tmp = o; o += B * std::max(std::max(beta * E, 2 * Lq), 2 * P) * N;
     L.extra = o;
     if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
-    if (op == NEO_OP_HROT || op == NEO_OP_HROT_HOISTED) o += B * 2 * Lq * N;
+    if (op == NEO_OP_HROT) o += B * Lq * N;                       // sigma_g(c0)
+    if (op == NEO_OP_HROT_HOISTED) o += B * 2 * Lq * N;
     L.total = o;
     return L;
 }
@@ -239,7 +240,7 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
 static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
                             u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
                             const u64* add0, const u64* add1, long long add_bs, cudaStream_t st,
-                            unsigned galois = 0) {
+                            unsigned galois = 0, bool add_galois = true) {
     const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p;
     u64 *up = ws + Ly.up, *acc = ws + Ly.acc, *conv = ws + Ly.conv, *pc = ws + Ly.pc, *tmp = ws + Ly.tmp;
     int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
@@ -307,7 +308,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         ep.acc_c = (long long)E * N;
         ep.add0 = add0; ep.add1 = add1; ep.add_b = add_bs;
         ep.out0 = out0; ep.out1 = out1; ep.out_b = out_bs;
-        ep.add_galois = galois;                // add0 is gathered through sigma_g
+        ep.add_galois = add_galois ? galois : 0;   // add0 gathered through sigma_g
         for (int i = 0; i < Lq; ++i) ep.pinv[i] = c->pinv[i];
         if ((s = ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st,
                           &ep, c->use_tc)))
@@ -319,10 +320,10 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
 static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
                           u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
                           const u64* add0, const u64* add1, long long add_bs, cudaStream_t st,
-                          unsigned galois = 0) {
+                          unsigned galois = 0, bool add_galois = true) {
     neo_status s = ks_modup(c, d, d_bs, l, B, ws, Ly, st, galois);
     if (s) return s;
-    return ks_finish(c, k, d, d_bs, l, B, ws, Ly, out0, out1, out_bs, add0, add1, add_bs, st, galois);
+    return ks_finish(c, k, d, d_bs, l, B, ws, Ly, out0, out1, out_bs, add0, add1, add_bs, st, galois, add_galois);
 }
 
 // ------------------------------------------------------------------ validation helpers
@@ -673,12 +674,16 @@ neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint6
     TRY(check_ws(c, NEO_OP_HROT, level, batch, ws, ws_bytes));
     KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HROT);
     u64* w = static_cast<u64*>(ws);
+    u64* sc0 = w + Ly.extra;                               // [B][l+1][N]: sigma_g(c0)
     const long long ls = (long long)(level + 1) * c->N;
     cudaStream_t s = S(st);
-    // AUTO fused into its consumers: the INTT's row pass and KeyIP read
-    // sigma_g(c1), the ModDown tail reads sigma_g(c0), each through the index map
-    return ks_core(c, rk, ct_in + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, ct_in, nullptr,
-                   2 * ls, s, g);
+    // AUTO on c1 is fused into its consumers: the INTT's row pass and KeyIP
+    // read sigma_g(c1) through the index map.  sigma_g(c0) is permuted by its own (streaming)
+    // launch up front: the ModDown tail then reads it with 16-byte loads instead of 8-byte
+    // gathers, which measured faster when HROTATE overlaps another key-switch
+    LAUNCH(PK_AUTO, s, launch_automorph(ct_in, sc0, g, c->N, level + 1, s, batch, 2 * ls, ls));
+    return ks_core(c, rk, ct_in + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, sc0, nullptr,
+                   ls, s, g, /*add_galois=*/false);
 }
 
 neo_status neo_hrot_hoisted(const neo_ctx* c, const neo_evk* const* keys, int32_t n_rot, const uint64_t* ct_in,

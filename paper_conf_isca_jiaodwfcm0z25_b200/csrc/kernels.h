@@ -74,7 +74,8 @@ cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t 
 cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStream_t st);
 cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, int limbs, int N, int batch,
                           cudaStream_t st);
-cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st);
+cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st, int batch = 1,
+                             long long in_bs = 0, long long out_bs = 0);
 cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st);
 cudaError_t launch_rescale_combine(const RescaleArgs& A, int bc, cudaStream_t st);
 cudaError_t launch_pack5(const u64* in, uint32_t* lo, uint8_t* hi, size_t n, cudaStream_t st);
