@@ -47,6 +47,7 @@ def lib():
             getattr(L, name).argtypes = [_U64P, _U64P, _U64P, i64, u64]
         L.or_vec_scalar_mulmod.argtypes = [_U64P, u64, _U64P, i64, u64]
         L.or_vec_mod.argtypes = [_U64P, _U64P, i64, u64]
+        L.or_crt_exact.argtypes = [_U64P, _U64P, _U64P, i32, _U64P, _U64P, i32, _U64P, i32, _U64P, i32, i32]
         L.or_num_threads.restype = i32
         _lib = L
     return _lib

@@ -20,6 +20,9 @@
  *   or_bconv                  Algorithm 1 (L296-319), literally: for i, for j, for coeff:
  *                             out_j += (c_i * qhat_i^-1 mod q_i) * qhat_i mod p_j.
  *   or_vec_*                  element-wise ModMUL / ModADD (L268, L456).
+ *   or_crt_exact              EXACT basis conversion by multi-word big-integer CRT (KLSS key
+ *                             decomposition and Recover Limbs, L155-180): x = sum_i y_i qhat_i
+ *                             mod Q in [0, Q) (optionally centred to (-Q/2, Q/2]), then x mod t.
  */
 #include <stdint.h>
 #include <stdlib.h>
@@ -185,6 +188,78 @@ void or_vec_scalar_mulmod(const u64 *a, u64 s, u64 *out, long n, u64 q) {
 void or_vec_mod(const u64 *a, u64 *out, long n, u64 q) {
 #pragma omp parallel for schedule(static)
     for (long k = 0; k < n; ++k) out[k] = a[k] % q;
+}
+
+/* ---------------------------------------------------------------- exact CRT (big integers) */
+
+/* Little-endian multi-word naturals of W <= 8 64-bit words. */
+#define CRT_MAXW 8
+
+static int mw_ge(const u64 *a, const u64 *b, int W) {         /* a >= b */
+    for (int w = W - 1; w >= 0; --w)
+        if (a[w] != b[w]) return a[w] > b[w];
+    return 1;
+}
+static void mw_sub(u64 *a, const u64 *b, int W) {              /* a -= b (a >= b) */
+    u64 borrow = 0;
+    for (int w = 0; w < W; ++w) {
+        u128 d = (u128)a[w] - b[w] - borrow;
+        a[w] = (u64)d;
+        borrow = (u64)(d >> 64) ? 1 : 0;
+    }
+}
+static u64 mw_mod(const u64 *a, int W, u64 t) {                /* a mod t, Horner over words */
+    u128 r = 0;
+    for (int w = W - 1; w >= 0; --w) r = ((r << 64) | a[w]) % t;
+    return (u64)r;
+}
+
+/* in[n_in][n]: residues c_i mod q_i; qhat_inv[i] = (Q/q_i)^-1 mod q_i; qhat[n_in][W] and Q[W]
+ * as W-word naturals (n_in * Q < 2^(64 W)); t[n_out].  For every coefficient:
+ *   y_i = c_i qhat_inv_i mod q_i,  x = sum_i y_i qhat_i  (exact),  x -= Q while x >= Q,
+ *   centred: x > Q/2 -> x - Q (negative);   out[j] = x mod t_j.
+ * This is the definition of the CRT lift (no floating point, no approximation). */
+void or_crt_exact(const u64 *in, const u64 *q, const u64 *qhat_inv, int n_in, const u64 *qhat,
+                  const u64 *Q, int W, const u64 *t, int n_out, u64 *out, int n, int centred) {
+#pragma omp parallel for schedule(static)
+    for (int k = 0; k < n; ++k) {
+        u64 acc[CRT_MAXW + 1] = {0};
+        for (int i = 0; i < n_in; ++i) {
+            const u64 y = mulmod(in[(size_t)i * n + k], qhat_inv[i], q[i]);
+            u64 carry = 0;
+            for (int w = 0; w < W; ++w) {
+                u128 v = (u128)y * qhat[(size_t)i * W + w] + acc[w] + carry;
+                acc[w] = (u64)v;
+                carry = (u64)(v >> 64);
+            }
+            acc[W] += carry;
+        }
+        u64 Qe[CRT_MAXW + 1];                                  /* Q as W + 1 words */
+        for (int w = 0; w < W; ++w) Qe[w] = Q[w];
+        Qe[W] = 0;
+        while (mw_ge(acc, Qe, W + 1)) mw_sub(acc, Qe, W + 1);  /* at most n_in subtractions */
+        int neg = 0;
+        if (centred) {                                         /* 2 x > Q  ->  x - Q */
+            u64 twice[CRT_MAXW + 1];
+            u64 c = 0;
+            for (int w = 0; w < W; ++w) {
+                twice[w] = (acc[w] << 1) | c;
+                c = acc[w] >> 63;
+            }
+            twice[W] = c;
+            if (!mw_ge(Qe, twice, W + 1)) {                    /* Q < 2x */
+                u64 m[CRT_MAXW];
+                for (int w = 0; w < W; ++w) m[w] = Q[w];
+                mw_sub(m, acc, W);                             /* |x - Q| = Q - x */
+                for (int w = 0; w < W; ++w) acc[w] = m[w];
+                neg = 1;
+            }
+        }
+        for (int j = 0; j < n_out; ++j) {
+            const u64 r = mw_mod(acc, W, t[j]);
+            out[(size_t)j * n + k] = (neg && r) ? t[j] - r : r;
+        }
+    }
 }
 
 int or_num_threads(void) {
