@@ -68,6 +68,10 @@ typedef struct {
     int32_t log_n, num_q, num_p, dnum, word_bits, device;
     const uint64_t* q;
     const uint64_t* p;
+    int32_t alpha_t;     /* KLSS key-decomposition group size alpha~ (Table 4); 0 = Hybrid only.
+                          * > 0 adds alpha' T primes (WordSize_T = word_bits, the Z4 rule continued
+                          * after p; alpha' from Eq. 4, reading K3) and the KLSS
+                          * tables; requires generated primes (q = p = NULL). */
 } neo_params_desc;
 
 /* Build the context: primes, psi, NTT twiddle tables, BConv tables for every
@@ -78,6 +82,10 @@ neo_status neo_params_destroy(neo_ctx* ctx);
 /* Copy the moduli and psi to host arrays (any may be NULL): q[num_q], p[num_p],
  * psi[num_q+num_p] (psi indexed by limb id). */
 neo_status neo_params_query(const neo_ctx* ctx, uint64_t* q, uint64_t* p, uint64_t* psi);
+
+/* KLSS extras of the context: alpha~, alpha' (number of T primes) and the T primes (host array
+ * of alpha' entries, may be NULL).  T limb ids are num_q+num_p .. num_q+num_p+alpha'-1. */
+neo_status neo_klss_query(const neo_ctx* ctx, int32_t* alpha_t, int32_t* alpha_p, uint64_t* t);
 
 /* Bytes of device workspace `ws` the caller must pass to op (NEO_OP_*) at this level
  * and batch; 0 on invalid arguments. */
@@ -119,6 +127,17 @@ neo_status neo_automorphism(const neo_ctx* ctx, const uint64_t* in, int32_t n_li
  * free its copy after return.  Synchronises the current device. */
 neo_status neo_evk_create(const neo_ctx* ctx, const uint64_t* evk, neo_evk** out);
 neo_status neo_evk_destroy(neo_evk* evk);
+
+/* KLSS evaluation key (L155-180, Alg. 3/4; readings K1-K6 in DESIGN.md): ekey is a DEVICE array
+ * [2][beta~][dnum][alpha'][N], NTT form over the T primes, ekey[c][i][j] = the Hybrid key
+ * component evk_{j,c} reduced modulo the group modulus P~_i (group i = limbs i*alpha~ ..
+ * of q_0..q_L, p_0..p_K).  Re-laid out to 5 bytes per residue; the caller may free its copy.
+ * neo_keyswitch / neo_hmult / neo_hrot given a KLSS key run the KLSS method:
+ *   INTT -> ModUp BConv to T (alpha' limbs) -> NTT over T -> IP (beta x beta~) -> INTT over T
+ *   -> Recover Limbs (exact centred CRT from T) -> ModDown -> NTT,
+ * whose output equals the Hybrid method's for the key it was derived from (reading K4).
+ * Needs a context created with alpha_t > 0. */
+neo_status neo_evk_create_klss(const neo_ctx* ctx, const uint64_t* ekey, neo_evk** out);
 
 /* Hybrid key-switch (Table 2, Eq. 2, Fig. 5) at `level`:
  *   INTT -> ModUp BConv (per digit) -> NTT -> KeyIP -> INTT(P part) -> ModDown BConv

@@ -9,6 +9,7 @@
 #include "bconv_tc.h"
 #include "context.h"
 #include "kernels.h"
+#include "klss.h"
 #include "ntt.h"
 
 namespace neo {
@@ -147,6 +148,10 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
     L.total = o;
     return L;
 }
+
+static size_t klss_total(const neo_ctx* c, int l, int B, int op);
+// offset (u64 words) of the op's extra buffers (tensor output d, sigma_g(c0)) in the workspace
+static size_t extra_offset(const neo_ctx* c, const neo_evk* k, int l, int B, int op);
 
 static size_t rescale_ws(const neo_ctx* c, int l, int B) {
     const size_t N = c->N;
@@ -317,10 +322,182 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     return NEO_OK;
 }
 
+// ------------------------------------------------------------------ KLSS key-switch
+// Workspace: y [B][Lq], up [B][beta][alpha'] (T basis), accT [B][2][beta~][alpha'],
+// rec [B][2][E] (PQ_l, coefficient form), conv [2B][Lq], diff [2B][Lq], NTT intermediate.
+struct KlssLayout {
+    size_t y, up, acc, rec, conv, diff, tmp, extra, total;
+};
+
+static KlssLayout klss_layout(const neo_ctx* c, int l, int B, int op) {
+    const size_t N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), ap = c->num_t,
+                 bt = c->klss_groups.size();
+    KlssLayout L;
+    size_t o = 0;
+    L.y = o; o += B * Lq * N;
+    L.up = o; o += B * beta * ap * N;
+    L.acc = o; o += B * 2 * bt * ap * N;
+    L.rec = o; o += B * 2 * E * N;
+    L.conv = o; o += B * 2 * Lq * N;
+    L.diff = o; o += B * 2 * Lq * N;
+    L.tmp = o; o += B * std::max(std::max(beta * ap, 2 * bt * ap), 2 * Lq) * N;
+    L.extra = o;
+    if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
+    if (op == NEO_OP_HROT) o += B * Lq * N;
+    L.total = o;
+    return L;
+}
+
+static size_t klss_total(const neo_ctx* c, int l, int B, int op) { return klss_layout(c, l, B, op).total; }
+static size_t extra_offset(const neo_ctx* c, const neo_evk* k, int l, int B, int op) {
+    return k->klss ? klss_layout(c, l, B, op).extra : ks_layout(c, l, B, op).extra;
+}
+
+// KLSS (L155-180, Fig. 5): INTT -> ModUp (Eq. 3) -> NTT over T -> IP (Alg. 3/4) -> INTT over T
+// -> Recover Limbs -> ModDown (Table 2) -> NTT; readings K1-K6.
+static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
+                            u64* ws, const KlssLayout& Ly, u64* out0, u64* out1, long long out_bs,
+                            const u64* add0, const u64* add1, long long add_bs, cudaStream_t st, unsigned galois) {
+    const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p, ap = c->num_t;
+    const int bt = (int)c->klss_groups.size(), nl = c->num_q + c->num_p;
+    if (beta > KLSS_MAX_BETA || bt > KLSS_MAX_GROUPS) FAIL(NEO_EUNSUPPORTED, "KLSS: too many digits or groups");
+    u64 *y = ws + Ly.y, *up = ws + Ly.up, *acc = ws + Ly.acc, *rec = ws + Ly.rec, *conv = ws + Ly.conv,
+        *diff = ws + Ly.diff, *tmp = ws + Ly.tmp;
+    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    neo_status s;
+    // 1. INTT of d; Algorithm 2's [c_i qhat_i^-1]_{q_i} folded in (the digits are Hybrid's)
+    for (int i = 0; i < Lq; ++i) { so[i] = i; dof[i] = i; pr[i] = i; }
+    {
+        TWD sc[NEO_MAX_ROWS];
+        if (c->use_tc)
+            for (int j = 0; j < beta; ++j)
+                for (size_t u = 0; u < c->digits[l][j].size(); ++u) sc[c->digits[l][j][u]] = c->klss_up_tc[l][j].qhat_inv[u];
+        if ((s = ntt_rows(c, false, d, d_bs, so, y, (long long)Lq * N, dof, pr, Lq, tmp, B, st, nullptr, false,
+                          c->use_tc ? sc : nullptr, galois)))
+            return s;
+    }
+    // 2. ModUp: every digit -> the alpha' T limbs (Eq. 3, Algorithm 1)
+    {
+        BConvMulti M;
+        M.dbg = nullptr;
+        M.njobs = 0;
+        M.pre_scaled = 1;
+        M.lazy_out = 1;
+        for (int j = 0; j < beta; ++j) {
+            const std::vector<int>& dj = c->digits[l][j];
+            BConvIO io;
+            io.in = y; io.out = up;
+            io.in_bstride = (long long)Lq * N;
+            io.out_bstride = (long long)beta * ap * N;
+            for (size_t i = 0; i < dj.size(); ++i) io.in_off[i] = dj[i];
+            for (int t = 0; t < ap; ++t) io.out_off[t] = j * ap + t;
+            if (c->use_tc) {
+                M.P[M.njobs] = c->klss_up_tc[l][j];
+                M.io[M.njobs] = io;
+                M.bmat[M.njobs] = c->d_bmat + c->klss_up_boff[l][j];
+                if (++M.njobs == 4) {
+                    LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, B, c->num_sms, st));
+                    M.njobs = 0;
+                }
+            } else {
+                LAUNCH(PK_BCONV, st, launch_bconv(c->klss_up[l][j], io, N, B, st));
+            }
+        }
+        if (M.njobs) LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, B, c->num_sms, st));
+    }
+    // 3. NTT over T of the beta * alpha' rows
+    for (int j = 0; j < beta; ++j)
+        for (int t = 0; t < ap; ++t) { so[j * ap + t] = dof[j * ap + t] = j * ap + t; pr[j * ap + t] = nl + t; }
+    if ((s = ntt_rows(c, true, up, (long long)beta * ap * N, so, up, (long long)beta * ap * N, dof, pr, beta * ap, tmp,
+                      B, st, nullptr, c->use_tc)))
+        return s;
+    // 4. IP over T for the groups present at level l
+    KlssIpArgs I;
+    I.up = up; I.key_lo = k->lo; I.key_hi = k->hi; I.acc = acc; I.mods = c->d_mods;
+    I.N = N; I.beta = beta; I.dnum = c->dnum; I.beta_t = bt; I.alpha_p = ap; I.t0 = nl;
+    KlssRecArgs R;
+    R.acc = acc; R.rec = rec; R.tab = c->d_rec; R.mods = c->d_mods;
+    R.N = N; R.alpha_p = ap; R.beta_t = bt; R.t0 = nl; R.E = E;
+    int ng = 0, no = 0;
+    for (int i = 0; i < bt; ++i) {
+        int first = no;
+        for (int id : c->klss_groups[i]) {
+            const bool present = id <= l || id >= c->num_q;
+            if (!present) continue;
+            R.out_id[no] = id;
+            R.out_pos[no] = id <= l ? id : Lq + (id - c->num_q);
+            ++no;
+        }
+        if (no > first) {
+            I.group[ng] = R.group[ng] = i;
+            R.first[ng] = first;
+            ++ng;
+        }
+    }
+    R.first[ng] = no;
+    I.n_groups = R.n_groups = ng;
+    LAUNCH(PK_KEYIP, st, launch_klss_ip(I, B, st));
+    // 5. INTT over T of the 2 * (present groups) * alpha' rows (in place, coefficient form)
+    int nr = 0;
+    for (int cc = 0; cc < 2; ++cc)
+        for (int g = 0; g < ng; ++g)
+            for (int t = 0; t < ap; ++t) {
+                so[nr] = dof[nr] = (cc * bt + I.group[g]) * ap + t;
+                pr[nr] = nl + t;
+                ++nr;
+            }
+    if (nr > NEO_MAX_ROWS) FAIL(NEO_EUNSUPPORTED, "KLSS: too many T rows for one transform");
+    if ((s = ntt_rows(c, false, acc, (long long)2 * bt * ap * N, so, acc, (long long)2 * bt * ap * N, dof, pr, nr,
+                      tmp, B, st)))
+        return s;
+    // 6. Recover Limbs: exact centred CRT from T to the PQ_l limbs (K4)
+    LAUNCH(PK_COMBINE, st, launch_klss_recover(R, B, st));
+    // 7. ModDown BConv P -> Q_l on the recovered (coefficient-form) P limbs, batch 2B
+    {
+        BConvIO io;
+        io.in = rec; io.out = conv;
+        io.in_bstride = (long long)E * N;
+        io.out_bstride = (long long)Lq * N;
+        for (int i = 0; i < P; ++i) io.in_off[i] = Lq + i;
+        for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
+        if (c->use_tc) {                        // canonical u64 out (the difference kernel reads it)
+            BConvMulti M;
+            M.dbg = nullptr;
+            M.njobs = 1;
+            M.pre_scaled = 0;
+            M.lazy_out = 0;
+            M.P[0] = c->moddown_tc[l];
+            M.io[0] = io;
+            M.bmat[0] = c->d_bmat + c->moddown_boff[l];
+            LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, 2 * B, c->num_sms, st));
+        } else {
+            LAUNCH(PK_BCONV, st, launch_bconv(c->moddown[l], io, N, 2 * B, st));
+        }
+    }
+    // 8. (conv - acc_Q) in coefficient form, then 9. its NTT with the tail
+    //    out_c = (0 - NTT(conv - acc_Q)) P^-1 (+ add_c) = NTT((acc_Q - conv) P^-1) (+ add_c)   (K5)
+    KlssDiffArgs D;
+    D.conv = conv; D.rec = rec; D.out = diff; D.mods = c->d_mods;
+    D.N = N; D.Lq = Lq; D.E = E;
+    LAUNCH(PK_COMBINE, st, launch_klss_diff(D, B, st));
+    for (int i = 0; i < Lq; ++i) { so[i] = dof[i] = i; pr[i] = i; }
+    RowEpi ep;
+    ep.acc = nullptr;
+    ep.acc_b = ep.acc_c = 0;
+    ep.add0 = add0; ep.add1 = add1; ep.add_b = add_bs;
+    ep.out0 = out0; ep.out1 = out1; ep.out_b = out_bs;
+    ep.add_galois = 0;
+    for (int i = 0; i < Lq; ++i) ep.pinv[i] = c->pinv[i];
+    return ntt_rows(c, true, diff, (long long)Lq * N, so, diff, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st, &ep);
+}
+
 static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
                           u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
                           const u64* add0, const u64* add1, long long add_bs, cudaStream_t st,
                           unsigned galois = 0, bool add_galois = true) {
+    if (k->klss)           // the key decides the method; c0's automorphism was applied by the caller
+        return klss_core(c, k, d, d_bs, l, B, ws, klss_layout(c, l, B, NEO_OP_KEYSWITCH), out0, out1, out_bs, add0,
+                         add1, add_bs, st, galois);
     neo_status s = ks_modup(c, d, d_bs, l, B, ws, Ly, st, galois);
     if (s) return s;
     return ks_finish(c, k, d, d_bs, l, B, ws, Ly, out0, out1, out_bs, add0, add1, add_bs, st, galois, add_galois);
@@ -404,7 +581,7 @@ neo_status neo_params_create(const neo_params_desc* desc, neo_ctx** out) {
     int alpha = (desc->num_q + desc->dnum - 1) / desc->dnum;
     if ((desc->num_q + alpha - 1) / alpha != desc->dnum) FAIL(NEO_EINVAL, "every digit must be non-empty");
     if (alpha > BC_MAX_IN) FAIL(NEO_EUNSUPPORTED, "alpha must be <= 16");
-    if (desc->dnum > KS_MAX_BETA) FAIL(NEO_EUNSUPPORTED, "dnum must be <= 8");
+    if (desc->dnum > KS_MAX_BETA) FAIL(NEO_EUNSUPPORTED, "dnum must be <= 12");
     if ((desc->q == nullptr) != (desc->p == nullptr)) FAIL(NEO_EINVAL, "give both q and p or neither");
     neo_ctx* c = new (std::nothrow) neo_ctx();
     if (!c) FAIL(NEO_ENOMEM, "host allocation failed");
@@ -436,8 +613,8 @@ neo_status neo_params_destroy(neo_ctx* c) {
 neo_status neo_params_query(const neo_ctx* c, uint64_t* q, uint64_t* p, uint64_t* psi) {
     TRY(check_ctx(c));
     if (q) std::copy(c->mod.begin(), c->mod.begin() + c->num_q, q);
-    if (p) std::copy(c->mod.begin() + c->num_q, c->mod.end(), p);
-    if (psi) std::copy(c->psi.begin(), c->psi.end(), psi);
+    if (p) std::copy(c->mod.begin() + c->num_q, c->mod.begin() + c->num_q + c->num_p, p);
+    if (psi) std::copy(c->psi.begin(), c->psi.begin() + c->num_q + c->num_p, psi);
     return NEO_OK;
 }
 
@@ -447,7 +624,11 @@ size_t neo_workspace_size(const neo_ctx* c, int32_t op, int32_t level, int32_t b
         case NEO_OP_KEYSWITCH:
         case NEO_OP_HMULT:
         case NEO_OP_HROT:
-        case NEO_OP_HROT_HOISTED: return ks_layout(c, level, batch, op).total * sizeof(u64);
+        case NEO_OP_HROT_HOISTED: {
+            size_t w = ks_layout(c, level, batch, op).total;
+            if (c->num_t && op != NEO_OP_HROT_HOISTED) w = std::max(w, klss_total(c, level, batch, op));
+            return w * sizeof(u64);
+        }
         case NEO_OP_RESCALE: return level >= 1 ? rescale_ws(c, level, batch) * sizeof(u64) : 0;
         case NEO_OP_DOUBLE_RESCALE: return level >= 2 ? ds_ws(c, level, batch) * sizeof(u64) : 0;
         default: return 0;
@@ -462,7 +643,7 @@ static neo_status ntt_api(const neo_ctx* c, bool fwd, uint64_t* poly, const int3
     if (!ids || n <= 0 || n > NEO_MAX_ROWS) FAIL(NEO_EINVAL, "need 1 <= n_limbs <= 160 limb ids");
     if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
     for (int k = 0; k < n; ++k)
-        if (ids[k] < 0 || ids[k] >= c->num_q + c->num_p) FAIL(NEO_EINVAL, "unknown limb id");
+        if (ids[k] < 0 || ids[k] >= c->limbs_total()) FAIL(NEO_EINVAL, "unknown limb id");
     size_t need = (size_t)batch * n * c->N * sizeof(u64);
     if (!ws || ws_bytes < need) FAIL(NEO_EINVAL, "ntt workspace must hold batch*n_limbs*N words");
     int off[NEO_MAX_ROWS];
@@ -613,6 +794,38 @@ static neo_status evk_create(const neo_ctx* c, const uint64_t* evk, uint32_t gal
 
 neo_status neo_evk_create(const neo_ctx* c, const uint64_t* evk, neo_evk** out) { return evk_create(c, evk, 0, out); }
 
+neo_status neo_evk_create_klss(const neo_ctx* c, const uint64_t* ekey, neo_evk** out) {
+    TRY(check_ctx(c));
+    if (!c->num_t) FAIL(NEO_EINVAL, "context has no KLSS T primes (create it with alpha_t > 0)");
+    if (!ekey || !out) FAIL(NEO_EINVAL, "null argument");
+    *out = nullptr;
+    neo_evk* k = new (std::nothrow) neo_evk();
+    if (!k) FAIL(NEO_ENOMEM, "host allocation failed");
+    k->ctx = c;
+    k->klss = 1;
+    const size_t n = (size_t)2 * c->klss_groups.size() * c->dnum * c->num_t * c->N;
+    if (cudaMalloc(&k->lo, n * sizeof(uint32_t)) != cudaSuccess || cudaMalloc(&k->hi, n) != cudaSuccess) {
+        neo_evk_destroy(k);
+        FAIL(NEO_ENOMEM, "cudaMalloc of the KLSS key failed");
+    }
+    cudaError_t e = launch_pack5(ekey, k->lo, k->hi, n, nullptr);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) {
+        neo_evk_destroy(k);
+        FAIL(NEO_ECUDA, std::string("KLSS key re-layout failed: ") + cudaGetErrorString(e));
+    }
+    *out = k;
+    return NEO_OK;
+}
+
+neo_status neo_klss_query(const neo_ctx* c, int32_t* alpha_t, int32_t* alpha_p, uint64_t* t) {
+    TRY(check_ctx(c));
+    if (alpha_t) *alpha_t = c->alpha_t;
+    if (alpha_p) *alpha_p = c->num_t;
+    if (t) std::copy(c->mod.begin() + c->num_q + c->num_p, c->mod.end(), t);
+    return NEO_OK;
+}
+
 neo_status neo_evk_create_hoisted(const neo_ctx* c, const uint64_t* evk, uint32_t galois_elt, neo_evk** out) {
     TRY(check_ctx(c));
     if ((galois_elt & 1) == 0 || galois_elt >= 2u * (unsigned)c->N) FAIL(NEO_EINVAL, "galois element must be odd and < 2N");
@@ -637,6 +850,7 @@ neo_status neo_keyswitch(const neo_ctx* c, const neo_evk* k, const uint64_t* d, 
     TRY(check_ptr(out0, "out0"));
     TRY(check_ptr(out1, "out1"));
     TRY(check_ws(c, NEO_OP_KEYSWITCH, level, batch, ws, ws_bytes));
+    if (k->klss && !c->num_t) FAIL(NEO_EINVAL, "KLSS key on a context without T primes");
     KsLayout Ly = ks_layout(c, level, batch, NEO_OP_KEYSWITCH);
     const long long ls = (long long)(level + 1) * c->N;
     return ks_core(c, k, d, ls, level, batch, static_cast<u64*>(ws), Ly, out0, out1, ls, nullptr, nullptr, 0, S(st));
@@ -652,9 +866,10 @@ neo_status neo_hmult(const neo_ctx* c, const neo_evk* relin, const uint64_t* ct_
     TRY(check_ptr(ct_b, "ct_b"));
     TRY(check_ptr(ct_out, "ct_out"));
     TRY(check_ws(c, NEO_OP_HMULT, level, batch, ws, ws_bytes));
+    if (relin->klss && !c->num_t) FAIL(NEO_EINVAL, "KLSS key on a context without T primes");
     KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HMULT);
     u64* w = static_cast<u64*>(ws);
-    u64* dd = w + Ly.extra;
+    u64* dd = w + extra_offset(c, relin, level, batch, NEO_OP_HMULT);
     const long long ls = (long long)(level + 1) * c->N;
     cudaStream_t s = S(st);
     LAUNCH(PK_TENSOR, s, launch_tensor(ct_a, ct_b, dd, c->d_mods, level + 1, c->N, batch, s));
@@ -672,9 +887,10 @@ neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint6
     TRY(check_ptr(ct_out, "ct_out"));
     if ((g & 1) == 0 || g >= 2u * (unsigned)c->N) FAIL(NEO_EINVAL, "galois element must be odd and < 2N");
     TRY(check_ws(c, NEO_OP_HROT, level, batch, ws, ws_bytes));
+    if (rk->klss && !c->num_t) FAIL(NEO_EINVAL, "KLSS key on a context without T primes");
     KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HROT);
     u64* w = static_cast<u64*>(ws);
-    u64* sc0 = w + Ly.extra;                               // [B][l+1][N]: sigma_g(c0)
+    u64* sc0 = w + extra_offset(c, rk, level, batch, NEO_OP_HROT);   // [B][l+1][N]: sigma_g(c0)
     const long long ls = (long long)(level + 1) * c->N;
     cudaStream_t s = S(st);
     // AUTO on c1 is fused into its consumers: the INTT's row pass and KeyIP
@@ -696,7 +912,7 @@ neo_status neo_hrot_hoisted(const neo_ctx* c, const neo_evk* const* keys, int32_
     TRY(check_ptr(ct_out, "ct_out"));
     if (!keys || n_rot < 1) FAIL(NEO_EINVAL, "need n_rot >= 1 hoisted rotation keys");
     for (int r = 0; r < n_rot; ++r)
-        if (!keys[r] || keys[r]->ctx != c || keys[r]->galois == 0)
+        if (!keys[r] || keys[r]->ctx != c || keys[r]->galois == 0 || keys[r]->klss)
             FAIL(NEO_EINVAL, "keys must come from neo_evk_create_hoisted on this context");
     TRY(check_ws(c, NEO_OP_HROT_HOISTED, level, batch, ws, ws_bytes));
     KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HROT_HOISTED);
@@ -719,7 +935,7 @@ neo_status neo_keyip(const neo_ctx* c, const neo_evk* k, const uint64_t* dhat, c
                      int32_t beta, uint64_t* acc, int32_t batch, neo_stream_t st) {
     g_launches = 0;
     TRY(check_ctx(c));
-    if (!k || k->ctx != c) FAIL(NEO_EINVAL, "evaluation key missing or from another context");
+    if (!k || k->ctx != c || k->klss) FAIL(NEO_EINVAL, "Hybrid evaluation key missing or from another context");
     TRY(check_ptr(dhat, "dhat"));
     TRY(check_ptr(acc, "acc"));
     if (!limb_ids || n < 1 || n > KS_MAX_EXT) FAIL(NEO_EINVAL, "need 1 <= n_limbs <= 64 limb ids");

@@ -54,6 +54,17 @@ struct BMatParam {                   // B passed by value (generic neo_bconv, no
     uint4 d[BCTC_MAX_PARTS * BCTC_PART_ROWS * 64 / 16];   // parts of 48 rows x 64 B
 };
 
+// KLSS Recover Limbs (exact centred CRT from T to a limb p of PQ), device table:
+//   y_k = [a_k That_k^-1]_{t_k},  u = rint(sum_k y_k / t_k),  out_p = sum_k y_k [That_k]_p - u [T]_p
+constexpr int KLSS_MAX_T = 16;
+constexpr int KLSS_MAX_EXT = 64;
+struct RecTab {
+    TW that_inv[KLSS_MAX_T];                 // That_k^-1 mod t_k
+    double tinv[KLSS_MAX_T];                 // fl(1 / t_k)
+    TW that_p[KLSS_MAX_EXT][KLSS_MAX_T];     // That_k mod p, by limb id p of PQ
+    TW T_p[KLSS_MAX_EXT];                    // T mod p
+};
+
 }  // namespace neo
 
 struct neo_ctx {
@@ -83,6 +94,14 @@ struct neo_ctx {
     // ds_qlinv_m[l] = q_l^-1 mod q_{l-1}
     std::vector<std::vector<TW>> ds_inv, ds_ql;
     std::vector<TW> ds_qlinv_m;
+    // KLSS (alpha_t > 0): T primes are limb ids num_q+num_p .. +num_t-1
+    int alpha_t = 0, num_t = 0;
+    std::vector<std::vector<int>> klss_groups;             // [i] limb ids of PQ_L in group i
+    std::vector<std::vector<neo::BConvTab>> klss_up;       // [l][j] digit -> T (CUDA-core control)
+    std::vector<std::vector<neo::BConvTC>> klss_up_tc;     // [l][j] digit -> T (tensor cores)
+    std::vector<std::vector<size_t>> klss_up_boff;
+    neo::RecTab* d_rec = nullptr;
+    int limbs_total() const { return num_q + num_p + num_t; }
 
     int beta(int level) const { return (level + 1 + alpha - 1) / alpha; }
     int ext(int level) const { return level + 1 + num_p; }          // limbs of PQ_l
@@ -98,4 +117,5 @@ struct neo_evk {
     uint32_t* lo = nullptr;
     uint8_t* hi = nullptr;
     uint32_t galois = 0;                  // hoisted rotation keys: the key is stored as sigma_{g^-1}(evk_g)
+    int klss = 0;                         // KLSS key: planes are [2][beta~][dnum][alpha'][N] over T
 };

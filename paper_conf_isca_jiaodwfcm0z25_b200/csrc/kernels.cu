@@ -271,7 +271,11 @@ cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t 
         case 5: return launch_k(k_keyip<5>, g, dim3(256), 0, st, A, batch);
         case 6: return launch_k(k_keyip<6>, g, dim3(256), 0, st, A, batch);
         case 7: return launch_k(k_keyip<7>, g, dim3(256), 0, st, A, batch);
-        default: return launch_k(k_keyip<8>, g, dim3(256), 0, st, A, batch);
+        case 8: return launch_k(k_keyip<8>, g, dim3(256), 0, st, A, batch);
+        case 9: return launch_k(k_keyip<9>, g, dim3(256), 0, st, A, batch);
+        case 10: return launch_k(k_keyip<10>, g, dim3(256), 0, st, A, batch);
+        case 11: return launch_k(k_keyip<11>, g, dim3(256), 0, st, A, batch);
+        default: return launch_k(k_keyip<12>, g, dim3(256), 0, st, A, batch);
     }
 }
 cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStream_t st) {

@@ -5,7 +5,7 @@
 namespace neo {
 
 constexpr int KS_MAX_EXT = 64;
-constexpr int KS_MAX_BETA = 8;
+constexpr int KS_MAX_BETA = 12;
 
 struct KeyIPArgs {
     const u64* d;          // KS input [B][l+1][N] (NTT form)

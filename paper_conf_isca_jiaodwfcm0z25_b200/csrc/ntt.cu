@@ -325,7 +325,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
             const u64* accr = ep.acc + bb * ep.acc_b + cc * ep.acc_c + (size_t)k * a.N + row0;
             const u64* addr = cc ? ep.add1 : ep.add0;
             for (int i2 = tid; i2 < N2; i2 += NT) {
-                pf_l2(accr + (size_t)N1 * i2);
+                if (ep.acc) pf_l2(accr + (size_t)N1 * i2);
                 if (addr && !(cc == 0 && ep.add_galois))
                     pf_l2(addr + bb * ep.add_b + (size_t)k * a.N + row0 + (size_t)N1 * i2);
             }
@@ -395,7 +395,8 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                     const int i2 = e >> 3, p = e & 7;
                     const size_t pos = row0 + (size_t)N1 * i2 + 2 * p;
                     const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
-                    const uint4 av = *reinterpret_cast<const uint4*>(accr + pos);
+                    const uint4 av = ep.acc ? *reinterpret_cast<const uint4*>(accr + pos)
+                                            : make_uint4(0u, 0u, 0u, 0u);   // acc = 0 (KLSS ModDown)
                     u64 r0 = shoup(sub_mod(((u64)av.y << 32) | av.x, ((u64)v.y << 32) | v.x, qq), pinv, qq);
                     u64 r1 = shoup(sub_mod(((u64)av.w << 32) | av.z, ((u64)v.w << 32) | v.z, qq), pinv, qq);
                     if (addr) {

@@ -6,6 +6,7 @@
 // Tables: NTT twiddles (ntt_tables.h), BConv constants per (level, digit) for ModUp
 // (Eq. 2) and per level for ModDown (Table 2), P^-1 mod q_i, q_l^-1 mod q_i.
 #include <algorithm>
+#include <cmath>
 #include <cstring>
 #include <stdexcept>
 
@@ -220,6 +221,8 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
     c->device = d->device;
     c->alpha = (c->num_q + c->dnum - 1) / c->dnum;
     const int nl = c->num_q + c->num_p;
+    c->alpha_t = d->alpha_t > 0 ? d->alpha_t : 0;
+    if (c->alpha_t && (d->q || d->p)) { err = "KLSS (alpha_t > 0) needs generated primes"; return NEO_EUNSUPPORTED; }
     if (d->q && d->p) {
         c->mod.assign(d->q, d->q + c->num_q);
         c->mod.insert(c->mod.end(), d->p, d->p + c->num_p);
@@ -229,28 +232,60 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
                 return NEO_EINVAL;
             }
     } else {
-        c->mod = gen_primes(c->log_n, c->word_bits, nl);
-        if ((int)c->mod.size() != nl) { err = "not enough NTT-friendly primes"; return NEO_ENOPRIME; }
+        c->mod = gen_primes(c->log_n, c->word_bits, nl + (c->alpha_t ? KLSS_MAX_T : 0));
+        if ((int)c->mod.size() < nl) { err = "not enough NTT-friendly primes"; return NEO_ENOPRIME; }
     }
-    c->psi.resize(nl);
-    c->h_mods.resize(nl);
-    for (int i = 0; i < nl; ++i) {
+    if (c->alpha_t) {
+        // KLSS (reading K1-K3, Eq. 4): groups of alpha~ consecutive limbs of q_0..q_L, p_0..p_K;
+        // alpha' = least number of T primes with T > 4 beta N B B~, B = alpha max_j Q_j (Algorithm 1's
+        // non-centred digit integer), B~ = max_i P~_i.  Compared in log2 (a margin of 1e-9 bits is
+        // checked; tests/ compare alpha' with the oracle's exact big-integer count).
+        std::vector<int> ext;
+        for (int i = 0; i < nl; ++i) ext.push_back(i);
+        for (int i = 0; i < nl; i += c->alpha_t)
+            c->klss_groups.push_back(std::vector<int>(ext.begin() + i, ext.begin() + std::min(nl, i + c->alpha_t)));
+        auto lg = [&](int id) { return std::log2((long double)c->mod[id]); };
+        long double lq = 0, lp = 0;
+        for (int j = 0; j < c->dnum; ++j) {
+            long double s = 0;
+            for (int i = j * c->alpha; i < std::min((j + 1) * c->alpha, c->num_q); ++i) s += lg(i);
+            lq = std::max(lq, s);
+        }
+        for (const auto& g : c->klss_groups) {
+            long double s = 0;
+            for (int id : g) s += lg(id);
+            lp = std::max(lp, s);
+        }
+        const long double need = 2.0L + std::log2((long double)c->dnum) + c->log_n + std::log2((long double)c->alpha) + lq + lp;
+        long double have = 0;
+        int k = 0;
+        while (have <= need && nl + k < (int)c->mod.size()) have += lg(nl + k++);
+        if (have <= need || k > KLSS_MAX_T) { err = "KLSS: too many T primes"; return NEO_EUNSUPPORTED; }
+        if (std::fabs((double)(have - need)) < 1e-9) { err = "KLSS: Eq. 4 bound too close to call in log2"; return NEO_EUNSUPPORTED; }
+        if (nl > KLSS_MAX_EXT) { err = "KLSS: num_q + num_p must be <= 64"; return NEO_EUNSUPPORTED; }
+        c->num_t = k;
+    }
+    c->mod.resize(nl + c->num_t);
+    const int ntot = nl + c->num_t;
+    c->psi.resize(ntot);
+    c->h_mods.resize(ntot);
+    for (int i = 0; i < ntot; ++i) {
         c->psi[i] = min_psi(c->mod[i], (u64)c->N);
         c->h_mods[i] = mk_mod(c->mod[i]);
     }
     c->L = make_ntt_layout(c->log_n);
 
     // ---- device tables
-    std::vector<TWD> tab((size_t)nl * c->L.total);
-    for (int i = 0; i < nl; ++i) fill_ntt_block(&tab[(size_t)i * c->L.total], c->L, c->mod[i], c->psi[i], c->N);
+    std::vector<TWD> tab((size_t)ntot * c->L.total);
+    for (int i = 0; i < ntot; ++i) fill_ntt_block(&tab[(size_t)i * c->L.total], c->L, c->mod[i], c->psi[i], c->N);
     if (cudaSetDevice(c->device) != cudaSuccess) { err = "cudaSetDevice failed"; return NEO_ECUDA; }
     if (cudaMalloc(&c->d_tab, tab.size() * sizeof(TWD)) != cudaSuccess ||
-        cudaMalloc(&c->d_mods, nl * sizeof(ModQ)) != cudaSuccess) {
+        cudaMalloc(&c->d_mods, ntot * sizeof(ModQ)) != cudaSuccess) {
         err = "cudaMalloc of constant tables failed";
         return NEO_ENOMEM;
     }
     if (cudaMemcpy(c->d_tab, tab.data(), tab.size() * sizeof(TWD), cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemcpy(c->d_mods, c->h_mods.data(), nl * sizeof(ModQ), cudaMemcpyHostToDevice) != cudaSuccess) {
+        cudaMemcpy(c->d_mods, c->h_mods.data(), ntot * sizeof(ModQ), cudaMemcpyHostToDevice) != cudaSuccess) {
         err = "cudaMemcpy of constant tables failed";
         return NEO_ECUDA;
     }
@@ -287,6 +322,12 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
             }
             c->digits[l].push_back(dj);
             c->modup[l].push_back(make_bconv(c, dj, tg));
+            if (c->num_t) {
+                std::vector<int> tids;
+                for (int k = 0; k < c->num_t; ++k) tids.push_back(nl + k);
+                c->klss_up.resize(c->num_q);
+                c->klss_up[l].push_back(make_bconv(c, dj, tids));
+            }
         }
         c->moddown[l] = make_bconv(c, pids, qids);
         for (int i = 0; i < l; ++i) c->ql_inv[l].push_back(mk_tw(invm(c->mod[l] % c->mod[i], c->mod[i]), c->mod[i]));
@@ -308,7 +349,7 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
         const char* e = std::getenv("NEO_BCONV");
         c->use_tc = !(e && std::string(e) == "cuda");
         // the epilogue's exact FP64 sum of the byte planes needs every modulus < 2^36 (bconv_tc.cu)
-        for (int k = 0; k < c->num_q + c->num_p; ++k)
+        for (int k = 0; k < ntot; ++k)
             if (c->mod[k] >> 36) c->use_tc = false;
         std::vector<uint8_t> all, bm;
         c->modup_tc.resize(c->num_q);
@@ -339,6 +380,20 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
             make_bconv_tc(pm, qm, c->moddown_tc[l], bm);
             c->moddown_boff[l] = all.size();
             all.insert(all.end(), bm.begin(), bm.end());
+            if (c->num_t) {                                     // KLSS ModUp: digit -> T
+                c->klss_up_tc.resize(c->num_q);
+                c->klss_up_boff.resize(c->num_q);
+                std::vector<u64> tm(c->mod.begin() + nl, c->mod.begin() + nl + c->num_t);
+                for (int j = 0; j < c->beta(l); ++j) {
+                    std::vector<u64> sm;
+                    for (int id : c->digits[l][j]) sm.push_back(c->mod[id]);
+                    BConvTC P;
+                    make_bconv_tc(sm, tm, P, bm);
+                    c->klss_up_tc[l].push_back(P);
+                    c->klss_up_boff[l].push_back(all.size());
+                    all.insert(all.end(), bm.begin(), bm.end());
+                }
+            }
         }
         if (!fits) c->use_tc = false;
         if (!all.empty()) {
@@ -347,6 +402,35 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
                 err = "cudaMemcpy of BConv tables failed";
                 return NEO_ECUDA;
             }
+        }
+    }
+    if (c->num_t) {                                             // KLSS Recover Limbs constants
+        RecTab R;
+        std::memset(&R, 0, sizeof(R));
+        for (int k = 0; k < c->num_t; ++k) {
+            const u64 tk = c->mod[nl + k];
+            u64 th = 1;
+            for (int m = 0; m < c->num_t; ++m)
+                if (m != k) th = mulm(th, c->mod[nl + m] % tk, tk);
+            R.that_inv[k] = mk_tw(invm(th, tk), tk);
+            R.tinv[k] = 1.0 / (double)tk;
+        }
+        for (int p = 0; p < nl; ++p) {
+            const u64 pm = c->mod[p];
+            u64 T = 1;
+            for (int k = 0; k < c->num_t; ++k) {
+                u64 th = 1;
+                for (int m = 0; m < c->num_t; ++m)
+                    if (m != k) th = mulm(th, c->mod[nl + m] % pm, pm);
+                R.that_p[p][k] = mk_tw(th, pm);
+                T = mulm(T, c->mod[nl + k] % pm, pm);
+            }
+            R.T_p[p] = mk_tw(T, pm);
+        }
+        if (cudaMalloc(&c->d_rec, sizeof(RecTab)) != cudaSuccess ||
+            cudaMemcpy(c->d_rec, &R, sizeof(RecTab), cudaMemcpyHostToDevice) != cudaSuccess) {
+            err = "KLSS table upload failed";
+            return NEO_ECUDA;
         }
     }
     c->pinv.resize(c->num_q);

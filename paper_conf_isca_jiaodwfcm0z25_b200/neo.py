@@ -26,7 +26,8 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_evk_destroy", "neo_keyswitch", "neo_hmult", "neo_hrot", "neo_rescale",
             "neo_keyip", "neo_moddown_combine", "neo_evk_create_hoisted", "neo_hrot_hoisted",
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
-            "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd")
+            "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
+            "neo_evk_create_klss", "neo_klss_query")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -40,7 +41,8 @@ class NeoError(RuntimeError):
 class ParamsDesc(ctypes.Structure):
     _fields_ = [("log_n", ctypes.c_int32), ("num_q", ctypes.c_int32), ("num_p", ctypes.c_int32),
                 ("dnum", ctypes.c_int32), ("word_bits", ctypes.c_int32), ("device", ctypes.c_int32),
-                ("q", ctypes.POINTER(ctypes.c_uint64)), ("p", ctypes.POINTER(ctypes.c_uint64))]
+                ("q", ctypes.POINTER(ctypes.c_uint64)), ("p", ctypes.POINTER(ctypes.c_uint64)),
+                ("alpha_t", ctypes.c_int32)]
 
 
 _lib = None
@@ -79,6 +81,8 @@ def lib() -> ctypes.CDLL:
             "neo_pmult": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
             "neo_hadd": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
             "neo_padd": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
+            "neo_evk_create_klss": [_vp, _vp, ctypes.POINTER(_vp)],
+            "neo_klss_query": [_vp, _i32p, _i32p, _u64p],
         }
         for name, args in sig.items():
             if not hasattr(L, name):        # an older build (A/B runs); tests/test_abi.py requires every symbol
@@ -155,11 +159,12 @@ def neo_debug_bconv_trace():
 class Context:
     """neo_params_create / neo_params_destroy; q, p, psi from neo_params_query."""
 
-    def __init__(self, log_n: int, num_q: int, num_p: int, dnum: int, word_bits: int = 36, device: int = 0):
+    def __init__(self, log_n: int, num_q: int, num_p: int, dnum: int, word_bits: int = 36, device: int = 0,
+                 alpha_t: int = 0):
         self.log_n, self.num_q, self.num_p, self.dnum = log_n, num_q, num_p, dnum
         self.N = 1 << log_n
         self.alpha = -(-num_q // dnum)
-        d = ParamsDesc(log_n, num_q, num_p, dnum, word_bits, device, None, None)
+        d = ParamsDesc(log_n, num_q, num_p, dnum, word_bits, device, None, None, alpha_t)
         h = ctypes.c_void_p()
         _check(lib().neo_params_create(ctypes.byref(d), ctypes.byref(h)), "neo_params_create")
         self.handle = h
@@ -169,6 +174,12 @@ class Context:
         _check(lib().neo_params_query(h, q, p, psi), "neo_params_query")
         self.q, self.p, self.psi = list(q), list(p), list(psi)
         self.moduli = self.q + self.p
+        at, ap = ctypes.c_int32(), ctypes.c_int32()
+        _check(lib().neo_klss_query(h, ctypes.byref(at), ctypes.byref(ap), None), "neo_klss_query")
+        self.alpha_t, self.alpha_p = at.value, ap.value
+        t = (ctypes.c_uint64 * max(1, self.alpha_p))()
+        _check(lib().neo_klss_query(h, None, None, t), "neo_klss_query")
+        self.t = list(t)[: self.alpha_p]
 
     def close(self):
         if self.handle:
@@ -195,10 +206,12 @@ class EvalKey:
     """neo_evk_create / neo_evk_destroy (device copy of [dnum][2][num_q+num_p][N]);
     with hoisted_galois=g, neo_evk_create_hoisted (key for neo_hrot_hoisted)."""
 
-    def __init__(self, ctx: Context, evk: torch.Tensor, hoisted_galois: int | None = None):
+    def __init__(self, ctx: Context, evk: torch.Tensor, hoisted_galois: int | None = None, klss: bool = False):
         self.ctx = ctx
         h = ctypes.c_void_p()
-        if hoisted_galois is None:
+        if klss:          # neo_evk_create_klss: evk is [2][beta~][dnum][alpha'][N] over the T primes
+            _check(lib().neo_evk_create_klss(ctx.handle, _ptr(evk), ctypes.byref(h)), "neo_evk_create_klss")
+        elif hoisted_galois is None:
             _check(lib().neo_evk_create(ctx.handle, _ptr(evk), ctypes.byref(h)), "neo_evk_create")
         else:
             _check(lib().neo_evk_create_hoisted(ctx.handle, _ptr(evk), hoisted_galois, ctypes.byref(h)),
