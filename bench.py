@@ -47,6 +47,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-hoisted", action="store_true")
+    ap.add_argument("--no-klss", action="store_true",
+                    help="skip the KLSS vs Hybrid key-switch comparison at Set-C (SURVEY §8(f) row 1)")
     ap.add_argument("--batch-hrot", type=int, default=256,
                     help="BASELINE configs[2]: this many independent HRot key-switches (one shared key) "
                          "split data-parallel over the ranks, plus a batch sweep up to it (0 = skip)")
@@ -457,6 +459,50 @@ def run_neo(args):
         del big_in, big_out, big_ws
         torch.cuda.empty_cache()
 
+    # SURVEY §8(f) row 1 (Table 8 / Fig. 16 analogue): one key-switch at Set-C (N=2^16, L=35,
+    # dnum=9, alpha~=5; WordSize_T=36 -> 10 T primes, reading K6) with the KLSS key and with the
+    # Hybrid key of the same parameters, B = 1 and B = 8 per GPU, CUDA events, max over ranks.
+    # Keys and inputs are uniform residues < 2^35 made on the device (timing is data-independent).
+    klss_block = None
+    if not args.no_klss:
+        cctx = neo.Context(16, 36, 4, 9, alpha_t=5, device=local)
+        gen = torch.Generator(device="cuda")
+        gen.manual_seed(seed + 91)
+        rnd = lambda *shape: torch.randint(0, 1 << 35, shape, dtype=torch.int64, device="cuda",
+                                           generator=gen).view(torch.uint64)
+        bt = -(-(36 + 4) // 5)
+        keys = {"klss": neo.EvalKey(cctx, rnd(2, bt, 9, cctx.alpha_p, N), klss=True),
+                "hybrid": neo.EvalKey(cctx, rnd(9, 2, 40, N))}
+        klss_block = {"config": "Set-C (Table 4): N=2^16, L=35, dnum=9, alpha~=5, WordSize_T=36 "
+                                f"(alpha'={cctx.alpha_p} T primes), level 35",
+                      "unit": "KS/s", "timing": "CUDA events around 20 neo_keyswitch calls after 3 warm-ups"}
+        for Bk in (1, 8):
+            dk = rnd(Bk, Lq, N)
+            o0, o1 = torch.empty_like(dk), torch.empty_like(dk)
+            wsk = torch.empty(cctx.workspace_size(neo.NEO_OP_KEYSWITCH, LEVEL, Bk) // 8, dtype=torch.uint64,
+                              device="cuda")
+            for meth, key in keys.items():
+                for _ in range(3):
+                    neo.neo_keyswitch(cctx, key, dk, LEVEL, o0, o1, Bk, wsk)
+                torch.cuda.synchronize()
+                barrier()
+                k0, k1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                k0.record()
+                for _ in range(20):
+                    neo.neo_keyswitch(cctx, key, dk, LEVEL, o0, o1, Bk, wsk)
+                k1.record()
+                torch.cuda.synchronize()
+                kms = k0.elapsed_time(k1) / 20
+                if world > 1:
+                    t = torch.tensor([kms], dtype=torch.float64, device="cuda")
+                    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                    kms = float(t.item())
+                klss_block[f"{meth}_B{Bk}"] = {"ms_per_call": round(kms, 4), "value": Bk * world / (kms / 1e3)}
+            del dk, o0, o1, wsk
+        del keys
+        cctx.close()
+        torch.cuda.empty_cache()
+
     # end-to-end through the public API with pinned host buffers: every step copies its three
     # input ciphertexts host->device and both results device->host.  Copies run on their own
     # streams, double-buffered, so the H2D of step k+1 and the D2H of step k-1 overlap the
@@ -539,7 +585,7 @@ def run_neo(args):
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted,
-                "batch_hrot": batch_block,
+                "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}
         print(json.dumps(line), flush=True)

@@ -34,6 +34,7 @@ static thread_local int g_launches = 0;
         }                                                                   \
     } while (0)
 
+constexpr int NEO_HOST_ROWS = 1024;   // host row lists (split into launches of <= NEO_MAX_ROWS)
 static inline cudaStream_t S(neo_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
 
 // BConv pipeline trace (debug only, NEO_BCONV_DBG=1): CTA 0's clock64 stamps of the last launch
@@ -92,7 +93,16 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
                            int batch, cudaStream_t st, const RowEpi* epi = nullptr, bool in_lazy = false,
                            const TWD* scale = nullptr, unsigned galois = 0) {
     if (n <= 0) return NEO_OK;
-    if (n > NEO_MAX_ROWS) FAIL(NEO_EUNSUPPORTED, "too many limb rows in one transform");
+    if (n > NEO_MAX_ROWS) {               // more rows than one launch's descriptor holds: chunks
+        if (epi) FAIL(NEO_EUNSUPPORTED, "too many limb rows for a fused-epilogue transform");
+        for (int k0 = 0; k0 < n; k0 += NEO_MAX_ROWS) {
+            const int m = std::min(NEO_MAX_ROWS, n - k0);
+            neo_status s = ntt_rows(c, fwd, src, src_bs, src_off + k0, dst, dst_bs, dst_off + k0, prime + k0, m, tmp,
+                                    batch, st, nullptr, in_lazy, scale ? scale + k0 : nullptr, galois);
+            if (s) return s;
+        }
+        return NEO_OK;
+    }
     RowSet a, b;
     const long long N = c->N;
     a.n = b.n = n;
@@ -170,7 +180,7 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
                            cudaStream_t st, unsigned galois = 0) {
     const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l);
     u64 *y = ws + Ly.y, *up = ws + Ly.up, *tmp = ws + Ly.tmp;
-    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
     neo_status s;
 
     // a3: INTT of d (l+1 limbs) -> y (coefficient form); on the tensor-core path the ModUp
@@ -248,7 +258,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
                             unsigned galois = 0, bool add_galois = true) {
     const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p;
     u64 *up = ws + Ly.up, *acc = ws + Ly.acc, *conv = ws + Ly.conv, *pc = ws + Ly.pc, *tmp = ws + Ly.tmp;
-    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
     neo_status s;
 
     // a6: KeyIP over all E limbs of PQ_l
@@ -363,7 +373,7 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     if (beta > KLSS_MAX_BETA || bt > KLSS_MAX_GROUPS) FAIL(NEO_EUNSUPPORTED, "KLSS: too many digits or groups");
     u64 *y = ws + Ly.y, *up = ws + Ly.up, *acc = ws + Ly.acc, *rec = ws + Ly.rec, *conv = ws + Ly.conv,
         *diff = ws + Ly.diff, *tmp = ws + Ly.tmp;
-    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
     neo_status s;
     // 1. INTT of d; Algorithm 2's [c_i qhat_i^-1]_{q_i} folded in (the digits are Hybrid's)
     for (int i = 0; i < Lq; ++i) { so[i] = i; dof[i] = i; pr[i] = i; }
@@ -998,7 +1008,7 @@ neo_status neo_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, u
     u64* last = w;                          // [2B][N]: INTT of c_l, canonical mod q_l
     u64* tmp = last + (size_t)B2 * N;       // NTT intermediate
     cudaStream_t s = S(st);
-    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
     // 1. coefficient form of the last limb of both components
     so[0] = l; dof[0] = 0; pr[0] = l;
     TRY(ntt_rows(c, false, ct_in, (long long)(l + 1) * N, so, last, N, dof, pr, 1, tmp, B2, s));
@@ -1064,7 +1074,7 @@ neo_status neo_double_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t l
     u64* corr = last2 + (size_t)B2 * 2 * N;           // [2B][l-1][N]
     u64* tmp = corr + (size_t)B2 * (l - 1) * N;       // NTT intermediate
     cudaStream_t s = S(st);
-    int so[NEO_MAX_ROWS], dof[NEO_MAX_ROWS], pr[NEO_MAX_ROWS];
+    int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
     // 1. coefficient form of the last two limbs of both components
     for (int k = 0; k < 2; ++k) { so[k] = l - 1 + k; dof[k] = k; pr[k] = l - 1 + k; }
     TRY(ntt_rows(c, false, ct_in, (long long)(l + 1) * N, so, last2, 2LL * N, dof, pr, 2, tmp, B2, s));

@@ -6,7 +6,7 @@ for v in $AB; do
   cp ab/$v.so $L
   echo "== $v"
   [ -z "$NO_NTT" ] && timeout 300 python tools/ntt_bench.py 108 50
-  timeout 600 python bench.py --steps 200 --warmup 10 --no-cpu-baseline --no-e2e --no-hoisted --batch-hrot 0 > gpurun_out/ab_$v.json 2>/dev/null
+  timeout 600 python bench.py --steps 200 --warmup 10 --no-cpu-baseline --no-e2e --no-hoisted --batch-hrot 0 --no-klss > gpurun_out/ab_$v.json 2>/dev/null
   python -c "
 import json; d=json.load(open('gpurun_out/ab_$v.json')); b=d['breakdown']
 print('bench', round(d['value'],1), 'KS/s ms', round(d['ms_per_step'],4), '1-stream', round(d['single_stream_profiled_ms_per_step'],4))

@@ -1,2 +1,4 @@
-timeout 1200 python -m pytest tests/test_gpu_klss.py -x -q 2>&1 | tail -25
-timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_ops.py -x -q 2>&1 | tail -3
+timeout 900 python bench.py --steps 100 --warmup 5 --no-cpu-baseline --no-e2e --no-hoisted --batch-hrot 0 > gpurun_out/bench_klss.json 2> gpurun_out/bench_klss.err
+tail -3 gpurun_out/bench_klss.err
+python -c "
+import json; d=json.load(open('gpurun_out/bench_klss.json')); print(round(d['value'],1), json.dumps(d['klss_vs_hybrid_setc'], indent=1))"
