@@ -199,6 +199,7 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
     // a4: ModUp BConv of all beta digits: y[D_j] -> up[j][targets]  (one launch on tensor cores)
     {
         BConvMulti M;
+        M.centred = 0;
         M.dbg = bconv_dbg();
         M.njobs = 0;
         M.pre_scaled = 1;
@@ -301,6 +302,8 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
         if (c->use_tc) {
             BConvMulti M;
+            M.centred = 0;
+        M.centred = 0;
             M.dbg = bconv_dbg() ? bconv_dbg() + 512 : nullptr;
             M.njobs = 1;
             M.pre_scaled = 1;
@@ -370,7 +373,8 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
                             const u64* add0, const u64* add1, long long add_bs, cudaStream_t st, unsigned galois) {
     const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p, ap = c->num_t;
     const int bt = (int)c->klss_groups.size(), nl = c->num_q + c->num_p;
-    if (beta > KLSS_MAX_BETA || bt > KLSS_MAX_GROUPS) FAIL(NEO_EUNSUPPORTED, "KLSS: too many digits or groups");
+    if (beta > KLSS_MAX_BETA || bt > KLSS_MAX_GROUPS || c->alpha_t > KLSS_MAX_OUT_G)
+        FAIL(NEO_EUNSUPPORTED, "KLSS: too many digits, groups (<= 8) or limbs per group (<= 16)");
     u64 *y = ws + Ly.y, *up = ws + Ly.up, *acc = ws + Ly.acc, *rec = ws + Ly.rec, *conv = ws + Ly.conv,
         *diff = ws + Ly.diff, *tmp = ws + Ly.tmp;
     int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
@@ -389,6 +393,7 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     // 2. ModUp: every digit -> the alpha' T limbs (Eq. 3, Algorithm 1)
     {
         BConvMulti M;
+        M.centred = 0;
         M.dbg = nullptr;
         M.njobs = 0;
         M.pre_scaled = 1;
@@ -457,11 +462,48 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
                 ++nr;
             }
     if (nr > NEO_MAX_ROWS) FAIL(NEO_EUNSUPPORTED, "KLSS: too many T rows for one transform");
+    // Recover Limbs engine: CUDA cores by default (16 small conversions: the tensor-core kernel's
+    // per-tile pipeline cost dominates, measured 0.136 vs 0.102 ms per KS at Set-C); NEO_KLSS_REC=tc
+    // selects the tensor-core conversion with the centred-correction column
+    static const bool rec_tc = [] { const char* e = std::getenv("NEO_KLSS_REC"); return e && std::string(e) == "tc"; }();
+    const bool use_rec_tc = c->use_tc && rec_tc;
+    TWD tsc[NEO_HOST_ROWS];                // tensor-core Recover: [That_k^-1]_{t_k} folded into the INTT
+    if (use_rec_tc)
+        for (int r = 0; r < nr; ++r) tsc[r] = c->klss_rec_tc[l][I.group[0]].qhat_inv[r % ap];
     if ((s = ntt_rows(c, false, acc, (long long)2 * bt * ap * N, so, acc, (long long)2 * bt * ap * N, dof, pr, nr,
-                      tmp, B, st)))
+                      tmp, B, st, nullptr, false, use_rec_tc ? tsc : nullptr)))
         return s;
-    // 6. Recover Limbs: exact centred CRT from T to the PQ_l limbs (K4)
-    LAUNCH(PK_COMBINE, st, launch_klss_recover(R, B, st));
+    // 6. Recover Limbs: exact centred CRT from T to the PQ_l limbs (K4): on tensor cores, one
+    //    conversion per (group, component) with the centred-correction column; else CUDA cores
+    if (use_rec_tc) {
+        BConvMulti M;
+        M.dbg = nullptr;
+        M.njobs = 0;
+        M.pre_scaled = 1;
+        M.lazy_out = 0;
+        M.centred = 1;
+        for (int cc = 0; cc < 2; ++cc)
+            for (int g = 0; g < ng; ++g) {
+                const int i = I.group[g];
+                BConvIO io;
+                io.in = acc + (size_t)(cc * bt + i) * ap * N;
+                io.out = rec + (size_t)cc * E * N;
+                io.in_bstride = (long long)2 * bt * ap * N;
+                io.out_bstride = (long long)2 * E * N;
+                for (int t = 0; t < ap; ++t) io.in_off[t] = t;
+                for (int o = R.first[g]; o < R.first[g + 1]; ++o) io.out_off[o - R.first[g]] = R.out_pos[o];
+                M.P[M.njobs] = c->klss_rec_tc[l][i];
+                M.io[M.njobs] = io;
+                M.bmat[M.njobs] = c->d_bmat + c->klss_rec_boff[l][i];
+                if (++M.njobs == 4) {
+                    LAUNCH(PK_COMBINE, st, launch_bconv_tc(M, N, B, c->num_sms, st));
+                    M.njobs = 0;
+                }
+            }
+        if (M.njobs) LAUNCH(PK_COMBINE, st, launch_bconv_tc(M, N, B, c->num_sms, st));
+    } else {
+        LAUNCH(PK_COMBINE, st, launch_klss_recover(R, B, st));
+    }
     // 7. ModDown BConv P -> Q_l on the recovered (coefficient-form) P limbs, batch 2B
     {
         BConvIO io;
@@ -472,6 +514,8 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
         if (c->use_tc) {                        // canonical u64 out (the difference kernel reads it)
             BConvMulti M;
+            M.centred = 0;
+        M.centred = 0;
             M.dbg = nullptr;
             M.njobs = 1;
             M.pre_scaled = 0;

@@ -72,7 +72,7 @@ static_assert(kSlots * kSlotCols == 512, "TMEM plan");
 // A tile of 36 targets is 4 parts, one per set.  Per-job / per-target constants and the tile
 // schedule are staged in shared memory during setup (register-indexed reads of the large
 // parameter block miss the constant cache on the critical path).
-template <bool kPre, bool kLazy, class LoadB>
+template <bool kPre, bool kLazy, class LoadB, bool kCorr = false>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
                                               int tiles_per_entry, int batch, int exp,
                                               const CUtensorMap* tmaps = nullptr, const int* use_tmap = nullptr,
@@ -197,6 +197,17 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                     w[wi + 1] |= (uint32_t)(y >> (32 - sh));
                     if (sh > 24) w[wi + 2] |= (uint32_t)(y >> (64 - sh));
                 }
+            }
+            if (kCorr) {          // centred lift: u = rint(sum_j y_j / q_j) into K column 5 n_in (byte)
+                double sacc = 0.0;
+#pragma unroll
+                for (int j = 0; j < BCTC_MAX_IN; ++j)
+                    if (j < n_in) sacc = __fma_rn(u2d(c[j]), PJ[jb].qinv_in[j], sacc);
+                const uint32_t u = (uint32_t)__double2int_rn(sacc);
+                const int byte = 5 * n_in;
+#pragma unroll
+                for (int kk = 0; kk < 16; ++kk)
+                    if (kk == (byte >> 2)) w[kk] |= u << (8 * (byte & 3));
             }
             const int s = i % kAStages, k = i / kAStages;
             WAIT(&empty_a[s], (k & 1) ^ 1, 2);
@@ -336,12 +347,12 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     if (warp == 0) tc::tmem_dealloc(tmem, kSlots * kSlotCols);
 }
 
-template <bool kPre, bool kLazy>
+template <bool kPre, bool kLazy, bool kCorr = false>
 __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_g(const __grid_constant__ BConvMulti M, int N, int tiles_per_entry, int batch, int exp) {
-    bconv_tc_body<kPre, kLazy>(M.P, M.io, M.njobs,
-                               [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; }, N,
-                               tiles_per_entry, batch, exp, M.tmap, M.use_tmap, M.dbg);
+    auto lb = [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; };
+    bconv_tc_body<kPre, kLazy, decltype(lb), kCorr>(M.P, M.io, M.njobs, lb, N, tiles_per_entry, batch, exp, M.tmap,
+                                                   M.use_tmap, M.dbg);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
@@ -360,6 +371,8 @@ static void bconv_tc_init() {
         cudaFuncSetAttribute(k_bconv_tc_g<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         cudaFuncSetAttribute(k_bconv_tc_g<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         cudaFuncSetAttribute(k_bconv_tc_p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
+        cudaFuncSetAttribute(k_bconv_tc_g<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)kSmemAlloc);
         init = true;
     }
 }
@@ -411,6 +424,10 @@ cudaError_t launch_bconv_tc(const BConvMulti& M0, int N, int batch, int num_sms,
     // exp != 0: timing experiments only (NEO_BCONV_EXP: 32 no TMA, 256 setup/teardown only)
     auto k = M.pre_scaled ? (M.lazy_out ? k_bconv_tc_g<true, true> : k_bconv_tc_g<true, false>)
                           : (M.lazy_out ? k_bconv_tc_g<false, true> : k_bconv_tc_g<false, false>);
+    if (M.centred) {                       // KLSS Recover Limbs: pre-scaled input, canonical output only
+        if (!M.pre_scaled || M.lazy_out) return cudaErrorInvalidValue;
+        k = k_bconv_tc_g<true, false, true>;
+    }
     return launch_k(k, dim3(grid), dim3(kThreads), kSmemAlloc, st, M, N, tiles_per_entry, batch, exp);
 }
 

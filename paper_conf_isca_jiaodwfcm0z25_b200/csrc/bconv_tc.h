@@ -11,8 +11,11 @@ namespace neo {
 
 // Host: the pre-shifted byte matrix B[n = 5t + b][k = 5i + a] = byte_b(2^(8a) qhat_i mod t),
 // stored in the SWIZZLE_NONE K-major core-matrix layout (ncols x 64 bytes).
+// corr (optional, KLSS Recover Limbs): corr[t] = (-Q_in) mod t fills the extra K column 5 n_in,
+// which the producers load with u = rint(sum_i y_i / q_i), so the GEMM returns the CENTRED lift
+// sum_i y_i qhat_i - u Q_in (exact while |x| < Q_in / 4); needs 5 n_in < 64.
 void make_bconv_tc(const std::vector<u64>& src_mod, const std::vector<u64>& dst_mod, BConvTC& P,
-                   std::vector<uint8_t>& bmat);
+                   std::vector<uint8_t>& bmat, const std::vector<u64>* corr = nullptr);
 
 size_t bconv_tc_smem(int ncols);
 
@@ -24,6 +27,7 @@ struct BConvMulti {
     int njobs;
     int pre_scaled;      // inputs already hold y_i = [c_i qhat_i^-1]_{q_i} (scale folded into the INTT)
     int lazy_out;        // write lazy doubles |x| < 2^40 for the next NTT instead of canonical u64
+    int centred;         // B has the correction column of make_bconv_tc(corr): producers supply u
     BConvTC P[4];
     BConvIO io[4];
     const uint8_t* bmat[4];

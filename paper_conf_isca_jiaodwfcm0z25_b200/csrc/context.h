@@ -62,6 +62,7 @@ struct RecTab {
     TW that_inv[KLSS_MAX_T];                 // That_k^-1 mod t_k
     double tinv[KLSS_MAX_T];                 // fl(1 / t_k)
     TW that_p[KLSS_MAX_EXT][KLSS_MAX_T];     // That_k mod p, by limb id p of PQ
+    unsigned that_lo[KLSS_MAX_EXT][KLSS_MAX_T], that_hi[KLSS_MAX_EXT][KLSS_MAX_T];   // its 18-bit halves
     TW T_p[KLSS_MAX_EXT];                    // T mod p
 };
 
@@ -101,6 +102,8 @@ struct neo_ctx {
     std::vector<std::vector<neo::BConvTC>> klss_up_tc;     // [l][j] digit -> T (tensor cores)
     std::vector<std::vector<size_t>> klss_up_boff;
     neo::RecTab* d_rec = nullptr;
+    std::vector<std::vector<neo::BConvTC>> klss_rec_tc;    // [l][i] T -> group i's limbs in PQ_l (centred)
+    std::vector<std::vector<size_t>> klss_rec_boff;
     int limbs_total() const { return num_q + num_p + num_t; }
 
     int beta(int level) const { return (level + 1 + alpha - 1) / alpha; }

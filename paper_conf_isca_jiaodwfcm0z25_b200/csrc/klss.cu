@@ -1,81 +1,127 @@
 // klss.cu -- KLSS key-switching kernels (Neo's default method, L155-180; readings K1-K6 in
 // DESIGN.md): the inner product over the T basis (Alg. 3 / Alg. 4) and Recover Limbs.
+#include <algorithm>
+
 #include "klss.h"
 
 namespace neo {
 
-// IP on CUDA cores (the paper's CUDA-core IP mapping, L488: its beta x beta~ products are
-// far too small for a tensor-core tile at B = 1).  One thread per (T limb k, coefficient n):
-// for each present group i and component c the beta key words stay in registers while the
-// batch is walked, so the key is read once per launch (Z21).
-__global__ void __launch_bounds__(256)
+// 36-bit x 36-bit products as four 18-bit x 18-bit IMADs (32x32->64) into three 64-bit partial
+// sums (the CUDA-core BConv's scheme): sum_j x_j e_j = A + 2^18 Bm + 2^36 C exactly.
+NEO_DEV void mac18(u64& A, u64& Bm, u64& C, unsigned xl, unsigned xh, unsigned el, unsigned eh) {
+    A += (u64)xl * el;
+    Bm += (u64)xl * eh + (u64)xh * el;
+    C += (u64)xh * eh;
+}
+NEO_DEV u64 reduce18(u64 A, u64 Bm, u64 C, ModQ m) {       // A, Bm, C < 2^41 (<= 16 terms)
+    const u64 t = A + (Bm << 18);
+    const u64 lo = t + (C << 36);
+    const u64 hi = (C >> 28) + (t < A) + (lo < t);
+    return barrett_reduce(hi, lo, m);
+}
+
+// IP on CUDA cores (the paper's CUDA-core IP mapping, L488: its beta x beta~ products are far
+// too small for a tensor-core tile).  One thread per (coefficient n, T limb k, group i): a warp
+// is 32 consecutive coefficients of one group, so every key plane access is a coalesced
+// 128-byte (32-bit plane) / 32-byte (8-bit plane) segment, and the 8 group warps of a CTA read
+// the same digit values (L1 hits).  The 2 x beta key words of the thread stay in registers
+// while the batch is walked: the key (the dominant traffic, 5 bytes per residue) is read once.
+constexpr int KLSS_IP_W = 32;
+
+template <int BETA>
+__global__ void __launch_bounds__(256, 3)
 k_klss_ip(const __grid_constant__ KlssIpArgs A, int batch) {
     pdl_wait();
-    const int n = blockIdx.x * blockDim.x + threadIdx.x;
-    const int k = blockIdx.y;
-    if (n >= A.N) return;
+    const int gi = threadIdx.y;
+    if (gi >= A.n_groups) return;
+    const int n = blockIdx.x * KLSS_IP_W + threadIdx.x;
+    const int k = blockIdx.y, i = A.group[gi];
     const ModQ m = A.mods[A.t0 + k];
-    const size_t NK = (size_t)A.alpha_p * A.N;                  // one [alpha'][N] block
+    const size_t NK = (size_t)A.alpha_p * A.N;
     const size_t col = (size_t)k * A.N + n;
-    for (int gi = 0; gi < A.n_groups; ++gi) {
-        const int i = A.group[gi];
-        for (int c = 0; c < 2; ++c) {
-            u64 e[KLSS_MAX_BETA];
-            const size_t kb = (size_t)(c * A.beta_t + i) * A.dnum * NK + col;
+    unsigned el[2][BETA], eh[2][BETA];
 #pragma unroll
-            for (int j = 0; j < KLSS_MAX_BETA; ++j) {
-                e[j] = 0;
-                if (j < A.beta) {
-                    const size_t o = kb + (size_t)j * NK;
-                    e[j] = (u64)A.key_lo[o] | ((u64)A.key_hi[o] << 32);
-                }
-            }
-            for (int b = 0; b < batch; ++b) {
-                const u64* up = A.up + (size_t)b * A.beta * NK + col;
-                u64 h = 0, l = 0;                               // < beta 2^72 <= 2^76
+    for (int c = 0; c < 2; ++c) {
+        const size_t kb = (size_t)(c * A.beta_t + i) * A.dnum * NK + col;
 #pragma unroll
-                for (int j = 0; j < KLSS_MAX_BETA; ++j)
-                    if (j < A.beta) mac128(h, l, up[(size_t)j * NK], e[j]);
-                A.acc[((size_t)(b * 2 + c) * A.beta_t + i) * NK + col] = barrett_reduce(h, l, m);
-            }
+        for (int j = 0; j < BETA; ++j) {
+            const size_t o = kb + (size_t)j * NK;
+            const u64 e = (u64)A.key_lo[o] | ((u64)A.key_hi[o] << 32);
+            el[c][j] = (unsigned)(e & 0x3FFFF);
+            eh[c][j] = (unsigned)(e >> 18);
         }
+    }
+    for (int b = 0; b < batch; ++b) {
+        const u64* up = A.up + (size_t)b * A.beta * NK + col;
+        u64 a0 = 0, a1 = 0, a2 = 0, c0 = 0, c1 = 0, c2 = 0;
+#pragma unroll
+        for (int j = 0; j < BETA; ++j) {
+            const u64 x = up[(size_t)j * NK];
+            const unsigned xl = (unsigned)(x & 0x3FFFF), xh = (unsigned)(x >> 18);
+            mac18(a0, a1, a2, xl, xh, el[0][j], eh[0][j]);
+            mac18(c0, c1, c2, xl, xh, el[1][j], eh[1][j]);
+        }
+        u64* acc = A.acc + (size_t)(b * 2) * A.beta_t * NK + (size_t)i * NK + col;
+        acc[0] = reduce18(a0, a1, a2, m);
+        acc[(size_t)A.beta_t * NK] = reduce18(c0, c1, c2, m);
     }
 }
 
 // Recover Limbs: x = the centred lift of acc from T (|x| < T/4 by Eq. 4 + guard bit, K3):
 //   y_k = [a_k That_k^-1]_{t_k};  X = sum_k y_k That_k = x + u T exactly, u = rint(sum_k y_k / t_k)
 //   (the FP64 sum is within 2^-44 of X / T, and |x / T| < 1/4, so the rounding is exact);
-//   out_p = sum_k y_k [That_k]_p - u [T]_p  mod p  = x mod p.
+//   out_p = sum_k y_k [That_k]_p - u [T]_p  mod p  = x mod p   (18-bit split products).
+template <int AP>
 __global__ void __launch_bounds__(256)
 k_klss_recover(const __grid_constant__ KlssRecArgs A) {
     pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
     const int gi = blockIdx.y >> 1, c = blockIdx.y & 1, b = blockIdx.z;
-    if (n >= A.N) return;
     const RecTab& R = *A.tab;
-    const size_t NK = (size_t)A.alpha_p * A.N;
-    const u64* a = A.acc + ((size_t)(b * 2 + c) * A.beta_t + A.group[gi]) * NK + n;
-    u64 y[KLSS_MAX_T];
-    double s = 0.0;
-#pragma unroll
-    for (int k = 0; k < KLSS_MAX_T; ++k) {
-        y[k] = 0;
-        if (k < A.alpha_p) {
-            const u64 tk = A.mods[A.t0 + k].q;
-            y[k] = shoup(a[(size_t)k * A.N], R.that_inv[k], tk);
-            s = __fma_rn((double)y[k], R.tinv[k], s);
+    const int o0 = A.first[gi], no = A.first[gi + 1] - o0;
+    __shared__ uint2 tc[KLSS_MAX_OUT_G][AP];                   // this group's [That_k]_p in 18-bit halves
+    __shared__ TW tT[KLSS_MAX_OUT_G];                          // [T]_p
+    __shared__ ModQ tm[KLSS_MAX_OUT_G];
+    __shared__ int tpos[KLSS_MAX_OUT_G];
+    for (int e = threadIdx.x; e < no * AP; e += blockDim.x) {
+        const int ro = e / AP, k = e - ro * AP, p = A.out_id[o0 + ro];
+        tc[ro][k] = make_uint2(R.that_lo[p][k], R.that_hi[p][k]);
+        if (k == 0) {
+            tT[ro] = R.T_p[p];
+            tm[ro] = A.mods[p];
+            tpos[ro] = A.out_pos[o0 + ro];
         }
     }
-    const u64 u = (u64)__double2ll_rn(s);
-    for (int o = A.first[gi]; o < A.first[gi + 1]; ++o) {
-        const int p = A.out_id[o];
-        const ModQ m = A.mods[p];
-        u64 h = 0, l = 0;                                       // < 16 * 2^72
+    __syncthreads();
+    if (n >= A.N) return;
+    const size_t NK = (size_t)AP * A.N;
+    const u64* a = A.acc + ((size_t)(b * 2 + c) * A.beta_t + A.group[gi]) * NK + n;
+    u64 av[AP];
 #pragma unroll
-        for (int k = 0; k < KLSS_MAX_T; ++k)
-            if (k < A.alpha_p) mac128(h, l, y[k], R.that_p[p][k].w);
-        const u64 r = barrett_reduce(h, l, m);
-        A.rec[((size_t)(b * 2 + c) * A.E + A.out_pos[o]) * A.N + n] = sub_mod(r, shoup(u, R.T_p[p], m.q), m.q);
+    for (int k = 0; k < AP; ++k) av[k] = a[(size_t)k * A.N];      // all loads in flight first
+    unsigned yl[AP], yh[AP];
+    double s = 0.0;
+#pragma unroll
+    for (int k = 0; k < AP; ++k) {
+        const u64 tk = A.mods[A.t0 + k].q;
+        const u64 y = shoup(av[k], R.that_inv[k], tk);
+        s = __fma_rn((double)y, R.tinv[k], s);
+        yl[k] = (unsigned)(y & 0x3FFFF);
+        yh[k] = (unsigned)(y >> 18);
+    }
+    const u64 u = (u64)__double2ll_rn(s);
+    u64* out = A.rec + (size_t)(b * 2 + c) * A.E * A.N + n;
+#pragma unroll 1
+    for (int ro = 0; ro < no; ++ro) {
+        u64 a0 = 0, a1 = 0, a2 = 0;
+#pragma unroll
+        for (int k = 0; k < AP; ++k) {
+            const uint2 cc = tc[ro][k];
+            mac18(a0, a1, a2, yl[k], yh[k], cc.x, cc.y);
+        }
+        const ModQ m = tm[ro];
+        const u64 r = reduce18(a0, a1, a2, m);
+        out[(size_t)tpos[ro] * A.N] = sub_mod(r, shoup(u, tT[ro], m.q), m.q);
     }
 }
 
@@ -93,10 +139,25 @@ k_klss_diff(const __grid_constant__ KlssDiffArgs A) {
 }
 
 cudaError_t launch_klss_ip(const KlssIpArgs& A, int batch, cudaStream_t st) {
-    return launch_k(k_klss_ip, dim3((A.N + 255) / 256, A.alpha_p), dim3(256), 0, st, A, batch);
+    const dim3 g(A.N / KLSS_IP_W, A.alpha_p), blk(KLSS_IP_W, 256 / KLSS_IP_W);
+    switch (A.beta) {
+#define NEO_IP_CASE(B) case B: return launch_k(k_klss_ip<B>, g, blk, 0, st, A, batch);
+        NEO_IP_CASE(1) NEO_IP_CASE(2) NEO_IP_CASE(3) NEO_IP_CASE(4) NEO_IP_CASE(5) NEO_IP_CASE(6)
+        NEO_IP_CASE(7) NEO_IP_CASE(8) NEO_IP_CASE(9) NEO_IP_CASE(10) NEO_IP_CASE(11) NEO_IP_CASE(12)
+#undef NEO_IP_CASE
+        default: return cudaErrorInvalidValue;
+    }
 }
 cudaError_t launch_klss_recover(const KlssRecArgs& A, int batch, cudaStream_t st) {
-    return launch_k(k_klss_recover, dim3((A.N + 255) / 256, 2 * A.n_groups, batch), dim3(256), 0, st, A);
+    const dim3 g((A.N + 255) / 256, 2 * A.n_groups, batch);
+    switch (A.alpha_p) {
+#define NEO_REC_CASE(K) case K: return launch_k(k_klss_recover<K>, g, dim3(256), 0, st, A);
+        NEO_REC_CASE(2) NEO_REC_CASE(3) NEO_REC_CASE(4) NEO_REC_CASE(5) NEO_REC_CASE(6) NEO_REC_CASE(7)
+        NEO_REC_CASE(8) NEO_REC_CASE(9) NEO_REC_CASE(10) NEO_REC_CASE(11) NEO_REC_CASE(12) NEO_REC_CASE(13)
+        NEO_REC_CASE(14) NEO_REC_CASE(15) NEO_REC_CASE(16)
+#undef NEO_REC_CASE
+        default: return cudaErrorInvalidValue;
+    }
 }
 cudaError_t launch_klss_diff(const KlssDiffArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_klss_diff, dim3((A.N + 255) / 256, A.Lq, 2 * batch), dim3(256), 0, st, A);

@@ -6,7 +6,8 @@
 namespace neo {
 
 constexpr int KLSS_MAX_BETA = 12;     // digits (beta <= dnum)
-constexpr int KLSS_MAX_GROUPS = 16;   // beta~
+constexpr int KLSS_MAX_GROUPS = 8;    // beta~ (one warp per group in the IP CTA)
+constexpr int KLSS_MAX_OUT_G = 16;    // limbs per group (alpha~)
 
 // IP (Alg. 3 L359-382 / Alg. 4): for every T limb k and coefficient n,
 //   acc[b][c][i][k] = sum_{j < beta} up[b][j][k] * e[c][i][j][k]  mod t_k

@@ -171,7 +171,8 @@ static BConvTab make_bconv(const neo_ctx* c, const std::vector<int>& src, const 
 
 // Tensor-core BConv constants (bconv_tc.cu): B[n = 5t + b][k = 5i + a] =
 // byte_b((2^(8a) qhat_i) mod t) in the SWIZZLE_NONE K-major core-matrix layout.
-void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BConvTC& P, std::vector<uint8_t>& bmat) {
+void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BConvTC& P, std::vector<uint8_t>& bmat,
+                   const std::vector<u64>* corr) {
     std::memset(&P, 0, sizeof(P));
     P.n_in = (int)src.size();
     P.n_out = (int)dst.size();
@@ -205,6 +206,15 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
                                  (n % 8) * 16 + (k % 16);
                     bmat[off] = (uint8_t)((v >> (8 * b)) & 0xFF);
                 }
+            }
+        }
+        if (corr) {                                            // column k = 5 n_in: (-Q_in) mod t, unshifted
+            const u64 v = (*corr)[t] % m;
+            for (int b = 0; b < 5; ++b) {
+                const int h = t / P.J, n = 5 * (t - h * P.J) + b, k = 5 * P.n_in;
+                size_t off = (size_t)h * BCTC_PART_ROWS * 64 + (size_t)(n / 8) * 512 + (k / 16) * 128 + (n % 8) * 16 +
+                             (k % 16);
+                bmat[off] = (uint8_t)((v >> (8 * b)) & 0xFF);
             }
         }
     }
@@ -383,7 +393,31 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
             if (c->num_t) {                                     // KLSS ModUp: digit -> T
                 c->klss_up_tc.resize(c->num_q);
                 c->klss_up_boff.resize(c->num_q);
+                c->klss_rec_tc.resize(c->num_q);
+                c->klss_rec_boff.resize(c->num_q);
                 std::vector<u64> tm(c->mod.begin() + nl, c->mod.begin() + nl + c->num_t);
+                if (5 * c->num_t >= 64) fits = false;           // Recover's correction column needs K = 5 alpha' + 1 <= 64
+                for (size_t gi = 0; gi < c->klss_groups.size(); ++gi) {   // Recover Limbs: T -> group (centred)
+                    std::vector<u64> dm, corr;
+                    for (int id : c->klss_groups[gi])
+                        if (id <= l || id >= c->num_q) {
+                            const u64 pm = c->mod[id];
+                            u64 T = 1;
+                            for (u64 t : tm) T = mulm(T, t % pm, pm);
+                            dm.push_back(pm);
+                            corr.push_back((pm - T) % pm);
+                        }
+                    BConvTC P;
+                    if (!dm.empty()) {
+                        make_bconv_tc(tm, dm, P, bm, &corr);
+                        c->klss_rec_boff[l].push_back(all.size());
+                        all.insert(all.end(), bm.begin(), bm.end());
+                    } else {
+                        std::memset(&P, 0, sizeof(P));
+                        c->klss_rec_boff[l].push_back(0);
+                    }
+                    c->klss_rec_tc[l].push_back(P);
+                }
                 for (int j = 0; j < c->beta(l); ++j) {
                     std::vector<u64> sm;
                     for (int id : c->digits[l][j]) sm.push_back(c->mod[id]);
@@ -423,6 +457,8 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
                 for (int m = 0; m < c->num_t; ++m)
                     if (m != k) th = mulm(th, c->mod[nl + m] % pm, pm);
                 R.that_p[p][k] = mk_tw(th, pm);
+                R.that_lo[p][k] = (unsigned)(th & 0x3FFFF);
+                R.that_hi[p][k] = (unsigned)(th >> 18);
                 T = mulm(T, c->mod[nl + k] % pm, pm);
             }
             R.T_p[p] = mk_tw(T, pm);
