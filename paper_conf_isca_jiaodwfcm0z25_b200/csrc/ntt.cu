@@ -391,27 +391,44 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                 const u64* addr = cc ? ep.add1 : ep.add0;
                 if (addr) addr += bb * ep.add_b + (size_t)k * a.N;
                 u64* outr = (cc ? ep.out1 : ep.out0) + bb * ep.out_b + (size_t)k * a.N;
-                for (int e = tid; e < N2 * 8; e += NT) {
-                    const int i2 = e >> 3, p = e & 7;
-                    const size_t pos = row0 + (size_t)N1 * i2 + 2 * p;
-                    const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
-                    const uint4 av = ep.acc ? *reinterpret_cast<const uint4*>(accr + pos)
-                                            : make_uint4(0u, 0u, 0u, 0u);   // acc = 0 (KLSS ModDown)
-                    u64 r0 = shoup(sub_mod(((u64)av.y << 32) | av.x, ((u64)v.y << 32) | v.x, qq), pinv, qq);
-                    u64 r1 = shoup(sub_mod(((u64)av.w << 32) | av.z, ((u64)v.w << 32) | v.z, qq), pinv, qq);
-                    if (addr) {
-                        if (cc == 0 && ep.add_galois) {        // sigma_g(c0) of HROTATE, gathered
-                            const unsigned gg = ep.add_galois, msk = (unsigned)a.N - 1;
-                            const unsigned s0 = (unsigned)(((unsigned long long)gg * pos + (gg - 1) / 2) & msk);
-                            r0 = add_mod(r0, addr[s0], qq);
-                            r1 = add_mod(r1, addr[(s0 + gg) & msk], qq);
-                        } else {
-                            const uint4 dv = *reinterpret_cast<const uint4*>(addr + pos);
-                            r0 = add_mod(r0, ((u64)dv.y << 32) | dv.x, qq);
-                            r1 = add_mod(r1, ((u64)dv.w << 32) | dv.z, qq);
+                // 8 chunks of 2 coefficients per thread, in two rounds of 4 whose global loads are
+                // all issued before any of their results is used (the loads' L2 latency overlaps)
+                constexpr int U = 4;
+                static_assert((N2 * 8) % (NT * U) == 0, "epilogue rounds");
+                const bool gat = cc == 0 && ep.add_galois;
+#pragma unroll 1
+                for (int e0 = tid; e0 < N2 * 8; e0 += NT * U) {
+                    uint4 av[U], dv[U];
+                    size_t pos[U];
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        const int e = e0 + u * NT, i2 = e >> 3, p = e & 7;
+                        pos[u] = row0 + (size_t)N1 * i2 + 2 * p;
+                        av[u] = ep.acc ? __ldg(reinterpret_cast<const uint4*>(accr + pos[u]))
+                                       : make_uint4(0u, 0u, 0u, 0u);        // acc = 0 (KLSS ModDown)
+                        dv[u] = make_uint4(0u, 0u, 0u, 0u);
+                        if (addr) {
+                            if (gat) {                                       // sigma_g(c0), gathered
+                                const unsigned gg = ep.add_galois, msk = (unsigned)a.N - 1;
+                                const unsigned s0 = (unsigned)(((unsigned long long)gg * pos[u] + (gg - 1) / 2) & msk);
+                                const u64 x0 = __ldg(addr + s0), x1 = __ldg(addr + ((s0 + gg) & msk));
+                                dv[u] = make_uint4((unsigned)x0, (unsigned)(x0 >> 32), (unsigned)x1, (unsigned)(x1 >> 32));
+                            } else {
+                                dv[u] = __ldg(reinterpret_cast<const uint4*>(addr + pos[u]));
+                            }
                         }
                     }
-                    *reinterpret_cast<uint4*>(outr + pos) = make_uint4((unsigned)r0, (unsigned)(r0 >> 32), (unsigned)r1, (unsigned)(r1 >> 32));
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        const int e = e0 + u * NT, i2 = e >> 3, p = e & 7;
+                        const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
+                        u64 r0 = shoup(sub_mod(((u64)av[u].y << 32) | av[u].x, ((u64)v.y << 32) | v.x, qq), pinv, qq);
+                        u64 r1 = shoup(sub_mod(((u64)av[u].w << 32) | av[u].z, ((u64)v.w << 32) | v.z, qq), pinv, qq);
+                        r0 = add_mod(r0, ((u64)dv[u].y << 32) | dv[u].x, qq);       // add = 0 when absent
+                        r1 = add_mod(r1, ((u64)dv[u].w << 32) | dv[u].z, qq);
+                        *reinterpret_cast<uint4*>(outr + pos[u]) =
+                            make_uint4((unsigned)r0, (unsigned)(r0 >> 32), (unsigned)r1, (unsigned)(r1 >> 32));
+                    }
                 }
             }
         } else {

@@ -175,6 +175,9 @@ class Context:
         self.q, self.p, self.psi = list(q), list(p), list(psi)
         self.moduli = self.q + self.p
         at, ap = ctypes.c_int32(), ctypes.c_int32()
+        if not hasattr(lib(), "neo_klss_query"):     # an older build in an A/B run
+            self.alpha_t, self.alpha_p, self.t = 0, 0, []
+            return
         _check(lib().neo_klss_query(h, ctypes.byref(at), ctypes.byref(ap), None), "neo_klss_query")
         self.alpha_t, self.alpha_p = at.value, ap.value
         t = (ctypes.c_uint64 * max(1, self.alpha_p))()
