@@ -236,6 +236,9 @@ enum { NEO_PK_NTT_COL = 0, NEO_PK_NTT_ROW, NEO_PK_BCONV, NEO_PK_KEYIP, NEO_PK_CO
        NEO_PK_TENSOR, NEO_PK_AUTO, NEO_PK_MODSW, NEO_PK_RESCALE, NEO_PK_EW, NEO_PK_COUNT };
 neo_status neo_profile_enable(int32_t on);
 neo_status neo_profile_read(int32_t kind, double* total_ms, int32_t* launches);
+/* Diagnostics: the recorded launches in issue order (at most max): kind and start / end time
+ * in ms relative to the first recorded launch's start event (events of every stream). */
+int32_t neo_profile_timeline(int32_t max, int32_t* kinds, float* start_ms, float* end_ms);
 
 /* Diagnostics: when NEO_BCONV_DBG=1 is set in the environment before the first key-switch,
  * the tensor-core BConv records per-role clock64 stamps of CTA 0 (tiles 0..61: producer

@@ -605,6 +605,24 @@ neo_status neo_profile_enable(int32_t on) {
     return NEO_OK;
 }
 
+int32_t neo_profile_timeline(int32_t max, int32_t* kinds, float* start_ms, float* end_ms) {
+    if (g_recs.empty()) return 0;
+    cudaEventSynchronize(g_recs.back().b);
+    int n = 0;
+    for (const ProfRec& r : g_recs) {
+        if (n >= max) break;
+        float a = 0, b = 0;
+        cudaEventSynchronize(r.b);
+        cudaEventElapsedTime(&a, g_recs[0].a, r.a);
+        cudaEventElapsedTime(&b, g_recs[0].a, r.b);
+        if (kinds) kinds[n] = r.kind;
+        if (start_ms) start_ms[n] = a;
+        if (end_ms) end_ms[n] = b;
+        ++n;
+    }
+    return n;
+}
+
 neo_status neo_profile_read(int32_t kind, double* total_ms, int32_t* launches) {
     if (kind < 0 || kind >= PK_COUNT || !total_ms || !launches) FAIL(NEO_EINVAL, "bad profile kind or null output");
     double t = 0;

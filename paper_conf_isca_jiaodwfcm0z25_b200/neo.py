@@ -27,7 +27,7 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_keyip", "neo_moddown_combine", "neo_evk_create_hoisted", "neo_hrot_hoisted",
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
-            "neo_evk_create_klss", "neo_klss_query")
+            "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -145,6 +145,17 @@ def neo_profile_read() -> dict:
         _check(lib().neo_profile_read(k, ctypes.byref(ms), ctypes.byref(n)), "neo_profile_read")
         out[name] = (ms.value, n.value)
     return out
+
+
+def neo_profile_timeline(max_n: int = 4096):
+    """[(kind name, start_ms, end_ms)] of the launches recorded since neo_profile_enable."""
+    L = lib()
+    k = (ctypes.c_int32 * max_n)()
+    a, b = (ctypes.c_float * max_n)(), (ctypes.c_float * max_n)()
+    L.neo_profile_timeline.restype = _i32
+    L.neo_profile_timeline.argtypes = [_i32, _i32p, ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_float)]
+    n = L.neo_profile_timeline(max_n, k, a, b)
+    return [(PROFILE_KINDS[k[i]], a[i], b[i]) for i in range(n)]
 
 
 def neo_debug_bconv_trace():
