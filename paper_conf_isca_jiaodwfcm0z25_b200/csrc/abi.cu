@@ -678,6 +678,7 @@ neo_status neo_params_destroy(neo_ctx* c) {
     if (c->d_tab) cudaFree(c->d_tab);
     if (c->d_mods) cudaFree(c->d_mods);
     if (c->d_bmat) cudaFree(c->d_bmat);
+    if (c->d_rec) cudaFree(c->d_rec);
     delete c;
     return NEO_OK;
 }
