@@ -383,6 +383,21 @@ def run_neo(args):
     n_launch_dom = prof[dom][1] / args.steps
     achieved = bm[dom] / (step_ms[dom] / 1e3) / 1e9 if step_ms[dom] > 0 else None
     traffic = load_traffic(dom)
+    # NTT passes are co-bound by the FP64 pipe: FP64 ops per element per pass
+    # counted from the radix-2 structure (col: fwd 45.4 / inv 48.4, row: fwd 30.8 / inv 27.8),
+    # limb transforms per step at B=1, l=35: forward 430, inverse 122; peak = 63 DFMA-pipe
+    # ops/clk/SM (tools/microbench/pipes.cu) x SMs x the max SM clock.
+    fp64 = None
+    if dom in ("ntt_col", "ntt_row"):
+        ops = {"ntt_col": 430 * 45.4 + 122 * 48.4, "ntt_row": 430 * 30.8 + 122 * 27.8}[dom] * (1 << LOG_N) * B
+        try:
+            mhz = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["sm_max_mhz"])
+        except Exception:
+            mhz = 1965.0
+        pk = 63 * torch.cuda.get_device_properties(local).multi_processor_count * mhz * 1e6
+        ach = ops / (step_ms[dom] / 1e3)
+        fp64 = {"bound": "fp64", "achieved": ach / 1e12, "peak": pk / 1e12, "unit": "Tops/s", "frac": ach / pk,
+                "ops_per_step": ops}
     breakdown = {k: {"ms_per_step": round(step_ms[k], 5), "launches_per_step": prof[k][1] / args.steps,
                      "share": round(step_ms[k] / ms_step_ref, 4) if ms_step_ref > 0 else None,
                      "algo_GBps": round(bm[k] / (step_ms[k] / 1e3) / 1e9, 1) if step_ms[k] > 0 else None,
@@ -578,7 +593,7 @@ def run_neo(args):
                              "peak_source": peak_src, "unit": "GB/s",
                              "frac": achieved / peak if achieved else None, "traffic": traffic,
                              "launches_per_step": n_launch_dom,
-                             "algo_bytes_per_step": bm[dom]},
+                             "algo_bytes_per_step": bm[dom], "alt": fp64},
                 "step_roofline": {"algo_bytes_per_step": sum(bm.values()),
                                   "achieved": sum(bm.values()) / (ms_step / 1e3) / 1e9,
                                   "peak": peak, "unit": "GB/s",
