@@ -51,7 +51,7 @@ typedef enum {
 
 /* Operation codes for neo_workspace_size. */
 enum { NEO_OP_KEYSWITCH = 0, NEO_OP_HMULT = 1, NEO_OP_HROT = 2, NEO_OP_RESCALE = 3, NEO_OP_HROT_HOISTED = 4,
-       NEO_OP_DOUBLE_RESCALE = 5 };
+       NEO_OP_DOUBLE_RESCALE = 5, NEO_OP_MODRAISE = 6 };
 
 /* Parameter description (Table 1, Table 4).
  *  log_n      : log2 N; this build supports 12 and 16 (N = 2^12 tiny config, 2^16 Set-B).
@@ -217,6 +217,23 @@ neo_status neo_hadd(const neo_ctx* ctx, const uint64_t* ct_a, const uint64_t* ct
                     uint64_t* ct_out, int32_t batch, neo_stream_t stream);
 neo_status neo_padd(const neo_ctx* ctx, const uint64_t* ct_in, const uint64_t* pt, int32_t level,
                     uint64_t* ct_out, int32_t batch, neo_stream_t stream);
+
+/* HSUB: (a0 - b0, a1 - b1), same conventions as neo_hadd. */
+neo_status neo_hsub(const neo_ctx* ctx, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level,
+                    uint64_t* ct_out, int32_t batch, neo_stream_t stream);
+
+/* Bootstrapping's ModRaise (the first step of PackBootstrap, L529):
+ * ct_in [batch][2][1][N] mod q_0 (NTT form) -> ct_out [batch][2][level+1][N]: each coefficient's
+ * centred representative in (-q_0/2, q_0/2] reduced mod q_0..q_level, NTT form, so that
+ * decryption gives m + q_0 I for a small integer polynomial I.
+ * ws >= neo_workspace_size(ctx, NEO_OP_MODRAISE, level, batch). */
+neo_status neo_modraise(const neo_ctx* ctx, const uint64_t* ct_in, int32_t level, uint64_t* ct_out,
+                        int32_t batch, void* ws, size_t ws_bytes, neo_stream_t stream);
+
+/* Level drop (modulus switch down without scaling): the first level_out+1 limbs of each
+ * component, ct_in [batch][2][level_in+1][N] -> ct_out [batch][2][level_out+1][N]. */
+neo_status neo_drop_levels(const neo_ctx* ctx, const uint64_t* ct_in, int32_t level_in, uint64_t* ct_out,
+                           int32_t level_out, int32_t batch, neo_stream_t stream);
 
 /* Thread-local message describing the last non-OK status returned on this thread. */
 const char* neo_last_error(void);

@@ -1,0 +1,238 @@
+"""CPU ORACLE of CKKS bootstrapping (PackBootstrap of L529) -- TEST
+INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+``--impl reference`` legs may import this module; it shares no code with the CUDA path.
+
+The paper names bootstrapping's three parts (CoeffToSlot, EvalMod, SlotToCoeff, L529) and the
+Double Rescale it needs at 36-bit words (L138, L151) but gives no algorithm or parameters (it
+cites Lattigo [34]).  Reading "BOOT" -- the textbook sparse-slot bootstrapping of
+Cheon, Han, Kim, Kim, Song (EUROCRYPT'18), built only from the operations pinned elsewhere
+(HROTATE, HMULT, PMULT, HADD/HSUB, Rescale) plus ModRaise:
+
+  ModRaise  ct mod q_0 -> mod Q_L, coefficients lifted centred: m + q_0 I, I small
+  SubSum    sum of the rotations by n 2^j: the trace onto the degree-2n subring (x M = N / 2n)
+  CoeffToSlot  slots <- A z with A = W^-1 / M, W[k][j] = xi^(j 5^k), xi = e^(i pi / 2n): the slot
+            j then holds (p_{Mj} + i p_{M(j+n)}) / q_0 (diagonal method, one PMULT level)
+  split     Re = (w + conj w) / 2, Im = (w - conj w) / 2i   (conjugation = HROTATE, g = 2N - 1)
+  EvalMod   y = theta t (theta = 2 pi / 2^r), E = sum_{k<=7} (i y)^k / k!, E <- E^2 r times
+            (= exp(2 pi i t)), f = (E - conj E) (-i / 4 pi) = sin(2 pi t) / 2 pi ~ t mod 1 = m / q_0
+  combine   f(Re) + i f(Im)  (i = the monomial X^(N/2): PMULT by a scale-1 plaintext, exact)
+  SlotToCoeff  slots <- W v (diagonal method): the message slots, value z Delta_in / q_0
+
+Every plaintext constant is encoded at a scale that makes the next rescale restore the
+ciphertext's scale, so scales are tracked exactly; the constants are returned so the GPU run
+uses the same ones (tests/test_gpu_boot.py: bit-exact).  Pinned by decoding (the output
+decrypts to the input slots) and by ModRaise's exact big-integer identity."""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import ckks
+
+D_TAYLOR = 7                                 # degree of the exp Taylor polynomial (powers y .. y^7)
+
+
+@dataclass
+class BootParams:
+    prm: ckks.Params
+    n: int                                   # complex slots (sparse packing), n | N/2
+    r: int                                   # squarings in EvalMod
+    h: int = 192                             # secret Hamming weight (bounds I)
+
+    @property
+    def M(self) -> int:
+        return self.prm.N // (2 * self.n)
+
+    @property
+    def top(self) -> int:
+        return self.prm.max_level
+
+    def levels_used(self) -> int:            # CtS 1, EvalMod 1 + 3 + 1 + r + 1, StC 1
+        return 1 + (1 + 3 + 1 + self.r + 1) + 1
+
+    def rotations(self) -> list[int]:
+        """Galois elements: SubSum (rotations by n 2^j), the diagonal method (1..n-1), conj."""
+        N = self.prm.N
+        gs = [pow(5, self.n << j, 2 * N) for j in range(int(math.log2(self.M)))]
+        gs += [pow(5, d, 2 * N) for d in range(1, self.n)]
+        return sorted(set(gs)) + [2 * N - 1]
+
+
+def tiny() -> BootParams:
+    """Test set: N = 2^12, 19 Q limbs + 2 P limbs (dnum 10: alpha = 2), 8 slots, r = 9, h = 32."""
+    return BootParams(ckks.Params(12, 19, 2, 10), n=8, r=9, h=32)
+
+
+def set_b() -> BootParams:
+    """Set-B (Table 4) with 8 sparse slots, r = 12 squarings (h = 192: |I| up to ~100)."""
+    return BootParams(ckks.set_b(), n=8, r=12, h=192)
+
+
+# --------------------------------------------------------------------------- slot algebra
+
+def _xi_matrix(n: int) -> np.ndarray:
+    """W[k][j] = xi^(j 5^k), xi = e^(i pi / 2n): slots of a degree-2n subring polynomial."""
+    e5 = [pow(5, k, 4 * n) for k in range(n)]
+    return np.array([[np.exp(1j * math.pi * ((j * e) % (4 * n)) / (2 * n)) for j in range(n)] for e in e5])
+
+
+def _diagonals(A: np.ndarray) -> list[np.ndarray]:
+    n = A.shape[0]
+    return [np.array([A[k][(k + d) % n] for k in range(n)]) for d in range(n)]
+
+
+def _pt(bp: BootParams, slots_n: np.ndarray, scale: float, level: int) -> np.ndarray:
+    """Plaintext (NTT form, level) whose full-slot vector is slots_n tiled, at `scale`."""
+    prm = bp.prm
+    ids = list(range(level + 1))
+    m = ckks.encode(prm.N, np.tile(np.asarray(slots_n, dtype=complex), bp.M), scale)
+    return ckks.ntt(prm, ckks.reduce_signed(prm, m, ids), ids)
+
+
+def _monomial(prm: ckks.Params, k: int, sign: int, level: int) -> np.ndarray:
+    """NTT form of sign * X^k (an exact scale-1 plaintext): X^(N/2) multiplies every slot by i."""
+    ids = list(range(level + 1))
+    c = np.zeros(prm.N, dtype=np.int64)
+    c[k] = sign
+    return ckks.ntt(prm, ckks.reduce_signed(prm, c, ids), ids)
+
+
+# --------------------------------------------------------------------------- ops
+
+def modraise(prm: ckks.Params, ct: np.ndarray, level: int) -> np.ndarray:
+    """ct [2][1][N] mod q_0 (NTT form) -> [2][level+1][N]: centred lift of each coefficient."""
+    q0 = prm.q[0]
+    ids = list(range(level + 1))
+    out = []
+    for c in range(2):
+        coef = ckks.intt(prm, ct[c][0:1], [0])[0].astype(np.int64)
+        signed = np.where(2 * coef > q0, coef - q0, coef)
+        out.append(ckks.ntt(prm, ckks.reduce_signed(prm, signed, ids), ids))
+    return np.stack(out)
+
+
+def hsub(prm, a, b, level):
+    ids = list(range(level + 1))
+    return np.stack([ckks.sub(prm, a[0], b[0], ids), ckks.sub(prm, a[1], b[1], ids)])
+
+
+def drop(ct: np.ndarray, level: int) -> np.ndarray:
+    return np.ascontiguousarray(ct[:, : level + 1])
+
+
+# --------------------------------------------------------------------------- keys
+
+def boot_keys(bp: BootParams, s: np.ndarray, seed: int) -> dict:
+    """Hybrid evaluation keys: 'relin' and one rotation key per Galois element of bp.rotations()."""
+    keys = {"relin": ckks.relin_key(bp.prm, s, seed)}
+    for t, g in enumerate(bp.rotations()):
+        keys[g] = ckks.rot_key(bp.prm, s, g, seed + 1 + t)
+    return keys
+
+
+# --------------------------------------------------------------------------- bootstrapping
+
+def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None = None):
+    """Bootstrap ct0 ([2][1][N], level 0).  Returns (ct, level, scale, consts) where the output
+    decodes (at `scale` Delta_in / q_0) to the input's slots.  `consts` (plaintexts by name) are
+    generated when None and returned, so another implementation can replay the same run."""
+    prm, N, n, M = bp.prm, bp.prm.N, bp.n, bp.M
+    gen = consts is None
+    consts = {} if gen else consts
+    q = prm.q
+
+    def const(name, make):
+        if gen:
+            consts[name] = make()
+        return consts[name]
+
+    def rot(ct, g, lv):
+        return ckks.hrot(prm, ct, g, lv, keys[g])
+
+    # ModRaise: value (m + q_0 I) / q_0 at scale q_0
+    L = bp.top
+    ct = modraise(prm, ct0, L)
+    scale = float(q[0])
+    # SubSum: M x the subring projection
+    for j in range(int(math.log2(M))):
+        ct = ckks.hadd(prm, ct, rot(ct, pow(5, n << j, 2 * N), L), L)
+
+    def lintrans(ct, lv, A, tag):        # slots <- A slots (diagonal method), scale kept, one level
+        acc = None
+        for d, dg in enumerate(_diagonals(A)):
+            src = ct if d == 0 else rot(ct, pow(5, d, 2 * N), lv)
+            pt = const(f"{tag}_{d}", lambda dg=dg: _pt(bp, dg, float(q[lv]), lv))
+            t = ckks.pmult(prm, src, pt, lv)
+            acc = t if acc is None else ckks.hadd(prm, acc, t, lv)
+        return ckks.rescale(prm, acc, lv)
+
+    W = _xi_matrix(n)
+    ct = lintrans(ct, L, np.linalg.inv(W) / M, "cts")              # CoeffToSlot
+    lv = L - 1
+    cj = rot(ct, 2 * N - 1, lv)
+    x1 = ckks.hadd(prm, ct, cj, lv)                                 # 2 Re(w)
+    x2 = ckks.pmult(prm, hsub(prm, ct, cj, lv), const("mono_mi", lambda: _monomial(prm, N // 2, -1, lv)), lv)  # 2 Im(w)
+    sx = 2.0 * scale                                                # value Re(w), Im(w) at scale 2 q_0
+
+    def evalmod(x, lv, sx, tag):
+        theta = 2 * math.pi / (1 << bp.r)
+        S = float(q[lv])                                            # y's scale after the theta product
+        y1 = ckks.rescale(prm, ckks.pmult(prm, x, const(f"{tag}theta", lambda: _pt(bp, np.full(n, theta), S * q[lv] / sx, lv)), lv), lv)
+        lv -= 1
+        sc = {1: S}
+        pw = {1: (y1, lv)}
+
+        def mul(a, b):                                              # y^a y^b, levels aligned, rescaled
+            (ca, la), (cb, lb) = pw[a], pw[b]
+            l0 = min(la, lb)
+            prod = ckks.hmult(prm, drop(ca, l0), drop(cb, l0), l0, keys["relin"])
+            pw[a + b] = (ckks.rescale(prm, prod, l0), l0 - 1)
+            sc[a + b] = sc[a] * sc[b] / q[l0]
+        mul(1, 1)
+        mul(2, 1)
+        mul(2, 2)
+        mul(4, 1)
+        mul(4, 2)
+        mul(4, 3)
+        lt = min(pw[k][1] for k in pw)                              # common level of the terms
+        St = float(q[lt])                                           # their common scale
+        E = None
+        for k in range(1, D_TAYLOR + 1):
+            ck, lk = pw[k]
+            coef = (1j ** k) / math.factorial(k)
+            pt = const(f"{tag}c{k}", lambda coef=coef, lk=lk, k=k: _pt(bp, np.full(n, coef), St * q[lk] / sc[k], lk))
+            term = drop(ckks.rescale(prm, ckks.pmult(prm, ck, pt, lk), lk), lt - 1)
+            E = term if E is None else ckks.hadd(prm, E, term, lt - 1)
+        lv = lt - 1
+        E = ckks.padd(prm, E, const(f"{tag}c0", lambda: _pt(bp, np.ones(n), St, lv)), lv)
+        s_e = St
+        for _ in range(bp.r):                                       # E <- E^2: exp(2 pi i t)
+            E = ckks.rescale(prm, ckks.hmult(prm, E, E, lv, keys["relin"]), lv)
+            s_e = s_e * s_e / q[lv]
+            lv -= 1
+        cE = rot(E, 2 * N - 1, lv)
+        Dm = hsub(prm, E, cE, lv)                                   # 2 i sin(2 pi t)
+        k = -1j / (4 * math.pi)
+        f = ckks.rescale(prm, ckks.pmult(prm, Dm, const(f"{tag}sin", lambda: _pt(bp, np.full(n, k), float(q[lv]), lv)), lv), lv)
+        return f, lv - 1, s_e
+
+    f1, lv1, s1 = evalmod(x1, lv, sx, "re")
+    f2, lv2, s2 = evalmod(x2, lv, sx, "im")
+    assert (lv1, s1) == (lv2, s2)
+    lv = lv1
+    w = ckks.hadd(prm, f1, ckks.pmult(prm, f2, const("mono_i", lambda: _monomial(prm, N // 2, 1, lv)), lv), lv)
+    out = lintrans(w, lv, W, "stc")                                 # SlotToCoeff
+    return out, lv - 1, s1, consts
+
+
+def encrypt_sparse(bp: BootParams, z: np.ndarray, delta: float, s: np.ndarray, seed: int) -> np.ndarray:
+    """Encrypt n slots (tiled to the full N/2) at level 0, scale delta: ct [2][1][N]."""
+    m = ckks.encode(bp.prm.N, np.tile(z, bp.M), delta)
+    return ckks.encrypt(bp.prm, m, s, 0, seed)
+
+
+def decode_sparse(bp: BootParams, ct: np.ndarray, level: int, scale: float, s: np.ndarray) -> np.ndarray:
+    m = ckks.crt_centered(bp.prm, ckks.decrypt_residues(bp.prm, ct, s, level), list(range(level + 1)))
+    return ckks.decode(bp.prm.N, m, scale)[: bp.n]

@@ -704,6 +704,7 @@ size_t neo_workspace_size(const neo_ctx* c, int32_t op, int32_t level, int32_t b
         }
         case NEO_OP_RESCALE: return level >= 1 ? rescale_ws(c, level, batch) * sizeof(u64) : 0;
         case NEO_OP_DOUBLE_RESCALE: return level >= 2 ? ds_ws(c, level, batch) * sizeof(u64) : 0;
+        case NEO_OP_MODRAISE: return (size_t)2 * batch * c->N * (2 + level) * sizeof(u64);
         default: return 0;
     }
 }
@@ -1120,6 +1121,44 @@ neo_status neo_hadd(const neo_ctx* c, const uint64_t* ct_a, const uint64_t* ct_b
 neo_status neo_padd(const neo_ctx* c, const uint64_t* ct_in, const uint64_t* pt, int32_t level, uint64_t* ct_out,
                     int32_t batch, neo_stream_t st) {
     return ew_api(c, EW_PADD, ct_in, pt, level, ct_out, batch, st);
+}
+
+neo_status neo_hsub(const neo_ctx* c, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level, uint64_t* ct_out,
+                    int32_t batch, neo_stream_t st) {
+    return ew_api(c, EW_HSUB, ct_a, ct_b, level, ct_out, batch, st);
+}
+
+neo_status neo_modraise(const neo_ctx* c, const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch,
+                        void* ws, size_t ws_bytes, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(ct_in, "ct_in"));
+    TRY(check_ptr(ct_out, "ct_out"));
+    TRY(check_ws(c, NEO_OP_MODRAISE, level, batch, ws, ws_bytes));
+    const int N = c->N, B2 = 2 * batch, Lq = level + 1;
+    u64* w = static_cast<u64*>(ws);
+    u64* coef = w;                                   // [2B][N]
+    u64* tmp = coef + (size_t)B2 * N;                // NTT intermediate [2B][Lq][N]
+    cudaStream_t s = S(st);
+    int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
+    so[0] = 0; dof[0] = 0; pr[0] = 0;
+    TRY(ntt_rows(c, false, ct_in, (long long)N, so, coef, (long long)N, dof, pr, 1, tmp, B2, s));
+    LAUNCH(PK_MODSW, s, launch_modraise(coef, ct_out, c->d_mods, Lq, N, B2, s));
+    for (int i = 0; i < Lq; ++i) { so[i] = dof[i] = pr[i] = i; }
+    return ntt_rows(c, true, ct_out, (long long)Lq * N, so, ct_out, (long long)Lq * N, dof, pr, Lq, tmp, B2, s);
+}
+
+neo_status neo_drop_levels(const neo_ctx* c, const uint64_t* ct_in, int32_t level_in, uint64_t* ct_out,
+                           int32_t level_out, int32_t batch, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level_in, batch));
+    if (level_out < 0 || level_out > level_in) FAIL(NEO_EINVAL, "need 0 <= level_out <= level_in");
+    TRY(check_ptr(ct_in, "ct_in"));
+    TRY(check_ptr(ct_out, "ct_out"));
+    LAUNCH(PK_EW, S(st), launch_drop(ct_in, ct_out, level_in + 1, level_out + 1, c->N, batch, S(st)));
+    return NEO_OK;
 }
 
 neo_status neo_double_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t level, uint64_t* ct_out,

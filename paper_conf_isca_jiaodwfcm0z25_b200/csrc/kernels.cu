@@ -198,6 +198,11 @@ k_ew(const __grid_constant__ EwArgs A) {
         const ulonglong2 b1 = *reinterpret_cast<const ulonglong2*>(A.b + ct + cs);
         y0 = make_ulonglong2(add_mod(x0.x, b0.x, m.q), add_mod(x0.y, b0.y, m.q));
         y1 = make_ulonglong2(add_mod(x1.x, b1.x, m.q), add_mod(x1.y, b1.y, m.q));
+    } else if (A.op == EW_HSUB) {
+        const ulonglong2 b0 = *reinterpret_cast<const ulonglong2*>(A.b + ct);
+        const ulonglong2 b1 = *reinterpret_cast<const ulonglong2*>(A.b + ct + cs);
+        y0 = make_ulonglong2(sub_mod(x0.x, b0.x, m.q), sub_mod(x0.y, b0.y, m.q));
+        y1 = make_ulonglong2(sub_mod(x1.x, b1.x, m.q), sub_mod(x1.y, b1.y, m.q));
     } else {
         const ulonglong2 p = *reinterpret_cast<const ulonglong2*>(A.b + pt);
         if (A.op == EW_PMULT) {
@@ -210,6 +215,36 @@ k_ew(const __grid_constant__ EwArgs A) {
     }
     *reinterpret_cast<ulonglong2*>(A.out + ct) = y0;
     *reinterpret_cast<ulonglong2*>(A.out + ct + cs) = y1;
+}
+
+// ------------------------------------------------------------------ ModRaise (bootstrapping)
+// c in [0, q_0) -> the centred representative in (-q_0/2, q_0/2] reduced mod q_i
+__global__ void __launch_bounds__(256)
+k_modraise(const u64* __restrict__ coef, u64* __restrict__ out, const ModQ* __restrict__ mods, int limbs, int N) {
+    pdl_wait();
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int i = blockIdx.y, bc = blockIdx.z;
+    if (n >= N) return;
+    const u64 q0 = mods[0].q, qi = mods[i].q;
+    const u64 c = coef[(size_t)bc * N + n];
+    u64 r;
+    if (2 * c > q0) {                                           // negative: c - q0
+        const u64 m = q0 - c;                                   // |value| < q_0 / 2 < q_i
+        r = m == 0 ? 0 : qi - (m % qi);
+    } else {
+        r = c % qi;
+    }
+    out[((size_t)bc * limbs + i) * N + n] = r;
+}
+
+__global__ void __launch_bounds__(256)
+k_drop(const u64* __restrict__ in, u64* __restrict__ out, int li, int lo, int N) {
+    pdl_wait();
+    const int n = 2 * (blockIdx.x * blockDim.x + threadIdx.x);
+    const int i = blockIdx.y, bc = blockIdx.z;
+    if (n >= N) return;
+    *reinterpret_cast<ulonglong2*>(out + ((size_t)bc * lo + i) * N + n) =
+        *reinterpret_cast<const ulonglong2*>(in + ((size_t)bc * li + i) * N + n);
 }
 
 // ------------------------------------------------------------------ Double Rescale (L138, L151)
@@ -248,6 +283,12 @@ k_pack5(const u64* __restrict__ in, uint32_t* __restrict__ lo, uint8_t* __restri
 // ------------------------------------------------------------------ launchers
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_ew, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);
+}
+cudaError_t launch_modraise(const u64* coef, u64* out, const ModQ* mods, int limbs, int N, int bc, cudaStream_t st) {
+    return launch_k(k_modraise, dim3((N + 255) / 256, limbs, bc), dim3(256), 0, st, coef, out, mods, limbs, N);
+}
+cudaError_t launch_drop(const u64* in, u64* out, int li, int lo, int N, int batch, cudaStream_t st) {
+    return launch_k(k_drop, dim3((N / 2 + 255) / 256, lo, 2 * batch), dim3(256), 0, st, in, out, li, lo, N);
 }
 cudaError_t launch_ds_corr(const DsArgs& A, int bc, cudaStream_t st) {
     return launch_k(k_ds_corr, dim3((A.N + 255) / 256, bc), dim3(256), 0, st, A);

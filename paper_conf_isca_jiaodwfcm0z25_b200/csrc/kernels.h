@@ -47,7 +47,7 @@ struct RescaleArgs {
 
 // Element-wise ciphertext ops (L133-135) on [batch][2][limbs][N] ciphertexts and
 // [batch][limbs][N] plaintexts, NTT form.
-enum EwOp { EW_PMULT = 0, EW_HADD = 1, EW_PADD = 2 };
+enum EwOp { EW_PMULT = 0, EW_HADD = 1, EW_PADD = 2, EW_HSUB = 3 };
 struct EwArgs {
     const u64* a;          // ct [B][2][limbs][N]
     const u64* b;          // ct (HADD) or plaintext [B][limbs][N]
@@ -68,6 +68,10 @@ struct DsArgs {
 };
 
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st);
+// ModRaise: coef[bc][N] (coefficient form mod q_0, canonical) -> out[bc][i][N] = centred lift mod q_i
+cudaError_t launch_modraise(const u64* coef, u64* out, const ModQ* mods, int limbs, int N, int bc, cudaStream_t st);
+// drop limbs: in [B][2][li][N] -> out [B][2][lo][N] (lo <= li), the first lo limbs of each component
+cudaError_t launch_drop(const u64* in, u64* out, int li, int lo, int N, int batch, cudaStream_t st);
 cudaError_t launch_ds_corr(const DsArgs& A, int bc, cudaStream_t st);
 cudaError_t launch_bconv(const BConvTab& T, const BConvIO& io, int N, int batch, cudaStream_t st);
 cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t st);

@@ -17,7 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libneo.so")
 
 NEO_OP_KEYSWITCH, NEO_OP_HMULT, NEO_OP_HROT, NEO_OP_RESCALE, NEO_OP_HROT_HOISTED = 0, 1, 2, 3, 4
-NEO_OP_DOUBLE_RESCALE = 5
+NEO_OP_DOUBLE_RESCALE, NEO_OP_MODRAISE = 5, 6
 _STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM", 4: "NEO_ECUDA",
            5: "NEO_ENCCL", 6: "NEO_ENOPRIME"}
 
@@ -27,7 +27,8 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_keyip", "neo_moddown_combine", "neo_evk_create_hoisted", "neo_hrot_hoisted",
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
-            "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline")
+            "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline", "neo_hsub", "neo_modraise",
+            "neo_drop_levels")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -82,6 +83,9 @@ def lib() -> ctypes.CDLL:
             "neo_hadd": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
             "neo_padd": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
             "neo_evk_create_klss": [_vp, _vp, ctypes.POINTER(_vp)],
+            "neo_hsub": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
+            "neo_modraise": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+            "neo_drop_levels": [_vp, _vp, _i32, _vp, _i32, _i32, _vp],
             "neo_klss_query": [_vp, _i32p, _i32p, _u64p],
         }
         for name, args in sig.items():
@@ -309,6 +313,21 @@ def neo_hadd(ctx: Context, ct_a, ct_b, level: int, ct_out, batch: int, stream=No
 def neo_padd(ctx: Context, ct_in, pt, level: int, ct_out, batch: int, stream=None):
     _check(lib().neo_padd(ctx.handle, _ptr(ct_in), _ptr(pt), level, _ptr(ct_out), batch, _stream(stream)),
            "neo_padd")
+
+
+def neo_hsub(ctx: Context, ct_a, ct_b, level: int, ct_out, batch: int, stream=None):
+    _check(lib().neo_hsub(ctx.handle, _ptr(ct_a), _ptr(ct_b), level, _ptr(ct_out), batch, _stream(stream)),
+           "neo_hsub")
+
+
+def neo_modraise(ctx: Context, ct_in, level: int, ct_out, batch: int, ws, stream=None):
+    _check(lib().neo_modraise(ctx.handle, _ptr(ct_in), level, _ptr(ct_out), batch, _ptr(ws), ws.numel() * 8,
+                              _stream(stream)), "neo_modraise")
+
+
+def neo_drop_levels(ctx: Context, ct_in, level_in: int, ct_out, level_out: int, batch: int, stream=None):
+    _check(lib().neo_drop_levels(ctx.handle, _ptr(ct_in), level_in, _ptr(ct_out), level_out, batch,
+                                 _stream(stream)), "neo_drop_levels")
 
 
 def neo_keyip(ctx: Context, evk: EvalKey, dhat, limb_ids, beta: int, acc, batch: int, stream=None):
