@@ -1,0 +1,43 @@
+"""GPU parity of bootstrapping (reading BOOT): the GPU run of
+paper_conf_isca_jiaodwfcm0z25_b200.boot with the oracle's keys and plaintext constants is
+bit-exact against oracle/boot.py, and decodes to the input slots."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import boot, ckks
+
+pytestmark = pytest.mark.gpu
+
+neo = pytest.importorskip("paper_conf_isca_jiaodwfcm0z25_b200.neo")
+gboot = pytest.importorskip("paper_conf_isca_jiaodwfcm0z25_b200.boot")
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint64)).cuda()
+
+
+def test_bootstrap_bit_exact_and_decodes():
+    bp = boot.tiny()
+    prm = bp.prm
+    s = ckks.secret(prm, 21, bp.h)
+    keys_np = boot.boot_keys(bp, s, 500)
+    z = synth.complex_slots(23, bp.n)
+    delta = 2.0 ** 31
+    ct0 = boot.encrypt_sparse(bp, z, delta, s, 25)
+    want, lv, scale, consts = boot.bootstrap(bp, ct0, keys_np)
+
+    ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+    assert gboot.rotations(prm.N, bp.n) == bp.rotations()
+    keys = {k: neo.EvalKey(ctx, dev(v)) for k, v in keys_np.items()}
+    cl = gboot.const_levels(bp.top, bp.n, bp.r)
+    assert set(cl) == set(consts) and all(consts[k].shape[0] == cl[k] + 1 for k in cl)
+    b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()})
+    got, glv = b.run(dev(ct0[None]))
+    torch.cuda.synchronize()
+    assert glv == lv
+    got = got.cpu().numpy()[0]
+    assert np.array_equal(got, want)
+    zz = boot.decode_sparse(bp, got, lv, scale * delta / prm.q[0], s)
+    assert np.max(np.abs(zz - z)) < 4e-3
