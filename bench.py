@@ -19,6 +19,7 @@ from __future__ import annotations
 
 import argparse
 import json
+import math
 import os
 import statistics
 import subprocess
@@ -49,6 +50,8 @@ def parse():
     ap.add_argument("--no-hoisted", action="store_true")
     ap.add_argument("--no-klss", action="store_true",
                     help="skip the KLSS vs Hybrid key-switch comparison at Set-C (SURVEY §8(f) row 1)")
+    ap.add_argument("--no-boot", action="store_true",
+                    help="skip the bootstrapping timing (Set-B, 8 sparse slots; SURVEY §8(f) row 2)")
     ap.add_argument("--batch-hrot", type=int, default=256,
                     help="BASELINE configs[2]: this many independent HRot key-switches (one shared key) "
                          "split data-parallel over the ranks, plus a batch sweep up to it (0 = skip)")
@@ -518,6 +521,49 @@ def run_neo(args):
         cctx.close()
         torch.cuda.empty_cache()
 
+    # SURVEY §8(f) row 2 / BASELINE metric "bootstrap ms": one sparse-slot bootstrapping
+    # (paper_conf_isca_jiaodwfcm0z25_b200.boot: ModRaise, SubSum, CoeffToSlot, EvalMod,
+    # SlotToCoeff; n = 8 slots, r = 12 squarings, 20 levels) at Set-B on every rank (DP).  Keys
+    # and plaintext constants are uniform residues made on the device (timing is data-independent;
+    # correctness: tests/test_gpu_boot.py).
+    boot_block = None
+    if not args.no_boot:
+        from paper_conf_isca_jiaodwfcm0z25_b200 import boot as gboot
+        nb, rb = 8, 12
+        gen = torch.Generator(device="cuda")
+        gen.manual_seed(seed + 123)
+        rnd = lambda *shape: torch.randint(0, 1 << 35, shape, dtype=torch.int64, device="cuda",
+                                           generator=gen).view(torch.uint64)
+        bkeys = {"relin": neo.EvalKey(ctx, rnd(DNUM, 2, NUM_Q + NUM_P, N))}
+        for gg in gboot.rotations(N, nb):
+            bkeys[gg] = neo.EvalKey(ctx, rnd(DNUM, 2, NUM_Q + NUM_P, N))
+        bconsts = {k: rnd(l + 1, N) for k, l in gboot.const_levels(LEVEL, nb, rb).items()}
+        bt = gboot.Bootstrapper(ctx, nb, rb, bkeys, bconsts)
+        bct = rnd(1, 2, 1, N)
+        for _ in range(2):
+            bt.run(bct)
+        torch.cuda.synchronize()
+        barrier()
+        nboot = 5
+        b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        b0.record()
+        for _ in range(nboot):
+            bt.run(bct)
+        b1.record()
+        torch.cuda.synchronize()
+        bms = b0.elapsed_time(b1) / nboot
+        if world > 1:
+            t = torch.tensor([bms], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            bms = float(t.item())
+        nks = int(math.log2(N // (2 * nb))) + 2 * (nb - 1) + 2 + 2 * (7 + rb)
+        boot_block = {"config": "Set-B (N=2^16, L=35, dnum=3), 8 sparse slots, r=12 squarings, levels 35 -> 15",
+                      "ms_per_bootstrap": round(bms, 3), "value": world / (bms / 1e3), "unit": "bootstraps/s",
+                      "key_switches": nks,
+                      "timing": f"CUDA events around {nboot} runs after 2 warm-ups, max over ranks"}
+        del bkeys, bconsts, bt
+        torch.cuda.empty_cache()
+
     # end-to-end through the public API with pinned host buffers: every step copies its three
     # input ciphertexts host->device and both results device->host.  Copies run on their own
     # streams, double-buffered, so the H2D of step k+1 and the D2H of step k-1 overlap the
@@ -600,7 +646,7 @@ def run_neo(args):
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted,
-                "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block,
+                "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}
         print(json.dumps(line), flush=True)
