@@ -59,53 +59,66 @@ class Bootstrapper:
         self.N = ctx.N
         self.top = ctx.num_q - 1
         ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_MODRAISE)
-        wsn = max(ctx.workspace_size(op, self.top, 1) for op in ops)
+        wsn = max(ctx.workspace_size(op, self.top, 2) for op in ops)
+        self._stack = {}
         self.ws = torch.empty(wsn // 8, dtype=torch.uint64, device="cuda")
 
-    def _ct(self, level):
-        return torch.empty((1, 2, level + 1, self.N), dtype=torch.uint64, device="cuda")
+    def _ct(self, level, B=1):
+        return torch.empty((B, 2, level + 1, self.N), dtype=torch.uint64, device="cuda")
 
     # ---- primitive ops (each one C-ABI call)
+    # a ciphertext tensor is [B][2][l+1][N]; B = 2 runs EvalMod's real and imaginary halves as
+    # one batch (plaintexts: one per batch entry, stacked)
     def rot(self, ct, g, lv):
-        out = self._ct(lv)
-        neo.neo_hrot(self.ctx, self.keys[g], g, ct, lv, out, 1, self.ws, self.stream)
+        B = ct.shape[0]
+        out = self._ct(lv, B)
+        neo.neo_hrot(self.ctx, self.keys[g], g, ct, lv, out, B, self.ws, self.stream)
         return out
 
-    def add(self, a, b, lv):
-        out = self._ct(lv)
-        neo.neo_hadd(self.ctx, a, b, lv, out, 1, self.stream)
+    def add(self, a, b, lv, out=None):
+        out = self._ct(lv, a.shape[0]) if out is None else out
+        neo.neo_hadd(self.ctx, a, b, lv, out, a.shape[0], self.stream)
         return out
 
     def sub(self, a, b, lv):
-        out = self._ct(lv)
-        neo.neo_hsub(self.ctx, a, b, lv, out, 1, self.stream)
+        out = self._ct(lv, a.shape[0])
+        neo.neo_hsub(self.ctx, a, b, lv, out, a.shape[0], self.stream)
         return out
 
-    def pmul(self, a, name, lv):
-        out = self._ct(lv)
-        neo.neo_pmult(self.ctx, a, self.consts[name], lv, out, 1, self.stream)
+    def _pt(self, names):
+        return self.consts[names] if isinstance(names, str) else self._stacked(names)
+
+    def _stacked(self, names):
+        key = tuple(names)
+        if key not in self._stack:
+            self._stack[key] = torch.stack([self.consts[k] for k in names]).contiguous()
+        return self._stack[key]
+
+    def pmul(self, a, name, lv, out=None):
+        out = self._ct(lv, a.shape[0]) if out is None else out
+        neo.neo_pmult(self.ctx, a, self._pt(name), lv, out, a.shape[0], self.stream)
         return out
 
     def padd(self, a, name, lv):
-        out = self._ct(lv)
-        neo.neo_padd(self.ctx, a, self.consts[name], lv, out, 1, self.stream)
+        out = self._ct(lv, a.shape[0])
+        neo.neo_padd(self.ctx, a, self._pt(name), lv, out, a.shape[0], self.stream)
         return out
 
     def rescale(self, a, lv):
-        out = self._ct(lv - 1)
-        neo.neo_rescale(self.ctx, a, lv, out, 1, self.ws, self.stream)
+        out = self._ct(lv - 1, a.shape[0])
+        neo.neo_rescale(self.ctx, a, lv, out, a.shape[0], self.ws, self.stream)
         return out
 
     def hmul(self, a, b, lv):
-        out = self._ct(lv)
-        neo.neo_hmult(self.ctx, self.keys["relin"], a, b, lv, out, 1, self.ws, self.stream)
+        out = self._ct(lv, a.shape[0])
+        neo.neo_hmult(self.ctx, self.keys["relin"], a, b, lv, out, a.shape[0], self.ws, self.stream)
         return out
 
     def drop(self, a, li, lo):
         if li == lo:
             return a
-        out = self._ct(lo)
-        neo.neo_drop_levels(self.ctx, a, li, out, lo, 1, self.stream)
+        out = self._ct(lo, a.shape[0])
+        neo.neo_drop_levels(self.ctx, a, li, out, lo, a.shape[0], self.stream)
         return out
 
     # ---- the run
@@ -129,11 +142,12 @@ class Bootstrapper:
         ct = lintrans(ct, L, "cts")                                    # CoeffToSlot
         lv = L - 1
         cj = self.rot(ct, 2 * N - 1, lv)
-        x1 = self.add(ct, cj, lv)
-        x2 = self.pmul(self.sub(ct, cj, lv), "mono_mi", lv)
+        xs = self._ct(lv, 2)                                            # [x1, x2]: one batch of 2
+        self.add(ct, cj, lv, out=xs[0:1])                               # 2 Re(w)
+        self.pmul(self.sub(ct, cj, lv), "mono_mi", lv, out=xs[1:2])     # 2 Im(w)
 
-        def evalmod(x, lv, tag):
-            y1 = self.rescale(self.pmul(x, f"{tag}theta", lv), lv)
+        def evalmod(x, lv, tags):
+            y1 = self.rescale(self.pmul(x, [f"{t}theta" for t in tags], lv), lv)
             lv -= 1
             pw = {1: (y1, lv)}
 
@@ -147,19 +161,19 @@ class Bootstrapper:
             E = None
             for k in range(1, D_TAYLOR + 1):
                 ck, lk = pw[k]
-                term = self.drop(self.rescale(self.pmul(ck, f"{tag}c{k}", lk), lk), lk - 1, lt - 1)
+                term = self.drop(self.rescale(self.pmul(ck, [f"{t}c{k}" for t in tags], lk), lk), lk - 1, lt - 1)
                 E = term if E is None else self.add(E, term, lt - 1)
             lv = lt - 1
-            E = self.padd(E, f"{tag}c0", lv)
+            E = self.padd(E, [f"{t}c0" for t in tags], lv)
             for _ in range(self.r):
                 E = self.rescale(self.hmul(E, E, lv), lv)
                 lv -= 1
             cE = self.rot(E, 2 * N - 1, lv)
-            f = self.rescale(self.pmul(self.sub(E, cE, lv), f"{tag}sin", lv), lv)
+            f = self.rescale(self.pmul(self.sub(E, cE, lv), [f"{t}sin" for t in tags], lv), lv)
             return f, lv - 1
 
-        f1, lv = evalmod(x1, lv, "re")
-        f2, _ = evalmod(x2, L - 1, "im")
-        w = self.add(f1, self.pmul(f2, "mono_i", lv), lv)
+        # EvalMod of the real and imaginary halves as one batch of 2
+        f, lv = evalmod(xs, lv, ("re", "im"))
+        w = self.add(f[0:1], self.pmul(f[1:2], "mono_i", lv), lv)
         out = lintrans(w, lv, "stc")                                   # SlotToCoeff
         return out, lv - 1
