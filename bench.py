@@ -41,7 +41,7 @@ HBM_FALLBACK = 6650.0   # GB/s, /opt/skills/guides/B200_PROFILING.md fallback
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=300)
+    ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--batch", type=int, default=1, help="ciphertexts per GPU per step")
     ap.add_argument("--impl", choices=["neo", "reference"], default="neo")
@@ -113,10 +113,23 @@ class ClockSampler:
 
     def _read(self):
         for line in self.proc.stdout:
-            self.lines.append(line.strip())
+            self.lines.append((time.monotonic(), line.strip()))
+
+    def wait_ready(self, timeout: float = 5.0):
+        """Block until nvidia-smi has produced its first sample (its start-up takes longer
+        than a short timed region), then mark the start of the window that counts."""
+        t0 = time.monotonic()
+        while self.proc and not self.lines and time.monotonic() - t0 < timeout:
+            time.sleep(0.01)
+        self.t_begin = time.monotonic()
+
+    def mark_end(self):
+        self.t_end = time.monotonic()
 
     def __exit__(self, *a):
         if self.proc:
+            if not hasattr(self, "t_end"):
+                self.t_end = time.monotonic()
             time.sleep(0.15)
             self.proc.terminate()
             try:
@@ -127,7 +140,10 @@ class ClockSampler:
     def summary(self) -> dict:
         sm, mx, reasons = [], [], set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        t0, t1 = getattr(self, "t_begin", 0.0), getattr(self, "t_end", float("inf"))
+        inside = [ln for t, ln in self.lines if t0 <= t <= t1 + 0.1]
+        # a sample taken within 100 ms after the region covers its tail (-lms 100)
+        for ln in inside:
             f = [x.strip() for x in ln.split(",")]
             if len(f) < 7:
                 continue
@@ -348,11 +364,15 @@ def run_neo(args):
     launches[0] = 0
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
+        clk.wait_ready()
+        barrier()
+        torch.cuda.synchronize()
         t_start.record()
         for k in range(args.steps):
             run_step(k)
         t_end.record()
         torch.cuda.synchronize()
+        clk.mark_end()
     barrier()
     torch.cuda.synchronize()
     ms = t_start.elapsed_time(t_end)
