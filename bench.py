@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--no-hoisted", action="store_true")
     ap.add_argument("--no-klss", action="store_true",
                     help="skip the KLSS vs Hybrid key-switch comparison at Set-C (SURVEY §8(f) row 1)")
+    ap.add_argument("--no-apps", action="store_true",
+                    help="skip the application traces (HELR iteration, ResNet-20 layer; SURVEY §8(f) row 4)")
     ap.add_argument("--no-boot", action="store_true",
                     help="skip the bootstrapping timing (Set-B, 8 sparse slots; SURVEY §8(f) row 2)")
     ap.add_argument("--batch-hrot", type=int, default=256,
@@ -584,6 +586,67 @@ def run_neo(args):
         del bkeys, bconsts, bt
         torch.cuda.empty_cache()
 
+    # SURVEY §8(f) row 4 / BASELINE configs[4]: the application traces (reading APP,
+    # paper_conf_isca_jiaodwfcm0z25_b200.apps) at Set-B on every rank (DP): one HELR iteration
+    # over 1,024 samples of 196 -> 256 features (8 ciphertexts of 128 x 256, L530) and one
+    # ResNet-20 convolution layer (16 channels of 32 x 32, [32]).  Keys (one random evk shared
+    # by every Galois element) and constants are uniform residues made on the device: the cost
+    # is data-independent (correctness: tests/test_gpu_apps.py).
+    apps_block = None
+    if not args.no_apps:
+        from paper_conf_isca_jiaodwfcm0z25_b200 import apps as gapps
+        gen = torch.Generator(device="cuda")
+        gen.manual_seed(seed + 321)
+        rnd = lambda *shape: torch.randint(0, 1 << 35, shape, dtype=torch.int64, device="cuda",
+                                           generator=gen).view(torch.uint64)
+        evk_r = rnd(DNUM, 2, NUM_Q + NUM_P, N)
+        f_h, B_h, C_c, H_c = 256, 8, 16, 32
+        baby, giant = gapps.conv_rotations(C_c, H_c)
+        akeys = {"relin": neo.EvalKey(ctx, evk_r)}
+        for r in gapps.helr_rotations(N, f_h) + giant:
+            akeys.setdefault(gapps.galois(N, r), neo.EvalKey(ctx, evk_r))
+        for r in baby:
+            akeys[("h", gapps.galois(N, r))] = neo.EvalKey(ctx, evk_r, hoisted_galois=gapps.galois(N, r))
+        del evk_r
+        aconsts = {k: rnd(LEVEL + 1, N) for k in gapps.helr_const_names() + gapps.conv_const_names(C_c)}
+        aev = gapps.Evaluator(ctx, akeys, aconsts, max_batch=B_h)
+        Zc, Wc, Xc = rnd(B_h, 2, LEVEL + 1, N), rnd(1, 2, LEVEL + 1, N), rnd(1, 2, LEVEL + 1, N)
+
+        def timed(fn, reps):
+            for _ in range(2):
+                fn()
+            torch.cuda.synchronize()
+            barrier()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record()
+            for _ in range(reps):
+                fn()
+            a1.record()
+            torch.cuda.synchronize()
+            tms = a0.elapsed_time(a1) / reps
+            if world > 1:
+                t = torch.tensor([tms], dtype=torch.float64, device="cuda")
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                tms = float(t.item())
+            return tms
+        hms = timed(lambda: gapps.helr_iteration(aev, f_h, Zc, Wc, LEVEL), 3)
+        cms = timed(lambda: gapps.conv_layer(aev, C_c, H_c, Xc, LEVEL), 3)
+        lf, lr = int(math.log2(f_h)), int(math.log2(N // 2 // f_h))
+        apps_block = {
+            "helr_iteration": {
+                "config": "Set-B, l=35, 1024 samples x 256 features (196 padded) = 8 ciphertexts of 128 x 256 slots",
+                "ms_per_iteration": round(hms, 3), "value": world / (hms / 1e3), "unit": "iterations/s",
+                "ops": {"hmult": 4 * B_h, "hrot": (2 * lf + lr) * B_h, "pmult": 3 * B_h + 1, "rescale": 7 * B_h + 1},
+                "paper_context": "Table 5 (L534-549): Neo 0.22 s per HELR iteration, Set-C, A100 (context only)"},
+            "resnet20_conv_layer": {
+                "config": "Set-B, l=35, 16 channels x 32 x 32, 3x3 conv (8 hoisted + 15 giant-step HROT, 144 fused PMULT terms) + bias + degree-4 ReLU",
+                "ms_per_layer": round(cms, 3), "value": world / (cms / 1e3), "unit": "layers/s",
+                "ops": {"hrot": len(baby) + len(giant), "hmult": 2, "pmult_terms": 9 * C_c + 3},
+                "paper_context": "Table 5: Neo 12.03 s for all of ResNet-20 incl. bootstrapping, Set-C, A100 (context only)"},
+            "timing": "CUDA events around 3 runs after 2 warm-ups, max over ranks; synthetic keys/constants"}
+        del akeys, aconsts, aev, Zc, Wc, Xc
+        torch.cuda.empty_cache()
+
     # end-to-end through the public API with pinned host buffers: every step copies its three
     # input ciphertexts host->device and both results device->host.  Copies run on their own
     # streams, double-buffered, so the H2D of step k+1 and the D2H of step k-1 overlap the
@@ -666,7 +729,7 @@ def run_neo(args):
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted,
-                "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block,
+                "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block, "apps": apps_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}
         print(json.dumps(line), flush=True)

@@ -222,6 +222,18 @@ neo_status neo_padd(const neo_ctx* ctx, const uint64_t* ct_in, const uint64_t* p
 neo_status neo_hsub(const neo_ctx* ctx, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level,
                     uint64_t* ct_out, int32_t batch, neo_stream_t stream);
 
+/* Plaintext inner product (the diagonal method's inner loop of CoeffToSlot / SlotToCoeff and of
+ * a packed convolution: PMULT L133 followed by HADD L134, fused):
+ *   ct_out[b] = sum_{k < n_terms} ( c0_k[b] * m_k, c1_k[b] * m_k )   mod q_i, NTT form.
+ * cts: host array of n_terms device pointers, each ciphertexts [batch][2][level+1][N];
+ * pts: host array of n_terms device pointers, each plaintexts [batch][level+1][N], or one
+ * plaintext [level+1][N] applied to every batch entry when pt_shared != 0.
+ * 1 <= n_terms <= 32; ct_out [batch][2][level+1][N] must not alias any cts[k] (NEO_EINVAL).
+ * Equal, residue for residue, to n_terms neo_pmult calls summed by neo_hadd; one launch. */
+neo_status neo_pmult_acc(const neo_ctx* ctx, const uint64_t* const* cts, const uint64_t* const* pts,
+                         int32_t n_terms, int32_t pt_shared, int32_t level, uint64_t* ct_out, int32_t batch,
+                         neo_stream_t stream);
+
 /* Bootstrapping's ModRaise (the first step of PackBootstrap, L529):
  * ct_in [batch][2][1][N] mod q_0 (NTT form) -> ct_out [batch][2][level+1][N]: each coefficient's
  * centred representative in (-q_0/2, q_0/2] reduced mod q_0..q_level, NTT form, so that

@@ -1,0 +1,189 @@
+"""CKKS application traces on the GPU (BASELINE configs[4]; reading APP in
+DESIGN.md): one HELR training iteration [17, 18] and one ResNet-20 convolution layer [32],
+issued through the C-ABI in the order the oracle (oracle/apps.py) defines -- the same
+operations on the same operands, so the results are bit-exact.
+
+HELR iteration (L530, "batch sizes of 1,024 images", 196 features -> f = 256):
+  T = Rescale(HMULT(Z, W)); T += HROT(T, 2^k) (k < log f); T = Rescale(PMULT(T, mask));
+  T += HROT(T, -2^k); S = sigma3(-T) (two HMULTs, two PMULTs); G = Rescale(HMULT(S, Z));
+  G += HROT(G, f 2^k) (k < log rows); G = sum over the batch; W' = W + Rescale(PMULT(G, gamma/n)).
+  The batch of ciphertexts is one batched call per step (the library's batch dimension).
+ResNet-20 layer (L572, [32]'s 16-channel 32 x 32 stage): 8 hoisted baby-step rotations of the
+  input (one ModUp), per channel diagonal d one fused plaintext inner product over the 9 kernel
+  offsets (neo_pmult_acc) and one giant-step HROT by d H^2, Rescale, bias PADD, and the degree-4
+  ReLU polynomial (two HMULTs, three PMULTs).
+
+Plaintext constants are inputs (name -> device tensor [l+1][N], NTT form), like evaluation
+keys: tests produce them with the oracle's encoder, bench.py with random residues (the cost is
+data-independent).  Keys: {'relin': EvalKey, g: EvalKey} plus, for the conv layer's baby steps,
+hoisted keys {('h', g): EvalKey(hoisted_galois=g)}."""
+from __future__ import annotations
+
+import math
+
+import torch
+
+from . import neo
+
+
+def galois(N: int, r: int) -> int:
+    """Galois element of a left rotation by r slots (Z11), r taken mod N/2."""
+    return pow(5, r % (N // 2), 2 * N)
+
+
+def helr_rotations(N: int, f: int) -> list[int]:
+    rows = N // 2 // f
+    lf, lr = int(math.log2(f)), int(math.log2(rows))
+    return [1 << k for k in range(lf)] + [-(1 << k) for k in range(lf)] + [f << k for k in range(lr)]
+
+
+def conv_rotations(C: int, H: int) -> tuple[list[int], list[int]]:
+    """(hoisted baby steps dy H + dx, giant steps d H^2)."""
+    baby = [dy * H + dx for dy in (-1, 0, 1) for dx in (-1, 0, 1) if (dy, dx) != (0, 0)]
+    return baby, [d * H * H for d in range(1, C)]
+
+
+def helr_const_names() -> list[str]:
+    return ["mask", "sig_c3", "sig_c1", "sig_c0", "gamma"]
+
+
+def conv_const_names(C: int) -> list[str]:
+    ws = [f"w_{d}_{dy}_{dx}" for d in range(C) for dy in (-1, 0, 1) for dx in (-1, 0, 1)]
+    return ws + ["bias", "relu_a4", "relu_a2", "relu_a1", "relu_a0"]
+
+
+class Evaluator:
+    """Thin sequencing of C-ABI calls on one stream; every op allocates its output."""
+
+    def __init__(self, ctx: neo.Context, keys: dict, consts: dict, max_batch: int = 1, stream=None):
+        self.ctx, self.keys, self.consts, self.stream = ctx, keys, consts, stream
+        self.N = ctx.N
+        top = ctx.num_q - 1
+        ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_HROT_HOISTED)
+        wsn = max(ctx.workspace_size(op, top, max_batch) for op in ops)
+        self.ws = torch.empty(wsn // 8, dtype=torch.uint64, device="cuda")
+        self._bc = {}
+
+    def _ct(self, level, B=1, lead=()):
+        return torch.empty((*lead, B, 2, level + 1, self.N), dtype=torch.uint64, device="cuda")
+
+    def _pt_batched(self, name, B):
+        """A shared plaintext repeated for B ciphertexts (neo_padd takes one per ciphertext)."""
+        if (name, B) not in self._bc:
+            self._bc[(name, B)] = self.consts[name].unsqueeze(0).expand(B, -1, -1).contiguous()
+        return self._bc[(name, B)]
+
+    def rot(self, ct, r, lv):
+        g = galois(self.N, r)
+        out = self._ct(lv, ct.shape[0])
+        neo.neo_hrot(self.ctx, self.keys[g], g, ct, lv, out, ct.shape[0], self.ws, self.stream)
+        return out
+
+    def rot_hoisted(self, ct, rs, lv):
+        keys = [self.keys[("h", galois(self.N, r))] for r in rs]
+        out = self._ct(lv, ct.shape[0], (len(rs),))
+        neo.neo_hrot_hoisted(self.ctx, keys, ct, lv, out, ct.shape[0], self.ws, self.stream)
+        return out
+
+    def add(self, a, b, lv):
+        out = self._ct(lv, a.shape[0])
+        neo.neo_hadd(self.ctx, a, b, lv, out, a.shape[0], self.stream)
+        return out
+
+    def hmul(self, a, b, lv):
+        out = self._ct(lv, a.shape[0])
+        neo.neo_hmult(self.ctx, self.keys["relin"], a, b, lv, out, a.shape[0], self.ws, self.stream)
+        return out
+
+    def rescale(self, a, lv):
+        out = self._ct(lv - 1, a.shape[0])
+        neo.neo_rescale(self.ctx, a, lv, out, a.shape[0], self.ws, self.stream)
+        return out
+
+    def drop(self, a, li, lo):
+        if li == lo:
+            return a
+        out = self._ct(lo, a.shape[0])
+        neo.neo_drop_levels(self.ctx, a, li, out, lo, a.shape[0], self.stream)
+        return out
+
+    def pmul(self, a, name, lv):
+        """PMULT by one shared plaintext (neo_pmult_acc with one term)."""
+        return self.pmul_acc([a], [name], lv)
+
+    def pmul_acc(self, cts, names, lv):
+        out = self._ct(lv, cts[0].shape[0])
+        neo.neo_pmult_acc(self.ctx, cts, [self.consts[n] for n in names], lv, out, cts[0].shape[0],
+                          pt_shared=True, stream=self.stream)
+        return out
+
+    def padd(self, a, name, lv):
+        out = self._ct(lv, a.shape[0])
+        neo.neo_padd(self.ctx, a, self._pt_batched(name, a.shape[0]), lv, out, a.shape[0], self.stream)
+        return out
+
+
+def helr_iteration(ev: Evaluator, f: int, Z: torch.Tensor, W: torch.Tensor, level: int):
+    """Z [B][2][level+1][N] (B ciphertexts of rows x f samples), W [1][2][level+1][N] ->
+    (W' [1][2][level-5][N], level - 6)."""
+    N, B = ev.N, Z.shape[0]
+    rows = N // 2 // f
+    lf, lr = int(math.log2(f)), int(math.log2(rows))
+    L = level
+    Wb = W.expand(B, -1, -1, -1).contiguous() if B > 1 else W
+    T = ev.rescale(ev.hmul(Z, Wb, L), L)                          # 1
+    lv = L - 1
+    for k in range(lf):                                           # 2
+        T = ev.add(T, ev.rot(T, 1 << k, lv), lv)
+    T = ev.rescale(ev.pmul(T, "mask", lv), lv)                    # 3
+    lv -= 1
+    for k in range(lf):                                           # 4
+        T = ev.add(T, ev.rot(T, -(1 << k), lv), lv)
+    lT = lv                                                       # 5
+    T2 = ev.rescale(ev.hmul(T, T, lT), lT)
+    U = ev.rescale(ev.pmul(T, "sig_c3", lT), lT)
+    T3 = ev.rescale(ev.hmul(T2, U, lT - 1), lT - 1)
+    T1 = ev.drop(ev.rescale(ev.pmul(T, "sig_c1", lT), lT), lT - 1, lT - 2)
+    S = ev.padd(ev.add(T3, T1, lT - 2), "sig_c0", lT - 2)
+    G = ev.rescale(ev.hmul(S, ev.drop(Z, L, lT - 2), lT - 2), lT - 2)   # 6
+    lg = lT - 3
+    for k in range(lr):                                           # 7
+        G = ev.add(G, ev.rot(G, f << k, lg), lg)
+    while G.shape[0] > 1:                                         # 8 (a tree: modular sums are exact)
+        h = G.shape[0] // 2
+        S2 = ev.add(G[:h], G[h:2 * h], lg)
+        G = S2 if G.shape[0] == 2 * h else torch.cat([S2, G[2 * h:]])
+    upd = ev.rescale(ev.pmul(G, "gamma", lg), lg)                 # 9
+    Wn = ev.add(ev.drop(W, L, lg - 1), upd, lg - 1)
+    return Wn, lg - 1
+
+
+def conv_layer(ev: Evaluator, C: int, H: int, X: torch.Tensor, level: int):
+    """X [1][2][level+1][N] -> (out [1][2][level-3][N], level - 4)."""
+    baby, _ = conv_rotations(C, H)
+    lv = level
+    R = ev.rot_hoisted(X, baby, lv)                               # 1: [8][1][2][l+1][N]
+    offs = [(dy, dx) for dy in (-1, 0, 1) for dx in (-1, 0, 1)]
+    src, k = [], 0
+    for o in offs:
+        if o == (0, 0):
+            src.append(X)
+        else:
+            src.append(R[k])
+            k += 1
+    Y = None
+    for d in range(C):                                            # 2
+        acc = ev.pmul_acc(src, [f"w_{d}_{dy}_{dx}" for dy, dx in offs], lv)
+        if d:
+            acc = ev.rot(acc, d * H * H, lv)
+        Y = acc if Y is None else ev.add(Y, acc, lv)
+    Y = ev.rescale(Y, lv)
+    lY = lv - 1
+    Y = ev.padd(Y, "bias", lY)                                    # 3
+    Y2 = ev.rescale(ev.hmul(Y, Y, lY), lY)                        # 4
+    U = ev.rescale(ev.pmul(Y2, "relu_a4", lY - 1), lY - 1)
+    Y4 = ev.rescale(ev.hmul(ev.drop(Y2, lY - 1, lY - 2), U, lY - 2), lY - 2)
+    Y2c = ev.drop(ev.rescale(ev.pmul(Y2, "relu_a2", lY - 1), lY - 1), lY - 2, lY - 3)
+    Y1c = ev.drop(ev.rescale(ev.pmul(Y, "relu_a1", lY), lY), lY - 1, lY - 3)
+    out = ev.padd(ev.add(ev.add(Y4, Y2c, lY - 3), Y1c, lY - 3), "relu_a0", lY - 3)
+    return out, lY - 3

@@ -1128,6 +1128,28 @@ neo_status neo_hsub(const neo_ctx* c, const uint64_t* ct_a, const uint64_t* ct_b
     return ew_api(c, EW_HSUB, ct_a, ct_b, level, ct_out, batch, st);
 }
 
+neo_status neo_pmult_acc(const neo_ctx* c, const uint64_t* const* cts, const uint64_t* const* pts, int32_t n_terms,
+                        int32_t pt_shared, int32_t level, uint64_t* ct_out, int32_t batch, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(ct_out, "ct_out"));
+    if (!cts || !pts) FAIL(NEO_EINVAL, "cts / pts arrays are null");
+    if (n_terms < 1 || n_terms > NEO_MAX_ACC) FAIL(NEO_EINVAL, "n_terms must be in [1, 32]");
+    PmaccArgs A;
+    for (int k = 0; k < n_terms; ++k) {
+        TRY(check_ptr(cts[k], "cts[k]"));
+        TRY(check_ptr(pts[k], "pts[k]"));
+        if (cts[k] == ct_out) FAIL(NEO_EINVAL, "ct_out must not alias an input ciphertext");
+        A.ct[k] = cts[k];
+        A.pt[k] = pts[k];
+    }
+    A.out = ct_out; A.mods = c->d_mods;
+    A.N = c->N; A.limbs = level + 1; A.n_terms = n_terms; A.pt_shared = pt_shared != 0;
+    LAUNCH(PK_EW, S(st), launch_pmult_acc(A, batch, S(st)));
+    return NEO_OK;
+}
+
 neo_status neo_modraise(const neo_ctx* c, const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch,
                         void* ws, size_t ws_bytes, neo_stream_t st) {
     g_launches = 0;

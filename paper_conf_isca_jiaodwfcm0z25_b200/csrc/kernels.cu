@@ -217,6 +217,38 @@ k_ew(const __grid_constant__ EwArgs A) {
     *reinterpret_cast<ulonglong2*>(A.out + ct + cs) = y1;
 }
 
+// ------------------------------------------------------------------ plaintext inner product
+// sum_k (c0_k m_k, c1_k m_k) (L133 PMULT + L134 HADD, the diagonal method's inner loop):
+// products < 2^72 accumulate exactly in 128 bits (n_terms <= 32: < 2^77), one Barrett
+// reduction per output.  Two coefficients per thread, 16-byte accesses; one read of every
+// operand and one write, against 2 k launches and k - 1 intermediate ciphertexts unfused.
+__global__ void __launch_bounds__(256)
+k_pmult_acc(const __grid_constant__ PmaccArgs A) {
+    pdl_wait();
+    const int n = 2 * (blockIdx.x * blockDim.x + threadIdx.x);
+    const int i = blockIdx.y, b = blockIdx.z;
+    if (n >= A.N) return;
+    const ModQ m = A.mods[i];
+    const size_t cs = (size_t)A.limbs * A.N;
+    const size_t ct = (size_t)b * 2 * cs + (size_t)i * A.N + n;
+    const size_t pt = (A.pt_shared ? 0 : (size_t)b * cs) + (size_t)i * A.N + n;
+    u64 h[4] = {0, 0, 0, 0}, l[4] = {0, 0, 0, 0};
+#pragma unroll 4
+    for (int k = 0; k < A.n_terms; ++k) {
+        const ulonglong2 x0 = __ldg(reinterpret_cast<const ulonglong2*>(A.ct[k] + ct));
+        const ulonglong2 x1 = __ldg(reinterpret_cast<const ulonglong2*>(A.ct[k] + ct + cs));
+        const ulonglong2 p = __ldg(reinterpret_cast<const ulonglong2*>(A.pt[k] + pt));
+        mac128(h[0], l[0], x0.x, p.x);
+        mac128(h[1], l[1], x0.y, p.y);
+        mac128(h[2], l[2], x1.x, p.x);
+        mac128(h[3], l[3], x1.y, p.y);
+    }
+    *reinterpret_cast<ulonglong2*>(A.out + ct) =
+        make_ulonglong2(barrett_reduce(h[0], l[0], m), barrett_reduce(h[1], l[1], m));
+    *reinterpret_cast<ulonglong2*>(A.out + ct + cs) =
+        make_ulonglong2(barrett_reduce(h[2], l[2], m), barrett_reduce(h[3], l[3], m));
+}
+
 // ------------------------------------------------------------------ ModRaise (bootstrapping)
 // c in [0, q_0) -> the centred representative in (-q_0/2, q_0/2] reduced mod q_i
 __global__ void __launch_bounds__(256)
@@ -283,6 +315,9 @@ k_pack5(const u64* __restrict__ in, uint32_t* __restrict__ lo, uint8_t* __restri
 // ------------------------------------------------------------------ launchers
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_ew, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);
+}
+cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st) {
+    return launch_k(k_pmult_acc, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);
 }
 cudaError_t launch_modraise(const u64* coef, u64* out, const ModQ* mods, int limbs, int N, int bc, cudaStream_t st) {
     return launch_k(k_modraise, dim3((N + 255) / 256, limbs, bc), dim3(256), 0, st, coef, out, mods, limbs, N);

@@ -56,6 +56,16 @@ struct EwArgs {
     int N, limbs, op;
 };
 
+// Plaintext inner product: out[b] = sum_k PMULT(ct[k][b], pt[k][b or 0]) (neo_pmult_acc)
+constexpr int NEO_MAX_ACC = 32;
+struct PmaccArgs {
+    const u64* ct[NEO_MAX_ACC];   // each [B][2][limbs][N]
+    const u64* pt[NEO_MAX_ACC];   // each [B][limbs][N], or [limbs][N] when pt_shared
+    u64* out;                     // [B][2][limbs][N]
+    const ModQ* mods;
+    int N, limbs, n_terms, pt_shared;
+};
+
 // Double Rescale step 2: from the coefficient form of the last two limbs r[bc][2][N]
 // (mod q_{l-1}, mod q_l) writes corr[bc][i][N] = [x mod q_{l-1} q_l]_{q_i} for i < l - 1.
 struct DsArgs {
@@ -68,6 +78,7 @@ struct DsArgs {
 };
 
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st);
+cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st);
 // ModRaise: coef[bc][N] (coefficient form mod q_0, canonical) -> out[bc][i][N] = centred lift mod q_i
 cudaError_t launch_modraise(const u64* coef, u64* out, const ModQ* mods, int limbs, int N, int bc, cudaStream_t st);
 // drop limbs: in [B][2][li][N] -> out [B][2][lo][N] (lo <= li), the first lo limbs of each component

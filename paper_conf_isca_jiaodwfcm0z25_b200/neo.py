@@ -28,7 +28,7 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
             "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline", "neo_hsub", "neo_modraise",
-            "neo_drop_levels")
+            "neo_drop_levels", "neo_pmult_acc")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -87,6 +87,7 @@ def lib() -> ctypes.CDLL:
             "neo_modraise": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_drop_levels": [_vp, _vp, _i32, _vp, _i32, _i32, _vp],
             "neo_klss_query": [_vp, _i32p, _i32p, _u64p],
+            "neo_pmult_acc": [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), _i32, _i32, _i32, _vp, _i32, _vp],
         }
         for name, args in sig.items():
             if not hasattr(L, name):        # an older build (A/B runs); tests/test_abi.py requires every symbol
@@ -338,6 +339,17 @@ def neo_keyip(ctx: Context, evk: EvalKey, dhat, limb_ids, beta: int, acc, batch:
 def neo_moddown_combine(ctx: Context, acc, conv, q_ids, out, batch: int, stream=None):
     _check(lib().neo_moddown_combine(ctx.handle, _ptr(acc), _ptr(conv), _ids(q_ids), len(q_ids), _ptr(out), batch,
                                      _stream(stream)), "neo_moddown_combine")
+
+
+def neo_pmult_acc(ctx: Context, cts, pts, level: int, ct_out, batch: int, pt_shared: bool = False, stream=None):
+    """sum_k PMULT(cts[k], pts[k]) in one launch; pts[k] is [batch][l+1][N] or, with pt_shared,
+    one [l+1][N] plaintext for every batch entry."""
+    if len(cts) != len(pts):
+        raise NeoError(1, "neo_pmult_acc", "cts and pts differ in length")
+    ca = (ctypes.c_void_p * len(cts))(*[_ptr(t).value for t in cts])
+    pa = (ctypes.c_void_p * len(pts))(*[_ptr(t).value for t in pts])
+    _check(lib().neo_pmult_acc(ctx.handle, ca, pa, len(cts), int(pt_shared), level, _ptr(ct_out), batch,
+                               _stream(stream)), "neo_pmult_acc")
 
 
 def neo_hrot_hoisted(ctx: Context, keys, ct_in, level: int, ct_out, batch: int, ws, stream=None):
