@@ -652,58 +652,103 @@ def run_neo(args):
     # streams, double-buffered, so the H2D of step k+1 and the D2H of step k-1 overlap the
     # compute of step k (PCIe is full duplex).
     e2e = None
+    e2e_u64 = None
     if not args.no_e2e:
+        # two variants through the public API: (u64) residues copied as 8-byte words; (wire) the
+        # library's 36-bit wire format (neo_wire_pack/unpack: 4.5 bytes per residue), unpacked
+        # on the device before the step and the results packed after it -- inside the region.
         pinned = [[torch.from_numpy(x).pin_memory() for x in slot] for slot in host_in]
         sets = [[torch.empty_like(x) for x in dev_in[0]] for _ in range(2)]
         outs = [new_outs() for _ in range(2)]
         host_out = [(torch.empty(o[1].shape, dtype=torch.uint64).pin_memory(),
                      torch.empty(o[2].shape, dtype=torch.uint64).pin_memory()) for o in outs]
+        n_in = [x.numel() for x in dev_in[0]]
+        wb_in = [neo.neo_wire_bytes(n) for n in n_in]
+        n_out = [outs[0][1].numel(), outs[0][2].numel()]
+        wb_out = [neo.neo_wire_bytes(n) for n in n_out]
+        off_in = [sum(wb_in[:i]) for i in range(3)]
+        off_out = [0, wb_out[0]]
+        pinned_w = []
+        for slot in dev_in:
+            wdev = torch.empty(sum(wb_in), dtype=torch.uint8, device="cuda")
+            for i, x in enumerate(slot):
+                neo.neo_wire_pack(ctx, x, wdev[off_in[i]:off_in[i] + wb_in[i]])
+            pinned_w.append(wdev.cpu().pin_memory())
+        wire_in = [torch.empty(sum(wb_in), dtype=torch.uint8, device="cuda") for _ in range(2)]
+        wire_out = [torch.empty(sum(wb_out), dtype=torch.uint8, device="cuda") for _ in range(2)]
+        host_wout = [torch.empty(sum(wb_out), dtype=torch.uint8).pin_memory() for _ in range(2)]
         h2d_st, d2h_st = torch.cuda.Stream(), torch.cuda.Stream()
         ev_in = [torch.cuda.Event() for _ in range(2)]
         ev_comp = [torch.cuda.Event() for _ in range(2)]
         ev_out = [torch.cuda.Event() for _ in range(2)]
         k_e2e = max(3, min(args.steps, 50))
 
-        def e2e_run(K):
+        def e2e_run(K, wire):
             main = torch.cuda.current_stream()
             for k in range(K):
                 s_ = k % 2
                 with torch.cuda.stream(h2d_st):
                     if k >= 2:
                         h2d_st.wait_event(ev_comp[s_])
-                    for i in range(3):
-                        sets[s_][i].copy_(pinned[k % SLOTS][i], non_blocking=True)
+                    if wire:
+                        wire_in[s_].copy_(pinned_w[k % SLOTS], non_blocking=True)
+                    else:
+                        for i in range(3):
+                            sets[s_][i].copy_(pinned[k % SLOTS][i], non_blocking=True)
                     ev_in[s_].record(h2d_st)
                 main.wait_event(ev_in[s_])
                 if k >= 2:
                     main.wait_event(ev_out[s_])
+                if wire:
+                    for i in range(3):
+                        neo.neo_wire_unpack(ctx, wire_in[s_][off_in[i]:off_in[i] + wb_in[i]], sets[s_][i])
                 step(0, *sets[s_], outs=outs[s_])
+                if wire:
+                    for j in range(2):
+                        neo.neo_wire_pack(ctx, outs[s_][1 + j], wire_out[s_][off_out[j]:off_out[j] + wb_out[j]])
                 ev_comp[s_].record(main)
                 with torch.cuda.stream(d2h_st):
                     d2h_st.wait_event(ev_comp[s_])
-                    host_out[s_][0].copy_(outs[s_][1], non_blocking=True)
-                    host_out[s_][1].copy_(outs[s_][2], non_blocking=True)
+                    if wire:
+                        host_wout[s_].copy_(wire_out[s_], non_blocking=True)
+                    else:
+                        host_out[s_][0].copy_(outs[s_][1], non_blocking=True)
+                        host_out[s_][1].copy_(outs[s_][2], non_blocking=True)
                     ev_out[s_].record(d2h_st)
             for s_ in range(2):
                 main.wait_event(ev_out[s_])
 
-        e2e_run(2)
+        def e2e_time(wire):
+            e2e_run(2, wire)
+            torch.cuda.synchronize()
+            barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            e2e_run(k_e2e, wire)
+            e1.record()
+            torch.cuda.synchronize()
+            ems = e0.elapsed_time(e1)
+            if world > 1:
+                t = torch.tensor([ems], dtype=torch.float64, device="cuda")
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                ems = float(t.item())
+            return ems
+
+        ems = e2e_time(False)
+        e2e_u64 = {"value": 2 * B * world / (ems / k_e2e / 1e3), "unit": UNIT,
+                   "h2d_bytes_per_step": sum(n * 8 for n in n_in), "d2h_bytes_per_step": sum(n * 8 for n in n_out),
+                   "steps": k_e2e, "ms_per_step": ems / k_e2e, "format": "u64 residues (8 bytes each)"}
+        wms = e2e_time(True)
+        # the wire round trip is lossless: the last step's packed results unpack to its outputs
+        chk = torch.empty_like(outs[(k_e2e - 1) % 2][2])
+        neo.neo_wire_unpack(ctx, host_wout[(k_e2e - 1) % 2].cuda()[off_out[1]:], chk)
         torch.cuda.synchronize()
-        barrier()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        e2e_run(k_e2e)
-        e1.record()
-        torch.cuda.synchronize()
-        ems = e0.elapsed_time(e1)
-        if world > 1:
-            t = torch.tensor([ems], dtype=torch.float64, device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ems = float(t.item())
-        h2d = sum(x.numel() * 8 for x in dev_in[0])
-        d2h = (outs[0][1].numel() + outs[0][2].numel()) * 8
-        e2e = {"value": 2 * B * world / (ems / k_e2e / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
-               "d2h_bytes_per_step": d2h, "steps": k_e2e, "ms_per_step": ems / k_e2e,
+        assert torch.equal(chk.view(torch.int64), outs[(k_e2e - 1) % 2][2].view(torch.int64)), "wire round trip"
+        e2e = {"value": 2 * B * world / (wms / k_e2e / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": sum(wb_in), "d2h_bytes_per_step": sum(wb_out),
+               "steps": k_e2e, "ms_per_step": wms / k_e2e,
+               "format": "36-bit wire format (neo_wire_pack/unpack, 4.5 bytes per residue), unpack/pack on the device inside the region",
                "overlap": "H2D / compute / D2H on separate streams, double-buffered"}
 
     cpu = None
@@ -728,7 +773,7 @@ def run_neo(args):
                                   "peak": peak, "unit": "GB/s",
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
-                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted,
+                "cpu_baseline": cpu, "e2e": e2e, "e2e_u64": e2e_u64, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted,
                 "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block, "apps": apps_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}

@@ -222,6 +222,18 @@ neo_status neo_padd(const neo_ctx* ctx, const uint64_t* ct_in, const uint64_t* p
 neo_status neo_hsub(const neo_ctx* ctx, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level,
                     uint64_t* ct_out, int32_t batch, neo_stream_t stream);
 
+/* 36-bit wire format for host<->device transfers of residues (serialization, no arithmetic):
+ * n canonical residues < 2^36 take neo_wire_bytes(n) = 4.5 n bytes instead of 8 n:
+ *   bytes [0, 4n):      the low 32 bits of residue i at 4 i (little endian),
+ *   bytes [4n, 4.5n):   byte k = (residue 2k >> 32) | (residue 2k+1 >> 32) << 4.
+ * neo_wire_pack: device u64 residues -> device wire buffer; neo_wire_unpack: the inverse.
+ * n must be a positive multiple of 8; the wire buffer 16-byte aligned; word_bits <= 36
+ * (NEO_EUNSUPPORTED otherwise).  A ciphertext [batch][2][l+1][N] is n = batch 2 (l+1) N.
+ * Residues >= 2^36 lose their high bits (the caller's inputs must be canonical). */
+size_t     neo_wire_bytes(size_t n);
+neo_status neo_wire_pack(const neo_ctx* ctx, const uint64_t* in, void* wire, size_t n, neo_stream_t stream);
+neo_status neo_wire_unpack(const neo_ctx* ctx, const void* wire, uint64_t* out, size_t n, neo_stream_t stream);
+
 /* Plaintext inner product (the diagonal method's inner loop of CoeffToSlot / SlotToCoeff and of
  * a packed convolution: PMULT L133 followed by HADD L134, fused):
  *   ct_out[b] = sum_{k < n_terms} ( c0_k[b] * m_k, c1_k[b] * m_k )   mod q_i, NTT form.

@@ -1128,6 +1128,26 @@ neo_status neo_hsub(const neo_ctx* c, const uint64_t* ct_a, const uint64_t* ct_b
     return ew_api(c, EW_HSUB, ct_a, ct_b, level, ct_out, batch, st);
 }
 
+size_t neo_wire_bytes(size_t n) { return 4 * n + n / 2; }
+
+static neo_status wire_api(const neo_ctx* c, bool pack, const void* in, void* out, size_t n, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_ptr(in, "in"));
+    TRY(check_ptr(out, "out"));
+    if (c->word_bits > 36) FAIL(NEO_EUNSUPPORTED, "the 36-bit wire format needs word_bits <= 36");
+    if (n == 0 || n % 8) FAIL(NEO_EINVAL, "n must be a positive multiple of 8");
+    if (reinterpret_cast<uintptr_t>(pack ? out : in) % 16) FAIL(NEO_EINVAL, "wire buffer must be 16-byte aligned");
+    LAUNCH(PK_EW, S(st), launch_wire(pack, in, out, n, S(st)));
+    return NEO_OK;
+}
+neo_status neo_wire_pack(const neo_ctx* c, const uint64_t* in, void* wire, size_t n, neo_stream_t st) {
+    return wire_api(c, true, in, wire, n, st);
+}
+neo_status neo_wire_unpack(const neo_ctx* c, const void* wire, uint64_t* out, size_t n, neo_stream_t st) {
+    return wire_api(c, false, wire, out, n, st);
+}
+
 neo_status neo_pmult_acc(const neo_ctx* c, const uint64_t* const* cts, const uint64_t* const* pts, int32_t n_terms,
                         int32_t pt_shared, int32_t level, uint64_t* ct_out, int32_t batch, neo_stream_t st) {
     g_launches = 0;

@@ -1,5 +1,7 @@
 // kernels.cu -- BConv (CUDA-core), KeyIP, combine, tensor, automorphism and rescale helpers.
 #include "context.h"
+#include <algorithm>
+
 #include "kernels.h"
 
 namespace neo {
@@ -312,7 +314,56 @@ k_pack5(const u64* __restrict__ in, uint32_t* __restrict__ lo, uint8_t* __restri
     }
 }
 
+// ------------------------------------------------------------------ 36-bit wire format
+// n residues < 2^36 as [4n bytes: u32 low words][n/2 bytes: byte k = hi4(2k) | hi4(2k+1) << 4]
+// (4.5 bytes per residue against 8: the host<->device copies of neo_wire_pack / _unpack).
+// One thread per 8 residues: 32-byte low-word loads, one 4-byte nibble word.
+__global__ void __launch_bounds__(256)
+k_wire_unpack(const uint8_t* __restrict__ wire, u64* __restrict__ out, size_t n) {
+    pdl_wait();
+    const uint4* lo = reinterpret_cast<const uint4*>(wire);
+    const uint32_t* hi = reinterpret_cast<const uint32_t*>(wire + 4 * n);
+    const size_t groups = n / 8;
+    for (size_t g = blockIdx.x * (size_t)blockDim.x + threadIdx.x; g < groups; g += (size_t)gridDim.x * blockDim.x) {
+        const uint4 a = lo[2 * g], b = lo[2 * g + 1];
+        const uint32_t h = hi[g];
+        const uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+        ulonglong2* o = reinterpret_cast<ulonglong2*>(out + 8 * g);
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+            o[k] = make_ulonglong2((u64)w[2 * k] | ((u64)((h >> (8 * k)) & 0xF) << 32),
+                                   (u64)w[2 * k + 1] | ((u64)((h >> (8 * k + 4)) & 0xF) << 32));
+    }
+}
+__global__ void __launch_bounds__(256)
+k_wire_pack(const u64* __restrict__ in, uint8_t* __restrict__ wire, size_t n) {
+    pdl_wait();
+    uint4* lo = reinterpret_cast<uint4*>(wire);
+    uint32_t* hi = reinterpret_cast<uint32_t*>(wire + 4 * n);
+    const size_t groups = n / 8;
+    for (size_t g = blockIdx.x * (size_t)blockDim.x + threadIdx.x; g < groups; g += (size_t)gridDim.x * blockDim.x) {
+        const ulonglong2* v = reinterpret_cast<const ulonglong2*>(in + 8 * g);
+        uint32_t w[8], h = 0;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const ulonglong2 x = v[k];
+            w[2 * k] = (uint32_t)x.x;
+            w[2 * k + 1] = (uint32_t)x.y;
+            h |= (uint32_t)(((x.x >> 32) & 0xF) | (((x.y >> 32) & 0xF) << 4)) << (8 * k);
+        }
+        lo[2 * g] = make_uint4(w[0], w[1], w[2], w[3]);
+        lo[2 * g + 1] = make_uint4(w[4], w[5], w[6], w[7]);
+        hi[g] = h;
+    }
+}
+
 // ------------------------------------------------------------------ launchers
+cudaError_t launch_wire(bool pack, const void* in, void* out, size_t n, cudaStream_t st) {
+    const size_t groups = n / 8;
+    const unsigned blocks = (unsigned)std::min<size_t>((groups + 255) / 256, 148 * 16);
+    if (pack) return launch_k(k_wire_pack, dim3(blocks), dim3(256), 0, st, (const u64*)in, (uint8_t*)out, n);
+    return launch_k(k_wire_unpack, dim3(blocks), dim3(256), 0, st, (const uint8_t*)in, (u64*)out, n);
+}
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_ew, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);
 }

@@ -79,6 +79,8 @@ struct DsArgs {
 
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st);
+// 36-bit wire format (neo_wire_pack / neo_wire_unpack); n % 8 == 0
+cudaError_t launch_wire(bool pack, const void* in, void* out, size_t n, cudaStream_t st);
 // ModRaise: coef[bc][N] (coefficient form mod q_0, canonical) -> out[bc][i][N] = centred lift mod q_i
 cudaError_t launch_modraise(const u64* coef, u64* out, const ModQ* mods, int limbs, int N, int bc, cudaStream_t st);
 // drop limbs: in [B][2][li][N] -> out [B][2][lo][N] (lo <= li), the first lo limbs of each component

@@ -28,7 +28,7 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
             "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline", "neo_hsub", "neo_modraise",
-            "neo_drop_levels", "neo_pmult_acc")
+            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -87,6 +87,8 @@ def lib() -> ctypes.CDLL:
             "neo_modraise": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_drop_levels": [_vp, _vp, _i32, _vp, _i32, _i32, _vp],
             "neo_klss_query": [_vp, _i32p, _i32p, _u64p],
+            "neo_wire_pack": [_vp, _vp, _vp, _sz, _vp],
+            "neo_wire_unpack": [_vp, _vp, _vp, _sz, _vp],
             "neo_pmult_acc": [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), _i32, _i32, _i32, _vp, _i32, _vp],
         }
         for name, args in sig.items():
@@ -95,6 +97,8 @@ def lib() -> ctypes.CDLL:
             f = getattr(L, name)
             f.argtypes = args
             f.restype = ctypes.c_int
+        L.neo_wire_bytes.argtypes = [_sz]
+        L.neo_wire_bytes.restype = _sz
         L.neo_workspace_size.argtypes = [_vp, _i32, _i32, _i32]
         L.neo_workspace_size.restype = _sz
         L.neo_last_error.restype = ctypes.c_char_p
@@ -339,6 +343,25 @@ def neo_keyip(ctx: Context, evk: EvalKey, dhat, limb_ids, beta: int, acc, batch:
 def neo_moddown_combine(ctx: Context, acc, conv, q_ids, out, batch: int, stream=None):
     _check(lib().neo_moddown_combine(ctx.handle, _ptr(acc), _ptr(conv), _ids(q_ids), len(q_ids), _ptr(out), batch,
                                      _stream(stream)), "neo_moddown_combine")
+
+
+def neo_wire_bytes(n: int) -> int:
+    return int(lib().neo_wire_bytes(n))
+
+
+def _u8ptr(t: torch.Tensor):
+    if t.dtype != torch.uint8 or not t.is_cuda or not t.is_contiguous():
+        raise TypeError("expected a contiguous torch.uint8 CUDA tensor")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def neo_wire_pack(ctx: Context, x: torch.Tensor, wire: torch.Tensor, stream=None):
+    """u64 residues x (any shape, numel n) -> uint8 wire [neo_wire_bytes(n)] (36-bit format)."""
+    _check(lib().neo_wire_pack(ctx.handle, _ptr(x), _u8ptr(wire), x.numel(), _stream(stream)), "neo_wire_pack")
+
+
+def neo_wire_unpack(ctx: Context, wire: torch.Tensor, x: torch.Tensor, stream=None):
+    _check(lib().neo_wire_unpack(ctx.handle, _u8ptr(wire), _ptr(x), x.numel(), _stream(stream)), "neo_wire_unpack")
 
 
 def neo_pmult_acc(ctx: Context, cts, pts, level: int, ct_out, batch: int, pt_shared: bool = False, stream=None):
