@@ -559,6 +559,8 @@ def run_neo(args):
         bkeys = {"relin": neo.EvalKey(ctx, rnd(DNUM, 2, NUM_Q + NUM_P, N))}
         for gg in gboot.rotations(N, nb):
             bkeys[gg] = neo.EvalKey(ctx, rnd(DNUM, 2, NUM_Q + NUM_P, N))
+        for gg in gboot.hoisted_rotations(N, nb):
+            bkeys[("h", gg)] = neo.EvalKey(ctx, rnd(DNUM, 2, NUM_Q + NUM_P, N), hoisted_galois=gg)
         bconsts = {k: rnd(l + 1, N) for k, l in gboot.const_levels(LEVEL, nb, rb).items()}
         bt = gboot.Bootstrapper(ctx, nb, rb, bkeys, bconsts)
         bct = rnd(1, 2, 1, N)

@@ -11,7 +11,8 @@ Cheon, Han, Kim, Kim, Song (EUROCRYPT'18), built only from the operations pinned
   ModRaise  ct mod q_0 -> mod Q_L, coefficients lifted centred: m + q_0 I, I small
   SubSum    sum of the rotations by n 2^j: the trace onto the degree-2n subring (x M = N / 2n)
   CoeffToSlot  slots <- A z with A = W^-1 / M, W[k][j] = xi^(j 5^k), xi = e^(i pi / 2n): the slot
-            j then holds (p_{Mj} + i p_{M(j+n)}) / q_0 (diagonal method, one PMULT level)
+            j then holds (p_{Mj} + i p_{M(j+n)}) / q_0 (diagonal method, one PMULT level; its
+            n - 1 rotations of one ciphertext are hoisted rotations: one ModUp, reading BOOT-H)
   split     Re = (w + conj w) / 2, Im = (w - conj w) / 2i   (conjugation = HROTATE, g = 2N - 1)
   EvalMod   y = theta t (theta = 2 pi / 2^r), E = sum_{k<=7} (i y)^k / k!, E <- E^2 r times
             (= exp(2 pi i t)), f = (E - conj E) (-i / 4 pi) = sin(2 pi t) / 2 pi ~ t mod 1 = m / q_0
@@ -160,11 +161,13 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
         ct = ckks.hadd(prm, ct, rot(ct, pow(5, n << j, 2 * N), L), L)
 
     def lintrans(ct, lv, A, tag):        # slots <- A slots (diagonal method), scale kept, one level
+        # the n - 1 rotations of the same ciphertext are hoisted (one ModUp, reading BOOT-H)
+        gs = [pow(5, d, 2 * N) for d in range(1, n)]
+        rots = [ct] + list(ckks.hrot_hoisted(prm, ct, gs, lv, [keys[g] for g in gs]))
         acc = None
         for d, dg in enumerate(_diagonals(A)):
-            src = ct if d == 0 else rot(ct, pow(5, d, 2 * N), lv)
             pt = const(f"{tag}_{d}", lambda dg=dg: _pt(bp, dg, float(q[lv]), lv))
-            t = ckks.pmult(prm, src, pt, lv)
+            t = ckks.pmult(prm, rots[d], pt, lv)
             acc = t if acc is None else ckks.hadd(prm, acc, t, lv)
         return ckks.rescale(prm, acc, lv)
 

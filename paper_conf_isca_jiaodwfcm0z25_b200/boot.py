@@ -51,20 +51,26 @@ def const_levels(top: int, n: int, r: int) -> dict:
     return lv
 
 
+def hoisted_rotations(N: int, n: int) -> list[int]:
+    """Galois elements of the diagonal method's hoisted rotations (5^d, d = 1 .. n-1)."""
+    return [pow(5, d, 2 * N) for d in range(1, n)]
+
+
 class Bootstrapper:
-    """keys: {'relin': EvalKey, g: EvalKey for g in rotations(N, n)}; consts: {name: tensor}."""
+    """keys: {'relin': EvalKey, g: EvalKey for g in rotations(N, n), ('h', g): hoisted EvalKey
+    (neo_evk_create_hoisted) for g in hoisted_rotations(N, n)}; consts: {name: tensor}."""
 
     def __init__(self, ctx: neo.Context, n: int, r: int, keys: dict, consts: dict, stream=None):
         self.ctx, self.n, self.r, self.keys, self.consts, self.stream = ctx, n, r, keys, consts, stream
         self.N = ctx.N
         self.top = ctx.num_q - 1
-        ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_MODRAISE)
+        ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_MODRAISE, neo.NEO_OP_HROT_HOISTED)
         wsn = max(ctx.workspace_size(op, self.top, 2) for op in ops)
         self._stack = {}
         self.ws = torch.empty(wsn // 8, dtype=torch.uint64, device="cuda")
 
-    def _ct(self, level, B=1):
-        return torch.empty((B, 2, level + 1, self.N), dtype=torch.uint64, device="cuda")
+    def _ct(self, level, B=1, lead=()):
+        return torch.empty((*lead, B, 2, level + 1, self.N), dtype=torch.uint64, device="cuda")
 
     # ---- primitive ops (each one C-ABI call)
     # a ciphertext tensor is [B][2][l+1][N]; B = 2 runs EvalMod's real and imaginary halves as
@@ -131,12 +137,14 @@ class Bootstrapper:
         for j in range(int(math.log2(M))):                             # SubSum
             ct = self.add(ct, self.rot(ct, pow(5, n << j, 2 * N), L), L)
 
-        def lintrans(ct, lv, tag):                                      # diagonal method
-            acc = None
-            for d in range(n):
-                src = ct if d == 0 else self.rot(ct, pow(5, d, 2 * N), lv)
-                t = self.pmul(src, f"{tag}_{d}", lv)
-                acc = t if acc is None else self.add(acc, t, lv)
+        def lintrans(ct, lv, tag):             # diagonal method: hoisted rotations + one fused PMULT sum
+            hk = [self.keys[("h", pow(5, d, 2 * N))] for d in range(1, n)]
+            rots = self._ct(lv, 1, (n - 1,))
+            neo.neo_hrot_hoisted(self.ctx, hk, ct, lv, rots, 1, self.ws, self.stream)
+            acc = self._ct(lv)
+            neo.neo_pmult_acc(self.ctx, [ct] + [rots[d] for d in range(n - 1)],
+                              [self.consts[f"{tag}_{d}"] for d in range(n)], lv, acc, 1, pt_shared=True,
+                              stream=self.stream)
             return self.rescale(acc, lv)
 
         ct = lintrans(ct, L, "cts")                                    # CoeffToSlot

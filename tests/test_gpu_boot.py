@@ -31,6 +31,8 @@ def test_bootstrap_bit_exact_and_decodes():
     ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
     assert gboot.rotations(prm.N, bp.n) == bp.rotations()
     keys = {k: neo.EvalKey(ctx, dev(v)) for k, v in keys_np.items()}
+    for g in gboot.hoisted_rotations(prm.N, bp.n):
+        keys[("h", g)] = neo.EvalKey(ctx, dev(keys_np[g]), hoisted_galois=g)
     cl = gboot.const_levels(bp.top, bp.n, bp.r)
     assert set(cl) == set(consts) and all(consts[k].shape[0] == cl[k] + 1 for k in cl)
     b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()})
