@@ -51,7 +51,7 @@ typedef enum {
 
 /* Operation codes for neo_workspace_size. */
 enum { NEO_OP_KEYSWITCH = 0, NEO_OP_HMULT = 1, NEO_OP_HROT = 2, NEO_OP_RESCALE = 3, NEO_OP_HROT_HOISTED = 4,
-       NEO_OP_DOUBLE_RESCALE = 5, NEO_OP_MODRAISE = 6 };
+       NEO_OP_DOUBLE_RESCALE = 5, NEO_OP_MODRAISE = 6, NEO_OP_HMULT_RESCALE = 7 };
 
 /* Parameter description (Table 1, Table 4).
  *  log_n      : log2 N; this build supports 12 and 16 (N = 2^12 tiny config, 2^16 Set-B).
@@ -154,6 +154,18 @@ neo_status neo_keyswitch(const neo_ctx* ctx, const neo_evk* evk, const uint64_t*
 neo_status neo_hmult(const neo_ctx* ctx, const neo_evk* relin, const uint64_t* ct_a,
                      const uint64_t* ct_b, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
                      size_t ws_bytes, neo_stream_t stream);
+
+/* HMULT followed by Rescale (L132 + L137) as one fused call: ct_out [batch][2][level][N] equals
+ * neo_rescale(neo_hmult(ct_a, ct_b)) residue for residue.  Rescale's correction is folded
+ * into the key-switch's ModDown: with c_l = INTT of the product's last limb (its coefficient
+ * form, from INTT(acc_l), INTT(d_l) and the ModDown BConv output), the BConv output of every
+ * q_i (i < l) gets P [c_l]_{q_l} added before the one forward NTT, whose fused tail writes
+ * ((acc_i - NTT_i) P^-1 + d_i) q_l^-1 -- so Rescale's own INTT / NTT passes disappear.
+ * Hybrid keys only (NEO_EUNSUPPORTED for a KLSS key); 1 <= level <= 64;
+ * ws >= neo_workspace_size(ctx, NEO_OP_HMULT_RESCALE, level, batch). */
+neo_status neo_hmult_rescale(const neo_ctx* ctx, const neo_evk* relin, const uint64_t* ct_a,
+                             const uint64_t* ct_b, int32_t level, uint64_t* ct_out, int32_t batch,
+                             void* ws, size_t ws_bytes, neo_stream_t stream);
 
 /* HROTATE (L136): (sigma_g(c0) + k0, k1) with (k0, k1) = KS(sigma_g(c1)) under rotkey
  * = KSGen(s, sigma_g(s)) (L184).  galois_elt = 5^r mod 2N rotates slots left by r (Z11). */

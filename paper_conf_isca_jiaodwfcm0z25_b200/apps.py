@@ -59,7 +59,8 @@ class Evaluator:
         self.ctx, self.keys, self.consts, self.stream = ctx, keys, consts, stream
         self.N = ctx.N
         top = ctx.num_q - 1
-        ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_HROT_HOISTED)
+        ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_HROT_HOISTED,
+               neo.NEO_OP_HMULT_RESCALE)
         wsn = max(ctx.workspace_size(op, top, max_batch) for op in ops)
         self.ws = torch.empty(wsn // 8, dtype=torch.uint64, device="cuda")
         self._bc = {}
@@ -93,6 +94,12 @@ class Evaluator:
     def hmul(self, a, b, lv):
         out = self._ct(lv, a.shape[0])
         neo.neo_hmult(self.ctx, self.keys["relin"], a, b, lv, out, a.shape[0], self.ws, self.stream)
+        return out
+
+    def hmul_rescale(self, a, b, lv):
+        """Rescale(HMULT(a, b)) as one fused call (bit-identical)."""
+        out = self._ct(lv - 1, a.shape[0])
+        neo.neo_hmult_rescale(self.ctx, self.keys["relin"], a, b, lv, out, a.shape[0], self.ws, self.stream)
         return out
 
     def rescale(self, a, lv):
@@ -131,7 +138,7 @@ def helr_iteration(ev: Evaluator, f: int, Z: torch.Tensor, W: torch.Tensor, leve
     lf, lr = int(math.log2(f)), int(math.log2(rows))
     L = level
     Wb = W.expand(B, -1, -1, -1).contiguous() if B > 1 else W
-    T = ev.rescale(ev.hmul(Z, Wb, L), L)                          # 1
+    T = ev.hmul_rescale(Z, Wb, L)                          # 1
     lv = L - 1
     for k in range(lf):                                           # 2
         T = ev.add(T, ev.rot(T, 1 << k, lv), lv)
@@ -140,12 +147,12 @@ def helr_iteration(ev: Evaluator, f: int, Z: torch.Tensor, W: torch.Tensor, leve
     for k in range(lf):                                           # 4
         T = ev.add(T, ev.rot(T, -(1 << k), lv), lv)
     lT = lv                                                       # 5
-    T2 = ev.rescale(ev.hmul(T, T, lT), lT)
+    T2 = ev.hmul_rescale(T, T, lT)
     U = ev.rescale(ev.pmul(T, "sig_c3", lT), lT)
-    T3 = ev.rescale(ev.hmul(T2, U, lT - 1), lT - 1)
+    T3 = ev.hmul_rescale(T2, U, lT - 1)
     T1 = ev.drop(ev.rescale(ev.pmul(T, "sig_c1", lT), lT), lT - 1, lT - 2)
     S = ev.padd(ev.add(T3, T1, lT - 2), "sig_c0", lT - 2)
-    G = ev.rescale(ev.hmul(S, ev.drop(Z, L, lT - 2), lT - 2), lT - 2)   # 6
+    G = ev.hmul_rescale(S, ev.drop(Z, L, lT - 2), lT - 2)   # 6
     lg = lT - 3
     for k in range(lr):                                           # 7
         G = ev.add(G, ev.rot(G, f << k, lg), lg)
@@ -180,9 +187,9 @@ def conv_layer(ev: Evaluator, C: int, H: int, X: torch.Tensor, level: int):
     Y = ev.rescale(Y, lv)
     lY = lv - 1
     Y = ev.padd(Y, "bias", lY)                                    # 3
-    Y2 = ev.rescale(ev.hmul(Y, Y, lY), lY)                        # 4
+    Y2 = ev.hmul_rescale(Y, Y, lY)                        # 4
     U = ev.rescale(ev.pmul(Y2, "relu_a4", lY - 1), lY - 1)
-    Y4 = ev.rescale(ev.hmul(ev.drop(Y2, lY - 1, lY - 2), U, lY - 2), lY - 2)
+    Y4 = ev.hmul_rescale(ev.drop(Y2, lY - 1, lY - 2), U, lY - 2)
     Y2c = ev.drop(ev.rescale(ev.pmul(Y2, "relu_a2", lY - 1), lY - 1), lY - 2, lY - 3)
     Y1c = ev.drop(ev.rescale(ev.pmul(Y, "relu_a1", lY), lY), lY - 1, lY - 3)
     out = ev.padd(ev.add(ev.add(Y4, Y2c, lY - 3), Y1c, lY - 3), "relu_a0", lY - 3)

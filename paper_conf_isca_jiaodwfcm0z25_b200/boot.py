@@ -1,7 +1,8 @@
 """Sparse-slot CKKS bootstrapping on the GPU (PackBootstrap, L529; reading
 BOOT in DESIGN.md): an orchestration of the library's own kernels through the C-ABI --
 ModRaise, HROTATE (SubSum, the diagonal method, conjugation), PMULT / HADD / HSUB / PADD,
-HMULT and Rescale -- in the order oracle/boot.py defines (same operations, same operands).
+HMULT and Rescale (every HMULT -> Rescale pair as one neo_hmult_rescale call, bit-identical)
+-- in the order oracle/boot.py defines (same operations, same operands).
 
 The plaintext constants (CoeffToSlot / SlotToCoeff diagonals, EvalMod's Taylor coefficients,
 the monomials +-X^(N/2)) are inputs, like evaluation keys: a dict name -> device tensor
@@ -64,7 +65,8 @@ class Bootstrapper:
         self.ctx, self.n, self.r, self.keys, self.consts, self.stream = ctx, n, r, keys, consts, stream
         self.N = ctx.N
         self.top = ctx.num_q - 1
-        ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_MODRAISE, neo.NEO_OP_HROT_HOISTED)
+        ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_MODRAISE, neo.NEO_OP_HROT_HOISTED,
+               neo.NEO_OP_HMULT_RESCALE)
         wsn = max(ctx.workspace_size(op, self.top, 2) for op in ops)
         self._stack = {}
         self.ws = torch.empty(wsn // 8, dtype=torch.uint64, device="cuda")
@@ -120,6 +122,11 @@ class Bootstrapper:
         neo.neo_hmult(self.ctx, self.keys["relin"], a, b, lv, out, a.shape[0], self.ws, self.stream)
         return out
 
+    def hmul_rescale(self, a, b, lv):
+        out = self._ct(lv - 1, a.shape[0])
+        neo.neo_hmult_rescale(self.ctx, self.keys["relin"], a, b, lv, out, a.shape[0], self.ws, self.stream)
+        return out
+
     def drop(self, a, li, lo):
         if li == lo:
             return a
@@ -162,7 +169,7 @@ class Bootstrapper:
             def mul(a, b):
                 (ca, la), (cb, lb) = pw[a], pw[b]
                 l0 = min(la, lb)
-                pw[a + b] = (self.rescale(self.hmul(self.drop(ca, la, l0), self.drop(cb, lb, l0), l0), l0), l0 - 1)
+                pw[a + b] = (self.hmul_rescale(self.drop(ca, la, l0), self.drop(cb, lb, l0), l0), l0 - 1)
             for a, b in ((1, 1), (2, 1), (2, 2), (4, 1), (4, 2), (4, 3)):
                 mul(a, b)
             lt = min(l for _, l in pw.values())
@@ -174,7 +181,7 @@ class Bootstrapper:
             lv = lt - 1
             E = self.padd(E, [f"{t}c0" for t in tags], lv)
             for _ in range(self.r):
-                E = self.rescale(self.hmul(E, E, lv), lv)
+                E = self.hmul_rescale(E, E, lv)
                 lv -= 1
             cE = self.rot(E, 2 * N - 1, lv)
             f = self.rescale(self.pmul(self.sub(E, cE, lv), [f"{t}sin" for t in tags], lv), lv)

@@ -153,6 +153,7 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
     L.tmp = o; o += B * std::max(std::max(beta * E, 2 * Lq), 2 * P) * N;
     L.extra = o;
     if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
+    if (op == NEO_OP_HMULT_RESCALE) o += B * 3 * Lq * N + 4 * B * N;   // d, then c_l scratch
     if (op == NEO_OP_HROT) o += B * Lq * N;                       // sigma_g(c0)
     if (op == NEO_OP_HROT_HOISTED) o += B * 2 * Lq * N;
     L.total = o;
@@ -256,7 +257,10 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
 static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
                             u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
                             const u64* add0, const u64* add1, long long add_bs, cudaStream_t st,
-                            unsigned galois = 0, bool add_galois = true) {
+                            unsigned galois = 0, bool add_galois = true, u64* hmr_last = nullptr) {
+    // hmr_last != nullptr: fused HMULT + Rescale (neo_hmult_rescale).  add0/add1 are then d0/d1
+    // (stride add_bs), out0/out1 receive the rescaled ciphertext at level l - 1, and hmr_last
+    // is scratch [2][2B][N] for the coefficient form of acc_c and d_c at limb l.
     const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l), P = c->num_p;
     u64 *up = ws + Ly.up, *acc = ws + Ly.acc, *conv = ws + Ly.conv, *pc = ws + Ly.pc, *tmp = ws + Ly.tmp;
     int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
@@ -316,6 +320,43 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
             LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, 2 * B, st));
     }
 
+    if (hmr_last) {
+        // Rescale folded into ModDown: c_l = INTT(acc_l - NTT(conv_l)) P^-1 + INTT(d_l) is the
+        // coefficient form of the HMULT output's last limb; conv_i += P c_l for i < l, and the
+        // tail below becomes ((acc_i - NTT(conv_i)) P^-1 + d_i) q_l^-1 = Rescale(HMULT) exactly.
+        u64* accl = hmr_last;
+        u64* dl = hmr_last + (size_t)2 * B * N;
+        so[0] = l; so[1] = E + l; dof[0] = 0; dof[1] = 1; pr[0] = pr[1] = l;
+        if ((s = ntt_rows(c, false, acc, (long long)2 * E * N, so, accl, (long long)2 * N, dof, pr, 2, tmp, B, st)))
+            return s;
+        so[1] = (int)(add1 - add0) / N + l;
+        if ((s = ntt_rows(c, false, add0, add_bs, so, dl, (long long)2 * N, dof, pr, 2, tmp, B, st))) return s;
+        HmrFoldArgs F;
+        F.conv = conv; F.accl = accl; F.dl = dl; F.mods = c->d_mods;
+        F.pinv_l = c->pinv[l];
+        for (int i = 0; i < l; ++i) {
+            const u64 qi = c->mod[i];
+            u64 pm = 1;
+            for (int k2 = 0; k2 < P; ++k2) pm = (u64)((u128)pm * (c->mod[c->num_q + k2] % qi) % qi);
+            F.pmod[i].w = (double)pm;
+            F.pmod[i].wq = (double)pm / (double)qi;
+        }
+        F.N = N; F.l = l; F.lazy = c->use_tc ? 1 : 0;
+        LAUNCH(PK_EW, st, launch_hmr_fold(F, 2 * B, st));
+        for (int i = 0; i < l; ++i) { so[i] = dof[i] = i; pr[i] = i; }
+        RowEpi ep;
+        ep.acc = acc;
+        ep.acc_b = (long long)2 * E * N;
+        ep.acc_c = (long long)E * N;
+        ep.add0 = add0; ep.add1 = add1; ep.add_b = add_bs;
+        ep.out0 = out0; ep.out1 = out1; ep.out_b = out_bs;
+        ep.add_galois = 0;
+        ep.has_post = 1;
+        for (int i = 0; i < l; ++i) { ep.pinv[i] = c->pinv[i]; ep.post[i] = c->ql_inv[l][i]; }
+        return ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, l, tmp, 2 * B, st,
+                        &ep, c->use_tc);
+    }
+
     // a9 + a10: NTT of conv, with the ModDown tail (acc - conv) * P^-1 (+ add) fused into the
     // epilogue of the row pass (conv is never written back)
     for (int i = 0; i < Lq; ++i) { so[i] = dof[i] = i; pr[i] = i; }
@@ -356,6 +397,7 @@ static KlssLayout klss_layout(const neo_ctx* c, int l, int B, int op) {
     L.tmp = o; o += B * std::max(std::max(beta * ap, 2 * bt * ap), 2 * Lq) * N;
     L.extra = o;
     if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
+    if (op == NEO_OP_HMULT_RESCALE) o += B * 3 * Lq * N + 4 * B * N;   // d, then c_l scratch
     if (op == NEO_OP_HROT) o += B * Lq * N;
     L.total = o;
     return L;
@@ -697,9 +739,11 @@ size_t neo_workspace_size(const neo_ctx* c, int32_t op, int32_t level, int32_t b
         case NEO_OP_KEYSWITCH:
         case NEO_OP_HMULT:
         case NEO_OP_HROT:
-        case NEO_OP_HROT_HOISTED: {
+        case NEO_OP_HROT_HOISTED:
+        case NEO_OP_HMULT_RESCALE: {
+            if (op == NEO_OP_HMULT_RESCALE && level < 1) return 0;
             size_t w = ks_layout(c, level, batch, op).total;
-            if (c->num_t && op != NEO_OP_HROT_HOISTED) w = std::max(w, klss_total(c, level, batch, op));
+            if (c->num_t && op != NEO_OP_HROT_HOISTED && op != NEO_OP_HMULT_RESCALE) w = std::max(w, klss_total(c, level, batch, op));
             return w * sizeof(u64);
         }
         case NEO_OP_RESCALE: return level >= 1 ? rescale_ws(c, level, batch) * sizeof(u64) : 0;
@@ -949,6 +993,32 @@ neo_status neo_hmult(const neo_ctx* c, const neo_evk* relin, const uint64_t* ct_
     LAUNCH(PK_TENSOR, s, launch_tensor(ct_a, ct_b, dd, c->d_mods, level + 1, c->N, batch, s));
     return ks_core(c, relin, dd + 2 * ls, 3 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, dd, dd + ls,
                    3 * ls, s);
+}
+
+neo_status neo_hmult_rescale(const neo_ctx* c, const neo_evk* relin, const uint64_t* ct_a, const uint64_t* ct_b,
+                             int32_t level, uint64_t* ct_out, int32_t batch, void* ws, size_t ws_bytes,
+                             neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    if (!relin || relin->ctx != c) FAIL(NEO_EINVAL, "relinearisation key missing or from another context");
+    if (relin->klss) FAIL(NEO_EUNSUPPORTED, "neo_hmult_rescale takes a Hybrid key (use neo_hmult + neo_rescale)");
+    TRY(check_level(c, level, batch));
+    if (level < 1) FAIL(NEO_EINVAL, "rescale needs level >= 1");
+    if (level > 64) FAIL(NEO_EUNSUPPORTED, "level > 64");
+    TRY(check_ptr(ct_a, "ct_a"));
+    TRY(check_ptr(ct_b, "ct_b"));
+    TRY(check_ptr(ct_out, "ct_out"));
+    TRY(check_ws(c, NEO_OP_HMULT_RESCALE, level, batch, ws, ws_bytes));
+    KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HMULT_RESCALE);
+    u64* w = static_cast<u64*>(ws);
+    u64* dd = w + Ly.extra;
+    u64* last = dd + (size_t)3 * batch * (level + 1) * c->N;
+    const long long ls = (long long)(level + 1) * c->N, lo = (long long)level * c->N;
+    cudaStream_t s = S(st);
+    LAUNCH(PK_TENSOR, s, launch_tensor(ct_a, ct_b, dd, c->d_mods, level + 1, c->N, batch, s));
+    TRY(ks_modup(c, dd + 2 * ls, 3 * ls, level, batch, w, Ly, s));
+    return ks_finish(c, relin, dd + 2 * ls, 3 * ls, level, batch, w, Ly, ct_out, ct_out + lo, 2 * lo, dd, dd + ls,
+                     3 * ls, s, 0, true, last);
 }
 
 neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint64_t* ct_in, int32_t level,

@@ -251,6 +251,34 @@ k_pmult_acc(const __grid_constant__ PmaccArgs A) {
         make_ulonglong2(barrett_reduce(h[2], l[2], m), barrett_reduce(h[3], l[3], m));
 }
 
+// ------------------------------------------------------------------ fused HMULT + Rescale
+// One thread per (bc, coefficient): c_l once, then the l rows i < l (coalesced per row).
+__global__ void __launch_bounds__(256)
+k_hmr_fold(const __grid_constant__ HmrFoldArgs A) {
+    pdl_wait();
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int bc = blockIdx.y;
+    if (n >= A.N) return;
+    const size_t row = (size_t)A.N, base = (size_t)bc * (A.l + 1) * row + n;
+    const ModQ ml = A.mods[A.l];
+    u64 cv;
+    if (A.lazy) cv = d2u(canon(__longlong_as_double((long long)A.conv[base + (size_t)A.l * row]), ml.qd, ml.qinv));
+    else cv = A.conv[base + (size_t)A.l * row];
+    const u64 cl = add_mod(shoup(sub_mod(A.accl[(size_t)bc * row + n], cv, ml.q), A.pinv_l, ml.q),
+                           A.dl[(size_t)bc * row + n], ml.q);
+    const double cld = u2d(cl);
+    for (int i = 0; i < A.l; ++i) {
+        const ModQ m = A.mods[i];
+        u64* p = A.conv + base + (size_t)i * row;
+        if (A.lazy) {
+            const double z = __dadd_rn(__longlong_as_double((long long)*p), mulc(cld, A.pmod[i], m.qd));
+            *p = (u64)__double_as_longlong(canon(z, m.qd, m.qinv));
+        } else {
+            *p = add_mod(*p, d2u(canon(mulc(cld, A.pmod[i], m.qd), m.qd, m.qinv)), m.q);
+        }
+    }
+}
+
 // ------------------------------------------------------------------ ModRaise (bootstrapping)
 // c in [0, q_0) -> the centred representative in (-q_0/2, q_0/2] reduced mod q_i
 __global__ void __launch_bounds__(256)
@@ -369,6 +397,9 @@ cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st) {
 }
 cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_pmult_acc, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);
+}
+cudaError_t launch_hmr_fold(const HmrFoldArgs& A, int bc, cudaStream_t st) {
+    return launch_k(k_hmr_fold, dim3((A.N + 255) / 256, bc), dim3(256), 0, st, A);
 }
 cudaError_t launch_modraise(const u64* coef, u64* out, const ModQ* mods, int limbs, int N, int bc, cudaStream_t st) {
     return launch_k(k_modraise, dim3((N + 255) / 256, limbs, bc), dim3(256), 0, st, coef, out, mods, limbs, N);

@@ -66,6 +66,20 @@ struct PmaccArgs {
     int N, limbs, n_terms, pt_shared;
 };
 
+// Fused HMULT + Rescale (neo_hmult_rescale): with c_l = INTT(HMULT output limb l) =
+// (accl - conv_l) P^-1 + dl mod q_l (coefficient form, canonical), rewrite the ModDown BConv
+// output rows i < l as z_i = conv_i + P c_l mod q_i, so one NTT of z carries both ModDown's
+// and Rescale's corrections.
+struct HmrFoldArgs {
+    u64* conv;             // [2B][l+1][N]: lazy doubles (lazy != 0) or canonical u64
+    const u64* accl;       // [2B][N] INTT(acc_c limb l), canonical mod q_l
+    const u64* dl;         // [2B][N] INTT(d_c limb l), canonical mod q_l
+    const ModQ* mods;
+    TW pinv_l;             // P^-1 mod q_l
+    TWD pmod[64];          // (P mod q_i, /q_i), i < l
+    int N, l, lazy;
+};
+
 // Double Rescale step 2: from the coefficient form of the last two limbs r[bc][2][N]
 // (mod q_{l-1}, mod q_l) writes corr[bc][i][N] = [x mod q_{l-1} q_l]_{q_i} for i < l - 1.
 struct DsArgs {
@@ -79,6 +93,7 @@ struct DsArgs {
 
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st);
+cudaError_t launch_hmr_fold(const HmrFoldArgs& A, int bc, cudaStream_t st);
 // 36-bit wire format (neo_wire_pack / neo_wire_unpack); n % 8 == 0
 cudaError_t launch_wire(bool pack, const void* in, void* out, size_t n, cudaStream_t st);
 // ModRaise: coef[bc][N] (coefficient form mod q_0, canonical) -> out[bc][i][N] = centred lift mod q_i

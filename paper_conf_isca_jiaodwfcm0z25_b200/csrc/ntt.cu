@@ -426,6 +426,11 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                         u64 r1 = shoup(sub_mod(((u64)av[u].w << 32) | av[u].z, ((u64)v.w << 32) | v.z, qq), pinv, qq);
                         r0 = add_mod(r0, ((u64)dv[u].y << 32) | dv[u].x, qq);       // add = 0 when absent
                         r1 = add_mod(r1, ((u64)dv[u].w << 32) | dv[u].z, qq);
+                        if (ep.has_post) {                       // fused Rescale: x q_l^-1 (uniform branch)
+                            const TW post = ep.post[k];
+                            r0 = shoup(r0, post, qq);
+                            r1 = shoup(r1, post, qq);
+                        }
                         *reinterpret_cast<uint4*>(outr + pos[u]) =
                             make_uint4((unsigned)r0, (unsigned)(r0 >> 32), (unsigned)r1, (unsigned)(r1 >> 32));
                     }

@@ -27,7 +27,9 @@ struct RowEpi {
     u64* out1;
     long long out_b;
     unsigned add_galois;  // != 0: the addend of component 0 is sigma_g(add0), gathered on the fly
+    int has_post = 0;     // != 0: the result is further multiplied by post[k] (fused HMULT + Rescale)
     TW pinv[64];          // per row k
+    TW post[64];          // per row k: q_l^-1 mod q_k
 };
 
 // One pass over batch x rs.n limb rows.  Forward NTT = column pass (src -> tmp) then row

@@ -17,7 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libneo.so")
 
 NEO_OP_KEYSWITCH, NEO_OP_HMULT, NEO_OP_HROT, NEO_OP_RESCALE, NEO_OP_HROT_HOISTED = 0, 1, 2, 3, 4
-NEO_OP_DOUBLE_RESCALE, NEO_OP_MODRAISE = 5, 6
+NEO_OP_DOUBLE_RESCALE, NEO_OP_MODRAISE, NEO_OP_HMULT_RESCALE = 5, 6, 7
 _STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM", 4: "NEO_ECUDA",
            5: "NEO_ENCCL", 6: "NEO_ENOPRIME"}
 
@@ -28,7 +28,7 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
             "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline", "neo_hsub", "neo_modraise",
-            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack")
+            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -72,6 +72,7 @@ def lib() -> ctypes.CDLL:
             "neo_evk_destroy": [_vp],
             "neo_keyswitch": [_vp, _vp, _vp, _i32, _vp, _vp, _i32, _vp, _sz, _vp],
             "neo_hmult": [_vp, _vp, _vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+            "neo_hmult_rescale": [_vp, _vp, _vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_hrot": [_vp, _vp, _u32, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_rescale": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_keyip": [_vp, _vp, _vp, _i32p, _i32, _i32, _vp, _i32, _vp],
@@ -287,6 +288,12 @@ def neo_keyswitch(ctx: Context, evk: EvalKey, d, level: int, out0, out1, batch: 
 def neo_hmult(ctx: Context, relin: EvalKey, ct_a, ct_b, level: int, ct_out, batch: int, ws, stream=None):
     _check(lib().neo_hmult(ctx.handle, relin.handle, _ptr(ct_a), _ptr(ct_b), level, _ptr(ct_out), batch,
                            _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_hmult")
+
+
+def neo_hmult_rescale(ctx: Context, relin: EvalKey, ct_a, ct_b, level: int, ct_out, batch: int, ws, stream=None):
+    """Rescale(HMULT(ct_a, ct_b)) in one call: ct_out [batch][2][level][N]."""
+    _check(lib().neo_hmult_rescale(ctx.handle, relin.handle, _ptr(ct_a), _ptr(ct_b), level, _ptr(ct_out), batch,
+                                   _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_hmult_rescale")
 
 
 def neo_hrot(ctx: Context, rotkey: EvalKey, galois_elt: int, ct_in, level: int, ct_out, batch: int, ws,

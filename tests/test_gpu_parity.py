@@ -250,3 +250,33 @@ def test_hrot_hoisted(name, level, batch, rs):
         want = ckks.hrot_hoisted(prm, ct[bb], gs, level, keys_np)
         for r in range(len(rs)):
             assert np.array_equal(got[r, bb], want[r])
+
+
+@pytest.mark.parametrize("name,level,batch", [("tiny", 2, 2), ("tiny", 1, 1), ("tiny3", 2, 3), ("setb", 35, 1),
+                                              ("setb", 20, 2), ("setb", 1, 1)])
+def test_hmult_rescale_fused(name, level, batch):
+    """neo_hmult_rescale == Rescale(HMULT) of the oracle, bit for bit (the fused ModDown tail)."""
+    ctx, prm = ctx_of(name)
+    evk_np = rand_evk(prm, 1100)
+    relin = neo.EvalKey(ctx, dev(evk_np))
+    a = np.stack([rand_ct(prm, level, 1110 + 4 * b) for b in range(batch)])
+    b_ = np.stack([rand_ct(prm, level, 1112 + 4 * b) for b in range(batch)])
+    out = torch.empty((batch, 2, level, prm.N), dtype=torch.uint64, device="cuda")
+    ws = ctx.workspace(neo.NEO_OP_HMULT_RESCALE, level, batch)
+    neo.neo_hmult_rescale(ctx, relin, dev(a), dev(b_), level, out, batch, ws)
+    got = host(out)
+    for bb in range(batch):
+        assert np.array_equal(got[bb], ckks.rescale(prm, ckks.hmult(prm, a[bb], b_[bb], level, evk_np), level))
+
+
+def test_hmult_rescale_fused_rejects():
+    ctx, prm = ctx_of("tiny")
+    relin = neo.EvalKey(ctx, dev(rand_evk(prm, 1200)))
+    ct = dev(rand_ct(prm, 2, 1210)[None])
+    ws = ctx.workspace(neo.NEO_OP_HMULT_RESCALE, 2, 1)
+    with pytest.raises(neo.NeoError):           # level 0 cannot be rescaled
+        neo.neo_hmult_rescale(ctx, relin, ct[:, :, :1].contiguous(), ct[:, :, :1].contiguous(), 0,
+                              torch.empty((1, 2, 1, prm.N), dtype=torch.uint64, device="cuda"), 1, ws)
+    with pytest.raises(neo.NeoError):           # workspace too small
+        neo.neo_hmult_rescale(ctx, relin, ct, ct, 2, torch.empty((1, 2, 2, prm.N), dtype=torch.uint64, device="cuda"),
+                              1, ws[: ws.numel() // 2])
