@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--no-hoisted", action="store_true")
     ap.add_argument("--no-klss", action="store_true",
                     help="skip the KLSS vs Hybrid key-switch comparison at Set-C (SURVEY §8(f) row 1)")
+    ap.add_argument("--fused-rescale", type=int, default=1, choices=[0, 1],
+                    help="1: the step's HMULT -> Rescale is one neo_hmult_rescale call (bit-identical)")
     ap.add_argument("--no-apps", action="store_true",
                     help="skip the application traces (HELR iteration, ResNet-20 layer; SURVEY §8(f) row 4)")
     ap.add_argument("--no-boot", action="store_true",
@@ -163,7 +165,7 @@ class ClockSampler:
 
 # ----------------------------------------------------------------------------- byte model
 
-def bytes_model(batch: int, l: int = LEVEL) -> dict:
+def bytes_model(batch: int, l: int = LEVEL, fused: bool = False) -> dict:
     """Algorithmic HBM bytes per step, per kernel kind: every limb a launch must read or write
     once (limb = N words of 8 bytes; SURVEY §8(d) per-limb figures x the limbs each launch
     processes).  Per KS with Lq = l+1 Q limbs, P special limbs, E = Lq + P:
@@ -173,7 +175,10 @@ def bytes_model(batch: int, l: int = LEVEL) -> dict:
       BConv: ModUp Lq + (beta*E - Lq), ModDown 2P + 2*Lq;  KeyIP: beta*E + 2E per ciphertext,
       2*beta*E key limbs once per launch.
     Rescale: INTT of 2 limbs (col 4, row 4), NTT of 2l rows reading 2 unique limbs
-    (col 2 + 2l, row 2l + 2l (c_i) + 2l (out))."""
+    (col 2 + 2l, row 2l + 2l (c_i) + 2l (out)).
+    fused (neo_hmult_rescale): no Rescale passes; the HMULT's final NTT covers l rows (col 4l,
+    row 2l + 2l (acc) + 2l (d) + 2l (out)), plus INTTs of acc_l, d_l (4 rows: col 8, row 8) and
+    the fold kernel (elementwise: read 2 Lq + 4, write 2 l)."""
     limb = (1 << LOG_N) * 8
     Lq, P = l + 1, NUM_P
     beta = -(-Lq // 12)
@@ -182,14 +187,22 @@ def bytes_model(batch: int, l: int = LEVEL) -> dict:
     ks_col = 2 * Lq + 2 * up + 4 * P + 4 * Lq
     ks_row_base = 2 * Lq + 2 * up + 4 * P + 6 * Lq
     add_hmult, add_hrot = 2 * Lq, Lq
-    ntt_col = batch * (2 * ks_col + 4 + 2 + 2 * l)
-    ntt_row = batch * (2 * ks_row_base + add_hmult + add_hrot + 4 + 6 * l)
+    if fused:
+        hm_col = 2 * Lq + 2 * up + 4 * P + 4 * l + 8
+        hm_row = 2 * Lq + 2 * up + 4 * P + 8 * l + 8
+        ntt_col = batch * (hm_col + ks_col)
+        ntt_row = batch * (hm_row + ks_row_base + add_hrot)
+        ew = batch * (2 * Lq + 4 + 2 * l)
+    else:
+        ntt_col = batch * (2 * ks_col + 4 + 2 + 2 * l)
+        ntt_row = batch * (2 * ks_row_base + add_hmult + add_hrot + 4 + 6 * l)
+        ew = 0
     bconv = batch * 2 * ((Lq + up) + (2 * P + 2 * Lq))
     keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E * 5 / 8)          # key stored in 5 bytes per residue
     tensor = batch * 7 * Lq
     auto = batch * 2 * Lq         # AUTO of c0 only (c1 is read through the index map by the INTT and KeyIP)
     out = {"ntt_col": ntt_col, "ntt_row": ntt_row, "bconv": bconv, "keyip": keyip, "combine": 0,
-           "tensor": tensor, "automorphism": auto, "rescale_modswitch": 0, "rescale_combine": 0, "elementwise": 0}
+           "tensor": tensor, "automorphism": auto, "rescale_modswitch": 0, "rescale_combine": 0, "elementwise": ew}
     return {k: v * limb for k, v in out.items()}
 
 
@@ -300,7 +313,7 @@ def run_neo(args):
                 torch.empty((B, 2, Lq, N), dtype=torch.uint64, device="cuda"))
     hm_o, rs_o, hr_o = new_outs()
     ws_n = max(ctx.workspace_size(neo.NEO_OP_HMULT, LEVEL, B), ctx.workspace_size(neo.NEO_OP_HROT, LEVEL, B),
-               ctx.workspace_size(neo.NEO_OP_RESCALE, LEVEL, B))
+               ctx.workspace_size(neo.NEO_OP_RESCALE, LEVEL, B), ctx.workspace_size(neo.NEO_OP_HMULT_RESCALE, LEVEL, B))
     ws = torch.empty(ws_n // 8, dtype=torch.uint64, device="cuda")
     ws2 = torch.empty(ws_n // 8, dtype=torch.uint64, device="cuda") if args.streams == 2 else ws
     main_st = torch.cuda.current_stream()
@@ -325,10 +338,14 @@ def run_neo(args):
             side.wait_event(ev_go)
         neo.neo_hrot(ctx, rot, g, c, LEVEL, hr_out, B, ws2 if two else ws, stream=side)
         n = neo.last_launch_count()
-        neo.neo_hmult(ctx, relin, a, b, LEVEL, hm_out, B, ws, stream=main)
-        n += neo.last_launch_count()
-        neo.neo_rescale(ctx, hm_out, LEVEL, rs_out, B, ws, stream=main)
-        n += neo.last_launch_count()
+        if args.fused_rescale:          # Rescale(HMULT) in one call, bit-identical to the pair
+            neo.neo_hmult_rescale(ctx, relin, a, b, LEVEL, rs_out, B, ws, stream=main)
+            n += neo.last_launch_count()
+        else:
+            neo.neo_hmult(ctx, relin, a, b, LEVEL, hm_out, B, ws, stream=main)
+            n += neo.last_launch_count()
+            neo.neo_rescale(ctx, hm_out, LEVEL, rs_out, B, ws, stream=main)
+            n += neo.last_launch_count()
         if two:
             ev_done.record(side)
             main.wait_event(ev_done)
@@ -401,7 +418,7 @@ def run_neo(args):
 
     # roofline of the dominant kernel kind
     peak, peak_src = load_peaks()
-    bm = bytes_model(B)
+    bm = bytes_model(B, fused=bool(args.fused_rescale))
     step_ms = {k: v[0] / args.steps for k, v in prof.items()}
     ms_step_ref = ms_step_1s
     dom = max(step_ms, key=lambda k: step_ms[k])
@@ -764,7 +781,9 @@ def run_neo(args):
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
                 "vs_baseline": None, "dtype": "u64", "data": "synthetic (uniform residues, random keys)",
-                "config": workload_config(B, world),
+                "config": dict(workload_config(B, world),
+                               hmult_rescale="one neo_hmult_rescale call" if args.fused_rescale
+                               else "neo_hmult then neo_rescale"),
                 "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
                              "peak_source": peak_src, "unit": "GB/s",
                              "frac": achieved / peak if achieved else None, "traffic": traffic,
