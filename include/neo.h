@@ -234,6 +234,24 @@ neo_status neo_padd(const neo_ctx* ctx, const uint64_t* ct_in, const uint64_t* p
 neo_status neo_hsub(const neo_ctx* ctx, const uint64_t* ct_a, const uint64_t* ct_b, int32_t level,
                     uint64_t* ct_out, int32_t batch, neo_stream_t stream);
 
+/* Limb-subset element-wise operations for the limb-sharded evaluator (SURVEY §8(e)/(f) row 2:
+ * each rank holds the rows limb_ids[0..n) of its ciphertexts, in that order; row k is reduced
+ * mod q_{limb_ids[k]}, ids index the concatenated basis q_0..q_L, p_0..p_K).  NTT form unless
+ * stated; ct_* [batch][2][n][N], pt [batch][n][N]; 1 <= n <= 64.
+ *   NEO_EWL_HADD / _HSUB / _PMULT / _PADD (0-3): as neo_hadd / neo_hsub / neo_pmult / neo_padd (L133-135)
+ *   NEO_EWL_TENSOR (4): out d [batch][3][n][N] = (a0 b0, a0 b1 + a1 b0, a1 b1) (L132)
+ *   NEO_EWL_SUBMUL (5): out = (a - b) * scal[k]; scal a HOST array of n residues (Rescale's
+ *                       (c_i - r_i) q_l^-1 on a rank's limbs, L137)
+ *   NEO_EWL_LIFT (6):   a = coefficient rows [batch][2][N], canonical mod q_{src_limb}; out
+ *                       [batch][2][n][N] = each value's centred representative reduced mod
+ *                       q_{limb_ids[k]} (coefficient form; ModRaise on a rank's limbs, L529)
+ * b is ignored for LIFT; scal only read for SUBMUL; out may alias a (same positions). */
+enum { NEO_EWL_HADD = 0, NEO_EWL_HSUB = 1, NEO_EWL_PMULT = 2, NEO_EWL_PADD = 3, NEO_EWL_TENSOR = 4,
+       NEO_EWL_SUBMUL = 5, NEO_EWL_LIFT = 6 };
+neo_status neo_ew_limbs(const neo_ctx* ctx, int32_t op, const uint64_t* a, const uint64_t* b,
+                        const int32_t* limb_ids, int32_t n, const uint64_t* scal, int32_t src_limb,
+                        uint64_t* out, int32_t batch, neo_stream_t stream);
+
 /* 36-bit wire format for host<->device transfers of residues (serialization, no arithmetic):
  * n canonical residues < 2^36 take neo_wire_bytes(n) = 4.5 n bytes instead of 8 n:
  *   bytes [0, 4n):      the low 32 bits of residue i at 4 i (little endian),

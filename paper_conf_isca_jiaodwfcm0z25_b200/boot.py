@@ -134,25 +134,31 @@ class Bootstrapper:
         neo.neo_drop_levels(self.ctx, a, li, out, lo, a.shape[0], self.stream)
         return out
 
+    def modraise(self, ct0, L):
+        ct = self._ct(L)
+        neo.neo_modraise(self.ctx, ct0, L, ct, 1, self.ws, self.stream)
+        return ct
+
+    def lintrans(self, ct, lv, tag):           # diagonal method: hoisted rotations + one fused PMULT sum
+        N, n = self.N, self.n
+        hk = [self.keys[("h", pow(5, d, 2 * N))] for d in range(1, n)]
+        rots = self._ct(lv, 1, (n - 1,))
+        neo.neo_hrot_hoisted(self.ctx, hk, ct, lv, rots, 1, self.ws, self.stream)
+        acc = self._ct(lv)
+        neo.neo_pmult_acc(self.ctx, [ct] + [rots[d] for d in range(n - 1)],
+                          [self.consts[f"{tag}_{d}"] for d in range(n)], lv, acc, 1, pt_shared=True,
+                          stream=self.stream)
+        return self.rescale(acc, lv)
+
     # ---- the run
     def run(self, ct0: torch.Tensor):
         """ct0 [1][2][1][N] (level 0) -> (ct, level)."""
         N, n, L = self.N, self.n, self.top
         M = N // (2 * n)
-        ct = self._ct(L)
-        neo.neo_modraise(self.ctx, ct0, L, ct, 1, self.ws, self.stream)
+        ct = self.modraise(ct0, L)
         for j in range(int(math.log2(M))):                             # SubSum
             ct = self.add(ct, self.rot(ct, pow(5, n << j, 2 * N), L), L)
-
-        def lintrans(ct, lv, tag):             # diagonal method: hoisted rotations + one fused PMULT sum
-            hk = [self.keys[("h", pow(5, d, 2 * N))] for d in range(1, n)]
-            rots = self._ct(lv, 1, (n - 1,))
-            neo.neo_hrot_hoisted(self.ctx, hk, ct, lv, rots, 1, self.ws, self.stream)
-            acc = self._ct(lv)
-            neo.neo_pmult_acc(self.ctx, [ct] + [rots[d] for d in range(n - 1)],
-                              [self.consts[f"{tag}_{d}"] for d in range(n)], lv, acc, 1, pt_shared=True,
-                              stream=self.stream)
-            return self.rescale(acc, lv)
+        lintrans = self.lintrans
 
         ct = lintrans(ct, L, "cts")                                    # CoeffToSlot
         lv = L - 1

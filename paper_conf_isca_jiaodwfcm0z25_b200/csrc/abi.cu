@@ -1198,6 +1198,38 @@ neo_status neo_hsub(const neo_ctx* c, const uint64_t* ct_a, const uint64_t* ct_b
     return ew_api(c, EW_HSUB, ct_a, ct_b, level, ct_out, batch, st);
 }
 
+neo_status neo_ew_limbs(const neo_ctx* c, int32_t op, const uint64_t* a, const uint64_t* b, const int32_t* limb_ids,
+                        int32_t n, const uint64_t* scal, int32_t src_limb, uint64_t* out, int32_t batch,
+                        neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    if (op < EWL_HADD || op > EWL_LIFT) FAIL(NEO_EINVAL, "unknown neo_ew_limbs op");
+    if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
+    if (n < 1 || n > 64 || !limb_ids) FAIL(NEO_EINVAL, "need 1 <= n <= 64 limb ids");
+    TRY(check_ptr(a, "a"));
+    TRY(check_ptr(out, "out"));
+    if (op != EWL_LIFT) TRY(check_ptr(b, "b"));
+    const int tot = c->num_q + c->num_p;
+    EwlArgs A;
+    for (int k = 0; k < n; ++k) {
+        if (limb_ids[k] < 0 || limb_ids[k] >= tot) FAIL(NEO_EINVAL, "unknown limb id");
+        A.lid[k] = (short)limb_ids[k];
+    }
+    if (op == EWL_SUBMUL) {
+        if (!scal) FAIL(NEO_EINVAL, "SUBMUL needs the host array scal[n]");
+        for (int k = 0; k < n; ++k) {
+            const u64 q = c->mod[limb_ids[k]];
+            if (scal[k] >= q) FAIL(NEO_EINVAL, "scal[k] must be a residue mod q_{limb_ids[k]}");
+            A.scal[k] = TW{scal[k], (u64)(((u128)scal[k] << 64) / q)};
+        }
+    }
+    if (op == EWL_LIFT && (src_limb < 0 || src_limb >= tot)) FAIL(NEO_EINVAL, "bad src_limb");
+    A.a = a; A.b = b; A.out = out; A.mods = c->d_mods;
+    A.N = c->N; A.n = n; A.op = op; A.src = src_limb;
+    LAUNCH(PK_EW, S(st), launch_ew_limbs(A, batch, S(st)));
+    return NEO_OK;
+}
+
 size_t neo_wire_bytes(size_t n) { return 4 * n + n / 2; }
 
 static neo_status wire_api(const neo_ctx* c, bool pack, const void* in, void* out, size_t n, neo_stream_t st) {

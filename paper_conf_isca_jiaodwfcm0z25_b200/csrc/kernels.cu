@@ -251,6 +251,73 @@ k_pmult_acc(const __grid_constant__ PmaccArgs A) {
         make_ulonglong2(barrett_reduce(h[2], l[2], m), barrett_reduce(h[3], l[3], m));
 }
 
+// ------------------------------------------------------------------ limb-subset element-wise ops
+// One thread per (coefficient, row k, batch b); both components in the thread.
+__global__ void __launch_bounds__(256)
+k_ew_limbs(const __grid_constant__ EwlArgs A) {
+    pdl_wait();
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int k = blockIdx.y, b = blockIdx.z;
+    if (n >= A.N) return;
+    const ModQ m = A.mods[A.lid[k]];
+    const size_t cs = (size_t)A.n * A.N;
+    const size_t ct = (size_t)b * 2 * cs + (size_t)k * A.N + n;
+    if (A.op == EWL_LIFT) {                                  // centred lift from q_src
+        const u64 qs = A.mods[A.src].q;
+#pragma unroll
+        for (int c = 0; c < 2; ++c) {
+            const u64 x = A.a[((size_t)b * 2 + c) * A.N + n];
+            u64 r;
+            if (2 * x > qs) {
+                const u64 mm = (qs - x) % m.q;
+                r = mm == 0 ? 0 : m.q - mm;
+            } else {
+                r = x % m.q;
+            }
+            A.out[ct + c * cs] = r;
+        }
+        return;
+    }
+    const u64 a0 = A.a[ct], a1 = A.a[ct + cs];
+    if (A.op == EWL_TENSOR) {
+        const u64 b0 = A.b[ct], b1 = A.b[ct + cs];
+        const size_t ob = (size_t)b * 3 * cs + (size_t)k * A.N + n;
+        A.out[ob] = mul_mod(a0, b0, m);
+        u64 h = 0, l = 0;
+        mac128(h, l, a0, b1);
+        mac128(h, l, a1, b0);
+        A.out[ob + cs] = barrett_reduce(h, l, m);
+        A.out[ob + 2 * cs] = mul_mod(a1, b1, m);
+        return;
+    }
+    u64 y0, y1;
+    if (A.op == EWL_HADD || A.op == EWL_HSUB || A.op == EWL_SUBMUL) {
+        const u64 b0 = A.b[ct], b1 = A.b[ct + cs];
+        if (A.op == EWL_HADD) {
+            y0 = add_mod(a0, b0, m.q);
+            y1 = add_mod(a1, b1, m.q);
+        } else {
+            y0 = sub_mod(a0, b0, m.q);
+            y1 = sub_mod(a1, b1, m.q);
+            if (A.op == EWL_SUBMUL) {
+                y0 = shoup(y0, A.scal[k], m.q);
+                y1 = shoup(y1, A.scal[k], m.q);
+            }
+        }
+    } else {
+        const u64 p = A.b[(size_t)b * cs + (size_t)k * A.N + n];
+        if (A.op == EWL_PMULT) {
+            y0 = mul_mod(a0, p, m);
+            y1 = mul_mod(a1, p, m);
+        } else {
+            y0 = add_mod(a0, p, m.q);
+            y1 = a1;
+        }
+    }
+    A.out[ct] = y0;
+    A.out[ct + cs] = y1;
+}
+
 // ------------------------------------------------------------------ fused HMULT + Rescale
 // One thread per (bc, coefficient): c_l once, then the l rows i < l (coalesced per row).
 __global__ void __launch_bounds__(256)
@@ -397,6 +464,9 @@ cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st) {
 }
 cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_pmult_acc, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);
+}
+cudaError_t launch_ew_limbs(const EwlArgs& A, int batch, cudaStream_t st) {
+    return launch_k(k_ew_limbs, dim3((A.N + 255) / 256, A.n, batch), dim3(256), 0, st, A);
 }
 cudaError_t launch_hmr_fold(const HmrFoldArgs& A, int bc, cudaStream_t st) {
     return launch_k(k_hmr_fold, dim3((A.N + 255) / 256, bc), dim3(256), 0, st, A);

@@ -66,6 +66,19 @@ struct PmaccArgs {
     int N, limbs, n_terms, pt_shared;
 };
 
+// Limb-subset element-wise operations (neo_ew_limbs; the limb-sharded evaluator): row k of
+// every polynomial is reduced mod q_{lid[k]}.
+enum EwlOp { EWL_HADD = 0, EWL_HSUB = 1, EWL_PMULT = 2, EWL_PADD = 3, EWL_TENSOR = 4, EWL_SUBMUL = 5, EWL_LIFT = 6 };
+struct EwlArgs {
+    const u64* a;          // ct [B][2][n][N]  (LIFT: coefficient rows [B][2][N] mod q_src)
+    const u64* b;          // ct [B][2][n][N] or pt [B][n][N]
+    u64* out;              // ct [B][2][n][N] (TENSOR: d [B][3][n][N])
+    const ModQ* mods;
+    int N, n, op, src;
+    short lid[64];
+    TW scal[64];           // SUBMUL: per row
+};
+
 // Fused HMULT + Rescale (neo_hmult_rescale): with c_l = INTT(HMULT output limb l) =
 // (accl - conv_l) P^-1 + dl mod q_l (coefficient form, canonical), rewrite the ModDown BConv
 // output rows i < l as z_i = conv_i + P c_l mod q_i, so one NTT of z carries both ModDown's
@@ -94,6 +107,7 @@ struct DsArgs {
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_hmr_fold(const HmrFoldArgs& A, int bc, cudaStream_t st);
+cudaError_t launch_ew_limbs(const EwlArgs& A, int batch, cudaStream_t st);
 // 36-bit wire format (neo_wire_pack / neo_wire_unpack); n % 8 == 0
 cudaError_t launch_wire(bool pack, const void* in, void* out, size_t n, cudaStream_t st);
 // ModRaise: coef[bc][N] (coefficient form mod q_0, canonical) -> out[bc][i][N] = centred lift mod q_i

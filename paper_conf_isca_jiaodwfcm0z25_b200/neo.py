@@ -28,7 +28,7 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
             "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline", "neo_hsub", "neo_modraise",
-            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale")
+            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale", "neo_ew_limbs")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -72,6 +72,7 @@ def lib() -> ctypes.CDLL:
             "neo_evk_destroy": [_vp],
             "neo_keyswitch": [_vp, _vp, _vp, _i32, _vp, _vp, _i32, _vp, _sz, _vp],
             "neo_hmult": [_vp, _vp, _vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+            "neo_ew_limbs": [_vp, _i32, _vp, _vp, _i32p, _i32, _u64p, _i32, _vp, _i32, _vp],
             "neo_hmult_rescale": [_vp, _vp, _vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_hrot": [_vp, _vp, _u32, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_rescale": [_vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
@@ -293,7 +294,7 @@ def neo_hmult(ctx: Context, relin: EvalKey, ct_a, ct_b, level: int, ct_out, batc
 def neo_hmult_rescale(ctx: Context, relin: EvalKey, ct_a, ct_b, level: int, ct_out, batch: int, ws, stream=None):
     """Rescale(HMULT(ct_a, ct_b)) in one call: ct_out [batch][2][level][N]."""
     _check(lib().neo_hmult_rescale(ctx.handle, relin.handle, _ptr(ct_a), _ptr(ct_b), level, _ptr(ct_out), batch,
-                                   _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_hmult_rescale")
+                                   _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_hmult_rescale", "neo_ew_limbs")
 
 
 def neo_hrot(ctx: Context, rotkey: EvalKey, galois_elt: int, ct_in, level: int, ct_out, batch: int, ws,
@@ -350,6 +351,17 @@ def neo_keyip(ctx: Context, evk: EvalKey, dhat, limb_ids, beta: int, acc, batch:
 def neo_moddown_combine(ctx: Context, acc, conv, q_ids, out, batch: int, stream=None):
     _check(lib().neo_moddown_combine(ctx.handle, _ptr(acc), _ptr(conv), _ids(q_ids), len(q_ids), _ptr(out), batch,
                                      _stream(stream)), "neo_moddown_combine")
+
+
+NEO_EWL_HADD, NEO_EWL_HSUB, NEO_EWL_PMULT, NEO_EWL_PADD, NEO_EWL_TENSOR, NEO_EWL_SUBMUL, NEO_EWL_LIFT = range(7)
+
+
+def neo_ew_limbs(ctx: Context, op: int, a, b, limb_ids, out, batch: int, scal=None, src_limb: int = 0,
+                 stream=None):
+    """Element-wise op on the rows limb_ids of a rank's polynomials (include/neo.h)."""
+    sc = (ctypes.c_uint64 * len(limb_ids))(*scal) if scal is not None else None
+    _check(lib().neo_ew_limbs(ctx.handle, op, _ptr(a), _ptr(b), _ids(limb_ids), len(limb_ids), sc, src_limb,
+                              _ptr(out), batch, _stream(stream)), "neo_ew_limbs")
 
 
 def neo_wire_bytes(n: int) -> int:

@@ -49,16 +49,30 @@ def max_over_ranks(value: float, group=None) -> float:
     return float(t.item())
 
 
-class ShardPlan:
-    """Limb ownership for a key-switch at `level` (digits of Z8: D_j = [j alpha, ...))."""
+def strided_blocks(ids: list[int], world: int) -> list[list[int]]:
+    """Round-robin ownership: position k goes to rank k mod world (level drops stay balanced)."""
+    return [ids[r::world] for r in range(world)]
 
-    def __init__(self, level: int, num_q: int, num_p: int, alpha: int, world: int, rank: int):
+
+class ShardPlan:
+    """Limb ownership for a key-switch at `level` (digits of Z8: D_j = [j alpha, ...)).
+    strided=False: contiguous blocks; strided=True: round-robin (the limb-sharded evaluator,
+    whose ciphertexts lose their top limb at every Rescale)."""
+
+    def __init__(self, level: int, num_q: int, num_p: int, alpha: int, world: int, rank: int,
+                 strided: bool = False):
         self.level, self.num_q, self.num_p, self.alpha = level, num_q, num_p, alpha
         self.world, self.rank = world, rank
         self.q_ids = list(range(level + 1))
         self.p_ids = list(range(num_q, num_q + num_p))
-        self.q_blocks = limb_blocks(self.q_ids, world)
-        self.p_blocks = limb_blocks(self.p_ids, world)
+        split = strided_blocks if strided else limb_blocks
+        self.q_blocks = split(self.q_ids, world)
+        self.p_blocks = split(self.p_ids, world)
+        # the all-gathers concatenate the blocks rank by rank: positions of the natural order
+        cq = [i for b in self.q_blocks for i in b]
+        cp = [i for b in self.p_blocks for i in b]
+        self.q_perm = None if cq == self.q_ids else [cq.index(i) for i in self.q_ids]
+        self.p_perm = None if cp == self.p_ids else [cp.index(i) for i in self.p_ids]
         self.my_q = self.q_blocks[rank]
         self.my_p = self.p_blocks[rank]
         self.mine = self.my_q + self.my_p                 # this rank's limbs of PQ_l
@@ -76,6 +90,8 @@ def limb_sharded_keyswitch(ops, plan: ShardPlan, d_local, evk):
     # a3: INTT of the rank's Q limbs, then exchange #1: every rank gets all Q limbs
     y_local = ops.intt(d_local, P.my_q)
     y_all = ops.allgather(y_local, [len(b) for b in P.q_blocks])          # [B][l+1][N]
+    if P.q_perm is not None:
+        y_all = ops.take(y_all, P.q_perm)
     # a4/a5: ModUp of every digit onto this rank's own target limbs, then NTT
     if not P.my_q:
         raise ValueError("limb-sharded key-switch needs world <= level + 1 (every rank owns a Q limb)")
@@ -95,6 +111,8 @@ def limb_sharded_keyswitch(ops, plan: ShardPlan, d_local, evk):
     p_pos = [P.mine.index(t) for t in P.my_p]
     acc_p_local = ops.intt2(ops.take2(acc, p_pos), P.my_p) if p_pos else ops.empty2(acc, 0)
     acc_p_all = ops.allgather2(acc_p_local, [len(b) for b in P.p_blocks])  # [B][2][num_p][N]
+    if P.p_perm is not None:
+        acc_p_all = ops.take2(acc_p_all, P.p_perm)
     # a8/a9: ModDown BConv onto the rank's Q limbs, NTT, a10: combine
     conv = ops.ntt2(ops.bconv2(acc_p_all, P.p_ids, P.my_q), P.my_q)
     q_pos = [P.mine.index(t) for t in P.my_q]
@@ -193,6 +211,38 @@ class NeoOps:
         acc = torch.empty((B, 2, len(ids), dhat.shape[-1]), dtype=torch.uint64, device=dhat.device)
         self.neo.neo_keyip(self.ctx, evk, dhat, ids, beta, acc, B, self.stream)
         return acc
+
+    def ew(self, op, a, b, ids, out=None, scal=None, src=0, batch=None):
+        """neo_ew_limbs on the rows `ids` (a new output unless `out` is given)."""
+        if out is None:
+            shape = list(a.shape)
+            if op == self.neo.NEO_EWL_TENSOR:
+                shape[1] = 3
+            elif op == self.neo.NEO_EWL_LIFT:
+                shape = [a.shape[0], 2, len(ids), a.shape[-1]]
+            out = torch.empty(shape, dtype=torch.uint64, device=a.device)
+        if ids:
+            self.neo.neo_ew_limbs(self.ctx, op, a, b if b is not None else a, ids, out,
+                                  a.shape[0] if batch is None else batch, scal=scal, src_limb=src, stream=self.stream)
+        return out
+
+    def automorphism(self, x, g):
+        """sigma_g on every row of x (any leading shape; rows of N)."""
+        out = torch.empty_like(x)
+        rows = x.numel() // x.shape[-1]
+        if rows:
+            self.neo.neo_automorphism(self.ctx, x, rows, g, out, 1, self.stream)
+        return out
+
+    def broadcast(self, x, src):
+        if not dist.is_initialized() or dist.get_world_size(self.group) == 1:
+            return x
+        if dist.get_backend(self.group) == "nccl":
+            dist.broadcast(x.view(torch.int64), src=src, group=self.group)
+            return x
+        host = x.view(torch.int64).cpu()
+        dist.broadcast(host, src=src, group=self.group)
+        return host.to(x.device).view(torch.uint64)
 
     def moddown_combine(self, acc, conv, q_ids):
         out = torch.empty_like(acc)

@@ -108,7 +108,7 @@ class OracleOps:
         return out
 
 
-def _worker(rank, world, port, cfg, level, q):
+def _worker(rank, world, port, cfg, level, q, strided=False):
     sys.path.insert(0, ROOT)
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
@@ -123,7 +123,7 @@ def _worker(rank, world, port, cfg, level, q):
                         for j in range(prm.dnum)])
         B = 2
         d = np.stack([synth.uniform_residues(60 + b, prm.q[: level + 1], prm.N) for b in range(B)])
-        plan = ShardPlan(level, prm.num_q, prm.num_p, prm.alpha, world, rank)
+        plan = ShardPlan(level, prm.num_q, prm.num_p, prm.alpha, world, rank, strided=strided)
         ops = OracleOps(prm)
         k0, k1 = limb_sharded_keyswitch(ops, plan, np.ascontiguousarray(d[:, plan.my_q]), evk)
         ok = True
@@ -145,16 +145,18 @@ def _free_port():
     return p
 
 
-@pytest.mark.parametrize("world,cfg,level", [
-    (2, (10, 6, 2, 3), 5),      # N=2^10, 6 Q + 2 P, dnum 3: both ranks own Q and P limbs
-    (3, (10, 6, 2, 3), 4),      # rank 2 owns no P limb; partial last digit
-    (2, (10, 3, 1, 1), 2),      # dnum = 1 (one digit spans both ranks)
+@pytest.mark.parametrize("world,cfg,level,strided", [
+    (2, (10, 6, 2, 3), 5, False),      # N=2^10, 6 Q + 2 P, dnum 3: both ranks own Q and P limbs
+    (3, (10, 6, 2, 3), 4, False),      # rank 2 owns no P limb; partial last digit
+    (2, (10, 3, 1, 1), 2, False),      # dnum = 1 (one digit spans both ranks)
+    (2, (10, 6, 2, 3), 4, True),       # round-robin ownership (the sharded evaluator's plan)
+    (3, (10, 6, 2, 3), 5, True),
 ])
-def test_limb_sharded_keyswitch_gloo(world, cfg, level):
+def test_limb_sharded_keyswitch_gloo(world, cfg, level, strided):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, cfg, level, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, cfg, level, q, strided)) for r in range(world)]
     for p in procs:
         p.start()
     res = dict(q.get(timeout=300) for _ in procs)
