@@ -602,7 +602,33 @@ def run_neo(args):
                       "ms_per_bootstrap": round(bms, 3), "value": world / (bms / 1e3), "unit": "bootstraps/s",
                       "key_switches": nks,
                       "timing": f"CUDA events around {nboot} runs after 2 warm-ups, max over ranks"}
-        del bkeys, bconsts, bt
+        # config 4's multi-GPU form: the same bootstrap limb-sharded over all ranks (round-robin
+        # limbs; two all-gathers per key-switch, one limb broadcast per Rescale; NCCL).  At N = 1
+        # it runs the sharded code path on one rank (the exchange steps degenerate to copies).
+        from paper_conf_isca_jiaodwfcm0z25_b200.sharded_boot import ShardedBootstrapper
+        sbt = ShardedBootstrapper(ctx, nb, rb, bkeys, bconsts, world, rank)
+        sct0 = sbt.shard(bct, 0)
+        for _ in range(1):
+            sbt.run(sct0)
+        torch.cuda.synchronize()
+        barrier()
+        nsb = 3
+        b0.record()
+        for _ in range(nsb):
+            sbt.run(sct0)
+        b1.record()
+        torch.cuda.synchronize()
+        sms = b0.elapsed_time(b1) / nsb
+        if world > 1:
+            t = torch.tensor([sms], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            sms = float(t.item())
+        boot_block["limb_sharded"] = {
+            "ranks": world, "ms_per_bootstrap": round(sms, 3), "value": 1 / (sms / 1e3), "unit": "bootstraps/s",
+            "exchanges": "per key-switch 2 all-gathers (Q limbs before ModUp, P limbs before ModDown); "
+                         "per Rescale / ModRaise 1 broadcast of one limb (2 rows)",
+            "timing": f"CUDA events around {nsb} runs after 1 warm-up, max over ranks (one bootstrap over all ranks)"}
+        del bkeys, bconsts, bt, sbt
         torch.cuda.empty_cache()
 
     # SURVEY §8(f) row 4 / BASELINE configs[4]: the application traces (reading APP,

@@ -294,7 +294,7 @@ def neo_hmult(ctx: Context, relin: EvalKey, ct_a, ct_b, level: int, ct_out, batc
 def neo_hmult_rescale(ctx: Context, relin: EvalKey, ct_a, ct_b, level: int, ct_out, batch: int, ws, stream=None):
     """Rescale(HMULT(ct_a, ct_b)) in one call: ct_out [batch][2][level][N]."""
     _check(lib().neo_hmult_rescale(ctx.handle, relin.handle, _ptr(ct_a), _ptr(ct_b), level, _ptr(ct_out), batch,
-                                   _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_hmult_rescale", "neo_ew_limbs")
+                                   _ptr(ws), ws.numel() * 8, _stream(stream)), "neo_hmult_rescale")
 
 
 def neo_hrot(ctx: Context, rotkey: EvalKey, galois_elt: int, ct_in, level: int, ct_out, batch: int, ws,
