@@ -1,6 +1,9 @@
 // abi.cpp -- the extern "C" entry points of libneo.so (include/neo.h) and the key-switch
 // orchestrator (Fig. 5: INTT -> ModUp -> NTT -> KeyIP -> INTT -> ModDown -> NTT).
 #include <algorithm>
+#include <atomic>
+#include <map>
+#include <memory>
 #include <cstdlib>
 #include <cstring>
 #include <new>
@@ -699,6 +702,8 @@ neo_status neo_params_create(const neo_params_desc* desc, neo_ctx** out) {
     if ((desc->q == nullptr) != (desc->p == nullptr)) FAIL(NEO_EINVAL, "give both q and p or neither");
     neo_ctx* c = new (std::nothrow) neo_ctx();
     if (!c) FAIL(NEO_ENOMEM, "host allocation failed");
+    static std::atomic<unsigned long long> next_uid{0};
+    c->uid = ++next_uid;
     std::string err;
     neo_status s;
     try {
@@ -796,37 +801,61 @@ neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids
     }
     for (int j = 0; j < n_out; ++j)
         if (out_ids[j] < 0 || out_ids[j] >= nl) FAIL(NEO_EINVAL, "unknown output limb id");
-    // constants of Algorithm 1 for this (in, out) pair, passed by value (no allocation)
-    BConvTab T;
-    std::memset(&T, 0, sizeof(T));
-    T.n_in = n_in;
-    T.n_out = n_out;
-    auto mulm = [](u64 a, u64 b, u64 m) { return (u64)((u128)a * b % m); };
-    auto powm = [&](u64 a, u64 e, u64 m) {
-        u64 r = 1;
-        for (a %= m; e; e >>= 1, a = mulm(a, a, m))
-            if (e & 1) r = mulm(r, a, m);
-        return r;
-    };
-    for (int i = 0; i < n_in; ++i) {
-        u64 qi = c->mod[in_ids[i]], qh = 1;
-        for (int k = 0; k < n_in; ++k)
-            if (k != i) qh = mulm(qh, c->mod[in_ids[k]] % qi, qi);
-        u64 inv = powm(qh, qi - 2, qi);
-        T.qin[i] = qi;
-        T.qhat_inv[i] = TW{inv, (u64)(((u128)inv << 64) / qi)};
-    }
-    for (int j = 0; j < n_out; ++j) {
-        u64 t = c->mod[out_ids[j]];
-        T.tmod[j] = ModQ{t, (u64)(((u128)1 << 98) / t), (double)t, 1.0 / (double)t};
+    // constants of Algorithm 1 for this (in, out) pair, passed by value (no allocation); built
+    // once per (context, in_ids, out_ids) and cached per thread (the limb-sharded path calls
+    // this with the same id lists at every key-switch)
+    struct BcEntry { BConvTab T; BConvTC P; BMatParam bp; };
+    static thread_local std::map<std::vector<long long>, std::unique_ptr<BcEntry>> cache;
+    std::vector<long long> key{(long long)c->uid, n_in, n_out};
+    key.insert(key.end(), in_ids, in_ids + n_in);
+    key.insert(key.end(), out_ids, out_ids + n_out);
+    auto hit = cache.find(key);
+    if (hit == cache.end()) {
+        if (cache.size() > 512) cache.clear();
+        std::unique_ptr<BcEntry> e(new BcEntry);
+        BConvTab& T = e->T;
+        std::memset(&T, 0, sizeof(T));
+        T.n_in = n_in;
+        T.n_out = n_out;
+        auto mulm = [](u64 a, u64 b, u64 m) { return (u64)((u128)a * b % m); };
+        auto powm = [&](u64 a, u64 x, u64 m) {
+            u64 r = 1;
+            for (a %= m; x; x >>= 1, a = mulm(a, a, m))
+                if (x & 1) r = mulm(r, a, m);
+            return r;
+        };
         for (int i = 0; i < n_in; ++i) {
-            u64 f = 1;
+            u64 qi = c->mod[in_ids[i]], qh = 1;
             for (int k = 0; k < n_in; ++k)
-                if (k != i) f = mulm(f, c->mod[in_ids[k]] % t, t);
-            T.f_lo[i][j] = (unsigned)(f & 0x3FFFF);
-            T.f_hi[i][j] = (unsigned)(f >> 18);
+                if (k != i) qh = mulm(qh, c->mod[in_ids[k]] % qi, qi);
+            u64 inv = powm(qh, qi - 2, qi);
+            T.qin[i] = qi;
+            T.qhat_inv[i] = TW{inv, (u64)(((u128)inv << 64) / qi)};
         }
+        for (int j = 0; j < n_out; ++j) {
+            u64 t = c->mod[out_ids[j]];
+            T.tmod[j] = ModQ{t, (u64)(((u128)1 << 98) / t), (double)t, 1.0 / (double)t};
+            for (int i = 0; i < n_in; ++i) {
+                u64 f = 1;
+                for (int k = 0; k < n_in; ++k)
+                    if (k != i) f = mulm(f, c->mod[in_ids[k]] % t, t);
+                T.f_lo[i][j] = (unsigned)(f & 0x3FFFF);
+                T.f_hi[i][j] = (unsigned)(f >> 18);
+            }
+        }
+
+        if (c->use_tc && n_in <= BCTC_MAX_IN && n_out <= BCTC_MAX_OUT) {
+            std::vector<u64> sm, tm;
+            for (int i = 0; i < n_in; ++i) sm.push_back(c->mod[in_ids[i]]);
+            for (int j = 0; j < n_out; ++j) tm.push_back(c->mod[out_ids[j]]);
+            std::vector<uint8_t> bm;
+            make_bconv_tc(sm, tm, e->P, bm);
+            std::memset(&e->bp, 0, sizeof(e->bp));
+            std::memcpy(&e->bp, bm.data(), bm.size());
+        }
+        hit = cache.emplace(key, std::move(e)).first;
     }
+    const BcEntry& E = *hit->second;
     BConvIO io;
     io.in = in; io.out = out;
     io.in_bstride = (long long)n_in * c->N;
@@ -834,18 +863,9 @@ neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids
     for (int i = 0; i < n_in; ++i) io.in_off[i] = i;
     for (int j = 0; j < n_out; ++j) io.out_off[j] = j;
     if (c->use_tc && n_in <= BCTC_MAX_IN && n_out <= BCTC_MAX_OUT) {
-        std::vector<u64> sm, tm;
-        for (int i = 0; i < n_in; ++i) sm.push_back(c->mod[in_ids[i]]);
-        for (int j = 0; j < n_out; ++j) tm.push_back(c->mod[out_ids[j]]);
-        BConvTC P;
-        std::vector<uint8_t> bm;
-        make_bconv_tc(sm, tm, P, bm);
-        static thread_local BMatParam bp;
-        std::memset(&bp, 0, sizeof(bp));
-        std::memcpy(&bp, bm.data(), bm.size());
-        LAUNCH(PK_BCONV, S(st), launch_bconv_tc_param(P, io, bp, c->N, batch, c->num_sms, S(st)));
+        LAUNCH(PK_BCONV, S(st), launch_bconv_tc_param(E.P, io, E.bp, c->N, batch, c->num_sms, S(st)));
     } else {
-        LAUNCH(PK_BCONV, S(st), launch_bconv(T, io, c->N, batch, S(st)));
+        LAUNCH(PK_BCONV, S(st), launch_bconv(E.T, io, c->N, batch, S(st)));
     }
     return NEO_OK;
 }

@@ -99,13 +99,12 @@ def limb_sharded_keyswitch(ops, plan: ShardPlan, d_local, evk):
     for dj in P.digits:
         targets = [t for t in P.mine if t not in dj]
         up = ops.ntt(ops.bconv(ops.take(y_all, dj), dj, targets), targets) if targets else None
-        rows = []
-        for t in P.mine:
-            if t in dj:
-                rows.append(ops.take(d_local, [P.my_q.index(t)]))           # digit's own limb: d_t
-            else:
-                rows.append(ops.take(up, [targets.index(t)]))
-        dhat_rows.append(ops.cat(rows, axis=1))
+        # rows of d_hat_j in P.mine order: the digit's own limbs are d_t itself, the rest ModUp's
+        # outputs -- one concatenation and one row selection (not one copy per limb)
+        n_d = len(P.my_q)
+        idx = [P.my_q.index(t) if t in dj else n_d + targets.index(t) for t in P.mine]
+        both = ops.cat([d_local, up], axis=1) if up is not None else d_local
+        dhat_rows.append(ops.take(both, idx))
     acc = ops.keyip(ops.stack(dhat_rows, axis=1), P.mine, P.beta, evk)       # a6 -> [B][2][n_mine][N]
     # a7: INTT of the rank's P limbs of acc, exchange #2: every rank gets all P limbs
     p_pos = [P.mine.index(t) for t in P.my_p]
@@ -125,17 +124,31 @@ class NeoOps:
 
     def __init__(self, ctx, group=None, stream=None):
         from . import neo
-        self.neo, self.ctx, self.group, self.stream = neo, ctx, group, stream
+        # resolve the stream once: torch.cuda.current_stream() per C-ABI call costs ~15 us of host time
+        self.neo, self.ctx, self.group = neo, ctx, group
+        self.stream = stream if stream is not None else torch.cuda.current_stream()
+        self._icache = {}
 
     # ---- tensor plumbing (torch.uint64 CUDA tensors, moved through int64 views because
     #      torch implements few uint64 CUDA ops; the bits are unchanged)
-    @staticmethod
-    def take(x, idx):
-        return x.view(torch.int64)[:, idx].contiguous().view(torch.uint64)
+    def _sel(self, x, idx, dim):
+        """Rows idx of x along dim: a slice when idx is a run, else index_select with a cached
+        device index (a Python list index would be copied host->device, synchronously, per call)."""
+        xi = x.view(torch.int64)
+        if idx and list(idx) == list(range(idx[0], idx[0] + len(idx))):
+            return xi.narrow(dim, idx[0], len(idx)).contiguous().view(torch.uint64)
+        key = (tuple(idx), x.device)
+        t = self._icache.get(key)
+        if t is None:
+            t = torch.tensor(list(idx), dtype=torch.int64, device=x.device)
+            self._icache[key] = t
+        return xi.index_select(dim, t).view(torch.uint64)
 
-    @staticmethod
-    def take2(x, idx):
-        return x.view(torch.int64)[:, :, idx].contiguous().view(torch.uint64)
+    def take(self, x, idx):
+        return self._sel(x, idx, 1)
+
+    def take2(self, x, idx):
+        return self._sel(x, idx, 2)
 
     @staticmethod
     def cat(xs, axis):
