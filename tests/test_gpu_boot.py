@@ -43,3 +43,32 @@ def test_bootstrap_bit_exact_and_decodes():
     assert np.array_equal(got, want)
     zz = boot.decode_sparse(bp, got, lv, scale * delta / prm.q[0], s)
     assert np.max(np.abs(zz - z)) < 4e-3
+
+
+def test_bootstrap_graph_replay_bit_exact():
+    """The bootstrap captured as one CUDA graph (how bench.py times it) replays to the oracle's
+    result."""
+    bp = boot.tiny()
+    prm = bp.prm
+    s = ckks.secret(prm, 21, bp.h)
+    keys_np = boot.boot_keys(bp, s, 500)
+    ct0 = boot.encrypt_sparse(bp, synth.complex_slots(23, bp.n), 2.0 ** 31, s, 25)
+    want, lv, scale, consts = boot.bootstrap(bp, ct0, keys_np)
+    ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+    keys = {k: neo.EvalKey(ctx, dev(v)) for k, v in keys_np.items()}
+    for g in gboot.hoisted_rotations(prm.N, bp.n):
+        keys[("h", g)] = neo.EvalKey(ctx, dev(keys_np[g]), hoisted_galois=g)
+    b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()})
+    x = dev(ct0[None])
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):
+        b.run(x)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=side):
+            out, glv = b.run(x)
+    torch.cuda.current_stream().wait_stream(side)
+    out.zero_()
+    g.replay()
+    torch.cuda.synchronize()
+    assert glv == lv and np.array_equal(out.cpu().numpy()[0], want)
