@@ -71,6 +71,7 @@ struct RecTab {
 struct neo_ctx {
     int log_n, N, num_q, num_p, dnum, alpha, word_bits, device;
     unsigned long long uid = 0;           // unique per created context (host-side caches key on it)
+    cudaStream_t side = nullptr;          // second stream for chunked batches (fork/join on the caller's)
     std::vector<u64> mod;                 // by limb id
     std::vector<u64> psi;                 // by limb id
     std::vector<ModQ> h_mods;

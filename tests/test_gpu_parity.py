@@ -280,3 +280,37 @@ def test_hmult_rescale_fused_rejects():
     with pytest.raises(neo.NeoError):           # workspace too small
         neo.neo_hmult_rescale(ctx, relin, ct, ct, 2, torch.empty((1, 2, 2, prm.N), dtype=torch.uint64, device="cuda"),
                               1, ws[: ws.numel() // 2])
+
+
+@pytest.mark.parametrize("op", ["hrot", "hmult_rescale", "keyswitch"])
+def test_batch_larger_than_chunk(op):
+    """Batches above the library's chunk (32 ciphertexts) run as several chunks alternating
+    over two streams: every ciphertext still equals the oracle's; the workspace is two chunks'."""
+    ctx, prm = ctx_of("tiny")
+    level, batch = 2, 35
+    evk_np = rand_evk(prm, 1300)
+    key = neo.EvalKey(ctx, dev(evk_np))
+    code = {"hrot": neo.NEO_OP_HROT, "hmult_rescale": neo.NEO_OP_HMULT_RESCALE, "keyswitch": neo.NEO_OP_KEYSWITCH}[op]
+    assert ctx.workspace_size(code, level, batch) == 2 * ctx.workspace_size(code, level, 32)   # two chunks in flight
+    ws = ctx.workspace(code, level, batch)
+    a = np.stack([rand_ct(prm, level, 1310 + 4 * b) for b in range(batch)])
+    g = pow(5, 3, 2 * prm.N)
+    if op == "hrot":
+        out = torch.empty((batch, 2, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+        neo.neo_hrot(ctx, key, g, dev(a), level, out, batch, ws)
+        want = [ckks.hrot(prm, a[b], g, level, evk_np) for b in range(batch)]
+    elif op == "hmult_rescale":
+        b_ = np.stack([rand_ct(prm, level, 1312 + 4 * b) for b in range(batch)])
+        out = torch.empty((batch, 2, level, prm.N), dtype=torch.uint64, device="cuda")
+        neo.neo_hmult_rescale(ctx, key, dev(a), dev(b_), level, out, batch, ws)
+        want = [ckks.rescale(prm, ckks.hmult(prm, a[b], b_[b], level, evk_np), level) for b in range(batch)]
+    else:
+        d = np.ascontiguousarray(a[:, 0])
+        o0 = torch.empty((batch, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+        o1 = torch.empty_like(o0)
+        neo.neo_keyswitch(ctx, key, dev(d), level, o0, o1, batch, ws)
+        out = torch.stack([o0, o1], dim=1)
+        want = [np.stack(ckks.keyswitch(prm, d[b], level, evk_np)) for b in range(batch)]
+    got = host(out)
+    for bb in range(batch):
+        assert np.array_equal(got[bb], want[bb]), bb
