@@ -41,6 +41,7 @@ class BootParams:
     n: int                                   # complex slots (sparse packing), n | N/2
     r: int                                   # squarings in EvalMod
     h: int = 192                             # secret Hamming weight (bounds I)
+    fft_levels: int = 0                      # 0: dense diagonal method; k: factored CtS / StC, k levels each
 
     @property
     def M(self) -> int:
@@ -50,15 +51,32 @@ class BootParams:
     def top(self) -> int:
         return self.prm.max_level
 
-    def levels_used(self) -> int:            # CtS 1, EvalMod 1 + 3 + 1 + r + 1, StC 1
-        return 1 + (1 + 3 + 1 + self.r + 1) + 1
+    def levels_used(self) -> int:            # CtS, EvalMod 1 + 3 + 1 + r + 1, StC
+        lt = max(1, self.fft_levels)
+        return lt + (1 + 3 + 1 + self.r + 1) + lt
 
     def rotations(self) -> list[int]:
-        """Galois elements: SubSum (rotations by n 2^j), the diagonal method (1..n-1), conj."""
+        """Galois elements: SubSum (rotations by n 2^j), the linear transforms' rotations, conj."""
         N = self.prm.N
         gs = [pow(5, self.n << j, 2 * N) for j in range(int(math.log2(self.M)))]
-        gs += [pow(5, d, 2 * N) for d in range(1, self.n)]
+        if self.fft_levels:
+            for grp in fft_groups(N, self.fft_levels, inverse=True) + fft_groups(N, self.fft_levels, inverse=False):
+                babies, giants = bsgs_amounts(grp, N)
+                gs += [pow(5, d % (N // 2), 2 * N) for d in babies + giants]
+        else:
+            gs += [pow(5, d, 2 * N) for d in range(1, self.n)]
         return sorted(set(gs)) + [2 * N - 1]
+
+
+def tiny_full() -> BootParams:
+    """Full-slot test set: N = 2^12 (2048 slots), 24 Q + 2 P limbs (dnum 12: alpha = 2), r = 9,
+    h = 32, CoeffToSlot / SlotToCoeff as 3 levels each (special-FFT groups of 4, 4, 3 stages)."""
+    return BootParams(ckks.Params(12, 24, 2, 12), n=2048, r=9, h=32, fft_levels=3)
+
+
+def set_b_full() -> BootParams:
+    """Set-B with all N/2 = 32768 slots, r = 12, CtS / StC as 3 levels of 5 special-FFT stages."""
+    return BootParams(ckks.set_b(), n=32768, r=12, h=192, fft_levels=3)
 
 
 def tiny() -> BootParams:
@@ -98,6 +116,144 @@ def _monomial(prm: ckks.Params, k: int, sign: int, level: int) -> np.ndarray:
     c = np.zeros(prm.N, dtype=np.int64)
     c[k] = sign
     return ckks.ntt(prm, ckks.reduce_signed(prm, c, ids), ids)
+
+
+# --------------------------------------------------------------------------- special FFT (full slots)
+# With n = N/2 slots the slot vector of a polynomial t (at scale 1) is z = U (t_lo + i t_hi),
+# U[j][k] = zeta^(5^j k), zeta = e^(i pi / N) (zeta^(5^j N/2) = i).  U factors into log2(n)
+# butterfly stages after a bit-reversal P (the "special FFT" of the CKKS encoder):
+#     U = F_n ... F_4 F_2 P,   F_len: out[i+j] = u + w v, out[i+j+len/2] = u - w v,
+#     u = in[i+j], v = in[i+j+len/2], w = zeta^((5^j mod 4 len) 2N / (4 len)),  j < len/2,
+# so CoeffToSlot = P U^-1 = F_2^-1 ... F_n^-1 (slots end in bit-reversed order, which the
+# slot-wise EvalMod does not see) and SlotToCoeff = U P^-1 = F_n ... F_2.  Every stage is three
+# rotation diagonals; a level applies a group of consecutive stages merged into one matrix
+# (2^(k+1) - 1 diagonals for k stages), evaluated baby-step giant-step.
+
+def _rot(v: np.ndarray, d: int) -> np.ndarray:
+    """rot_d(v)[p] = v[(p + d) mod n] (a left rotation by d, Z11)."""
+    return np.roll(v, -d)
+
+
+def sfft_stages(N: int, inverse: bool) -> list[dict]:
+    """[F_2, F_4, ..., F_n] (inverse=False) or [F_2^-1, ..., F_n^-1], each {amount d: diagonal}
+    with (F x)[p] = sum_d diag_d[p] x[p + d]."""
+    n = N // 2
+    e5 = np.array([pow(5, j, 2 * N) for j in range(n)], dtype=np.int64)
+    p = np.arange(n)
+    out = []
+    ln = 2
+    while ln <= n:
+        lenh, lenq = ln // 2, 4 * ln
+        j = p % ln
+        first = j < lenh
+        jj = np.where(first, j, j - lenh)
+        w = np.exp(1j * np.pi * ((e5[jj] % lenq) * (2 * N // lenq)) / N)
+        if not inverse:
+            d0 = np.where(first, 1.0, -w)
+            dp = np.where(first, w, 0.0)
+            dm = np.where(first, 0.0, 1.0)
+        else:                                    # [[1, w], [1, -w]]^-1 = 1/2 [[1, 1], [w^-1, -w^-1]]
+            wi = np.conj(w)
+            d0 = np.where(first, 0.5, -0.5 * wi)
+            dp = np.where(first, 0.5, 0.0)
+            dm = np.where(first, 0.0, 0.5 * wi)
+        out.append({0: d0.astype(complex), lenh: dp.astype(complex), -lenh: dm.astype(complex)})
+        ln *= 2
+    return out
+
+
+def diag_compose(B: dict, A: dict, n: int) -> dict:
+    """Diagonals of B A: (B A x)[p] = sum_{d1, d2} B_d1[p] A_d2[p + d1] x[p + d1 + d2]."""
+    out = {}
+    for d1, b in B.items():
+        for d2, a in A.items():
+            d = d1 + d2
+            d = (d + n // 2) % n - n // 2                     # signed representative
+            out[d] = out.get(d, 0) + b * _rot(a, d1)
+    return out
+
+
+def fft_groups(N: int, levels: int, inverse: bool) -> list[dict]:
+    """The merged matrices applied one per level.  CoeffToSlot (inverse=True) applies
+    F_n^-1 first and F_2^-1 last; SlotToCoeff applies F_2 first.  The log2(n) stages split into
+    `levels` consecutive groups (sizes differ by at most one, larger groups first)."""
+    n = N // 2
+    st = sfft_stages(N, inverse)
+    order = st[::-1] if inverse else st
+    L = len(order)
+    sizes = [L // levels + (1 if i < L % levels else 0) for i in range(levels)]
+    groups, k = [], 0
+    for sz in sizes:
+        M = order[k]
+        for F in order[k + 1:k + sz]:
+            M = diag_compose(F, M, n)
+        groups.append(M)
+        k += sz
+    return groups
+
+
+def bsgs_amounts(diags: dict, N: int) -> tuple[list[int], list[int]]:
+    """Baby-step rotations (b h, b = 1 .. b1-1) and giant-step rotations (g b1 h, g != 0) of the
+    baby-step giant-step evaluation of a merged group (amounts d = m h, m = g b1 + b)."""
+    b1, h, ms = _bsgs_shape(diags)
+    babies = sorted({m % b1 for m in ms} - {0})
+    giants = sorted({m // b1 for m in ms} - {0})
+    return [b * h for b in babies], [g * b1 * h for g in giants]
+
+
+def _bsgs_shape(diags: dict):
+    h = min(abs(d) for d in diags if d != 0)
+    ms = sorted(d // h for d in diags)
+    b1 = 1
+    while b1 * b1 < len(ms):
+        b1 *= 2
+    return b1, h, ms
+
+
+def _lintrans_bsgs(prm, ct, lv, diags: dict, name: str, keys: dict, const):
+    """sum_d diag_d (.) rot_d(ct) = sum_g rot_{g b1 h}( sum_b rot_{-g b1 h}(diag_m) (.) rot_{b h}(ct) ),
+    babies hoisted (one ModUp), one PMULT level at scale q_lv, then Rescale."""
+    N, n = prm.N, prm.N // 2
+    b1, h, ms = _bsgs_shape(diags)
+    babies = sorted({m % b1 for m in ms} - {0})
+    gs = [pow(5, (b * h) % n, 2 * N) for b in babies]
+    rots = {0: ct}
+    if gs:
+        for b, r in zip(babies, ckks.hrot_hoisted(prm, ct, gs, lv, [keys[g] for g in gs])):
+            rots[b] = r
+    acc = None
+    for g in sorted({m // b1 for m in ms}):
+        inner = None
+        for m in ms:
+            if m // b1 != g:
+                continue
+            b = m % b1
+            pt = const(f"{name}_g{g}_b{b}", lambda m=m, g=g: _pt_full(prm, _rot(diags[m * h], -g * b1 * h),
+                                                                      float(prm.q[lv]), lv))
+            t = ckks.pmult(prm, rots[b], pt, lv)
+            inner = t if inner is None else ckks.hadd(prm, inner, t, lv)
+        if g:
+            ga = pow(5, (g * b1 * h) % n, 2 * N)
+            inner = ckks.hrot(prm, inner, ga, lv, keys[ga])
+        acc = inner if acc is None else ckks.hadd(prm, acc, inner, lv)
+    return ckks.rescale(prm, acc, lv)
+
+
+def fft_transform(bp: BootParams, ct: np.ndarray, lv: int, keys: dict, inverse: bool, tag: str, const=None):
+    """CoeffToSlot (inverse=True: slots <- P U^-1 slots) or SlotToCoeff (slots <- U P^-1 slots)
+    as bp.fft_levels BSGS levels from level lv.  Returns (ct, lv - fft_levels).  `const(name,
+    make)` supplies / records the plaintext diagonals (default: encode on the fly)."""
+    const = const or (lambda name, make: make())
+    for k, grp in enumerate(fft_groups(bp.prm.N, bp.fft_levels, inverse)):
+        ct = _lintrans_bsgs(bp.prm, ct, lv, grp, f"{tag}{k}", keys, const)
+        lv -= 1
+    return ct, lv
+
+
+def _pt_full(prm: ckks.Params, slots: np.ndarray, scale: float, level: int) -> np.ndarray:
+    ids = list(range(level + 1))
+    m = ckks.encode(prm.N, np.asarray(slots, dtype=complex), scale)
+    return ckks.ntt(prm, ckks.reduce_signed(prm, m, ids), ids)
 
 
 # --------------------------------------------------------------------------- ops
@@ -160,6 +316,9 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
     for j in range(int(math.log2(M))):
         ct = ckks.hadd(prm, ct, rot(ct, pow(5, n << j, 2 * N), L), L)
 
+    def lintrans_fft(ct, lv, inverse, tag):   # factored: fft_levels levels, BSGS per level
+        return fft_transform(bp, ct, lv, keys, inverse, tag, const)
+
     def lintrans(ct, lv, A, tag):        # slots <- A slots (diagonal method), scale kept, one level
         # the n - 1 rotations of the same ciphertext are hoisted (one ModUp, reading BOOT-H)
         gs = [pow(5, d, 2 * N) for d in range(1, n)]
@@ -171,9 +330,13 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
             acc = t if acc is None else ckks.hadd(prm, acc, t, lv)
         return ckks.rescale(prm, acc, lv)
 
-    W = _xi_matrix(n)
-    ct = lintrans(ct, L, np.linalg.inv(W) / M, "cts")              # CoeffToSlot
-    lv = L - 1
+    if bp.fft_levels:
+        W = None
+        ct, lv = lintrans_fft(ct, L, True, "cts")                  # CoeffToSlot (bit-reversed slots)
+    else:
+        W = _xi_matrix(n)
+        ct = lintrans(ct, L, np.linalg.inv(W) / M, "cts")          # CoeffToSlot
+        lv = L - 1
     cj = rot(ct, 2 * N - 1, lv)
     x1 = ckks.hadd(prm, ct, cj, lv)                                 # 2 Re(w)
     x2 = ckks.pmult(prm, hsub(prm, ct, cj, lv), const("mono_mi", lambda: _monomial(prm, N // 2, -1, lv)), lv)  # 2 Im(w)
@@ -226,6 +389,9 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
     assert (lv1, s1) == (lv2, s2)
     lv = lv1
     w = ckks.hadd(prm, f1, ckks.pmult(prm, f2, const("mono_i", lambda: _monomial(prm, N // 2, 1, lv)), lv), lv)
+    if bp.fft_levels:
+        out, lo = lintrans_fft(w, lv, False, "stc")                 # SlotToCoeff
+        return out, lo, s1, consts
     out = lintrans(w, lv, W, "stc")                                 # SlotToCoeff
     return out, lv - 1, s1, consts
 

@@ -62,3 +62,110 @@ def test_bootstrap_decodes_to_input(booted):
     assert lv == bp.top - bp.levels_used()
     got = boot.decode_sparse(bp, out, lv, scale * delta / bp.prm.q[0], s)
     assert np.max(np.abs(got - z)) < 4e-3
+
+
+# --------------------------------------------------------------------------- full-slot (special FFT)
+
+def _u_matrix(N):
+    n = N // 2
+    e5 = [pow(5, j, 2 * N) for j in range(n)]
+    return np.array([[np.exp(1j * math.pi * ((e5[j] * k) % (2 * N)) / N) for k in range(n)] for j in range(n)])
+
+
+def _brev_perm(n):
+    bits = n.bit_length() - 1
+    return np.array([int(format(i, f"0{bits}b")[::-1], 2) for i in range(n)])
+
+
+def _apply(diags, x):
+    return sum(v * np.roll(x, -d) for d, v in diags.items())
+
+
+def test_special_fft_factorises_the_slot_matrix():
+    """U = F_n ... F_2 P with U[j][k] = zeta^(5^j k) (decode's definition, checked against
+    ckks.decode) and P the bit reversal; the inverse stages give P U^-1."""
+    N = 1 << 8
+    n = N // 2
+    U = _u_matrix(N)
+    rng = np.random.default_rng(5)
+    t = rng.standard_normal(N)
+    z_dec = ckks.decode(N, [float(v) for v in t], 1.0)
+    assert np.max(np.abs(U @ (t[:n] + 1j * t[n:]) - z_dec)) < 1e-9
+    x = rng.standard_normal(n) + 1j * rng.standard_normal(n)
+    px = np.empty(n, dtype=complex)
+    px[_brev_perm(n)] = x                                   # (P x)[brev(i)] = x[i]
+    y = px
+    for F in boot.sfft_stages(N, inverse=False):
+        y = _apply(F, y)
+    assert np.max(np.abs(y - U @ x)) < 1e-9
+    y = U @ x
+    for F in boot.sfft_stages(N, inverse=True)[::-1]:
+        y = _apply(F, y)
+    assert np.max(np.abs(y - px)) < 1e-9
+
+
+def test_fft_groups_equal_the_stage_products():
+    N = 1 << 10
+    rng = np.random.default_rng(6)
+    x = rng.standard_normal(N // 2) + 1j * rng.standard_normal(N // 2)
+    for inverse in (True, False):
+        st = boot.sfft_stages(N, inverse)
+        want = x
+        for F in (st[::-1] if inverse else st):
+            want = _apply(F, want)
+        got = x
+        for G in boot.fft_groups(N, 3, inverse):
+            got = _apply(G, got)
+        assert np.max(np.abs(got - want)) < 1e-9
+        for G in boot.fft_groups(N, 3, inverse):          # k = 3 stages: <= 2^(k+1) - 1 diagonals
+            assert len(G) <= 15                          # (fewer when amounts wrap mod n)
+
+
+def test_homomorphic_coeff_to_slot_full():
+    """Encrypted full-slot CoeffToSlot decodes to P U^-1 z (the bit-reversed complex packing of
+    the coefficients), and SlotToCoeff brings it back to z.  Tolerances: CoeffToSlot's entries
+    are O(1/n), so its output carries only the key-switch noise of ~10 rotations per level at
+    scale ~2^36 (~2^-26 relative each): 1e-5 absolute.  SlotToCoeff = U P^-1 has entries of
+    modulus 1 summed over n = 2048 terms, so iid input noise of rms s becomes sqrt(n) s ~ 45 s
+    (s ~ 2^-22 here), plus its own rotations: 2e-4 absolute on the round trip."""
+    bp = boot.tiny_full()
+    prm = bp.prm
+    s = ckks.secret(prm, 41, bp.h)
+    keys = boot.boot_keys(bp, s, 900)
+    z = synth.complex_slots(43, prm.N // 2)
+    delta = float(prm.q[prm.max_level])
+    L = prm.max_level
+    ct = ckks.encrypt(prm, ckks.encode(prm.N, z, delta), s, L, 45)
+    cts, lv = boot.fft_transform(bp, ct, L, keys, True, "cts")
+    assert lv == L - bp.fft_levels
+    m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, cts, s, lv), list(range(lv + 1)))
+    w = ckks.decode(prm.N, m, delta)
+    U = _u_matrix(prm.N)
+    want = np.empty_like(z)
+    want[_brev_perm(prm.N // 2)] = np.linalg.solve(U, z)
+    assert np.max(np.abs(w - want)) < 1e-5
+    back, lv2 = boot.fft_transform(bp, cts, lv, keys, False, "stc")
+    m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, back, s, lv2), list(range(lv2 + 1)))
+    assert np.max(np.abs(ckks.decode(prm.N, m, delta) - z)) < 2e-4
+
+
+@pytest.fixture(scope="module")
+def booted_full():
+    bp = boot.tiny_full()
+    s = ckks.secret(bp.prm, 51, bp.h)
+    keys = boot.boot_keys(bp, s, 600)
+    z = synth.complex_slots(53, bp.prm.N // 2)
+    delta = 2.0 ** 31
+    ct0 = boot.encrypt_sparse(bp, z, delta, s, 55)
+    out, lv, scale, consts = boot.bootstrap(bp, ct0, keys)
+    return bp, s, z, delta, out, lv, scale
+
+
+def test_full_slot_bootstrap_decodes_to_input(booted_full):
+    """All N/2 slots.  Same error budget as the sparse test (EvalMod's 2^r amplification of
+    the coefficient-level noise, the sine's cubic error), with the coefficient-to-slot gain
+    sqrt(N) instead of sqrt(2n) of the sparse case: 4e-3 absolute."""
+    bp, s, z, delta, out, lv, scale = booted_full
+    assert lv == bp.top - bp.levels_used()
+    got = boot.decode_sparse(bp, out, lv, scale * delta / bp.prm.q[0], s)
+    assert np.max(np.abs(got - z)) < 4e-3

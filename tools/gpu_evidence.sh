@@ -1,12 +1,14 @@
 # Round evidence: GPU tests, smoke, full bench line, ncu launch list and full captures.
 set -x
-timeout 1200 python -m pytest tests -m gpu -q 2>&1 | tail -5
+timeout 1500 python -m pytest tests -m gpu -q 2>&1 | tail -5
 timeout 300 python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -3
-timeout 900 python bench.py > gpurun_out/bench_full.json 2> gpurun_out/bench_full.err; tail -3 gpurun_out/bench_full.err
+timeout 1200 python bench.py > gpurun_out/bench_full.json 2> gpurun_out/bench_full.err; tail -3 gpurun_out/bench_full.err
 cat gpurun_out/bench_full.json
+# launch list / full captures of the headline step only (the secondary blocks are skipped)
+NCUARGS="--steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-hoisted --no-klss --no-boot --no-apps --batch-hrot 0 --graph 0 --streams 1"
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
-    python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-hoisted --graph 0 --streams 1 > /dev/null 2>&1
+    python bench.py $NCUARGS > /dev/null 2>&1
 wc -l gpurun_out/launches.csv
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_ntt_col|k_ntt_row|k_bconv_tc|k_keyip" -s 40 -c 8 \
-    -o gpurun_out/prof_top python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-hoisted --graph 0 --streams 1 > gpurun_out/ncu_top.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_ntt_col|k_ntt_row|k_bconv_tc|k_keyip|k_hmr_fold|k_tensor" -s 40 -c 10 \
+    -o gpurun_out/prof_top python bench.py $NCUARGS > gpurun_out/ncu_top.log 2>&1
 tail -2 gpurun_out/ncu_top.log
