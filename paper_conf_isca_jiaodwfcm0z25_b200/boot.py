@@ -19,22 +19,79 @@ from . import neo
 D_TAYLOR = 7
 
 
-def levels_used(r: int) -> int:
-    return 1 + (1 + 3 + 1 + r + 1) + 1
+def levels_used(r: int, fft_levels: int = 0) -> int:
+    lt = max(1, fft_levels)
+    return lt + (1 + 3 + 1 + r + 1) + lt
 
 
-def rotations(N: int, n: int) -> list[int]:
-    """Galois elements the run needs: SubSum (n 2^j), the diagonal method (1..n-1), conj (2N-1)."""
+# ---- full-slot linear transforms (n = N/2): the special FFT's log2(n) butterfly stages, stage
+# F_len mixing slots p and p + len/2 (rotation amounts 0, +-len/2), merged into fft_levels
+# groups; CoeffToSlot applies the stages from len = n down to 2, SlotToCoeff from 2 up to n.
+# Only the rotation structure is computed here (the diagonals are plaintext inputs).
+
+def fft_plan(N: int, fft_levels: int, inverse: bool) -> list[tuple[int, int, list[int]]]:
+    """Per level: (h, b1, ms) -- the group's rotation amounts are m h (m in ms, signed mod N/2),
+    evaluated baby-step giant-step with m = g b1 + b, b in [0, b1)."""
+    n = N // 2
+    lenhs = [1 << k for k in range(int(math.log2(n)))]           # F_2 .. F_n: len/2 = 1 .. n/2
+    order = lenhs[::-1] if inverse else lenhs
+    L = len(order)
+    sizes = [L // fft_levels + (1 if i < L % fft_levels else 0) for i in range(fft_levels)]
+    plan, k = [], 0
+    for sz in sizes:
+        amounts = {0}
+        for lh in order[k:k + sz]:
+            amounts = {((a + e * lh) + n // 2) % n - n // 2 for a in amounts for e in (-1, 0, 1)}
+        if sz == 1:                                                # an unmerged stage keeps +-n/2 apart
+            amounts = {0, order[k], -order[k]}
+        h = min(abs(a) for a in amounts if a)
+        ms = sorted(a // h for a in amounts)
+        b1 = 1
+        while b1 * b1 < len(ms):
+            b1 *= 2
+        plan.append((h, b1, ms))
+        k += sz
+    return plan
+
+
+def fft_rotations(N: int, fft_levels: int) -> tuple[list[int], list[int]]:
+    """(hoisted baby-step Galois elements, giant-step Galois elements) of both transforms."""
+    n = N // 2
+    hoisted, giant = set(), set()
+    for inverse in (True, False):
+        for h, b1, ms in fft_plan(N, fft_levels, inverse):
+            hoisted |= {pow(5, ((m % b1) * h) % n, 2 * N) for m in ms if m % b1}
+            giant |= {pow(5, ((m // b1) * b1 * h) % n, 2 * N) for m in ms if m // b1}
+    return sorted(hoisted), sorted(giant)
+
+
+def rotations(N: int, n: int, fft_levels: int = 0) -> list[int]:
+    """Galois elements the run needs: SubSum (n 2^j), the linear transforms, conj (2N-1)."""
     M = N // (2 * n)
     gs = [pow(5, n << j, 2 * N) for j in range(int(math.log2(M)))]
-    gs += [pow(5, d, 2 * N) for d in range(1, n)]
+    if fft_levels:
+        hz, gz = fft_rotations(N, fft_levels)
+        gs += hz + gz
+    else:
+        gs += [pow(5, d, 2 * N) for d in range(1, n)]
     return sorted(set(gs)) + [2 * N - 1]
 
 
-def const_levels(top: int, n: int, r: int) -> dict:
+def _fft_const_names(N: int, fft_levels: int, inverse: bool, tag: str) -> list[list[str]]:
+    out = []
+    for k, (h, b1, ms) in enumerate(fft_plan(N, fft_levels, inverse)):
+        out.append([f"{tag}{k}_g{m // b1}_b{m % b1}" for m in ms])
+    return out
+
+
+def const_levels(top: int, n: int, r: int, N: int = 0, fft_levels: int = 0) -> dict:
     """Level of every plaintext constant (the same schedule as run())."""
-    lv = {f"cts_{d}": top for d in range(n)}
-    l1 = top - 1
+    F = max(1, fft_levels)
+    if fft_levels:
+        lv = {nm: top - k for k, names in enumerate(_fft_const_names(N, fft_levels, True, "cts")) for nm in names}
+    else:
+        lv = {f"cts_{d}": top for d in range(n)}
+    l1 = top - F
     lv["mono_mi"] = l1
     for tag in ("re", "im"):
         lv[f"{tag}theta"] = l1
@@ -47,13 +104,20 @@ def const_levels(top: int, n: int, r: int) -> dict:
         lv[f"{tag}sin"] = lt - 1 - r
     lf = l1 - (1 + 3 + 1 + r + 1)
     lv["mono_i"] = lf
-    for d in range(n):
-        lv[f"stc_{d}"] = lf
+    if fft_levels:
+        for k, names in enumerate(_fft_const_names(N, fft_levels, False, "stc")):
+            lv.update({nm: lf - k for nm in names})
+    else:
+        for d in range(n):
+            lv[f"stc_{d}"] = lf
     return lv
 
 
-def hoisted_rotations(N: int, n: int) -> list[int]:
-    """Galois elements of the diagonal method's hoisted rotations (5^d, d = 1 .. n-1)."""
+def hoisted_rotations(N: int, n: int, fft_levels: int = 0) -> list[int]:
+    """Galois elements of the hoisted rotations: the diagonal method's 5^d (d = 1 .. n-1), or the
+    full-slot transforms' baby steps."""
+    if fft_levels:
+        return fft_rotations(N, fft_levels)[0]
     return [pow(5, d, 2 * N) for d in range(1, n)]
 
 
@@ -61,8 +125,10 @@ class Bootstrapper:
     """keys: {'relin': EvalKey, g: EvalKey for g in rotations(N, n), ('h', g): hoisted EvalKey
     (neo_evk_create_hoisted) for g in hoisted_rotations(N, n)}; consts: {name: tensor}."""
 
-    def __init__(self, ctx: neo.Context, n: int, r: int, keys: dict, consts: dict, stream=None):
+    def __init__(self, ctx: neo.Context, n: int, r: int, keys: dict, consts: dict, stream=None,
+                 fft_levels: int = 0):
         self.ctx, self.n, self.r, self.keys, self.consts, self.stream = ctx, n, r, keys, consts, stream
+        self.fft_levels = fft_levels
         self.N = ctx.N
         self.top = ctx.num_q - 1
         ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_MODRAISE, neo.NEO_OP_HROT_HOISTED,
@@ -150,6 +216,39 @@ class Bootstrapper:
                           stream=self.stream)
         return self.rescale(acc, lv)
 
+    def rot_hoisted(self, ct, gs, lv):
+        """[sigma-rotations of ct by the Galois elements gs] sharing one ModUp."""
+        out = self._ct(lv, ct.shape[0], (len(gs),))
+        neo.neo_hrot_hoisted(self.ctx, [self.keys[("h", g)] for g in gs], ct, lv, out, ct.shape[0], self.ws,
+                             self.stream)
+        return [out[i] for i in range(len(gs))]
+
+    def pmul_sum(self, cts, names, lv):
+        """sum_k PMULT(cts[k], consts[names[k]]) in one launch."""
+        out = self._ct(lv, cts[0].shape[0])
+        neo.neo_pmult_acc(self.ctx, cts, [self.consts[nm] for nm in names], lv, out, cts[0].shape[0],
+                          pt_shared=True, stream=self.stream)
+        return out
+
+    def lintrans_fft(self, ct, lv, inverse, tag):
+        """Full-slot CoeffToSlot / SlotToCoeff: fft_levels baby-step giant-step levels."""
+        N, n = self.N, self.N // 2
+        for k, (h, b1, ms) in enumerate(fft_plan(N, self.fft_levels, inverse)):
+            babies = sorted({m % b1 for m in ms} - {0})
+            rots = {0: ct}
+            if babies:
+                rots.update(zip(babies, self.rot_hoisted(ct, [pow(5, (b * h) % n, 2 * N) for b in babies], lv)))
+            acc = None
+            for g in sorted({m // b1 for m in ms}):
+                bs = [m % b1 for m in ms if m // b1 == g]
+                inner = self.pmul_sum([rots[b] for b in bs], [f"{tag}{k}_g{g}_b{b}" for b in bs], lv)
+                if g:
+                    inner = self.rot(inner, pow(5, (g * b1 * h) % n, 2 * N), lv)
+                acc = inner if acc is None else self.add(acc, inner, lv)
+            ct = self.rescale(acc, lv)
+            lv -= 1
+        return ct, lv
+
     # ---- the run
     def run(self, ct0: torch.Tensor):
         """ct0 [1][2][1][N] (level 0) -> (ct, level)."""
@@ -160,8 +259,11 @@ class Bootstrapper:
             ct = self.add(ct, self.rot(ct, pow(5, n << j, 2 * N), L), L)
         lintrans = self.lintrans
 
-        ct = lintrans(ct, L, "cts")                                    # CoeffToSlot
-        lv = L - 1
+        if self.fft_levels:
+            ct, lv = self.lintrans_fft(ct, L, True, "cts")             # CoeffToSlot (bit-reversed)
+        else:
+            ct = lintrans(ct, L, "cts")                                # CoeffToSlot
+            lv = L - 1
         cj = self.rot(ct, 2 * N - 1, lv)
         xs = self._ct(lv, 2)                                            # [x1, x2]: one batch of 2
         self.add(ct, cj, lv, out=xs[0:1])                               # 2 Re(w)
@@ -196,5 +298,7 @@ class Bootstrapper:
         # EvalMod of the real and imaginary halves as one batch of 2
         f, lv = evalmod(xs, lv, ("re", "im"))
         w = self.add(f[0:1], self.pmul(f[1:2], "mono_i", lv), lv)
+        if self.fft_levels:
+            return self.lintrans_fft(w, lv, False, "stc")              # SlotToCoeff
         out = lintrans(w, lv, "stc")                                   # SlotToCoeff
         return out, lv - 1

@@ -29,8 +29,9 @@ class ShardedBootstrapper(Bootstrapper):
     consts: full plaintexts [l+1][N] (each rank keeps its own rows)."""
 
     def __init__(self, ctx: neo.Context, n: int, r: int, keys: dict, consts: dict, world: int, rank: int,
-                 group=None, stream=None):
+                 group=None, stream=None, fft_levels: int = 0):
         self.ctx, self.n, self.r, self.keys, self.stream = ctx, n, r, keys, stream
+        self.fft_levels = fft_levels
         self.N = ctx.N
         self.top = ctx.num_q - 1
         self.world, self.rank = world, rank
@@ -135,6 +136,21 @@ class ShardedBootstrapper(Bootstrapper):
         ids = self.own(L)
         lifted = self.ops.ew(neo.NEO_EWL_LIFT, coef, None, ids, src=0)        # [1][2][n][N] coefficients
         return self.ops.ntt(lifted.view(2, len(ids), self.N), ids).view(1, 2, len(ids), self.N)
+
+    def rot_hoisted(self, ct, gs, lv):
+        """Hoisted rotations (BOOT-H) on shards: per g the key-switch of c1 under the hoisted key,
+        then sigma_g of (c0 + k0', k1')."""
+        out = []
+        for g in gs:
+            k0, k1 = self._ks(ct[:, 1].contiguous(), lv, self.keys[("h", g)])
+            out.append(self.ops.automorphism(self._plus_k(ct[:, 0].contiguous(), k0, k1, lv), g))
+        return out
+
+    def pmul_sum(self, cts, names, lv):
+        acc = self.pmul(cts[0], names[0], lv)
+        for c, nm in zip(cts[1:], names[1:]):
+            acc = self.add(acc, self.pmul(c, nm, lv), lv)
+        return acc
 
     def lintrans(self, ct, lv, tag):
         """The diagonal method with hoisted rotations (BOOT-H): for g = 5^d the key-switch of c1

@@ -72,3 +72,31 @@ def test_bootstrap_graph_replay_bit_exact():
     g.replay()
     torch.cuda.synchronize()
     assert glv == lv and np.array_equal(out.cpu().numpy()[0], want)
+
+
+def test_full_slot_bootstrap_bit_exact_and_decodes():
+    """All N/2 slots: factored CoeffToSlot / SlotToCoeff (3 BSGS levels each, hoisted baby steps,
+    fused PMULT sums) + EvalMod, bit-exact vs oracle/boot.py and decoding to the input."""
+    bp = boot.tiny_full()
+    prm = bp.prm
+    s = ckks.secret(prm, 51, bp.h)
+    keys_np = boot.boot_keys(bp, s, 600)
+    z = synth.complex_slots(53, prm.N // 2)
+    delta = 2.0 ** 31
+    ct0 = boot.encrypt_sparse(bp, z, delta, s, 55)
+    want, lv, scale, consts = boot.bootstrap(bp, ct0, keys_np)
+    ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+    assert gboot.rotations(prm.N, bp.n, bp.fft_levels) == bp.rotations()
+    cl = gboot.const_levels(bp.top, bp.n, bp.r, prm.N, bp.fft_levels)
+    assert set(cl) == set(consts) and all(consts[k].shape[0] == cl[k] + 1 for k in cl)
+    keys = {k: neo.EvalKey(ctx, dev(v)) for k, v in keys_np.items()}
+    for g in gboot.hoisted_rotations(prm.N, bp.n, bp.fft_levels):
+        keys[("h", g)] = neo.EvalKey(ctx, dev(keys_np[g]), hoisted_galois=g)
+    b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()}, fft_levels=bp.fft_levels)
+    got, glv = b.run(dev(ct0[None]))
+    torch.cuda.synchronize()
+    assert glv == lv
+    got = got.cpu().numpy()[0]
+    assert np.array_equal(got, want)
+    zz = boot.decode_sparse(bp, got, lv, scale * delta / prm.q[0], s)
+    assert np.max(np.abs(zz - z)) < 4e-3
