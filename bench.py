@@ -595,106 +595,89 @@ def run_neo(args):
     boot_block = None
     if not args.no_boot:
         from paper_conf_isca_jiaodwfcm0z25_b200 import boot as gboot
-        nb, rb = 8, 12
+        from paper_conf_isca_jiaodwfcm0z25_b200.sharded_boot import ShardedBootstrapper
         gen = torch.Generator(device="cuda")
         gen.manual_seed(seed + 123)
         rnd = lambda *shape: torch.randint(0, 1 << 35, shape, dtype=torch.int64, device="cuda",
                                            generator=gen).view(torch.uint64)
-        bkeys = {"relin": neo.EvalKey(ctx, rnd(DNUM, 2, NUM_Q + NUM_P, N))}
-        for gg in gboot.rotations(N, nb):
-            bkeys[gg] = neo.EvalKey(ctx, rnd(DNUM, 2, NUM_Q + NUM_P, N))
-        for gg in gboot.hoisted_rotations(N, nb):
-            bkeys[("h", gg)] = neo.EvalKey(ctx, rnd(DNUM, 2, NUM_Q + NUM_P, N), hoisted_galois=gg)
-        bconsts = {k: rnd(l + 1, N) for k, l in gboot.const_levels(LEVEL, nb, rb).items()}
-        bt = gboot.Bootstrapper(ctx, nb, rb, bkeys, bconsts)
+        evk_b = rnd(DNUM, 2, NUM_Q + NUM_P, N)          # one random key serves every Galois element
         bct = rnd(1, 2, 1, N)
-        for _ in range(2):
-            bt.run(bct)
-        torch.cuda.synchronize()
-        barrier()
-        nboot = 5
-        b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        b0.record()
-        for _ in range(nboot):
-            bt.run(bct)
-        b1.record()
-        torch.cuda.synchronize()
-        bms = b0.elapsed_time(b1) / nboot
-        if world > 1:
-            t = torch.tensor([bms], dtype=torch.float64, device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            bms = float(t.item())
-        # the Python orchestration issues ~1,500 C-ABI calls per bootstrap: replay it as a CUDA
-        # graph (captured once; the same calls on the same buffers) -- the headline number
-        ref_out = bt.run(bct)[0].clone()
-        bgraph, bg_out = graph_capture(lambda: bt.run(bct)[0])
-        gms = None
-        if bgraph is not None:
-            bgraph.replay()
-            torch.cuda.synchronize()
-            assert _same(bg_out, ref_out), "graph replay of the bootstrap differs from the eager run"
+
+        def time_runs(run, reps):
             barrier()
+            b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             b0.record()
-            for _ in range(nboot):
-                bgraph.replay()
+            for _ in range(reps):
+                run()
             b1.record()
             torch.cuda.synchronize()
-            gms = b0.elapsed_time(b1) / nboot
+            t_ = b0.elapsed_time(b1) / reps
             if world > 1:
-                t = torch.tensor([gms], dtype=torch.float64, device="cuda")
+                t = torch.tensor([t_], dtype=torch.float64, device="cuda")
                 dist.all_reduce(t, op=dist.ReduceOp.MAX)
-                gms = float(t.item())
-        nks = int(math.log2(N // (2 * nb))) + 2 * (nb - 1) + 2 + 2 * (7 + rb)
-        best = gms if gms is not None else bms
-        boot_block = {"config": "Set-B (N=2^16, L=35, dnum=3), 8 sparse slots, r=12 squarings, levels 35 -> 15",
-                      "ms_per_bootstrap": round(best, 3), "value": world / (best / 1e3), "unit": "bootstraps/s",
-                      "graph": gms is not None, "ms_eager": round(bms, 3),
-                      "key_switches": nks,
-                      "timing": f"CUDA events around {nboot} graph replays (and {nboot} eager runs) after warm-ups, "
-                                "max over ranks; replay output checked equal to the eager run"}
-        # config 4's multi-GPU form: the same bootstrap limb-sharded over all ranks (round-robin
-        # limbs; two all-gathers per key-switch, one limb broadcast per Rescale; NCCL).  At N = 1
-        # it runs the sharded code path on one rank (the exchange steps degenerate to copies).
-        from paper_conf_isca_jiaodwfcm0z25_b200.sharded_boot import ShardedBootstrapper
-        sbt = ShardedBootstrapper(ctx, nb, rb, bkeys, bconsts, world, rank)
-        sct0 = sbt.shard(bct, 0)
-        for _ in range(1):
-            sbt.run(sct0)
-        torch.cuda.synchronize()
-        # the orchestration is host-bound (~25 C-ABI calls per key-switch from Python), so the
-        # whole run is captured once as a CUDA graph (NCCL collectives are capturable; the gloo
-        # fallback used when ranks share a GPU is not, and then this times eagerly)
-        sref = sbt.run(sct0)[0].clone()
-        s_side = torch.cuda.Stream()
-        sbt_g = ShardedBootstrapper(ctx, nb, rb, bkeys, bconsts, world, rank, stream=s_side)
-        sgraph, sg_out = graph_capture(lambda: sbt_g.run(sct0)[0], side=s_side)
-        if sgraph is not None:
-            sgraph.replay()
+                t_ = float(t.item())
+            return t_
+
+        def boot_case(nb, rb, fl, sharded):
+            """Time one bootstrap configuration: eager and as a CUDA-graph replay (output checked
+            equal), and optionally the limb-sharded form over all ranks (graph, NCCL)."""
+            keys = {"relin": neo.EvalKey(ctx, evk_b)}
+            for gg in gboot.rotations(N, nb, fl):
+                keys[gg] = neo.EvalKey(ctx, evk_b)
+            for gg in gboot.hoisted_rotations(N, nb, fl):
+                keys[("h", gg)] = neo.EvalKey(ctx, evk_b, hoisted_galois=gg)
+            consts = {k: rnd(l + 1, N) for k, l in gboot.const_levels(LEVEL, nb, rb, N, fl).items()}
+            bt = gboot.Bootstrapper(ctx, nb, rb, keys, consts, fft_levels=fl)
+            for _ in range(2):
+                bt.run(bct)
             torch.cuda.synchronize()
-            assert _same(sg_out, sref), "graph replay of the sharded bootstrap differs from the eager run"
-        barrier()
-        nsb = 3
-        b0.record()
-        for _ in range(nsb):
-            if sgraph is not None:
-                sgraph.replay()
-            else:
-                sbt.run(sct0)
-        b1.record()
-        torch.cuda.synchronize()
-        sms = b0.elapsed_time(b1) / nsb
-        if world > 1:
-            t = torch.tensor([sms], dtype=torch.float64, device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            sms = float(t.item())
-        boot_block["limb_sharded"] = {
-            "ranks": world, "ms_per_bootstrap": round(sms, 3), "value": 1 / (sms / 1e3), "unit": "bootstraps/s",
-            "exchanges": "per key-switch 2 all-gathers (Q limbs before ModUp, P limbs before ModDown); "
-                         "per Rescale / ModRaise 1 broadcast of one limb (2 rows)",
-            "graph": sgraph is not None,
-            "timing": f"CUDA events around {nsb} runs after 1 warm-up, max over ranks (one bootstrap over all ranks)"}
-        del bkeys, bconsts, bt, sbt, sbt_g, sgraph, bgraph
-        torch.cuda.empty_cache()
+            eager = time_runs(lambda: bt.run(bct), 3)
+            ref_out = bt.run(bct)[0].clone()
+            bgraph, bg_out = graph_capture(lambda: bt.run(bct)[0])
+            gms = None
+            if bgraph is not None:
+                bgraph.replay()
+                torch.cuda.synchronize()
+                assert _same(bg_out, ref_out), "graph replay of the bootstrap differs from the eager run"
+                gms = time_runs(bgraph.replay, 5)
+            best = gms if gms is not None else eager
+            out = {"ms_per_bootstrap": round(best, 3), "value": world / (best / 1e3), "unit": "bootstraps/s",
+                   "graph": gms is not None, "ms_eager": round(eager, 3),
+                   "levels": f"{LEVEL} -> {LEVEL - gboot.levels_used(rb, fl)}",
+                   "rotation_keys": len(gboot.rotations(N, nb, fl)) + len(gboot.hoisted_rotations(N, nb, fl))}
+            if sharded:
+                # config 4's multi-GPU form: the same bootstrap limb-sharded over all ranks
+                # (round-robin limbs; two all-gathers per key-switch, one limb broadcast per
+                # Rescale; NCCL).  At N = 1 the sharded code path runs on one rank.
+                sbt = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, fft_levels=fl)
+                sct0 = sbt.shard(bct, 0)
+                sref = sbt.run(sct0)[0].clone()
+                s_side = torch.cuda.Stream()
+                sbt_g = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, stream=s_side, fft_levels=fl)
+                sgraph, sg_out = graph_capture(lambda: sbt_g.run(sct0)[0], side=s_side)
+                if sgraph is not None:
+                    sgraph.replay()
+                    torch.cuda.synchronize()
+                    assert _same(sg_out, sref), "graph replay of the sharded bootstrap differs from the eager run"
+                sms = time_runs(sgraph.replay if sgraph is not None else (lambda: sbt.run(sct0)), 3)
+                out["limb_sharded"] = {
+                    "ranks": world, "ms_per_bootstrap": round(sms, 3), "value": 1 / (sms / 1e3),
+                    "unit": "bootstraps/s", "graph": sgraph is not None,
+                    "exchanges": "per key-switch 2 all-gathers (Q limbs before ModUp, P limbs before ModDown); "
+                                 "per Rescale / ModRaise 1 broadcast of one limb (2 rows)"}
+                del sbt, sbt_g, sgraph
+            del keys, consts, bt, bgraph
+            torch.cuda.empty_cache()
+            return out
+
+        full = boot_case(N // 2, 12, 3, sharded=True)
+        sparse = boot_case(8, 12, 0, sharded=False)
+        boot_block = dict(full, config="Set-B (N=2^16, L=35, dnum=3), full slots (32768), r=12 squarings, "
+                                       "CoeffToSlot / SlotToCoeff as 3 special-FFT BSGS levels each",
+                          timing="CUDA events around 5 graph replays (3 eager runs) after warm-ups, max over "
+                                 "ranks; replay output checked equal to the eager run; keys / constants synthetic",
+                          sparse_8_slots=sparse)
+        del evk_b
 
     # SURVEY §8(f) row 4 / BASELINE configs[4]: the application traces (reading APP,
     # paper_conf_isca_jiaodwfcm0z25_b200.apps) at Set-B on every rank (DP): one HELR iteration
