@@ -319,22 +319,26 @@ k_ew_limbs(const __grid_constant__ EwlArgs A) {
 }
 
 // ------------------------------------------------------------------ fused HMULT + Rescale
-// One thread per (bc, coefficient): c_l once, then the l rows i < l (coalesced per row).
+// One thread per (coefficient, group of kFoldRows rows, bc): c_l once per thread from three
+// L2-resident reads, then its rows (a single loop over all l rows per thread was latency-bound
+// at 512 CTAs; one row per thread re-read c_l's inputs 35 times: 18.8 / 30 us per step).
+constexpr int kFoldRows = 6;
 __global__ void __launch_bounds__(256)
 k_hmr_fold(const __grid_constant__ HmrFoldArgs A) {
     pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
-    const int bc = blockIdx.y;
+    const int i0 = blockIdx.y * kFoldRows, bc = blockIdx.z;
     if (n >= A.N) return;
     const size_t row = (size_t)A.N, base = (size_t)bc * (A.l + 1) * row + n;
     const ModQ ml = A.mods[A.l];
     u64 cv;
-    if (A.lazy) cv = d2u(canon(__longlong_as_double((long long)A.conv[base + (size_t)A.l * row]), ml.qd, ml.qinv));
-    else cv = A.conv[base + (size_t)A.l * row];
-    const u64 cl = add_mod(shoup(sub_mod(A.accl[(size_t)bc * row + n], cv, ml.q), A.pinv_l, ml.q),
-                           A.dl[(size_t)bc * row + n], ml.q);
+    if (A.lazy) cv = d2u(canon(__longlong_as_double((long long)__ldg(A.conv + base + (size_t)A.l * row)), ml.qd, ml.qinv));
+    else cv = __ldg(A.conv + base + (size_t)A.l * row);
+    const u64 cl = add_mod(shoup(sub_mod(__ldg(A.accl + (size_t)bc * row + n), cv, ml.q), A.pinv_l, ml.q),
+                           __ldg(A.dl + (size_t)bc * row + n), ml.q);
     const double cld = u2d(cl);
-    for (int i = 0; i < A.l; ++i) {
+    const int i1 = min(A.l, i0 + kFoldRows);
+    for (int i = i0; i < i1; ++i) {
         const ModQ m = A.mods[i];
         u64* p = A.conv + base + (size_t)i * row;
         if (A.lazy) {
@@ -469,7 +473,7 @@ cudaError_t launch_ew_limbs(const EwlArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_ew_limbs, dim3((A.N + 255) / 256, A.n, batch), dim3(256), 0, st, A);
 }
 cudaError_t launch_hmr_fold(const HmrFoldArgs& A, int bc, cudaStream_t st) {
-    return launch_k(k_hmr_fold, dim3((A.N + 255) / 256, bc), dim3(256), 0, st, A);
+    return launch_k(k_hmr_fold, dim3((A.N + 255) / 256, (A.l + kFoldRows - 1) / kFoldRows, bc), dim3(256), 0, st, A);
 }
 cudaError_t launch_modraise(const u64* coef, u64* out, const ModQ* mods, int limbs, int N, int bc, cudaStream_t st) {
     return launch_k(k_modraise, dim3((N + 255) / 256, limbs, bc), dim3(256), 0, st, coef, out, mods, limbs, N);
