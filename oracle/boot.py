@@ -252,7 +252,7 @@ def fft_transform(bp: BootParams, ct: np.ndarray, lv: int, keys: dict, inverse: 
 
 def _pt_full(prm: ckks.Params, slots: np.ndarray, scale: float, level: int) -> np.ndarray:
     ids = list(range(level + 1))
-    m = ckks.encode(prm.N, np.asarray(slots, dtype=complex), scale)
+    m = ckks.encode_fft(prm.N, np.asarray(slots, dtype=complex), scale)
     return ckks.ntt(prm, ckks.reduce_signed(prm, m, ids), ids)
 
 

@@ -560,15 +560,40 @@ def _slot_exponents(N: int) -> np.ndarray:
     return e
 
 
+_ROOTS = {}
+
+
+def _roots(N: int, sign: int) -> np.ndarray:
+    """exp(sign i pi e / N) for e < 2N: the same float operations as evaluating the exponential
+    at the angle (e mod 2N) pi / N directly, tabulated (a lookup instead of a complex exp)."""
+    key = (N, sign)
+    if key not in _ROOTS:
+        _ROOTS[key] = np.exp(sign * 1j * (np.arange(2 * N, dtype=np.int64).astype(np.float64) * (np.pi / N)))
+    return _ROOTS[key]
+
+
 def encode(N: int, z: np.ndarray, delta: float) -> np.ndarray:
     """m = round(Delta * tau^-1(z)), m_k = (2/N) Re sum_j z_j zeta_j^-k (half away from 0)."""
     ej = _slot_exponents(N)
     k = np.arange(N, dtype=np.int64)
     acc = np.zeros(N, dtype=np.float64)
+    roots = _roots(N, -1)
     for lo in range(0, N // 2, 64):
-        ang = (np.outer(ej[lo:lo + 64], k) % (2 * N)).astype(np.float64) * (np.pi / N)
-        acc += np.real(z[lo:lo + 64] @ np.exp(-1j * ang))
+        acc += np.real(z[lo:lo + 64] @ roots[np.outer(ej[lo:lo + 64], k) % (2 * N)])
     x = delta * (2.0 / N) * acc
+    return (np.sign(x) * np.floor(np.abs(x) + 0.5)).astype(np.int64)
+
+
+def encode_fft(N: int, z: np.ndarray, delta: float) -> np.ndarray:
+    """encode() evaluated with one length-2N FFT: the slots and their conjugates placed at the
+    odd exponents 5^j and 2N - 5^j give sum_e Z_e zeta^(-e k) = 2 Re sum_j z_j zeta_j^-k.  Same
+    value up to floating-point rounding order (|difference| <= 1 after rounding, pinned in
+    tests/test_oracle_ntt.py); used for the many plaintext diagonals of bootstrapping."""
+    ej = _slot_exponents(N)
+    Z = np.zeros(2 * N, dtype=np.complex128)
+    Z[ej] = z
+    Z[2 * N - ej] = np.conj(z)
+    x = delta / N * np.real(np.fft.fft(Z)[:N])
     return (np.sign(x) * np.floor(np.abs(x) + 0.5)).astype(np.int64)
 
 
@@ -578,7 +603,7 @@ def decode(N: int, m: list, delta: float) -> np.ndarray:
     k = np.arange(N, dtype=np.int64)
     mf = np.array([float(v) for v in m], dtype=np.float64)
     z = np.empty(N // 2, dtype=np.complex128)
+    roots = _roots(N, 1)
     for lo in range(0, N // 2, 64):
-        ang = (np.outer(ej[lo:lo + 64], k) % (2 * N)).astype(np.float64) * (np.pi / N)
-        z[lo:lo + 64] = np.exp(1j * ang) @ mf
+        z[lo:lo + 64] = roots[np.outer(ej[lo:lo + 64], k) % (2 * N)] @ mf
     return z / delta

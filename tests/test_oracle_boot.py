@@ -121,17 +121,22 @@ def test_fft_groups_equal_the_stage_products():
             assert len(G) <= 15                          # (fewer when amounts wrap mod n)
 
 
-def test_homomorphic_coeff_to_slot_full():
+@pytest.fixture(scope="module")
+def full_keys():
+    bp = boot.tiny_full()
+    s = ckks.secret(bp.prm, 51, bp.h)
+    return bp, s, boot.boot_keys(bp, s, 600)
+
+
+def test_homomorphic_coeff_to_slot_full(full_keys):
     """Encrypted full-slot CoeffToSlot decodes to P U^-1 z (the bit-reversed complex packing of
     the coefficients), and SlotToCoeff brings it back to z.  Tolerances: CoeffToSlot's entries
     are O(1/n), so its output carries only the key-switch noise of ~10 rotations per level at
     scale ~2^36 (~2^-26 relative each): 1e-5 absolute.  SlotToCoeff = U P^-1 has entries of
     modulus 1 summed over n = 2048 terms, so iid input noise of rms s becomes sqrt(n) s ~ 45 s
     (s ~ 2^-22 here), plus its own rotations: 2e-4 absolute on the round trip."""
-    bp = boot.tiny_full()
+    bp, s, keys = full_keys
     prm = bp.prm
-    s = ckks.secret(prm, 41, bp.h)
-    keys = boot.boot_keys(bp, s, 900)
     z = synth.complex_slots(43, prm.N // 2)
     delta = float(prm.q[prm.max_level])
     L = prm.max_level
@@ -150,10 +155,8 @@ def test_homomorphic_coeff_to_slot_full():
 
 
 @pytest.fixture(scope="module")
-def booted_full():
-    bp = boot.tiny_full()
-    s = ckks.secret(bp.prm, 51, bp.h)
-    keys = boot.boot_keys(bp, s, 600)
+def booted_full(full_keys):
+    bp, s, keys = full_keys
     z = synth.complex_slots(53, bp.prm.N // 2)
     delta = 2.0 ** 31
     ct0 = boot.encrypt_sparse(bp, z, delta, s, 55)

@@ -93,3 +93,15 @@ def test_set_b_fast_ntt_sampled_against_definition():
             assert int(f[k, idx]) == L.or_ntt_point(_core.ptr(row), prm.N, prm.moduli[i],
                                                     prm.psi[i], int(idx))
     assert np.array_equal(ckks.intt(prm, f, ids), x)
+
+
+def test_encode_fft_matches_the_definition():
+    """encode_fft (one FFT) and encode (the definition, direct sums) agree to within one after
+    rounding (floating-point order only; almost all coefficients equal), and decode back."""
+    import synth
+    for N, delta in ((1 << 8, 2.0 ** 30), (1 << 12, 2.0 ** 36)):
+        z = synth.complex_slots(17, N // 2)
+        a, b = ckks.encode(N, z, delta), ckks.encode_fft(N, z, delta)
+        assert np.max(np.abs(a - b)) <= 1
+        assert np.mean(a != b) < 0.01
+        assert np.max(np.abs(ckks.decode(N, [float(v) for v in b], delta) - z)) < 1e-6
