@@ -17,9 +17,9 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _run(rank, world, port, path, q):
+def _run(rank, world, port, path, q, full=False):
     try:
-        q.put((rank, _run_inner(rank, world, port, path)))
+        q.put((rank, _run_full(rank, world, port) if full else _run_inner(rank, world, port, path)))
     except Exception as e:                       # report instead of hanging the parent
         import traceback
         q.put((rank, "".join(traceback.format_exception(e))))
@@ -74,6 +74,50 @@ def _run_inner(rank, world, port, path):
             dist.destroy_process_group()
 
 
+def _run_full(rank, world, port):
+    """Full-slot bootstrap (special-FFT CoeffToSlot / SlotToCoeff) on shards against the
+    single-GPU Bootstrapper on the same inputs (bit-exact; the single-GPU full-slot run is
+    itself checked against oracle/boot.py in test_gpu_boot.py).  Keys, constants and the input
+    are seeded uniform residues: the comparison is exact modular arithmetic, so no oracle run
+    (and no multi-GB key file) is needed here."""
+    sys.path.insert(0, ROOT)
+    import synth
+    from oracle import boot
+    from paper_conf_isca_jiaodwfcm0z25_b200 import boot as gboot
+    from paper_conf_isca_jiaodwfcm0z25_b200 import neo
+    from paper_conf_isca_jiaodwfcm0z25_b200.sharded_boot import ShardedBootstrapper
+    if world > 1:
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        bp = boot.tiny_full()
+        prm = bp.prm
+        ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+        dev = lambda a: torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint64)).cuda()
+        evk = np.stack([np.stack([synth.uniform_residues(800 + 2 * j + c, prm.moduli, prm.N) for c in range(2)])
+                        for j in range(prm.dnum)])
+        keys = {"relin": neo.EvalKey(ctx, dev(evk))}
+        for g in gboot.rotations(prm.N, bp.n, bp.fft_levels):
+            keys[g] = neo.EvalKey(ctx, dev(evk))
+        for g in gboot.hoisted_rotations(prm.N, bp.n, bp.fft_levels):
+            keys[("h", g)] = neo.EvalKey(ctx, dev(evk), hoisted_galois=g)
+        cl = gboot.const_levels(bp.top, bp.n, bp.r, prm.N, bp.fft_levels)
+        consts = {k: dev(synth.uniform_residues(900 + i, prm.q[: l + 1], prm.N)) for i, (k, l) in
+                  enumerate(sorted(cl.items()))}
+        ct0 = dev(np.stack([synth.uniform_residues(990 + c, prm.q[:1], prm.N) for c in range(2)])[None])
+        ref, lv = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, consts, fft_levels=bp.fft_levels).run(ct0)
+        sb = ShardedBootstrapper(ctx, bp.n, bp.r, keys, consts, world, rank, fft_levels=bp.fft_levels)
+        out, glv = sb.run(sb.shard(ct0, 0))
+        torch.cuda.synchronize()
+        ok = glv == lv and np.array_equal(out.cpu().numpy(), ref.cpu().numpy()[:, :, sb.own(lv)])
+        return True if ok else ["full-slot bootstrap"]
+    finally:
+        if world > 1:
+            dist.destroy_process_group()
+
+
 def _port():
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
@@ -116,6 +160,20 @@ def test_sharded_bootstrap_bit_exact(world, oracle_file):
     for p in procs:
         p.start()
     res = dict(q.get(timeout=600) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+    assert all(res[r] is True for r in range(world)), res
+
+
+def test_sharded_full_slot_bootstrap_bit_exact():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_run, args=(r, world, port, None, q, True)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=900) for _ in procs)
     for p in procs:
         p.join(timeout=60)
     assert all(res[r] is True for r in range(world)), res
