@@ -458,7 +458,10 @@ def run_neo(args):
     # ops/clk/SM (tools/microbench/pipes.cu) x SMs x the max SM clock.
     fp64 = None
     if dom in ("ntt_col", "ntt_row"):
-        ops = {"ntt_col": 430 * 45.4 + 122 * 48.4, "ntt_row": 430 * 30.8 + 122 * 27.8}[dom] * (1 << LOG_N) * B
+        # forward / inverse limb rows per step: HROT 180 / 60; HMULT+Rescale 178 / 64 fused
+        # (250 / 62 as separate calls); per-element FP64 ops from the SASS counts (ncu)
+        fw, iv = (358, 124) if args.fused_rescale else (430, 122)
+        ops = {"ntt_col": fw * 45.4 + iv * 48.4, "ntt_row": fw * 30.8 + iv * 27.8}[dom] * (1 << LOG_N) * B
         try:
             mhz = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["sm_max_mhz"])
         except Exception:
