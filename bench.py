@@ -673,10 +673,10 @@ def run_neo(args):
             torch.cuda.empty_cache()
             return out
 
-        full = boot_case(N // 2, 12, 3, sharded=True)
+        full = boot_case(N // 2, 12, 4, sharded=True)
         sparse = boot_case(8, 12, 0, sharded=False)
         boot_block = dict(full, config="Set-B (N=2^16, L=35, dnum=3), full slots (32768), r=12 squarings, "
-                                       "CoeffToSlot / SlotToCoeff as 3 special-FFT BSGS levels each",
+                                       "CoeffToSlot / SlotToCoeff as 4 special-FFT BSGS levels each (stages 4-4-4-3)",
                           timing="CUDA events around 5 graph replays (3 eager runs) after warm-ups, max over "
                                  "ranks; replay output checked equal to the eager run; keys / constants synthetic",
                           sparse_8_slots=sparse)

@@ -68,15 +68,20 @@ class BootParams:
         return sorted(set(gs)) + [2 * N - 1]
 
 
-def tiny_full() -> BootParams:
-    """Full-slot test set: N = 2^12 (2048 slots), 24 Q + 2 P limbs (dnum 12: alpha = 2), r = 9,
-    h = 32, CoeffToSlot / SlotToCoeff as 3 levels each (special-FFT groups of 4, 4, 3 stages)."""
-    return BootParams(ckks.Params(12, 24, 2, 12), n=2048, r=9, h=32, fft_levels=3)
+def tiny_full(fft_levels: int = 3) -> BootParams:
+    """Full-slot test set: N = 2^12 (2048 slots), r = 9, h = 32, CoeffToSlot / SlotToCoeff as
+    fft_levels levels each.  3 levels: 24 Q + 2 P limbs (dnum 12: alpha = 2), output level 2;
+    4 levels: 25 Q + 3 P limbs (dnum 9: alpha = 3), output level 1."""
+    if fft_levels == 3:
+        return BootParams(ckks.Params(12, 24, 2, 12), n=2048, r=9, h=32, fft_levels=3)
+    return BootParams(ckks.Params(12, 21 + fft_levels, 3, -(-(21 + fft_levels) // 3)), n=2048, r=9, h=32,
+                      fft_levels=fft_levels)
 
 
 def set_b_full() -> BootParams:
-    """Set-B with all N/2 = 32768 slots, r = 12, CtS / StC as 3 levels of 5 special-FFT stages."""
-    return BootParams(ckks.set_b(), n=32768, r=12, h=192, fft_levels=3)
+    """Set-B with all N/2 = 32768 slots, r = 12, CtS / StC as 4 levels of 4-4-4-3 special-FFT
+    stages (levels 35 -> 9)."""
+    return BootParams(ckks.set_b(), n=32768, r=12, h=192, fft_levels=4)
 
 
 def tiny() -> BootParams:

@@ -74,10 +74,11 @@ def test_bootstrap_graph_replay_bit_exact():
     assert glv == lv and np.array_equal(out.cpu().numpy()[0], want)
 
 
-def test_full_slot_bootstrap_bit_exact_and_decodes():
+@pytest.mark.parametrize("fft_levels", [3, 4])
+def test_full_slot_bootstrap_bit_exact_and_decodes(fft_levels):
     """All N/2 slots: factored CoeffToSlot / SlotToCoeff (3 BSGS levels each, hoisted baby steps,
     fused PMULT sums) + EvalMod, bit-exact vs oracle/boot.py and decoding to the input."""
-    bp = boot.tiny_full()
+    bp = boot.tiny_full(fft_levels)
     prm = bp.prm
     s = ckks.secret(prm, 51, bp.h)
     keys_np = boot.boot_keys(bp, s, 600)
@@ -99,4 +100,4 @@ def test_full_slot_bootstrap_bit_exact_and_decodes():
     got = got.cpu().numpy()[0]
     assert np.array_equal(got, want)
     zz = boot.decode_sparse(bp, got, lv, scale * delta / prm.q[0], s)
-    assert np.max(np.abs(zz - z)) < 4e-3
+    assert np.max(np.abs(zz - z)) < 1e-2          # test_oracle_boot.py: sqrt(N) slot gain
