@@ -51,7 +51,7 @@ typedef enum {
 
 /* Operation codes for neo_workspace_size. */
 enum { NEO_OP_KEYSWITCH = 0, NEO_OP_HMULT = 1, NEO_OP_HROT = 2, NEO_OP_RESCALE = 3, NEO_OP_HROT_HOISTED = 4,
-       NEO_OP_DOUBLE_RESCALE = 5, NEO_OP_MODRAISE = 6, NEO_OP_HMULT_RESCALE = 7 };
+       NEO_OP_DOUBLE_RESCALE = 5, NEO_OP_MODRAISE = 6, NEO_OP_HMULT_RESCALE = 7, NEO_OP_HROT_SUM = 8 };
 
 /* Parameter description (Table 1, Table 4).
  *  log_n      : log2 N; this build supports 12 and 16 (N = 2^12 tiny config, 2^16 Set-B).
@@ -186,6 +186,18 @@ neo_status neo_evk_create_hoisted(const neo_ctx* ctx, const uint64_t* evk, uint3
 neo_status neo_hrot_hoisted(const neo_ctx* ctx, const neo_evk* const* keys, int32_t n_rot,
                             const uint64_t* ct_in, int32_t level, uint64_t* ct_out, int32_t batch,
                             void* ws, size_t ws_bytes, neo_stream_t stream);
+
+/* Sum of rotations with one ModDown (the giant steps of a baby-step giant-step linear
+ * transform; reading BOOT-G):  ct_out = (sum_k sigma_{g_k}(c0_k) + k0, k1) with
+ * (k0, k1) = ModDown( sum_k KeyIP(ModUp(sigma_{g_k}(c1_k)), keys[k]) ), the KeyIP outputs summed
+ * in PQ_l (Table 2).  Decrypts to sum_k rot_{g_k}(m_k); saves n - 1 ModDowns against n
+ * neo_hrot calls (a different, equally valid ciphertext: ModDown's floor rounding is applied once).
+ * keys[k]: neo_evk_create rotation keys (KSGen(s, sigma_{g_k}(s)), L184); galois[k] odd < 2N;
+ * cts: host array of n device pointers, each [batch][2][level+1][N]; ct_out likewise, not
+ * aliasing any input; 1 <= n <= 64; ws >= neo_workspace_size(ctx, NEO_OP_HROT_SUM, level, batch). */
+neo_status neo_hrot_sum(const neo_ctx* ctx, const neo_evk* const* keys, const uint32_t* galois, int32_t n,
+                        const uint64_t* const* cts, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
+                        size_t ws_bytes, neo_stream_t stream);
 
 /* Building blocks of the limb-sharded key-switch (each rank owns a subset of
  * the limbs of PQ_l and calls these on its own limbs between NCCL all-gathers):

@@ -226,7 +226,7 @@ def _lintrans_bsgs(prm, ct, lv, diags: dict, name: str, keys: dict, const):
     if gs:
         for b, r in zip(babies, ckks.hrot_hoisted(prm, ct, gs, lv, [keys[g] for g in gs])):
             rots[b] = r
-    acc = None
+    acc, rot_in, rot_g = None, [], []
     for g in sorted({m // b1 for m in ms}):
         inner = None
         for m in ms:
@@ -238,10 +238,49 @@ def _lintrans_bsgs(prm, ct, lv, diags: dict, name: str, keys: dict, const):
             t = ckks.pmult(prm, rots[b], pt, lv)
             inner = t if inner is None else ckks.hadd(prm, inner, t, lv)
         if g:
-            ga = pow(5, (g * b1 * h) % n, 2 * N)
-            inner = ckks.hrot(prm, inner, ga, lv, keys[ga])
-        acc = inner if acc is None else ckks.hadd(prm, acc, inner, lv)
+            rot_in.append(inner)
+            rot_g.append(pow(5, (g * b1 * h) % n, 2 * N))
+        else:
+            acc = inner
+    if rot_in:                                   # the giant steps' rotations share one ModDown
+        r = hrot_sum(prm, rot_in, rot_g, lv, [keys[ga] for ga in rot_g])
+        acc = r if acc is None else ckks.hadd(prm, acc, r, lv)
     return ckks.rescale(prm, acc, lv)
+
+
+def moddown(prm: ckks.Params, acc: np.ndarray, level: int) -> tuple:
+    """Steps a7-a10 of the key-switch (Table 2, Z9) on a KeyIP output acc [2][E][N] (PQ_l,
+    NTT form): (acc_c[Q] - NTT(BConv_{P->Q}(INTT(acc_c[P])))) P^-1."""
+    q_ids = list(range(level + 1))
+    p_ids = prm.p_ids
+    pinv = [pow(prm.P % prm.moduli[i], -1, prm.moduli[i]) for i in q_ids]
+    out = []
+    for c in range(2):
+        acc_p = ckks.intt(prm, acc[c][level + 1:], p_ids)
+        conv = ckks.ntt(prm, ckks.bconv(prm, acc_p, p_ids, q_ids), q_ids)
+        out.append(ckks.scalar_mul(prm, ckks.sub(prm, acc[c][: level + 1], conv, q_ids), pinv, q_ids))
+    return out[0], out[1]
+
+
+def hrot_sum(prm: ckks.Params, cts: list, gs: list, level: int, rotkeys: list) -> np.ndarray:
+    """sum_k HROTATE(cts[k], gs[k]) with one ModDown (reading BOOT-G, the giant steps of a
+    baby-step giant-step transform): the KeyIP outputs acc_k = KeyIP(ModUp(sigma_g(c1_k))) are
+    summed in PQ_l and ModDown runs once:  (sum_k sigma_g(c0_k) + k0, k1), (k0, k1) =
+    ModDown(sum_k acc_k).  Decrypts to the sum of the rotations (ModDown is linear up to its
+    floor rounding), a different but equally valid ciphertext than summing separate HROTATEs."""
+    ids = list(range(level + 1))
+    E = level + 1 + prm.num_p
+    ext = ids + prm.p_ids
+    acc = np.zeros((2, E, prm.N), dtype=np.uint64)
+    c0 = np.zeros((level + 1, prm.N), dtype=np.uint64)
+    for ct, g, key in zip(cts, gs, rotkeys):
+        tr = {}
+        ckks.keyswitch(prm, ckks.automorphism_ntt(ct[1], g), level, key, trace=tr)
+        for c in range(2):
+            acc[c] = ckks.add(prm, acc[c], tr["acc"][c], ext)
+        c0 = ckks.add(prm, c0, ckks.automorphism_ntt(ct[0], g), ids)
+    k0, k1 = moddown(prm, acc, level)
+    return np.stack([ckks.add(prm, c0, k0, ids), k1])
 
 
 def fft_transform(bp: BootParams, ct: np.ndarray, lv: int, keys: dict, inverse: bool, tag: str, const=None):

@@ -132,7 +132,7 @@ class Bootstrapper:
         self.N = ctx.N
         self.top = ctx.num_q - 1
         ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_MODRAISE, neo.NEO_OP_HROT_HOISTED,
-               neo.NEO_OP_HMULT_RESCALE)
+               neo.NEO_OP_HMULT_RESCALE, neo.NEO_OP_HROT_SUM)
         wsn = max(ctx.workspace_size(op, self.top, 2) for op in ops)
         self._stack = {}
         self.ws = torch.empty(wsn // 8, dtype=torch.uint64, device="cuda")
@@ -223,6 +223,13 @@ class Bootstrapper:
                              self.stream)
         return [out[i] for i in range(len(gs))]
 
+    def rot_sum(self, cts, gs, lv):
+        """sum_k HROTATE(cts[k], gs[k]) with one ModDown (neo_hrot_sum, reading BOOT-G)."""
+        out = self._ct(lv, cts[0].shape[0])
+        neo.neo_hrot_sum(self.ctx, [self.keys[g] for g in gs], gs, cts, lv, out, cts[0].shape[0], self.ws,
+                         self.stream)
+        return out
+
     def pmul_sum(self, cts, names, lv):
         """sum_k PMULT(cts[k], consts[names[k]]) in one launch."""
         out = self._ct(lv, cts[0].shape[0])
@@ -238,13 +245,18 @@ class Bootstrapper:
             rots = {0: ct}
             if babies:
                 rots.update(zip(babies, self.rot_hoisted(ct, [pow(5, (b * h) % n, 2 * N) for b in babies], lv)))
-            acc = None
+            acc, rin, rg = None, [], []
             for g in sorted({m // b1 for m in ms}):
                 bs = [m % b1 for m in ms if m // b1 == g]
                 inner = self.pmul_sum([rots[b] for b in bs], [f"{tag}{k}_g{g}_b{b}" for b in bs], lv)
                 if g:
-                    inner = self.rot(inner, pow(5, (g * b1 * h) % n, 2 * N), lv)
-                acc = inner if acc is None else self.add(acc, inner, lv)
+                    rin.append(inner)
+                    rg.append(pow(5, (g * b1 * h) % n, 2 * N))
+                else:
+                    acc = inner
+            if rin:                                            # giant steps: one shared ModDown
+                r = self.rot_sum(rin, rg, lv)
+                acc = r if acc is None else self.add(acc, r, lv)
             ct = self.rescale(acc, lv)
             lv -= 1
         return ct, lv

@@ -169,6 +169,7 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
     if (op == NEO_OP_HMULT_RESCALE) o += B * 3 * Lq * N + 4 * B * N;   // d, then c_l scratch
     if (op == NEO_OP_HROT) o += B * Lq * N;                       // sigma_g(c0)
     if (op == NEO_OP_HROT_HOISTED) o += B * 2 * Lq * N;
+    if (op == NEO_OP_HROT_SUM) o += B * 2 * Lq * N;                // sum of sigma_g(c0), one sigma_g(c0)
     L.total = o;
     return L;
 }
@@ -270,7 +271,10 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
 static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
                             u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
                             const u64* add0, const u64* add1, long long add_bs, cudaStream_t st,
-                            unsigned galois = 0, bool add_galois = true, u64* hmr_last = nullptr) {
+                            unsigned galois = 0, bool add_galois = true, u64* hmr_last = nullptr,
+                            int phase = 0) {
+    // phase 0: KeyIP then ModDown; 1: KeyIP only (acc overwritten); 2: KeyIP only, accumulated
+    // into acc; 3: ModDown only (of the acc already in the workspace) -- neo_hrot_sum
     // hmr_last != nullptr: fused HMULT + Rescale (neo_hmult_rescale).  add0/add1 are then d0/d1
     // (stride add_bs), out0/out1 receive the rescaled ciphertext at level l - 1, and hmr_last
     // is scratch [2][2B][N] for the coefficient form of acc_c and d_c at limb l.
@@ -280,7 +284,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     neo_status s;
 
     // a6: KeyIP over all E limbs of PQ_l
-    {
+    if (phase != 3) {
         KeyIPArgs A;
         A.d = d; A.up = up; A.evk_lo = k->lo; A.evk_hi = k->hi; A.acc = acc; A.mods = c->d_mods;
         A.d_bstride = d_bs;
@@ -289,6 +293,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         A.acc_cstride = (long long)E * N;
         A.N = N; A.beta = beta; A.evk_limbs = c->num_q + c->num_p;
         A.galois = galois;                     // d's own digit limbs are read as sigma_g(d)
+        A.accumulate = phase == 2;
         for (int pos = 0; pos < E; ++pos) {
             int id = c->ext_id(l, pos);
             A.limb[pos] = id;
@@ -301,6 +306,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         }
         LAUNCH(PK_KEYIP, st, launch_keyip(A, E, B, st));
     }
+    if (phase == 1 || phase == 2) return NEO_OK;
 
     // a7: INTT of the P part of acc_0, acc_1 -> pc [2B][P][N], with ModDown's [a_k Phat_k^-1] folded in
     for (int k2 = 0; k2 < P; ++k2) { so[k2] = Lq + k2; dof[k2] = k2; pr[k2] = c->num_q + k2; }
@@ -796,10 +802,11 @@ size_t neo_workspace_size(const neo_ctx* c, int32_t op, int32_t level, int32_t b
         case NEO_OP_HMULT:
         case NEO_OP_HROT:
         case NEO_OP_HROT_HOISTED:
+        case NEO_OP_HROT_SUM:
         case NEO_OP_HMULT_RESCALE: {
             if (op == NEO_OP_HMULT_RESCALE && level < 1) return 0;
             size_t w = ks_layout(c, level, batch, op).total;
-            if (c->num_t && op != NEO_OP_HROT_HOISTED && op != NEO_OP_HMULT_RESCALE) w = std::max(w, klss_total(c, level, batch, op));
+            if (c->num_t && op != NEO_OP_HROT_HOISTED && op != NEO_OP_HMULT_RESCALE && op != NEO_OP_HROT_SUM) w = std::max(w, klss_total(c, level, batch, op));
             return w * sizeof(u64);
         }
         case NEO_OP_RESCALE: return level >= 1 ? rescale_ws(c, level, batch) * sizeof(u64) : 0;
@@ -1150,6 +1157,50 @@ neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint6
     LAUNCH(PK_AUTO, s, launch_automorph(ct_in, sc0, g, c->N, level + 1, s, batch, 2 * ls, ls));
     return ks_core(c, rk, ct_in + ls, 2 * ls, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, sc0, nullptr,
                    ls, s, g, /*add_galois=*/false);
+}
+
+neo_status neo_hrot_sum(const neo_ctx* c, const neo_evk* const* keys, const uint32_t* galois, int32_t n,
+                        const uint64_t* const* cts, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
+                        size_t ws_bytes, neo_stream_t st) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    TRY(check_level(c, level, batch));
+    TRY(check_ptr(ct_out, "ct_out"));
+    if (!keys || !galois || !cts || n < 1 || n > 64) FAIL(NEO_EINVAL, "need 1 <= n <= 64 keys, Galois elements, ciphertexts");
+    for (int k = 0; k < n; ++k) {
+        if (!keys[k] || keys[k]->ctx != c || keys[k]->klss || keys[k]->galois)
+            FAIL(NEO_EINVAL, "keys must be Hybrid rotation keys from neo_evk_create on this context");
+        if ((galois[k] & 1) == 0 || galois[k] >= 2u * (unsigned)c->N) FAIL(NEO_EINVAL, "galois element must be odd and < 2N");
+        TRY(check_ptr(cts[k], "cts[k]"));
+        if (cts[k] == ct_out) FAIL(NEO_EINVAL, "ct_out must not alias an input");
+    }
+    TRY(check_ws(c, NEO_OP_HROT_SUM, level, batch, ws, ws_bytes));
+    KsLayout Ly = ks_layout(c, level, batch, NEO_OP_HROT_SUM);
+    u64* w = static_cast<u64*>(ws);
+    const long long ls = (long long)(level + 1) * c->N;
+    u64* c0sum = w + Ly.extra;                                 // [B][l+1][N]: sum_k sigma_g(c0_k)
+    u64* c0k = c0sum + (size_t)batch * ls;                     // [B][l+1][N]: sigma_g(c0_k)
+    cudaStream_t s = S(st);
+    int launches = 0;
+    for (int k = 0; k < n; ++k) {
+        // KeyIP(ModUp(sigma_g(c1_k))) accumulated in PQ_l; sigma_g(c1) read through the index map
+        TRY(ks_modup(c, cts[k] + ls, 2 * ls, level, batch, w, Ly, s, galois[k]));
+        launches += g_launches;
+        TRY(ks_finish(c, keys[k], cts[k] + ls, 2 * ls, level, batch, w, Ly, nullptr, nullptr, 0, nullptr, nullptr,
+                      0, s, galois[k], false, nullptr, k == 0 ? 1 : 2));
+        launches += g_launches;
+        g_launches = 0;
+        LAUNCH(PK_AUTO, s, launch_automorph(cts[k], k == 0 ? c0sum : c0k, galois[k], c->N, level + 1, s, batch,
+                                           2 * ls, ls));
+        if (k > 0) LAUNCH(PK_EW, s, launch_add_rows(c0sum, c0k, c0sum, c->d_mods, level + 1, c->N, batch, s));
+        launches += g_launches;
+        g_launches = 0;
+    }
+    // one ModDown of the summed acc, with the summed sigma_g(c0) added to component 0
+    TRY(ks_finish(c, keys[0], nullptr, 0, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, c0sum, nullptr, ls, s,
+                  0, false, nullptr, 3));
+    g_launches += launches;
+    return NEO_OK;
 }
 
 neo_status neo_hrot_hoisted(const neo_ctx* c, const neo_evk* const* keys, int32_t n_rot, const uint64_t* ct_in,

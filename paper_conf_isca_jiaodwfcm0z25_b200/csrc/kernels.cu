@@ -85,8 +85,13 @@ __device__ __forceinline__ void keyip_body(const KeyIPArgs& A, int n, int t, int
             mac128(h1, l1, x[j], e1[j]);
         }
         u64* o = acc + b * A.acc_bstride;
-        o[0] = barrett_reduce(h0, l0, m);
-        o[(size_t)A.acc_cstride] = barrett_reduce(h1, l1, m);
+        u64 r0 = barrett_reduce(h0, l0, m), r1 = barrett_reduce(h1, l1, m);
+        if (A.accumulate) {
+            r0 = add_mod(r0, o[0], m.q);
+            r1 = add_mod(r1, o[(size_t)A.acc_cstride], m.q);
+        }
+        o[0] = r0;
+        o[(size_t)A.acc_cstride] = r1;
     }
 }
 
@@ -217,6 +222,19 @@ k_ew(const __grid_constant__ EwArgs A) {
     }
     *reinterpret_cast<ulonglong2*>(A.out + ct) = y0;
     *reinterpret_cast<ulonglong2*>(A.out + ct + cs) = y1;
+}
+
+__global__ void __launch_bounds__(256)
+k_add_rows(const u64* __restrict__ a, const u64* __restrict__ b, u64* out, const ModQ* __restrict__ mods, int limbs,
+           int N) {
+    pdl_wait();
+    const int n = 2 * (blockIdx.x * blockDim.x + threadIdx.x);
+    const int i = blockIdx.y;
+    if (n >= N) return;
+    const u64 q = mods[i].q;
+    const size_t o = ((size_t)blockIdx.z * limbs + i) * N + n;
+    const ulonglong2 x = *reinterpret_cast<const ulonglong2*>(a + o), y = *reinterpret_cast<const ulonglong2*>(b + o);
+    *reinterpret_cast<ulonglong2*>(out + o) = make_ulonglong2(add_mod(x.x, y.x, q), add_mod(x.y, y.y, q));
 }
 
 // ------------------------------------------------------------------ plaintext inner product
@@ -465,6 +483,10 @@ cudaError_t launch_wire(bool pack, const void* in, void* out, size_t n, cudaStre
 }
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_ew, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);
+}
+cudaError_t launch_add_rows(const u64* a, const u64* b, u64* out, const ModQ* mods, int limbs, int N, int batch,
+                            cudaStream_t st) {
+    return launch_k(k_add_rows, dim3((N / 2 + 255) / 256, limbs, batch), dim3(256), 0, st, a, b, out, mods, limbs, N);
 }
 cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st) {
     return launch_k(k_pmult_acc, dim3((A.N / 2 + 255) / 256, A.limbs, batch), dim3(256), 0, st, A);

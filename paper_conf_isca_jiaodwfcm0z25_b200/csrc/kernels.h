@@ -17,6 +17,7 @@ struct KeyIPArgs {
     long long d_bstride, up_bstride, acc_bstride, acc_cstride;
     int N, beta, evk_limbs;
     unsigned galois;                         // != 0: rows of kind 0 (d) are read as sigma_g(d)
+    int accumulate = 0;                      // != 0: acc += (sum over the giant steps, neo_hrot_sum)
     int limb[KS_MAX_EXT];                    // position -> limb id
     unsigned char src_kind[KS_MAX_BETA][KS_MAX_EXT];   // 0: d, 1: up
     int src_off[KS_MAX_BETA][KS_MAX_EXT];    // row (in N units) inside the chosen buffer
@@ -105,6 +106,9 @@ struct DsArgs {
 };
 
 cudaError_t launch_ew(const EwArgs& A, int batch, cudaStream_t st);
+// out = a + b mod q_i for polynomials [batch][limbs][N] (one component; out may alias a)
+cudaError_t launch_add_rows(const u64* a, const u64* b, u64* out, const ModQ* mods, int limbs, int N, int batch,
+                            cudaStream_t st);
 cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_hmr_fold(const HmrFoldArgs& A, int bc, cudaStream_t st);
 cudaError_t launch_ew_limbs(const EwlArgs& A, int batch, cudaStream_t st);

@@ -17,7 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libneo.so")
 
 NEO_OP_KEYSWITCH, NEO_OP_HMULT, NEO_OP_HROT, NEO_OP_RESCALE, NEO_OP_HROT_HOISTED = 0, 1, 2, 3, 4
-NEO_OP_DOUBLE_RESCALE, NEO_OP_MODRAISE, NEO_OP_HMULT_RESCALE = 5, 6, 7
+NEO_OP_DOUBLE_RESCALE, NEO_OP_MODRAISE, NEO_OP_HMULT_RESCALE, NEO_OP_HROT_SUM = 5, 6, 7, 8
 _STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM", 4: "NEO_ECUDA",
            5: "NEO_ENCCL", 6: "NEO_ENOPRIME"}
 
@@ -28,7 +28,7 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
             "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline", "neo_hsub", "neo_modraise",
-            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale", "neo_ew_limbs")
+            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale", "neo_ew_limbs", "neo_hrot_sum")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -72,6 +72,8 @@ def lib() -> ctypes.CDLL:
             "neo_evk_destroy": [_vp],
             "neo_keyswitch": [_vp, _vp, _vp, _i32, _vp, _vp, _i32, _vp, _sz, _vp],
             "neo_hmult": [_vp, _vp, _vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
+            "neo_hrot_sum": [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_u32), _i32, ctypes.POINTER(_vp), _i32, _vp,
+                             _i32, _vp, _sz, _vp],
             "neo_ew_limbs": [_vp, _i32, _vp, _vp, _i32p, _i32, _u64p, _i32, _vp, _i32, _vp],
             "neo_hmult_rescale": [_vp, _vp, _vp, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
             "neo_hrot": [_vp, _vp, _u32, _vp, _i32, _vp, _i32, _vp, _sz, _vp],
@@ -392,6 +394,18 @@ def neo_pmult_acc(ctx: Context, cts, pts, level: int, ct_out, batch: int, pt_sha
     pa = (ctypes.c_void_p * len(pts))(*[_ptr(t).value for t in pts])
     _check(lib().neo_pmult_acc(ctx.handle, ca, pa, len(cts), int(pt_shared), level, _ptr(ct_out), batch,
                                _stream(stream)), "neo_pmult_acc")
+
+
+def neo_hrot_sum(ctx: Context, keys, galois, cts, level: int, ct_out, batch: int, ws, stream=None):
+    """sum_k HROTATE(cts[k], galois[k]) with one ModDown (include/neo.h)."""
+    n = len(keys)
+    if not (len(galois) == len(cts) == n):
+        raise NeoError(1, "neo_hrot_sum", "keys, galois and cts differ in length")
+    ka = (ctypes.c_void_p * n)(*[k.handle.value for k in keys])
+    ga = (ctypes.c_uint32 * n)(*[int(g) for g in galois])
+    ca = (ctypes.c_void_p * n)(*[_ptr(t).value for t in cts])
+    _check(lib().neo_hrot_sum(ctx.handle, ka, ga, n, ca, level, _ptr(ct_out), batch, _ptr(ws), ws.numel() * 8,
+                              _stream(stream)), "neo_hrot_sum")
 
 
 def neo_hrot_hoisted(ctx: Context, keys, ct_in, level: int, ct_out, batch: int, ws, stream=None):

@@ -86,6 +86,12 @@ def limb_sharded_keyswitch(ops, plan: ShardPlan, d_local, evk):
 
     Returns (k0, k1) restricted to this rank's Q limbs, each [B][len(my_q)][N].
     """
+    return limb_sharded_moddown(ops, plan, limb_sharded_keyip(ops, plan, d_local, evk))
+
+
+def limb_sharded_keyip(ops, plan: ShardPlan, d_local, evk):
+    """Steps a3-a6 (INTT, exchange #1, ModUp, NTT, KeyIP): the rank's rows of the KeyIP output
+    acc [B][2][len(plan.mine)][N] (PQ_l, NTT form)."""
     P = plan
     # a3: INTT of the rank's Q limbs, then exchange #1: every rank gets all Q limbs
     y_local = ops.intt(d_local, P.my_q)
@@ -105,7 +111,12 @@ def limb_sharded_keyswitch(ops, plan: ShardPlan, d_local, evk):
         idx = [P.my_q.index(t) if t in dj else n_d + targets.index(t) for t in P.mine]
         both = ops.cat([d_local, up], axis=1) if up is not None else d_local
         dhat_rows.append(ops.take(both, idx))
-    acc = ops.keyip(ops.stack(dhat_rows, axis=1), P.mine, P.beta, evk)       # a6 -> [B][2][n_mine][N]
+    return ops.keyip(ops.stack(dhat_rows, axis=1), P.mine, P.beta, evk)     # a6 -> [B][2][n_mine][N]
+
+
+def limb_sharded_moddown(ops, plan: ShardPlan, acc):
+    """Steps a7-a10 (INTT of P, exchange #2, ModDown BConv, NTT, combine) of a KeyIP output."""
+    P = plan
     # a7: INTT of the rank's P limbs of acc, exchange #2: every rank gets all P limbs
     p_pos = [P.mine.index(t) for t in P.my_p]
     acc_p_local = ops.intt2(ops.take2(acc, p_pos), P.my_p) if p_pos else ops.empty2(acc, 0)

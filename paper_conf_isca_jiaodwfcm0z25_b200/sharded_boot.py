@@ -21,7 +21,7 @@ import torch
 
 from . import neo
 from .boot import Bootstrapper
-from .sharded import NeoOps, ShardPlan, limb_sharded_keyswitch
+from .sharded import NeoOps, ShardPlan, limb_sharded_keyip, limb_sharded_keyswitch, limb_sharded_moddown
 
 
 class ShardedBootstrapper(Bootstrapper):
@@ -145,6 +145,19 @@ class ShardedBootstrapper(Bootstrapper):
             k0, k1 = self._ks(ct[:, 1].contiguous(), lv, self.keys[("h", g)])
             out.append(self.ops.automorphism(self._plus_k(ct[:, 0].contiguous(), k0, k1, lv), g))
         return out
+
+    def rot_sum(self, cts, gs, lv):
+        """sum_k HROTATE(cts[k], gs[k]) with one ModDown (BOOT-G): KeyIP outputs summed on the
+        rank's PQ_l rows, one sharded ModDown, plus the summed sigma_g(c0)."""
+        plan = ShardPlan(lv, self.ctx.num_q, self.ctx.num_p, self.ctx.alpha, self.world, self.rank, strided=True)
+        acc = sig = None
+        for ct, g in zip(cts, gs):
+            sg = self.ops.automorphism(ct, g)
+            a = limb_sharded_keyip(self.ops, plan, sg[:, 1].contiguous(), self.keys[g])
+            acc = a if acc is None else self.ops.ew(neo.NEO_EWL_HADD, acc, a, plan.mine)
+            sig = sg if sig is None else self.add(sig, sg, lv)
+        k0, k1 = limb_sharded_moddown(self.ops, plan, acc)
+        return self._plus_k(sig[:, 0].contiguous(), k0, k1, lv)
 
     def pmul_sum(self, cts, names, lv):
         acc = self.pmul(cts[0], names[0], lv)

@@ -314,3 +314,22 @@ def test_batch_larger_than_chunk(op):
     got = host(out)
     for bb in range(batch):
         assert np.array_equal(got[bb], want[bb]), bb
+
+
+@pytest.mark.parametrize("name,level,n", [("tiny", 2, 1), ("tiny3", 2, 3), ("setb", 35, 3), ("setb", 20, 2)])
+def test_hrot_sum(name, level, n):
+    """neo_hrot_sum (rotations summed with one ModDown) equals the oracle's hrot_sum bit for bit;
+    with one term it is HROTATE itself."""
+    from oracle import boot as oboot
+    ctx, prm = ctx_of(name)
+    gs = [pow(5, r, 2 * prm.N) for r in (1, 4, 9)[:n]]
+    evks = [rand_evk(prm, 1400 + 10 * k) for k in range(n)]
+    keys = [neo.EvalKey(ctx, dev(e)) for e in evks]
+    cts = [rand_ct(prm, level, 1450 + 4 * k) for k in range(n)]
+    out = torch.empty((1, 2, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+    ws = ctx.workspace(neo.NEO_OP_HROT_SUM, level, 1)
+    neo.neo_hrot_sum(ctx, keys, gs, [dev(c[None]) for c in cts], level, out, 1, ws)
+    got = host(out)[0]
+    assert np.array_equal(got, oboot.hrot_sum(prm, cts, gs, level, evks))
+    if n == 1:
+        assert np.array_equal(got, ckks.hrot(prm, cts[0], gs[0], level, evks[0]))

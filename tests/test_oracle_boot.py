@@ -175,3 +175,21 @@ def test_full_slot_bootstrap_decodes_to_input(booted_full):
     assert lv == bp.top - bp.levels_used()
     got = boot.decode_sparse(bp, out, lv, scale * delta / bp.prm.q[0], s)
     assert np.max(np.abs(got - z)) < 1e-2
+
+
+def test_hrot_sum_pins():
+    """hrot_sum of one ciphertext is HROTATE itself (moddown = the key-switch's a7-a10), and a
+    sum of several decrypts to the sum of the slot rotations (BOOT-G)."""
+    prm = ckks.Params(12, 4, 2, 2)
+    s = ckks.secret(prm, 61, 32)
+    L = prm.max_level
+    gs = [pow(5, r, 2 * prm.N) for r in (1, 3, 7)]
+    keys = [ckks.rot_key(prm, s, g, 620 + i) for i, g in enumerate(gs)]
+    zs = [synth.complex_slots(630 + i, prm.N // 2) for i in range(3)]
+    delta = 2.0 ** 40
+    cts = [ckks.encrypt(prm, ckks.encode(prm.N, z, delta), s, L, 640 + i) for i, z in enumerate(zs)]
+    assert np.array_equal(boot.hrot_sum(prm, cts[:1], gs[:1], L, keys[:1]), ckks.hrot(prm, cts[0], gs[0], L, keys[0]))
+    out = boot.hrot_sum(prm, cts, gs, L, keys)
+    m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, out, s, L), list(range(L + 1)))
+    want = sum(np.roll(z, -r) for z, r in zip(zs, (1, 3, 7)))
+    assert np.max(np.abs(ckks.decode(prm.N, m, delta) - want)) < 1e-6
