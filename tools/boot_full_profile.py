@@ -8,7 +8,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_isca_jiaodwfcm0z25_b200 import neo, boot as gboot  # noqa: E402
 
 N, NQ, NP, DNUM, L = 1 << 16, 36, 12, 3, 35
-nb, rb, fl = N // 2, 12, int(os.environ.get("FL", "3"))
+nb, rb, fl = N // 2, int(os.environ.get("R", "12")), int(os.environ.get("FL", "4"))
 ctx = neo.Context(16, NQ, NP, DNUM)
 rnd = lambda *s: torch.randint(0, 1 << 35, s, dtype=torch.int64, device="cuda").view(torch.uint64)
 evk = rnd(DNUM, 2, NQ + NP, N)
