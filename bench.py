@@ -692,9 +692,14 @@ def run_neo(args):
                 sbt = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, fft_levels=fl)
                 sct0 = sbt.shard(bct, 0)
                 sref = sbt.run(sct0)[0].clone()
-                s_side = torch.cuda.Stream()
-                sbt_g = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, stream=s_side, fft_levels=fl)
-                sgraph, sg_out = graph_capture(lambda: sbt_g.run(sct0)[0], side=s_side)
+                # graph capture only on one rank: a capture that failed on some ranks mid-way
+                # through NCCL collectives could desynchronise them; with N > 1 the exchanges
+                # are timed eagerly (host-issued)
+                sgraph = sg_out = sbt_g = None
+                if world == 1:
+                    s_side = torch.cuda.Stream()
+                    sbt_g = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, stream=s_side, fft_levels=fl)
+                    sgraph, sg_out = graph_capture(lambda: sbt_g.run(sct0)[0], side=s_side)
                 if sgraph is not None:
                     sgraph.replay()
                     torch.cuda.synchronize()
