@@ -52,6 +52,7 @@ def parse():
                     help="skip the KLSS vs Hybrid key-switch comparison at Set-C (SURVEY §8(f) row 1)")
     ap.add_argument("--fused-rescale", type=int, default=1, choices=[0, 1],
                     help="1: the step's HMULT -> Rescale is one neo_hmult_rescale call (bit-identical)")
+    ap.add_argument("--no-latency", action="store_true", help="skip the per-operation latency distributions")
     ap.add_argument("--no-apps", action="store_true",
                     help="skip the application traces (HELR iteration, ResNet-20 layer; SURVEY §8(f) row 4)")
     ap.add_argument("--no-boot", action="store_true",
@@ -513,6 +514,49 @@ def run_neo(args):
                      "frac_hbm": round(bm[k] / (step_ms[k] / 1e3) / 1e9 / peak, 4) if step_ms[k] > 0 else None}
                  for k in step_ms}
 
+    # per-operation latency at Set-B (l = 35, B = 1) -- median / p10 / p90
+    # of 100 single calls, each bracketed by CUDA events on the calling stream after 10 warm-ups;
+    # "warm": the same inputs back to back; "flushed": a 256 MB buffer (> the 126 MB L2) is
+    # overwritten before every call.  Context: the paper's Table 6 (A100, Set-C): HMult 3472.5 us,
+    # HRotate 3422.1 us, Rescale 114.3 us, PMult 81.7 us, HAdd 46.1 us.
+    latency = None
+    if not args.no_latency:
+        a_, b_, c_ = dev_in[0]
+        o1, o2, o3 = new_outs()
+        flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+        d_ks = a_[:, 1].contiguous()
+        k0_, k1_ = torch.empty_like(d_ks), torch.empty_like(d_ks)
+        ops_ = {
+            "keyswitch": lambda: neo.neo_keyswitch(ctx, relin, d_ks, LEVEL, k0_, k1_, B, ws),
+            "hmult": lambda: neo.neo_hmult(ctx, relin, a_, b_, LEVEL, o1, B, ws),
+            "hmult_rescale": lambda: neo.neo_hmult_rescale(ctx, relin, a_, b_, LEVEL, o2, B, ws),
+            "hrot": lambda: neo.neo_hrot(ctx, rot, g, c_, LEVEL, o3, B, ws),
+            "rescale": lambda: neo.neo_rescale(ctx, o1, LEVEL, o2, B, ws),
+        }
+        latency = {"config": "Set-B l=35, B=1, one call per sample", "unit": "us",
+                   "paper_context_table6_a100_setc_us": {"hmult": 3472.5, "hrot": 3422.1, "rescale": 114.3}}
+        for name, fn in ops_.items():
+            res = {}
+            for mode in ("warm", "flushed"):
+                for _ in range(10):
+                    fn()
+                torch.cuda.synchronize()
+                samples = []
+                for _ in range(100):
+                    if mode == "flushed":
+                        flush.fill_(1)
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record()
+                    fn()
+                    e1.record()
+                    e1.synchronize()
+                    samples.append(e0.elapsed_time(e1) * 1e3)
+                samples.sort()
+                res[mode] = {"median": round(samples[50], 1), "p10": round(samples[10], 1),
+                             "p90": round(samples[90], 1)}
+            latency[name] = res
+        del flush
+
     # secondary: hoisted rotations (one ModUp shared by n_rot rotations of the same ciphertext)
     hoisted = None
     if not args.no_hoisted:
@@ -930,7 +974,7 @@ def run_neo(args):
                                   "peak": peak, "unit": "GB/s",
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
-                "cpu_baseline": cpu, "e2e": e2e, "e2e_u64": e2e_u64, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted,
+                "cpu_baseline": cpu, "e2e": e2e, "e2e_u64": e2e_u64, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted, "latency": latency,
                 "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block, "apps": apps_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}
