@@ -557,6 +557,34 @@ def run_neo(args):
             latency[name] = res
         del flush
 
+    # one Set-B key-switch (l = 35, B = 1) limb-sharded over all
+    # ranks (round-robin limbs; two all-gathers, NCCL when N > 1), eager; at N = 1 the same code
+    # path on one rank.  Latency = the slowest rank's CUDA-event time per key-switch.
+    sharded_ks = None
+    if not args.no_latency:
+        from paper_conf_isca_jiaodwfcm0z25_b200.sharded import NeoOps, ShardPlan, limb_sharded_keyswitch
+        plan = ShardPlan(LEVEL, NUM_Q, NUM_P, ctx.alpha, world, rank, strided=True)
+        sops = NeoOps(ctx)
+        d_loc = dev_in[0][0][:, 1].contiguous().view(torch.int64)[:, plan.my_q].contiguous().view(torch.uint64)
+        for _ in range(3):
+            limb_sharded_keyswitch(sops, plan, d_loc, relin)
+        torch.cuda.synchronize()
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(20):
+            limb_sharded_keyswitch(sops, plan, d_loc, relin)
+        e1.record()
+        torch.cuda.synchronize()
+        sks = e0.elapsed_time(e1) / 20
+        if world > 1:
+            t = torch.tensor([sks], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            sks = float(t.item())
+        sharded_ks = {"ranks": world, "ms_per_keyswitch": round(sks, 4), "unit": "ms",
+                      "limbs_per_rank": len(plan.mine),
+                      "note": "eager Python orchestration over C-ABI building blocks (host-issued launches)"}
+
     # secondary: hoisted rotations (one ModUp shared by n_rot rotations of the same ciphertext)
     hoisted = None
     if not args.no_hoisted:
@@ -975,6 +1003,7 @@ def run_neo(args):
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
                 "cpu_baseline": cpu, "e2e": e2e, "e2e_u64": e2e_u64, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted, "latency": latency,
+                "limb_sharded_keyswitch": sharded_ks,
                 "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block, "apps": apps_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}
