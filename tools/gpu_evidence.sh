@@ -5,7 +5,7 @@ timeout 300 python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 |
 timeout 1200 python bench.py > gpurun_out/bench_full.json 2> gpurun_out/bench_full.err; tail -3 gpurun_out/bench_full.err
 cat gpurun_out/bench_full.json
 # launch list / full captures of the headline step only (the secondary blocks are skipped)
-NCUARGS="--steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-hoisted --no-klss --no-boot --no-apps --batch-hrot 0 --graph 0 --streams 1"
+NCUARGS="--steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-hoisted --no-klss --no-boot --no-apps --no-latency --batch-hrot 0 --graph 0 --streams 1"
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
     python bench.py $NCUARGS > /dev/null 2>&1
 wc -l gpurun_out/launches.csv
