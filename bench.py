@@ -360,6 +360,15 @@ def run_neo(args):
         if world > 1:
             dist.barrier()
 
+    def agree(ok: bool) -> bool:
+        """True on every rank iff true on all ranks (keeps the ranks' collectives in step when
+        something optional -- a graph capture -- succeeded on some ranks only)."""
+        if world == 1:
+            return ok
+        t = torch.tensor([1.0 if ok else 0.0], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MIN)
+        return bool(t.item() > 0.5)
+
     B = args.batch
     ctx = neo.Context(LOG_N, NUM_Q, NUM_P, DNUM, device=local)
     N, Lq = ctx.N, LEVEL + 1
@@ -747,6 +756,8 @@ def run_neo(args):
             ref_out = bt.run(bct)[0].clone()
             bgraph, bg_out = graph_capture(lambda: bt.run(bct)[0])
             gms = None
+            if not agree(bgraph is not None):
+                bgraph = None
             if bgraph is not None:
                 bgraph.replay()
                 torch.cuda.synchronize()
@@ -834,6 +845,8 @@ def run_neo(args):
                 gr.replay()
                 torch.cuda.synchronize()
                 assert _same(gout, ref), "graph replay of the trace differs from the eager run"
+            if not agree(gr is not None):
+                gr = None
             for i, run in enumerate([fn, gr.replay if gr is not None else None]):
                 if run is None:
                     continue
