@@ -352,9 +352,17 @@ def run_neo(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # NEO_BENCH_BACKEND=gloo runs several ranks on one GPU (a functional check of the N > 1
+    # paths on a 1-GPU box; not a measurement).  The driver's runs use NCCL, one GPU per rank.
+    backend = os.environ.get("NEO_BENCH_BACKEND", "nccl")
+    if backend != "nccl":
+        local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
 
     def barrier():
         if world > 1:
