@@ -333,3 +333,34 @@ def test_hrot_sum(name, level, n):
     assert np.array_equal(got, oboot.hrot_sum(prm, cts, gs, level, evks))
     if n == 1:
         assert np.array_equal(got, ckks.hrot(prm, cts[0], gs[0], level, evks[0]))
+
+
+def test_batch_chunks_setb_sampled():
+    """Set-B HROTATE over 33 ciphertexts (chunks of 32 + 1 on two streams, the configuration
+    bench.py's batch_hrot times): sampled ciphertexts from both chunks equal the oracle."""
+    ctx, prm = ctx_of("setb")
+    level, batch = 35, 33
+    evk_np = rand_evk(prm, 1500)
+    key = neo.EvalKey(ctx, dev(evk_np))
+    g = pow(5, 1, 2 * prm.N)
+    a = np.stack([rand_ct(prm, level, 1510 + 2 * b) for b in range(batch)])
+    out = torch.empty((batch, 2, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+    neo.neo_hrot(ctx, key, g, dev(a), level, out, batch, ctx.workspace(neo.NEO_OP_HROT, level, batch))
+    got = host(out)
+    for bb in (0, 31, 32):
+        assert np.array_equal(got[bb], ckks.hrot(prm, a[bb], g, level, evk_np)), bb
+
+
+def test_pmult_acc_setb():
+    """neo_pmult_acc at Set-B l = 35 (9 terms, the conv layer's inner sum) equals PMULT + HADD."""
+    ctx, prm = ctx_of("setb")
+    level, k = 35, 9
+    cts = [rand_ct(prm, level, 1600 + 2 * i) for i in range(k)]
+    pts = [rand_poly(prm, list(range(level + 1)), 1700 + i) for i in range(k)]
+    out = torch.empty((1, 2, level + 1, prm.N), dtype=torch.uint64, device="cuda")
+    neo.neo_pmult_acc(ctx, [dev(c[None]) for c in cts], [dev(p) for p in pts], level, out, 1, pt_shared=True)
+    want = None
+    for c, p in zip(cts, pts):
+        t = ckks.pmult(prm, c, p, level)
+        want = t if want is None else ckks.hadd(prm, want, t, level)
+    assert np.array_equal(host(out)[0], want)
