@@ -993,7 +993,35 @@ def run_neo(args):
         neo.neo_wire_unpack(ctx, host_wout[(k_e2e - 1) % 2].cuda()[off_out[1]:], chk)
         torch.cuda.synchronize()
         assert torch.equal(chk.view(torch.int64), outs[(k_e2e - 1) % 2][2].view(torch.int64)), "wire round trip"
+        # the PCIe ceiling of this e2e: raw pinned copies of 64 MB, both directions at once
+        # (tools/pcie_bw.py): the step's H2D bytes at the per-direction duplex rate
+        nb_ = 64 << 20
+        hb_i, hb_o = torch.empty(nb_, dtype=torch.uint8).pin_memory(), torch.empty(nb_, dtype=torch.uint8).pin_memory()
+        db_i, db_o = torch.empty(nb_, dtype=torch.uint8, device="cuda"), torch.empty(nb_, dtype=torch.uint8, device="cuda")
+
+        def duplex():
+            with torch.cuda.stream(h2d_st):
+                db_i.copy_(hb_i, non_blocking=True)
+            with torch.cuda.stream(d2h_st):
+                hb_o.copy_(db_o, non_blocking=True)
+            torch.cuda.current_stream().wait_stream(h2d_st)
+            torch.cuda.current_stream().wait_stream(d2h_st)
+        duplex()
+        torch.cuda.synchronize()
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        p0.record()
+        for _ in range(10):
+            duplex()
+        p1.record()
+        torch.cuda.synchronize()
+        per_dir = nb_ / (p0.elapsed_time(p1) / 10 / 1e3) / 1e9            # GB/s per direction
+        bound_ms = max(sum(wb_in), sum(wb_out)) / (per_dir * 1e9) * 1e3
+        del hb_i, hb_o, db_i, db_o
         e2e = {"value": 2 * B * world / (wms / k_e2e / 1e3), "unit": UNIT,
+               "pcie": {"duplex_GBps_per_direction": round(per_dir, 1), "bound_ms_per_step": round(bound_ms, 4),
+                        "frac_of_bound": round(bound_ms / (wms / k_e2e), 3),
+                        "note": "raw pinned 64 MB copies in both directions at once; the step's larger "
+                                "direction (H2D) at that rate is the e2e ceiling"},
                "h2d_bytes_per_step": sum(wb_in), "d2h_bytes_per_step": sum(wb_out),
                "steps": k_e2e, "ms_per_step": wms / k_e2e,
                "format": "36-bit wire format (neo_wire_pack/unpack, 4.5 bytes per residue), unpack/pack on the device inside the region",
