@@ -170,10 +170,12 @@ def test_hmult(name, level, batch):
         assert np.array_equal(got[bb], ckks.hmult(prm, a[bb], b_[bb], level, evk_np))
 
 
-@pytest.mark.parametrize("name,level,batch,r", [("tiny", 2, 2, 1), ("setb", 35, 1, 1), ("setb", 20, 1, 7)])
+@pytest.mark.parametrize("name,level,batch,r", [("tiny", 2, 2, 1), ("setb", 35, 1, 1), ("setb", 20, 1, 7),
+                                                ("tiny", 2, 1, 0), ("tiny", 1, 2, "conj"), ("setb", 35, 1, "conj")])
 def test_hrot(name, level, batch, r):
+    """r = 0 is the identity Galois element g = 1 (Z11's special case); "conj" is g = 2N - 1."""
     ctx, prm = ctx_of(name)
-    g = pow(5, r, 2 * prm.N)
+    g = 2 * prm.N - 1 if r == "conj" else pow(5, r, 2 * prm.N)
     evk_np = rand_evk(prm, 900)
     rk = neo.EvalKey(ctx, dev(evk_np))
     ct = np.stack([rand_ct(prm, level, 910 + 2 * b) for b in range(batch)])
