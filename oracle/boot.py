@@ -222,29 +222,21 @@ def _lintrans_bsgs(prm, ct, lv, diags: dict, name: str, keys: dict, const):
     b1, h, ms = _bsgs_shape(diags)
     babies = sorted({m % b1 for m in ms} - {0})
     gs = [pow(5, (b * h) % n, 2 * N) for b in babies]
-    ext_ids = list(range(lv + 1)) + prm.p_ids
-    exts = {}
-    if gs:                                       # double hoisting (BOOT-DH): baby steps kept in PQ_l
-        for b, x in zip(babies, hoisted_ext(prm, ct, gs, lv, [keys[g] for g in gs])):
-            exts[b] = x
+    rots = {0: ct}
+    if gs:
+        for b, r in zip(babies, ckks.hrot_hoisted(prm, ct, gs, lv, [keys[g] for g in gs])):
+            rots[b] = r
     acc, rot_in, rot_g = None, [], []
     for g in sorted({m // b1 for m in ms}):
-        inner, yext = None, None
+        inner = None
         for m in ms:
             if m // b1 != g:
                 continue
             b = m % b1
-            slots = _rot(diags[m * h], -g * b1 * h)
-            if b == 0:                           # the unrotated term stays in Q_l
-                pt = const(f"{name}_g{g}_b0", lambda slots=slots: _pt_full(prm, slots, float(prm.q[lv]), lv))
-                inner = ckks.pmult(prm, ct, pt, lv)
-            else:                                # rotated terms: PMULT in PQ_l, one ModDown per giant step
-                pt = const(f"{name}_g{g}_b{b}x", lambda slots=slots: _pt_ext(prm, slots, float(prm.q[lv]), ext_ids))
-                t = np.stack([ckks.mul(prm, exts[b][c], pt, ext_ids) for c in range(2)])
-                yext = t if yext is None else np.stack([ckks.add(prm, yext[c], t[c], ext_ids) for c in range(2)])
-        if yext is not None:                     # ModDown(P x + y) = x + ModDown(y): b = 0 added after
-            md = np.stack(moddown(prm, yext, lv))
-            inner = md if inner is None else ckks.hadd(prm, inner, md, lv)
+            pt = const(f"{name}_g{g}_b{b}", lambda m=m, g=g: _pt_full(prm, _rot(diags[m * h], -g * b1 * h),
+                                                                      float(prm.q[lv]), lv))
+            t = ckks.pmult(prm, rots[b], pt, lv)
+            inner = t if inner is None else ckks.hadd(prm, inner, t, lv)
         if g:
             rot_in.append(inner)
             rot_g.append(pow(5, (g * b1 * h) % n, 2 * N))
@@ -254,32 +246,6 @@ def _lintrans_bsgs(prm, ct, lv, diags: dict, name: str, keys: dict, const):
         r = hrot_sum(prm, rot_in, rot_g, lv, [keys[ga] for ga in rot_g])
         acc = r if acc is None else ckks.hadd(prm, acc, r, lv)
     return ckks.rescale(prm, acc, lv)
-
-
-def hoisted_ext(prm: ckks.Params, ct: np.ndarray, gs: list, level: int, rotkeys: list) -> list:
-    """Double-hoisted baby steps (reading BOOT-DH): for each g the rotation of ct kept in PQ_l,
-    before ModDown:  sigma_g( (P c0 + acc0, acc1) ),  acc = KeyIP(ModUp(c1)) under the key
-    sigma_g^-1(rotkey_g) (the hoisted rotation of ckks.hrot_hoisted, without its ModDown; P c0 is
-    0 on the P limbs).  Returns [n][2][E][N] (NTT form over q_0..q_l, p_0..p_K)."""
-    ids = list(range(level + 1))
-    ext = ids + prm.p_ids
-    pmod = [prm.P % prm.moduli[i] for i in ids]
-    c0p = np.concatenate([ckks.scalar_mul(prm, ct[0], pmod, ids),
-                          np.zeros((prm.num_p, prm.N), dtype=np.uint64)])
-    out = []
-    for g, key in zip(gs, rotkeys):
-        kp = ckks.automorphism_ntt(key, pow(g, -1, 2 * prm.N))
-        tr = {}
-        ckks.keyswitch(prm, ct[1], level, kp, trace=tr)
-        x = np.stack([ckks.add(prm, tr["acc"][0], c0p, ext), tr["acc"][1]])
-        out.append(ckks.automorphism_ntt(x, g))
-    return out
-
-
-def _pt_ext(prm: ckks.Params, slots: np.ndarray, scale: float, ext_ids: list) -> np.ndarray:
-    """A plaintext diagonal encoded over PQ_l (for the PQ-basis sums of double hoisting)."""
-    m = ckks.encode_fft(prm.N, np.asarray(slots, dtype=complex), scale)
-    return ckks.ntt(prm, ckks.reduce_signed(prm, m, ext_ids), ext_ids)
 
 
 def moddown(prm: ckks.Params, acc: np.ndarray, level: int) -> tuple:

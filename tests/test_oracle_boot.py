@@ -193,29 +193,3 @@ def test_hrot_sum_pins():
     m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, out, s, L), list(range(L + 1)))
     want = sum(np.roll(z, -r) for z, r in zip(zs, (1, 3, 7)))
     assert np.max(np.abs(ckks.decode(prm.N, m, delta) - want)) < 1e-6
-
-
-def test_hoisted_ext_pins():
-    """BOOT-DH: ModDown of a double-hoisted baby step decrypts to the slot rotation, and
-    ModDown(P x + y) = x + ModDown(y) exactly (the identity that keeps the unrotated term in Q)."""
-    prm = ckks.Params(12, 4, 2, 2)
-    s = ckks.secret(prm, 71, 32)
-    L = prm.max_level
-    gs = [pow(5, r, 2 * prm.N) for r in (1, 6)]
-    keys = [ckks.rot_key(prm, s, g, 720 + i) for i, g in enumerate(gs)]
-    z = synth.complex_slots(73, prm.N // 2)
-    delta = 2.0 ** 40
-    ct = ckks.encrypt(prm, ckks.encode(prm.N, z, delta), s, L, 74)
-    for x, r in zip(boot.hoisted_ext(prm, ct, gs, L, keys), (1, 6)):
-        md = np.stack(boot.moddown(prm, x, L))
-        m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, md, s, L), list(range(L + 1)))
-        assert np.max(np.abs(ckks.decode(prm.N, m, delta) - np.roll(z, -r))) < 1e-6
-    ids = list(range(L + 1))
-    ext = ids + prm.p_ids
-    y = np.stack([synth.uniform_residues(75 + c, [prm.moduli[i] for i in ext], prm.N) for c in range(2)])
-    pmod = [prm.P % prm.moduli[i] for i in ids]
-    lifted = np.stack([np.concatenate([ckks.add(prm, y[c][: L + 1], ckks.scalar_mul(prm, ct[c], pmod, ids), ids),
-                                       y[c][L + 1:]]) for c in range(2)])
-    a = np.stack(boot.moddown(prm, lifted, L))
-    b = ckks.hadd(prm, ct, np.stack(boot.moddown(prm, y, L)), L)
-    assert np.array_equal(a, b)
