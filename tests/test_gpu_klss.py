@@ -45,7 +45,8 @@ def test_klss_params_match_oracle(name):
     assert ctx.alpha_t == kp.alpha_t and ctx.alpha_p == kp.alpha_p and ctx.t == kp.t
 
 
-@pytest.mark.parametrize("name,level,batch", [("tiny", 5, 2), ("tiny", 3, 1), ("tiny", 0, 1), ("setc", 35, 1)])
+@pytest.mark.parametrize("name,level,batch", [("tiny", 5, 2), ("tiny", 3, 1), ("tiny", 0, 1), ("setc", 35, 1),
+                                              ("tiny", 5, 34)])     # 34: two chunks on two streams
 def test_klss_keyswitch(name, level, batch):
     kp, ctx, evk, ek, key = setup(name)
     b = kp.base
