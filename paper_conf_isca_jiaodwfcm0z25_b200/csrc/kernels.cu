@@ -150,14 +150,29 @@ k_tensor(const u64* __restrict__ cta, const u64* __restrict__ ctb, u64* __restri
 
 // ------------------------------------------------------------------ automorphism (AUTO)
 // out[i] = in[(g i + (g-1)/2) mod N]: X -> X^g in the natural-order NTT domain.
+#ifndef AUTO_ILP
+#define AUTO_ILP 4
+#endif
 __global__ void __launch_bounds__(256)
 k_automorph(const u64* __restrict__ in, u64* __restrict__ out, unsigned g, int N, long long in_bs, long long out_bs) {
     pdl_wait();
-    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    // AUTO_ILP gathers per thread, all issued before the stores (loads in flight per SM).
     const size_t row = (size_t)blockIdx.y * N;
-    if (i >= N) return;
-    const unsigned src = (unsigned)(((unsigned long long)g * i + (g - 1) / 2) & (N - 1));
-    out[blockIdx.z * out_bs + row + i] = in[blockIdx.z * in_bs + row + src];
+    const u64* src_row = in + blockIdx.z * in_bs + row;
+    u64* dst_row = out + blockIdx.z * out_bs + row;
+    const int i0 = blockIdx.x * blockDim.x * AUTO_ILP + threadIdx.x;
+    u64 v[AUTO_ILP];
+#pragma unroll
+    for (int k = 0; k < AUTO_ILP; ++k) {
+        const int i = i0 + k * blockDim.x;
+        const unsigned src = (unsigned)(((unsigned long long)g * i + (g - 1) / 2) & (N - 1));
+        if (i < N) v[k] = src_row[src];
+    }
+#pragma unroll
+    for (int k = 0; k < AUTO_ILP; ++k) {
+        const int i = i0 + k * blockDim.x;
+        if (i < N) dst_row[i] = v[k];
+    }
 }
 
 // ------------------------------------------------------------------ rescale helpers (L137)
@@ -544,7 +559,7 @@ cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, 
 }
 cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st, int batch,
                              long long in_bs, long long out_bs) {
-    return launch_k(k_automorph, dim3(g1(N).x, rows, batch), dim3(256), 0, st, in, out, g, N, in_bs, out_bs);
+    return launch_k(k_automorph, dim3((N + 256 * AUTO_ILP - 1) / (256 * AUTO_ILP), rows, batch), dim3(256), 0, st, in, out, g, N, in_bs, out_bs);
 }
 cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st) {
     return launch_k(k_modswitch, dim3(g1(N).x, l, bc), dim3(256), 0, st, last, r, mods, l, N);
