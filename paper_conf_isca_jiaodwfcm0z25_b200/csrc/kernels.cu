@@ -374,14 +374,21 @@ k_hmr_fold(const __grid_constant__ HmrFoldArgs A) {
                            __ldg(A.dl + (size_t)bc * row + n), ml.q);
     const double cld = u2d(cl);
     const int i1 = min(A.l, i0 + kFoldRows);
-    for (int i = i0; i < i1; ++i) {
+    u64* p = A.conv + base + (size_t)i0 * row;
+    u64 v[kFoldRows];                                // all rows' loads in flight before the stores
+#pragma unroll
+    for (int k = 0; k < kFoldRows; ++k)
+        if (i0 + k < i1) v[k] = p[(size_t)k * row];
+#pragma unroll
+    for (int k = 0; k < kFoldRows; ++k) {
+        const int i = i0 + k;
+        if (i >= i1) break;
         const ModQ m = A.mods[i];
-        u64* p = A.conv + base + (size_t)i * row;
         if (A.lazy) {
-            const double z = __dadd_rn(__longlong_as_double((long long)*p), mulc(cld, A.pmod[i], m.qd));
-            *p = (u64)__double_as_longlong(canon(z, m.qd, m.qinv));
+            const double z = __dadd_rn(__longlong_as_double((long long)v[k]), mulc(cld, A.pmod[i], m.qd));
+            p[(size_t)k * row] = (u64)__double_as_longlong(canon(z, m.qd, m.qinv));
         } else {
-            *p = add_mod(*p, d2u(canon(mulc(cld, A.pmod[i], m.qd), m.qd, m.qinv)), m.q);
+            p[(size_t)k * row] = add_mod(v[k], d2u(canon(mulc(cld, A.pmod[i], m.qd), m.qd, m.qinv)), m.q);
         }
     }
 }
