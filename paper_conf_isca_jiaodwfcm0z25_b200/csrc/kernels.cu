@@ -98,8 +98,11 @@ __device__ __forceinline__ void keyip_body(const KeyIPArgs& A, int n, int t, int
 // At beta = 3 (Set-B) the body fits 40 registers without spilling: 6 CTAs per SM instead of
 // 5 (48 registers) gives more loads in flight (KeyIP 0.112 -> 0.106 ms per step).  Larger
 // beta would spill at that bound and keeps the default.
+#ifndef KEYIP_NT
+#define KEYIP_NT 128
+#endif
 template <int BETA>
-__global__ void __launch_bounds__(256, BETA == 3 ? 6 : 1)
+__global__ void __launch_bounds__(KEYIP_NT, BETA == 3 ? 6 * 256 / KEYIP_NT : 1)
 k_keyip(const __grid_constant__ KeyIPArgs A, int batch) {
     pdl_wait();
     const int n = blockIdx.x * blockDim.x + threadIdx.x;
@@ -541,20 +544,20 @@ cudaError_t launch_bconv(const BConvTab& T, const BConvIO& io, int N, int batch,
     return launch_k(k_bconv, dim3((N + 255) / 256, batch), dim3(256), 0, st, T, io, N);
 }
 cudaError_t launch_keyip(const KeyIPArgs& A, int limbs, int batch, cudaStream_t st) {
-    const dim3 g((A.N + 255) / 256, limbs);
+    const dim3 g((A.N + KEYIP_NT - 1) / KEYIP_NT, limbs);
     switch (A.beta) {
-        case 1: return launch_k(k_keyip<1>, g, dim3(256), 0, st, A, batch);
-        case 2: return launch_k(k_keyip<2>, g, dim3(256), 0, st, A, batch);
-        case 3: return launch_k(k_keyip<3>, g, dim3(256), 0, st, A, batch);
-        case 4: return launch_k(k_keyip<4>, g, dim3(256), 0, st, A, batch);
-        case 5: return launch_k(k_keyip<5>, g, dim3(256), 0, st, A, batch);
-        case 6: return launch_k(k_keyip<6>, g, dim3(256), 0, st, A, batch);
-        case 7: return launch_k(k_keyip<7>, g, dim3(256), 0, st, A, batch);
-        case 8: return launch_k(k_keyip<8>, g, dim3(256), 0, st, A, batch);
-        case 9: return launch_k(k_keyip<9>, g, dim3(256), 0, st, A, batch);
-        case 10: return launch_k(k_keyip<10>, g, dim3(256), 0, st, A, batch);
-        case 11: return launch_k(k_keyip<11>, g, dim3(256), 0, st, A, batch);
-        default: return launch_k(k_keyip<12>, g, dim3(256), 0, st, A, batch);
+        case 1: return launch_k(k_keyip<1>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 2: return launch_k(k_keyip<2>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 3: return launch_k(k_keyip<3>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 4: return launch_k(k_keyip<4>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 5: return launch_k(k_keyip<5>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 6: return launch_k(k_keyip<6>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 7: return launch_k(k_keyip<7>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 8: return launch_k(k_keyip<8>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 9: return launch_k(k_keyip<9>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 10: return launch_k(k_keyip<10>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        case 11: return launch_k(k_keyip<11>, g, dim3(KEYIP_NT), 0, st, A, batch);
+        default: return launch_k(k_keyip<12>, g, dim3(KEYIP_NT), 0, st, A, batch);
     }
 }
 cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStream_t st) {
