@@ -101,6 +101,20 @@ neo_status neo_ntt(const neo_ctx* ctx, uint64_t* poly, const int32_t* limb_ids, 
 neo_status neo_intt(const neo_ctx* ctx, uint64_t* poly, const int32_t* limb_ids, int32_t n_limbs,
                     int32_t batch, void* ws, size_t ws_bytes, neo_stream_t stream);
 
+/* Select the NTT implementation every transform of this context uses (neo_ntt / neo_intt and
+ * every NTT inside the key-switching operations); the result is bit-identical either way.
+ *   NEO_NTT_TC   : both radix-16 DFT stages of each 256-point pass as tcgen05 kind::i8 GEMMs
+ *                  (Neo's matrix-multiplication NTT, L438-450 / Fig. 9, on the int8 tensor
+ *                  cores; N = 2^16 with 36-bit primes only) -- the default where supported
+ *                  (environment NEO_NTT=fp64 at context creation selects the other);
+ *   NEO_NTT_FP64 : radix-2 butterflies in FP64 on the CUDA cores (any supported N).
+ * Returns NEO_EUNSUPPORTED (selection unchanged) if NEO_NTT_TC is not available for this
+ * context.  Not thread-safe with respect to operations running on the same context. */
+enum { NEO_NTT_FP64 = 0, NEO_NTT_TC = 1 };
+neo_status neo_ntt_select(neo_ctx* ctx, int32_t impl);
+/* The implementation currently selected (NEO_NTT_*), or -1 for a NULL context. */
+int32_t neo_ntt_selected(const neo_ctx* ctx);
+
 /* Basis conversion, Algorithm 1 (L296-319), non-centred (Z7), coefficient form:
  *   out[t] = sum_i [in_i * qhat_i^-1]_{q_i} * (qhat_i mod t) mod t,
  *   qhat_i = prod_{i' != i} q_{i'} over the input limbs.

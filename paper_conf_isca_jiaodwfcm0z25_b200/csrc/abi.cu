@@ -14,6 +14,7 @@
 #include "kernels.h"
 #include "klss.h"
 #include "ntt.h"
+#include "ntt_tc.h"
 
 namespace neo {
 neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err);
@@ -144,8 +145,13 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
         b.src_off[k] = k; b.dst_off[k] = dst_off[k]; b.prime[k] = (short)prime[k];
     }
     // forward: column pass then row pass; inverse: row pass then column pass
-    LAUNCH(fwd ? PK_NTT_COL : PK_NTT_ROW, st, ntt_pass(fwd, a, c->ntt, batch, fwd, st));
-    LAUNCH(fwd ? PK_NTT_ROW : PK_NTT_COL, st, ntt_pass(!fwd, b, c->ntt, batch, fwd, st, epi));
+    if (c->ntt_impl == NEO_NTT_TC && c->ntt.tct) {     // both DFT stages of each pass on tcgen05
+        LAUNCH(fwd ? PK_NTT_COL : PK_NTT_ROW, st, ntt_pass_tc(fwd, a, c->ntt, batch, fwd, st));
+        LAUNCH(fwd ? PK_NTT_ROW : PK_NTT_COL, st, ntt_pass_tc(!fwd, b, c->ntt, batch, fwd, st, epi));
+    } else {                                           // FP64 butterflies on the CUDA cores
+        LAUNCH(fwd ? PK_NTT_COL : PK_NTT_ROW, st, ntt_pass(fwd, a, c->ntt, batch, fwd, st));
+        LAUNCH(fwd ? PK_NTT_ROW : PK_NTT_COL, st, ntt_pass(!fwd, b, c->ntt, batch, fwd, st, epi));
+    }
     return NEO_OK;
 }
 
@@ -777,12 +783,23 @@ neo_status neo_params_destroy(neo_ctx* c) {
     if (!c) return NEO_OK;
     if (c->side) cudaStreamDestroy(c->side);
     if (c->d_tab) cudaFree(c->d_tab);
+    if (c->d_ntt_tc) cudaFree(c->d_ntt_tc);
     if (c->d_mods) cudaFree(c->d_mods);
     if (c->d_bmat) cudaFree(c->d_bmat);
     if (c->d_rec) cudaFree(c->d_rec);
     delete c;
     return NEO_OK;
 }
+
+neo_status neo_ntt_select(neo_ctx* c, int32_t impl) {
+    if (!c) FAIL(NEO_EINVAL, "null context");
+    if (impl != NEO_NTT_FP64 && impl != NEO_NTT_TC) FAIL(NEO_EINVAL, "unknown NTT implementation");
+    if (impl == NEO_NTT_TC && !c->ntt.tct) FAIL(NEO_EUNSUPPORTED, "tensor-core NTT needs N = 2^16 and 36-bit primes");
+    c->ntt_impl = impl;
+    return NEO_OK;
+}
+
+int32_t neo_ntt_selected(const neo_ctx* c) { return c ? c->ntt_impl : -1; }
 
 neo_status neo_params_query(const neo_ctx* c, uint64_t* q, uint64_t* p, uint64_t* psi) {
     TRY(check_ctx(c));

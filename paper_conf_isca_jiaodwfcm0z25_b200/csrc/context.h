@@ -77,6 +77,8 @@ struct neo_ctx {
     std::vector<ModQ> h_mods;
     NttLayout L;
     TWD* d_tab = nullptr;                 // [limb id][L.total]
+    uint8_t* d_ntt_tc = nullptr;          // [limb id][NTC_PRIME_BYTES]: tensor-core NTT tables (N = 2^16), or null
+    int ntt_impl = 0;                     // NEO_NTT_FP64 (0) or NEO_NTT_TC (1); neo_ntt_select
     ModQ* d_mods = nullptr;
     neo::NttArgs ntt;
     // per level l (index l = 0..num_q-1)

@@ -104,17 +104,7 @@ NEO_DEV void cyc_dif(double (&a)[R], const TWD* tab, double q) {
 
 constexpr int kC = 16;   // columns per column-pass tile / rows per row-pass tile
 
-struct TileMap {        // rows (b, k) in limb-major order: consecutive tiles share a prime
-    int batch, tpr, total;
-    int tpr_log;            // tpr = 2^tpr_log
-    unsigned bmagic;        // floor(2^32 / batch) + 1 (batch > 1): exact for ri * batch < 2^32
-    NEO_DEV void decode(int t, int& b, int& k, int& blk) const {
-        const int ri = t >> tpr_log;
-        blk = t & (tpr - 1);
-        k = (batch == 1) ? ri : (int)__umulhi((unsigned)ri, bmagic);
-        b = ri - k * batch;
-    }
-};
+// TileMap: ntt.h
 
 // 16-byte chunk swizzle for [row][16 doubles] tiles read/written column-wise
 NEO_DEV int swz(int row, int col) { return row * 16 + ((((col >> 1) ^ (row & 7)) << 1) | (col & 1)); }

@@ -5,6 +5,19 @@
 
 namespace neo {
 
+// rows (b, k) in limb-major order: consecutive tiles share a prime
+struct TileMap {        // rows (b, k) in limb-major order: consecutive tiles share a prime
+    int batch, tpr, total;
+    int tpr_log;            // tpr = 2^tpr_log
+    unsigned bmagic;        // floor(2^32 / batch) + 1 (batch > 1): exact for ri * batch < 2^32
+    NEO_DEV void decode(int t, int& b, int& k, int& blk) const {
+        const int ri = t >> tpr_log;
+        blk = t & (tpr - 1);
+        k = (batch == 1) ? ri : (int)__umulhi((unsigned)ri, bmagic);
+        b = ri - k * batch;
+    }
+};
+
 struct NttArgs {
     const TWD* tabd;      // device: [limb id][L.total] twiddle blocks (w, w/q) in FP64
     long long tab_stride; // = L.total
@@ -12,6 +25,7 @@ struct NttArgs {
     int N, N1, N2;
     int num_sms;          // persistent grid = 2 CTAs per SM
     NttLayout L;
+    const uint8_t* tct = nullptr;   // device: tensor-core pass tables [limb id][NTC_PRIME_BYTES] (ntt_tc.h), or null
 };
 
 // Optional epilogue of the forward row pass for the ModDown NTT (a9 + a10 fused):

@@ -14,6 +14,7 @@
 
 #include "bconv_tc.h"
 #include "context.h"
+#include "ntt_tc.h"
 
 namespace neo {
 
@@ -312,6 +313,23 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
         c->num_sms = dev_sms > 0 ? dev_sms : 148;
     }
     c->ntt.num_sms = c->num_sms;
+    // tensor-core NTT tables (ntt_tc.cu): N = 2^16 and every prime in (2^35, 2^36)
+    {
+        std::vector<uint8_t> tct((size_t)ntot * NTC_PRIME_BYTES);
+        bool ok = c->N == 65536;
+        for (int i = 0; i < ntot && ok; ++i)
+            ok = make_ntt_tc_block(&tct[(size_t)i * NTC_PRIME_BYTES], c->mod[i], c->psi[i], c->N);
+        if (ok) {
+            if (cudaMalloc(&c->d_ntt_tc, tct.size()) != cudaSuccess) { err = "cudaMalloc of NTT tables failed"; return NEO_ENOMEM; }
+            if (cudaMemcpy(c->d_ntt_tc, tct.data(), tct.size(), cudaMemcpyHostToDevice) != cudaSuccess) {
+                err = "cudaMemcpy of NTT tables failed";
+                return NEO_ECUDA;
+            }
+            c->ntt.tct = c->d_ntt_tc;
+            const char* e = std::getenv("NEO_NTT");
+            c->ntt_impl = (e && std::string(e) == "fp64") ? NEO_NTT_FP64 : NEO_NTT_TC;
+        }
+    }
 
     // ---- BConv / ModDown / rescale constants per level
     std::vector<int> pids;

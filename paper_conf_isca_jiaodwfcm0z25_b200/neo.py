@@ -17,6 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libneo.so")
 
 NEO_OP_KEYSWITCH, NEO_OP_HMULT, NEO_OP_HROT, NEO_OP_RESCALE, NEO_OP_HROT_HOISTED = 0, 1, 2, 3, 4
+NEO_NTT_FP64, NEO_NTT_TC = 0, 1
 NEO_OP_DOUBLE_RESCALE, NEO_OP_MODRAISE, NEO_OP_HMULT_RESCALE, NEO_OP_HROT_SUM = 5, 6, 7, 8
 _STATUS = {0: "NEO_OK", 1: "NEO_EINVAL", 2: "NEO_EUNSUPPORTED", 3: "NEO_ENOMEM", 4: "NEO_ECUDA",
            5: "NEO_ENCCL", 6: "NEO_ENOPRIME"}
@@ -28,7 +29,8 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_last_error", "neo_last_launch_count", "neo_profile_enable", "neo_profile_read",
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
             "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline", "neo_hsub", "neo_modraise",
-            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale", "neo_ew_limbs", "neo_hrot_sum")
+            "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale", "neo_ew_limbs", "neo_hrot_sum",
+            "neo_ntt_select", "neo_ntt_selected")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -94,6 +96,8 @@ def lib() -> ctypes.CDLL:
             "neo_wire_pack": [_vp, _vp, _vp, _sz, _vp],
             "neo_wire_unpack": [_vp, _vp, _vp, _sz, _vp],
             "neo_pmult_acc": [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), _i32, _i32, _i32, _vp, _i32, _vp],
+            "neo_ntt_select": [_vp, _i32],
+            "neo_ntt_selected": [_vp],
         }
         for name, args in sig.items():
             if not hasattr(L, name):        # an older build (A/B runs); tests/test_abi.py requires every symbol
@@ -218,6 +222,14 @@ class Context:
             self.close()
         except Exception:
             pass
+
+    def ntt_select(self, impl: int):
+        """neo_ntt_select: NEO_NTT_TC (tcgen05 DFT stages) or NEO_NTT_FP64 (CUDA-core butterflies)."""
+        _check(lib().neo_ntt_select(self.handle, impl), "neo_ntt_select")
+
+    @property
+    def ntt_impl(self) -> int:
+        return int(lib().neo_ntt_selected(self.handle))
 
     def workspace_size(self, op: int, level: int, batch: int) -> int:
         return int(lib().neo_workspace_size(self.handle, op, level, batch))
