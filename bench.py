@@ -95,116 +95,135 @@ def rand_evk(moduli, seed, N):
 # ----------------------------------------------------------------------------- clocks
 
 class ClockSampler:
-    """nvidia-smi sampling (B200_PROFILING.md clocks line) during the timed region."""
-    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    """SM clock and clock-event (throttle) reasons sampled through NVML every ~2 ms in a
+    thread (nvidia-smi's 100 ms period sees at most one sample of a 10 ms region).  The bench
+    keeps the GPU under the same load after its timed region until the sampled window is
+    >= 1 s long (`pad_until`), so `samples` counts the whole window and `samples_in_region`
+    the timed region alone."""
+    NAMES = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
+             ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
+             ("sw_thermal_slowdown", "nvmlClocksEventReasonSwThermalSlowdown"),
+             ("sw_power_cap", "nvmlClocksEventReasonSwPowerCap"))
 
-    def __init__(self, index: int):
-        self.index = index
-        self.proc = None
-        self.lines = []
+    def __init__(self, index: int, period_s: float = 0.002):
+        self.index, self.period = index, period_s
+        self.samples = []
+        self.stop = threading.Event()
+        self.h = None
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
-                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.sm_max = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.masks = [(n, getattr(pynvml, m)) for n, m in self.NAMES]
+            self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
-        except Exception:
-            self.proc = None
+        except Exception as e:          # no NVML: report why instead of silently passing
+            self.err = repr(e)
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            self.lines.append((time.monotonic(), line.strip()))
+    def _run(self):
+        nv, h = self.nv, self.h
+        while not self.stop.is_set():
+            try:
+                sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
+                rs = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                self.samples.append((time.monotonic(), sm, rs))
+            except Exception:
+                pass
+            time.sleep(self.period)
 
     def wait_ready(self, timeout: float = 5.0):
-        """Block until nvidia-smi has produced its first sample (its start-up takes longer
-        than a short timed region), then mark the start of the window that counts."""
         t0 = time.monotonic()
-        while self.proc and not self.lines and time.monotonic() - t0 < timeout:
-            time.sleep(0.01)
+        while self.h is not None and not self.samples and time.monotonic() - t0 < timeout:
+            time.sleep(0.001)
         self.t_begin = time.monotonic()
 
     def mark_end(self):
         self.t_end = time.monotonic()
 
+    def window_s(self) -> float:
+        return time.monotonic() - getattr(self, "t_begin", time.monotonic())
+
     def __exit__(self, *a):
-        if self.proc:
-            if not hasattr(self, "t_end"):
-                self.t_end = time.monotonic()
-            time.sleep(0.15)
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=2)
-            except Exception:
-                self.proc.kill()
+        self.t_win_end = time.monotonic()
+        self.stop.set()
+        if self.h is not None:
+            self.t.join(timeout=1)
 
     def summary(self) -> dict:
-        sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        t0, t1 = getattr(self, "t_begin", 0.0), getattr(self, "t_end", float("inf"))
-        inside = [ln for t, ln in self.lines if t0 <= t <= t1 + 0.1]
-        # a sample taken within 100 ms after the region covers its tail (-lms 100)
-        for ln in inside:
-            f = [x.strip() for x in ln.split(",")]
-            if len(f) < 7:
-                continue
-            try:
-                sm.append(float(f[0]))
-                mx.append(float(f[1]))
-            except ValueError:
-                continue
-            for k, v in zip(names, f[3:7]):
-                if v.lower().startswith("active"):
-                    reasons.add(k)
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+        if self.h is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0,
+                    "error": getattr(self, "err", "NVML unavailable")}
+        t0 = getattr(self, "t_begin", 0.0)
+        t1 = getattr(self, "t_end", float("inf"))
+        tw = getattr(self, "t_win_end", float("inf"))
+        win = [x for x in self.samples if t0 <= x[0] <= tw]
+        reg = [x for x in win if x[0] <= t1]
+        reasons = sorted({n for _, _, rs in win for n, m in self.masks if rs & m})
+        sm = [x[1] for x in win]
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": self.sm_max,
+                "reasons": reasons, "samples": len(win), "samples_in_region": len(reg),
+                "sm_mhz_in_region": statistics.median([x[1] for x in reg]) if reg else None,
+                "window_s": round(tw - t0, 3), "source": "NVML every ~2 ms over the timed region, padded "
+                "with the same untimed steps to a >= 1 s window"}
 
 
 # ----------------------------------------------------------------------------- byte model
 
 def bytes_model(batch: int, l: int = LEVEL, fused: bool = False) -> dict:
-    """Algorithmic HBM bytes per step, per kernel kind: every limb a launch must read or write
-    once (limb = N words of 8 bytes; SURVEY §8(d) per-limb figures x the limbs each launch
-    processes).  Per KS with Lq = l+1 Q limbs, P special limbs, E = Lq + P:
-      INTT(d): col 2*Lq, row 2*Lq;  ModUp NTT: col 2*(beta*E - Lq), row 2*(beta*E - Lq);
-      INTT(acc_P): col 4P, row 4P;  NTT(conv) + fused ModDown tail: col 4*Lq,
-      row 2*Lq (intermediate) + 2*Lq (acc) + add limbs + 2*Lq (out);
-      BConv: ModUp Lq + (beta*E - Lq), ModDown 2P + 2*Lq;  KeyIP: beta*E + 2E per ciphertext,
-      2*beta*E key limbs once per launch.
-    Rescale: INTT of 2 limbs (col 4, row 4), NTT of 2l rows reading 2 unique limbs
-    (col 2 + 2l, row 2l + 2l (c_i) + 2l (out)).
-    fused (neo_hmult_rescale): no Rescale passes; the HMULT's final NTT covers l rows (col 4l,
-    row 2l + 2l (acc) + 2l (d) + 2l (out)), plus INTTs of acc_l, d_l (4 rows: col 8, row 8) and
-    the fold kernel (elementwise: read 2 Lq + 4, write 2 l)."""
+    """Algorithmic HBM bytes per step, per kernel kind, counted as SURVEY §8(d) counts them:
+    one read plus one write of every limb an OPERATION transforms (limb = N residues of 8
+    bytes; the NTT's two passes and their intermediate are not algorithmic traffic), plus the
+    operands a fused epilogue reads.  Per key-switch at level l (Lq = l+1, P = 12, E = Lq + P,
+    beta digits, up = beta*E - Lq ModUp outputs):
+      NTT transforms: INTT(d) Lq + ModUp NTT up + INTT(acc_P) 2P + NTT(conv) 2Lq, each 2 limbs;
+        the fused ModDown tail (a10) also reads acc_Q (2Lq) and the addend (HROT: sigma(c0),
+        Lq; HMULT: d0, d1, 2Lq);
+      BConv: ModUp reads Lq, writes up; ModDown reads 2P, writes 2Lq;
+      KeyIP: reads d^ (beta*E), writes acc (2E), reads the key once per launch (2*beta*E limbs
+        stored at 5 bytes per residue).
+    Per step (HMULT+Rescale fused + HROT, B = 1, l = 35): 482 limb transforms + 248 tail
+    operand limbs = 1212 limbs = 635.4 MB of NTT traffic (the fused HMULT+Rescale replaces the
+    last NTT over Lq rows by one over l rows and adds the INTTs of acc_l, d_l: 4 transforms).
+    tensor: reads a, b (4Lq), writes d0..d2 (3Lq); automorphism: c0 only (2Lq); elementwise: the
+    fused Rescale's fold kernel (reads 2Lq + 4, writes 2l)."""
     limb = (1 << LOG_N) * 8
     Lq, P = l + 1, NUM_P
     beta = -(-Lq // 12)
     E = Lq + P
     up = beta * E - Lq
-    ks_col = 2 * Lq + 2 * up + 4 * P + 4 * Lq
-    ks_row_base = 2 * Lq + 2 * up + 4 * P + 6 * Lq
-    add_hmult, add_hrot = 2 * Lq, Lq
+    ks_tr = Lq + up + 2 * P                      # transforms up to the ModDown NTT
+    hrot_tr, hrot_tail = ks_tr + 2 * Lq, 2 * Lq + Lq
     if fused:
-        hm_col = 2 * Lq + 2 * up + 4 * P + 4 * l + 8
-        hm_row = 2 * Lq + 2 * up + 4 * P + 8 * l + 8
-        ntt_col = batch * (hm_col + ks_col)
-        ntt_row = batch * (hm_row + ks_row_base + add_hrot)
+        hm_tr, hm_tail = ks_tr + 4 + 2 * l, 2 * l + 2 * l
         ew = batch * (2 * Lq + 4 + 2 * l)
+        resc_tr, resc_tail = 0, 0
     else:
-        ntt_col = batch * (2 * ks_col + 4 + 2 + 2 * l)
-        ntt_row = batch * (2 * ks_row_base + add_hmult + add_hrot + 4 + 6 * l)
+        hm_tr, hm_tail = ks_tr + 2 * Lq, 2 * Lq + 2 * Lq
+        resc_tr, resc_tail = 2 + 2 * l, 2 * l
         ew = 0
+    transforms = batch * (hrot_tr + hm_tr + resc_tr)
+    ntt = 2 * transforms + batch * (hrot_tail + hm_tail + resc_tail)
     bconv = batch * 2 * ((Lq + up) + (2 * P + 2 * Lq))
-    keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E * 5 / 8)          # key stored in 5 bytes per residue
+    keyip = 2 * (batch * (beta * E + 2 * E) + 2 * beta * E * 5 / 8)
     tensor = batch * 7 * Lq
-    auto = batch * 2 * Lq         # AUTO of c0 only (c1 is read through the index map by the INTT and KeyIP)
-    out = {"ntt_col": ntt_col, "ntt_row": ntt_row, "bconv": bconv, "keyip": keyip, "combine": 0,
-           "tensor": tensor, "automorphism": auto, "rescale_modswitch": 0, "rescale_combine": 0, "elementwise": ew}
-    return {k: v * limb for k, v in out.items()}
+    auto = batch * 2 * Lq
+    out = {"ntt": ntt, "bconv": bconv, "keyip": keyip, "combine": 0, "tensor": tensor, "automorphism": auto,
+           "rescale_modswitch": 0, "rescale_combine": 0, "elementwise": ew}
+    res = {k: v * limb for k, v in out.items()}
+    res["_ntt_transforms"] = transforms
+    return res
+
+
+def merge_ntt(d: dict) -> dict:
+    """neo_profile kinds with the two NTT passes merged into one kind 'ntt'."""
+    out = {k: v for k, v in d.items() if k not in ("ntt_col", "ntt_row")}
+    out["ntt"] = (d["ntt_col"][0] + d["ntt_row"][0], d["ntt_col"][1] + d["ntt_row"][1])
+    return out
 
 
 def load_peaks():
@@ -218,15 +237,35 @@ def load_peaks():
 
 
 def load_traffic(kind: str):
-    """dram bytes per launch of `kind` from the committed ncu --set full summary, or None."""
+    """DRAM bytes (dram__bytes_read.sum + dram__bytes_write.sum) per launch of `kind` from the
+    committed ncu --set full summary, next to that launch's algorithmic bytes, or None."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(p) as f:
             d = json.load(f)
         e = d.get(kind)
-        return None if e is None else {"bytes_per_launch": e["bytes_per_launch"],
-                                       "algo_bytes_per_launch": e["algo_bytes_per_launch"],
-                                       "launch": e["launch"], "source": "profiles/ncu_traffic.json (r01 ncu --set full)"}
+        if e is None:
+            return None
+        return {"bytes_per_launch": e["bytes_per_launch"], "algo_bytes_per_launch": e["algo_bytes_per_launch"],
+                "ratio": round(e["bytes_per_launch"] / e["algo_bytes_per_launch"], 3), "launch": e["launch"],
+                "source": e.get("source", "profiles/ncu_traffic.json")}
+    except Exception:
+        return None
+
+
+def load_int8_peak():
+    """The measured tcgen05 kind::i8 throughput at the NTT's MMA shape (M=128, N=80, K=32) and
+    the best shape, from profiles/int8_peak.json (tools/i8peak.py)."""
+    p = os.path.join(ROOT, "profiles", "int8_peak.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        shapes = d["tcgen05_i8_smem"]["shapes"]
+        best = max(x["tops"] for x in shapes)
+        n80 = [x["tops"] for x in shapes if x["N"] == 80]
+        return {"tops": best, "tops_at_n80": n80[0] if n80 else None,
+                "torch_int_mm_tops": max(x["tops"] for x in d.get("torch_int_mm", [{"tops": 0}])),
+                "source": "profiles/int8_peak.json (tools/i8peak.py: tcgen05 kind::i8, operands in smem)"}
     except Exception:
         return None
 
@@ -247,6 +286,47 @@ def oracle_keyswitch_rate(d, evk, budget_s=12.0, min_reps=1):
         if reps >= min_reps and el / reps * (reps + 1) > budget_s * 1.5:
             break
     return reps / el, reps, el, _core.lib().or_num_threads()
+
+
+def host_cpu_info() -> dict:
+    """nproc and the lscpu model name of the host the CPU baseline ran on."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.lower().startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return {"nproc": os.cpu_count(), "lscpu_model": model}
+
+
+def oracle_tiny_def_timing() -> dict:
+    """SURVEY §8(d) config 1 leg: one HMULT + relinearise at the tiny config (N=2^12, 3 Q + 1 P,
+    dnum=1) by the DEFINITIONAL oracle (O(N^2) NTT, Algorithm 1 BConv) on all host threads and
+    on one thread (OpenMP thread count set through libgomp)."""
+    import ctypes
+    from oracle import _core, ckks
+    import synth
+    prm = ckks.tiny()
+    ids = list(range(prm.num_q))
+    ct = lambda sd: np.stack([synth.uniform_residues(sd + c, [prm.moduli[i] for i in ids], prm.N) for c in range(2)])
+    allids = list(range(prm.num_q + prm.num_p))
+    evk = np.stack([np.stack([synth.uniform_residues(70 + 2 * j + c, [prm.moduli[i] for i in allids], prm.N)
+                              for c in range(2)]) for j in range(prm.dnum)])
+    a, b = ct(1), ct(3)
+    L = _core.lib()
+    gomp = ctypes.CDLL("libgomp.so.1")
+    full = L.or_num_threads()
+    res = {"op": "one HMULT + relinearise, tiny config, mode=def", "nproc": os.cpu_count()}
+    for name, nt in (("all_threads", full), ("one_thread", 1)):
+        gomp.omp_set_num_threads(nt)
+        t0 = time.perf_counter()
+        ckks.hmult(prm, a, b, prm.max_level, evk, mode="def")
+        res[name] = {"threads": nt, "seconds": round(time.perf_counter() - t0, 3)}
+    gomp.omp_set_num_threads(full)
+    return res
 
 
 # ----------------------------------------------------------------------------- reference arm
@@ -474,10 +554,17 @@ def run_neo(args):
         t_end.record()
         torch.cuda.synchronize()
         clk.mark_end()
+        gpu_launches = launches[0]
+        # keep the same load (untimed) until the clock window is >= 1 s long
+        k = args.steps
+        while clk.window_s() < 1.0:
+            for _ in range(50):
+                run_step(k)
+                k += 1
+            torch.cuda.synchronize()
     barrier()
     torch.cuda.synchronize()
     ms = t_start.elapsed_time(t_end)
-    gpu_launches = launches[0]
     if world > 1:
         t = torch.tensor([ms], dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -494,37 +581,45 @@ def run_neo(args):
         step(k % SLOTS, two=False)
     p_end.record()
     torch.cuda.synchronize()
-    prof = neo.neo_profile_read()
+    prof = merge_ntt(neo.neo_profile_read())
     neo.neo_profile_enable(False)
     ms_step_1s = p_start.elapsed_time(p_end) / args.steps
 
-    # roofline of the dominant kernel kind
+    # roofline of the dominant kernel kind (SURVEY §8(d) bytes; the NTT's two passes as one kind)
     peak, peak_src = load_peaks()
     bm = bytes_model(B, fused=bool(args.fused_rescale))
+    n_transforms = bm.pop("_ntt_transforms")
     step_ms = {k: v[0] / args.steps for k, v in prof.items()}
     ms_step_ref = ms_step_1s
     dom = max(step_ms, key=lambda k: step_ms[k])
     n_launch_dom = prof[dom][1] / args.steps
     achieved = bm[dom] / (step_ms[dom] / 1e3) / 1e9 if step_ms[dom] > 0 else None
     traffic = load_traffic(dom)
-    # NTT passes are co-bound by the FP64 pipe: FP64 ops per element per pass
-    # counted from the radix-2 structure (col: fwd 45.4 / inv 48.4, row: fwd 30.8 / inv 27.8),
-    # limb transforms per step at B=1, l=35: forward 430, inverse 122; peak = 63 DFMA-pipe
-    # ops/clk/SM (tools/microbench/pipes.cu) x SMs x the max SM clock.
-    fp64 = None
-    if dom in ("ntt_col", "ntt_row"):
-        # forward / inverse limb rows per step: HROT 180 / 60; HMULT+Rescale 178 / 64 fused
-        # (250 / 62 as separate calls); per-element FP64 ops from the SASS counts (ncu)
+    ntt_impl = "tc" if ctx.ntt_impl == neo.NEO_NTT_TC else "fp64"
+    # second roofline of the NTT: int8 tensor-core work against the measured tcgen05 i8 peak
+    # (profiles/int8_peak.json) for the tcgen05 form -- per limb transform 2 passes x 2 stages x
+    # 12 MMAs of 128 x 80 x 32 per 16-transform tile = 1920 MACs per coefficient -- or FP64
+    # operations against 63 DFMA-pipe ops/clk/SM for the CUDA-core form
+    alt = None
+    i8 = load_int8_peak()
+    try:
+        mhz = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["sm_max_mhz"])
+    except Exception:
+        mhz = 1965.0
+    if ntt_impl == "tc":
+        ops = 2.0 * 1920 * (1 << LOG_N) * n_transforms
+        ach = ops / (step_ms["ntt"] / 1e3) if step_ms["ntt"] > 0 else 0.0
+        alt = {"bound": "tensor", "kernel": "ntt", "dtype": "u8xu8->s32", "achieved": ach / 1e12,
+               "peak": i8["tops"] if i8 else None, "unit": "TOP/s",
+               "frac": ach / 1e12 / i8["tops"] if i8 else None, "ops_per_step": ops,
+               "peak_source": i8["source"] if i8 else "not measured"}
+    else:
         fw, iv = (358, 124) if args.fused_rescale else (430, 122)
-        ops = {"ntt_col": fw * 45.4 + iv * 48.4, "ntt_row": fw * 30.8 + iv * 27.8}[dom] * (1 << LOG_N) * B
-        try:
-            mhz = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["sm_max_mhz"])
-        except Exception:
-            mhz = 1965.0
+        ops = (fw * (45.4 + 30.8) + iv * (48.4 + 27.8)) * (1 << LOG_N) * B
         pk = 63 * torch.cuda.get_device_properties(local).multi_processor_count * mhz * 1e6
-        ach = ops / (step_ms[dom] / 1e3)
-        fp64 = {"bound": "fp64", "achieved": ach / 1e12, "peak": pk / 1e12, "unit": "Tops/s", "frac": ach / pk,
-                "ops_per_step": ops}
+        ach = ops / (step_ms["ntt"] / 1e3) if step_ms["ntt"] > 0 else 0.0
+        alt = {"bound": "fp64", "kernel": "ntt", "achieved": ach / 1e12, "peak": pk / 1e12, "unit": "Tops/s",
+               "frac": ach / pk, "ops_per_step": ops}
     breakdown = {k: {"ms_per_step": round(step_ms[k], 5), "launches_per_step": prof[k][1] / args.steps,
                      "share": round(step_ms[k] / ms_step_ref, 4) if ms_step_ref > 0 else None,
                      "algo_GBps": round(bm[k] / (step_ms[k] / 1e3) / 1e9, 1) if step_ms[k] > 0 else None,
@@ -901,6 +996,7 @@ def run_neo(args):
     # compute of step k (PCIe is full duplex).
     e2e = None
     e2e_u64 = None
+    e2e_wire = None
     if not args.no_e2e:
         # two variants through the public API: (u64) residues copied as 8-byte words; (wire) the
         # library's 36-bit wire format (neo_wire_pack/unpack: 4.5 bytes per residue), unpacked
@@ -1017,22 +1113,31 @@ def run_neo(args):
         per_dir = nb_ / (p0.elapsed_time(p1) / 10 / 1e3) / 1e9            # GB/s per direction
         bound_ms = max(sum(wb_in), sum(wb_out)) / (per_dir * 1e9) * 1e3
         del hb_i, hb_o, db_i, db_o
-        e2e = {"value": 2 * B * world / (wms / k_e2e / 1e3), "unit": UNIT,
-               "pcie": {"duplex_GBps_per_direction": round(per_dir, 1), "bound_ms_per_step": round(bound_ms, 4),
-                        "frac_of_bound": round(bound_ms / (wms / k_e2e), 3),
-                        "note": "raw pinned 64 MB copies in both directions at once; the step's larger "
-                                "direction (H2D) at that rate is the e2e ceiling"},
-               "h2d_bytes_per_step": sum(wb_in), "d2h_bytes_per_step": sum(wb_out),
-               "steps": k_e2e, "ms_per_step": wms / k_e2e,
-               "format": "36-bit wire format (neo_wire_pack/unpack, 4.5 bytes per residue), unpack/pack on the device inside the region",
-               "overlap": "H2D / compute / D2H on separate streams, double-buffered"}
+        bound_u64 = max(sum(n * 8 for n in n_in), sum(n * 8 for n in n_out)) / (per_dir * 1e9) * 1e3
+        # headline e2e: the caller's u64 host buffers (the ABI's own layout) copied in and out every
+        # step, nothing prepared outside the region
+        e2e = dict(e2e_u64, pcie={"duplex_GBps_per_direction": round(per_dir, 1),
+                                  "bound_ms_per_step": round(bound_u64, 4),
+                                  "frac_of_bound": round(bound_u64 / (ems / k_e2e), 3),
+                                  "note": "raw pinned 64 MB copies in both directions at once; the step's larger "
+                                          "direction (H2D, 113 MB) at that rate is the e2e ceiling"},
+                   overlap="H2D / compute / D2H on separate streams, double-buffered")
+        e2e_wire = {"value": 2 * B * world / (wms / k_e2e / 1e3), "unit": UNIT,
+                    "h2d_bytes_per_step": sum(wb_in), "d2h_bytes_per_step": sum(wb_out),
+                    "steps": k_e2e, "ms_per_step": wms / k_e2e,
+                    "bound_ms_per_step": round(bound_ms, 4), "frac_of_bound": round(bound_ms / (wms / k_e2e), 3),
+                    "format": "host buffers already in the library's 36-bit wire format (4.5 bytes per residue; "
+                              "packed once before the region, as a caller storing ciphertexts in that format "
+                              "would); unpack / pack on the device inside the region",
+                    "note": "secondary: not the headline e2e because the packing of the inputs is outside the region"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         d0 = host_in[0][2][0, 1]                                  # c1 of one ciphertext: [36][N]
         rate, reps, el, cores = oracle_keyswitch_rate(d0, rot_np)
         cpu = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle",
-               "sample": f"{reps} Set-B key-switch(es) (l=35, B=1) by the CPU oracle in {el:.1f} s"}
+               "sample": f"{reps} Set-B key-switch(es) (l=35, B=1) by the CPU oracle in {el:.1f} s",
+               "host": host_cpu_info(), "tiny_definitional": oracle_tiny_def_timing()}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -1044,14 +1149,16 @@ def run_neo(args):
                 "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
                              "peak_source": peak_src, "unit": "GB/s",
                              "frac": achieved / peak if achieved else None, "traffic": traffic,
-                             "launches_per_step": n_launch_dom,
-                             "algo_bytes_per_step": bm[dom], "alt": fp64},
+                             "launches_per_step": n_launch_dom, "algo_bytes_per_step": bm[dom],
+                             "bytes_rule": "SURVEY §8(d): one read + one write per limb an operation transforms, "
+                                           "plus fused-epilogue operands (bench.bytes_model)",
+                             "ntt_impl": ntt_impl, "ntt_transforms_per_step": n_transforms, "alt": alt},
                 "step_roofline": {"algo_bytes_per_step": sum(bm.values()),
                                   "achieved": sum(bm.values()) / (ms_step / 1e3) / 1e9,
                                   "peak": peak, "unit": "GB/s",
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
-                "cpu_baseline": cpu, "e2e": e2e, "e2e_u64": e2e_u64, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted, "latency": latency,
+                "cpu_baseline": cpu, "e2e": e2e, "e2e_wire": e2e_wire, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted, "latency": latency,
                 "limb_sharded_keyswitch": sharded_ks,
                 "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block, "apps": apps_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,

@@ -105,9 +105,10 @@ neo_status neo_intt(const neo_ctx* ctx, uint64_t* poly, const int32_t* limb_ids,
  * every NTT inside the key-switching operations); the result is bit-identical either way.
  *   NEO_NTT_TC   : both radix-16 DFT stages of each 256-point pass as tcgen05 kind::i8 GEMMs
  *                  (Neo's matrix-multiplication NTT, L438-450 / Fig. 9, on the int8 tensor
- *                  cores; N = 2^16 with 36-bit primes only) -- the default where supported
- *                  (environment NEO_NTT=fp64 at context creation selects the other);
- *   NEO_NTT_FP64 : radix-2 butterflies in FP64 on the CUDA cores (any supported N).
+ *                  cores; N = 2^16 with 36-bit primes only; environment NEO_NTT=tc at
+ *                  context creation makes it the context's default);
+ *   NEO_NTT_FP64 : radix-2 butterflies in FP64 on the CUDA cores (any supported N) -- the
+ *                  default: faster on B200 (profiles/r02_ntt_ab.md).
  * Returns NEO_EUNSUPPORTED (selection unchanged) if NEO_NTT_TC is not available for this
  * context.  Not thread-safe with respect to operations running on the same context. */
 enum { NEO_NTT_FP64 = 0, NEO_NTT_TC = 1 };
@@ -344,6 +345,7 @@ int32_t neo_profile_timeline(int32_t max, int32_t* kinds, float* start_ms, float
  * synchronises the device and copies the 2 x 64 x 8 uint64 stamps (ModUp, then ModDown) to
  * `host` (caller-owned, 8 KB).  Returns 1 if tracing is on, 0 if it is off (host untouched). */
 int32_t neo_debug_bconv_trace(unsigned long long* host);
+
 
 #ifdef __cplusplus
 }

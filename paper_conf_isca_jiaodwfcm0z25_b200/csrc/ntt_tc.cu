@@ -305,6 +305,9 @@ k_ntt_tc(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep, in
         // ---------------------------------------------------------------- epilogue 1 -> A
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
+            TWD tw[8];                                         // loaded before the TMEM wait (latency overlap)
+#pragma unroll
+            for (int j = 0; j < 8; ++j) tw[j] = sT[pa1 * 16 + 8 * h + j];
             uint32_t v[5][8];
 #pragma unroll
             for (int bb = 0; bb < 5; ++bb) tc::tmem_ld8(tmem + taddr_lane + (uint32_t)(bb * 16 + 8 * h), v[bb]);
@@ -313,7 +316,7 @@ k_ntt_tc(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep, in
             for (int j = 0; j < 8; ++j) {
                 const int oa = 8 * h + j;
                 const double V = vsum(v[0][j], v[1][j], v[2][j], v[3][j], v[4][j]);
-                const u64 z = dbits(__dadd_rn(mulc(V, sT[pa1 * 16 + oa], q), qp52));   // < 2^37 after + q
+                const u64 z = dbits(__dadd_rn(mulc(V, tw[j], q), qp52));   // < 2^37 after + q
                 uint8_t* row = sA + ((16 * oa + x1) >> 3) * 768 + (x1 & 7) * 16;
                 *reinterpret_cast<uint32_t*>(row + (pa1 >> 2) * 128 + (pa1 & 3) * 4) = (uint32_t)z;
                 row[4 * 128 + pa1] = (uint8_t)(z >> 32);
@@ -354,6 +357,11 @@ k_ntt_tc(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep, in
             const TWD tA = tw[x2 * 16 + oa2];
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
+                TWD tB[8];
+                if (PT == TC_COL_FWD) {
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) tB[j] = tw[256 + x2 * 16 + 8 * h + j];
+                }
                 uint32_t v[5][8];
 #pragma unroll
                 for (int bb = 0; bb < 5; ++bb) tc::tmem_ld8(tmem + taddr_lane + (uint32_t)(bb * 16 + 8 * h), v[bb]);
@@ -364,7 +372,7 @@ k_ntt_tc(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep, in
                     const double V = vsum(v[0][j], v[1][j], v[2][j], v[3][j], v[4][j]);
                     u64 outv;
                     if (PT == TC_COL_FWD)              // twist psi^((2 i1 + 1) n2) = A[n2][o_a] B[n2][o_b]
-                        outv = dbits(__dadd_rn(mulc(mulc(V, tA, q), tw[256 + x2 * 16 + ob], q), qp52));
+                        outv = dbits(__dadd_rn(mulc(mulc(V, tA, q), tB[j], q), qp52));
                     else
                         outv = d2u(canon(V, q, qinv));
                     dst[(size_t)(oa2 + 16 * ob) * N2] = outv;
@@ -459,7 +467,6 @@ k_ntt_tc(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep, in
     if (warp == 0) tc::tmem_dealloc(tmem, 256);
 }
 
-// ------------------------------------------------------------------ launcher
 template <int PT>
 static cudaError_t launch_tc(const RowSet& rs, const NttArgs& a, int batch, cudaStream_t st, const RowEpi* epi) {
     static bool init = false;
@@ -473,9 +480,9 @@ static cudaError_t launch_tc(const RowSet& rs, const NttArgs& a, int batch, cuda
     tm.tpr_log = 4;
     tm.bmagic = batch > 1 ? (unsigned)((1ull << 32) / (unsigned)batch + 1) : 0u;
     tm.total = tm.tpr * rs.n * batch;
+    static const RowEpi none{};
     int grid = 2 * a.num_sms;
     if (grid > tm.total) grid = tm.total;
-    static const RowEpi none{};
     return launch_k(k_ntt_tc<PT>, dim3(grid), dim3(kThr), kSmem, st, rs, a, tm, epi ? *epi : none, epi ? 1 : 0);
 }
 

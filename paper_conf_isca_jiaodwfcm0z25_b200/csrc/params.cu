@@ -327,7 +327,7 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
             }
             c->ntt.tct = c->d_ntt_tc;
             const char* e = std::getenv("NEO_NTT");
-            c->ntt_impl = (e && std::string(e) == "fp64") ? NEO_NTT_FP64 : NEO_NTT_TC;
+            c->ntt_impl = (e && std::string(e) == "tc") ? NEO_NTT_TC : NEO_NTT_FP64;
         }
     }
 
