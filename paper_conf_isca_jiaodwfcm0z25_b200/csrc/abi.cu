@@ -678,7 +678,15 @@ static neo_status run_chunked(const neo_ctx* c, int batch, void* ws, size_t ws_b
         void* wk = alt ? static_cast<void*>(static_cast<char*>(ws) + chunk_ws) : ws;
         neo_status s = f(b0, nb, wk, alt ? chunk_ws : (two ? chunk_ws : ws_bytes), alt ? c->side : st);
         launches += g_launches;
-        if (s != NEO_OK) return s;
+        if (s != NEO_OK) {
+            if (two) {                     // still join the side stream (keeps a graph capture valid)
+                const std::string msg = g_err;
+                cudaEventRecord(ev_join, c->side);
+                cudaStreamWaitEvent(st, ev_join, 0);
+                g_err = msg;
+            }
+            return s;
+        }
     }
     if (two) {
         CK(cudaEventRecord(ev_join, c->side));
@@ -840,6 +848,8 @@ static neo_status ntt_api(const neo_ctx* c, bool fwd, uint64_t* poly, const int3
     TRY(check_ptr(poly, "poly"));
     if (!ids || n <= 0 || n > NEO_MAX_ROWS) FAIL(NEO_EINVAL, "need 1 <= n_limbs <= 160 limb ids");
     if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
+    if ((long long)n * batch * batch >= (1ll << 32))      // the tile decode's 32-bit magic division
+        FAIL(NEO_EUNSUPPORTED, "neo_ntt / neo_intt: n_limbs * batch^2 must be < 2^32");
     for (int k = 0; k < n; ++k)
         if (ids[k] < 0 || ids[k] >= c->limbs_total()) FAIL(NEO_EINVAL, "unknown limb id");
     size_t need = (size_t)batch * n * c->N * sizeof(u64);
@@ -868,6 +878,7 @@ neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids
     if (!in_ids || !out_ids || n_in < 1 || n_in > BC_MAX_IN || n_out < 1 || n_out > BC_MAX_OUT)
         FAIL(NEO_EINVAL, "need 1 <= n_in <= 16 and 1 <= n_out <= 64");
     if (batch <= 0) FAIL(NEO_EINVAL, "batch must be positive");
+    if (batch >= 4096) FAIL(NEO_EUNSUPPORTED, "neo_bconv: batch must be < 4096 (12-bit tile schedule field)");
     const int nl = c->num_q + c->num_p;
     for (int i = 0; i < n_in; ++i) {
         if (in_ids[i] < 0 || in_ids[i] >= nl) FAIL(NEO_EINVAL, "unknown input limb id");
@@ -982,10 +993,12 @@ static neo_status evk_create(const neo_ctx* c, const uint64_t* evk, uint32_t gal
         neo_evk_destroy(k);
         FAIL(NEO_ENOMEM, "cudaMalloc of the evaluation key failed");
     }
-    cudaError_t e = cudaSuccess;
+    // the key may have been written on any of the caller's streams (e.g. a non-blocking torch
+    // stream, which the legacy stream does not wait for): finish all device work first
+    cudaError_t e = cudaDeviceSynchronize();
     const u64* src = evk;
     u64* perm = nullptr;
-    if (galois) {                          // sigma_{g^-1} of every key polynomial (NTT-domain gather)
+    if (e == cudaSuccess && galois) {                          // sigma_{g^-1} of every key polynomial (NTT-domain gather)
         const u64 two_n = 2ull * c->N;
         u64 ginv = 1, b = galois, ex = c->N - 1;            // g^-1 = g^(N-1) mod 2N (odd g)
         for (; ex; ex >>= 1, b = b * b % two_n)
@@ -1021,7 +1034,10 @@ neo_status neo_evk_create_klss(const neo_ctx* c, const uint64_t* ekey, neo_evk**
         neo_evk_destroy(k);
         FAIL(NEO_ENOMEM, "cudaMalloc of the KLSS key failed");
     }
-    cudaError_t e = launch_pack5(ekey, k->lo, k->hi, n, nullptr);
+    // the key may have been written on any of the caller's streams (e.g. a non-blocking torch
+    // stream, which the legacy stream does not wait for): finish all device work first
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e == cudaSuccess) e = launch_pack5(ekey, k->lo, k->hi, n, nullptr);
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
     if (e != cudaSuccess) {
         neo_evk_destroy(k);

@@ -93,14 +93,14 @@ def limb_sharded_keyip(ops, plan: ShardPlan, d_local, evk):
     """Steps a3-a6 (INTT, exchange #1, ModUp, NTT, KeyIP): the rank's rows of the KeyIP output
     acc [B][2][len(plan.mine)][N] (PQ_l, NTT form)."""
     P = plan
-    # a3: INTT of the rank's Q limbs, then exchange #1: every rank gets all Q limbs
-    y_local = ops.intt(d_local, P.my_q)
+    # a3: INTT of the rank's Q limbs, then exchange #1: every rank gets all Q limbs.  A rank
+    # that owns no Q limb (world > level + 1) still joins both exchanges: it owns P limbs the
+    # other ranks' ModDown needs, and returns empty outputs.
+    y_local = ops.intt(d_local, P.my_q) if P.my_q else d_local
     y_all = ops.allgather(y_local, [len(b) for b in P.q_blocks])          # [B][l+1][N]
     if P.q_perm is not None:
         y_all = ops.take(y_all, P.q_perm)
     # a4/a5: ModUp of every digit onto this rank's own target limbs, then NTT
-    if not P.my_q:
-        raise ValueError("limb-sharded key-switch needs world <= level + 1 (every rank owns a Q limb)")
     dhat_rows = []                                                          # per digit: [B][n_mine][N]
     for dj in P.digits:
         targets = [t for t in P.mine if t not in dj]
@@ -124,6 +124,9 @@ def limb_sharded_moddown(ops, plan: ShardPlan, acc):
     if P.p_perm is not None:
         acc_p_all = ops.take2(acc_p_all, P.p_perm)
     # a8/a9: ModDown BConv onto the rank's Q limbs, NTT, a10: combine
+    if not P.my_q:
+        empty = ops.empty2(acc, 0)
+        return ops.component(empty, 0), ops.component(empty, 1)
     conv = ops.ntt2(ops.bconv2(acc_p_all, P.p_ids, P.my_q), P.my_q)
     q_pos = [P.mine.index(t) for t in P.my_q]
     out = ops.moddown_combine(ops.take2(acc, q_pos), conv, P.my_q)          # [B][2][n_q][N]

@@ -126,7 +126,7 @@ def _worker(rank, world, port, cfg, level, q, strided=False):
         plan = ShardPlan(level, prm.num_q, prm.num_p, prm.alpha, world, rank, strided=strided)
         ops = OracleOps(prm)
         k0, k1 = limb_sharded_keyswitch(ops, plan, np.ascontiguousarray(d[:, plan.my_q]), evk)
-        ok = True
+        ok = k0.shape == (B, len(plan.my_q), prm.N) and k1.shape == k0.shape
         for b in range(B):
             r0, r1 = ckks.keyswitch(prm, d[b], level, evk)
             ok &= np.array_equal(k0[b], r0[plan.my_q]) and np.array_equal(k1[b], r1[plan.my_q])
@@ -151,6 +151,8 @@ def _free_port():
     (2, (10, 3, 1, 1), 2, False),      # dnum = 1 (one digit spans both ranks)
     (2, (10, 6, 2, 3), 4, True),       # round-robin ownership (the sharded evaluator's plan)
     (3, (10, 6, 2, 3), 5, True),
+    (3, (10, 6, 3, 3), 1, False),      # world > level + 1: rank 2 owns no Q limb, only P limbs
+    (4, (10, 6, 4, 3), 1, True),       # round-robin, ranks 2 and 3 own P limbs only
 ])
 def test_limb_sharded_keyswitch_gloo(world, cfg, level, strided):
     ctx = mp.get_context("spawn")

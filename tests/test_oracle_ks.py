@@ -229,3 +229,26 @@ def test_hrot_hoisted_rotates_slots(enc_setup):
     for r, ct in zip(rs, out):
         m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, ct, s, 2), [0, 1, 2])
         assert np.max(np.abs(ckks.decode(prm.N, m, delta) - np.roll(za, -r))) < 1e-6
+
+
+@pytest.mark.parametrize("mk,level", [(ckks.tiny, 2), (ckks.tiny_dnum3, 2), (ckks.tiny_dnum3, 0)])
+def test_moddown_exact_floor_pin(mk, level):
+    """Z9 pinned on its own (not through a noise bound, which a sign error in the combine
+    (acc - conv) -> (acc + conv) survives: with e_j = 0 the extra 2 conv / P term decrypts to a
+    small multiple of (1 + h)).  For every coefficient, with A the exact big-integer CRT lift of
+    the KeyIP output acc_c over PQ_l, ModDown's output must equal floor(A / P) - u (mod Q_l) with
+    the BConv overflow u in [0, K+1) (Algorithm 1 non-centred, Z7)."""
+    prm = mk()
+    q_ids = list(range(level + 1))
+    ext = q_ids + prm.p_ids
+    d = synth.uniform_residues(41, prm.q[: level + 1], prm.N)
+    evk = np.stack([np.stack([synth.uniform_residues(50 + 2 * j + c, prm.moduli, prm.N) for c in range(2)])
+                    for j in range(prm.dnum)])
+    tr = {}
+    out = ckks.keyswitch(prm, d, level, evk, trace=tr)
+    Q = math.prod(prm.q[: level + 1])
+    for c in range(2):
+        A = ckks.crt_lift(prm, ckks.intt(prm, tr["acc"][c], ext), ext)
+        got = ckks.crt_lift(prm, ckks.intt(prm, out[c], q_ids), q_ids)
+        us = {((a // prm.P) - g) % Q for a, g in zip(A, got)}
+        assert us <= set(range(prm.num_p)), sorted(us)[:4]
