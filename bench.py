@@ -697,6 +697,59 @@ def run_neo(args):
                       "limbs_per_rank": len(plan.mine),
                       "note": "eager Python orchestration over C-ABI building blocks (host-issued launches)"}
 
+    # the same key-switch through the NATIVE limb-sharded call (neo_keyswitch_sharded: both
+    # exchanges inside the library, NCCL over NVLink for N > 1, per-digit gathers overlapped with
+    # the previous digit's BConv + NTT), eager and as a captured CUDA graph
+    sharded_native = None
+    if not args.no_latency:
+        if world > 1:
+            uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
+            if rank == 0:
+                uid.copy_(torch.frombuffer(bytearray(neo.Comm.unique_id()), dtype=torch.uint8))
+            dist.broadcast(uid, src=0)
+            ncomm = neo.Comm.create(ctx, bytes(uid.cpu().numpy().tobytes()), world, rank)
+        else:
+            ncomm = neo.Comm.create(ctx, bytes(128), 1, 0)
+        nq_ids, _ = ncomm.limbs(LEVEL)
+        full_d = dev_in[0][0][:, 1].contiguous()
+        dl = full_d.view(torch.int64)[:, nq_ids].contiguous().view(torch.uint64) if nq_ids else None
+        so0 = torch.empty((B, len(nq_ids), N), dtype=torch.uint64, device="cuda") if nq_ids else None
+        so1 = torch.empty_like(so0) if nq_ids else None
+        sws = ncomm.workspace(LEVEL, B)
+        run_native = lambda: neo.neo_keyswitch_sharded(ctx, ncomm, relin, dl, LEVEL, so0, so1, B, sws)
+        for _ in range(3):
+            run_native()
+        torch.cuda.synchronize()
+        barrier()
+
+        def time_native(fn, reps=20):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(reps):
+                fn()
+            e1.record()
+            torch.cuda.synchronize()
+            v = e0.elapsed_time(e1) / reps
+            if world > 1:
+                t = torch.tensor([v], dtype=torch.float64, device="cuda")
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                v = float(t.item())
+            return v
+        eager_ms = time_native(run_native)
+        graph_ms = None
+        try:
+            gr = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gr):
+                run_native()
+            graph_ms = time_native(gr.replay)
+        except Exception as e:          # noqa: BLE001 -- reported in the line
+            graph_ms = f"capture failed: {e!r}"[:200]
+        sharded_native = {"ranks": world, "unit": "ms", "ms_per_keyswitch_eager": round(eager_ms, 4),
+                          "ms_per_keyswitch_graph": round(graph_ms, 4) if isinstance(graph_ms, float) else graph_ms,
+                          "q_limbs_per_rank": len(nq_ids), "transport": "nccl" if world > 1 else "none (1 rank)",
+                          "note": "neo_keyswitch_sharded (native C-ABI); slowest rank, CUDA events"}
+        ncomm.close()
+
     # secondary: hoisted rotations (one ModUp shared by n_rot rotations of the same ciphertext)
     hoisted = None
     if not args.no_hoisted:
@@ -1159,7 +1212,7 @@ def run_neo(args):
                                   "frac": sum(bm.values()) / (ms_step / 1e3) / 1e9 / peak,
                                   "note": "whole step (all kernels, 2 streams) against HBM, per GPU"},
                 "cpu_baseline": cpu, "e2e": e2e, "e2e_wire": e2e_wire, "gpu_launches": gpu_launches, "hoisted_rotations": hoisted, "latency": latency,
-                "limb_sharded_keyswitch": sharded_ks,
+                "limb_sharded_keyswitch": sharded_ks, "limb_sharded_keyswitch_native": sharded_native,
                 "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block, "apps": apps_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}

@@ -37,6 +37,7 @@ extern "C" {
 
 typedef struct neo_ctx neo_ctx;   /* parameters + device constant tables */
 typedef struct neo_evk neo_evk;   /* a device-resident evaluation (key-switching) key */
+typedef struct neo_comm neo_comm; /* limb-sharded key-switching communicator (one per rank) */
 typedef void* neo_stream_t;       /* cudaStream_t */
 
 typedef enum {
@@ -45,7 +46,7 @@ typedef enum {
     NEO_EUNSUPPORTED = 2,  /* valid request outside what this build implements (e.g. log_n) */
     NEO_ENOMEM = 3,        /* device/host allocation failed in a create call */
     NEO_ECUDA = 4,         /* a CUDA call or kernel launch failed */
-    NEO_ENCCL = 5,         /* reserved for the limb-sharded path */
+    NEO_ENCCL = 5,         /* NCCL unavailable or failed (limb-sharded key-switch) */
     NEO_ENOPRIME = 6       /* not enough word_bits-bit primes p = 1 mod 2N */
 } neo_status;
 
@@ -213,6 +214,46 @@ neo_status neo_hrot_hoisted(const neo_ctx* ctx, const neo_evk* const* keys, int3
 neo_status neo_hrot_sum(const neo_ctx* ctx, const neo_evk* const* keys, const uint32_t* galois, int32_t n,
                         const uint64_t* const* cts, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
                         size_t ws_bytes, neo_stream_t stream);
+
+/* ------------------------------------------------------------------ limb-sharded key-switch
+ * One Hybrid key-switch (Table 2, Fig. 5) split by RNS limb over nranks ranks, one
+ * GPU each (the paper has no multi-GPU design, L648 cites HE-Booster).  Limb
+ * ownership at level l (round-robin, so a Rescale's dropped top limb rotates over the ranks):
+ * rank r owns the Q limbs q_i with i = r (mod nranks), i <= l, and the P limbs p_k with
+ * k = r (mod nranks).  NTT, KeyIP and the ModDown tail are limb-local; BConv needs every limb,
+ * so the library runs two all-gathers of coefficient-form limbs inside the call: one per ModUp
+ * digit (overlapped with the previous digit's BConv + NTT on a communication stream) and one of
+ * the P limbs before ModDown.  The result equals neo_keyswitch restricted to the rank's limbs,
+ * bit for bit.
+ *
+ * neo_comm_unique_id : a 128-byte NCCL unique id (ncclGetUniqueId); rank 0 creates it and the
+ *                      caller distributes it (e.g. a torch.distributed broadcast).
+ * neo_comm_create    : collective over the nranks processes (same uid); NCCL over NVLink for
+ *                      nranks > 1 (libnccl.so.2 is loaded with dlopen; NEO_ENCCL if absent or if
+ *                      ncclCommInitRank fails, e.g. two ranks on one GPU); nranks = 1 needs no NCCL.
+ *                      Builds this rank's BConv tables for every level (synchronises the device).
+ * neo_comm_create_local : nranks communicators sharing the context's GPU inside ONE process (one
+ *                      host thread per rank must call each sharded operation concurrently; the
+ *                      exchanges are device-to-device copies after a host barrier; not capturable
+ *                      in a CUDA graph).  For tests and single-GPU runs of the sharded path.
+ * neo_comm_limbs     : this rank's Q limb ids (return value = their count) and P limb ids
+ *                      (count in *n_p) at `level`; arrays may be NULL; -1 on invalid arguments.
+ * neo_keyswitch_sharded : d_local [batch][nq][N] = the rank's Q limbs of the KS input, rising
+ *                      limb order, NTT form; out0/out1 [batch][nq][N] the rank's rows of (k0, k1).
+ *                      A rank with nq = 0 (nranks > level + 1) passes NULL buffers and still
+ *                      takes part in both exchanges.  evk: the full Hybrid key (neo_evk_create)
+ *                      on every rank.  1 <= batch <= 32.  ws: neo_workspace_size_sharded bytes.
+ *                      Asynchronous on `stream` (NCCL transport: graph-capturable). */
+neo_status neo_comm_unique_id(uint8_t uid[128]);
+neo_status neo_comm_create(const neo_ctx* ctx, const uint8_t uid[128], int32_t nranks, int32_t rank,
+                           neo_comm** out);
+neo_status neo_comm_create_local(const neo_ctx* ctx, int32_t nranks, neo_comm** comms);
+neo_status neo_comm_destroy(neo_comm* comm);
+int32_t neo_comm_limbs(const neo_comm* comm, int32_t level, int32_t* q_ids, int32_t* p_ids, int32_t* n_p);
+size_t neo_workspace_size_sharded(const neo_comm* comm, int32_t level, int32_t batch);
+neo_status neo_keyswitch_sharded(const neo_ctx* ctx, const neo_comm* comm, const neo_evk* evk,
+                                 const uint64_t* d_local, int32_t level, uint64_t* out0, uint64_t* out1,
+                                 int32_t batch, void* ws, size_t ws_bytes, neo_stream_t stream);
 
 /* Building blocks of the limb-sharded key-switch (each rank owns a subset of
  * the limbs of PQ_l and calls these on its own limbs between NCCL all-gathers):

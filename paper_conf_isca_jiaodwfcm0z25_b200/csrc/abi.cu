@@ -1539,3 +1539,476 @@ neo_status neo_double_rescale(const neo_ctx* c, const uint64_t* ct_in, int32_t l
 }
 
 }  // extern "C"
+
+// ==================================================================== limb-sharded key-switch
+// one key-switch split by RNS limb over `nranks` ranks, NCCL inside the
+// library.  Ownership (round-robin, so every Rescale's dropped top limb rotates over the ranks):
+// rank r owns the Q limbs i = r (mod nranks) of q_0..q_l and the P limbs p_k, k = r (mod nranks).
+// Only BConv needs other ranks' limbs, so the path has two exchange steps, both all-gathers of
+// coefficient-form limbs (Table 2, Fig. 5):
+//   INTT(own Q, q^_i^-1 folded) -> ALL-GATHER per digit j -> ModUp BConv of digit j onto own
+//   targets -> NTT  (digit j+1's gather runs on the communication stream meanwhile)
+//   -> KeyIP (own limbs) -> INTT(own P, P^_k^-1 folded) -> ALL-GATHER P -> ModDown BConv onto own
+//   Q -> NTT with the fused tail (acc - conv) P^-1.
+// Gathers land directly in the BConv input layout ([digit][rank][B][rows][N]; BConv addresses a
+// limb by its owner and local index), so nothing is padded, concatenated or copied around them.
+// Transports: NCCL (ncclAllGather; libnccl.so.2 resolved with dlopen when the communicator is
+// created, so the library has no link-time NCCL dependency), or an in-process group of ranks on
+// one GPU (one host thread per rank; device-to-device copies after a host barrier) for tests.
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <chrono>
+#include <condition_variable>
+#include <mutex>
+
+namespace {
+struct NcclApi {
+    ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    const char* (*GetErrorString)(ncclResult_t) = nullptr;
+    bool ok = false;
+};
+const NcclApi& nccl_api() {
+    static NcclApi A = [] {
+        NcclApi a;
+        void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) return a;
+        a.GetUniqueId = reinterpret_cast<decltype(a.GetUniqueId)>(dlsym(h, "ncclGetUniqueId"));
+        a.CommInitRank = reinterpret_cast<decltype(a.CommInitRank)>(dlsym(h, "ncclCommInitRank"));
+        a.AllGather = reinterpret_cast<decltype(a.AllGather)>(dlsym(h, "ncclAllGather"));
+        a.CommDestroy = reinterpret_cast<decltype(a.CommDestroy)>(dlsym(h, "ncclCommDestroy"));
+        a.GetErrorString = reinterpret_cast<decltype(a.GetErrorString)>(dlsym(h, "ncclGetErrorString"));
+        a.ok = a.GetUniqueId && a.CommInitRank && a.AllGather && a.CommDestroy && a.GetErrorString;
+        return a;
+    }();
+    return A;
+}
+
+// in-process group: all-gather = publish (pointer + ready event), barrier, copy every peer's
+// block on the rank's communication stream, barrier, wait for every peer's copies to finish
+// reading this rank's block (so it may be overwritten by later work on its stream)
+struct LocalGroup {
+    int n;
+    std::mutex m;
+    std::condition_variable cv;
+    int arrived = 0;
+    long long gen = 0;
+    std::vector<const void*> send;
+    std::vector<cudaEvent_t> ready, done;
+    int refs = 0;
+    bool barrier() {                                   // false: a rank did not arrive within 120 s
+        std::unique_lock<std::mutex> lk(m);
+        const long long g = gen;
+        if (++arrived == n) {
+            arrived = 0;
+            ++gen;
+            cv.notify_all();
+            return true;
+        }
+        return cv.wait_for(lk, std::chrono::seconds(120), [&] { return gen != g; });
+    }
+};
+}  // namespace
+
+struct neo_comm {
+    const neo_ctx* ctx;
+    int nranks, rank;
+    ncclComm_t nccl = nullptr;
+    LocalGroup* local = nullptr;
+    cudaStream_t cs = nullptr;                         // communication stream
+    cudaEvent_t ev_prod = nullptr, ev_p = nullptr;
+    std::vector<cudaEvent_t> ev_gath;                // one per digit
+    // per level l: BConv tables for this rank's targets
+    std::vector<std::vector<neo::BConvTC>> up_tc;      // [l][j]: digit j -> mine \ D_j
+    std::vector<std::vector<size_t>> up_off;
+    std::vector<neo::BConvTC> down_tc;                 // [l]: P -> my Q limbs (empty if none)
+    std::vector<size_t> down_off;
+    uint8_t* d_bmat = nullptr;
+};
+
+namespace {
+struct ShardGeo {                                      // this rank's limbs at level l
+    int W, r, Lq, beta, alpha, P, maxd, maxp;
+    std::vector<int> my_q, my_p, mine;                 // limb ids (mine = my_q then my_p)
+    std::vector<std::vector<int>> dig_own;             // [j] my limbs of digit j
+};
+ShardGeo shard_geo(const neo_ctx* c, int W, int r, int l) {
+    ShardGeo g;
+    g.W = W; g.r = r; g.Lq = l + 1; g.beta = c->beta(l); g.alpha = c->alpha; g.P = c->num_p;
+    g.maxd = (c->alpha + W - 1) / W;
+    g.maxp = (c->num_p + W - 1) / W;
+    for (int i = r; i < g.Lq; i += W) g.my_q.push_back(i);
+    for (int k = r; k < g.P; k += W) g.my_p.push_back(c->num_q + k);
+    g.mine = g.my_q;
+    g.mine.insert(g.mine.end(), g.my_p.begin(), g.my_p.end());
+    g.dig_own.resize(g.beta);
+    for (int j = 0; j < g.beta; ++j)
+        for (int i : c->digits[l][j])
+            if (i % W == r) g.dig_own[j].push_back(i);
+    return g;
+}
+struct ShardLayout {
+    size_t ysend, yall, up, acc, psend, pall, conv, tmp, total;   // u64 offsets
+};
+ShardLayout shard_layout(const neo_ctx* c, const ShardGeo& g, int B) {
+    const size_t N = c->N, nm = g.mine.size(), nq = g.my_q.size();
+    ShardLayout L;
+    size_t o = 0;
+    L.ysend = o; o += (size_t)g.beta * B * g.maxd * N;
+    L.yall = o; o += (size_t)g.beta * g.W * B * g.maxd * N;
+    L.up = o; o += (size_t)B * g.beta * nm * N;
+    L.acc = o; o += (size_t)B * 2 * nm * N;
+    L.psend = o; o += (size_t)B * 2 * g.maxp * N;
+    L.pall = o; o += (size_t)g.W * B * 2 * g.maxp * N;
+    L.conv = o; o += (size_t)B * 2 * std::max<size_t>(nq, 1) * N;
+    L.tmp = o; o += (size_t)B * std::max<size_t>(std::max<size_t>((size_t)g.beta * nm, 2 * nq), 2 * g.my_p.size() + 1) * N;
+    L.total = o;
+    return L;
+}
+}  // namespace
+
+// all-gather of `bytes` per rank from send (this rank's block) into recv ([nranks][bytes]), on
+// the communication stream, after the work recorded in ev_prod on `st`; completion is recorded
+// in `done` (the compute stream waits on it before reading recv)
+static neo_status comm_allgather(const neo_comm* cm, const void* send, void* recv, size_t bytes, cudaStream_t st,
+                                 cudaEvent_t done) {
+    CK(cudaEventRecord(cm->ev_prod, st));
+    CK(cudaStreamWaitEvent(cm->cs, cm->ev_prod, 0));
+    if (cm->nranks == 1) {
+        if (recv != send) CK(cudaMemcpyAsync(recv, send, bytes, cudaMemcpyDeviceToDevice, cm->cs));
+    } else if (cm->nccl) {
+        ncclResult_t e = nccl_api().AllGather(send, recv, bytes, ncclUint8, cm->nccl, cm->cs);
+        if (e != ncclSuccess) FAIL(NEO_ENCCL, std::string("ncclAllGather: ") + nccl_api().GetErrorString(e));
+    } else {
+        LocalGroup* G = cm->local;
+        G->send[cm->rank] = send;
+        CK(cudaEventRecord(G->ready[cm->rank], cm->cs));
+        if (!G->barrier()) FAIL(NEO_ECUDA, "local group: a rank did not reach the exchange (barrier timeout)");
+        for (int s = 0; s < G->n; ++s) {
+            CK(cudaStreamWaitEvent(cm->cs, G->ready[s], 0));
+            CK(cudaMemcpyAsync(static_cast<char*>(recv) + (size_t)s * bytes, G->send[s], bytes,
+                               cudaMemcpyDeviceToDevice, cm->cs));
+        }
+        CK(cudaEventRecord(G->done[cm->rank], cm->cs));
+        if (!G->barrier()) FAIL(NEO_ECUDA, "local group: a rank did not reach the exchange (barrier timeout)");
+        for (int s = 0; s < G->n; ++s) CK(cudaStreamWaitEvent(cm->cs, G->done[s], 0));
+    }
+    CK(cudaEventRecord(done, cm->cs));
+    return NEO_OK;
+}
+
+static neo_status comm_tables(neo_comm* cm) {
+    const neo_ctx* c = cm->ctx;
+    std::vector<uint8_t> all, bm;
+    cm->up_tc.assign(c->num_q, {});
+    cm->up_off.assign(c->num_q, {});
+    cm->down_tc.assign(c->num_q, BConvTC{});
+    cm->down_off.assign(c->num_q, 0);
+    std::vector<u64> pm;
+    for (int k = 0; k < c->num_p; ++k) pm.push_back(c->mod[c->num_q + k]);
+    for (int l = 0; l < c->num_q; ++l) {
+        ShardGeo g = shard_geo(c, cm->nranks, cm->rank, l);
+        for (int j = 0; j < g.beta; ++j) {
+            const std::vector<int>& dj = c->digits[l][j];
+            std::vector<u64> sm, tm;
+            for (int id : dj) sm.push_back(c->mod[id]);
+            for (int t : g.mine)
+                if (std::find(dj.begin(), dj.end(), t) == dj.end()) tm.push_back(c->mod[t]);
+            BConvTC P;
+            std::memset(&P, 0, sizeof(P));
+            if (!tm.empty()) {
+                if ((int)tm.size() > BCTC_MAX_OUT) FAIL(NEO_EUNSUPPORTED, "too many ModUp targets per rank");
+                make_bconv_tc(sm, tm, P, bm);
+                cm->up_off[l].push_back(all.size());
+                all.insert(all.end(), bm.begin(), bm.end());
+            } else {
+                cm->up_off[l].push_back(0);
+            }
+            cm->up_tc[l].push_back(P);
+        }
+        if (!g.my_q.empty()) {
+            std::vector<u64> qm;
+            for (int i : g.my_q) qm.push_back(c->mod[i]);
+            make_bconv_tc(pm, qm, cm->down_tc[l], bm);
+            cm->down_off[l] = all.size();
+            all.insert(all.end(), bm.begin(), bm.end());
+        }
+    }
+    if (!all.empty()) {
+        CK(cudaMalloc(&cm->d_bmat, all.size()));
+        CK(cudaMemcpy(cm->d_bmat, all.data(), all.size(), cudaMemcpyHostToDevice));
+    }
+    return NEO_OK;
+}
+
+static neo_status comm_common(const neo_ctx* c, neo_comm* cm) {
+    if (!c->use_tc) FAIL(NEO_EUNSUPPORTED, "the limb-sharded key-switch needs the tensor-core BConv tables");
+    CK(cudaSetDevice(c->device));
+    CK(cudaStreamCreateWithFlags(&cm->cs, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&cm->ev_prod, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&cm->ev_p, cudaEventDisableTiming));
+    cm->ev_gath.assign(c->dnum, nullptr);
+    for (auto& e : cm->ev_gath) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    return comm_tables(cm);
+}
+
+extern "C" {
+
+neo_status neo_comm_unique_id(uint8_t uid[128]) {
+    if (!uid) FAIL(NEO_EINVAL, "null uid buffer");
+    const NcclApi& A = nccl_api();
+    if (!A.ok) FAIL(NEO_ENCCL, "libnccl.so.2 not found");
+    ncclUniqueId id;
+    ncclResult_t e = A.GetUniqueId(&id);
+    if (e != ncclSuccess) FAIL(NEO_ENCCL, std::string("ncclGetUniqueId: ") + A.GetErrorString(e));
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId is 128 bytes");
+    std::memcpy(uid, &id, 128);
+    return NEO_OK;
+}
+
+neo_status neo_comm_create(const neo_ctx* c, const uint8_t uid[128], int32_t nranks, int32_t rank, neo_comm** out) {
+    TRY(check_ctx(c));
+    if (!out || !uid) FAIL(NEO_EINVAL, "null argument");
+    *out = nullptr;
+    if (nranks < 1 || rank < 0 || rank >= nranks) FAIL(NEO_EINVAL, "need 0 <= rank < nranks");
+    std::unique_ptr<neo_comm> cm(new (std::nothrow) neo_comm());
+    if (!cm) FAIL(NEO_ENOMEM, "out of host memory");
+    cm->ctx = c; cm->nranks = nranks; cm->rank = rank;
+    TRY(comm_common(c, cm.get()));
+    if (nranks > 1) {
+        const NcclApi& A = nccl_api();
+        if (!A.ok) FAIL(NEO_ENCCL, "libnccl.so.2 not found");
+        ncclUniqueId id;
+        std::memcpy(&id, uid, 128);
+        ncclResult_t e = A.CommInitRank(&cm->nccl, nranks, id, rank);
+        if (e != ncclSuccess) FAIL(NEO_ENCCL, std::string("ncclCommInitRank: ") + A.GetErrorString(e));
+    }
+    *out = cm.release();
+    return NEO_OK;
+}
+
+neo_status neo_comm_create_local(const neo_ctx* c, int32_t nranks, neo_comm** comms) {
+    TRY(check_ctx(c));
+    if (!comms || nranks < 1 || nranks > 64) FAIL(NEO_EINVAL, "need 1 <= nranks <= 64 and an output array");
+    LocalGroup* G = new (std::nothrow) LocalGroup();
+    if (!G) FAIL(NEO_ENOMEM, "out of host memory");
+    G->n = nranks;
+    G->send.assign(nranks, nullptr);
+    G->ready.assign(nranks, nullptr);
+    G->done.assign(nranks, nullptr);
+    for (int r = 0; r < nranks; ++r) {
+        cudaEventCreateWithFlags(&G->ready[r], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&G->done[r], cudaEventDisableTiming);
+    }
+    for (int r = 0; r < nranks; ++r) {
+        comms[r] = nullptr;
+        neo_comm* cm = new (std::nothrow) neo_comm();
+        if (!cm) FAIL(NEO_ENOMEM, "out of host memory");
+        cm->ctx = c; cm->nranks = nranks; cm->rank = r; cm->local = G;
+        G->refs++;
+        comms[r] = cm;
+        neo_status s = comm_common(c, cm);
+        if (s) return s;
+    }
+    return NEO_OK;
+}
+
+neo_status neo_comm_destroy(neo_comm* cm) {
+    if (!cm) return NEO_OK;
+    if (cm->nccl) nccl_api().CommDestroy(cm->nccl);
+    if (cm->cs) cudaStreamDestroy(cm->cs);
+    if (cm->ev_prod) cudaEventDestroy(cm->ev_prod);
+    if (cm->ev_p) cudaEventDestroy(cm->ev_p);
+    for (auto e : cm->ev_gath)
+        if (e) cudaEventDestroy(e);
+    if (cm->d_bmat) cudaFree(cm->d_bmat);
+    if (cm->local && --cm->local->refs == 0) {
+        for (auto e : cm->local->ready) cudaEventDestroy(e);
+        for (auto e : cm->local->done) cudaEventDestroy(e);
+        delete cm->local;
+    }
+    delete cm;
+    return NEO_OK;
+}
+
+int32_t neo_comm_limbs(const neo_comm* cm, int32_t level, int32_t* q_ids, int32_t* p_ids, int32_t* n_p) {
+    if (!cm || level < 0 || level >= cm->ctx->num_q) return -1;
+    ShardGeo g = shard_geo(cm->ctx, cm->nranks, cm->rank, level);
+    if (q_ids) for (size_t i = 0; i < g.my_q.size(); ++i) q_ids[i] = g.my_q[i];
+    if (p_ids) for (size_t i = 0; i < g.my_p.size(); ++i) p_ids[i] = g.my_p[i];
+    if (n_p) *n_p = (int32_t)g.my_p.size();
+    return (int32_t)g.my_q.size();
+}
+
+size_t neo_workspace_size_sharded(const neo_comm* cm, int32_t level, int32_t batch) {
+    if (!cm || level < 0 || level >= cm->ctx->num_q || batch <= 0) return 0;
+    ShardGeo g = shard_geo(cm->ctx, cm->nranks, cm->rank, level);
+    return shard_layout(cm->ctx, g, batch).total * sizeof(u64);
+}
+
+neo_status neo_keyswitch_sharded(const neo_ctx* c, const neo_comm* cm, const neo_evk* k, const uint64_t* d_local,
+                                 int32_t level, uint64_t* out0, uint64_t* out1, int32_t batch, void* ws,
+                                 size_t ws_bytes, neo_stream_t stream) {
+    g_launches = 0;
+    TRY(check_ctx(c));
+    if (!cm || cm->ctx != c) FAIL(NEO_EINVAL, "communicator missing or from another context");
+    if (!k || k->ctx != c || k->klss || k->galois) FAIL(NEO_EINVAL, "Hybrid evaluation key missing or from another context");
+    if (level < 0 || level >= c->num_q) FAIL(NEO_EINVAL, "level out of range");
+    if (batch <= 0 || batch > 32) FAIL(NEO_EINVAL, "batch must be in [1, 32]");
+    const int l = level, B = batch, N = c->N;
+    ShardGeo g = shard_geo(c, cm->nranks, cm->rank, l);
+    const int nq = (int)g.my_q.size(), nm = (int)g.mine.size(), np = (int)g.my_p.size();
+    if (nq > 0) { TRY(check_ptr(d_local, "d_local")); TRY(check_ptr(out0, "out0")); TRY(check_ptr(out1, "out1")); }
+    ShardLayout Ly = shard_layout(c, g, B);
+    if (!ws || ws_bytes < Ly.total * sizeof(u64)) FAIL(NEO_EINVAL, "workspace smaller than neo_workspace_size_sharded");
+    cudaStream_t st = S(stream);
+    u64* W64 = static_cast<u64*>(ws);
+    u64 *ysend = W64 + Ly.ysend, *yall = W64 + Ly.yall, *up = W64 + Ly.up, *acc = W64 + Ly.acc;
+    u64 *psend = W64 + Ly.psend, *pall = W64 + Ly.pall, *conv = W64 + Ly.conv, *tmp = W64 + Ly.tmp;
+    if (g.W == 1) {                        // one rank: the gathered layouts are the send blocks
+        yall = ysend;
+        pall = psend;
+    }
+    int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
+    auto qpos = [&](int id) { return (int)(std::find(g.my_q.begin(), g.my_q.end(), id) - g.my_q.begin()); };
+    auto mpos = [&](int id) { return (int)(std::find(g.mine.begin(), g.mine.end(), id) - g.mine.begin()); };
+    int launches = 0;
+
+    // a3: INTT of the own Q limbs, ModUp's [d_i qhat_i^-1]_{q_i} folded in, straight into the
+    // send block of each limb's digit: ysend[j][b][u]
+    if (nq > 0) {
+        TWD sc[NEO_MAX_ROWS];
+        int n = 0;
+        for (int j = 0; j < g.beta; ++j)
+            for (size_t u = 0; u < g.dig_own[j].size(); ++u) {
+                const int id = g.dig_own[j][u];
+                const std::vector<int>& dj = c->digits[l][j];
+                so[n] = qpos(id);
+                dof[n] = j * B * g.maxd + (int)u;
+                pr[n] = id;
+                sc[n] = c->modup_tc[l][j].qhat_inv[std::find(dj.begin(), dj.end(), id) - dj.begin()];
+                ++n;
+            }
+        TRY(ntt_rows(c, false, d_local, (long long)nq * N, so, ysend, (long long)g.maxd * N, dof, pr, n, tmp, B, st,
+                     nullptr, false, sc));
+        launches += g_launches;
+    }
+    // exchange #1, one all-gather per digit on the communication stream
+    const size_t dbytes = (size_t)B * g.maxd * N * sizeof(u64);
+    for (int j = 0; j < g.beta; ++j)
+        TRY(comm_allgather(cm, ysend + (size_t)j * B * g.maxd * N, yall + (size_t)j * g.W * B * g.maxd * N, dbytes,
+                           st, cm->ev_gath[j]));
+    // a4/a5 per digit, as soon as its gather has landed
+    for (int j = 0; j < g.beta; ++j) {
+        CK(cudaStreamWaitEvent(st, cm->ev_gath[j], 0));
+        const BConvTC& P = cm->up_tc[l][j];
+        if (P.n_out == 0) continue;
+        const std::vector<int>& dj = c->digits[l][j];
+        BConvMulti M;
+        M.centred = 0; M.dbg = nullptr; M.njobs = 1; M.pre_scaled = 1; M.lazy_out = 1;
+        BConvIO io;
+        io.in = yall + (size_t)j * g.W * B * g.maxd * N;
+        io.out = up;
+        io.in_bstride = (long long)g.maxd * N;
+        io.out_bstride = (long long)g.beta * nm * N;
+        for (size_t i = 0; i < dj.size(); ++i) {
+            const int id = dj[i], w = id % g.W;
+            // local index of id among its owner's limbs of digit j
+            int u = 0;
+            for (int t : dj) if (t < id && t % g.W == w) ++u;
+            io.in_off[i] = w * B * g.maxd + u;
+        }
+        int n = 0;
+        for (int t : g.mine)
+            if (std::find(dj.begin(), dj.end(), t) == dj.end()) {
+                io.out_off[n] = j * nm + mpos(t);
+                so[n] = dof[n] = j * nm + mpos(t);
+                pr[n] = t;
+                ++n;
+            }
+        M.P[0] = P; M.io[0] = io; M.bmat[0] = cm->d_bmat + cm->up_off[l][j];
+        LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, B, c->num_sms, st));
+        ++launches;
+        TRY(ntt_rows(c, true, up, (long long)g.beta * nm * N, so, up, (long long)g.beta * nm * N, dof, pr, n, tmp, B,
+                     st, nullptr, true));
+        launches += g_launches;
+    }
+    // a6: KeyIP over the own limbs; a digit's own Q limbs are read from d_local
+    if (nm > 0) {
+        KeyIPArgs A;
+        A.galois = 0; A.accumulate = 0;
+        A.d = d_local ? d_local : up; A.up = up; A.evk_lo = k->lo; A.evk_hi = k->hi; A.acc = acc; A.mods = c->d_mods;
+        A.d_bstride = (long long)std::max(nq, 1) * N;
+        A.up_bstride = (long long)g.beta * nm * N;
+        A.acc_bstride = (long long)2 * nm * N;
+        A.acc_cstride = (long long)nm * N;
+        A.N = N; A.beta = g.beta; A.evk_limbs = c->num_q + c->num_p;
+        for (int pos = 0; pos < nm; ++pos) {
+            const int id = g.mine[pos];
+            A.limb[pos] = id;
+            for (int j = 0; j < g.beta; ++j) {
+                const std::vector<int>& dj = c->digits[l][j];
+                const bool own = std::find(dj.begin(), dj.end(), id) != dj.end();
+                A.src_kind[j][pos] = own ? 0 : 1;
+                A.src_off[j][pos] = own ? qpos(id) : j * nm + pos;
+            }
+        }
+        LAUNCH(PK_KEYIP, st, launch_keyip(A, nm, B, st));
+        ++launches;
+    }
+    // a7: INTT of the own P rows of acc (both components), P^_k^-1 folded, into the send block
+    if (np > 0) {
+        TWD sc[NEO_MAX_ROWS];
+        for (int u = 0; u < np; ++u) {
+            so[u] = nq + u;
+            dof[u] = u;
+            pr[u] = g.my_p[u];
+            sc[u] = c->moddown_tc[l].qhat_inv[g.my_p[u] - c->num_q];
+        }
+        TRY(ntt_rows(c, false, acc, (long long)nm * N, so, psend, (long long)g.maxp * N, dof, pr, np, tmp, 2 * B, st,
+                     nullptr, false, sc));
+        launches += g_launches;
+    }
+    // exchange #2
+    TRY(comm_allgather(cm, psend, pall, (size_t)2 * B * g.maxp * N * sizeof(u64), st, cm->ev_p));
+    CK(cudaStreamWaitEvent(st, cm->ev_p, 0));
+    if (nq == 0) {
+        g_launches = launches;
+        return NEO_OK;                                      // this rank owns P limbs only
+    }
+    // a8: ModDown BConv P -> own Q limbs, batch 2B
+    {
+        BConvMulti M;
+        M.centred = 0; M.dbg = nullptr; M.njobs = 1; M.pre_scaled = 1; M.lazy_out = 1;
+        BConvIO io;
+        io.in = pall; io.out = conv;
+        io.in_bstride = (long long)g.maxp * N;
+        io.out_bstride = (long long)nq * N;
+        for (int kk = 0; kk < g.P; ++kk) io.in_off[kk] = (kk % g.W) * 2 * B * g.maxp + kk / g.W;
+        for (int i = 0; i < nq; ++i) io.out_off[i] = i;
+        M.P[0] = cm->down_tc[l]; M.io[0] = io; M.bmat[0] = cm->d_bmat + cm->down_off[l];
+        LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, 2 * B, c->num_sms, st));
+        ++launches;
+    }
+    // a9 + a10: NTT of conv with the fused tail out_c = (acc_c - NTT(conv_c)) P^-1
+    for (int i = 0; i < nq; ++i) { so[i] = dof[i] = i; pr[i] = g.my_q[i]; }
+    RowEpi ep;
+    ep.acc = acc;
+    ep.acc_b = (long long)2 * nm * N;
+    ep.acc_c = (long long)nm * N;
+    ep.add0 = ep.add1 = nullptr;
+    ep.add_b = 0;
+    ep.add_galois = 0;
+    ep.out0 = out0; ep.out1 = out1;
+    ep.out_b = (long long)nq * N;
+    for (int i = 0; i < nq; ++i) ep.pinv[i] = c->pinv[g.my_q[i]];
+    TRY(ntt_rows(c, true, conv, (long long)nq * N, so, conv, (long long)nq * N, dof, pr, nq, tmp, 2 * B, st, &ep, true));
+    g_launches = launches + g_launches;
+    return NEO_OK;
+}
+
+}  // extern "C"

@@ -30,7 +30,9 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_debug_bconv_trace", "neo_double_rescale", "neo_pmult", "neo_hadd", "neo_padd",
             "neo_evk_create_klss", "neo_klss_query", "neo_profile_timeline", "neo_hsub", "neo_modraise",
             "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale", "neo_ew_limbs", "neo_hrot_sum",
-            "neo_ntt_select", "neo_ntt_selected")
+            "neo_ntt_select", "neo_ntt_selected", "neo_comm_unique_id", "neo_comm_create",
+            "neo_comm_create_local", "neo_comm_destroy", "neo_comm_limbs", "neo_workspace_size_sharded",
+            "neo_keyswitch_sharded")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -97,6 +99,11 @@ def lib() -> ctypes.CDLL:
             "neo_wire_unpack": [_vp, _vp, _vp, _sz, _vp],
             "neo_pmult_acc": [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), _i32, _i32, _i32, _vp, _i32, _vp],
             "neo_ntt_select": [_vp, _i32],
+            "neo_comm_unique_id": [_vp],
+            "neo_comm_create": [_vp, _vp, _i32, _i32, ctypes.POINTER(_vp)],
+            "neo_comm_create_local": [_vp, _i32, ctypes.POINTER(_vp)],
+            "neo_comm_destroy": [_vp],
+            "neo_keyswitch_sharded": [_vp, _vp, _vp, _vp, _i32, _vp, _vp, _i32, _vp, _sz, _vp],
             "neo_ntt_selected": [_vp],
         }
         for name, args in sig.items():
@@ -107,6 +114,11 @@ def lib() -> ctypes.CDLL:
             f.restype = ctypes.c_int
         L.neo_wire_bytes.argtypes = [_sz]
         L.neo_wire_bytes.restype = _sz
+        if hasattr(L, "neo_comm_limbs"):
+            L.neo_comm_limbs.argtypes = [_vp, _i32, _i32p, _i32p, _i32p]
+            L.neo_comm_limbs.restype = _i32
+            L.neo_workspace_size_sharded.argtypes = [_vp, _i32, _i32]
+            L.neo_workspace_size_sharded.restype = _sz
         L.neo_workspace_size.argtypes = [_vp, _i32, _i32, _i32]
         L.neo_workspace_size.restype = _sz
         L.neo_last_error.restype = ctypes.c_char_p
@@ -424,3 +436,66 @@ def neo_hrot_hoisted(ctx: Context, keys, ct_in, level: int, ct_out, batch: int, 
     arr = (ctypes.c_void_p * len(keys))(*[k.handle.value for k in keys])
     _check(lib().neo_hrot_hoisted(ctx.handle, arr, len(keys), _ptr(ct_in), level, _ptr(ct_out), batch, _ptr(ws),
                                   ws.numel() * 8, _stream(stream)), "neo_hrot_hoisted")
+
+
+class Comm:
+    """A limb-sharded key-switching communicator (neo_comm_create / neo_comm_create_local)."""
+
+    def __init__(self, ctx: Context, handle):
+        self.ctx, self.handle = ctx, handle
+
+    @staticmethod
+    def unique_id() -> bytes:
+        """neo_comm_unique_id: the 128-byte NCCL unique id rank 0 distributes."""
+        buf = (ctypes.c_uint8 * 128)()
+        _check(lib().neo_comm_unique_id(buf), "neo_comm_unique_id")
+        return bytes(buf)
+
+    @classmethod
+    def create(cls, ctx: Context, uid: bytes, nranks: int, rank: int) -> "Comm":
+        buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
+        h = ctypes.c_void_p()
+        _check(lib().neo_comm_create(ctx.handle, buf, nranks, rank, ctypes.byref(h)), "neo_comm_create")
+        return cls(ctx, h)
+
+    @classmethod
+    def create_local(cls, ctx: Context, nranks: int) -> list:
+        arr = (ctypes.c_void_p * nranks)()
+        _check(lib().neo_comm_create_local(ctx.handle, nranks, arr), "neo_comm_create_local")
+        return [cls(ctx, ctypes.c_void_p(arr[r])) for r in range(nranks)]
+
+    def limbs(self, level: int):
+        """(Q limb ids, P limb ids) this rank owns at `level` (neo_comm_limbs)."""
+        q = (ctypes.c_int32 * 64)()
+        p = (ctypes.c_int32 * 64)()
+        n_p = ctypes.c_int32()
+        nq = lib().neo_comm_limbs(self.handle, level, q, p, ctypes.byref(n_p))
+        if nq < 0:
+            raise NeoError(1, "neo_comm_limbs", "invalid level")
+        return list(q)[:nq], list(p)[: n_p.value]
+
+    def workspace(self, level: int, batch: int, device="cuda") -> torch.Tensor:
+        n = int(lib().neo_workspace_size_sharded(self.handle, level, batch))
+        if n == 0:
+            raise NeoError(1, "neo_workspace_size_sharded", "invalid level/batch")
+        return torch.empty(n // 8, dtype=torch.uint64, device=device)
+
+    def close(self):
+        if self.handle:
+            lib().neo_comm_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def neo_keyswitch_sharded(ctx: Context, comm: Comm, evk: EvalKey, d_local, level: int, out0, out1, batch: int, ws,
+                          stream=None):
+    """One key-switch of this rank's Q limbs (d_local [batch][nq][N]); out0/out1 [batch][nq][N].
+    A rank without Q limbs passes None for d_local / out0 / out1."""
+    nb = ws.numel() * 8
+    _check(lib().neo_keyswitch_sharded(ctx.handle, comm.handle, evk.handle, _ptr(d_local), level, _ptr(out0),
+                                       _ptr(out1), batch, _ptr(ws), nb, _stream(stream)), "neo_keyswitch_sharded")
