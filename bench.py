@@ -895,7 +895,7 @@ def run_neo(args):
                 t_ = float(t.item())
             return t_
 
-        def boot_case(nb, rb, fl, sharded):
+        def boot_case(nb, rb, fl, sharded, boost=(0, 0), ds_sq=0):
             """Time one bootstrap configuration: eager and as a CUDA-graph replay (output checked
             equal), and optionally the limb-sharded form over all ranks (graph, NCCL)."""
             keys = {"relin": neo.EvalKey(ctx, evk_b)}
@@ -903,8 +903,8 @@ def run_neo(args):
                 keys[gg] = neo.EvalKey(ctx, evk_b)
             for gg in gboot.hoisted_rotations(N, nb, fl):
                 keys[("h", gg)] = neo.EvalKey(ctx, evk_b, hoisted_galois=gg)
-            consts = {k: rnd(l + 1, N) for k, l in gboot.const_levels(LEVEL, nb, rb, N, fl).items()}
-            bt = gboot.Bootstrapper(ctx, nb, rb, keys, consts, fft_levels=fl)
+            consts = {k: rnd(l + 1, N) for k, l in gboot.const_levels(LEVEL, nb, rb, N, fl, boost, ds_sq).items()}
+            bt = gboot.Bootstrapper(ctx, nb, rb, keys, consts, fft_levels=fl, boost=boost, ds_sq=ds_sq)
             for _ in range(2):
                 bt.run(bct)
             torch.cuda.synchronize()
@@ -922,13 +922,14 @@ def run_neo(args):
             best = gms if gms is not None else eager
             out = {"ms_per_bootstrap": round(best, 3), "value": world / (best / 1e3), "unit": "bootstraps/s",
                    "graph": gms is not None, "ms_eager": round(eager, 3),
-                   "levels": f"{LEVEL} -> {LEVEL - gboot.levels_used(rb, fl)}",
+                   "levels": f"{LEVEL} -> {LEVEL - gboot.levels_used(rb, fl, boost, ds_sq)}", "boost": list(boost),
+                   "ds_squarings": ds_sq,
                    "rotation_keys": len(gboot.rotations(N, nb, fl)) + len(gboot.hoisted_rotations(N, nb, fl))}
             if sharded:
                 # config 4's multi-GPU form: the same bootstrap limb-sharded over all ranks
                 # (round-robin limbs; two all-gathers per key-switch, one limb broadcast per
                 # Rescale; NCCL).  At N = 1 the sharded code path runs on one rank.
-                sbt = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, fft_levels=fl)
+                sbt = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, fft_levels=fl, boost=boost, ds_sq=ds_sq)
                 sct0 = sbt.shard(bct, 0)
                 sref = sbt.run(sct0)[0].clone()
                 # graph capture only on one rank: a capture that failed on some ranks mid-way
@@ -937,7 +938,8 @@ def run_neo(args):
                 sgraph = sg_out = sbt_g = None
                 if world == 1:
                     s_side = torch.cuda.Stream()
-                    sbt_g = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, stream=s_side, fft_levels=fl)
+                    sbt_g = ShardedBootstrapper(ctx, nb, rb, keys, consts, world, rank, stream=s_side, fft_levels=fl,
+                                                boost=boost, ds_sq=ds_sq)
                     sgraph, sg_out = graph_capture(lambda: sbt_g.run(sct0)[0], side=s_side)
                 if sgraph is not None:
                     sgraph.replay()
@@ -954,9 +956,9 @@ def run_neo(args):
             torch.cuda.empty_cache()
             return out
 
-        full = boot_case(N // 2, 12, 4, sharded=True)
+        full = boot_case(N // 2, 9, 4, sharded=True, boost=(20, 20), ds_sq=4)     # oracle.boot.set_b_full()
         sparse = boot_case(8, 12, 0, sharded=False)
-        boot_block = dict(full, config="Set-B (N=2^16, L=35, dnum=3), full slots (32768), r=12 squarings, "
+        boot_block = dict(full, config="Set-B (N=2^16, L=35, dnum=3), full slots (32768), r=9 squarings (4 at ~q^2 scale, Double Rescale), "
                                        "CoeffToSlot / SlotToCoeff as 4 special-FFT BSGS levels each (stages 4-4-4-3)",
                           timing="CUDA events around 5 graph replays (3 eager runs) after warm-ups, max over "
                                  "ranks; replay output checked equal to the eager run; keys / constants synthetic",

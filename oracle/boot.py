@@ -25,6 +25,7 @@ uses the same ones (tests/test_gpu_boot.py: bit-exact).  Pinned by decoding (the
 decrypts to the input slots) and by ModRaise's exact big-integer identity."""
 from __future__ import annotations
 
+import collections
 import math
 from dataclasses import dataclass
 
@@ -42,6 +43,8 @@ class BootParams:
     r: int                                   # squarings in EvalMod
     h: int = 192                             # secret Hamming weight (bounds I)
     fft_levels: int = 0                      # 0: dense diagonal method; k: factored CtS / StC, k levels each
+    boost: tuple = (0, 0)                    # (k1, k2): exact x 2^k scale boosts before CoeffToSlot / SlotToCoeff
+    ds_sq: int = 0                           # EvalMod at ~q^2 (Double Rescale) up to this many squarings (< r)
 
     @property
     def M(self) -> int:
@@ -51,9 +54,12 @@ class BootParams:
     def top(self) -> int:
         return self.prm.max_level
 
-    def levels_used(self) -> int:            # CtS, EvalMod 1 + 3 + 1 + r + 1, StC
+    def levels_used(self) -> int:            # CtS, EvalMod 1 + 3 + 1 + r + 1, StC (+ the Double Rescales)
         lt = max(1, self.fft_levels)
-        return lt + (1 + 3 + 1 + self.r + 1) + lt
+        extra = 1 if (self.boost[0] or self.ds_sq) else 0            # theta
+        if self.ds_sq:
+            extra += 3 + 1 + self.ds_sq + 2                          # powers, Taylor terms, squarings, 3-prime one
+        return lt + (1 + 3 + 1 + self.r + 1) + lt + extra
 
     def rotations(self) -> list[int]:
         """Galois elements: SubSum (rotations by n 2^j), the linear transforms' rotations, conj."""
@@ -78,10 +84,28 @@ def tiny_full(fft_levels: int = 3) -> BootParams:
                       fft_levels=fft_levels)
 
 
+def tiny_full_boost() -> BootParams:
+    """tiny_full(4) with the reading-BOOT-S scale boosts (2^12) and theta's Double Rescale:
+    N = 2^12, 26 Q + 3 P limbs (dnum 9), output level 1 (its 72-bit modulus holds the
+    2^12-boosted output scale; the GPU replays it bit for bit)."""
+    return BootParams(ckks.Params(12, 26, 3, 9), n=2048, r=9, h=32, fft_levels=4, boost=(12, 12))
+
+
+def tiny_full_ds() -> BootParams:
+    """The reading-BOOT-S schedule Set-B runs with, at N = 2^12: 2^12 boosts, EvalMod at ~q^2 (Double
+    Rescale) for the theta product, the Taylor powers and terms and the first 4 of r = 9 squarings;
+    37 Q + 4 P limbs (dnum 10), output level 2."""
+    return BootParams(ckks.Params(12, 37, 4, 10), n=2048, r=9, h=32, fft_levels=4, boost=(12, 12), ds_sq=4)
+
+
 def set_b_full() -> BootParams:
-    """Set-B with all N/2 = 32768 slots, r = 12, CtS / StC as 4 levels of 4-4-4-3 special-FFT
-    stages (levels 35 -> 9)."""
-    return BootParams(ckks.set_b(), n=32768, r=12, h=192, fft_levels=4)
+    """Set-B with all N/2 = 32768 slots, CtS / StC as 4 levels of 4-4-4-3 special-FFT stages, and
+    reading BOOT-S: 2^20 scale boosts before both linear transforms, EvalMod with r = 9 squarings
+    whose theta product, Taylor powers and terms and first 4 squarings run at ~q^2 scale with
+    Double Rescales (L138, L151: what keeps 36-bit words precise) -- levels 35 -> 1.  With
+    single-prime rescales throughout (r = 12) the key-switch and rescale noise at ~2^36 scale,
+    amplified 2^r by the squarings, swamps the message (decode error ~1, tools/boot_setb_diag.py)."""
+    return BootParams(ckks.set_b(), n=32768, r=9, h=192, fft_levels=4, boost=(20, 20), ds_sq=4)
 
 
 def tiny() -> BootParams:
@@ -107,12 +131,37 @@ def _diagonals(A: np.ndarray) -> list[np.ndarray]:
     return [np.array([A[k][(k + d) % n] for k in range(n)]) for d in range(n)]
 
 
+def _round_big(scale: float, x: float) -> int:
+    """round(scale x), half away from zero, exactly in integers for any float scale (the product
+    of two doubles is formed exactly from their integer mantissas)."""
+    from fractions import Fraction
+    y = Fraction(scale) * Fraction(x)
+    r = abs(y).__floor__() + (1 if abs(y) - abs(y).__floor__() >= Fraction(1, 2) else 0)
+    return r if y >= 0 else -r
+
+
 def _pt(bp: BootParams, slots_n: np.ndarray, scale: float, level: int) -> np.ndarray:
-    """Plaintext (NTT form, level) whose full-slot vector is slots_n tiled, at `scale`."""
+    """Plaintext (NTT form, level) whose full-slot vector is slots_n tiled, at `scale`.  A
+    constant vector c is encoded in closed form, m = round(scale Re c) + round(scale Im c) X^(N/2)
+    (X^(N/2) is i in every slot; encode()'s sum is zero at every other coefficient), which is
+    encode()'s result without its O(N^2) sum (pinned equal in tests/test_oracle_boot.py)."""
     prm = bp.prm
     ids = list(range(level + 1))
-    m = ckks.encode(prm.N, np.tile(np.asarray(slots_n, dtype=complex), bp.M), scale)
+    v = np.asarray(slots_n, dtype=complex)
+    if np.all(v == v[0]):
+        m = np.zeros(prm.N, dtype=object)                                  # scales up to ~2^110: Python ints
+        m[:] = 0
+        m[0] = _round_big(scale, v[0].real)
+        m[prm.N // 2] = _round_big(scale, v[0].imag)
+    else:
+        m = ckks.encode(prm.N, np.tile(v, bp.M), scale)
     return ckks.ntt(prm, ckks.reduce_signed(prm, m, ids), ids)
+
+
+def _const_int(prm: ckks.Params, c: int, level: int) -> np.ndarray:
+    """NTT form of the constant polynomial c (an exact integer plaintext: PMULT by it multiplies
+    the message by c without a Rescale)."""
+    return np.stack([np.full(prm.N, c % prm.moduli[i], dtype=np.uint64) for i in range(level + 1)])
 
 
 def _monomial(prm: ckks.Params, k: int, sign: int, level: int) -> np.ndarray:
@@ -248,6 +297,32 @@ def _lintrans_bsgs(prm, ct, lv, diags: dict, name: str, keys: dict, const):
     return ckks.rescale(prm, acc, lv)
 
 
+def _lintrans_plain(prm, ct, lv, diags: dict, keys: dict):
+    """The textbook diagonal method (reading BOOT-P): sum_d diag_d (.) rot_d(ct) with one separate
+    HROTATE per diagonal amount d and one PMULT per diagonal at scale q_lv, then Rescale -- no
+    hoisting, no baby-step giant-step split, no shared ModDown.  The reference the GPU's schedule
+    (hoisted baby steps, BOOT-H; giant steps summed before one ModDown, BOOT-G) is checked
+    against by decryption (tests/test_oracle_boot.py, tests/test_gpu_boot.py)."""
+    N, n = prm.N, prm.N // 2
+    acc = None
+    for d in sorted(diags):
+        r = ct if d % n == 0 else ckks.hrot(prm, ct, pow(5, d % n, 2 * N), lv, keys[pow(5, d % n, 2 * N)])
+        t = ckks.pmult(prm, r, _pt_full(prm, diags[d], float(prm.q[lv]), lv), lv)
+        acc = t if acc is None else ckks.hadd(prm, acc, t, lv)
+    return ckks.rescale(prm, acc, lv)
+
+
+def plain_rotations(bp: "BootParams") -> list[int]:
+    """Galois elements the plain (textbook) schedule needs beyond bp.rotations(): one per
+    diagonal amount of every merged CoeffToSlot / SlotToCoeff group."""
+    N = bp.prm.N
+    gs = set()
+    if bp.fft_levels:
+        for grp in fft_groups(N, bp.fft_levels, inverse=True) + fft_groups(N, bp.fft_levels, inverse=False):
+            gs |= {pow(5, d % (N // 2), 2 * N) for d in grp if d % (N // 2)}
+    return sorted(gs - set(bp.rotations()))
+
+
 def moddown(prm: ckks.Params, acc: np.ndarray, level: int) -> tuple:
     """Steps a7-a10 of the key-switch (Table 2, Z9) on a KeyIP output acc [2][E][N] (PQ_l,
     NTT form): (acc_c[Q] - NTT(BConv_{P->Q}(INTT(acc_c[P])))) P^-1."""
@@ -283,13 +358,18 @@ def hrot_sum(prm: ckks.Params, cts: list, gs: list, level: int, rotkeys: list) -
     return np.stack([ckks.add(prm, c0, k0, ids), k1])
 
 
-def fft_transform(bp: BootParams, ct: np.ndarray, lv: int, keys: dict, inverse: bool, tag: str, const=None):
+def fft_transform(bp: BootParams, ct: np.ndarray, lv: int, keys: dict, inverse: bool, tag: str, const=None,
+                  plain: bool = False):
     """CoeffToSlot (inverse=True: slots <- P U^-1 slots) or SlotToCoeff (slots <- U P^-1 slots)
     as bp.fft_levels BSGS levels from level lv.  Returns (ct, lv - fft_levels).  `const(name,
-    make)` supplies / records the plaintext diagonals (default: encode on the fly)."""
+    make)` supplies / records the plaintext diagonals (default: encode on the fly).  plain: the
+    textbook diagonal method per level (_lintrans_plain)."""
     const = const or (lambda name, make: make())
     for k, grp in enumerate(fft_groups(bp.prm.N, bp.fft_levels, inverse)):
-        ct = _lintrans_bsgs(bp.prm, ct, lv, grp, f"{tag}{k}", keys, const)
+        if plain:
+            ct = _lintrans_plain(bp.prm, ct, lv, grp, keys)
+        else:
+            ct = _lintrans_bsgs(bp.prm, ct, lv, grp, f"{tag}{k}", keys, const)
         lv -= 1
     return ct, lv
 
@@ -325,20 +405,26 @@ def drop(ct: np.ndarray, level: int) -> np.ndarray:
 
 # --------------------------------------------------------------------------- keys
 
-def boot_keys(bp: BootParams, s: np.ndarray, seed: int) -> dict:
-    """Hybrid evaluation keys: 'relin' and one rotation key per Galois element of bp.rotations()."""
+def boot_keys(bp: BootParams, s: np.ndarray, seed: int, plain: bool = False) -> dict:
+    """Hybrid evaluation keys: 'relin' and one rotation key per Galois element of bp.rotations()
+    (plain: also the textbook schedule's extra rotations, plain_rotations(bp))."""
     keys = {"relin": ckks.relin_key(bp.prm, s, seed)}
-    for t, g in enumerate(bp.rotations()):
+    gs = bp.rotations() + (plain_rotations(bp) if plain else [])
+    for t, g in enumerate(gs):
         keys[g] = ckks.rot_key(bp.prm, s, g, seed + 1 + t)
     return keys
 
 
 # --------------------------------------------------------------------------- bootstrapping
 
-def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None = None):
+def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None = None, plain: bool = False,
+              stop_after_cts: bool = False):
     """Bootstrap ct0 ([2][1][N], level 0).  Returns (ct, level, scale, consts) where the output
     decodes (at `scale` Delta_in / q_0) to the input's slots.  `consts` (plaintexts by name) are
-    generated when None and returned, so another implementation can replay the same run."""
+    generated when None and returned, so another implementation can replay the same run.
+    plain: the textbook schedule (separate HROTATEs, dense diagonal sums; reading BOOT-P) for
+    both linear transforms -- the reference the GPU's hoisted / BOOT-G schedule is checked
+    against by decryption.  stop_after_cts: return right after CoeffToSlot (ct, level, scale)."""
     prm, N, n, M = bp.prm, bp.prm.N, bp.n, bp.M
     gen = consts is None
     consts = {} if gen else consts
@@ -360,13 +446,25 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
     for j in range(int(math.log2(M))):
         ct = ckks.hadd(prm, ct, rot(ct, pow(5, n << j, 2 * N), L), L)
 
+    # reading BOOT-S: an exact x 2^k1 (PMULT by the integer constant, no level) raises the scale of
+    # the ModRaised ciphertext before CoeffToSlot, so the key-switch noise its rotations add is
+    # 2^k1 smaller relative to the message (at Set-B, full slots, it otherwise swamps it)
+    k1, k2 = bp.boost
+    if k1:
+        ct = ckks.pmult(prm, ct, const("boost_cts", lambda: _const_int(prm, 1 << k1, L)), L)
+        scale *= float(1 << k1)
+
     def lintrans_fft(ct, lv, inverse, tag):   # factored: fft_levels levels, BSGS per level
-        return fft_transform(bp, ct, lv, keys, inverse, tag, const)
+        return fft_transform(bp, ct, lv, keys, inverse, tag, const, plain=plain)
 
     def lintrans(ct, lv, A, tag):        # slots <- A slots (diagonal method), scale kept, one level
-        # the n - 1 rotations of the same ciphertext are hoisted (one ModUp, reading BOOT-H)
+        # the n - 1 rotations of the same ciphertext are hoisted (one ModUp, reading BOOT-H);
+        # plain: n - 1 separate HROTATEs
         gs = [pow(5, d, 2 * N) for d in range(1, n)]
-        rots = [ct] + list(ckks.hrot_hoisted(prm, ct, gs, lv, [keys[g] for g in gs]))
+        if plain:
+            rots = [ct] + [rot(ct, g, lv) for g in gs]
+        else:
+            rots = [ct] + list(ckks.hrot_hoisted(prm, ct, gs, lv, [keys[g] for g in gs]))
         acc = None
         for d, dg in enumerate(_diagonals(A)):
             pt = const(f"{tag}_{d}", lambda dg=dg: _pt(bp, dg, float(q[lv]), lv))
@@ -381,16 +479,32 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
         W = _xi_matrix(n)
         ct = lintrans(ct, L, np.linalg.inv(W) / M, "cts")          # CoeffToSlot
         lv = L - 1
+    if stop_after_cts:
+        return ct, lv, scale, consts
     cj = rot(ct, 2 * N - 1, lv)
     x1 = ckks.hadd(prm, ct, cj, lv)                                 # 2 Re(w)
     x2 = ckks.pmult(prm, hsub(prm, ct, cj, lv), const("mono_mi", lambda: _monomial(prm, N // 2, -1, lv)), lv)  # 2 Im(w)
-    sx = 2.0 * scale                                                # value Re(w), Im(w) at scale 2 q_0
+    sx = 2.0 * scale                                                # value Re(w), Im(w) at scale 2 q_0 (x 2^k1)
+
+    ds = bp.ds_sq                     # reading BOOT-S: EvalMod's first steps at scale ~q^2 (Double Rescale)
+
+    def rs(ct, lv, m):                # divide by m primes: Rescale (1), Double Rescale (2, L138), both (3)
+        if m == 1:
+            return ckks.rescale(prm, ct, lv)
+        ct = ckks.double_rescale(prm, ct, lv)
+        return ckks.rescale(prm, ct, lv - 2) if m == 3 else ct
+
+    def qq(lv, m):                    # the product of the m primes rs() divides by
+        return math.prod(float(q[lv - i]) for i in range(m))
 
     def evalmod(x, lv, sx, tag):
         theta = 2 * math.pi / (1 << bp.r)
-        S = float(q[lv])                                            # y's scale after the theta product
-        y1 = ckks.rescale(prm, ckks.pmult(prm, x, const(f"{tag}theta", lambda: _pt(bp, np.full(n, theta), S * q[lv] / sx, lv)), lv), lv)
-        lv -= 1
+        m = 2 if ds else 1                                          # primes per rescale while at q^2
+        S = qq(lv, m) if ds else float(q[lv])                       # y's scale after the theta product
+        m_th = 2 if (k1 or ds) else 1   # a boosted input needs q_lv q_lv-1 for theta to keep ~52 bits
+        y1 = rs(ckks.pmult(prm, x, const(f"{tag}theta", lambda: _pt(bp, np.full(n, theta), S * qq(lv, m_th) / sx, lv)),
+                           lv), lv, m_th)
+        lv -= m_th
         sc = {1: S}
         pw = {1: (y1, lv)}
 
@@ -398,8 +512,8 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
             (ca, la), (cb, lb) = pw[a], pw[b]
             l0 = min(la, lb)
             prod = ckks.hmult(prm, drop(ca, l0), drop(cb, l0), l0, keys["relin"])
-            pw[a + b] = (ckks.rescale(prm, prod, l0), l0 - 1)
-            sc[a + b] = sc[a] * sc[b] / q[l0]
+            pw[a + b] = (rs(prod, l0, m), l0 - m)
+            sc[a + b] = sc[a] * sc[b] / qq(l0, m)
         mul(1, 1)
         mul(2, 1)
         mul(2, 2)
@@ -407,21 +521,23 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
         mul(4, 2)
         mul(4, 3)
         lt = min(pw[k][1] for k in pw)                              # common level of the terms
-        St = float(q[lt])                                           # their common scale
+        St = qq(lt, m)                                              # their common scale
         E = None
         for k in range(1, D_TAYLOR + 1):
             ck, lk = pw[k]
             coef = (1j ** k) / math.factorial(k)
-            pt = const(f"{tag}c{k}", lambda coef=coef, lk=lk, k=k: _pt(bp, np.full(n, coef), St * q[lk] / sc[k], lk))
-            term = drop(ckks.rescale(prm, ckks.pmult(prm, ck, pt, lk), lk), lt - 1)
-            E = term if E is None else ckks.hadd(prm, E, term, lt - 1)
-        lv = lt - 1
+            pt = const(f"{tag}c{k}", lambda coef=coef, lk=lk, k=k: _pt(bp, np.full(n, coef), St * qq(lk, m) / sc[k], lk))
+            term = drop(rs(ckks.pmult(prm, ck, pt, lk), lk, m), lt - m)
+            E = term if E is None else ckks.hadd(prm, E, term, lt - m)
+        lv = lt - m
         E = ckks.padd(prm, E, const(f"{tag}c0", lambda: _pt(bp, np.ones(n), St, lv)), lv)
         s_e = St
-        for _ in range(bp.r):                                       # E <- E^2: exp(2 pi i t)
-            E = ckks.rescale(prm, ckks.hmult(prm, E, E, lv, keys["relin"]), lv)
-            s_e = s_e * s_e / q[lv]
-            lv -= 1
+        for i in range(bp.r):                                       # E <- E^2: exp(2 pi i t)
+            # ds squarings at ~q^2, then one dividing by 3 primes back to ~q, then single ones
+            mi = (2 if i < ds else 3 if i == ds else 1) if ds else 1
+            E = rs(ckks.hmult(prm, E, E, lv, keys["relin"]), lv, mi)
+            s_e = s_e * s_e / qq(lv, mi)
+            lv -= mi
         cE = rot(E, 2 * N - 1, lv)
         Dm = hsub(prm, E, cE, lv)                                   # 2 i sin(2 pi t)
         k = -1j / (4 * math.pi)
@@ -433,6 +549,9 @@ def bootstrap(bp: BootParams, ct0: np.ndarray, keys: dict, consts: dict | None =
     assert (lv1, s1) == (lv2, s2)
     lv = lv1
     w = ckks.hadd(prm, f1, ckks.pmult(prm, f2, const("mono_i", lambda: _monomial(prm, N // 2, 1, lv)), lv), lv)
+    if k2:                                                          # the same boost before SlotToCoeff
+        w = ckks.pmult(prm, w, const("boost_stc", lambda: _const_int(prm, 1 << k2, lv)), lv)
+        s1 *= float(1 << k2)
     if bp.fft_levels:
         out, lo = lintrans_fft(w, lv, False, "stc")                 # SlotToCoeff
         return out, lo, s1, consts
@@ -449,3 +568,43 @@ def encrypt_sparse(bp: BootParams, z: np.ndarray, delta: float, s: np.ndarray, s
 def decode_sparse(bp: BootParams, ct: np.ndarray, level: int, scale: float, s: np.ndarray) -> np.ndarray:
     m = ckks.crt_centered(bp.prm, ckks.decrypt_residues(bp.prm, ct, s, level), list(range(level + 1)))
     return ckks.decode(bp.prm.N, m, scale)[: bp.n]
+
+
+def make_consts(bp: BootParams) -> dict:
+    """The plaintext constants bootstrap(bp, ...) generates (see dry_run)."""
+    return dry_run(bp)[2]
+
+
+def dry_run(bp: BootParams) -> tuple:
+    """(output level, output scale, plaintext constants) of bootstrap(bp, ...), without its ciphertext arithmetic:
+    the schedule's levels and scales are data-independent, so the run is replayed with every
+    ciphertext operation replaced by a shape-preserving stand-in (used to give the GPU the real
+    constants at Set-B, where running the oracle's bootstrap itself would take hours)."""
+    N = bp.prm.N
+    z = lambda L: np.zeros((2, L + 1, N), dtype=np.uint64)
+    lim = lambda ct, lv: np.ascontiguousarray(ct[:, : lv + 1])
+    stand_in = {
+        "hrot": lambda prm, ct, g, lv, key: ct,
+        "hrot_hoisted": lambda prm, ct, gs, lv, keys: [ct] * len(gs),
+        "hmult": lambda prm, a, b, lv, relin, mode="fast": a,
+        "pmult": lambda prm, ct, pt, lv: ct,
+        "hadd": lambda prm, a, b, lv: a,
+        "padd": lambda prm, ct, pt, lv: ct,
+        "rescale": lambda prm, ct, lv, mode="fast": lim(ct, lv - 1),
+        "double_rescale": lambda prm, ct, lv, mode="fast": lim(ct, lv - 2),
+    }
+    saved_ckks = {k: getattr(ckks, k) for k in stand_in}
+    g = globals()
+    saved_boot = {k: g[k] for k in ("modraise", "hrot_sum", "hsub")}
+    try:
+        for k, f in stand_in.items():
+            setattr(ckks, k, f)
+        g["modraise"] = lambda prm, ct, L: z(L)
+        g["hrot_sum"] = lambda prm, cts, gs, lv, keys: cts[0]
+        g["hsub"] = lambda prm, a, b, lv: a
+        _, lv, scale, consts = bootstrap(bp, z(0), collections.defaultdict(lambda: None))
+    finally:
+        for k, f in saved_ckks.items():
+            setattr(ckks, k, f)
+        g.update(saved_boot)
+    return lv, scale, consts

@@ -19,9 +19,19 @@ from . import neo
 D_TAYLOR = 7
 
 
-def levels_used(r: int, fft_levels: int = 0) -> int:
+def levels_used(r: int, fft_levels: int = 0, boost: tuple = (0, 0), ds_sq: int = 0) -> int:
     lt = max(1, fft_levels)
-    return lt + (1 + 3 + 1 + r + 1) + lt
+    extra = 1 if (boost[0] or ds_sq) else 0                  # theta's Double Rescale
+    if ds_sq:
+        extra += 3 + 1 + ds_sq + 2                           # powers, Taylor terms, squarings, the 3-prime one
+    return lt + (1 + 3 + 1 + r + 1) + lt + extra
+
+
+def _sq_primes(i: int, ds_sq: int) -> int:
+    """Primes the i-th EvalMod squaring divides by: 2 while at ~q^2, 3 once to return to ~q, then 1."""
+    if not ds_sq:
+        return 1
+    return 2 if i < ds_sq else 3 if i == ds_sq else 1
 
 
 # ---- full-slot linear transforms (n = N/2): the special FFT's log2(n) butterfly stages, stage
@@ -84,26 +94,36 @@ def _fft_const_names(N: int, fft_levels: int, inverse: bool, tag: str) -> list[l
     return out
 
 
-def const_levels(top: int, n: int, r: int, N: int = 0, fft_levels: int = 0) -> dict:
+def const_levels(top: int, n: int, r: int, N: int = 0, fft_levels: int = 0, boost: tuple = (0, 0),
+                 ds_sq: int = 0) -> dict:
     """Level of every plaintext constant (the same schedule as run())."""
     F = max(1, fft_levels)
     if fft_levels:
         lv = {nm: top - k for k, names in enumerate(_fft_const_names(N, fft_levels, True, "cts")) for nm in names}
     else:
         lv = {f"cts_{d}": top for d in range(n)}
+    if boost[0]:
+        lv["boost_cts"] = top
     l1 = top - F
     lv["mono_mi"] = l1
+    m = 2 if ds_sq else 1                                   # primes per rescale while EvalMod is at ~q^2
+    m_th = 2 if (boost[0] or ds_sq) else 1                  # theta's product ends in a Double Rescale
     for tag in ("re", "im"):
         lv[f"{tag}theta"] = l1
-        y = l1 - 1                                          # y^1 level
-        lk = {1: y, 2: y - 1, 3: y - 2, 4: y - 2, 5: y - 3, 6: y - 3, 7: y - 3}
+        pw = {1: l1 - m_th}                                 # y^k levels
+        for a, b in ((1, 1), (2, 1), (2, 2), (4, 1), (4, 2), (4, 3)):
+            pw[a + b] = min(pw[a], pw[b]) - m
         for k in range(1, D_TAYLOR + 1):
-            lv[f"{tag}c{k}"] = lk[k]
-        lt = y - 3
-        lv[f"{tag}c0"] = lt - 1
-        lv[f"{tag}sin"] = lt - 1 - r
-    lf = l1 - (1 + 3 + 1 + r + 1)
+            lv[f"{tag}c{k}"] = pw[k]
+        le = min(pw.values()) - m
+        lv[f"{tag}c0"] = le
+        for i in range(r):
+            le -= _sq_primes(i, ds_sq)
+        lv[f"{tag}sin"] = le
+    lf = lv["resin"] - 1
     lv["mono_i"] = lf
+    if boost[1]:
+        lv["boost_stc"] = lf
     if fft_levels:
         for k, names in enumerate(_fft_const_names(N, fft_levels, False, "stc")):
             lv.update({nm: lf - k for nm in names})
@@ -126,13 +146,15 @@ class Bootstrapper:
     (neo_evk_create_hoisted) for g in hoisted_rotations(N, n)}; consts: {name: tensor}."""
 
     def __init__(self, ctx: neo.Context, n: int, r: int, keys: dict, consts: dict, stream=None,
-                 fft_levels: int = 0):
+                 fft_levels: int = 0, boost: tuple = (0, 0), ds_sq: int = 0):
         self.ctx, self.n, self.r, self.keys, self.consts, self.stream = ctx, n, r, keys, consts, stream
         self.fft_levels = fft_levels
+        self.boost = tuple(boost)
+        self.ds_sq = ds_sq
         self.N = ctx.N
         self.top = ctx.num_q - 1
         ops = (neo.NEO_OP_HMULT, neo.NEO_OP_HROT, neo.NEO_OP_RESCALE, neo.NEO_OP_MODRAISE, neo.NEO_OP_HROT_HOISTED,
-               neo.NEO_OP_HMULT_RESCALE, neo.NEO_OP_HROT_SUM)
+               neo.NEO_OP_HMULT_RESCALE, neo.NEO_OP_HROT_SUM, neo.NEO_OP_DOUBLE_RESCALE)
         wsn = max(ctx.workspace_size(op, self.top, 2) for op in ops)
         self._stack = {}
         self.ws = torch.empty(wsn // 8, dtype=torch.uint64, device="cuda")
@@ -181,6 +203,11 @@ class Bootstrapper:
     def rescale(self, a, lv):
         out = self._ct(lv - 1, a.shape[0])
         neo.neo_rescale(self.ctx, a, lv, out, a.shape[0], self.ws, self.stream)
+        return out
+
+    def double_rescale(self, a, lv):
+        out = self._ct(lv - 2, a.shape[0])
+        neo.neo_double_rescale(self.ctx, a, lv, out, a.shape[0], self.ws, self.stream)
         return out
 
     def hmul(self, a, b, lv):
@@ -270,6 +297,9 @@ class Bootstrapper:
         for j in range(int(math.log2(M))):                             # SubSum
             ct = self.add(ct, self.rot(ct, pow(5, n << j, 2 * N), L), L)
         lintrans = self.lintrans
+        k1, k2 = self.boost
+        if k1:                                                         # exact x 2^k1 (reading BOOT-S)
+            ct = self.pmul(ct, "boost_cts", L)
 
         if self.fft_levels:
             ct, lv = self.lintrans_fft(ct, L, True, "cts")             # CoeffToSlot (bit-reversed)
@@ -281,28 +311,42 @@ class Bootstrapper:
         self.add(ct, cj, lv, out=xs[0:1])                               # 2 Re(w)
         self.pmul(self.sub(ct, cj, lv), "mono_mi", lv, out=xs[1:2])     # 2 Im(w)
 
+        ds = self.ds_sq
+
+        def rs(ct, lv, m):             # Rescale (1), Double Rescale (2), both (3) -- the oracle's rs()
+            if m == 1:
+                return self.rescale(ct, lv)
+            ct = self.double_rescale(ct, lv)
+            return self.rescale(ct, lv - 2) if m == 3 else ct
+
         def evalmod(x, lv, tags):
-            y1 = self.rescale(self.pmul(x, [f"{t}theta" for t in tags], lv), lv)
-            lv -= 1
+            m = 2 if ds else 1
+            m_th = 2 if (k1 or ds) else 1                              # theta: Double Rescale
+            y1 = rs(self.pmul(x, [f"{t}theta" for t in tags], lv), lv, m_th)
+            lv -= m_th
             pw = {1: (y1, lv)}
 
             def mul(a, b):
                 (ca, la), (cb, lb) = pw[a], pw[b]
                 l0 = min(la, lb)
-                pw[a + b] = (self.hmul_rescale(self.drop(ca, la, l0), self.drop(cb, lb, l0), l0), l0 - 1)
+                if m == 1:
+                    pw[a + b] = (self.hmul_rescale(self.drop(ca, la, l0), self.drop(cb, lb, l0), l0), l0 - 1)
+                else:
+                    pw[a + b] = (rs(self.hmul(self.drop(ca, la, l0), self.drop(cb, lb, l0), l0), l0, m), l0 - m)
             for a, b in ((1, 1), (2, 1), (2, 2), (4, 1), (4, 2), (4, 3)):
                 mul(a, b)
             lt = min(l for _, l in pw.values())
             E = None
             for k in range(1, D_TAYLOR + 1):
                 ck, lk = pw[k]
-                term = self.drop(self.rescale(self.pmul(ck, [f"{t}c{k}" for t in tags], lk), lk), lk - 1, lt - 1)
-                E = term if E is None else self.add(E, term, lt - 1)
-            lv = lt - 1
+                term = self.drop(rs(self.pmul(ck, [f"{t}c{k}" for t in tags], lk), lk, m), lk - m, lt - m)
+                E = term if E is None else self.add(E, term, lt - m)
+            lv = lt - m
             E = self.padd(E, [f"{t}c0" for t in tags], lv)
-            for _ in range(self.r):
-                E = self.hmul_rescale(E, E, lv)
-                lv -= 1
+            for i in range(self.r):
+                mi = _sq_primes(i, ds)
+                E = self.hmul_rescale(E, E, lv) if mi == 1 else rs(self.hmul(E, E, lv), lv, mi)
+                lv -= mi
             cE = self.rot(E, 2 * N - 1, lv)
             f = self.rescale(self.pmul(self.sub(E, cE, lv), [f"{t}sin" for t in tags], lv), lv)
             return f, lv - 1
@@ -310,6 +354,8 @@ class Bootstrapper:
         # EvalMod of the real and imaginary halves as one batch of 2
         f, lv = evalmod(xs, lv, ("re", "im"))
         w = self.add(f[0:1], self.pmul(f[1:2], "mono_i", lv), lv)
+        if k2:
+            w = self.pmul(w, "boost_stc", lv)
         if self.fft_levels:
             return self.lintrans_fft(w, lv, False, "stc")              # SlotToCoeff
         out = lintrans(w, lv, "stc")                                   # SlotToCoeff

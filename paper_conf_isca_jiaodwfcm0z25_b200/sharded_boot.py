@@ -29,9 +29,11 @@ class ShardedBootstrapper(Bootstrapper):
     consts: full plaintexts [l+1][N] (each rank keeps its own rows)."""
 
     def __init__(self, ctx: neo.Context, n: int, r: int, keys: dict, consts: dict, world: int, rank: int,
-                 group=None, stream=None, fft_levels: int = 0):
+                 group=None, stream=None, fft_levels: int = 0, boost: tuple = (0, 0), ds_sq: int = 0):
         self.ctx, self.n, self.r, self.keys, self.stream = ctx, n, r, keys, stream
         self.fft_levels = fft_levels
+        self.boost = tuple(boost)
+        self.ds_sq = ds_sq
         self.N = ctx.N
         self.top = ctx.num_q - 1
         self.world, self.rank = world, rank
@@ -54,6 +56,11 @@ class ShardedBootstrapper(Bootstrapper):
     def shard(self, ct_full: torch.Tensor, level: int) -> torch.Tensor:
         """This rank's rows of a full ciphertext [B][2][level+1][N]."""
         return ct_full.view(torch.int64)[:, :, self.own(level)].contiguous().view(torch.uint64)
+
+    def double_rescale(self, a, lv):
+        """Double Rescale as two sharded Rescales (bit-identical: floor(floor(x/a)/b) = floor(x/ab),
+        pinned in test_oracle_ops.py)."""
+        return self.rescale(self.rescale(a, lv), lv - 1)
 
     def _ks(self, d_local, lv, key):
         plan = ShardPlan(lv, self.ctx.num_q, self.ctx.num_p, self.ctx.alpha, self.world, self.rank, strided=True)

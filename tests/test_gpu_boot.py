@@ -74,11 +74,12 @@ def test_bootstrap_graph_replay_bit_exact():
     assert glv == lv and np.array_equal(out.cpu().numpy()[0], want)
 
 
-@pytest.mark.parametrize("fft_levels", [3, 4])
+@pytest.mark.parametrize("fft_levels", [3, 4, "boost", "ds"])
 def test_full_slot_bootstrap_bit_exact_and_decodes(fft_levels):
     """All N/2 slots: factored CoeffToSlot / SlotToCoeff (3 BSGS levels each, hoisted baby steps,
-    fused PMULT sums) + EvalMod, bit-exact vs oracle/boot.py and decoding to the input."""
-    bp = boot.tiny_full(fft_levels)
+    fused PMULT sums) + EvalMod, bit-exact vs oracle/boot.py and decoding to the input; "boost":
+    the reading-BOOT-S schedule (2^12 scale boosts, theta's Double Rescale) Set-B runs with."""
+    bp = {"boost": boot.tiny_full_boost, "ds": boot.tiny_full_ds}.get(fft_levels, lambda: boot.tiny_full(fft_levels))()
     prm = bp.prm
     s = ckks.secret(prm, 51, bp.h)
     keys_np = boot.boot_keys(bp, s, 600)
@@ -88,12 +89,13 @@ def test_full_slot_bootstrap_bit_exact_and_decodes(fft_levels):
     want, lv, scale, consts = boot.bootstrap(bp, ct0, keys_np)
     ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
     assert gboot.rotations(prm.N, bp.n, bp.fft_levels) == bp.rotations()
-    cl = gboot.const_levels(bp.top, bp.n, bp.r, prm.N, bp.fft_levels)
+    cl = gboot.const_levels(bp.top, bp.n, bp.r, prm.N, bp.fft_levels, bp.boost, bp.ds_sq)
     assert set(cl) == set(consts) and all(consts[k].shape[0] == cl[k] + 1 for k in cl)
     keys = {k: neo.EvalKey(ctx, dev(v)) for k, v in keys_np.items()}
     for g in gboot.hoisted_rotations(prm.N, bp.n, bp.fft_levels):
         keys[("h", g)] = neo.EvalKey(ctx, dev(keys_np[g]), hoisted_galois=g)
-    b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()}, fft_levels=bp.fft_levels)
+    b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()}, fft_levels=bp.fft_levels,
+                           boost=bp.boost, ds_sq=bp.ds_sq)
     got, glv = b.run(dev(ct0[None]))
     torch.cuda.synchronize()
     assert glv == lv
@@ -101,3 +103,74 @@ def test_full_slot_bootstrap_bit_exact_and_decodes(fft_levels):
     assert np.array_equal(got, want)
     zz = boot.decode_sparse(bp, got, lv, scale * delta / prm.q[0], s)
     assert np.max(np.abs(zz - z)) < 1e-2          # test_oracle_boot.py: sqrt(N) slot gain
+
+
+def test_gpu_schedule_vs_plain_oracle_by_decryption():
+    """The GPU's schedule (hoisted baby steps, BOOT-H; one ModDown per giant-step group, BOOT-G)
+    against the TEXTBOOK oracle schedule (separate HROTATEs, dense diagonal sums; reading BOOT-P)
+    on the same input: both decrypt to the input slots, and to each other within twice the
+    decode gate (the two differ only in key-switch / rescale rounding, which EvalMod's 2^r
+    squarings amplify -- test_oracle_boot.py pins the CoeffToSlot stage to a Z9-derived bound)."""
+    bp = boot.tiny()
+    prm = bp.prm
+    s = ckks.secret(prm, 21, bp.h)
+    keys_np = boot.boot_keys(bp, s, 500, plain=True)
+    z = synth.complex_slots(23, bp.n)
+    delta = 2.0 ** 31
+    ct0 = boot.encrypt_sparse(bp, z, delta, s, 25)
+    lv, scale, consts = boot.dry_run(bp)
+    ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+    keys = {k: neo.EvalKey(ctx, dev(v)) for k, v in keys_np.items()}
+    for g in gboot.hoisted_rotations(prm.N, bp.n):
+        keys[("h", g)] = neo.EvalKey(ctx, dev(keys_np[g]), hoisted_galois=g)
+    b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()})
+    got, glv = b.run(dev(ct0[None]))
+    torch.cuda.synchronize()
+    assert glv == lv
+    zg = boot.decode_sparse(bp, got.cpu().numpy()[0], lv, scale * delta / prm.q[0], s)
+    plain, lp, sp, _ = boot.bootstrap(bp, ct0, keys_np, plain=True)
+    zp = boot.decode_sparse(bp, plain, lp, sp * delta / prm.q[0], s)
+    assert np.max(np.abs(zg - z)) < 4e-3 and np.max(np.abs(zp - z)) < 4e-3
+    assert np.max(np.abs(zg - zp)) < 8e-3
+
+
+def _decode_sample(prm, ct, level, scale, s, js):
+    """decode() restricted to slots js: z_j = m(zeta^(5^j)) / scale (its definition, per slot)."""
+    m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, ct, s, level), list(range(level + 1)))
+    mf = np.array([float(v) for v in m])
+    N = prm.N
+    e = np.array([pow(5, int(j), 2 * N) for j in js], dtype=np.int64)
+    k = np.arange(N, dtype=np.int64)
+    return np.array([np.exp(1j * np.pi * ((ej * k) % (2 * N)) / N) @ mf for ej in e]) / scale
+
+
+@pytest.mark.slow
+def test_set_b_full_slot_bootstrap_decodes():
+    """The configuration bench.py times (oracle.boot.set_b_full: Set-B, all 32768 slots, CoeffToSlot /
+    SlotToCoeff as 4 BSGS levels, EvalMod r = 9 with its first steps at ~q^2 via Double Rescale,
+    levels 35 -> 1) with real keys and the schedule's real constants (oracle.boot.dry_run): the
+    output decrypts to the input slots (256 sampled slots)."""
+    bp = boot.set_b_full()
+    prm = bp.prm
+    s = ckks.secret(prm, 61, bp.h)
+    keys_np = boot.boot_keys(bp, s, 700)
+    lv, scale, consts = boot.dry_run(bp)
+    z = synth.complex_slots(63, prm.N // 2)
+    delta = 2.0 ** 31
+    ct0 = ckks.encrypt(prm, ckks.encode_fft(prm.N, z, delta), s, 0, 65)
+    ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+    keys = {k: neo.EvalKey(ctx, dev(v)) for k, v in keys_np.items()}
+    for g in gboot.hoisted_rotations(prm.N, bp.n, bp.fft_levels):
+        keys[("h", g)] = neo.EvalKey(ctx, dev(keys_np[g]), hoisted_galois=g)
+    b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()}, fft_levels=bp.fft_levels,
+                           boost=bp.boost, ds_sq=bp.ds_sq)
+    got, glv = b.run(dev(ct0[None]))
+    torch.cuda.synchronize()
+    assert glv == lv == 1
+    js = np.random.default_rng(7).choice(prm.N // 2, 256, replace=False)
+    zz = _decode_sample(prm, got.cpu().numpy()[0], lv, scale * delta / prm.q[0], s, js)
+    err = np.max(np.abs(zz - z[js]))
+    print(f"Set-B full-slot bootstrap: max slot error {err:.3e} over {len(js)} sampled slots")
+    # measured 2.0e-3 (r02); single-prime rescales throughout gave ~1 (EvalMod's 2^12 amplification
+    # of ~2^-36-relative key-switch / rescale noise).  1e-2: the tiny full-slot gate.
+    assert err < 1e-2

@@ -40,6 +40,9 @@ def test_xi_matrix_maps_subring_coefficients_to_slots():
     assert np.max(np.abs(boot._xi_matrix(n) @ w - z)) < 1e-9
 
 
+_RUN = {}
+
+
 @pytest.fixture(scope="module")
 def booted():
     bp = boot.tiny()
@@ -49,6 +52,7 @@ def booted():
     delta = 2.0 ** 31
     ct0 = boot.encrypt_sparse(bp, z, delta, s, 25)
     out, lv, scale, consts = boot.bootstrap(bp, ct0, keys)
+    _RUN["sparse"] = consts
     return bp, s, z, delta, out, lv, scale
 
 
@@ -193,3 +197,129 @@ def test_hrot_sum_pins():
     m = ckks.crt_centered(prm, ckks.decrypt_residues(prm, out, s, L), list(range(L + 1)))
     want = sum(np.roll(z, -r) for z, r in zip(zs, (1, 3, 7)))
     assert np.max(np.abs(ckks.decode(prm.N, m, delta) - want)) < 1e-6
+
+
+# --------------------------------------------------------------------------- plain vs schedule
+# The GPU replays oracle/boot.py's schedule bit for bit (tests/test_gpu_boot.py): hoisted baby
+# rotations (BOOT-H), giant steps summed before one ModDown (BOOT-G), baby-step giant-step
+# levels.  These tests pin that schedule to the textbook one (reading BOOT-P: separate HROTATEs,
+# dense diagonal sums) by decryption, so a performance choice in the schedule cannot silently
+# change what is computed.
+#
+# Derived bound at the CoeffToSlot output.  Both schedules compute the same linear map; they
+# differ only in rounding: the key noise terms of a rotation are identical (sigma commutes with
+# the digit decomposition), so each key-switch contributes at most its ModDown floor rounding,
+# ||e||_inf <= (K+2)(1+h) (Z9, pinned in test_oracle_ks.py), and each Rescale its floor rounding
+# <= 1 + h; a coefficient error e becomes a slot error <= ||e||_1 <= N ||e||_inf, multiplied by
+# the largest diagonal entry it is later scaled with (D_max) and divided by the ciphertext scale
+# q_0.  Summing over every key-switch and Rescale of both runs gives B_cts below.
+
+def _cts_bound(bp, n_ks, n_rs, dmax):
+    prm = bp.prm
+    e_ks = (prm.num_p + 1) * (1 + bp.h)
+    return prm.N * (n_ks * e_ks * dmax + n_rs * (1 + bp.h)) / prm.q[0]
+
+
+def _slot_values(bp, ct, lv, s):
+    """Decrypt + decode at scale q_0 (the CoeffToSlot output's value scale), all N/2 slots."""
+    m = ckks.crt_centered(bp.prm, ckks.decrypt_residues(bp.prm, ct, s, lv), list(range(lv + 1)))
+    return ckks.decode(bp.prm.N, m, float(bp.prm.q[0]))
+
+
+def test_plain_vs_schedule_sparse(booted):
+    bp, s, z, delta, out, lv, scale = booted
+    keys = boot.boot_keys(bp, s, 500, plain=True)
+    ct0 = boot.encrypt_sparse(bp, z, delta, s, 25)
+    # CoeffToSlot stage: hoisted n - 1 rotations vs n - 1 separate HROTATEs
+    a, la, _, _ = boot.bootstrap(bp, ct0, keys, stop_after_cts=True)
+    b, lb, _, _ = boot.bootstrap(bp, ct0, keys, plain=True, stop_after_cts=True)
+    assert la == lb
+    dmax = np.max(np.abs(np.linalg.inv(boot._xi_matrix(bp.n)) / bp.M))
+    B = _cts_bound(bp, 2 * (bp.n - 1), 2, dmax)
+    diff = np.max(np.abs(_slot_values(bp, a, la, s) - _slot_values(bp, b, lb, s)))
+    assert diff <= B, (diff, B)
+    # whole bootstrap: both decode to the input (test_bootstrap_decodes_to_input's gate)
+    p, lp, sp, _ = boot.bootstrap(bp, ct0, keys, plain=True)
+    assert (lp, sp) == (lv, scale)
+    assert np.max(np.abs(boot.decode_sparse(bp, p, lp, sp * delta / bp.prm.q[0], s) - z)) < 4e-3
+
+
+@pytest.mark.slow
+def test_plain_vs_schedule_full_slot():
+    """Full slots, 3 factored levels per transform: BSGS + hoisting + shared giant-step ModDown
+    against one HROTATE and one PMULT per diagonal."""
+    bp = boot.tiny_full(3)
+    prm = bp.prm
+    s = ckks.secret(prm, 51, bp.h)
+    keys = boot.boot_keys(bp, s, 600, plain=True)
+    z = synth.complex_slots(53, prm.N // 2)
+    delta = 2.0 ** 31
+    ct0 = boot.encrypt_sparse(bp, z, delta, s, 55)
+    a, la, _, _ = boot.bootstrap(bp, ct0, keys, stop_after_cts=True)
+    b, lb, _, _ = boot.bootstrap(bp, ct0, keys, plain=True, stop_after_cts=True)
+    assert la == lb
+    groups = boot.fft_groups(prm.N, bp.fft_levels, inverse=True)
+    n_ks = sum(len(g) for g in groups) * 2            # >= the key-switches of either schedule
+    dmax = max(np.max(np.abs(v)) for g in groups for v in g.values())
+    B = _cts_bound(bp, n_ks, 2 * len(groups), max(1.0, dmax))
+    diff = np.max(np.abs(_slot_values(bp, a, la, s) - _slot_values(bp, b, lb, s)))
+    assert diff <= B, (diff, B)
+    p, lp, sp, _ = boot.bootstrap(bp, ct0, keys, plain=True)
+    assert np.max(np.abs(boot.decode_sparse(bp, p, lp, sp * delta / prm.q[0], s) - z)) < 1e-2
+
+
+def test_constant_plaintext_closed_form():
+    """_pt's closed form for a constant slot vector c (round(D Re c) + round(D Im c) X^(N/2)) equals
+    encode()'s O(N^2) definition, for the constants and scales bootstrapping uses."""
+    bp = boot.tiny()
+    prm = bp.prm
+    rng = np.random.default_rng(9)
+    for scale in (2.0 ** 20, 2.0 ** 36, float(prm.q[3]) * 3.7):
+        c = complex(rng.standard_normal(), rng.standard_normal())
+        lv = 4
+        ids = list(range(lv + 1))
+        want = ckks.ntt(prm, ckks.reduce_signed(prm, ckks.encode(prm.N, np.full(prm.N // 2, c), scale), ids), ids)
+        assert np.array_equal(boot._pt(bp, np.full(bp.n, c), scale, lv), want)
+
+
+def test_make_consts_matches_a_real_run(booted):
+    """make_consts (the schedule replayed without arithmetic) gives the constants a real run makes."""
+    bp, s, z, delta, out, lv, scale = booted
+    real = _RUN.get("sparse")
+    dlv, dscale, dry = boot.dry_run(bp)
+    assert (dlv, dscale) == (lv, scale)
+    if real is None:
+        real = boot.bootstrap(bp, boot.encrypt_sparse(bp, z, delta, s, 25), boot.boot_keys(bp, s, 500))[3]
+    assert set(dry) == set(real) and all(np.array_equal(dry[k], real[k]) for k in real)
+
+
+def test_boosted_full_slot_bootstrap_decodes():
+    """Reading BOOT-S (exact x 2^k scale boosts before both linear transforms, theta's product as a
+    Double Rescale, L138): the same full-slot bootstrap decodes, at least as accurately as without
+    (the boosts shrink the key-switch noise relative to the message; EvalMod's noise remains)."""
+    bp = boot.tiny_full_boost()
+    prm = bp.prm
+    s = ckks.secret(prm, 51, bp.h)
+    keys = boot.boot_keys(bp, s, 600)
+    z = synth.complex_slots(53, prm.N // 2)
+    delta = 2.0 ** 31
+    out, lv, scale, _ = boot.bootstrap(bp, boot.encrypt_sparse(bp, z, delta, s, 55), keys)
+    assert lv == bp.top - bp.levels_used() == 1
+    assert np.max(np.abs(boot.decode_sparse(bp, out, lv, scale * delta / prm.q[0], s) - z)) < 1e-2
+
+
+def test_ds_evalmod_bootstrap_decodes():
+    """Reading BOOT-S with EvalMod's theta product, Taylor powers and terms and first 4 squarings at
+    ~q^2 scale (Double Rescale, L138/L151), the schedule Set-B runs with, at N = 2^12."""
+    bp = boot.tiny_full_ds()
+    prm = bp.prm
+    s = ckks.secret(prm, 51, bp.h)
+    keys = boot.boot_keys(bp, s, 600)
+    z = synth.complex_slots(53, prm.N // 2)
+    delta = 2.0 ** 31
+    out, lv, scale, _ = boot.bootstrap(bp, boot.encrypt_sparse(bp, z, delta, s, 55), keys)
+    assert lv == bp.top - bp.levels_used() == 2
+    # 1e-3 (the single-scale schedule's gate is 1e-2, measured 5.0e-3; this one measures 1.8e-4: the
+    # noise EvalMod amplifies now enters at ~2^72 scale, what remains is the last 4 squarings' and
+    # the sine's noise at ~2^36, amplified at most 2^4)
+    assert np.max(np.abs(boot.decode_sparse(bp, out, lv, scale * delta / prm.q[0], s) - z)) < 1e-3
