@@ -351,11 +351,23 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         // tail below becomes ((acc_i - NTT(conv_i)) P^-1 + d_i) q_l^-1 = Rescale(HMULT) exactly.
         u64* accl = hmr_last;
         u64* dl = hmr_last + (size_t)2 * B * N;
-        so[0] = l; so[1] = E + l; dof[0] = 0; dof[1] = 1; pr[0] = pr[1] = l;
-        if ((s = ntt_rows(c, false, acc, (long long)2 * E * N, so, accl, (long long)2 * N, dof, pr, 2, tmp, B, st)))
-            return s;
-        so[1] = (int)(add1 - add0) / N + l;
-        if ((s = ntt_rows(c, false, add0, add_bs, so, dl, (long long)2 * N, dof, pr, 2, tmp, B, st))) return s;
+        // the 4 rows acc_0,l acc_1,l d_0,l d_1,l of every batch entry in ONE inverse transform
+        // (rows addressed from the lower of the two workspace buffers; batch entries as rows)
+        {
+            const u64* base = std::min<const u64*>(acc, add0);
+            const long long oa = (acc - base) / N, od = (add0 - base) / N, d1 = (add1 - add0) / N;
+            int n = 0;
+            for (int b = 0; b < B; ++b)
+                for (int cc = 0; cc < 2; ++cc) {
+                    so[n] = (int)(oa + (long long)b * 2 * E + (long long)cc * E + l);
+                    dof[n] = 2 * b + cc;
+                    pr[n++] = l;
+                    so[n] = (int)(od + (long long)b * (add_bs / N) + cc * d1 + l);
+                    dof[n] = 2 * B + 2 * b + cc;
+                    pr[n++] = l;
+                }
+            if ((s = ntt_rows(c, false, base, 0, so, hmr_last, 0, dof, pr, n, tmp, 1, st))) return s;
+        }
         HmrFoldArgs F;
         F.conv = conv; F.accl = accl; F.dl = dl; F.mods = c->d_mods;
         F.pinv_l = c->pinv[l];
