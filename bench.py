@@ -957,7 +957,7 @@ def run_neo(args):
             return out
 
         full = boot_case(N // 2, 9, 4, sharded=True, boost=(20, 20), ds_sq=4)     # oracle.boot.set_b_full()
-        sparse = boot_case(8, 12, 0, sharded=False)
+        sparse = boot_case(8, 9, 0, sharded=False, boost=(20, 20), ds_sq=4)    # oracle.boot.set_b()
         boot_block = dict(full, config="Set-B (N=2^16, L=35, dnum=3), full slots (32768), r=9 squarings (4 at ~q^2 scale, Double Rescale), "
                                        "CoeffToSlot / SlotToCoeff as 4 special-FFT BSGS levels each (stages 4-4-4-3)",
                           timing="CUDA events around 5 graph replays (3 eager runs) after warm-ups, max over "
@@ -982,12 +982,14 @@ def run_neo(args):
         f_h, B_h, C_c, H_c = 256, 8, 16, 32
         baby, giant = gapps.conv_rotations(C_c, H_c)
         akeys = {"relin": neo.EvalKey(ctx, evk_r)}
-        for r in gapps.helr_rotations(N, f_h) + giant:
+        pool_r, fc_r = gapps.head_rotations(C_c, H_c)
+        for r in gapps.helr_rotations(N, f_h) + giant + pool_r:
             akeys.setdefault(gapps.galois(N, r), neo.EvalKey(ctx, evk_r))
-        for r in baby:
-            akeys[("h", gapps.galois(N, r))] = neo.EvalKey(ctx, evk_r, hoisted_galois=gapps.galois(N, r))
+        for r in baby + fc_r:
+            akeys.setdefault(("h", gapps.galois(N, r)), neo.EvalKey(ctx, evk_r, hoisted_galois=gapps.galois(N, r)))
         del evk_r
-        aconsts = {k: rnd(LEVEL + 1, N) for k in gapps.helr_const_names() + gapps.conv_const_names(C_c)}
+        aconsts = {k: rnd(LEVEL + 1, N) for k in gapps.helr_const_names() + gapps.conv_const_names(C_c)
+                   + gapps.block_const_names(C_c) + gapps.head_const_names(C_c)}
         aev = gapps.Evaluator(ctx, akeys, aconsts, max_batch=B_h)
         Zc, Wc, Xc = rnd(B_h, 2, LEVEL + 1, N), rnd(1, 2, LEVEL + 1, N), rnd(1, 2, LEVEL + 1, N)
 
@@ -1024,8 +1026,10 @@ def run_neo(args):
             return out
         hms_e, hms_g = timed(lambda: gapps.helr_iteration(aev, f_h, Zc, Wc, LEVEL)[0], 3)
         cms_e, cms_g = timed(lambda: gapps.conv_layer(aev, C_c, H_c, Xc, LEVEL)[0], 3)
+        bms_e, bms_g = timed(lambda: gapps.head(aev, C_c, H_c, *gapps.basic_block(aev, C_c, H_c, Xc, LEVEL))[0], 3)
         hms = hms_g if hms_g is not None else hms_e
         cms = cms_g if cms_g is not None else cms_e
+        bms = bms_g if bms_g is not None else bms_e
         lf, lr = int(math.log2(f_h)), int(math.log2(N // 2 // f_h))
         apps_block = {
             "helr_iteration": {
@@ -1040,6 +1044,13 @@ def run_neo(args):
                 "graph": cms_g is not None, "ms_eager": round(cms_e, 3),
                 "ops": {"hrot": len(baby) + len(giant), "hmult": 2, "pmult_terms": 9 * C_c + 3},
                 "paper_context": "Table 5: Neo 12.03 s for all of ResNet-20 incl. bootstrapping, Set-C, A100 (context only)"},
+            "resnet20_block_and_head": {
+                "config": "Set-B, l=35 -> 25: a stride-1 basic block (conv, ReLU, conv, + shortcut, ReLU) at 16 x 32 x 32, "
+                          "then global average pooling (10 rotate-and-sum HROT) and a 16 -> 16 fully connected layer",
+                "ms": round(bms, 3), "value": world / (bms / 1e3), "unit": "block+head/s", "graph": bms_g is not None,
+                "ms_eager": round(bms_e, 3),
+                "ops": {"hrot": 2 * (len(baby) + len(giant)) + len(pool_r) + len(fc_r), "hmult": 4,
+                        "pmult_terms": 2 * (9 * C_c + 3) + 1 + C_c}},
             "timing": "CUDA events around 3 graph replays (headline) and 3 eager runs after warm-ups, max over "
                       "ranks; replay output checked equal to the eager run; synthetic keys/constants"}
         del akeys, aconsts, aev, Zc, Wc, Xc

@@ -272,12 +272,12 @@ def conv_diag(sh: ConvShape, w: np.ndarray, d: int, dy: int, dx: int) -> np.ndar
     return np.tile(v, sh.N // 2 // v.size)
 
 
-def conv_layer(sh: ConvShape, prm: ckks.Params, X, w: np.ndarray, bias: np.ndarray, keys: dict,
-               consts: dict | None = None):
-    """X = (ct, level, scale).  Returns (out, consts, counts); out at level - 4, X's scale."""
-    ev = Ev(prm, keys, consts)
+def _conv(sh: ConvShape, ev: Ev, X, w: np.ndarray, bias: np.ndarray, pre: str = ""):
+    """Steps 1-3: 3x3 convolution (hoisted baby steps, baby-step giant-step diagonal method),
+    Rescale, bias.  One level; the output keeps X's scale."""
+    prm = ev.prm
     C, H, half = sh.C, sh.H, sh.N // 2
-    lx, sx = X[1], X[2]
+    lx = X[1]
     offs = [(dy, dx) for dy in (-1, 0, 1) for dx in (-1, 0, 1)]
     rots = dict(zip([o for o in offs if o != (0, 0)], ev.rot_hoisted(X, sh.offsets)))   # 1
     rots[(0, 0)] = X
@@ -286,25 +286,121 @@ def conv_layer(sh: ConvShape, prm: ckks.Params, X, w: np.ndarray, bias: np.ndarr
     for d in range(C):                                            # 2
         acc = None
         for dy, dx in offs:
-            t = ev.pmul(rots[(dy, dx)], f"w_{d}_{dy}_{dx}", conv_diag(sh, w, d, dy, dx), S_w)
+            t = ev.pmul(rots[(dy, dx)], f"{pre}w_{d}_{dy}_{dx}", conv_diag(sh, w, d, dy, dx), S_w)
             acc = t if acc is None else ev.add(acc, t)
         if d:
             acc = ev.rot(acc, d * H * H)
         Y = acc if Y is None else ev.add(Y, acc)
     Y = ev.rescale(Y)
     bias_slots = np.tile(np.repeat(bias, H * H), half // (C * H * H))
-    Y = ev.padd(Y, "bias", bias_slots)                            # 3
-    a0, a1, a2, a4 = RELU_A                                       # 4
-    lY, S_a = Y[1], sx
+    return ev.padd(Y, f"{pre}bias", bias_slots)                   # 3
+
+
+def _relu(sh: ConvShape, ev: Ev, Y, pre: str = ""):
+    """Step 4: the degree-4 ReLU polynomial; three levels, the output keeps Y's scale."""
+    prm, half = ev.prm, sh.N // 2
+    a0, a1, a2, a4 = RELU_A
+    lY, S_a = Y[1], Y[2]
     Y2 = ev.rescale(ev.mul(Y, Y))                                 # level lY-1
     sU = S_a * prm.q[lY - 2] / Y2[2]                              # Y2 * U / q_{lY-2} = S_a
-    U = ev.pmul_to(Y2, "relu_a4", np.full(half, a4), sU)          # level lY-2
+    U = ev.pmul_to(Y2, f"{pre}relu_a4", np.full(half, a4), sU)    # level lY-2
     Y4 = ev.rescale(ev.mul(ev.drop(Y2, lY - 2), U))               # level lY-3
-    Y2c = ev.drop(ev.pmul_to(Y2, "relu_a2", np.full(half, a2), S_a), lY - 3)
-    Y1c = ev.drop(ev.pmul_to(Y, "relu_a1", np.full(half, a1), S_a), lY - 3)
-    out = ev.padd(ev.add(ev.add(Y4, Y2c), Y1c), "relu_a0", np.full(half, a0))
-    assert out[1] == lx - CONV_LEVELS
+    Y2c = ev.drop(ev.pmul_to(Y2, f"{pre}relu_a2", np.full(half, a2), S_a), lY - 3)
+    Y1c = ev.drop(ev.pmul_to(Y, f"{pre}relu_a1", np.full(half, a1), S_a), lY - 3)
+    return ev.padd(ev.add(ev.add(Y4, Y2c), Y1c), f"{pre}relu_a0", np.full(half, a0))
+
+
+def conv_layer(sh: ConvShape, prm: ckks.Params, X, w: np.ndarray, bias: np.ndarray, keys: dict,
+               consts: dict | None = None):
+    """X = (ct, level, scale).  Returns (out, consts, counts); out at level - 4, X's scale."""
+    ev = Ev(prm, keys, consts)
+    out = _relu(sh, ev, _conv(sh, ev, X, w, bias))
+    assert out[1] == X[1] - CONV_LEVELS
     return out, ev.consts, ev.counts
+
+
+# --------------------------------------------------------------------------- ResNet-20 mix
+# Reading R4 (APP): the layer types of [32]'s ResNet-20 beyond one convolution -- a stride-1
+# basic block (conv, ReLU, conv, + shortcut, ReLU: the block of all three stages, here at the
+# first stage's shape) and the network head (global average pooling, 64 -> 10 fully connected
+# layer, here C -> K with K <= C).  The stride-2 blocks that change the packing between stages
+# are not built.
+
+BLOCK_LEVELS = 2 * CONV_LEVELS
+HEAD_LEVELS = 2
+
+
+def basic_block(sh: ConvShape, prm: ckks.Params, X, w1, b1, w2, b2, keys: dict, consts: dict | None = None):
+    """out = ReLU(conv2(ReLU(conv1(X))) + X): 8 levels, X's scale.  Returns (out, consts, counts)."""
+    ev = Ev(prm, keys, consts)
+    h = _relu(sh, ev, _conv(sh, ev, X, w1, b1, "c1_"), "r1_")
+    y = _conv(sh, ev, h, w2, b2, "c2_")
+    out = _relu(sh, ev, ev.add(y, ev.drop(X, y[1])), "r2_")
+    assert out[1] == X[1] - BLOCK_LEVELS
+    return out, ev.consts, ev.counts
+
+
+def head_rotations(sh: ConvShape) -> tuple[list[int], list[int]]:
+    """(pooling's rotate-and-sum amounts 2^k < H^2, the FC layer's hoisted amounts d H^2)."""
+    return [1 << k for k in range(int(math.log2(sh.H * sh.H)))], [d * sh.H * sh.H for d in range(1, sh.C)]
+
+
+def head(sh: ConvShape, prm: ckks.Params, X, wfc: np.ndarray, bfc: np.ndarray, keys: dict,
+         consts: dict | None = None):
+    """Global average pooling per channel then a K x C fully connected layer (K = len(bfc) <= C):
+    class k at slot k H^2.  2 levels, X's scale.  Returns (out, consts, counts)."""
+    ev = Ev(prm, keys, consts)
+    C, H, half = sh.C, sh.H, sh.N // 2
+    K = len(bfc)
+    pool_r, fc_r = head_rotations(sh)
+    P = X
+    for r in pool_r:                                              # slot c H^2: sum over channel c
+        P = ev.add(P, ev.rot(P, r))
+    m = np.zeros(C * H * H)
+    m[:: H * H] = 1.0 / (H * H)
+    P = ev.pmul_to(P, "pool_mask", np.tile(m, half // m.size), X[2])   # pooled[c] at slot c H^2
+    rots = [P] + ev.rot_hoisted(P, fc_r)
+    S_w = float(prm.q[P[1]])
+    acc = None
+    for d in range(C):                                            # diagonal method on the H^2 grid
+        diag = np.zeros(C * H * H)
+        for k in range(K):
+            diag[k * H * H] = wfc[k, (k + d) % C]
+        t = ev.pmul(rots[d], f"fc_{d}", np.tile(diag, half // diag.size), S_w)
+        acc = t if acc is None else ev.add(acc, t)
+    out = ev.rescale(acc)
+    bb = np.zeros(C * H * H)
+    bb[: K * H * H: H * H] = bfc
+    out = ev.padd(out, "fc_bias", np.tile(bb, half // bb.size))
+    assert out[1] == X[1] - HEAD_LEVELS
+    return out, ev.consts, ev.counts
+
+
+def relu_poly(y):
+    a0, a1, a2, a4 = RELU_A
+    return a0 + a1 * y + a2 * y ** 2 + a4 * y ** 4
+
+
+def conv_linear_plain(sh: ConvShape, x, w, bias) -> np.ndarray:
+    """3x3 conv (stride 1, zero padding) + bias, no activation."""
+    C, H = sh.C, sh.H
+    xp = np.zeros((C, H + 2, H + 2))
+    xp[:, 1:-1, 1:-1] = x
+    y = np.zeros((C, H, H))
+    for co in range(C):
+        for ci in range(C):
+            for dy in (-1, 0, 1):
+                for dx in (-1, 0, 1):
+                    y[co] += w[co, ci, dy + 1, dx + 1] * xp[ci, 1 + dy:1 + dy + H, 1 + dx:1 + dx + H]
+    return y + bias[:, None, None]
+
+
+def block_plain(sh: ConvShape, x, w1, b1, w2, b2) -> np.ndarray:
+    return relu_poly(conv_linear_plain(sh, relu_poly(conv_linear_plain(sh, x, w1, b1)), w2, b2) + x)
+
+
+def head_plain(x, wfc, bfc) -> np.ndarray:
+    return wfc @ x.mean(axis=(1, 2)) + bfc
 
 
 # --------------------------------------------------------------------------- keys, encryption

@@ -114,8 +114,9 @@ def tiny() -> BootParams:
 
 
 def set_b() -> BootParams:
-    """Set-B (Table 4) with 8 sparse slots, r = 12 squarings (h = 192: |I| up to ~100)."""
-    return BootParams(ckks.set_b(), n=8, r=12, h=192)
+    """Set-B (Table 4) with 8 sparse slots and the schedule of set_b_full (reading BOOT-S: 2^20
+    boosts, EvalMod r = 9 with its first steps at ~q^2 via Double Rescale), levels 35 -> 7."""
+    return BootParams(ckks.set_b(), n=8, r=9, h=192, boost=(20, 20), ds_sq=4)
 
 
 # --------------------------------------------------------------------------- slot algebra
@@ -153,8 +154,9 @@ def _pt(bp: BootParams, slots_n: np.ndarray, scale: float, level: int) -> np.nda
         m[:] = 0
         m[0] = _round_big(scale, v[0].real)
         m[prm.N // 2] = _round_big(scale, v[0].imag)
-    else:
-        m = ckks.encode(prm.N, np.tile(v, bp.M), scale)
+    else:   # N >= 2^14: encode_fft (within 1 of encode, pinned; any valid encoding, reading BOOT-F)
+        enc = ckks.encode_fft if prm.N >= 1 << 14 else ckks.encode
+        m = enc(prm.N, np.tile(v, bp.M), scale)
     return ckks.ntt(prm, ckks.reduce_signed(prm, m, ids), ids)
 
 

@@ -11,7 +11,9 @@ HELR iteration (L530, "batch sizes of 1,024 images", 196 features -> f = 256):
 ResNet-20 layer (L572, [32]'s 16-channel 32 x 32 stage): 8 hoisted baby-step rotations of the
   input (one ModUp), per channel diagonal d one fused plaintext inner product over the 9 kernel
   offsets (neo_pmult_acc) and one giant-step HROT by d H^2, Rescale, bias PADD, and the degree-4
-  ReLU polynomial (two HMULTs, three PMULTs).
+  ReLU polynomial (two HMULTs, three PMULTs).  The layer mix (reading R4): a stride-1 basic
+  block (conv, ReLU, conv, + shortcut, ReLU) and the head (average pooling by rotate-and-sum,
+  a fully connected layer by the diagonal method on the H^2-strided grid).
 
 Plaintext constants are inputs (name -> device tensor [l+1][N], NTT form), like evaluation
 keys: tests produce them with the oracle's encoder, bench.py with random residues (the cost is
@@ -165,8 +167,8 @@ def helr_iteration(ev: Evaluator, f: int, Z: torch.Tensor, W: torch.Tensor, leve
     return Wn, lg - 1
 
 
-def conv_layer(ev: Evaluator, C: int, H: int, X: torch.Tensor, level: int):
-    """X [1][2][level+1][N] -> (out [1][2][level-3][N], level - 4)."""
+def conv(ev: Evaluator, C: int, H: int, X: torch.Tensor, level: int, pre: str = ""):
+    """Convolution + Rescale + bias (the oracle's _conv): X at `level` -> level - 1."""
     baby, _ = conv_rotations(C, H)
     lv = level
     R = ev.rot_hoisted(X, baby, lv)                               # 1: [8][1][2][l+1][N]
@@ -180,17 +182,67 @@ def conv_layer(ev: Evaluator, C: int, H: int, X: torch.Tensor, level: int):
             k += 1
     Y = None
     for d in range(C):                                            # 2
-        acc = ev.pmul_acc(src, [f"w_{d}_{dy}_{dx}" for dy, dx in offs], lv)
+        acc = ev.pmul_acc(src, [f"{pre}w_{d}_{dy}_{dx}" for dy, dx in offs], lv)
         if d:
             acc = ev.rot(acc, d * H * H, lv)
         Y = acc if Y is None else ev.add(Y, acc, lv)
     Y = ev.rescale(Y, lv)
-    lY = lv - 1
-    Y = ev.padd(Y, "bias", lY)                                    # 3
-    Y2 = ev.hmul_rescale(Y, Y, lY)                        # 4
-    U = ev.rescale(ev.pmul(Y2, "relu_a4", lY - 1), lY - 1)
+    return ev.padd(Y, f"{pre}bias", lv - 1)                       # 3
+
+
+def relu(ev: Evaluator, Y: torch.Tensor, lY: int, pre: str = ""):
+    """The degree-4 ReLU polynomial (the oracle's _relu): lY -> lY - 3."""
+    Y2 = ev.hmul_rescale(Y, Y, lY)                                # 4
+    U = ev.rescale(ev.pmul(Y2, f"{pre}relu_a4", lY - 1), lY - 1)
     Y4 = ev.hmul_rescale(ev.drop(Y2, lY - 1, lY - 2), U, lY - 2)
-    Y2c = ev.drop(ev.rescale(ev.pmul(Y2, "relu_a2", lY - 1), lY - 1), lY - 2, lY - 3)
-    Y1c = ev.drop(ev.rescale(ev.pmul(Y, "relu_a1", lY), lY), lY - 1, lY - 3)
-    out = ev.padd(ev.add(ev.add(Y4, Y2c, lY - 3), Y1c, lY - 3), "relu_a0", lY - 3)
-    return out, lY - 3
+    Y2c = ev.drop(ev.rescale(ev.pmul(Y2, f"{pre}relu_a2", lY - 1), lY - 1), lY - 2, lY - 3)
+    Y1c = ev.drop(ev.rescale(ev.pmul(Y, f"{pre}relu_a1", lY), lY), lY - 1, lY - 3)
+    return ev.padd(ev.add(ev.add(Y4, Y2c, lY - 3), Y1c, lY - 3), f"{pre}relu_a0", lY - 3)
+
+
+def conv_layer(ev: Evaluator, C: int, H: int, X: torch.Tensor, level: int):
+    """X [1][2][level+1][N] -> (out [1][2][level-3][N], level - 4)."""
+    return relu(ev, conv(ev, C, H, X, level), level - 1), level - 4
+
+
+# ---- ResNet-20 layer mix (reading R4): a stride-1 basic block and the network head
+
+def block_const_names(C: int) -> list[str]:
+    names = []
+    for pre in ("c1_", "c2_"):
+        names += [f"{pre}w_{d}_{dy}_{dx}" for d in range(C) for dy in (-1, 0, 1) for dx in (-1, 0, 1)]
+        names.append(f"{pre}bias")
+    for pre in ("r1_", "r2_"):
+        names += [f"{pre}relu_a{k}" for k in (4, 2, 1, 0)]
+    return names
+
+
+def head_rotations(C: int, H: int) -> tuple[list[int], list[int]]:
+    """(pooling's rotate-and-sum amounts 2^k < H^2, the FC layer's hoisted amounts d H^2)."""
+    return [1 << k for k in range(int(math.log2(H * H)))], [d * H * H for d in range(1, C)]
+
+
+def head_const_names(C: int) -> list[str]:
+    return ["pool_mask"] + [f"fc_{d}" for d in range(C)] + ["fc_bias"]
+
+
+def basic_block(ev: Evaluator, C: int, H: int, X: torch.Tensor, level: int):
+    """ReLU(conv2(ReLU(conv1(X))) + X): level -> level - 8."""
+    h = relu(ev, conv(ev, C, H, X, level, "c1_"), level - 1, "r1_")
+    y = conv(ev, C, H, h, level - 4, "c2_")
+    z = ev.add(y, ev.drop(X, level, level - 5), level - 5)
+    return relu(ev, z, level - 5, "r2_"), level - 8
+
+
+def head(ev: Evaluator, C: int, H: int, X: torch.Tensor, level: int):
+    """Global average pooling + fully connected layer (class k at slot k H^2): level -> level - 2."""
+    pool_r, fc_r = head_rotations(C, H)
+    P = X
+    for r in pool_r:
+        P = ev.add(P, ev.rot(P, r, level), level)
+    P = ev.rescale(ev.pmul(P, "pool_mask", level), level)
+    lv = level - 1
+    R = ev.rot_hoisted(P, fc_r, lv)
+    acc = ev.pmul_acc([P] + [R[k] for k in range(C - 1)], [f"fc_{d}" for d in range(C)], lv)
+    out = ev.rescale(acc, lv)
+    return ev.padd(out, "fc_bias", lv - 1), lv - 1

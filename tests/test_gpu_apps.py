@@ -119,3 +119,35 @@ def test_pmult_acc_rejects_bad_arguments():
         neo.neo_pmult_acc(ctx, [ct], [pt], 2, ct, 1, pt_shared=True)          # aliasing
     with pytest.raises(neo.NeoError):
         neo.neo_pmult_acc(ctx, [ct], [pt], prm.max_level + 1, torch.empty_like(ct), 1, pt_shared=True)
+
+
+def test_resnet_block_and_head_bit_exact():
+    """The ResNet-20 layer mix (reading R4): a stride-1 basic block then the head, GPU vs oracle bit
+    for bit, decoding to the plain computation."""
+    from test_oracle_apps import block_inputs, block_params
+    prm = block_params()
+    sh = apps.ConvShape(prm.N, C=4, H=8)
+    s = ckks.secret(prm, 35, 64)
+    baby, giant = sh.rotations()
+    pool_r, fc_r = apps.head_rotations(sh)
+    assert gapps.head_rotations(sh.C, sh.H) == (pool_r, fc_r)
+    keys_np = apps.app_keys(prm, s, baby + giant + pool_r, 810)
+    x, w1, b1, w2, b2, wfc, bfc = block_inputs(sh)
+    L = prm.max_level
+    X = apps.encrypt_slots(prm, apps.conv_pack(sh, x), DELTA, s, L, 71)
+    want_b, cb, _ = apps.basic_block(sh, prm, X, w1, b1, w2, b2, keys_np)
+    want_h, ch, _ = apps.head(sh, prm, want_b, wfc, bfc, keys_np)
+    assert sorted(cb) == sorted(gapps.block_const_names(sh.C)) and sorted(ch) == sorted(gapps.head_const_names(sh.C))
+    ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+    hoisted = [gapps.galois(prm.N, r) for r in baby + fc_r]
+    consts = {k: dev(v) for k, v in {**cb, **ch}.items()}
+    ev = gapps.Evaluator(ctx, gpu_keys(ctx, keys_np, hoisted), consts)
+    gb, lb = gapps.basic_block(ev, sh.C, sh.H, dev(X[0][None]), L)
+    gh, lh = gapps.head(ev, sh.C, sh.H, gb, lb)
+    torch.cuda.synchronize()
+    assert (lb, lh) == (want_b[1], want_h[1])
+    assert np.array_equal(gb.cpu().numpy()[0], want_b[0])
+    assert np.array_equal(gh.cpu().numpy()[0], want_h[0])
+    z = np.real(apps.decrypt_slots(prm, (gh.cpu().numpy()[0], lh, want_h[2]), s))
+    got = z[: 3 * sh.H * sh.H: sh.H * sh.H]
+    assert np.max(np.abs(got - apps.head_plain(apps.block_plain(sh, x, w1, b1, w2, b2), wfc, bfc))) < TOL

@@ -174,3 +174,30 @@ def test_set_b_full_slot_bootstrap_decodes():
     # measured 2.0e-3 (r02); single-prime rescales throughout gave ~1 (EvalMod's 2^12 amplification
     # of ~2^-36-relative key-switch / rescale noise).  1e-2: the tiny full-slot gate.
     assert err < 1e-2
+
+
+@pytest.mark.slow
+def test_set_b_sparse_bootstrap_decodes():
+    """bench.py's second bootstrap configuration (oracle.boot.set_b: Set-B, 8 sparse slots, the
+    same reading-BOOT-S schedule) with real keys and constants decodes to the input slots."""
+    bp = boot.set_b()
+    prm = bp.prm
+    s = ckks.secret(prm, 71, bp.h)
+    keys_np = boot.boot_keys(bp, s, 720)
+    lv, scale, consts = boot.dry_run(bp)
+    z = synth.complex_slots(73, bp.n)
+    delta = 2.0 ** 31
+    ct0 = ckks.encrypt(prm, ckks.encode_fft(prm.N, np.tile(z, bp.M), delta), s, 0, 75)
+    ctx = neo.Context(prm.log_n, prm.num_q, prm.num_p, prm.dnum)
+    keys = {k: neo.EvalKey(ctx, dev(v)) for k, v in keys_np.items()}
+    for g in gboot.hoisted_rotations(prm.N, bp.n):
+        keys[("h", g)] = neo.EvalKey(ctx, dev(keys_np[g]), hoisted_galois=g)
+    b = gboot.Bootstrapper(ctx, bp.n, bp.r, keys, {k: dev(v) for k, v in consts.items()}, boost=bp.boost,
+                           ds_sq=bp.ds_sq)
+    got, glv = b.run(dev(ct0[None]))
+    torch.cuda.synchronize()
+    assert glv == lv
+    zz = _decode_sample(prm, got.cpu().numpy()[0], lv, scale * delta / prm.q[0], s, np.arange(bp.n))
+    err = np.max(np.abs(zz - z))
+    print(f"Set-B sparse bootstrap: max slot error {err:.3e}")
+    assert err < 1e-2

@@ -124,3 +124,56 @@ def test_conv_op_counts(conv_run):
     assert counts["hrot"] == 8 + (sh.C - 1)
     assert counts["pmult"] == 9 * sh.C + 3
     assert counts["hmult"] == 2
+
+
+def block_params() -> ckks.Params:
+    """N = 2^12, 13 Q limbs + 2 P limbs, dnum 7 (alpha = 2): 12 levels for a block + the head."""
+    return ckks.Params(12, 13, 2, 7)
+
+
+def block_inputs(sh):
+    r = lambda k, n: synth.uniform_unit(synth.derive(47, k), n)
+    x = 2.0 * r(1, sh.C * sh.H * sh.H).reshape(sh.C, sh.H, sh.H) - 1.0
+    w1 = (2.0 * r(2, sh.C * sh.C * 9).reshape(sh.C, sh.C, 3, 3) - 1.0) / 6.0
+    w2 = (2.0 * r(3, sh.C * sh.C * 9).reshape(sh.C, sh.C, 3, 3) - 1.0) / 6.0
+    b1, b2 = 0.2 * (2.0 * r(4, sh.C) - 1.0), 0.2 * (2.0 * r(5, sh.C) - 1.0)
+    wfc = (2.0 * r(6, 3 * sh.C).reshape(3, sh.C) - 1.0) / 2.0
+    bfc = 0.1 * (2.0 * r(7, 3) - 1.0)
+    return x, w1, b1, w2, b2, wfc, bfc
+
+
+def test_block_plain_is_the_residual_definition():
+    """block_plain = relu(conv2(relu(conv1 x)) + x) with conv_plain's convolution (pinned above)."""
+    sh = apps.ConvShape(4096, C=3, H=5)
+    rng = np.random.default_rng(4)
+    x, w1, w2 = rng.standard_normal((3, 5, 5)), rng.standard_normal((3, 3, 3, 3)), rng.standard_normal((3, 3, 3, 3))
+    b1, b2 = rng.standard_normal(3), rng.standard_normal(3)
+    assert np.allclose(apps.relu_poly(apps.conv_linear_plain(sh, x, w1, b1)), apps.conv_plain(sh, x, w1, b1))
+    h = apps.conv_plain(sh, x, w1, b1)
+    want = apps.relu_poly(apps.conv_linear_plain(sh, h, w2, b2) + x)
+    assert np.allclose(apps.block_plain(sh, x, w1, b1, w2, b2), want)
+
+
+def test_resnet_block_and_head_decode():
+    """A stride-1 ResNet-20 basic block then the network head (pooling + FC) decode to the plain
+    computation (tolerance as above: the block's key-switches and rescales at ~2^36 scales)."""
+    prm = block_params()
+    sh = apps.ConvShape(prm.N, C=4, H=8)
+    s = ckks.secret(prm, 35, 64)
+    baby, giant = sh.rotations()
+    pool_r, fc_r = apps.head_rotations(sh)
+    keys = apps.app_keys(prm, s, baby + giant + pool_r, 810)
+    x, w1, b1, w2, b2, wfc, bfc = block_inputs(sh)
+    L = prm.max_level
+    X = apps.encrypt_slots(prm, apps.conv_pack(sh, x), DELTA, s, L, 71)
+    out, _, counts = apps.basic_block(sh, prm, X, w1, b1, w2, b2, keys)
+    assert out[1] == L - apps.BLOCK_LEVELS
+    want_b = apps.block_plain(sh, x, w1, b1, w2, b2)
+    got_b = apps.conv_unpack(sh, apps.decrypt_slots(prm, out, s))
+    assert np.max(np.abs(got_b - want_b)) < TOL
+    assert counts["hrot"] == 2 * (8 + sh.C - 1) and counts["hmult"] == 4
+    hd, _, hc = apps.head(sh, prm, out, wfc, bfc, keys)
+    z = np.real(apps.decrypt_slots(prm, hd, s))
+    got_h = z[: 3 * sh.H * sh.H: sh.H * sh.H]
+    assert np.max(np.abs(got_h - apps.head_plain(want_b, wfc, bfc))) < TOL
+    assert hc["hrot"] == len(pool_r) + sh.C - 1
