@@ -105,10 +105,11 @@ struct ProfScope {
 static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long src_bs, const int* src_off,
                            u64* dst, long long dst_bs, const int* dst_off, const int* prime, int n, u64* tmp,
                            int batch, cudaStream_t st, const RowEpi* epi = nullptr, bool in_lazy = false,
-                           const TWD* scale = nullptr, unsigned galois = 0) {
+                           const TWD* scale = nullptr, unsigned galois = 0, const u64* fold = nullptr,
+                           const TWD* fold_w = nullptr) {
     if (n <= 0) return NEO_OK;
     if (n > NEO_MAX_ROWS) {               // more rows than one launch's descriptor holds: chunks
-        if (epi) FAIL(NEO_EUNSUPPORTED, "too many limb rows for a fused-epilogue transform");
+        if (epi || fold) FAIL(NEO_EUNSUPPORTED, "too many limb rows for a fused-epilogue transform");
         for (int k0 = 0; k0 < n; k0 += NEO_MAX_ROWS) {
             const int m = std::min(NEO_MAX_ROWS, n - k0);
             neo_status s = ntt_rows(c, fwd, src, src_bs, src_off + k0, dst, dst_bs, dst_off + k0, prime + k0, m, tmp,
@@ -135,6 +136,10 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
     }
     if (b.has_scale)
         for (int k = 0; k < n; ++k) b.scale[k] = scale[k];
+    if (fwd && fold) {                    // forward column pass: x += fold[b] * fold_w[k]
+        a.fold = fold;
+        for (int k = 0; k < n; ++k) a.scale[k] = fold_w[k];
+    }
     // first pass: src -> tmp ; second pass: tmp -> dst
     a.src = src; a.src_bstride = src_bs;
     a.dst = tmp; a.dst_bstride = (long long)n * N;
@@ -169,7 +174,9 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
     L.acc = o; o += B * 2 * E * N;
     L.conv = o; o += B * 2 * Lq * N;
     L.pc = o; o += B * 2 * P * N;
-    L.tmp = o; o += B * std::max(std::max(beta * E, 2 * Lq), 2 * P) * N;
+    size_t tmp_rows = std::max(std::max(beta * E, 2 * Lq), 2 * P);
+    if (op == NEO_OP_HMULT_RESCALE) tmp_rows = std::max(tmp_rows, 2 * P + 4);   // merged P-part + last-limb INTT
+    L.tmp = o; o += B * tmp_rows * N;
     L.extra = o;
     if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
     if (op == NEO_OP_HMULT_RESCALE) o += B * 3 * Lq * N + 4 * B * N;   // d, then c_l scratch
@@ -197,8 +204,25 @@ static size_t ds_ws(const neo_ctx* c, int l, int B) {
 
 // ------------------------------------------------------------------ key-switch core
 // a3-a5: ModUp of d (INTT, BConv of every digit onto PQ_l, NTT) into the workspace.
+// The ModUp NTT's row pass can be fused with KeyIP (ntt.h KipArgs): ks_modup(..., fused) then
+// stops after the column pass and ks_finish(..., fused) runs the fused pass instead of KeyIP.
+// FP64 NTT only; the ModUp rows must fit one launch descriptor.
+static bool kip_ok(const neo_ctx* c, int l) {
+    if (c->ntt_impl == NEO_NTT_TC && c->ntt.tct) return false;
+    const int E = c->ext(l), beta = c->beta(l);
+    if (E > KIP_MAX_EXT || beta > KIP_MAX_BETA) return false;
+    int n = 0;
+    for (int j = 0; j < beta; ++j) n += E - (int)c->digits[l][j].size();
+    static int on = -1;                  // measured slower than the separate KeyIP: opt-in
+    if (on < 0) {
+        const char* e = std::getenv("NEO_KIP");
+        on = (e && e[0] == '1') ? 1 : 0;
+    }
+    return on && n <= NEO_MAX_ROWS;
+}
+
 static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l, int B, u64* ws, const KsLayout& Ly,
-                           cudaStream_t st, unsigned galois = 0) {
+                           cudaStream_t st, unsigned galois = 0, bool fused = false) {
     const int N = c->N, Lq = l + 1, E = c->ext(l), beta = c->beta(l);
     u64 *y = ws + Ly.y, *up = ws + Ly.up, *tmp = ws + Ly.tmp;
     int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
@@ -266,6 +290,19 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
             ++n;
         }
     }
+    if (fused) {            // column pass only: the row pass runs fused with KeyIP in ks_finish
+        RowSet a;
+        a.n = n;
+        a.in_lazy = c->use_tc ? 1 : 0;
+        a.has_scale = 0;
+        a.galois = 0;
+        a.galois_inv_n1 = 0;
+        a.src = up; a.src_bstride = (long long)beta * E * N;
+        a.dst = tmp; a.dst_bstride = (long long)n * N;
+        for (int k = 0; k < n; ++k) { a.src_off[k] = so[k]; a.dst_off[k] = k; a.prime[k] = (short)pr[k]; }
+        LAUNCH(PK_NTT_COL, st, ntt_pass(true, a, c->ntt, B, true, st));
+        return NEO_OK;
+    }
     if ((s = ntt_rows(c, true, up, (long long)beta * E * N, so, up, (long long)beta * E * N, dof, pr, n, tmp, B, st,
                       nullptr, c->use_tc)))
         return s;
@@ -278,7 +315,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
                             u64* ws, const KsLayout& Ly, u64* out0, u64* out1, long long out_bs,
                             const u64* add0, const u64* add1, long long add_bs, cudaStream_t st,
                             unsigned galois = 0, bool add_galois = true, u64* hmr_last = nullptr,
-                            int phase = 0) {
+                            int phase = 0, bool fused = false) {
     // phase 0: KeyIP then ModDown; 1: KeyIP only (acc overwritten); 2: KeyIP only, accumulated
     // into acc; 3: ModDown only (of the acc already in the workspace) -- neo_hrot_sum
     // hmr_last != nullptr: fused HMULT + Rescale (neo_hmult_rescale).  add0/add1 are then d0/d1
@@ -289,8 +326,32 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
     neo_status s;
 
-    // a6: KeyIP over all E limbs of PQ_l
-    if (phase != 3) {
+    // a5 row pass + a6 fused: acc straight from the column-pass intermediates (ntt.h KipArgs)
+    if (phase != 3 && fused) {
+        KipArgs A;
+        A.tmp = reinterpret_cast<const double*>(ws + Ly.tmp);
+        int n = 0;
+        for (int pos = 0; pos < E; ++pos) { A.ntr[pos] = 0; A.own[pos] = -1; }
+        for (int j = 0; j < beta; ++j) {                 // the row order of ks_modup's column pass
+            const std::vector<int>& dj = c->digits[l][j];
+            for (int pos = 0; pos < E; ++pos) {
+                const int id = c->ext_id(l, pos);
+                if (std::find(dj.begin(), dj.end(), id) != dj.end()) { A.own[pos] = (signed char)j; continue; }
+                A.dig[pos][A.ntr[pos]] = (unsigned char)j;
+                A.row[pos][A.ntr[pos]++] = (short)n++;
+            }
+        }
+        for (int pos = 0; pos < E; ++pos) A.limb[pos] = c->ext_id(l, pos);
+        A.tmp_bstride = (long long)n * N;
+        A.d = d; A.d_bstride = d_bs; A.galois = galois;
+        A.evk_lo = k->lo; A.evk_hi = k->hi; A.evk_limbs = c->num_q + c->num_p;
+        A.acc = acc;
+        A.acc_bstride = (long long)2 * E * N;
+        A.acc_cstride = (long long)E * N;
+        A.mods = c->d_mods;
+        A.accumulate = phase == 2;
+        LAUNCH(PK_NTT_ROW, st, ntt_row_kip(c->ntt, A, E, B, st));
+    } else if (phase != 3) {   // a6: KeyIP over all E limbs of PQ_l
         KeyIPArgs A;
         A.d = d; A.up = up; A.evk_lo = k->lo; A.evk_hi = k->hi; A.acc = acc; A.mods = c->d_mods;
         A.d_bstride = d_bs;
@@ -314,11 +375,43 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     }
     if (phase == 1 || phase == 2) return NEO_OK;
 
-    // a7: INTT of the P part of acc_0, acc_1 -> pc [2B][P][N], with ModDown's [a_k Phat_k^-1] folded in
-    for (int k2 = 0; k2 < P; ++k2) { so[k2] = Lq + k2; dof[k2] = k2; pr[k2] = c->num_q + k2; }
-    if ((s = ntt_rows(c, false, acc, (long long)E * N, so, pc, (long long)P * N, dof, pr, P, tmp, 2 * B, st, nullptr,
-                      false, c->use_tc ? c->moddown_tc[l].qhat_inv : nullptr)))
-        return s;
+    // a7: INTT of the P part of acc_0, acc_1 -> pc [2B][P][N], with ModDown's [a_k Phat_k^-1] folded in.
+    // Fused HMULT + Rescale at small batch: the 4B last-limb rows (acc_c,l and d_c,l, needed in
+    // coefficient form below) join the same launch as extra rows (scale 1), one INTT instead of two.
+    const bool hmr_merged = hmr_last && (2 * P + 4) * B <= NEO_MAX_ROWS;
+    if (hmr_merged) {
+        const u64* base = std::min<const u64*>(acc, add0);
+        const long long oa = (acc - base) / N, od = (add0 - base) / N, d1 = (add1 - add0) / N;
+        const long long oh = (hmr_last - pc) / N;            // hmr_last lies after pc in the workspace
+        TWD sc[NEO_MAX_ROWS];
+        const TWD one{1.0, 1.0 / (double)c->mod[l]};
+        int n = 0;
+        for (int b = 0; b < B; ++b)
+            for (int cc = 0; cc < 2; ++cc)
+                for (int k2 = 0; k2 < P; ++k2) {
+                    so[n] = (int)(oa + (long long)b * 2 * E + (long long)cc * E + Lq + k2);
+                    dof[n] = (2 * b + cc) * P + k2;
+                    pr[n] = c->num_q + k2;
+                    sc[n++] = c->use_tc ? c->moddown_tc[l].qhat_inv[k2] : TWD{1.0, 1.0 / (double)c->mod[c->num_q + k2]};
+                }
+        for (int b = 0; b < B; ++b)
+            for (int cc = 0; cc < 2; ++cc) {
+                so[n] = (int)(oa + (long long)b * 2 * E + (long long)cc * E + l);
+                dof[n] = (int)(oh + 2 * b + cc);
+                pr[n] = l;
+                sc[n++] = one;
+                so[n] = (int)(od + (long long)b * (add_bs / N) + cc * d1 + l);
+                dof[n] = (int)(oh + 2 * B + 2 * b + cc);
+                pr[n] = l;
+                sc[n++] = one;
+            }
+        if ((s = ntt_rows(c, false, base, 0, so, pc, 0, dof, pr, n, tmp, 1, st, nullptr, false, sc))) return s;
+    } else {
+        for (int k2 = 0; k2 < P; ++k2) { so[k2] = Lq + k2; dof[k2] = k2; pr[k2] = c->num_q + k2; }
+        if ((s = ntt_rows(c, false, acc, (long long)E * N, so, pc, (long long)P * N, dof, pr, P, tmp, 2 * B, st, nullptr,
+                          false, c->use_tc ? c->moddown_tc[l].qhat_inv : nullptr)))
+            return s;
+    }
 
     // a8: ModDown BConv P -> q_0..q_l, batch 2B
     {
@@ -352,8 +445,9 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         u64* accl = hmr_last;
         u64* dl = hmr_last + (size_t)2 * B * N;
         // the 4 rows acc_0,l acc_1,l d_0,l d_1,l of every batch entry in ONE inverse transform
-        // (rows addressed from the lower of the two workspace buffers; batch entries as rows)
-        {
+        // (rows addressed from the lower of the two workspace buffers; batch entries as rows),
+        // unless they already went with the P part above
+        if (!hmr_merged) {
             const u64* base = std::min<const u64*>(acc, add0);
             const long long oa = (acc - base) / N, od = (add0 - base) / N, d1 = (add1 - add0) / N;
             int n = 0;
@@ -379,7 +473,10 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
             F.pmod[i].wq = (double)pm / (double)qi;
         }
         F.N = N; F.l = l; F.lazy = c->use_tc ? 1 : 0;
-        LAUNCH(PK_EW, st, launch_hmr_fold(F, 2 * B, st));
+        // FP64 NTT: c_l alone here, conv_i += P c_l inside the next column pass (RowSet::fold)
+        const bool fold_fused = !(c->ntt_impl == NEO_NTT_TC && c->ntt.tct);
+        if (fold_fused) LAUNCH(PK_EW, st, launch_hmr_cl(F, 2 * B, st));
+        else LAUNCH(PK_EW, st, launch_hmr_fold(F, 2 * B, st));
         for (int i = 0; i < l; ++i) { so[i] = dof[i] = i; pr[i] = i; }
         RowEpi ep;
         ep.acc = acc;
@@ -391,7 +488,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         ep.has_post = 1;
         for (int i = 0; i < l; ++i) { ep.pinv[i] = c->pinv[i]; ep.post[i] = c->ql_inv[l][i]; }
         return ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, l, tmp, 2 * B, st,
-                        &ep, c->use_tc);
+                        &ep, c->use_tc, nullptr, 0, fold_fused ? accl : nullptr, F.pmod);
     }
 
     // a9 + a10: NTT of conv, with the ModDown tail (acc - conv) * P^-1 (+ add) fused into the
@@ -631,9 +728,11 @@ static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long
     if (k->klss)           // the key decides the method; c0's automorphism was applied by the caller
         return klss_core(c, k, d, d_bs, l, B, ws, klss_layout(c, l, B, NEO_OP_KEYSWITCH), out0, out1, out_bs, add0,
                          add1, add_bs, st, galois);
-    neo_status s = ks_modup(c, d, d_bs, l, B, ws, Ly, st, galois);
+    const bool fused = kip_ok(c, l);
+    neo_status s = ks_modup(c, d, d_bs, l, B, ws, Ly, st, galois, fused);
     if (s) return s;
-    return ks_finish(c, k, d, d_bs, l, B, ws, Ly, out0, out1, out_bs, add0, add1, add_bs, st, galois, add_galois);
+    return ks_finish(c, k, d, d_bs, l, B, ws, Ly, out0, out1, out_bs, add0, add1, add_bs, st, galois, add_galois,
+                     nullptr, 0, fused);
 }
 
 // ------------------------------------------------------------------ validation helpers
@@ -1170,9 +1269,10 @@ neo_status neo_hmult_rescale(const neo_ctx* c, const neo_evk* relin, const uint6
     const long long ls = (long long)(level + 1) * c->N, lo = (long long)level * c->N;
     cudaStream_t s = S(st);
     LAUNCH(PK_TENSOR, s, launch_tensor(ct_a, ct_b, dd, c->d_mods, level + 1, c->N, batch, s));
-    TRY(ks_modup(c, dd + 2 * ls, 3 * ls, level, batch, w, Ly, s));
+    const bool fused = kip_ok(c, level);
+    TRY(ks_modup(c, dd + 2 * ls, 3 * ls, level, batch, w, Ly, s, 0, fused));
     return ks_finish(c, relin, dd + 2 * ls, 3 * ls, level, batch, w, Ly, ct_out, ct_out + lo, 2 * lo, dd, dd + ls,
-                     3 * ls, s, 0, true, last);
+                     3 * ls, s, 0, true, last, 0, fused);
 }
 
 neo_status neo_hrot(const neo_ctx* c, const neo_evk* rk, uint32_t g, const uint64_t* ct_in, int32_t level,
@@ -1229,10 +1329,11 @@ neo_status neo_hrot_sum(const neo_ctx* c, const neo_evk* const* keys, const uint
     int launches = 0;
     for (int k = 0; k < n; ++k) {
         // KeyIP(ModUp(sigma_g(c1_k))) accumulated in PQ_l; sigma_g(c1) read through the index map
-        TRY(ks_modup(c, cts[k] + ls, 2 * ls, level, batch, w, Ly, s, galois[k]));
+        const bool fused = kip_ok(c, level);
+        TRY(ks_modup(c, cts[k] + ls, 2 * ls, level, batch, w, Ly, s, galois[k], fused));
         launches += g_launches;
         TRY(ks_finish(c, keys[k], cts[k] + ls, 2 * ls, level, batch, w, Ly, nullptr, nullptr, 0, nullptr, nullptr,
-                      0, s, galois[k], false, nullptr, k == 0 ? 1 : 2));
+                      0, s, galois[k], false, nullptr, k == 0 ? 1 : 2, fused));
         launches += g_launches;
         g_launches = 0;
         LAUNCH(PK_AUTO, s, launch_automorph(cts[k], k == 0 ? c0sum : c0k, galois[k], c->N, level + 1, s, batch,

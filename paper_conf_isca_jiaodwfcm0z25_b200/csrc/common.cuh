@@ -136,6 +136,9 @@ struct RowSet {
     int has_scale;                         // inverse column pass: multiply row k by scale[k]
     unsigned galois;                       // inverse row pass: read sigma_g(src) (X -> X^g, NTT domain); 0 = none
     unsigned galois_inv_n1;                //   g^-1 mod N1
+    const u64* fold = nullptr;             // forward column pass: x += [fold[b][n]] * scale[k] (fused
+                                           //   HMULT + Rescale: conv_i + P c_l), canonical mod the row's
+                                           //   limb ... or nullptr; fold row b of batch entry b, stride N
     int src_off[NEO_MAX_ROWS];
     int dst_off[NEO_MAX_ROWS];
     short prime[NEO_MAX_ROWS];

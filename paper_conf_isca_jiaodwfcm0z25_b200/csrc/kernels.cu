@@ -396,6 +396,23 @@ k_hmr_fold(const __grid_constant__ HmrFoldArgs A) {
     }
 }
 
+// c_l only (the fold itself goes into the next NTT's column pass, RowSet::fold): writes
+// c_l = ((accl - [conv_l]) P^-1 + dl) mod q_l over accl
+__global__ void __launch_bounds__(256)
+k_hmr_cl(const __grid_constant__ HmrFoldArgs A) {
+    pdl_wait();
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int bc = blockIdx.y;
+    if (n >= A.N) return;
+    const size_t row = (size_t)A.N, base = (size_t)bc * (A.l + 1) * row + n;
+    const ModQ ml = A.mods[A.l];
+    u64 cv;
+    if (A.lazy) cv = d2u(canon(__longlong_as_double((long long)__ldg(A.conv + base + (size_t)A.l * row)), ml.qd, ml.qinv));
+    else cv = __ldg(A.conv + base + (size_t)A.l * row);
+    u64* cl = const_cast<u64*>(A.accl) + (size_t)bc * row + n;
+    *cl = add_mod(shoup(sub_mod(*cl, cv, ml.q), A.pinv_l, ml.q), __ldg(A.dl + (size_t)bc * row + n), ml.q);
+}
+
 // ------------------------------------------------------------------ ModRaise (bootstrapping)
 // c in [0, q_0) -> the centred representative in (-q_0/2, q_0/2] reduced mod q_i
 __global__ void __launch_bounds__(256)
@@ -524,6 +541,9 @@ cudaError_t launch_ew_limbs(const EwlArgs& A, int batch, cudaStream_t st) {
 }
 cudaError_t launch_hmr_fold(const HmrFoldArgs& A, int bc, cudaStream_t st) {
     return launch_k(k_hmr_fold, dim3((A.N + 255) / 256, (A.l + kFoldRows - 1) / kFoldRows, bc), dim3(256), 0, st, A);
+}
+cudaError_t launch_hmr_cl(const HmrFoldArgs& A, int bc, cudaStream_t st) {
+    return launch_k(k_hmr_cl, dim3((A.N + 255) / 256, bc), dim3(256), 0, st, A);
 }
 cudaError_t launch_modraise(const u64* coef, u64* out, const ModQ* mods, int limbs, int N, int bc, cudaStream_t st) {
     return launch_k(k_modraise, dim3((N + 255) / 256, limbs, bc), dim3(256), 0, st, coef, out, mods, limbs, N);

@@ -111,6 +111,7 @@ cudaError_t launch_add_rows(const u64* a, const u64* b, u64* out, const ModQ* mo
                             cudaStream_t st);
 cudaError_t launch_pmult_acc(const PmaccArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_hmr_fold(const HmrFoldArgs& A, int bc, cudaStream_t st);
+cudaError_t launch_hmr_cl(const HmrFoldArgs& A, int bc, cudaStream_t st);   // c_l only, over accl
 cudaError_t launch_ew_limbs(const EwlArgs& A, int batch, cudaStream_t st);
 // 36-bit wire format (neo_wire_pack / neo_wire_unpack); n % 8 == 0
 cudaError_t launch_wire(bool pack, const void* in, void* out, size_t n, cudaStream_t st);

@@ -206,6 +206,15 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
 #pragma unroll
                 for (int na = 0; na < R; ++na) x[na] = u2d(d64[(R * na + r) * C + c]);
             }
+            if (rs.fold) {                                 // + [c_l]_{q_i} * (P mod q_i): |x| < 2^40 + q
+                const u64* fr = rs.fold + (size_t)b * a.N + n2;
+                u64 fv[R];
+#pragma unroll
+                for (int na = 0; na < R; ++na) fv[na] = __ldg(fr + (size_t)(R * na + r) * N2);
+                const TWD fw = rs.scale[k];
+#pragma unroll
+                for (int na = 0; na < R; ++na) x[na] = __dadd_rn(x[na], mulc(u2d(fv[na]), fw, q));
+            }
             neg_fwd<R>(x, NEG, q);
             __syncthreads();                               // tile consumed: exchange in place
 #pragma unroll
@@ -463,6 +472,200 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
     cp_wait<0>();
 }
 
+// ------------------------------------------------------------------ row pass + KeyIP (a5 + a6)
+// ntt.h KipArgs.  Work items are (tile, i) with i over the ntr[k] transforms of the tile's
+// target (at least one item per tile: with beta = 1 a Q target has only its own-digit term);
+// the CTA walks its tiles in order, so the accumulator of item i > 0 is read back by the same
+// thread that stored it in item i - 1 (plain loads, not the non-coherent path).
+template <int R, int MINB, int U>
+__global__ void __launch_bounds__(RowCfg<R>::NT, MINB)
+k_ntt_row_kip(NttArgs a, TileMap tm, const __grid_constant__ KipArgs A) {
+    using CF = RowCfg<R>;
+    constexpr int RR = kC, NT = CF::NT, N2 = CF::N2;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int tid = threadIdx.x, rho = tid / R, r = tid % R;
+    const int N1 = a.N1, N = a.N;
+    TWD* sT = reinterpret_cast<TWD*>(smem_raw);
+    double* sD = reinterpret_cast<double*>(smem_raw + CF::NS * sizeof(TWD));
+
+    auto issue = [&](int t, int i) {
+        if (t < tm.total) {
+            int b, k, blk;
+            tm.decode(t, b, k, blk);
+            if (A.ntr[k] > 0) {
+                const TWD* ptab = a.tabd + (size_t)A.limb[k] * a.tab_stride;
+                for (int e = tid; e < CF::NS; e += NT) {
+                    int dd = e;
+                    if (e >= R / 2) {
+                        const int f = e - R / 2;
+                        dd = R / 2 + (f % R) * R + f / R;
+                    }
+                    cp16(sT + dd, ptab + a.L.rowf_cyc + e);
+                }
+                const double* g = A.tmp + b * A.tmp_bstride + (size_t)A.row[k][i] * N + (size_t)blk * RR * N2;
+                for (int e = tid; e < RR * N2 / 2; e += NT) cp16(sD + 2 * e, g + 2 * e);
+            }
+        }
+        cp_commit();
+    };
+    auto next = [&](int t, int i, int& tn, int& in) {
+        int b, k, blk;
+        tm.decode(t, b, k, blk);
+        const int items = A.ntr[k] > 0 ? A.ntr[k] : 1;
+        if (i + 1 < items) { tn = t; in = i + 1; } else { tn = t + gridDim.x; in = 0; }
+    };
+
+    int t = blockIdx.x, i = 0;
+    pdl_wait();
+    pdl_trigger();
+    issue(t, 0);
+    while (t < tm.total) {
+        int tn, in;
+        next(t, i, tn, in);
+        int b, k, blk;
+        tm.decode(t, b, k, blk);
+        const int row0 = blk * RR, nt = A.ntr[k], lid = A.limb[k];
+        // L2 prefetch: this item's key rows (consumed after the transform) and the next item's tile
+        const int j = nt > 0 ? A.dig[k][i] : -1;
+        const int jo = i == 0 ? A.own[k] : -1;
+        if (j >= 0)
+            for (int i2 = tid; i2 < N2; i2 += NT)
+                for (int c = 0; c < 2; ++c)
+                    pf_l2(A.evk_lo + ((size_t)(2 * j + c) * A.evk_limbs + lid) * N + row0 + (size_t)N1 * i2);
+        if (tn < tm.total) {
+            int b2, k2, blk2;
+            tm.decode(tn, b2, k2, blk2);
+            if (A.ntr[k2] > 0) {
+                const double* g = A.tmp + b2 * A.tmp_bstride + (size_t)A.row[k2][in] * N + (size_t)blk2 * RR * N2;
+                for (int e = tid; e < RR * N2 / 16; e += NT) pf_l2(g + 16 * e);
+            }
+        }
+        cp_wait<0>();
+        __syncthreads();
+        const u64* T = reinterpret_cast<const u64*>(sD);
+        if (nt > 0) {
+            const TWD* CYC = sT;
+            const double q = CYC[0].w, qinv = CYC[0].wq;
+            const TWD* TW2 = CYC + R / 2;
+            double* S = sD + rho * CF::XP;
+            double x[R];
+#pragma unroll
+            for (int na = 0; na < R; ++na) x[na] = sD[rho * N2 + R * na + r];
+            cyc_dif<R>(x, CYC, q);
+            __syncthreads();
+#pragma unroll
+            for (int ia = 0; ia < R; ++ia) S[ia + CF::EP * r] = mulc(x[BitRev<R>::of(ia)], TW2[ia * R + r], q);
+            __syncthreads();
+#pragma unroll
+            for (int nb = 0; nb < R; ++nb) x[nb] = S[r + CF::EP * nb];
+            cyc_dif<R>(x, CYC, q);
+            __syncthreads();
+            u64* Tw = reinterpret_cast<u64*>(sD);
+#pragma unroll
+            for (int ib = 0; ib < R; ++ib) Tw[swz(r + R * ib, rho)] = d2u(canon(x[BitRev<R>::of(ib)], q, qinv));
+            __syncthreads();
+        }
+        // epilogue: acc_c = (i > 0 || accumulate ? acc_c : 0) + x * evk_{j,c} (+ dhat * evk_{own,c})
+        {
+            const ModQ m = A.mods[lid];
+            const bool prev = i > 0 || A.accumulate;
+            const size_t kr = (size_t)A.evk_limbs * N;
+            const uint32_t* klo = A.evk_lo + ((size_t)(2 * (j < 0 ? 0 : j)) * A.evk_limbs + lid) * N;
+            const uint8_t* khi = A.evk_hi + ((size_t)(2 * (j < 0 ? 0 : j)) * A.evk_limbs + lid) * N;
+            const uint32_t* olo = A.evk_lo + ((size_t)(2 * (jo < 0 ? 0 : jo)) * A.evk_limbs + lid) * N;
+            const uint8_t* ohi = A.evk_hi + ((size_t)(2 * (jo < 0 ? 0 : jo)) * A.evk_limbs + lid) * N;
+            const u64* dsrc = A.d + b * A.d_bstride + (size_t)lid * N;
+            u64* acc0 = A.acc + b * A.acc_bstride + (size_t)k * N;
+            u64* acc1 = acc0 + A.acc_cstride;
+            static_assert((N2 * 8) % (NT * U) == 0, "epilogue rounds");
+#pragma unroll 1
+            for (int e0 = tid; e0 < N2 * 8; e0 += NT * U) {
+                uint2 kl0[U], kl1[U], ol0[U], ol1[U];
+                unsigned kh[U], oh[U];
+                uint4 p0[U], p1[U], dv[U];
+                size_t pos[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const int e = e0 + u * NT, i2 = e >> 3, p = e & 7;
+                    pos[u] = row0 + (size_t)N1 * i2 + 2 * p;
+                    if (j >= 0) {
+                        kl0[u] = __ldg(reinterpret_cast<const uint2*>(klo + pos[u]));
+                        kl1[u] = __ldg(reinterpret_cast<const uint2*>(klo + kr + pos[u]));
+                        kh[u] = (unsigned)__ldg(reinterpret_cast<const unsigned short*>(khi + pos[u])) |
+                                ((unsigned)__ldg(reinterpret_cast<const unsigned short*>(khi + kr + pos[u])) << 16);
+                    }
+                    if (jo >= 0) {
+                        ol0[u] = __ldg(reinterpret_cast<const uint2*>(olo + pos[u]));
+                        ol1[u] = __ldg(reinterpret_cast<const uint2*>(olo + kr + pos[u]));
+                        oh[u] = (unsigned)__ldg(reinterpret_cast<const unsigned short*>(ohi + pos[u])) |
+                                ((unsigned)__ldg(reinterpret_cast<const unsigned short*>(ohi + kr + pos[u])) << 16);
+                        if (A.galois) {                              // sigma_g(d), gathered
+                            const unsigned gg = A.galois, msk = (unsigned)N - 1;
+                            const unsigned s0 = (unsigned)(((unsigned long long)gg * pos[u] + (gg - 1) / 2) & msk);
+                            const u64 x0 = __ldg(dsrc + s0), x1 = __ldg(dsrc + ((s0 + gg) & msk));
+                            dv[u] = make_uint4((unsigned)x0, (unsigned)(x0 >> 32), (unsigned)x1, (unsigned)(x1 >> 32));
+                        } else {
+                            dv[u] = __ldg(reinterpret_cast<const uint4*>(dsrc + pos[u]));
+                        }
+                    }
+                    if (prev) {
+                        p0[u] = __ldcg(reinterpret_cast<const uint4*>(acc0 + pos[u]));   // ld.global.cg: coherent
+                        p1[u] = __ldcg(reinterpret_cast<const uint4*>(acc1 + pos[u]));
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const int e = e0 + u * NT, i2 = e >> 3, p = e & 7;
+                    u64 xv[2] = {0, 0}, dd[2] = {0, 0};
+                    if (nt > 0) {
+                        const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
+                        xv[0] = ((u64)v.y << 32) | v.x;
+                        xv[1] = ((u64)v.w << 32) | v.z;
+                    }
+                    if (jo >= 0) {
+                        dd[0] = ((u64)dv[u].y << 32) | dv[u].x;
+                        dd[1] = ((u64)dv[u].w << 32) | dv[u].z;
+                    }
+                    u64 rr[2][2];
+#pragma unroll
+                    for (int c = 0; c < 2; ++c) {
+#pragma unroll
+                        for (int h = 0; h < 2; ++h) {
+                            u64 hi = 0, lo = 0;
+                            if (j >= 0) {
+                                const uint2 kl = c ? kl1[u] : kl0[u];
+                                const u64 kv = (u64)(h ? kl.y : kl.x) | ((u64)((kh[u] >> (16 * c + 8 * h)) & 0xffu) << 32);
+                                mac128(hi, lo, xv[h], kv);
+                            }
+                            if (jo >= 0) {
+                                const uint2 ol = c ? ol1[u] : ol0[u];
+                                const u64 ov = (u64)(h ? ol.y : ol.x) | ((u64)((oh[u] >> (16 * c + 8 * h)) & 0xffu) << 32);
+                                mac128(hi, lo, dd[h], ov);
+                            }
+                            if (prev) {
+                                const uint4 pv = c ? p1[u] : p0[u];
+                                const u64 pw = h ? (((u64)pv.w << 32) | pv.z) : (((u64)pv.y << 32) | pv.x);
+                                lo += pw;
+                                hi += lo < pw;
+                            }
+                            rr[c][h] = barrett_reduce(hi, lo, m);
+                        }
+                    }
+                    *reinterpret_cast<uint4*>(acc0 + pos[u]) =
+                        make_uint4((unsigned)rr[0][0], (unsigned)(rr[0][0] >> 32), (unsigned)rr[0][1], (unsigned)(rr[0][1] >> 32));
+                    *reinterpret_cast<uint4*>(acc1 + pos[u]) =
+                        make_uint4((unsigned)rr[1][0], (unsigned)(rr[1][0] >> 32), (unsigned)rr[1][1], (unsigned)(rr[1][1] >> 32));
+                }
+            }
+        }
+        __syncthreads();
+        issue(tn, in);
+        t = tn;
+        i = in;
+    }
+    cp_wait<0>();
+}
+
 // ------------------------------------------------------------------ launchers
 
 // Pipeline depth / occupancy variant: 0 = 2 stages x 2 CTAs/SM, 1 = 1 stage x 3,
@@ -530,6 +733,43 @@ cudaError_t ntt_pass(bool col, const RowSet& rs, const NttArgs& a, int batch, bo
     switch (a.L.R) {
         case 8: return fwd ? launch_pass<8, true>(col, rs, a, batch, st, epi) : launch_pass<8, false>(col, rs, a, batch, st, epi);
         case 16: return fwd ? launch_pass<16, true>(col, rs, a, batch, st, epi) : launch_pass<16, false>(col, rs, a, batch, st, epi);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+// fused ModUp row pass + KeyIP: npos target positions x batch, 1 stage x 4 CTAs per SM
+cudaError_t ntt_row_kip(const NttArgs& a, const KipArgs& A, int npos, int batch, cudaStream_t st) {
+    if (npos == 0 || batch == 0) return cudaSuccess;
+    TileMap tm;
+    tm.batch = batch;
+    tm.tpr = a.N1 / kC;
+    tm.tpr_log = 0;
+    while ((1 << tm.tpr_log) < tm.tpr) ++tm.tpr_log;
+    tm.bmagic = batch > 1 ? (unsigned)((1ull << 32) / (unsigned)batch + 1) : 0u;
+    tm.total = tm.tpr * npos * batch;
+    auto go = [&](auto kern, int nt, size_t sm, int minb) -> cudaError_t {
+        static bool init = false;
+        if (!init) {
+            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            init = true;
+        }
+        int grid = minb * a.num_sms;
+        if (grid > tm.total) grid = tm.total;
+        return launch_k(kern, dim3(grid), dim3(nt), sm, st, a, tm, A);
+    };
+    switch (a.L.R) {
+        case 8: return go(k_ntt_row_kip<8, 4, 2>, RowCfg<8>::NT, RowCfg<8>::STAGE, 4);
+        case 16: {
+            // occupancy x loads-in-flight variant (NEO_KIP_CFG): 0 = 4 CTAs x 1 chunk, 1 = 3 x 2, 2 = 2 x 4
+            static int v = -1;
+            if (v < 0) {
+                const char* e = std::getenv("NEO_KIP_CFG");
+                v = e ? std::atoi(e) : 0;
+            }
+            if (v == 1) return go(k_ntt_row_kip<16, 3, 2>, RowCfg<16>::NT, RowCfg<16>::STAGE, 3);
+            if (v == 2) return go(k_ntt_row_kip<16, 2, 4>, RowCfg<16>::NT, RowCfg<16>::STAGE, 2);
+            return go(k_ntt_row_kip<16, 4, 1>, RowCfg<16>::NT, RowCfg<16>::STAGE, 4);
+        }
         default: return cudaErrorInvalidValue;
     }
 }

@@ -46,6 +46,34 @@ struct RowEpi {
     TW post[64];          // per row k: q_l^-1 mod q_k
 };
 
+// KeyIP fused into the forward row pass of the ModUp NTT (a5 + a6): one tile = 16 rows x N2
+// of ONE target limb (position k of PQ_l) of one batch entry; the CTA transforms that tile of
+// each digit j whose ModUp output reaches k (ntr[k] of them, column-pass intermediates in tmp)
+// and accumulates acc_c[k] = sum_j NTT(up_j[k]) * evk_{j,c}[k] (+ dhat[k] * evk_{own,c}[k] for
+// the digit that owns k) in its epilogue, so the ModUp outputs never reach HBM (Alg. 3).
+constexpr int KIP_MAX_EXT = 64;
+constexpr int KIP_MAX_BETA = 12;
+struct KipArgs {
+    const double* tmp;          // column-pass output [B][rows][N] (lazy doubles)
+    long long tmp_bstride;
+    const u64* d;               // KS input [B][l+1][N] in NTT form (the own-digit term)
+    long long d_bstride;
+    unsigned galois;            // != 0: the own-digit term reads sigma_g(d) (fused HROTATE)
+    const uint32_t* evk_lo;     // [dnum][2][evk_limbs][N]
+    const uint8_t* evk_hi;
+    int evk_limbs;
+    u64* acc;                   // [B][2][E][N]
+    long long acc_bstride, acc_cstride;
+    const ModQ* mods;
+    int accumulate;             // acc += (neo_hrot_sum's giant steps)
+    int limb[KIP_MAX_EXT];      // position -> limb id
+    signed char ntr[KIP_MAX_EXT];                // transformed digits reaching position k
+    signed char own[KIP_MAX_EXT];                // digit owning position k, or -1
+    unsigned char dig[KIP_MAX_EXT][KIP_MAX_BETA];   // digit of the i-th transform of k
+    short row[KIP_MAX_EXT][KIP_MAX_BETA];           // its row in tmp
+};
+cudaError_t ntt_row_kip(const NttArgs& a, const KipArgs& A, int npos, int batch, cudaStream_t st);
+
 // One pass over batch x rs.n limb rows.  Forward NTT = column pass (src -> tmp) then row
 // pass (tmp -> dst); inverse = row pass then column pass.  src and dst of one pass must
 // not overlap.
