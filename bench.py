@@ -821,28 +821,31 @@ def run_neo(args):
         torch.cuda.empty_cache()
 
     # SURVEY §8(f) row 1 (Table 8 / Fig. 16 analogue): one key-switch at Set-C (N=2^16, L=35,
-    # dnum=9, alpha~=5; WordSize_T=36 -> 10 T primes, reading K6) with the KLSS key and with the
-    # Hybrid key of the same parameters, B = 1 and B = 8 per GPU, CUDA events, max over ranks.
-    # Keys and inputs are uniform residues < 2^35 made on the device (timing is data-independent).
+    # dnum=9, alpha~=5) with the KLSS key at WordSize_T = 48 (Table 4 as printed, L511: 8 T primes)
+    # and at WordSize_T = 36 (10 T primes), and with the Hybrid key of the same parameters, B = 1
+    # and B = 8 per GPU, CUDA events, max over ranks.  Keys and inputs are uniform residues < 2^35
+    # made on the device (timing is data-independent).
     klss_block = None
     if not args.no_klss:
-        cctx = neo.Context(16, 36, 4, 9, alpha_t=5, device=local)
         gen = torch.Generator(device="cuda")
         gen.manual_seed(seed + 91)
         rnd = lambda *shape: torch.randint(0, 1 << 35, shape, dtype=torch.int64, device="cuda",
                                            generator=gen).view(torch.uint64)
         bt = -(-(36 + 4) // 5)
-        keys = {"klss": neo.EvalKey(cctx, rnd(2, bt, 9, cctx.alpha_p, N), klss=True),
-                "hybrid": neo.EvalKey(cctx, rnd(9, 2, 40, N))}
-        klss_block = {"config": "Set-C (Table 4): N=2^16, L=35, dnum=9, alpha~=5, WordSize_T=36 "
-                                f"(alpha'={cctx.alpha_p} T primes), level 35",
+        ctxs = {48: neo.Context(16, 36, 4, 9, alpha_t=5, word_bits_t=48, device=local),
+                36: neo.Context(16, 36, 4, 9, alpha_t=5, device=local)}
+        keys = {"klss_t48": (ctxs[48], neo.EvalKey(ctxs[48], rnd(2, bt, 9, ctxs[48].alpha_p, N), klss=True)),
+                "klss_t36": (ctxs[36], neo.EvalKey(ctxs[36], rnd(2, bt, 9, ctxs[36].alpha_p, N), klss=True)),
+                "hybrid": (ctxs[48], neo.EvalKey(ctxs[48], rnd(9, 2, 40, N)))}
+        klss_block = {"config": "Set-C (Table 4): N=2^16, L=35, dnum=9, alpha~=5, level 35; KLSS with "
+                                f"WordSize_T=48 (alpha'={ctxs[48].alpha_p}) and 36 (alpha'={ctxs[36].alpha_p})",
                       "unit": "KS/s", "timing": "CUDA events around 20 neo_keyswitch calls after 3 warm-ups"}
         for Bk in (1, 8):
             dk = rnd(Bk, Lq, N)
             o0, o1 = torch.empty_like(dk), torch.empty_like(dk)
-            wsk = torch.empty(cctx.workspace_size(neo.NEO_OP_KEYSWITCH, LEVEL, Bk) // 8, dtype=torch.uint64,
-                              device="cuda")
-            for meth, key in keys.items():
+            for meth, (cctx, key) in keys.items():
+                wsk = torch.empty(cctx.workspace_size(neo.NEO_OP_KEYSWITCH, LEVEL, Bk) // 8, dtype=torch.uint64,
+                                  device="cuda")
                 for _ in range(3):
                     neo.neo_keyswitch(cctx, key, dk, LEVEL, o0, o1, Bk, wsk)
                 torch.cuda.synchronize()
@@ -859,9 +862,11 @@ def run_neo(args):
                     dist.all_reduce(t, op=dist.ReduceOp.MAX)
                     kms = float(t.item())
                 klss_block[f"{meth}_B{Bk}"] = {"ms_per_call": round(kms, 4), "value": Bk * world / (kms / 1e3)}
-            del dk, o0, o1, wsk
+                del wsk
+            del dk, o0, o1
         del keys
-        cctx.close()
+        for cctx in ctxs.values():
+            cctx.close()
         torch.cuda.empty_cache()
 
     # SURVEY §8(f) row 2 / BASELINE metric "bootstrap ms": one sparse-slot bootstrapping

@@ -70,9 +70,12 @@ typedef struct {
     const uint64_t* q;
     const uint64_t* p;
     int32_t alpha_t;     /* KLSS key-decomposition group size alpha~ (Table 4); 0 = Hybrid only.
-                          * > 0 adds alpha' T primes (WordSize_T = word_bits, the Z4 rule continued
-                          * after p; alpha' from Eq. 4, reading K3) and the KLSS
-                          * tables; requires generated primes (q = p = NULL). */
+                          * > 0 adds alpha' T primes (alpha' from Eq. 4, reading K3)
+                          * and the KLSS tables; requires generated primes (q = p = NULL). */
+    int32_t word_bits_t; /* WordSize_T of the T primes (Table 4: 48 for Set-C), used when
+                          * alpha_t > 0: 0 or word_bits = the Z4 rule continued after p; up to 48 =
+                          * the Z4 rule at word_bits_t bits (reading K6).  Values outside
+                          * [word_bits, 48] fail with NEO_EUNSUPPORTED. */
 } neo_params_desc;
 
 /* Build the context: primes, psi, NTT twiddle tables, BConv tables for every

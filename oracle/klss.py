@@ -28,8 +28,10 @@ K4 Recover Limbs = the exact centred CRT lift from T, reduced modulo each limb o
    KeySwitch bit for bit (pinned in tests/test_oracle_klss.py).
 K5 ModDown on the recovered (coefficient-form) limbs: (acc_Q - BConv_{P->Q}(acc_P)) P^-1,
    then NTT over Q_l (Z9; by linearity identical to Hybrid's NTT-domain combine).
-K6 T primes: WordSize_T = 36 (Fig. 16 evaluates 36, 48, 64; this build's residue arithmetic
-   is 36-bit), the Z4 rule continued after the Q and P primes.
+K6 T primes: the Z4 rule at WordSize_T bits (Table 4: 48 for Set-C; Fig. 16 evaluates
+   36, 48, 64).  When WordSize_T equals the Q/P word size the sequence continues after the Q
+   and P primes; otherwise it starts afresh at the top of the WordSize_T range (disjoint from
+   Q and P by bit length).
 """
 from __future__ import annotations
 
@@ -53,11 +55,14 @@ class KlssParams:
 
     def __post_init__(self):
         b = self.base
-        assert self.word_bits_t == b.word_bits, "K6: T primes continue the Z4 sequence (same width)"
+        assert b.word_bits <= self.word_bits_t <= 64
         ext = list(range(b.num_q)) + b.p_ids                              # PQ_L limb ids
         self.groups = [ext[i:i + self.alpha_t] for i in range(0, len(ext), self.alpha_t)]
         self.bound = self.ip_bound()
-        cand = ckks.gen_primes(b.log_n, self.word_bits_t, b.num_q + b.num_p + 64)[b.num_q + b.num_p:]
+        if self.word_bits_t == b.word_bits:                               # K6
+            cand = ckks.gen_primes(b.log_n, self.word_bits_t, b.num_q + b.num_p + 64)[b.num_q + b.num_p:]
+        else:
+            cand = ckks.gen_primes(b.log_n, self.word_bits_t, 64)
         T, k = 1, 0
         while T <= 4 * self.bound:                                        # K3 (Eq. 4 + guard bit)
             T *= cand[k]
@@ -96,6 +101,17 @@ def set_c_t36() -> KlssParams:
     """Table 4 Set-C (L504-517): N=2^16, L=35, WordSize 36, dnum=9 (P: alpha = 4 limbs, Z3),
     alpha~ = 5, with WordSize_T = 36 (K6)."""
     return KlssParams(ckks.Params(16, 36, 4, 9), alpha_t=5)
+
+
+def set_c() -> KlssParams:
+    """Table 4 Set-C as printed (L504-517): N=2^16, L=35, WordSize 36, WordSize_T = 48, dnum=9,
+    alpha~ = 5 (P: alpha = 4 limbs, Z3)."""
+    return KlssParams(ckks.Params(16, 36, 4, 9), alpha_t=5, word_bits_t=48)
+
+
+def tiny48() -> KlssParams:
+    """tiny() with 48-bit T primes (WordSize_T = 48, K6)."""
+    return KlssParams(ckks.Params(12, 6, 2, 3), alpha_t=3, word_bits_t=48)
 
 
 def tiny() -> KlssParams:

@@ -551,6 +551,9 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     const int bt = (int)c->klss_groups.size(), nl = c->num_q + c->num_p;
     if (beta > KLSS_MAX_BETA || bt > KLSS_MAX_GROUPS || c->alpha_t > KLSS_MAX_OUT_G)
         FAIL(NEO_EUNSUPPORTED, "KLSS: too many digits, groups (<= 8) or limbs per group (<= 16)");
+    const bool wide = c->word_bits_t > 40;     // 48-bit T words: 6-byte BConv constants, 64-bit IP / Recover
+    if (wide && !c->use_tc) FAIL(NEO_EUNSUPPORTED, "KLSS with WordSize_T > 40 needs the tensor-core BConv");
+    if ((k->hi_bytes == 2) != wide) FAIL(NEO_EINVAL, "KLSS key packed for another WordSize_T");
     u64 *y = ws + Ly.y, *up = ws + Ly.up, *acc = ws + Ly.acc, *rec = ws + Ly.rec, *conv = ws + Ly.conv,
         *diff = ws + Ly.diff, *tmp = ws + Ly.tmp;
     int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
@@ -627,7 +630,7 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     }
     R.first[ng] = no;
     I.n_groups = R.n_groups = ng;
-    LAUNCH(PK_KEYIP, st, launch_klss_ip(I, B, st));
+    LAUNCH(PK_KEYIP, st, wide ? launch_klss_ip48(I, B, st) : launch_klss_ip(I, B, st));
     // 5. INTT over T of the 2 * (present groups) * alpha' rows (in place, coefficient form)
     int nr = 0;
     for (int cc = 0; cc < 2; ++cc)
@@ -642,7 +645,7 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     // per-tile pipeline cost dominates, measured 0.136 vs 0.102 ms per KS at Set-C); NEO_KLSS_REC=tc
     // selects the tensor-core conversion with the centred-correction column
     static const bool rec_tc = [] { const char* e = std::getenv("NEO_KLSS_REC"); return e && std::string(e) == "tc"; }();
-    const bool use_rec_tc = c->use_tc && rec_tc;
+    const bool use_rec_tc = c->use_tc && rec_tc && c->klss_rec_tc_ok;
     TWD tsc[NEO_HOST_ROWS];                // tensor-core Recover: [That_k^-1]_{t_k} folded into the INTT
     if (use_rec_tc)
         for (int r = 0; r < nr; ++r) tsc[r] = c->klss_rec_tc[l][I.group[0]].qhat_inv[r % ap];
@@ -678,7 +681,7 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
             }
         if (M.njobs) LAUNCH(PK_COMBINE, st, launch_bconv_tc(M, N, B, c->num_sms, st));
     } else {
-        LAUNCH(PK_COMBINE, st, launch_klss_recover(R, B, st));
+        LAUNCH(PK_COMBINE, st, wide ? launch_klss_recover48(R, B, st) : launch_klss_recover(R, B, st));
     }
     // 7. ModDown BConv P -> Q_l on the recovered (coefficient-form) P limbs, batch 2B
     {
@@ -877,6 +880,8 @@ neo_status neo_params_create(const neo_params_desc* desc, neo_ctx** out) {
     if (alpha > BC_MAX_IN) FAIL(NEO_EUNSUPPORTED, "alpha must be <= 16");
     if (desc->dnum > KS_MAX_BETA) FAIL(NEO_EUNSUPPORTED, "dnum must be <= 12");
     if ((desc->q == nullptr) != (desc->p == nullptr)) FAIL(NEO_EINVAL, "give both q and p or neither");
+    if (desc->alpha_t > 0 && desc->word_bits_t != 0 && (desc->word_bits_t < desc->word_bits || desc->word_bits_t > 48))
+        FAIL(NEO_EUNSUPPORTED, "word_bits_t must be 0 or in [word_bits, 48]");
     neo_ctx* c = new (std::nothrow) neo_ctx();
     if (!c) FAIL(NEO_ENOMEM, "host allocation failed");
     static std::atomic<unsigned long long> next_uid{0};
@@ -1141,14 +1146,17 @@ neo_status neo_evk_create_klss(const neo_ctx* c, const uint64_t* ekey, neo_evk**
     k->ctx = c;
     k->klss = 1;
     const size_t n = (size_t)2 * c->klss_groups.size() * c->dnum * c->num_t * c->N;
-    if (cudaMalloc(&k->lo, n * sizeof(uint32_t)) != cudaSuccess || cudaMalloc(&k->hi, n) != cudaSuccess) {
+    k->hi_bytes = c->word_bits_t > 40 ? 2 : 1;             // 48-bit T residues: 6 bytes per key word
+    if (cudaMalloc(&k->lo, n * sizeof(uint32_t)) != cudaSuccess || cudaMalloc(&k->hi, n * k->hi_bytes) != cudaSuccess) {
         neo_evk_destroy(k);
         FAIL(NEO_ENOMEM, "cudaMalloc of the KLSS key failed");
     }
     // the key may have been written on any of the caller's streams (e.g. a non-blocking torch
     // stream, which the legacy stream does not wait for): finish all device work first
     cudaError_t e = cudaDeviceSynchronize();
-    if (e == cudaSuccess) e = launch_pack5(ekey, k->lo, k->hi, n, nullptr);
+    if (e == cudaSuccess)
+        e = k->hi_bytes == 2 ? launch_pack6(ekey, k->lo, reinterpret_cast<uint16_t*>(k->hi), n, nullptr)
+                             : launch_pack5(ekey, k->lo, k->hi, n, nullptr);
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
     if (e != cudaSuccess) {
         neo_evk_destroy(k);

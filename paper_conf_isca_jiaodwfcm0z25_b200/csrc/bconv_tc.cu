@@ -72,7 +72,7 @@ static_assert(kSlots * kSlotCols == 512, "TMEM plan");
 // A tile of 36 targets is 4 parts, one per set.  Per-job / per-target constants and the tile
 // schedule are staged in shared memory during setup (register-indexed reads of the large
 // parameter block miss the constant cache on the critical path).
-template <bool kPre, bool kLazy, class LoadB, bool kCorr = false>
+template <bool kPre, bool kLazy, class LoadB, bool kCorr = false, int NB = 5>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
                                               int tiles_per_entry, int batch, int exp,
                                               const CUtensorMap* tmaps = nullptr, const int* use_tmap = nullptr,
@@ -263,15 +263,25 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                 // (D0 + 2^8 D1) + 2^16 D2 + 2^24 D3 as a 64-bit word, then D4 and the exponent of
                 // 2^52 added to the high word (no carry: hi + D4 < 2^20).
 #pragma unroll
-                for (int u = 0; u < BCTC_PART_J; ++u) {
+                for (int u = 0; u < (NB == 5 ? BCTC_PART_J : BCTC_PART_ROWS / 6); ++u) {
                     const TgtC& C = tg[u];
-                    const uint32_t* D = &v[5 * u];
+                    const uint32_t* D = &v[NB * u];
                     u64 w = (u64)(D[0] + (D[1] << 8)) + (u64)D[2] * 65536ull;
                     w += (u64)D[3] * 16777216ull;
-                    const double Vd = __dadd_rn(__hiloint2double((int)((uint32_t)(w >> 32) + D[4] + 0x43300000u),
-                                                                 (int)(uint32_t)w), -kTwo52);
-                    const double qf = __dadd_rn(__fma_rn(Vd, C.tinv, kMagic), -kMagic);
-                    double r = __fma_rn(-qf, C.t, Vd);                 // V mod t, |r| <= t/2 + 1 (exact)
+                    double r;
+                    if (NB == 5) {
+                        const double Vd = __dadd_rn(__hiloint2double((int)((uint32_t)(w >> 32) + D[4] + 0x43300000u),
+                                                                     (int)(uint32_t)w), -kTwo52);
+                        const double qf = __dadd_rn(__fma_rn(Vd, C.tinv, kMagic), -kMagic);
+                        r = __fma_rn(-qf, C.t, Vd);                    // V mod t, |r| <= t/2 + 1 (exact)
+                    } else {
+                        // 48-bit targets: V = sum_b 2^(8b) D_b < 2^62 exactly in 64 bits; the quotient
+                        // rint(V / t) < 2^15 from an FP64 estimate (off by < 2^-30), the remainder in
+                        // integers: |r| <= t/2 + 1 < 2^48, exact as a double
+                        w += ((u64)D[4] << 32) + ((u64)D[5] << 40);
+                        const double qf = rint(__dmul_rn(__ull2double_rn(w), C.tinv));
+                        r = (double)(long long)(w - (u64)qf * (u64)C.t);
+                    }
                     if (!kLazy) r = __dadd_rn(r, r < 0.0 ? C.t : 0.0);
                     const u64 val = kLazy ? (u64)__double_as_longlong(r) : d2u(r);
                     const uint32_t ok = u < nt;
@@ -347,12 +357,12 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     if (warp == 0) tc::tmem_dealloc(tmem, kSlots * kSlotCols);
 }
 
-template <bool kPre, bool kLazy, bool kCorr = false>
+template <bool kPre, bool kLazy, bool kCorr = false, int NB = 5>
 __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_g(const __grid_constant__ BConvMulti M, int N, int tiles_per_entry, int batch, int exp) {
     auto lb = [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; };
-    bconv_tc_body<kPre, kLazy, decltype(lb), kCorr>(M.P, M.io, M.njobs, lb, N, tiles_per_entry, batch, exp, M.tmap,
-                                                   M.use_tmap, M.dbg);
+    bconv_tc_body<kPre, kLazy, decltype(lb), kCorr, NB>(M.P, M.io, M.njobs, lb, N, tiles_per_entry, batch, exp,
+                                                       M.tmap, M.use_tmap, M.dbg);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
@@ -372,6 +382,8 @@ static void bconv_tc_init() {
         cudaFuncSetAttribute(k_bconv_tc_g<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         cudaFuncSetAttribute(k_bconv_tc_p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemAlloc);
         cudaFuncSetAttribute(k_bconv_tc_g<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)kSmemAlloc);
+        cudaFuncSetAttribute(k_bconv_tc_g<true, true, false, 6>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)kSmemAlloc);
         init = true;
     }
@@ -427,6 +439,12 @@ cudaError_t launch_bconv_tc(const BConvMulti& M0, int N, int batch, int num_sms,
     if (M.centred) {                       // KLSS Recover Limbs: pre-scaled input, canonical output only
         if (!M.pre_scaled || M.lazy_out) return cudaErrorInvalidValue;
         k = k_bconv_tc_g<true, false, true>;
+    }
+    for (int j = 0; j < M.njobs; ++j)
+        if ((M.P[j].nb == 6) != (M.P[0].nb == 6)) return cudaErrorInvalidValue;
+    if (M.P[0].nb == 6) {                  // 48-bit targets (KLSS ModUp to WordSize_T = 48)
+        if (!M.pre_scaled || !M.lazy_out || M.centred) return cudaErrorInvalidValue;
+        k = k_bconv_tc_g<true, true, false, 6>;
     }
     return launch_k(k, dim3(grid), dim3(kThreads), kSmemAlloc, st, M, N, tiles_per_entry, batch, exp);
 }

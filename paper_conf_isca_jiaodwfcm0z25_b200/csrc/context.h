@@ -44,7 +44,8 @@ constexpr int BCTC_MAX_PARTS = (BCTC_MAX_OUT + BCTC_PART_J - 1) / BCTC_PART_J;  
 struct BConvTC {
     int n_in, n_out;
     int nparts, J;                  // targets split in nparts jobs of J (last may be shorter)
-    int ncols;                      // MMA N per job = round_up(5 J, 16) <= 48
+    int ncols;                      // MMA N per job = round_up(nb J, 16) <= 48
+    int nb;                         // bytes per target in B: 5 (targets < 2^40) or 6 (48-bit T primes)
     double qin[BCTC_MAX_IN], qinv_in[BCTC_MAX_IN];
     TWD qhat_inv[BCTC_MAX_IN];      // [qhat_i^-1]_{q_i}
     double t[BCTC_MAX_OUT], tinv[BCTC_MAX_OUT];
@@ -101,6 +102,8 @@ struct neo_ctx {
     std::vector<TW> ds_qlinv_m;
     // KLSS (alpha_t > 0): T primes are limb ids num_q+num_p .. +num_t-1
     int alpha_t = 0, num_t = 0;
+    int word_bits_t = 0;                                   // WordSize_T of the T primes (Table 4; 36 or 48)
+    bool klss_rec_tc_ok = true;                            // tensor-core Recover needs T primes < 2^40
     std::vector<std::vector<int>> klss_groups;             // [i] limb ids of PQ_L in group i
     std::vector<std::vector<neo::BConvTab>> klss_up;       // [l][j] digit -> T (CUDA-core control)
     std::vector<std::vector<neo::BConvTC>> klss_up_tc;     // [l][j] digit -> T (tensor cores)
@@ -125,4 +128,5 @@ struct neo_evk {
     uint8_t* hi = nullptr;
     uint32_t galois = 0;                  // hoisted rotation keys: the key is stored as sigma_{g^-1}(evk_g)
     int klss = 0;                         // KLSS key: planes are [2][beta~][dnum][alpha'][N] over T
+    int hi_bytes = 1;                     // bytes per residue in the hi plane: 1 (5-byte key) or 2 (48-bit T: 6 bytes)
 };

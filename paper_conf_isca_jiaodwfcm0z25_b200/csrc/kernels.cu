@@ -476,6 +476,17 @@ k_pack5(const u64* __restrict__ in, uint32_t* __restrict__ lo, uint8_t* __restri
     }
 }
 
+// 6-byte packing (48-bit KLSS T residues): low 32 bits and a 16-bit plane
+__global__ void __launch_bounds__(256)
+k_pack6(const u64* __restrict__ in, uint32_t* __restrict__ lo, uint16_t* __restrict__ hi, size_t n) {
+    pdl_wait();
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+        const u64 v = in[i];
+        lo[i] = (uint32_t)v;
+        hi[i] = (uint16_t)(v >> 32);
+    }
+}
+
 // ------------------------------------------------------------------ 36-bit wire format
 // n residues < 2^36 as [4n bytes: u32 low words][n/2 bytes: byte k = hi4(2k) | hi4(2k+1) << 4]
 // (4.5 bytes per residue against 8: the host<->device copies of neo_wire_pack / _unpack).
@@ -556,6 +567,9 @@ cudaError_t launch_ds_corr(const DsArgs& A, int bc, cudaStream_t st) {
 }
 cudaError_t launch_pack5(const u64* in, uint32_t* lo, uint8_t* hi, size_t n, cudaStream_t st) {
     return launch_k(k_pack5, dim3(4096), dim3(256), 0, st, in, lo, hi, n);
+}
+cudaError_t launch_pack6(const u64* in, uint32_t* lo, uint16_t* hi, size_t n, cudaStream_t st) {
+    return launch_k(k_pack6, dim3(4096), dim3(256), 0, st, in, lo, hi, n);
 }
 
 static inline dim3 g1(int N) { return dim3((N + 255) / 256); }

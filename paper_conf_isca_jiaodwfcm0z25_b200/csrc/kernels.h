@@ -130,5 +130,6 @@ cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int row
 cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st);
 cudaError_t launch_rescale_combine(const RescaleArgs& A, int bc, cudaStream_t st);
 cudaError_t launch_pack5(const u64* in, uint32_t* lo, uint8_t* hi, size_t n, cudaStream_t st);
+cudaError_t launch_pack6(const u64* in, uint32_t* lo, uint16_t* hi, size_t n, cudaStream_t st);
 
 }  // namespace neo

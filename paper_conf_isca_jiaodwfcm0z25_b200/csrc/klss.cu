@@ -67,6 +67,104 @@ k_klss_ip(const __grid_constant__ KlssIpArgs A, int batch) {
     }
 }
 
+// WordSize_T = 48 (Table 4 Set-C, L511): residues and key words < 2^48, 64-bit products
+// (IMAD.WIDE pairs) into a 128-bit sum; pairs of products (< 2^97) are folded through the
+// Barrett reduction (valid for X < 2^98, q < 2^48: common.cuh) with the running remainder.
+NEO_DEV void mac2_reduce(u64& r, u64 x0, u64 e0, u64 x1, u64 e1, ModQ m) {
+    u64 hi = 0, lo = r;
+    mac128(hi, lo, x0, e0);
+    mac128(hi, lo, x1, e1);
+    r = barrett_reduce(hi, lo, m);
+}
+
+template <int BETA>
+__global__ void __launch_bounds__(256, 2)
+k_klss_ip48(const __grid_constant__ KlssIpArgs A, int batch) {
+    pdl_wait();
+    const int gi = threadIdx.y;
+    if (gi >= A.n_groups) return;
+    const int n = blockIdx.x * KLSS_IP_W + threadIdx.x;
+    const int k = blockIdx.y, i = A.group[gi];
+    const ModQ m = A.mods[A.t0 + k];
+    const size_t NK = (size_t)A.alpha_p * A.N;
+    const size_t col = (size_t)k * A.N + n;
+    const uint16_t* hi16 = reinterpret_cast<const uint16_t*>(A.key_hi);
+    u64 e[2][BETA];
+#pragma unroll
+    for (int c = 0; c < 2; ++c) {
+        const size_t kb = (size_t)(c * A.beta_t + i) * A.dnum * NK + col;
+#pragma unroll
+        for (int j = 0; j < BETA; ++j) {
+            const size_t o = kb + (size_t)j * NK;
+            e[c][j] = (u64)A.key_lo[o] | ((u64)hi16[o] << 32);
+        }
+    }
+    for (int b = 0; b < batch; ++b) {
+        const u64* up = A.up + (size_t)b * A.beta * NK + col;
+        u64 x[BETA];
+#pragma unroll
+        for (int j = 0; j < BETA; ++j) x[j] = up[(size_t)j * NK];
+        u64 r0 = 0, r1 = 0;
+#pragma unroll
+        for (int j = 0; j < BETA; j += 2) {
+            const u64 x1 = j + 1 < BETA ? x[j + 1] : 0;
+            mac2_reduce(r0, x[j], e[0][j], x1, j + 1 < BETA ? e[0][j + 1] : 0, m);
+            mac2_reduce(r1, x[j], e[1][j], x1, j + 1 < BETA ? e[1][j + 1] : 0, m);
+        }
+        u64* acc = A.acc + (size_t)(b * 2) * A.beta_t * NK + (size_t)i * NK + col;
+        acc[0] = r0;
+        acc[(size_t)A.beta_t * NK] = r1;
+    }
+}
+
+// Recover Limbs with 48-bit T primes: as k_klss_recover, the products y_k [That_k]_p
+// (< 2^84) summed in 128 bits (alpha' <= 16 terms < 2^88) and Barrett-reduced mod p.
+template <int AP>
+__global__ void __launch_bounds__(256)
+k_klss_recover48(const __grid_constant__ KlssRecArgs A) {
+    pdl_wait();
+    const int n = blockIdx.x * blockDim.x + threadIdx.x;
+    const int gi = blockIdx.y >> 1, c = blockIdx.y & 1, b = blockIdx.z;
+    const RecTab& R = *A.tab;
+    const int o0 = A.first[gi], no = A.first[gi + 1] - o0;
+    __shared__ u64 tc[KLSS_MAX_OUT_G][AP];                     // this group's [That_k]_p
+    __shared__ TW tT[KLSS_MAX_OUT_G];                          // [T]_p
+    __shared__ ModQ tm[KLSS_MAX_OUT_G];
+    __shared__ int tpos[KLSS_MAX_OUT_G];
+    for (int e = threadIdx.x; e < no * AP; e += blockDim.x) {
+        const int ro = e / AP, k = e - ro * AP, p = A.out_id[o0 + ro];
+        tc[ro][k] = R.that_p[p][k].w;
+        if (k == 0) {
+            tT[ro] = R.T_p[p];
+            tm[ro] = A.mods[p];
+            tpos[ro] = A.out_pos[o0 + ro];
+        }
+    }
+    __syncthreads();
+    if (n >= A.N) return;
+    const size_t NK = (size_t)AP * A.N;
+    const u64* a = A.acc + ((size_t)(b * 2 + c) * A.beta_t + A.group[gi]) * NK + n;
+    u64 y[AP];
+#pragma unroll
+    for (int k = 0; k < AP; ++k) y[k] = a[(size_t)k * A.N];        // all loads in flight first
+    double s = 0.0;
+#pragma unroll
+    for (int k = 0; k < AP; ++k) {
+        y[k] = shoup(y[k], R.that_inv[k], A.mods[A.t0 + k].q);     // y_k = [a_k That_k^-1]_{t_k}
+        s = __fma_rn((double)y[k], R.tinv[k], s);
+    }
+    const u64 u = (u64)__double2ll_rn(s);
+    u64* out = A.rec + (size_t)(b * 2 + c) * A.E * A.N + n;
+#pragma unroll 1
+    for (int ro = 0; ro < no; ++ro) {
+        u64 hi = 0, lo = 0;
+#pragma unroll
+        for (int k = 0; k < AP; ++k) mac128(hi, lo, y[k], tc[ro][k]);
+        const ModQ m = tm[ro];
+        out[(size_t)tpos[ro] * A.N] = sub_mod(barrett_reduce(hi, lo, m), shoup(u, tT[ro], m.q), m.q);
+    }
+}
+
 // Recover Limbs: x = the centred lift of acc from T (|x| < T/4 by Eq. 4 + guard bit, K3):
 //   y_k = [a_k That_k^-1]_{t_k};  X = sum_k y_k That_k = x + u T exactly, u = rint(sum_k y_k / t_k)
 //   (the FP64 sum is within 2^-44 of X / T, and |x / T| < 1/4, so the rounding is exact);
@@ -145,6 +243,27 @@ cudaError_t launch_klss_ip(const KlssIpArgs& A, int batch, cudaStream_t st) {
         NEO_IP_CASE(1) NEO_IP_CASE(2) NEO_IP_CASE(3) NEO_IP_CASE(4) NEO_IP_CASE(5) NEO_IP_CASE(6)
         NEO_IP_CASE(7) NEO_IP_CASE(8) NEO_IP_CASE(9) NEO_IP_CASE(10) NEO_IP_CASE(11) NEO_IP_CASE(12)
 #undef NEO_IP_CASE
+        default: return cudaErrorInvalidValue;
+    }
+}
+cudaError_t launch_klss_ip48(const KlssIpArgs& A, int batch, cudaStream_t st) {
+    const dim3 g(A.N / KLSS_IP_W, A.alpha_p), blk(KLSS_IP_W, 256 / KLSS_IP_W);
+    switch (A.beta) {
+#define NEO_IP_CASE(B) case B: return launch_k(k_klss_ip48<B>, g, blk, 0, st, A, batch);
+        NEO_IP_CASE(1) NEO_IP_CASE(2) NEO_IP_CASE(3) NEO_IP_CASE(4) NEO_IP_CASE(5) NEO_IP_CASE(6)
+        NEO_IP_CASE(7) NEO_IP_CASE(8) NEO_IP_CASE(9) NEO_IP_CASE(10) NEO_IP_CASE(11) NEO_IP_CASE(12)
+#undef NEO_IP_CASE
+        default: return cudaErrorInvalidValue;
+    }
+}
+cudaError_t launch_klss_recover48(const KlssRecArgs& A, int batch, cudaStream_t st) {
+    const dim3 g((A.N + 255) / 256, 2 * A.n_groups, batch);
+    switch (A.alpha_p) {
+#define NEO_REC_CASE(K) case K: return launch_k(k_klss_recover48<K>, g, dim3(256), 0, st, A);
+        NEO_REC_CASE(2) NEO_REC_CASE(3) NEO_REC_CASE(4) NEO_REC_CASE(5) NEO_REC_CASE(6) NEO_REC_CASE(7)
+        NEO_REC_CASE(8) NEO_REC_CASE(9) NEO_REC_CASE(10) NEO_REC_CASE(11) NEO_REC_CASE(12) NEO_REC_CASE(13)
+        NEO_REC_CASE(14) NEO_REC_CASE(15) NEO_REC_CASE(16)
+#undef NEO_REC_CASE
         default: return cudaErrorInvalidValue;
     }
 }

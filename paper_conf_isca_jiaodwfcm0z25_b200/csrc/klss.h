@@ -51,6 +51,9 @@ struct KlssDiffArgs {
 
 cudaError_t launch_klss_ip(const KlssIpArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_klss_recover(const KlssRecArgs& A, int batch, cudaStream_t st);
+// WordSize_T = 48 variants (64-bit products; the key's hi plane holds 16 bits per residue)
+cudaError_t launch_klss_ip48(const KlssIpArgs& A, int batch, cudaStream_t st);
+cudaError_t launch_klss_recover48(const KlssRecArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_klss_diff(const KlssDiffArgs& A, int batch, cudaStream_t st);
 
 }  // namespace neo

@@ -179,9 +179,14 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
     P.n_out = (int)dst.size();
     // targets in parts of J = 9 (45 MMA columns, padded to 48): one TMEM job and one
     // tcgen05.ld batch per part in the epilogue
-    P.J = std::min(P.n_out, BCTC_PART_J);
+    // 48-bit targets (KLSS T primes at WordSize_T = 48) need 6 constant bytes: 8 targets per part
+    u64 tmax = 0;
+    for (u64 m : dst) tmax = std::max(tmax, m);
+    P.nb = (tmax >> 40) ? 6 : 5;
+    const int nb = P.nb;
+    P.J = std::min(P.n_out, nb == 5 ? BCTC_PART_J : BCTC_PART_ROWS / 6);
     P.nparts = (P.n_out + P.J - 1) / P.J;
-    P.ncols = ((5 * P.J + 15) / 16) * 16;
+    P.ncols = ((nb * P.J + 15) / 16) * 16;
     bmat.assign((size_t)P.nparts * BCTC_PART_ROWS * 64, 0);
     for (int i = 0; i < P.n_in; ++i) {
         u64 qi = src[i], qh = 1;
@@ -201,8 +206,8 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
                 if (k != i) f = mulm(f, src[k] % m, m);
             for (int a = 0; a < 5; ++a) {
                 u64 v = mulm(f, (1ull << (8 * a)) % m, m);      // (2^(8a) qhat_i) mod t
-                for (int b = 0; b < 5; ++b) {
-                    const int h = t / P.J, n = 5 * (t - h * P.J) + b, k = 5 * i + a;
+                for (int b = 0; b < nb; ++b) {
+                    const int h = t / P.J, n = nb * (t - h * P.J) + b, k = 5 * i + a;
                     size_t off = (size_t)h * BCTC_PART_ROWS * 64 + (size_t)(n / 8) * 512 + (k / 16) * 128 +
                                  (n % 8) * 16 + (k % 16);
                     bmat[off] = (uint8_t)((v >> (8 * b)) & 0xFF);
@@ -211,8 +216,8 @@ void make_bconv_tc(const std::vector<u64>& src, const std::vector<u64>& dst, BCo
         }
         if (corr) {                                            // column k = 5 n_in: (-Q_in) mod t, unshifted
             const u64 v = (*corr)[t] % m;
-            for (int b = 0; b < 5; ++b) {
-                const int h = t / P.J, n = 5 * (t - h * P.J) + b, k = 5 * P.n_in;
+            for (int b = 0; b < nb; ++b) {
+                const int h = t / P.J, n = nb * (t - h * P.J) + b, k = 5 * P.n_in;
                 size_t off = (size_t)h * BCTC_PART_ROWS * 64 + (size_t)(n / 8) * 512 + (k / 16) * 128 + (n % 8) * 16 +
                              (k % 16);
                 bmat[off] = (uint8_t)((v >> (8 * b)) & 0xFF);
@@ -243,8 +248,21 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
                 return NEO_EINVAL;
             }
     } else {
-        c->mod = gen_primes(c->log_n, c->word_bits, nl + (c->alpha_t ? KLSS_MAX_T : 0));
+        c->word_bits_t = c->alpha_t ? (d->word_bits_t > 0 ? d->word_bits_t : c->word_bits) : 0;
+        // T primes (K6): the Z4 rule at WordSize_T bits; at WordSize_T = word_bits the sequence
+        // continues after q and p, otherwise it starts afresh (disjoint from Q and P by width)
+        const bool same = c->word_bits_t == c->word_bits;
+        c->mod = gen_primes(c->log_n, c->word_bits, nl + (c->alpha_t && same ? KLSS_MAX_T : 0));
         if ((int)c->mod.size() < nl) { err = "not enough NTT-friendly primes"; return NEO_ENOPRIME; }
+        if (c->alpha_t && !same) {
+            if (c->word_bits_t < c->word_bits || c->word_bits_t > 48) {
+                err = "KLSS: WordSize_T must be in [word_bits, 48]";
+                return NEO_EUNSUPPORTED;
+            }
+            c->mod.resize(nl);
+            std::vector<u64> tp = gen_primes(c->log_n, c->word_bits_t, KLSS_MAX_T);
+            c->mod.insert(c->mod.end(), tp.begin(), tp.end());
+        }
     }
     if (c->alpha_t) {
         // KLSS (reading K1-K3, Eq. 4): groups of alpha~ consecutive limbs of q_0..q_L, p_0..p_K;
@@ -376,9 +394,14 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
     {
         const char* e = std::getenv("NEO_BCONV");
         c->use_tc = !(e && std::string(e) == "cuda");
-        // the epilogue's exact FP64 sum of the byte planes needs every modulus < 2^36 (bconv_tc.cu)
-        for (int k = 0; k < ntot; ++k)
+        // the epilogue's exact FP64 sum of the byte planes needs every Q / P modulus < 2^36
+        // (bconv_tc.cu); 48-bit T targets take the 6-byte integer epilogue, 48-bit T inputs the
+        // CUDA-core Recover Limbs
+        for (int k = 0; k < nl; ++k)
             if (c->mod[k] >> 36) c->use_tc = false;
+        c->klss_rec_tc_ok = true;
+        for (int k = nl; k < ntot; ++k)
+            if (c->mod[k] >> 36) c->klss_rec_tc_ok = false;
         std::vector<uint8_t> all, bm;
         c->modup_tc.resize(c->num_q);
         c->modup_boff.resize(c->num_q);
@@ -414,8 +437,8 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
                 c->klss_rec_tc.resize(c->num_q);
                 c->klss_rec_boff.resize(c->num_q);
                 std::vector<u64> tm(c->mod.begin() + nl, c->mod.begin() + nl + c->num_t);
-                if (5 * c->num_t >= 64) fits = false;           // Recover's correction column needs K = 5 alpha' + 1 <= 64
-                for (size_t gi = 0; gi < c->klss_groups.size(); ++gi) {   // Recover Limbs: T -> group (centred)
+                if (5 * c->num_t >= 64) c->klss_rec_tc_ok = false;   // Recover's correction column: K = 5 alpha' + 1 <= 64
+                for (size_t gi = 0; gi < c->klss_groups.size() && c->klss_rec_tc_ok; ++gi) {   // Recover Limbs: T -> group (centred)
                     std::vector<u64> dm, corr;
                     for (int id : c->klss_groups[gi])
                         if (id <= l || id >= c->num_q) {

@@ -47,7 +47,8 @@ class ParamsDesc(ctypes.Structure):
     _fields_ = [("log_n", ctypes.c_int32), ("num_q", ctypes.c_int32), ("num_p", ctypes.c_int32),
                 ("dnum", ctypes.c_int32), ("word_bits", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("q", ctypes.POINTER(ctypes.c_uint64)), ("p", ctypes.POINTER(ctypes.c_uint64)),
-                ("alpha_t", ctypes.c_int32)]
+                ("alpha_t", ctypes.c_int32),
+                ("word_bits_t", ctypes.c_int32)]
 
 
 _lib = None
@@ -200,11 +201,11 @@ class Context:
     """neo_params_create / neo_params_destroy; q, p, psi from neo_params_query."""
 
     def __init__(self, log_n: int, num_q: int, num_p: int, dnum: int, word_bits: int = 36, device: int = 0,
-                 alpha_t: int = 0):
+                 alpha_t: int = 0, word_bits_t: int = 0):
         self.log_n, self.num_q, self.num_p, self.dnum = log_n, num_q, num_p, dnum
         self.N = 1 << log_n
         self.alpha = -(-num_q // dnum)
-        d = ParamsDesc(log_n, num_q, num_p, dnum, word_bits, device, None, None, alpha_t)
+        d = ParamsDesc(log_n, num_q, num_p, dnum, word_bits, device, None, None, alpha_t, word_bits_t)
         h = ctypes.c_void_p()
         _check(lib().neo_params_create(ctypes.byref(d), ctypes.byref(h)), "neo_params_create")
         self.handle = h

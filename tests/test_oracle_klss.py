@@ -57,10 +57,28 @@ def test_alpha_prime_follows_eq4_set_c():
     assert not set(kp.t) & set(b.moduli)
 
 
-def test_klss_key_is_evk_mod_group():
+def test_alpha_prime_follows_eq4_set_c_t48():
+    """Eq. 4 (L173) at Set-C as printed in Table 4 (WordSize_T = 48, L511): alpha' = 8 T primes of
+    48 bits, the Z4 rule at 48 bits (K6): the largest 48-bit k 2N + 1 primes in order."""
+    kp = klss.set_c()
+    b = kp.base
+    T = math.prod(kp.t)
+    assert T > 4 * kp.bound and T // kp.t[-1] <= 4 * kp.bound
+    assert kp.alpha_p == 8 == math.ceil(math.log2(4 * kp.bound) / 48)
+    assert all(ckks.is_prime(t) and t % (2 * b.N) == 1 and t.bit_length() == 48 for t in kp.t)
+    two_n = 2 * b.N
+    ks = [(t - 1) // two_n for t in kp.t]
+    assert ks == sorted(ks, reverse=True) and ks[0] <= ((1 << 48) - 1) // two_n
+    for k in range(ks[-1] + 1, ((1 << 48) - 1) // two_n + 1):         # every skipped candidate composite
+        if k not in ks:
+            assert not ckks.is_prime(k * two_n + 1)
+
+
+@pytest.mark.parametrize("mk", [klss.tiny, klss.tiny48])
+def test_klss_key_is_evk_mod_group(mk):
     """K1: INTT_T of the key, lifted exactly from T, is [evk]_{P~_i} in [0, P~_i) and agrees
     with evk modulo every limb of the group."""
-    kp = klss.tiny()
+    kp = mk()
     b = kp.base
     evk = np.stack([np.stack([synth.uniform_residues(60 + 2 * j + c, b.moduli, b.N) for c in range(2)])
                     for j in range(b.dnum)])
@@ -76,10 +94,12 @@ def test_klss_key_is_evk_mod_group():
                 assert [e % b.moduli[t] for t in g] == [int(v) for v in evk_coef[:, n]]
 
 
+@pytest.mark.parametrize("mk", [klss.tiny, klss.tiny48])
 @pytest.mark.parametrize("level", [5, 3, 0])
-def test_klss_keyswitch_equals_hybrid(level):
-    """K4: with the key of K1, KLSS KeySwitch returns exactly Hybrid's output (every residue)."""
-    kp = klss.tiny()
+def test_klss_keyswitch_equals_hybrid(level, mk):
+    """K4: with the key of K1, KLSS KeySwitch returns exactly Hybrid's output (every residue);
+    WordSize_T = 36 and 48 (K6)."""
+    kp = mk()
     b = kp.base
     evk = np.stack([np.stack([synth.uniform_residues(80 + 2 * j + c, b.moduli, b.N) for c in range(2)])
                     for j in range(b.dnum)])
@@ -113,9 +133,11 @@ def test_klss_hmult_rescale_decrypts():
     assert np.max(np.abs(z - za * zb)) < 1e-6
 
 
-def test_klss_equals_hybrid_set_c():
-    """K4 at Set-C (dnum = 9, alpha~ = 5, 10 T primes), level 35: sampled residues of every limb."""
-    kp = klss.set_c_t36()
+@pytest.mark.parametrize("mk", [klss.set_c_t36, klss.set_c])
+def test_klss_equals_hybrid_set_c(mk):
+    """K4 at Set-C (dnum = 9, alpha~ = 5; 10 T primes of 36 bits or 8 of 48), level 35: every
+    residue of every limb."""
+    kp = mk()
     b = kp.base
     evk = np.stack([np.stack([synth.uniform_residues(400 + 2 * j + c, b.moduli, b.N) for c in range(2)])
                     for j in range(b.dnum)])
