@@ -73,9 +73,9 @@ typedef struct {
                           * > 0 adds alpha' T primes (alpha' from Eq. 4, reading K3)
                           * and the KLSS tables; requires generated primes (q = p = NULL). */
     int32_t word_bits_t; /* WordSize_T of the T primes (Table 4: 48 for Set-C), used when
-                          * alpha_t > 0: 0 or word_bits = the Z4 rule continued after p; up to 48 =
-                          * the Z4 rule at word_bits_t bits (reading K6).  Values outside
-                          * [word_bits, 48] fail with NEO_EUNSUPPORTED. */
+                          * alpha_t > 0: 0 or word_bits = the Z4 rule continued after p; 48 = the
+                          * Z4 rule at 48 bits (reading K6).  Other values fail with
+                          * NEO_EUNSUPPORTED. */
 } neo_params_desc;
 
 /* Build the context: primes, psi, NTT twiddle tables, BConv tables for every

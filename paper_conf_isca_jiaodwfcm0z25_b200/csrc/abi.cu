@@ -106,10 +106,10 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
                            u64* dst, long long dst_bs, const int* dst_off, const int* prime, int n, u64* tmp,
                            int batch, cudaStream_t st, const RowEpi* epi = nullptr, bool in_lazy = false,
                            const TWD* scale = nullptr, unsigned galois = 0, const u64* fold = nullptr,
-                           const TWD* fold_w = nullptr) {
+                           const TWD* fold_w = nullptr, const u64* sub = nullptr, long long sub_bs = 0) {
     if (n <= 0) return NEO_OK;
     if (n > NEO_MAX_ROWS) {               // more rows than one launch's descriptor holds: chunks
-        if (epi || fold) FAIL(NEO_EUNSUPPORTED, "too many limb rows for a fused-epilogue transform");
+        if (epi || fold || sub) FAIL(NEO_EUNSUPPORTED, "too many limb rows for a fused-epilogue transform");
         for (int k0 = 0; k0 < n; k0 += NEO_MAX_ROWS) {
             const int m = std::min(NEO_MAX_ROWS, n - k0);
             neo_status s = ntt_rows(c, fwd, src, src_bs, src_off + k0, dst, dst_bs, dst_off + k0, prime + k0, m, tmp,
@@ -136,6 +136,10 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
     }
     if (b.has_scale)
         for (int k = 0; k < n; ++k) b.scale[k] = scale[k];
+    if (fwd && sub) {                     // forward column pass: x -= sub row k of entry b
+        a.sub = sub;
+        a.sub_bstride = sub_bs;
+    }
     if (fwd && fold) {                    // forward column pass: x += fold[b] * fold_w[k]
         a.fold = fold;
         for (int k = 0; k < n; ++k) a.scale[k] = fold_w[k];
@@ -264,13 +268,14 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
                 io.out_off[o++] = j * E + pos;
             }
             if (c->use_tc) {
-                M.P[M.njobs] = c->modup_tc[l][j];
-                M.io[M.njobs] = io;
-                M.bmat[M.njobs] = c->d_bmat + c->modup_boff[l][j];
-                if (++M.njobs == 4) {                      // at most 4 conversions per launch
+                if (M.njobs && !bconv_multi_fits(M, c->modup_tc[l][j])) {   // job / part limits of one launch
                     LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, B, c->num_sms, st));
                     M.njobs = 0;
                 }
+                M.P[M.njobs] = c->modup_tc[l][j];
+                M.io[M.njobs] = io;
+                M.bmat[M.njobs] = c->d_bmat + c->modup_boff[l][j];
+                ++M.njobs;
             } else {
                 LAUNCH(PK_BCONV, st, launch_bconv(T, io, N, B, st));
             }
@@ -512,9 +517,9 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
 
 // ------------------------------------------------------------------ KLSS key-switch
 // Workspace: y [B][Lq], up [B][beta][alpha'] (T basis), accT [B][2][beta~][alpha'],
-// rec [B][2][E] (PQ_l, coefficient form), conv [2B][Lq], diff [2B][Lq], NTT intermediate.
+// rec [B][2][E] (PQ_l, coefficient form), conv [2B][Lq], NTT intermediate.
 struct KlssLayout {
-    size_t y, up, acc, rec, conv, diff, tmp, extra, total;
+    size_t y, up, acc, rec, conv, tmp, extra, total;
 };
 
 static KlssLayout klss_layout(const neo_ctx* c, int l, int B, int op) {
@@ -527,7 +532,6 @@ static KlssLayout klss_layout(const neo_ctx* c, int l, int B, int op) {
     L.acc = o; o += B * 2 * bt * ap * N;
     L.rec = o; o += B * 2 * E * N;
     L.conv = o; o += B * 2 * Lq * N;
-    L.diff = o; o += B * 2 * Lq * N;
     L.tmp = o; o += B * std::max(std::max(beta * ap, 2 * bt * ap), 2 * Lq) * N;
     L.extra = o;
     if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
@@ -555,7 +559,7 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     if (wide && !c->use_tc) FAIL(NEO_EUNSUPPORTED, "KLSS with WordSize_T > 40 needs the tensor-core BConv");
     if ((k->hi_bytes == 2) != wide) FAIL(NEO_EINVAL, "KLSS key packed for another WordSize_T");
     u64 *y = ws + Ly.y, *up = ws + Ly.up, *acc = ws + Ly.acc, *rec = ws + Ly.rec, *conv = ws + Ly.conv,
-        *diff = ws + Ly.diff, *tmp = ws + Ly.tmp;
+        *tmp = ws + Ly.tmp;
     int so[NEO_HOST_ROWS], dof[NEO_HOST_ROWS], pr[NEO_HOST_ROWS];
     neo_status s;
     // 1. INTT of d; Algorithm 2's [c_i qhat_i^-1]_{q_i} folded in (the digits are Hybrid's)
@@ -586,13 +590,14 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
             for (size_t i = 0; i < dj.size(); ++i) io.in_off[i] = dj[i];
             for (int t = 0; t < ap; ++t) io.out_off[t] = j * ap + t;
             if (c->use_tc) {
-                M.P[M.njobs] = c->klss_up_tc[l][j];
-                M.io[M.njobs] = io;
-                M.bmat[M.njobs] = c->d_bmat + c->klss_up_boff[l][j];
-                if (++M.njobs == 4) {
+                if (M.njobs && !bconv_multi_fits(M, c->klss_up_tc[l][j])) {
                     LAUNCH(PK_BCONV, st, launch_bconv_tc(M, N, B, c->num_sms, st));
                     M.njobs = 0;
                 }
+                M.P[M.njobs] = c->klss_up_tc[l][j];
+                M.io[M.njobs] = io;
+                M.bmat[M.njobs] = c->d_bmat + c->klss_up_boff[l][j];
+                ++M.njobs;
             } else {
                 LAUNCH(PK_BCONV, st, launch_bconv(c->klss_up[l][j], io, N, B, st));
             }
@@ -671,13 +676,14 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
                 io.out_bstride = (long long)2 * E * N;
                 for (int t = 0; t < ap; ++t) io.in_off[t] = t;
                 for (int o = R.first[g]; o < R.first[g + 1]; ++o) io.out_off[o - R.first[g]] = R.out_pos[o];
-                M.P[M.njobs] = c->klss_rec_tc[l][i];
-                M.io[M.njobs] = io;
-                M.bmat[M.njobs] = c->d_bmat + c->klss_rec_boff[l][i];
-                if (++M.njobs == 4) {
+                if (M.njobs && !bconv_multi_fits(M, c->klss_rec_tc[l][i])) {
                     LAUNCH(PK_COMBINE, st, launch_bconv_tc(M, N, B, c->num_sms, st));
                     M.njobs = 0;
                 }
+                M.P[M.njobs] = c->klss_rec_tc[l][i];
+                M.io[M.njobs] = io;
+                M.bmat[M.njobs] = c->d_bmat + c->klss_rec_boff[l][i];
+                ++M.njobs;
             }
         if (M.njobs) LAUNCH(PK_COMBINE, st, launch_bconv_tc(M, N, B, c->num_sms, st));
     } else {
@@ -691,7 +697,7 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         io.out_bstride = (long long)Lq * N;
         for (int i = 0; i < P; ++i) io.in_off[i] = Lq + i;
         for (int i = 0; i < Lq; ++i) io.out_off[i] = i;
-        if (c->use_tc) {                        // canonical u64 out (the difference kernel reads it)
+        if (c->use_tc) {                        // canonical u64 out (the next column pass reads it)
             BConvMulti M;
             M.centred = 0;
         M.centred = 0;
@@ -707,12 +713,8 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
             LAUNCH(PK_BCONV, st, launch_bconv(c->moddown[l], io, N, 2 * B, st));
         }
     }
-    // 8. (conv - acc_Q) in coefficient form, then 9. its NTT with the tail
-    //    out_c = (0 - NTT(conv - acc_Q)) P^-1 (+ add_c) = NTT((acc_Q - conv) P^-1) (+ add_c)   (K5)
-    KlssDiffArgs D;
-    D.conv = conv; D.rec = rec; D.out = diff; D.mods = c->d_mods;
-    D.N = N; D.Lq = Lq; D.E = E;
-    LAUNCH(PK_COMBINE, st, launch_klss_diff(D, B, st));
+    // 8. (conv - acc_Q) in coefficient form, subtracted inside the column pass of 9. its NTT with
+    //    the tail out_c = (0 - NTT(conv - acc_Q)) P^-1 (+ add_c) = NTT((acc_Q - conv) P^-1) (+ add_c)   (K5)
     for (int i = 0; i < Lq; ++i) { so[i] = dof[i] = i; pr[i] = i; }
     RowEpi ep;
     ep.acc = nullptr;
@@ -721,7 +723,8 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     ep.out0 = out0; ep.out1 = out1; ep.out_b = out_bs;
     ep.add_galois = 0;
     for (int i = 0; i < Lq; ++i) ep.pinv[i] = c->pinv[i];
-    return ntt_rows(c, true, diff, (long long)Lq * N, so, diff, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st, &ep);
+    return ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st, &ep,
+                    false, nullptr, 0, nullptr, nullptr, rec, (long long)E * N);
 }
 
 static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,
@@ -880,8 +883,8 @@ neo_status neo_params_create(const neo_params_desc* desc, neo_ctx** out) {
     if (alpha > BC_MAX_IN) FAIL(NEO_EUNSUPPORTED, "alpha must be <= 16");
     if (desc->dnum > KS_MAX_BETA) FAIL(NEO_EUNSUPPORTED, "dnum must be <= 12");
     if ((desc->q == nullptr) != (desc->p == nullptr)) FAIL(NEO_EINVAL, "give both q and p or neither");
-    if (desc->alpha_t > 0 && desc->word_bits_t != 0 && (desc->word_bits_t < desc->word_bits || desc->word_bits_t > 48))
-        FAIL(NEO_EUNSUPPORTED, "word_bits_t must be 0 or in [word_bits, 48]");
+    if (desc->alpha_t > 0 && desc->word_bits_t != 0 && desc->word_bits_t != desc->word_bits && desc->word_bits_t != 48)
+        FAIL(NEO_EUNSUPPORTED, "word_bits_t must be 0, word_bits or 48");
     neo_ctx* c = new (std::nothrow) neo_ctx();
     if (!c) FAIL(NEO_ENOMEM, "host allocation failed");
     static std::atomic<unsigned long long> next_uid{0};

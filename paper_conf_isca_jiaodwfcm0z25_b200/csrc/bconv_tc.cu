@@ -36,14 +36,14 @@ constexpr int kInStages = 8;                       // TMA input ring (12 KB each
 constexpr int kEpiWarps = 4 * kSets;
 constexpr int kThreads = (4 + kEpiWarps + 2) * 32; // producers, epilogue, MMA, TMA
 constexpr size_t kInBytes = (size_t)BCTC_MAX_IN * kTileM * 8;
-constexpr int kMaxJobs = 4;                        // conversions fused into one launch (ModUp digits)
+constexpr int kMaxJobs = BCTC_MULTI_JOBS;          // conversions fused into one launch (ModUp digits)
 constexpr size_t kPartBytes = (size_t)BCTC_PART_ROWS * 64;
-constexpr size_t kBBytes = BCTC_MAX_PARTS * kPartBytes;   // 15 KB per conversion
+constexpr size_t kBAll = BCTC_MULTI_PARTS * kPartBytes;  // all jobs' B, packed (60 KB)
 struct JobH {                                      // per-conversion header, staged in smem
     const u64* in;
     u64* out;
     long long in_bs, out_bs;
-    int n_in, n_out, nparts, J, ncols, in_off0, use_tmap, pad;
+    int n_in, n_out, nparts, J, ncols, in_off0, use_tmap, boff;   // boff: B offset in parts
 };
 struct TgtC {                                      // per-target epilogue constants, staged in smem
     double t, tinv;
@@ -53,7 +53,7 @@ struct TgtC {                                      // per-target epilogue consta
 constexpr int kTgtRow = (BCTC_MAX_PARTS * BCTC_PART_J + 7) / 8 * 8;   // padded: parts need no clamp
 constexpr int kMaxSched = 1024;                    // per-CTA tile schedule entries staged in smem
 constexpr size_t kTabBytes = kMaxJobs * (sizeof(JobH) + kTgtRow * sizeof(TgtC)) + kMaxSched * 4;
-constexpr size_t kSmemBytes = kAStages * kTileM * 64 + kMaxJobs * kBBytes + kInStages * kInBytes + kTabBytes;
+constexpr size_t kSmemBytes = kAStages * kTileM * 64 + kBAll + kInStages * kInBytes + kTabBytes;
 constexpr size_t kSmemAlloc = 214 * 1024;          // > half an SM: one CTA (and 512 TMEM cols) per SM
 static_assert(kSmemBytes <= kSmemAlloc, "shared memory plan exceeds the allocation");
 static_assert(kSlots * kSlotCols == 512, "TMEM plan");
@@ -90,8 +90,8 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     };
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t* sA = smem;                                  // kAStages x (128 rows x 64 B)
-    uint8_t* sB0 = smem + kAStages * kTileM * 64;        // kMaxJobs x parts x (48 rows x 64 B)
-    u64* sIn = reinterpret_cast<u64*>(sB0 + kMaxJobs * kBBytes);   // kInStages x [n_in][128]
+    uint8_t* sB0 = smem + kAStages * kTileM * 64;        // all jobs' parts x (48 rows x 64 B), packed
+    u64* sIn = reinterpret_cast<u64*>(sB0 + kBAll);      // kInStages x [n_in][128]
     JobH* sJob = reinterpret_cast<JobH*>(sIn + kInStages * BCTC_MAX_IN * kTileM);    // [job]
     TgtC* sTgt = reinterpret_cast<TgtC*>(sJob + kMaxJobs);                           // [job][target]
     uint32_t* sSched = reinterpret_cast<uint32_t*>(sTgt + kMaxJobs * kTgtRow);       // [i] -> jb | b | m-tile
@@ -134,16 +134,18 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             tc::mbar_init(&in_empty[s], 4);
         }
     }
-    for (int j = 0; j < njobs; ++j) {
-        uint4* s4 = reinterpret_cast<uint4*>(sB0 + j * kBBytes);
+    for (int j = 0, bo = 0; j < njobs; bo += PJ[j].nparts, ++j) {
+        uint4* s4 = reinterpret_cast<uint4*>(sB0 + (size_t)bo * kPartBytes);
         const int n16 = PJ[j].nparts * (int)(kPartBytes / 16);
         for (int e = tid; e < n16; e += kThreads) s4[e] = loadB(j, e);
     }
     if (tid < njobs) {
         const BConvTC& P = PJ[tid];
         const BConvIO& io = IOJ[tid];
+        int bo = 0;
+        for (int j = 0; j < tid; ++j) bo += PJ[j].nparts;
         sJob[tid] = JobH{io.in, io.out, io.in_bstride, io.out_bstride, P.n_in, P.n_out, P.nparts, P.J, P.ncols,
-                         io.in_off[0], use_tmap ? use_tmap[tid] : 0, 0};
+                         io.in_off[0], use_tmap ? use_tmap[tid] : 0, bo};
     }
     for (int x = tid; x < kMaxSched && blockIdx.x + x * G < total_tiles; x += kThreads) {
         int j, b, m0;
@@ -309,7 +311,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
                 WAIT(&tempty[slot], (kq & 1) ^ 1, 5);
                 tc::fence_after();
                 const uint32_t acc = tmem + (uint32_t)(slot * kSlotCols);
-                const uint32_t bs = tc::smem_u32(sB0 + jb * kBBytes);
+                const uint32_t bs = tc::smem_u32(sB0 + (size_t)H.boff * kPartBytes);
                 if (!(exp & 16)) {
                     // K = 64 as two K = 32 steps (LBO = 128 B between K chunks, SBO = 512 B between row groups)
                     tc::mma_u8(acc, tc::sdesc(as, 128, 512), tc::sdesc(bs, 128, 512), idesc, 0);
@@ -428,7 +430,11 @@ cudaError_t launch_bconv_tc(const BConvMulti& M0, int N, int batch, int num_sms,
     bconv_tc_init();
     BConvMulti M = M0;
     static const bool no_tmap = [] { const char* e = std::getenv("NEO_BCONV_TMAP"); return e && e[0] == '0'; }();
-    for (int j = 0; j < 4; ++j) M.use_tmap[j] = (j < M.njobs && !no_tmap) ? make_input_tmap(M.P[j], M.io[j], N, batch, &M.tmap[j]) : 0;
+    if (M.njobs < 1 || M.njobs > kMaxJobs) return cudaErrorInvalidValue;
+    int parts = 0;
+    for (int j = 0; j < M.njobs; ++j) parts += M.P[j].nparts;
+    if (parts > BCTC_MULTI_PARTS) return cudaErrorInvalidValue;
+    for (int j = 0; j < kMaxJobs; ++j) M.use_tmap[j] = (j < M.njobs && !no_tmap) ? make_input_tmap(M.P[j], M.io[j], N, batch, &M.tmap[j]) : 0;
     const int tiles_per_entry = N / kTileM;
     const int total = tiles_per_entry * batch * M.njobs;
     const int grid = num_sms < total ? num_sms : total;
@@ -447,6 +453,13 @@ cudaError_t launch_bconv_tc(const BConvMulti& M0, int N, int batch, int num_sms,
         k = k_bconv_tc_g<true, true, false, 6>;
     }
     return launch_k(k, dim3(grid), dim3(kThreads), kSmemAlloc, st, M, N, tiles_per_entry, batch, exp);
+}
+
+bool bconv_multi_fits(const BConvMulti& M, const BConvTC& P) {
+    if (M.njobs >= kMaxJobs) return false;
+    int parts = P.nparts;
+    for (int j = 0; j < M.njobs; ++j) parts += M.P[j].nparts;
+    return parts <= BCTC_MULTI_PARTS;
 }
 
 cudaError_t launch_bconv_tc_param(const BConvTC& P, const BConvIO& io, const BMatParam& bp, int N, int batch,

@@ -19,21 +19,26 @@ void make_bconv_tc(const std::vector<u64>& src_mod, const std::vector<u64>& dst_
 
 size_t bconv_tc_smem(int ncols);
 
-// Up to 4 conversions with the same input/output batch geometry in one launch (e.g. the
-// beta ModUp digits); B matrices from device memory.
+// Up to BCTC_MULTI_JOBS conversions with the same input/output batch geometry in one launch (e.g.
+// the beta ModUp digits), with at most BCTC_MULTI_PARTS target parts in total (B matrices packed
+// back to back in shared memory); B matrices from device memory.
+constexpr int BCTC_MULTI_JOBS = 12;
+constexpr int BCTC_MULTI_PARTS = 20;
 struct BConvMulti {
-    CUtensorMap tmap[4];     // filled by launch_bconv_tc: 3-D map {N, rows, batch} of job j's input
-    int use_tmap[4];         // 1: one tensor TMA per tile (inputs rows contiguous), 0: per-row bulk copies
+    CUtensorMap tmap[BCTC_MULTI_JOBS];     // filled by launch_bconv_tc: 3-D map {N, rows, batch} of job j's input
+    int use_tmap[BCTC_MULTI_JOBS];         // 1: one tensor TMA per tile (inputs rows contiguous), 0: per-row bulk copies
     int njobs;
     int pre_scaled;      // inputs already hold y_i = [c_i qhat_i^-1]_{q_i} (scale folded into the INTT)
     int lazy_out;        // write lazy doubles |x| < 2^40 for the next NTT instead of canonical u64
     int centred;         // B has the correction column of make_bconv_tc(corr): producers supply u
-    BConvTC P[4];
-    BConvIO io[4];
-    const uint8_t* bmat[4];
+    BConvTC P[BCTC_MULTI_JOBS];
+    BConvIO io[BCTC_MULTI_JOBS];
+    const uint8_t* bmat[BCTC_MULTI_JOBS];
     unsigned long long* dbg;   // optional clock64 trace of CTA 0 (NEO_BCONV_DBG): [tile][8]
 };
 cudaError_t launch_bconv_tc(const BConvMulti& M, int N, int batch, int num_sms, cudaStream_t st);
+// true if job P still fits a BConvMulti holding M.njobs jobs (job and part limits)
+bool bconv_multi_fits(const BConvMulti& M, const BConvTC& P);
 // One conversion with B passed by value (generic neo_bconv).
 cudaError_t launch_bconv_tc_param(const BConvTC& P, const BConvIO& io, const BMatParam& bp, int N, int batch,
                                   int num_sms, cudaStream_t st);

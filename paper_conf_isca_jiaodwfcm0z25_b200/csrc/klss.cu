@@ -67,18 +67,33 @@ k_klss_ip(const __grid_constant__ KlssIpArgs A, int batch) {
     }
 }
 
-// WordSize_T = 48 (Table 4 Set-C, L511): residues and key words < 2^48, 64-bit products
-// (IMAD.WIDE pairs) into a 128-bit sum; pairs of products (< 2^97) are folded through the
-// Barrett reduction (valid for X < 2^98, q < 2^48: common.cuh) with the running remainder.
-NEO_DEV void mac2_reduce(u64& r, u64 x0, u64 e0, u64 x1, u64 e1, ModQ m) {
-    u64 hi = 0, lo = r;
-    mac128(hi, lo, x0, e0);
-    mac128(hi, lo, x1, e1);
-    r = barrett_reduce(hi, lo, m);
+// WordSize_T = 48 (Table 4 Set-C, L511): residues and key words < 2^48 split into 24-bit halves,
+// so every product is four 24 x 24-bit IMAD.WIDE.U32 multiply-adds into three 64-bit partial sums
+// (sum_j x_j e_j = A + 2^24 Bm + 2^48 C, A, C < 12 * 2^48 and Bm < 24 * 2^48: no overflow for
+// beta <= 12), and ONE reduction per output: X < 2^101 via an FP64 quotient estimate
+// qf = rint(X / t) (|qf - X / t| < 4), the remainder X - qf t exactly in signed 64-bit
+// arithmetic (|.| < 5 t < 2^51) and at most four corrections each way.  Karatsuba: the middle
+// sum is S - A - C with S = sum (xl + xh)(el + eh) < 12 * 2^50, so three IMAD.WIDE per product.
+NEO_DEV void mac24k(u64& A, u64& S, u64& C, unsigned xl, unsigned xh, unsigned xs, unsigned el, unsigned eh,
+                    unsigned es) {
+    A += (u64)xl * el;
+    S += (u64)xs * es;
+    C += (u64)xh * eh;
+}
+NEO_DEV u64 reduce24(u64 A, u64 Bm, u64 C, ModQ m) {
+    const double Xd = __fma_rn((double)C, 281474976710656.0, __fma_rn((double)Bm, 16777216.0, (double)A));
+    const u64 qf = (u64)rint(Xd * m.qinv);
+    long long r = (long long)(A + (Bm << 24) + (C << 48) - qf * m.q);   // low 64 bits; true |r| < 2^51
+    const long long q = (long long)m.q;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) r += (r < 0) ? q : 0;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) r -= (r >= q) ? q : 0;
+    return (u64)r;
 }
 
 template <int BETA>
-__global__ void __launch_bounds__(256, 2)
+__global__ void __launch_bounds__(256, 3)
 k_klss_ip48(const __grid_constant__ KlssIpArgs A, int batch) {
     pdl_wait();
     const int gi = threadIdx.y;
@@ -89,14 +104,16 @@ k_klss_ip48(const __grid_constant__ KlssIpArgs A, int batch) {
     const size_t NK = (size_t)A.alpha_p * A.N;
     const size_t col = (size_t)k * A.N + n;
     const uint16_t* hi16 = reinterpret_cast<const uint16_t*>(A.key_hi);
-    u64 e[2][BETA];
+    unsigned el[2][BETA], eh[2][BETA];
 #pragma unroll
     for (int c = 0; c < 2; ++c) {
         const size_t kb = (size_t)(c * A.beta_t + i) * A.dnum * NK + col;
 #pragma unroll
         for (int j = 0; j < BETA; ++j) {
             const size_t o = kb + (size_t)j * NK;
-            e[c][j] = (u64)A.key_lo[o] | ((u64)hi16[o] << 32);
+            const unsigned lo = A.key_lo[o], hi = hi16[o];
+            el[c][j] = lo & 0xFFFFFFu;
+            eh[c][j] = (lo >> 24) | (hi << 8);
         }
     }
     for (int b = 0; b < batch; ++b) {
@@ -104,21 +121,21 @@ k_klss_ip48(const __grid_constant__ KlssIpArgs A, int batch) {
         u64 x[BETA];
 #pragma unroll
         for (int j = 0; j < BETA; ++j) x[j] = up[(size_t)j * NK];
-        u64 r0 = 0, r1 = 0;
+        u64 a0 = 0, s0 = 0, c0 = 0, a1 = 0, s1 = 0, c1 = 0;
 #pragma unroll
-        for (int j = 0; j < BETA; j += 2) {
-            const u64 x1 = j + 1 < BETA ? x[j + 1] : 0;
-            mac2_reduce(r0, x[j], e[0][j], x1, j + 1 < BETA ? e[0][j + 1] : 0, m);
-            mac2_reduce(r1, x[j], e[1][j], x1, j + 1 < BETA ? e[1][j + 1] : 0, m);
+        for (int j = 0; j < BETA; ++j) {
+            const unsigned xl = (unsigned)x[j] & 0xFFFFFFu, xh = (unsigned)(x[j] >> 24);
+            mac24k(a0, s0, c0, xl, xh, xl + xh, el[0][j], eh[0][j], el[0][j] + eh[0][j]);
+            mac24k(a1, s1, c1, xl, xh, xl + xh, el[1][j], eh[1][j], el[1][j] + eh[1][j]);
         }
         u64* acc = A.acc + (size_t)(b * 2) * A.beta_t * NK + (size_t)i * NK + col;
-        acc[0] = r0;
-        acc[(size_t)A.beta_t * NK] = r1;
+        acc[0] = reduce24(a0, s0 - a0 - c0, c0, m);
+        acc[(size_t)A.beta_t * NK] = reduce24(a1, s1 - a1 - c1, c1, m);
     }
 }
 
-// Recover Limbs with 48-bit T primes: as k_klss_recover, the products y_k [That_k]_p
-// (< 2^84) summed in 128 bits (alpha' <= 16 terms < 2^88) and Barrett-reduced mod p.
+// Recover Limbs with 48-bit T primes (reading K4, as k_klss_recover below).
+
 template <int AP>
 __global__ void __launch_bounds__(256)
 k_klss_recover48(const __grid_constant__ KlssRecArgs A) {
@@ -127,16 +144,19 @@ k_klss_recover48(const __grid_constant__ KlssRecArgs A) {
     const int gi = blockIdx.y >> 1, c = blockIdx.y & 1, b = blockIdx.z;
     const RecTab& R = *A.tab;
     const int o0 = A.first[gi], no = A.first[gi + 1] - o0;
-    __shared__ u64 tc[KLSS_MAX_OUT_G][AP];                     // this group's [That_k]_p
-    __shared__ TW tT[KLSS_MAX_OUT_G];                          // [T]_p
-    __shared__ ModQ tm[KLSS_MAX_OUT_G];
+    // outputs on the FP64 pipe (the y_k on the integer pipe): out_p = sum_k mulc(y_k, [That_k]_p)
+    // - mulc(u, [T]_p), each |mulc| <= 0.75 p for |y_k| < 2^48 (common.cuh bound), |sum| < 18 p
+    __shared__ TWD tc[KLSS_MAX_OUT_G][AP];                     // this group's ([That_k]_p, /p)
+    __shared__ TWD tT[KLSS_MAX_OUT_G];                         // ([T]_p, /p)
+    __shared__ double2 tm[KLSS_MAX_OUT_G];                     // (p, 1/p)
     __shared__ int tpos[KLSS_MAX_OUT_G];
     for (int e = threadIdx.x; e < no * AP; e += blockDim.x) {
         const int ro = e / AP, k = e - ro * AP, p = A.out_id[o0 + ro];
-        tc[ro][k] = R.that_p[p][k].w;
+        const double pd = (double)A.mods[p].q;
+        tc[ro][k] = TWD{(double)R.that_p[p][k].w, (double)R.that_p[p][k].w / pd};
         if (k == 0) {
-            tT[ro] = R.T_p[p];
-            tm[ro] = A.mods[p];
+            tT[ro] = TWD{(double)R.T_p[p].w, (double)R.T_p[p].w / pd};
+            tm[ro] = make_double2(pd, 1.0 / pd);
             tpos[ro] = A.out_pos[o0 + ro];
         }
     }
@@ -144,24 +164,26 @@ k_klss_recover48(const __grid_constant__ KlssRecArgs A) {
     if (n >= A.N) return;
     const size_t NK = (size_t)AP * A.N;
     const u64* a = A.acc + ((size_t)(b * 2 + c) * A.beta_t + A.group[gi]) * NK + n;
-    u64 y[AP];
+    u64 av[AP];
 #pragma unroll
-    for (int k = 0; k < AP; ++k) y[k] = a[(size_t)k * A.N];        // all loads in flight first
+    for (int k = 0; k < AP; ++k) av[k] = a[(size_t)k * A.N];      // all loads in flight first
+    double yd[AP];
     double s = 0.0;
 #pragma unroll
     for (int k = 0; k < AP; ++k) {
-        y[k] = shoup(y[k], R.that_inv[k], A.mods[A.t0 + k].q);     // y_k = [a_k That_k^-1]_{t_k}
-        s = __fma_rn((double)y[k], R.tinv[k], s);
+        const u64 y = shoup(av[k], R.that_inv[k], A.mods[A.t0 + k].q);   // y_k = [a_k That_k^-1]_{t_k}
+        yd[k] = u2d(y);
+        s = __fma_rn(yd[k], R.tinv[k], s);
     }
-    const u64 u = (u64)__double2ll_rn(s);
+    const double u = rint(s);
     u64* out = A.rec + (size_t)(b * 2 + c) * A.E * A.N + n;
 #pragma unroll 1
     for (int ro = 0; ro < no; ++ro) {
-        u64 hi = 0, lo = 0;
+        const double p = tm[ro].x, pinv = tm[ro].y;
+        double acc = -mulc(u, tT[ro], p);
 #pragma unroll
-        for (int k = 0; k < AP; ++k) mac128(hi, lo, y[k], tc[ro][k]);
-        const ModQ m = tm[ro];
-        out[(size_t)tpos[ro] * A.N] = sub_mod(barrett_reduce(hi, lo, m), shoup(u, tT[ro], m.q), m.q);
+        for (int k = 0; k < AP; ++k) acc = __dadd_rn(acc, mulc(yd[k], tc[ro][k], p));
+        out[(size_t)tpos[ro] * A.N] = d2u(canon(acc, p, pinv));
     }
 }
 

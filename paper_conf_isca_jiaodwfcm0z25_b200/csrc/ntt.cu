@@ -206,6 +206,14 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
 #pragma unroll
                 for (int na = 0; na < R; ++na) x[na] = u2d(d64[(R * na + r) * C + c]);
             }
+            if (rs.sub) {                                  // - sub (KLSS ModDown: conv - acc_Q), |x| < 2^40 + q
+                const u64* sr = rs.sub + b * rs.sub_bstride + (size_t)k * a.N + n2;
+                u64 sv[R];
+#pragma unroll
+                for (int na = 0; na < R; ++na) sv[na] = __ldg(sr + (size_t)(R * na + r) * N2);
+#pragma unroll
+                for (int na = 0; na < R; ++na) x[na] = __dadd_rn(x[na], -u2d(sv[na]));
+            }
             if (rs.fold) {                                 // + [c_l]_{q_i} * (P mod q_i): |x| < 2^40 + q
                 const u64* fr = rs.fold + (size_t)b * a.N + n2;
                 u64 fv[R];

@@ -255,8 +255,8 @@ neo_status build_context(neo_ctx* c, const neo_params_desc* d, std::string& err)
         c->mod = gen_primes(c->log_n, c->word_bits, nl + (c->alpha_t && same ? KLSS_MAX_T : 0));
         if ((int)c->mod.size() < nl) { err = "not enough NTT-friendly primes"; return NEO_ENOPRIME; }
         if (c->alpha_t && !same) {
-            if (c->word_bits_t < c->word_bits || c->word_bits_t > 48) {
-                err = "KLSS: WordSize_T must be in [word_bits, 48]";
+            if (c->word_bits_t != 48) {
+                err = "KLSS: WordSize_T must be word_bits or 48";
                 return NEO_EUNSUPPORTED;
             }
             c->mod.resize(nl);

@@ -1,5 +1,5 @@
-"""Per-kernel-kind breakdown of one Set-C key-switch, KLSS vs Hybrid (neo_profile events).
-usage: python tools/klss_profile.py [batch]"""
+"""Per-launch breakdown of one Set-C key-switch (level 35), KLSS vs Hybrid (neo_profile events).
+usage: python tools/klss_profile.py [batch] [word_bits_t]   (default 1, 48)"""
 import os
 import sys
 
@@ -9,7 +9,8 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_isca_jiaodwfcm0z25_b200 import neo  # noqa: E402
 
 B = int(sys.argv[1]) if len(sys.argv) > 1 else 1
-ctx = neo.Context(16, 36, 4, 9, alpha_t=5)
+WT = int(sys.argv[2]) if len(sys.argv) > 2 else 48
+ctx = neo.Context(16, 36, 4, 9, alpha_t=5, word_bits_t=WT)
 N, L = ctx.N, 35
 g = torch.Generator(device="cuda")
 g.manual_seed(1)
@@ -18,14 +19,21 @@ keys = {"klss": neo.EvalKey(ctx, rnd(2, 8, 9, ctx.alpha_p, N), klss=True), "hybr
 d = rnd(B, L + 1, N)
 o0, o1 = torch.empty_like(d), torch.empty_like(d)
 ws = ctx.workspace(neo.NEO_OP_KEYSWITCH, L, B)
+reps = 10
+print(f"Set-C l=35 B={B} WordSize_T={WT} alpha'={ctx.alpha_p}")
 for name, k in keys.items():
     for _ in range(3):
         neo.neo_keyswitch(ctx, k, d, L, o0, o1, B, ws)
     torch.cuda.synchronize()
-    neo.neo_profile_enable(True)
-    for _ in range(10):
+    acc = {}
+    for _ in range(reps):
+        neo.neo_profile_enable(True)
         neo.neo_keyswitch(ctx, k, d, L, o0, o1, B, ws)
-    pr = neo.neo_profile_read()
-    neo.neo_profile_enable(False)
-    tot = sum(v[0] for v in pr.values()) / 10
-    print(name, f"B={B} total {tot:.4f} ms/KS:", " ".join(f"{kk}={v[0] / 10:.4f}({v[1] // 10})" for kk, v in pr.items() if v[1]))
+        tl = neo.neo_profile_timeline()
+        neo.neo_profile_enable(False)
+        for i, (kind, s, e) in enumerate(tl):
+            acc.setdefault(i, [kind, 0.0])[1] += (e - s) * 1e3 / reps
+    tot = sum(v for _, v in acc.values())
+    print(f"{name}: {len(acc)} launches, {tot:.1f} us")
+    for i, (kind, us) in acc.items():
+        print(f"  {i:3d} {kind:18s} {us:8.1f} us")
