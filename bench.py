@@ -186,11 +186,12 @@ def bytes_model(batch: int, l: int = LEVEL, fused: bool = False) -> dict:
       BConv: ModUp reads Lq, writes up; ModDown reads 2P, writes 2Lq;
       KeyIP: reads d^ (beta*E), writes acc (2E), reads the key once per launch (2*beta*E limbs
         stored at 5 bytes per residue).
-    Per step (HMULT+Rescale fused + HROT, B = 1, l = 35): 482 limb transforms + 248 tail
-    operand limbs = 1212 limbs = 635.4 MB of NTT traffic (the fused HMULT+Rescale replaces the
+    Per step (HMULT+Rescale fused + HROT, B = 1, l = 35): 482 limb transforms + 250 tail
+    operand limbs = 1214 limbs = 636.5 MB of NTT traffic (the fused HMULT+Rescale replaces the
     last NTT over Lq rows by one over l rows and adds the INTTs of acc_l, d_l: 4 transforms).
     tensor: reads a, b (4Lq), writes d0..d2 (3Lq); automorphism: c0 only (2Lq); elementwise: the
-    fused Rescale's fold kernel (reads 2Lq + 4, writes 2l)."""
+    fused Rescale's c_l kernel (reads acc_l, conv_l, d_l of both components, writes c_l: 8 limbs;
+    the fold P*c_l itself is an operand of the next column pass, its 2 c_l limbs counted there)."""
     limb = (1 << LOG_N) * 8
     Lq, P = l + 1, NUM_P
     beta = -(-Lq // 12)
@@ -199,8 +200,8 @@ def bytes_model(batch: int, l: int = LEVEL, fused: bool = False) -> dict:
     ks_tr = Lq + up + 2 * P                      # transforms up to the ModDown NTT
     hrot_tr, hrot_tail = ks_tr + 2 * Lq, 2 * Lq + Lq
     if fused:
-        hm_tr, hm_tail = ks_tr + 4 + 2 * l, 2 * l + 2 * l
-        ew = batch * (2 * Lq + 4 + 2 * l)
+        hm_tr, hm_tail = ks_tr + 4 + 2 * l, 2 * l + 2 * l + 2
+        ew = batch * 8
         resc_tr, resc_tail = 0, 0
     else:
         hm_tr, hm_tail = ks_tr + 2 * Lq, 2 * Lq + 2 * Lq

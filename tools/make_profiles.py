@@ -69,6 +69,14 @@ def traffic(rnd, full):
         out[kind] = {"bytes_per_launch": int((d["dram_rd"] + d["dram_wr"]) * 1e6), "algo_bytes_per_launch": algo,
                      "launch": desc, "dram_read": int(d["dram_rd"] * 1e6), "dram_write": int(d["dram_wr"] * 1e6),
                      "dur_us_cold": d["dur_us"]}
+    if "ntt_row" in out and "ntt_col" in out:        # the NTT as one kind (bench.py's roofline.traffic)
+        r, c = out["ntt_row"], out["ntt_col"]
+        out["ntt"] = {"bytes_per_launch": r["bytes_per_launch"] + c["bytes_per_launch"],
+                      "algo_bytes_per_launch": 108 * 2 * LIMB,
+                      "launch": "forward NTT of the 108 ModUp limbs (Set-B, l=35, B=1): column + row pass, FP64 form",
+                      "dram_read": r["dram_read"] + c["dram_read"], "dram_write": r["dram_write"] + c["dram_write"],
+                      "dur_us_cold": round(r["dur_us_cold"] + c["dur_us_cold"], 3),
+                      "source": f"profiles/{rnd}_ncu_full_top_kernels.jsonl (ncu --set full, --clock-control none)"}
     json.dump(out, open(os.path.join(ROOT, "profiles", "ncu_traffic.json"), "w"), indent=1)
 
 
