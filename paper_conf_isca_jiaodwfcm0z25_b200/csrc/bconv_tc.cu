@@ -452,7 +452,10 @@ cudaError_t launch_bconv_tc(const BConvMulti& M0, int N, int batch, int num_sms,
         if (!M.pre_scaled || !M.lazy_out || M.centred) return cudaErrorInvalidValue;
         k = k_bconv_tc_g<true, true, false, 6>;
     }
-    return launch_k(k, dim3(grid), dim3(kThreads), kSmemAlloc, st, M, N, tiles_per_entry, batch, exp);
+    // with NEO_PDL=2 the launch may start while its predecessor drains: the setup (TMEM, B matrices,
+    // barriers, schedule) runs before griddepcontrol.wait
+    return launch_k_pdl(neo_pdl_bconv(), k, dim3(grid), dim3(kThreads), kSmemAlloc, st, M, N, tiles_per_entry, batch,
+                        exp);
 }
 
 bool bconv_multi_fits(const BConvMulti& M, const BConvTC& P) {

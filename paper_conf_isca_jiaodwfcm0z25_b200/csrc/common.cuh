@@ -105,6 +105,24 @@ NEO_DEV void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;\n" 
 
 bool neo_pdl_enabled();   // NEO_PDL=1 enables (launch.cu); griddepcontrol.* are no-ops otherwise
 
+bool neo_pdl_bconv();      // NEO_PDL=2: programmatic dependent launch for the BConv launches only (launch.cu)
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_k_pdl(bool pdl, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                                cudaStream_t st, Args&&... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_k(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
                             Args&&... args) {

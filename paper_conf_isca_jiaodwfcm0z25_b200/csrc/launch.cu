@@ -12,3 +12,10 @@ bool neo_pdl_enabled() {
     }();
     return on;
 }
+bool neo_pdl_bconv() {
+    static const bool on = [] {
+        const char* e = std::getenv("NEO_PDL");
+        return e && e[0] == '2';
+    }();
+    return on || neo_pdl_enabled();
+}
