@@ -167,6 +167,15 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
 // ------------------------------------------------------------------ workspace layout
 struct KsLayout {
     size_t y, up, acc, conv, pc, tmp, extra, total;   // u64 offsets
+    // second scratch area for the two-stream forms (neo_hrot_hoisted: acc, conv, pc, tmp, extra;
+    // neo_hrot_sum: y, up, tmp), 0 when the op has none
+    size_t y2 = 0, up2 = 0, acc2 = 0, conv2 = 0, pc2 = 0, tmp2 = 0, extra2 = 0;
+    KsLayout area2() const {               // the same layout with the second area's buffers
+        KsLayout L = *this;
+        if (acc2) { L.acc = acc2; L.conv = conv2; L.pc = pc2; L.tmp = tmp2; L.extra = extra2; }
+        if (up2) { L.y = y2; L.up = up2; L.tmp = tmp2; }
+        return L;
+    }
 };
 
 static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
@@ -185,10 +194,28 @@ static KsLayout ks_layout(const neo_ctx* c, int l, int B, int op) {
     if (op == NEO_OP_HMULT) o += B * 3 * Lq * N;
     if (op == NEO_OP_HMULT_RESCALE) o += B * 3 * Lq * N + 4 * B * N;   // d, then c_l scratch
     if (op == NEO_OP_HROT) o += B * Lq * N;                       // sigma_g(c0)
-    if (op == NEO_OP_HROT_HOISTED) o += B * 2 * Lq * N;
-    if (op == NEO_OP_HROT_SUM) o += B * 2 * Lq * N;                // sum of sigma_g(c0), one sigma_g(c0)
+    if (op == NEO_OP_HROT_HOISTED) {
+        o += B * 2 * Lq * N;                                       // pre (before the automorphism)
+        L.acc2 = o; o += B * 2 * E * N;                            // second ModDown area (side stream)
+        L.conv2 = o; o += B * 2 * Lq * N;
+        L.pc2 = o; o += B * 2 * P * N;
+        L.tmp2 = o; o += B * tmp_rows * N;
+        L.extra2 = o; o += B * 2 * Lq * N;
+    }
+    if (op == NEO_OP_HROT_SUM) {
+        o += B * 2 * Lq * N;                                       // sum of sigma_g(c0), one sigma_g(c0)
+        L.y2 = o; o += B * Lq * N;                                 // second ModUp area (side stream)
+        L.up2 = o; o += B * beta * E * N;
+        L.tmp2 = o; o += B * tmp_rows * N;
+    }
     L.total = o;
     return L;
+}
+
+// Two-stream forms of neo_hrot_hoisted / neo_hrot_sum at batch <= one chunk (NEO_TWO_STREAM=0 disables)
+static bool two_stream_ok(const neo_ctx* c) {
+    static const bool off = [] { const char* e = std::getenv("NEO_TWO_STREAM"); return e && e[0] == '0'; }();
+    return c->side && !off;
 }
 
 static size_t klss_total(const neo_ctx* c, int l, int B, int op);
@@ -1338,13 +1365,49 @@ neo_status neo_hrot_sum(const neo_ctx* c, const neo_evk* const* keys, const uint
     u64* c0k = c0sum + (size_t)batch * ls;                     // [B][l+1][N]: sigma_g(c0_k)
     cudaStream_t s = S(st);
     int launches = 0;
+    // two streams: the ModUps of odd k run on the context's side stream into a second ModUp area,
+    // overlapping the main stream's KeyIP of k - 1 and ModUp of k + 1; the KeyIPs accumulate in
+    // order on the main stream (each after its ModUp's event)
+    static thread_local cudaEvent_t ev_f = nullptr, ev_mu = nullptr, ev_kd = nullptr, ev_j = nullptr;
+    if (!ev_f) {
+        for (cudaEvent_t* e : {&ev_f, &ev_mu, &ev_kd, &ev_j}) cudaEventCreateWithFlags(e, cudaEventDisableTiming);
+    }
+    const bool fused = kip_ok(c, level);
+    const bool two = n > 1 && !fused && two_stream_ok(c);
+    const KsLayout Ly2 = Ly.area2();
+    if (two) {
+        CK(cudaEventRecord(ev_f, s));
+        CK(cudaStreamWaitEvent(c->side, ev_f, 0));
+    }
+    auto join = [&]() {
+        if (two) {
+            const std::string msg = g_err;
+            cudaEventRecord(ev_j, c->side);
+            cudaStreamWaitEvent(s, ev_j, 0);
+            g_err = msg;
+        }
+    };
     for (int k = 0; k < n; ++k) {
         // KeyIP(ModUp(sigma_g(c1_k))) accumulated in PQ_l; sigma_g(c1) read through the index map
-        const bool fused = kip_ok(c, level);
-        TRY(ks_modup(c, cts[k] + ls, 2 * ls, level, batch, w, Ly, s, galois[k], fused));
+        const bool alt = two && (k & 1);
+        const KsLayout& Lk = alt ? Ly2 : Ly;
+        if (alt) {
+            if (k >= 2 && cudaStreamWaitEvent(c->side, ev_kd, 0) != cudaSuccess) { join(); FAIL(NEO_ECUDA, "event wait"); }
+            neo_status r = ks_modup(c, cts[k] + ls, 2 * ls, level, batch, w, Lk, c->side, galois[k], fused);
+            if (r == NEO_OK && (cudaEventRecord(ev_mu, c->side) != cudaSuccess || cudaStreamWaitEvent(s, ev_mu, 0) != cudaSuccess))
+                r = NEO_ECUDA;
+            if (r != NEO_OK) { join(); return r; }
+        } else {
+            const neo_status r = ks_modup(c, cts[k] + ls, 2 * ls, level, batch, w, Lk, s, galois[k], fused);
+            if (r != NEO_OK) { join(); return r; }
+        }
         launches += g_launches;
-        TRY(ks_finish(c, keys[k], cts[k] + ls, 2 * ls, level, batch, w, Ly, nullptr, nullptr, 0, nullptr, nullptr,
-                      0, s, galois[k], false, nullptr, k == 0 ? 1 : 2, fused));
+        {
+            const neo_status r = ks_finish(c, keys[k], cts[k] + ls, 2 * ls, level, batch, w, Lk, nullptr, nullptr, 0,
+                                           nullptr, nullptr, 0, s, galois[k], false, nullptr, k == 0 ? 1 : 2, fused);
+            if (r != NEO_OK) { join(); return r; }
+        }
+        if (alt && cudaEventRecord(ev_kd, s) != cudaSuccess) { join(); FAIL(NEO_ECUDA, "event record"); }
         launches += g_launches;
         g_launches = 0;
         LAUNCH(PK_AUTO, s, launch_automorph(cts[k], k == 0 ? c0sum : c0k, galois[k], c->N, level + 1, s, batch,
@@ -1353,6 +1416,7 @@ neo_status neo_hrot_sum(const neo_ctx* c, const neo_evk* const* keys, const uint
         launches += g_launches;
         g_launches = 0;
     }
+    join();
     // one ModDown of the summed acc, with the summed sigma_g(c0) added to component 0
     TRY(ks_finish(c, keys[0], nullptr, 0, level, batch, w, Ly, ct_out, ct_out + ls, 2 * ls, c0sum, nullptr, ls, s,
                   0, false, nullptr, 3));
@@ -1380,13 +1444,47 @@ neo_status neo_hrot_hoisted(const neo_ctx* c, const neo_evk* const* keys, int32_
     cudaStream_t s = S(st);
     // one ModUp of c1 for all rotations (hoisting): sigma_g(KS'(c1)) with KS' under sigma_g^-1(key)
     TRY(ks_modup(c, ct_in + ls, 2 * ls, level, batch, w, Ly, s));
-    for (int r = 0; r < n_rot; ++r) {
-        TRY(ks_finish(c, keys[r], ct_in + ls, 2 * ls, level, batch, w, Ly, pre, pre + ls, 2 * ls, ct_in, nullptr,
-                      2 * ls, s));
-        u64* dst = ct_out + (size_t)r * batch * 2 * ls;
-        LAUNCH(PK_AUTO, s, launch_automorph(pre, dst, keys[r]->galois, c->N, 2 * (level + 1) * batch, s));
+    // the rotations' KeyIP + ModDown are independent: odd ones on the context's side stream with
+    // their own ModDown area (latency-bound small launches at B = 1 overlap); fork / join by events
+    static thread_local cudaEvent_t ev_f = nullptr, ev_j = nullptr;
+    if (!ev_f) {
+        cudaEventCreateWithFlags(&ev_f, cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&ev_j, cudaEventDisableTiming);
     }
-    return NEO_OK;
+    const bool two = n_rot > 1 && two_stream_ok(c);
+    const KsLayout Ly2 = Ly.area2();
+    u64* pre2 = w + Ly.extra2;
+    if (two) {
+        CK(cudaEventRecord(ev_f, s));
+        CK(cudaStreamWaitEvent(c->side, ev_f, 0));
+    }
+    int launches = g_launches;
+    neo_status res = NEO_OK;
+    for (int r = 0; r < n_rot && res == NEO_OK; ++r) {
+        const bool alt = two && (r & 1);
+        cudaStream_t sr = alt ? c->side : s;
+        u64* pr = alt ? pre2 : pre;
+        g_launches = 0;
+        res = ks_finish(c, keys[r], ct_in + ls, 2 * ls, level, batch, w, alt ? Ly2 : Ly, pr, pr + ls, 2 * ls, ct_in,
+                        nullptr, 2 * ls, sr);
+        launches += g_launches;
+        if (res != NEO_OK) break;
+        u64* dst = ct_out + (size_t)r * batch * 2 * ls;
+        g_launches = 0;
+        res = [&]() -> neo_status {
+            LAUNCH(PK_AUTO, sr, launch_automorph(pr, dst, keys[r]->galois, c->N, 2 * (level + 1) * batch, sr));
+            return NEO_OK;
+        }();
+        launches += g_launches;
+    }
+    if (two) {                                 // join (also on error: keeps a graph capture valid)
+        const std::string msg = g_err;
+        cudaEventRecord(ev_j, c->side);
+        cudaStreamWaitEvent(s, ev_j, 0);
+        g_err = msg;
+    }
+    g_launches = launches;
+    return res;
 }
 
 neo_status neo_keyip(const neo_ctx* c, const neo_evk* k, const uint64_t* dhat, const int32_t* limb_ids, int32_t n,
