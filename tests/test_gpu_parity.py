@@ -366,3 +366,19 @@ def test_pmult_acc_setb():
         t = ckks.pmult(prm, c, p, level)
         want = t if want is None else ckks.hadd(prm, want, t, level)
     assert np.array_equal(host(out)[0], want)
+
+
+# The library's environment-selected variants are read once per process, so each runs the parity
+# tests above in a fresh interpreter: NEO_TWO_STREAM=0 (hoisted rotations / giant-step sums on one
+# stream) and NEO_KIP=1 (KeyIP fused into the ModUp NTT's row pass, opt-in).
+@pytest.mark.parametrize("env,sel", [("NEO_TWO_STREAM=0", "hoisted or hrot_sum"),
+                                     ("NEO_KIP=1", "keyswitch or hmult or hrot")])
+def test_env_variants_bit_exact(env, sel):
+    import os
+    import subprocess
+    import sys
+    k, v = env.split("=")
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k",
+                        f"({sel}) and not env_variants", __file__],
+                       env=dict(os.environ, **{k: v}), capture_output=True, text=True, timeout=1200)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
