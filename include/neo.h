@@ -120,11 +120,19 @@ neo_status neo_ntt_select(neo_ctx* ctx, int32_t impl);
 /* The implementation currently selected (NEO_NTT_*), or -1 for a NULL context. */
 int32_t neo_ntt_selected(const neo_ctx* ctx);
 
+/* Rescale constants (L137, Z10): out[k] = q_level^-1 mod q_{limb_ids[k]} for n limb ids < level
+ * (host arrays), from the context's tables -- for callers that sequence a Rescale themselves
+ * (the limb-sharded bootstrapping).  NEO_EINVAL for a limb id outside [0, level). */
+neo_status neo_query_ql_inv(const neo_ctx* ctx, int32_t level, const int32_t* limb_ids, int32_t n, uint64_t* out);
+
 /* Basis conversion, Algorithm 1 (L296-319), non-centred (Z7), coefficient form:
  *   out[t] = sum_i [in_i * qhat_i^-1]_{q_i} * (qhat_i mod t) mod t,
  *   qhat_i = prod_{i' != i} q_{i'} over the input limbs.
  * in [batch][n_in][N] with limb ids in_ids (1 <= n_in <= 16, distinct);
- * out [batch][n_out][N] with limb ids out_ids (1 <= n_out <= 64). */
+ * out [batch][n_out][N] with limb ids out_ids (1 <= n_out <= 64).
+ * The first call for a given (context, in_ids, out_ids) builds that conversion's constants on the
+ * host and caches them per thread (one host allocation); later calls with the same ids do no
+ * host work beyond argument validation.  No device allocation. */
 neo_status neo_bconv(const neo_ctx* ctx, const uint64_t* in, const int32_t* in_ids, int32_t n_in,
                      uint64_t* out, const int32_t* out_ids, int32_t n_out, int32_t batch,
                      neo_stream_t stream);

@@ -57,10 +57,17 @@ def _g(N: int, r: int) -> int:
     return pow(5, r % (N // 2), 2 * N)
 
 
+def _encode(N: int, z, scale: float) -> np.ndarray:
+    """ckks.encode below N = 2^14; its one-FFT evaluation encode_fft above (within 1 of encode,
+    pinned in tests/test_oracle_ntt.py; any valid encoding -- as for bootstrapping, reading BOOT-F)."""
+    z = np.asarray(z, dtype=complex)
+    return ckks.encode(N, z, scale) if N < (1 << 14) else ckks.encode_fft(N, z, scale)
+
+
 def _enc(prm: ckks.Params, slots, scale: float, level: int) -> np.ndarray:
     """Plaintext (NTT form, [level+1][N]) of the slot vector `slots` (length N/2) at `scale`."""
     ids = list(range(level + 1))
-    m = ckks.encode(prm.N, np.asarray(slots, dtype=complex), scale)
+    m = _encode(prm.N, slots, scale)
     return ckks.ntt(prm, ckks.reduce_signed(prm, m, ids), ids)
 
 
@@ -136,6 +143,60 @@ class Ev:
         return self.rescale(self.pmul(v, name, slots, target * self.prm.q[l] / s))
 
 
+class DryEv(Ev):
+    """Ev without the ciphertext arithmetic: levels and scales tracked exactly as Ev tracks them,
+    plaintext constants made as Ev makes them.  A value is (None, level, scale).  Gives the
+    constants of a trace at sizes where running the oracle's ciphertext arithmetic is too slow
+    (Set-B); the GPU run with those constants is then checked by decryption."""
+
+    def __init__(self, prm: ckks.Params):
+        super().__init__(prm, {}, None)
+
+    def rescale(self, v):
+        _, l, s = v
+        self.counts["rescale"] += 1
+        return None, l - 1, s / self.prm.q[l]
+
+    def drop(self, v, level):
+        return None, level, v[2]
+
+    def add(self, a, b):
+        (_, la, sa), (_, lb, sb) = a, b
+        assert la == lb and abs(sa - sb) <= 1e-9 * sa, (la, lb, sa, sb)
+        self.counts["hadd"] += 1
+        return None, la, sa
+
+    def mul(self, a, b):
+        (_, la, sa), (_, lb, sb) = a, b
+        assert la == lb
+        self.counts["hmult"] += 1
+        return None, la, sa * sb
+
+    def rot(self, v, r):
+        self.counts["hrot"] += 1
+        return None, v[1], v[2]
+
+    def rot_hoisted(self, v, rs):
+        self.counts["hrot"] += len(rs)
+        return [(None, v[1], v[2]) for _ in rs]
+
+    def pmul(self, v, name, slots, scale):
+        _, l, s = v
+        self.counts["pmult"] += 1
+        self.const(name, slots, scale, l)
+        return None, l, s * scale
+
+    def padd(self, v, name, slots):
+        _, l, s = v
+        self.counts["padd"] += 1
+        self.const(name, slots, s, l)
+        return None, l, s
+
+
+def _ev(prm, keys, consts, dry):
+    return DryEv(prm) if dry else Ev(prm, keys, consts)
+
+
 # --------------------------------------------------------------------------- HELR
 
 @dataclass
@@ -175,10 +236,11 @@ def helr_plain(sh: HelrShape, Z: np.ndarray, w: np.ndarray) -> np.ndarray:
     return w + sh.gamma / sh.n * (s @ Z)
 
 
-def helr_iteration(sh: HelrShape, prm: ckks.Params, Zs: list, W, keys: dict, consts: dict | None = None):
+def helr_iteration(sh: HelrShape, prm: ckks.Params, Zs: list, W, keys: dict, consts: dict | None = None,
+                   dry: bool = False):
     """Zs: list of `batch` values (ct, level, scale); W likewise (same level and scale).
-    Returns (W', consts, counts); W' = (ct, level - 6, W's scale)."""
-    ev = Ev(prm, keys, consts)
+    Returns (W', consts, counts); W' = (ct, level - 6, W's scale).  dry: constants only (DryEv)."""
+    ev = _ev(prm, keys, consts, dry)
     N, f, rows = sh.N, sh.f, sh.rows
     lf, lr = int(math.log2(f)), int(math.log2(rows))
     half = N // 2
@@ -311,9 +373,10 @@ def _relu(sh: ConvShape, ev: Ev, Y, pre: str = ""):
 
 
 def conv_layer(sh: ConvShape, prm: ckks.Params, X, w: np.ndarray, bias: np.ndarray, keys: dict,
-               consts: dict | None = None):
-    """X = (ct, level, scale).  Returns (out, consts, counts); out at level - 4, X's scale."""
-    ev = Ev(prm, keys, consts)
+               consts: dict | None = None, dry: bool = False):
+    """X = (ct, level, scale).  Returns (out, consts, counts); out at level - 4, X's scale.
+    dry: constants only (DryEv)."""
+    ev = _ev(prm, keys, consts, dry)
     out = _relu(sh, ev, _conv(sh, ev, X, w, bias))
     assert out[1] == X[1] - CONV_LEVELS
     return out, ev.consts, ev.counts
@@ -414,7 +477,7 @@ def app_keys(prm: ckks.Params, s: np.ndarray, rotations: list[int], seed: int) -
 
 
 def encrypt_slots(prm: ckks.Params, z, delta: float, s: np.ndarray, level: int, seed: int):
-    m = ckks.encode(prm.N, np.asarray(z, dtype=complex), delta)
+    m = _encode(prm.N, z, delta)
     return ckks.encrypt(prm, m, s, level, seed), level, delta
 
 

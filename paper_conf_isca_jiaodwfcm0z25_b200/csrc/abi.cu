@@ -1015,6 +1015,17 @@ neo_status neo_intt(const neo_ctx* c, uint64_t* poly, const int32_t* ids, int32_
     return ntt_api(c, false, poly, ids, n, batch, ws, ws_bytes, st);
 }
 
+neo_status neo_query_ql_inv(const neo_ctx* c, int32_t level, const int32_t* limb_ids, int32_t n, uint64_t* out) {
+    TRY(check_ctx(c));
+    if (level < 1 || level >= c->num_q) FAIL(NEO_EINVAL, "level out of range");
+    if (n < 0 || (n > 0 && (!limb_ids || !out))) FAIL(NEO_EINVAL, "null argument");
+    for (int k = 0; k < n; ++k) {
+        if (limb_ids[k] < 0 || limb_ids[k] >= level) FAIL(NEO_EINVAL, "limb id outside [0, level)");
+        out[k] = c->ql_inv[level][limb_ids[k]].w;
+    }
+    return NEO_OK;
+}
+
 neo_status neo_bconv(const neo_ctx* c, const uint64_t* in, const int32_t* in_ids, int32_t n_in, uint64_t* out,
                      const int32_t* out_ids, int32_t n_out, int32_t batch, neo_stream_t st) {
     g_launches = 0;

@@ -32,7 +32,7 @@ EXPORTED = ("neo_params_create", "neo_params_destroy", "neo_params_query", "neo_
             "neo_drop_levels", "neo_pmult_acc", "neo_wire_bytes", "neo_wire_pack", "neo_wire_unpack", "neo_hmult_rescale", "neo_ew_limbs", "neo_hrot_sum",
             "neo_ntt_select", "neo_ntt_selected", "neo_comm_unique_id", "neo_comm_create",
             "neo_comm_create_local", "neo_comm_destroy", "neo_comm_limbs", "neo_workspace_size_sharded",
-            "neo_keyswitch_sharded")
+            "neo_keyswitch_sharded", "neo_query_ql_inv")
 PROFILE_KINDS = ("ntt_col", "ntt_row", "bconv", "keyip", "combine", "tensor", "automorphism",
                  "rescale_modswitch", "rescale_combine", "elementwise")
 
@@ -71,6 +71,7 @@ def lib() -> ctypes.CDLL:
             "neo_ntt": [_vp, _vp, _i32p, _i32, _i32, _vp, _sz, _vp],
             "neo_intt": [_vp, _vp, _i32p, _i32, _i32, _vp, _sz, _vp],
             "neo_bconv": [_vp, _vp, _i32p, _i32, _vp, _i32p, _i32, _i32, _vp],
+            "neo_query_ql_inv": [_vp, _i32, _i32p, _i32, _u64p],
             "neo_tensor": [_vp, _vp, _vp, _i32, _vp, _i32, _vp],
             "neo_automorphism": [_vp, _vp, _i32, _u32, _vp, _i32, _vp],
             "neo_evk_create": [_vp, _vp, ctypes.POINTER(_vp)],
@@ -296,6 +297,13 @@ def neo_intt(ctx: Context, poly: torch.Tensor, limb_ids, batch: int, ws: torch.T
 def neo_bconv(ctx: Context, inp: torch.Tensor, in_ids, out: torch.Tensor, out_ids, batch: int, stream=None):
     _check(lib().neo_bconv(ctx.handle, _ptr(inp), _ids(in_ids), len(in_ids), _ptr(out), _ids(out_ids),
                            len(out_ids), batch, _stream(stream)), "neo_bconv")
+
+
+def neo_query_ql_inv(ctx: Context, level: int, limb_ids) -> list:
+    """q_level^-1 mod q_i for the limb ids i < level (the context's Rescale constants)."""
+    out = (ctypes.c_uint64 * max(1, len(limb_ids)))()
+    _check(lib().neo_query_ql_inv(ctx.handle, level, _ids(limb_ids), len(limb_ids), out), "neo_query_ql_inv")
+    return list(out)[: len(limb_ids)]
 
 
 def neo_tensor(ctx: Context, ct_a, ct_b, level: int, d, batch: int, stream=None):

@@ -131,9 +131,8 @@ class ShardedBootstrapper(Bootstrapper):
         if not ids:
             return self._ct(lv - 1, B)
         r = self.ops.ntt(self.ops.bconv(coef.view(2 * B, 1, self.N), [lv], ids), ids).view(B, 2, len(ids), self.N)
-        if (lv, tuple(ids)) not in self._qinv:
-            ql = self.ctx.q[lv]
-            self._qinv[(lv, tuple(ids))] = [pow(ql % self.ctx.q[i], -1, self.ctx.q[i]) for i in ids]
+        if (lv, tuple(ids)) not in self._qinv:                    # the context's constants (C-ABI)
+            self._qinv[(lv, tuple(ids))] = neo.neo_query_ql_inv(self.ctx, lv, ids)
         return self._ew(neo.NEO_EWL_SUBMUL, self.drop(a, lv, lv - 1), r, lv - 1, scal=self._qinv[(lv, tuple(ids))])
 
     def modraise(self, ct0, L):

@@ -38,11 +38,11 @@ def helr_run():
     Zs = [apps.encrypt_slots(prm, zs[b], DELTA, s, L, 50 + b) for b in range(sh.batch)]
     W = apps.encrypt_slots(prm, wv, DELTA, s, L, 60)
     Wn, consts, counts = apps.helr_iteration(sh, prm, Zs, W, keys)
-    return prm, sh, s, Z, w, Wn, counts
+    return prm, sh, s, Z, w, Wn, counts, consts, Zs, W
 
 
 def test_helr_iteration_decodes_to_plain_step(helr_run):
-    prm, sh, s, Z, w, Wn, counts = helr_run
+    prm, sh, s, Z, w, Wn, counts, *_ = helr_run
     got = np.real(apps.decrypt_slots(prm, Wn, s))
     want = apps.helr_plain(sh, Z, w)
     assert Wn[1] == prm.max_level - apps.HELR_LEVELS
@@ -52,7 +52,7 @@ def test_helr_iteration_decodes_to_plain_step(helr_run):
 
 
 def test_helr_op_counts(helr_run):
-    prm, sh, s, Z, w, Wn, counts = helr_run
+    prm, sh, s, Z, w, Wn, counts, *_ = helr_run
     lf, lr = int(math.log2(sh.f)), int(math.log2(sh.rows))
     B = sh.batch
     assert counts["hmult"] == 4 * B
@@ -177,3 +177,24 @@ def test_resnet_block_and_head_decode():
     got_h = z[: 3 * sh.H * sh.H: sh.H * sh.H]
     assert np.max(np.abs(got_h - apps.head_plain(want_b, wfc, bfc))) < TOL
     assert hc["hrot"] == len(pool_r) + sh.C - 1
+
+
+def test_dry_run_gives_the_same_constants(helr_run):
+    """apps.DryEv (no ciphertext arithmetic, used for the Set-B GPU decode tests) makes exactly the
+    constants, levels and scales the full evaluation makes: HELR and the convolution layer."""
+    prm, sh, s, Z, w, Wn, counts, consts, Zs, W = helr_run
+    dry_in = [(None, z[1], z[2]) for z in Zs]
+    Wd, cd, nd = apps.helr_iteration(sh, prm, dry_in, (None, W[1], W[2]), {}, dry=True)
+    assert (Wd[1], Wd[2]) == (Wn[1], Wn[2]) and nd == counts
+    assert sorted(cd) == sorted(consts) and all(np.array_equal(cd[k], consts[k]) for k in consts)
+    sh2 = apps.ConvShape(prm.N, C=4, H=8)
+    baby, giant = sh2.rotations()
+    keys = apps.app_keys(prm, s, baby + giant, 800)
+    x = 2.0 * synth.uniform_unit(synth.derive(43, 1), sh2.C * sh2.H * sh2.H).reshape(sh2.C, sh2.H, sh2.H) - 1.0
+    wc = (2.0 * synth.uniform_unit(synth.derive(43, 2), sh2.C * sh2.C * 9).reshape(sh2.C, sh2.C, 3, 3) - 1.0) / 6.0
+    bias = 0.2 * (2.0 * synth.uniform_unit(synth.derive(43, 3), sh2.C) - 1.0)
+    X = apps.encrypt_slots(prm, apps.conv_pack(sh2, x), DELTA, s, prm.max_level, 70)
+    out, cc, nc = apps.conv_layer(sh2, prm, X, wc, bias, keys)
+    outd, ccd, ncd = apps.conv_layer(sh2, prm, (None, X[1], X[2]), wc, bias, {}, dry=True)
+    assert (outd[1], outd[2]) == (out[1], out[2]) and ncd == nc
+    assert sorted(ccd) == sorted(cc) and all(np.array_equal(ccd[k], cc[k]) for k in cc)
