@@ -398,7 +398,7 @@ def run_reference(args):
                                        "the CPU oracle (INTT; ModUp+NTT+KeyIP of digit 0/1/2; ModDown of c0/c1); "
                                        "6 steps = 1 key-switch"},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    emit(line)
 
 
 # ----------------------------------------------------------------------------- neo arm
@@ -733,15 +733,25 @@ def run_neo(args):
     # exchanges inside the library, NCCL over NVLink for N > 1, per-digit gathers overlapped with
     # the previous digit's BConv + NTT), eager and as a captured CUDA graph
     sharded_native = None
+    ncomm, comm_err = None, None
     if not args.no_latency:
-        if world > 1:
-            uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
-            if rank == 0:
-                uid.copy_(torch.frombuffer(bytearray(neo.Comm.unique_id()), dtype=torch.uint8))
-            dist.broadcast(uid, src=0)
-            ncomm = neo.Comm.create(ctx, bytes(uid.cpu().numpy().tobytes()), world, rank)
-        else:
-            ncomm = neo.Comm.create(ctx, bytes(128), 1, 0)
+        try:
+            if world > 1:
+                uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
+                if rank == 0:
+                    uid.copy_(torch.frombuffer(bytearray(neo.Comm.unique_id()), dtype=torch.uint8))
+                dist.broadcast(uid, src=0)
+                ncomm = neo.Comm.create(ctx, bytes(uid.cpu().numpy().tobytes()), world, rank)
+            else:
+                ncomm = neo.Comm.create(ctx, bytes(128), 1, 0)
+        except neo.NeoError as e:       # e.g. several ranks on one GPU (NEO_BENCH_BACKEND=gloo): NCCL refuses
+            ncomm, comm_err = None, str(e)[:200]
+        if not agree(ncomm is not None):
+            if ncomm is not None:
+                ncomm.close()
+                ncomm = None
+            sharded_native = {"ranks": world, "unavailable": comm_err or "the communicator failed on another rank"}
+    if ncomm is not None:
         nq_ids, _ = ncomm.limbs(LEVEL)
         full_d = dev_in[0][0][:, 1].contiguous()
         dl = full_d.view(torch.int64)[:, nq_ids].contiguous().view(torch.uint64) if nq_ids else None
@@ -1270,12 +1280,27 @@ def run_neo(args):
                 "batch_hrot": batch_block, "klss_vs_hybrid_setc": klss_block, "bootstrap": boot_block, "apps": apps_block,
                 "clocks": clk.summary(), "graph": bool(args.graph), "streams": args.streams,
                 "single_stream_profiled_ms_per_step": ms_step_1s, "breakdown": breakdown}
-        print(json.dumps(line), flush=True)
+        emit(line)
     if world > 1:
         dist.destroy_process_group()
 
 
+_JSON_OUT = None
+
+
+def emit(line: dict):
+    """The one JSON line, on the process's original stdout (everything else goes to stderr)."""
+    out = _JSON_OUT if _JSON_OUT is not None else sys.stdout
+    out.write(json.dumps(line) + "\n")
+    out.flush()
+
+
 def main():
+    global _JSON_OUT
+    # keep stdout to the JSON line alone: libraries (NCCL's version banner, ...) print to fd 1
+    sys.stdout.flush()
+    _JSON_OUT = os.fdopen(os.dup(1), "w")
+    os.dup2(2, 1)
     args = parse()
     if args.impl == "reference":
         run_reference(args)
