@@ -7,6 +7,8 @@
 namespace neo {
 
 // ------------------------------------------------------------------ BConv (Algorithm 1)
+// CONTROL kernel, off the default path: the CUDA-core form kept for A/B against the tcgen05
+// BConv (NEO_BCONV=cuda) and for neo_bconv's generic conversions that have no tensor-core table.
 // One thread per coefficient: y_i = [c_i qhat_i^-1]_{q_i} (Shoup), then every output
 // out_j = sum_i y_i f_ij mod t_j with y and f split in 18-bit halves so that each MAC is
 // four 32x32->64 IMADs into three 64-bit partial sums (12 inputs: < 2^41 each), followed
@@ -112,7 +114,9 @@ k_keyip(const __grid_constant__ KeyIPArgs A, int batch) {
 }
 
 // ------------------------------------------------------------------ combine (ModDown tail)
-// out_c[i] = (acc_c[i] - conv_c[i]) * P^-1 mod q_i  (+ add_c[i]); Fig. 5, Z9.
+// out_c[i] = (acc_c[i] - conv_c[i]) * P^-1 mod q_i  (+ add_c[i]); Fig. 5, Z9.  Off the
+// single-GPU path (there the tail is the NTT row pass's epilogue); used by neo_moddown_combine,
+// the limb-sharded building block.
 __global__ void __launch_bounds__(256)
 k_combine(CombineArgs A) {
     pdl_wait();
@@ -178,32 +182,6 @@ k_automorph(const u64* __restrict__ in, u64* __restrict__ out, unsigned g, int N
     }
 }
 
-// ------------------------------------------------------------------ rescale helpers (L137)
-// r[bc][i] = last[bc] mod q_i for i < l  (last < q_l < 2 q_i for equal-width primes)
-__global__ void __launch_bounds__(256)
-k_modswitch(const u64* __restrict__ last, u64* __restrict__ r, const ModQ* __restrict__ mods, int l, int N) {
-    pdl_wait();
-    const int n = blockIdx.x * blockDim.x + threadIdx.x;
-    const int i = blockIdx.y, bc = blockIdx.z;
-    if (n >= N) return;
-    const u64 q = mods[i].q;
-    u64 v = last[(size_t)bc * N + n];
-    v = v >= q ? v - q : v;
-    r[((size_t)bc * l + i) * N + n] = v;
-}
-
-// out[bc][i] = (in[bc][i] - r[bc][i]) * q_l^-1 mod q_i, in has l+1 limbs, out has l.
-__global__ void __launch_bounds__(256)
-k_rescale_combine(RescaleArgs A) {
-    pdl_wait();
-    const int n = blockIdx.x * blockDim.x + threadIdx.x;
-    const int i = blockIdx.y, bc = blockIdx.z;
-    if (n >= A.N) return;
-    const u64 q = A.mods[i].q;
-    u64 x = A.in[((size_t)bc * (A.l + 1) + i) * A.N + n];
-    u64 v = A.r[((size_t)bc * A.l + i) * A.N + n];
-    A.out[((size_t)bc * A.l + i) * A.N + n] = shoup(sub_mod(x, v, q), A.qlinv[i], q);
-}
 
 // ------------------------------------------------------------------ PMULT / HADD / PADD
 // L133-135, two coefficients per thread (16-byte accesses):
@@ -604,12 +582,6 @@ cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, 
 cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st, int batch,
                              long long in_bs, long long out_bs) {
     return launch_k(k_automorph, dim3((N + 256 * AUTO_ILP - 1) / (256 * AUTO_ILP), rows, batch), dim3(256), 0, st, in, out, g, N, in_bs, out_bs);
-}
-cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st) {
-    return launch_k(k_modswitch, dim3(g1(N).x, l, bc), dim3(256), 0, st, last, r, mods, l, N);
-}
-cudaError_t launch_rescale_combine(const RescaleArgs& A, int bc, cudaStream_t st) {
-    return launch_k(k_rescale_combine, dim3(g1(A.N).x, A.l, bc), dim3(256), 0, st, A);
 }
 
 }  // namespace neo

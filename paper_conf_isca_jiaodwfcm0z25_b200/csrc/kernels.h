@@ -37,14 +37,6 @@ struct CombineArgs {
     int limb[64];          // position -> limb id (modulus)
 };
 
-struct RescaleArgs {
-    const u64* in;         // [2B][l+1][N]
-    const u64* r;          // [2B][l][N]
-    u64* out;              // [2B][l][N]
-    const ModQ* mods;
-    int N, l;
-    TW qlinv[64];
-};
 
 // Element-wise ciphertext ops (L133-135) on [batch][2][limbs][N] ciphertexts and
 // [batch][limbs][N] plaintexts, NTT form.
@@ -127,8 +119,6 @@ cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, 
                           cudaStream_t st);
 cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st, int batch = 1,
                              long long in_bs = 0, long long out_bs = 0);
-cudaError_t launch_modswitch(const u64* last, u64* r, const ModQ* mods, int l, int N, int bc, cudaStream_t st);
-cudaError_t launch_rescale_combine(const RescaleArgs& A, int bc, cudaStream_t st);
 cudaError_t launch_pack5(const u64* in, uint32_t* lo, uint8_t* hi, size_t n, cudaStream_t st);
 cudaError_t launch_pack6(const u64* in, uint32_t* lo, uint16_t* hi, size_t n, cudaStream_t st);
 

@@ -245,19 +245,6 @@ k_klss_recover(const __grid_constant__ KlssRecArgs A) {
     }
 }
 
-// ModDown difference in coefficient form: (conv - acc_q) mod q_i, canonical.
-__global__ void __launch_bounds__(256)
-k_klss_diff(const __grid_constant__ KlssDiffArgs A) {
-    pdl_wait();
-    const int n = blockIdx.x * blockDim.x + threadIdx.x;
-    const int i = blockIdx.y, bc = blockIdx.z;
-    if (n >= A.N) return;
-    const u64 q = A.mods[i].q;
-    const size_t o = ((size_t)bc * A.Lq + i) * A.N + n;
-    const u64 a = A.rec[((size_t)bc * A.E + i) * A.N + n];      // bc = 2 b + c, position i = q_i
-    A.out[o] = sub_mod(A.conv[o], a, q);
-}
-
 cudaError_t launch_klss_ip(const KlssIpArgs& A, int batch, cudaStream_t st) {
     const dim3 g(A.N / KLSS_IP_W, A.alpha_p), blk(KLSS_IP_W, 256 / KLSS_IP_W);
     switch (A.beta) {
@@ -299,9 +286,6 @@ cudaError_t launch_klss_recover(const KlssRecArgs& A, int batch, cudaStream_t st
 #undef NEO_REC_CASE
         default: return cudaErrorInvalidValue;
     }
-}
-cudaError_t launch_klss_diff(const KlssDiffArgs& A, int batch, cudaStream_t st) {
-    return launch_k(k_klss_diff, dim3((A.N + 255) / 256, A.Lq, 2 * batch), dim3(256), 0, st, A);
 }
 
 }  // namespace neo

@@ -39,21 +39,11 @@ struct KlssRecArgs {
     int out_pos[KLSS_MAX_EXT];                // its position in PQ_l
 };
 
-// ModDown difference in coefficient form: out[b][c][i] = (conv - rec_Q) mod q_i, canonical;
-// conv [2B][Lq][N] canonical (BConv output), rec [B][2][E][N].
-struct KlssDiffArgs {
-    const u64* conv;
-    const u64* rec;
-    u64* out;                 // [2B][Lq][N]
-    const ModQ* mods;
-    int N, Lq, E;
-};
 
 cudaError_t launch_klss_ip(const KlssIpArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_klss_recover(const KlssRecArgs& A, int batch, cudaStream_t st);
 // WordSize_T = 48 variants (64-bit products; the key's hi plane holds 16 bits per residue)
 cudaError_t launch_klss_ip48(const KlssIpArgs& A, int batch, cudaStream_t st);
 cudaError_t launch_klss_recover48(const KlssRecArgs& A, int batch, cudaStream_t st);
-cudaError_t launch_klss_diff(const KlssDiffArgs& A, int batch, cudaStream_t st);
 
 }  // namespace neo
