@@ -130,7 +130,8 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
     constexpr int C = kC, NT = CF::NT;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int tid = threadIdx.x, c = tid % C, r = tid / C;
-    const int N1 = a.N1, N2 = a.N2;
+    constexpr int N1 = R * R, N2 = R * R;       // compile-time strides: immediate address offsets
+    constexpr long long NN = (long long)N1 * N2;
 
     auto stage_ptr = [&](int s) { return smem_raw + s * CF::STAGE; };
     auto issue = [&](int t, int s) {
@@ -152,7 +153,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
                 cp16(sT + CF::NS + xx * C + cc, ptab + oa + e);
                 cp16(sT + CF::NS + C * R + xx * C + cc, ptab + ob + e);
             }
-            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N + col0;
+            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * NN + col0;
             for (int e = tid; e < N1 * (C / 2); e += NT) {
                 const int row = e / (C / 2), part = e % (C / 2);
                 cp16(sD + row * C + 2 * part, src + (size_t)row * N2 + 2 * part);
@@ -167,7 +168,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
         if (STAGES == 1 && t < tm.total) {
             int b, k, blk;
             tm.decode(t, b, k, blk);
-            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N + blk * C;
+            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * NN + blk * C;
             for (int row = tid; row < N1; row += NT) pf_l2(src + (size_t)row * N2);
         }
     };
@@ -195,7 +196,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
         double* sD = reinterpret_cast<double*>(st + (CF::NS + CF::NO) * sizeof(TWD));
         double* S = sD + c * CF::XP;
         const int n2 = blk * C + c;
-        u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * a.N;
+        u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * NN;
         double x[R];
         if (FWD) {
             if (rs.in_lazy) {                              // lazy doubles (BConv outputs), |x| < 2^40
@@ -207,7 +208,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
                 for (int na = 0; na < R; ++na) x[na] = u2d(d64[(R * na + r) * C + c]);
             }
             if (rs.sub) {                                  // - sub (KLSS ModDown: conv - acc_Q), |x| < 2^40 + q
-                const u64* sr = rs.sub + b * rs.sub_bstride + (size_t)k * a.N + n2;
+                const u64* sr = rs.sub + b * rs.sub_bstride + (size_t)k * NN + n2;
                 u64 sv[R];
 #pragma unroll
                 for (int na = 0; na < R; ++na) sv[na] = __ldg(sr + (size_t)(R * na + r) * N2);
@@ -215,7 +216,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
                 for (int na = 0; na < R; ++na) x[na] = __dadd_rn(x[na], -u2d(sv[na]));
             }
             if (rs.fold) {                                 // + [c_l]_{q_i} * (P mod q_i): |x| < 2^40 + q
-                const u64* fr = rs.fold + (size_t)b * a.N + n2;
+                const u64* fr = rs.fold + (size_t)b * NN + n2;
                 u64 fv[R];
 #pragma unroll
                 for (int na = 0; na < R; ++na) fv[na] = __ldg(fr + (size_t)(R * na + r) * N2);
@@ -284,7 +285,8 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
     constexpr int RR = kC, NT = CF::NT, N2 = CF::N2;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int tid = threadIdx.x, rho = tid / R, r = tid % R;
-    const int N1 = a.N1;
+    constexpr int N1 = R * R;                   // compile-time strides: immediate address offsets
+    constexpr long long NN = (long long)N1 * N1;
 
     auto stage_ptr = [&](int s) { return smem_raw + s * CF::STAGE; };
     auto issue = [&](int t, int s) {
@@ -306,7 +308,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                 cp16(sT + d, ptab + off + e);
             }
             const int row0 = blk * RR;
-            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N;
+            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * NN;
             if (FWD) {   // 16 contiguous rows
                 const u64* g = src + (size_t)row0 * N2;
                 for (int e = tid; e < RR * N2 / 2; e += NT) cp16(sD + 2 * e, g + 2 * e);
@@ -329,15 +331,15 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
         const int row0 = blk * RR;
         if (epi_rows) {
             const int bb = b >> 1, cc = b & 1;
-            const u64* accr = ep.acc + bb * ep.acc_b + cc * ep.acc_c + (size_t)k * a.N + row0;
+            const u64* accr = ep.acc + bb * ep.acc_b + cc * ep.acc_c + (size_t)k * NN + row0;
             const u64* addr = cc ? ep.add1 : ep.add0;
             for (int i2 = tid; i2 < N2; i2 += NT) {
                 if (ep.acc) pf_l2(accr + (size_t)N1 * i2);
                 if (addr && !(cc == 0 && ep.add_galois))
-                    pf_l2(addr + bb * ep.add_b + (size_t)k * a.N + row0 + (size_t)N1 * i2);
+                    pf_l2(addr + bb * ep.add_b + (size_t)k * NN + row0 + (size_t)N1 * i2);
             }
         } else if (STAGES == 1) {
-            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * a.N;
+            const u64* src = rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * NN;
             if (FWD)
                 for (int e = tid; e < RR * N2 / 16; e += NT) pf_l2(src + (size_t)row0 * N2 + 16 * e);
             else
@@ -366,7 +368,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
         double* sD = reinterpret_cast<double*>(st + CF::NS * sizeof(TWD));
         double* S = sD + rho * CF::XP;
         const int row0 = blk * RR, i1 = row0 + rho;
-        u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * a.N;
+        u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * NN;
         double x[R];
         if (FWD) {
 #pragma unroll
@@ -394,10 +396,10 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                 const int bb = b >> 1, cc = b & 1;
                 const u64 qq = d2u(q);
                 const TW pinv = ep.pinv[k];
-                const u64* accr = ep.acc + bb * ep.acc_b + cc * ep.acc_c + (size_t)k * a.N;
+                const u64* accr = ep.acc + bb * ep.acc_b + cc * ep.acc_c + (size_t)k * NN;
                 const u64* addr = cc ? ep.add1 : ep.add0;
-                if (addr) addr += bb * ep.add_b + (size_t)k * a.N;
-                u64* outr = (cc ? ep.out1 : ep.out0) + bb * ep.out_b + (size_t)k * a.N;
+                if (addr) addr += bb * ep.add_b + (size_t)k * NN;
+                u64* outr = (cc ? ep.out1 : ep.out0) + bb * ep.out_b + (size_t)k * NN;
                 // 8 chunks of 2 coefficients per thread, in two rounds of 4 whose global loads are
                 // all issued before any of their results is used (the loads' L2 latency overlaps)
                 constexpr int U = 4;
@@ -416,7 +418,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                         dv[u] = make_uint4(0u, 0u, 0u, 0u);
                         if (addr) {
                             if (gat) {                                       // sigma_g(c0), gathered
-                                const unsigned gg = ep.add_galois, msk = (unsigned)a.N - 1;
+                                const unsigned gg = ep.add_galois, msk = (unsigned)NN - 1;
                                 const unsigned s0 = (unsigned)(((unsigned long long)gg * pos[u] + (gg - 1) / 2) & msk);
                                 const u64 x0 = __ldg(addr + s0), x1 = __ldg(addr + ((s0 + gg) & msk));
                                 dv[u] = make_uint4((unsigned)x0, (unsigned)(x0 >> 32), (unsigned)x1, (unsigned)(x1 >> 32));
@@ -453,7 +455,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                 const unsigned g = rs.galois, cst = (g - 1) / 2;
                 const unsigned ginv = rs.galois_inv_n1;
                 i1o = (int)((ginv * (unsigned)(i1 + N1 - (int)(cst & (unsigned)(N1 - 1)))) & (unsigned)(N1 - 1));
-                const unsigned s0 = (unsigned)(((unsigned long long)g * (unsigned)i1o + cst) & (unsigned long long)(a.N - 1));
+                const unsigned s0 = (unsigned)(((unsigned long long)g * (unsigned)i1o + cst) & (unsigned long long)(NN - 1));
                 const unsigned kk = s0 / (unsigned)N1;
 #pragma unroll
                 for (int ib = 0; ib < R; ++ib)
@@ -492,7 +494,8 @@ k_ntt_row_kip(NttArgs a, TileMap tm, const __grid_constant__ KipArgs A) {
     constexpr int RR = kC, NT = CF::NT, N2 = CF::N2;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int tid = threadIdx.x, rho = tid / R, r = tid % R;
-    const int N1 = a.N1, N = a.N;
+    constexpr int N1 = R * R;                   // compile-time strides
+    constexpr long long N = (long long)N1 * N1;
     TWD* sT = reinterpret_cast<TWD*>(smem_raw);
     double* sD = reinterpret_cast<double*>(smem_raw + CF::NS * sizeof(TWD));
 
