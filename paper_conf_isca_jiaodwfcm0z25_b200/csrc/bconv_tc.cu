@@ -76,7 +76,8 @@ template <bool kPre, bool kLazy, class LoadB, bool kCorr = false, int NB = 5>
 __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* IOJ, int njobs, LoadB loadB, int N,
                                               int tiles_per_entry, int batch, int exp,
                                               const CUtensorMap* tmaps = nullptr, const int* use_tmap = nullptr,
-                                              unsigned long long* dbg = nullptr) {
+                                              unsigned long long* dbg = nullptr,
+                                              const uint8_t* const* bglob = nullptr) {
     // NEO_BCONV_DBG trace of CTA 0: [i][0..3] producer in / A ready, MMA start / committed,
     // [i][4..5] epilogue part 0 start / last part end; row 60: waiting cycles per barrier
     unsigned long long wacc[6] = {0, 0, 0, 0, 0, 0};
@@ -116,10 +117,24 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     __shared__ uint64_t full_a[kAStages], empty_a[kAStages], tfull[kSlots], tempty[kSlots];
     __shared__ uint64_t in_full[kInStages], in_empty[kInStages];
     __shared__ uint32_t tmem_base;
+    __shared__ uint64_t bar_b;                           // B matrices landed (bulk copies, bglob != null)
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int G = gridDim.x;
+    unsigned long long st0 = dbg ? clock64() : 0, st1 = 0, st2 = 0;   // setup stamps (debug trace, row 61)
+    if (bglob && tid == 32 * (4 + kEpiWarps + 1)) {
+        // B matrices from device memory: one bulk copy per conversion, issued first so that they
+        // land while the rest of the setup runs (only the MMA issuer waits for them)
+        uint32_t bytes = 0;
+        for (int j = 0; j < njobs; ++j) bytes += (uint32_t)(PJ[j].nparts * kPartBytes);
+        tc::mbar_init(&bar_b, 1);
+        tc::fence_proxy_async();
+        tc::mbar_arrive_tx(&bar_b, bytes);
+        for (int j = 0, bo = 0; j < njobs; bo += PJ[j].nparts, ++j)
+            tc::bulk_g2s(sB0 + (size_t)bo * kPartBytes, bglob[j], (uint32_t)(PJ[j].nparts * kPartBytes), &bar_b);
+    }
     if (warp == 0) tc::tmem_alloc(&tmem_base, kSlots * kSlotCols);
+    if (dbg) st1 = clock64();
     if (tid == 0) {
         for (int s = 0; s < kAStages; ++s) {
             tc::mbar_init(&full_a[s], 4);                // one arrival per producer warp
@@ -134,10 +149,12 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
             tc::mbar_init(&in_empty[s], 4);
         }
     }
-    for (int j = 0, bo = 0; j < njobs; bo += PJ[j].nparts, ++j) {
-        uint4* s4 = reinterpret_cast<uint4*>(sB0 + (size_t)bo * kPartBytes);
-        const int n16 = PJ[j].nparts * (int)(kPartBytes / 16);
-        for (int e = tid; e < n16; e += kThreads) s4[e] = loadB(j, e);
+    if (!bglob) {
+        for (int j = 0, bo = 0; j < njobs; bo += PJ[j].nparts, ++j) {
+            uint4* s4 = reinterpret_cast<uint4*>(sB0 + (size_t)bo * kPartBytes);
+            const int n16 = PJ[j].nparts * (int)(kPartBytes / 16);
+            for (int e = tid; e < n16; e += kThreads) s4[e] = loadB(j, e);
+        }
     }
     if (tid < njobs) {
         const BConvTC& P = PJ[tid];
@@ -160,7 +177,14 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
+    if (dbg) st2 = clock64();
     pdl_wait();            // B matrices / TMEM / barriers were set up while the predecessor drained
+    if (dbg && blockIdx.x == 0 && tid == 0) {
+        dbg[61 * 8 + 0] = st0;
+        dbg[61 * 8 + 1] = st1;
+        dbg[61 * 8 + 2] = st2;
+        dbg[61 * 8 + 3] = clock64();
+    }
     pdl_trigger();
     const uint32_t tmem = tmem_base;
     const int total_run = (exp & 256) ? 0 : total_tiles;      // exp 256: setup/teardown only
@@ -297,6 +321,7 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         // ------------------------------------------------ MMA issuer
         if (lane == 0) {
             const uint32_t aaddr = tc::smem_u32(sA);
+            if (bglob) tc::mbar_wait(&bar_b, 0);
             int i = 0;
             for (int tile = blockIdx.x; tile < total_run; tile += G, ++i) {
                 const int s = i % kAStages, k = i / kAStages;
@@ -364,7 +389,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 k_bconv_tc_g(const __grid_constant__ BConvMulti M, int N, int tiles_per_entry, int batch, int exp) {
     auto lb = [&](int j, int e) { return reinterpret_cast<const uint4*>(M.bmat[j])[e]; };
     bconv_tc_body<kPre, kLazy, decltype(lb), kCorr, NB>(M.P, M.io, M.njobs, lb, N, tiles_per_entry, batch, exp,
-                                                       M.tmap, M.use_tmap, M.dbg);
+                                                       M.tmap, M.use_tmap, M.dbg, M.bmat);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)

@@ -40,3 +40,8 @@ for which, w in (("ModUp", 0), ("ModDown", 1)):
     print(f"  waiting cycles (span from tile 0 {span}):", {"tma in_empty": int(a[60, 0]), "prod in_full": int(a[60, 1]),
           "prod empty_a": int(a[60, 2]), "epi tfull (set 0)": int(a[60, 3]), "mma full_a": int(a[60, 4]),
           "mma tempty": int(a[60, 5])})
+    st = a[61, :4]                                   # setup stamps of CTA 0: entry, TMEM allocated, set up, past PDL wait
+    if st[0]:
+        print(f"  setup (cycles from kernel entry): TMEM alloc {int(st[1] - st[0])}, tables / barriers / B "
+              f"{int(st[2] - st[1])}, PDL wait {int(st[3] - st[2])}, to tile 0 input {int(t0 - st[3])}, "
+              f"last epilogue end {int(max(a[60, 6], a[60, 7]) - st[0])}")
