@@ -33,6 +33,7 @@ constexpr int kSlots = 2;                          // TMEM accumulator ring: 2 t
 constexpr int kSlotCols = 256;                     // a tile's parts at 48-column stride
 constexpr int kSets = 4;                           // epilogue sets of 4 warps: set e drains parts q = e (mod 4)
 constexpr int kInStages = 8;                       // TMA input ring (12 KB each)
+constexpr int kPreIn = kInStages;                  // input stages issued before the setup barrier (2: 4260 KS/s, 8: 4315-4350)
 constexpr int kEpiWarps = 4 * kSets;
 constexpr int kThreads = (4 + kEpiWarps + 2) * 32; // producers, epilogue, MMA, TMA
 constexpr size_t kInBytes = (size_t)BCTC_MAX_IN * kTileM * 8;
@@ -133,6 +134,34 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         for (int j = 0, bo = 0; j < njobs; bo += PJ[j].nparts, ++j)
             tc::bulk_g2s(sB0 + (size_t)bo * kPartBytes, bglob[j], (uint32_t)(PJ[j].nparts * kPartBytes), &bar_b);
     }
+    const int total_run = (exp & 256) ? 0 : total_tiles;      // exp 256: setup/teardown only
+    // the input ring's first stages are issued before the CTA-wide setup barrier by the TMA thread
+    // itself (its barriers initialised here), so the first tiles' HBM latency overlaps the setup
+    const int n_pre = (exp & 32) ? 0 : min(kPreIn, (total_run - (int)blockIdx.x + G - 1) / G);
+    auto issue_in = [&](int i, int s, int jb, int b, int m0, const BConvIO& io, int n_in, int use_tm, int off0) {
+        u64* dst = sIn + (size_t)s * BCTC_MAX_IN * kTileM;
+        tc::mbar_arrive_tx(&in_full[s], (uint32_t)n_in * kTileM * 8);
+        if (use_tm) {                      // one instruction for the [n_in][128] box
+            tc::tensor_g2s_3d(dst, &tmaps[jb], m0, off0, b, &in_full[s]);
+        } else {                           // each 1-D bulk copy costs ~170 issue cycles
+            const u64* in = io.in + b * io.in_bstride + m0;
+            for (int j = 0; j < n_in; ++j)
+                tc::bulk_g2s(dst + j * kTileM, in + (size_t)io.in_off[j] * N, kTileM * 8, &in_full[s]);
+        }
+    };
+    if (tid == 32 * (4 + kEpiWarps + 1)) {
+        for (int s = 0; s < kInStages; ++s) {
+            tc::mbar_init(&in_full[s], 1);
+            tc::mbar_init(&in_empty[s], 4);
+        }
+        tc::fence_proxy_async();
+        if (n_pre > 0) pdl_wait();         // the inputs are the predecessor's output
+        for (int i = 0; i < n_pre; ++i) {
+            int jb, b, m0;
+            decode(blockIdx.x + i * G, jb, b, m0);
+            issue_in(i, i, jb, b, m0, IOJ[jb], PJ[jb].n_in, use_tmap ? use_tmap[jb] : 0, IOJ[jb].in_off[0]);
+        }
+    }
     if (warp == 0) tc::tmem_alloc(&tmem_base, kSlots * kSlotCols);
     if (dbg) st1 = clock64();
     if (tid == 0) {
@@ -143,10 +172,6 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         for (int s = 0; s < kSlots; ++s) {
             tc::mbar_init(&tfull[s], 1);
             tc::mbar_init(&tempty[s], kEpiWarps);        // one arrival per epilogue warp
-        }
-        for (int s = 0; s < kInStages; ++s) {
-            tc::mbar_init(&in_full[s], 1);
-            tc::mbar_init(&in_empty[s], 4);
         }
     }
     if (!bglob) {
@@ -169,10 +194,6 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         decode(blockIdx.x + x * G, j, b, m0);
         sSched[x] = ((uint32_t)j << 28) | ((uint32_t)b << 16) | (uint32_t)(m0 / kTileM);
     }
-    for (int x = tid; x < njobs * kTgtRow; x += kThreads) {
-        const int j = x / kTgtRow, t = min(x - j * kTgtRow, PJ[j].n_out - 1);   // pad: repeat the last target
-        sTgt[x] = TgtC{PJ[j].t[t], PJ[j].tinv[t], (long long)IOJ[j].out_off[t] * N * 8, 0};
-    }
     tc::fence_proxy_async();
     tc::fence_before();
     __syncthreads();
@@ -187,7 +208,6 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     }
     pdl_trigger();
     const uint32_t tmem = tmem_base;
-    const int total_run = (exp & 256) ? 0 : total_tiles;      // exp 256: setup/teardown only
 
     if (warp < 4) {
         // ------------------------------------------------ producers
@@ -248,6 +268,13 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
         }
     } else if (warp < 4 + kEpiWarps) {
         // ------------------------------------------------ epilogue: set e drains parts q = e (mod 4)
+        // the per-target constants are staged here, off the setup's critical path (the first tile's
+        // accumulators are thousands of cycles away); named barrier 1 over the epilogue warps
+        for (int x = tid - 128; x < njobs * kTgtRow; x += 32 * kEpiWarps) {
+            const int j = x / kTgtRow, t = min(x - j * kTgtRow, PJ[j].n_out - 1);   // pad: repeat the last target
+            sTgt[x] = TgtC{PJ[j].t[t], PJ[j].tinv[t], (long long)IOJ[j].out_off[t] * N * 8, 0};
+        }
+        asm volatile("bar.sync 1, %0;\n" ::"r"(32 * kEpiWarps) : "memory");
         const int ew = warp - 4, quarter = ew & 3, e = ew >> 2;
         const int et = quarter * 32 + lane;                  // TMEM lane = A row = coefficient
         int q = 0, i = 0;                                    // part counter, tile counter of this CTA
@@ -351,22 +378,14 @@ __device__ __forceinline__ void bconv_tc_body(const BConvTC* PJ, const BConvIO* 
     } else {
         // ------------------------------------------------ TMA issuer (input ring, 7 tiles ahead)
         if (lane == 0) {
-            int i = 0;
-            for (int tile = blockIdx.x; tile < total_run && !(exp & 32); tile += G, ++i) {
+            int i = n_pre;
+            for (int tile = blockIdx.x + n_pre * G; tile < total_run && !(exp & 32); tile += G, ++i) {
                 const int s = i % kInStages, k = i / kInStages;
                 WAIT(&in_empty[s], (k & 1) ^ 1, 0);
                 int jb, b, m0;
                 tile_at(i, jb, b, m0);
                 const JobH& H = sJob[jb];
-                u64* dst = sIn + (size_t)s * BCTC_MAX_IN * kTileM;
-                tc::mbar_arrive_tx(&in_full[s], (uint32_t)H.n_in * kTileM * 8);
-                if (H.use_tmap) {                  // one instruction for the [n_in][128] box
-                    tc::tensor_g2s_3d(dst, &tmaps[jb], m0, H.in_off0, b, &in_full[s]);
-                } else {                           // each 1-D bulk copy costs ~170 issue cycles
-                    const u64* in = H.in + b * H.in_bs + m0;
-                    for (int j = 0; j < H.n_in; ++j)
-                        tc::bulk_g2s(dst + j * kTileM, in + (size_t)IOJ[jb].in_off[j] * N, kTileM * 8, &in_full[s]);
-                }
+                issue_in(i, s, jb, b, m0, IOJ[jb], H.n_in, H.use_tmap, H.in_off0);
             }
         }
         __syncwarp();
