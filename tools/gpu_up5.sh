@@ -1,0 +1,8 @@
+# 5-byte planar ModUp outputs (row pass -> KeyIP): parity and A/B
+set -x
+timeout 1800 python -m pytest tests -m gpu -q -x 2>&1 | tail -2
+Q="--steps 2000 --warmup 10 --no-cpu-baseline --no-e2e --no-hoisted --no-boot --no-apps --no-latency --batch-hrot 256"
+for v in 1 0 1 0; do
+  NEO_UP5=$v timeout 300 python bench.py $Q > gpurun_out/u5_$v.json 2>/dev/null
+  python -c "import json; d=json.load(open('gpurun_out/u5_$v.json')); b=d['breakdown']; print('up5=$v', round(d['value'],1), round(d['ms_per_step'],4), 'keyip', b['keyip']['ms_per_step'], 'ntt', b['ntt']['ms_per_step'], 'single', d['single_stream_profiled_ms_per_step'], 'B256', round(d['batch_hrot']['value']), 'hyb_setc', d['klss_vs_hybrid_setc']['hybrid_B1']['ms_per_call'])"
+done
