@@ -144,7 +144,9 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
         a.fold = fold;
         for (int k = 0; k < n; ++k) a.scale[k] = fold_w[k];
     }
-    // first pass: src -> tmp ; second pass: tmp -> dst
+    // first pass: src -> tmp ; second pass: tmp -> dst (tmp kept in L2, discarded once read: NEO_L2HINT=0 off)
+    static const int l2h = [] { const char* e = std::getenv("NEO_L2HINT"); return (e && e[0] == '0') ? 0 : 1; }();
+    a.l2hint = b.l2hint = l2h;
     a.src = src; a.src_bstride = src_bs;
     a.dst = tmp; a.dst_bstride = (long long)n * N;
     b.src = tmp; b.src_bstride = (long long)n * N;

@@ -154,6 +154,9 @@ struct RowSet {
     int has_scale;                         // inverse column pass: multiply row k by scale[k]
     unsigned galois;                       // inverse row pass: read sigma_g(src) (X -> X^g, NTT domain); 0 = none
     unsigned galois_inv_n1;                //   g^-1 mod N1
+    int l2hint = 0;                        // the pass's intermediate side (first pass: dst, second: src):
+                                           //   stores keep it in L2 (evict_last), the consumer discards its
+                                           //   lines after reading them (no write-back of dead data)
     const u64* sub = nullptr;              // forward column pass: x -= sub[b][k][n] (canonical, row k of
     long long sub_bstride = 0;             //   batch entry b at sub + b * sub_bstride + k * N), or nullptr
     const u64* fold = nullptr;             // forward column pass: x += [fold[b][n]] * scale[k] (fused

@@ -33,6 +33,17 @@ NEO_DEV void cp_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory")
 NEO_DEV void pf_l2(const void* g) { asm volatile("prefetch.global.L2 [%0];\n" ::"l"(g)); }
 template <int N>
 NEO_DEV void cp_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+// L2 residency of the pass-to-pass intermediate: evict_last stores, and a discard (invalidate
+// without write-back) of each 128-byte line once the next pass has read it
+NEO_DEV uint64_t l2_keep_policy() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;\n" : "=l"(p));
+    return p;
+}
+NEO_DEV void st_keep(double* a, double v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.f64 [%0], %1, %2;\n" ::"l"(a), "d"(v), "l"(pol) : "memory");
+}
+NEO_DEV void discard_line(const void* a) { asm volatile("discard.global.L2 [%0], 128;\n" ::"l"(a) : "memory"); }
 
 // ------------------------------------------------------------------ in-register transforms
 
@@ -234,10 +245,20 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
             cyc_dif<R>(x, CYC, q);
             const TWD ta = sA[r * C + c];
             double* dd = reinterpret_cast<double*>(dst);
+            if (rs.l2hint) {
+                const uint64_t pol = l2_keep_policy();
 #pragma unroll
-            for (int ib = 0; ib < R; ++ib)
-                dd[(size_t)(r + R * ib) * N2 + n2] = mulc(mulc(x[BitRev<R>::of(ib)], ta, q), sB[ib * C + c], q);
+                for (int ib = 0; ib < R; ++ib)
+                    st_keep(dd + (size_t)(r + R * ib) * N2 + n2, mulc(mulc(x[BitRev<R>::of(ib)], ta, q), sB[ib * C + c], q),
+                            pol);
+            } else {
+#pragma unroll
+                for (int ib = 0; ib < R; ++ib)
+                    dd[(size_t)(r + R * ib) * N2 + n2] = mulc(mulc(x[BitRev<R>::of(ib)], ta, q), sB[ib * C + c], q);
+            }
         } else {
+            if (rs.l2hint && tid < N1)                     // the intermediate's lines of this tile are dead now
+                discard_line(rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * NN + (size_t)tid * N2 + blk * C);
             TWD ta = sA[r * C + c];
             if (rs.has_scale) {                            // fold a per-row constant (e.g. qhat^-1) into the twist
                 double w = mulc(ta.w, rs.scale[k], q);
@@ -371,6 +392,9 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
         u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * NN;
         double x[R];
         if (FWD) {
+            if (rs.l2hint)                                 // the intermediate's lines of this tile are dead now
+                for (int e = tid; e < RR * N2 / 16; e += NT)
+                    discard_line(rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * NN + (size_t)row0 * N2 + 16 * e);
 #pragma unroll
             for (int na = 0; na < R; ++na) x[na] = sD[rho * N2 + R * na + r];
             cyc_dif<R>(x, CYC, q);
@@ -473,8 +497,14 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
             for (int ia = 0; ia < R; ++ia) x[ia] = S[ia + CF::EP * r];
             cyc_dif<R>(x, CYC, q);
             double* dd = reinterpret_cast<double*>(dst);
+            if (rs.l2hint) {
+                const uint64_t pol = l2_keep_policy();
 #pragma unroll
-            for (int na = 0; na < R; ++na) dd[(size_t)i1o * N2 + R * na + r] = x[BitRev<R>::of(na)];
+                for (int na = 0; na < R; ++na) st_keep(dd + (size_t)i1o * N2 + R * na + r, x[BitRev<R>::of(na)], pol);
+            } else {
+#pragma unroll
+                for (int na = 0; na < R; ++na) dd[(size_t)i1o * N2 + R * na + r] = x[BitRev<R>::of(na)];
+            }
         }
         __syncthreads();
         issue(t + STAGES * G, s);
