@@ -106,14 +106,16 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
                            u64* dst, long long dst_bs, const int* dst_off, const int* prime, int n, u64* tmp,
                            int batch, cudaStream_t st, const RowEpi* epi = nullptr, bool in_lazy = false,
                            const TWD* scale = nullptr, unsigned galois = 0, const u64* fold = nullptr,
-                           const TWD* fold_w = nullptr, const u64* sub = nullptr, long long sub_bs = 0) {
+                           const TWD* fold_w = nullptr, const u64* sub = nullptr, long long sub_bs = 0,
+                           bool src_dead = false) {
     if (n <= 0) return NEO_OK;
     if (n > NEO_MAX_ROWS) {               // more rows than one launch's descriptor holds: chunks
         if (epi || fold || sub) FAIL(NEO_EUNSUPPORTED, "too many limb rows for a fused-epilogue transform");
         for (int k0 = 0; k0 < n; k0 += NEO_MAX_ROWS) {
             const int m = std::min(NEO_MAX_ROWS, n - k0);
             neo_status s = ntt_rows(c, fwd, src, src_bs, src_off + k0, dst, dst_bs, dst_off + k0, prime + k0, m, tmp,
-                                    batch, st, nullptr, in_lazy, scale ? scale + k0 : nullptr, galois);
+                                    batch, st, nullptr, in_lazy, scale ? scale + k0 : nullptr, galois, nullptr,
+                                    nullptr, nullptr, 0, src_dead);
             if (s) return s;
         }
         return NEO_OK;
@@ -146,7 +148,10 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
     }
     // first pass: src -> tmp ; second pass: tmp -> dst (tmp kept in L2, discarded once read: NEO_L2HINT=0 off)
     static const int l2h = [] { const char* e = std::getenv("NEO_L2HINT"); return (e && e[0] == '0') ? 0 : 1; }();
-    a.l2hint = b.l2hint = l2h;
+    // evict_last only while the intermediate fits comfortably in L2 (large batched launches would
+    // pin more than the L2 holds: discard only)
+    a.l2hint = b.l2hint = l2h ? (((size_t)n * batch * N * 8 <= ((size_t)48 << 20)) ? 2 : 1) : 0;
+    a.src_dead = (src_dead && l2h) ? 1 : 0;
     a.src = src; a.src_bstride = src_bs;
     a.dst = tmp; a.dst_bstride = (long long)n * N;
     b.src = tmp; b.src_bstride = (long long)n * N;
@@ -338,7 +343,7 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
         return NEO_OK;
     }
     if ((s = ntt_rows(c, true, up, (long long)beta * E * N, so, up, (long long)beta * E * N, dof, pr, n, tmp, B, st,
-                      nullptr, c->use_tc)))
+                      nullptr, c->use_tc, nullptr, 0, nullptr, nullptr, nullptr, 0, true)))   // BConv output: dead
         return s;
 
     return NEO_OK;
@@ -439,11 +444,14 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
                 pr[n] = l;
                 sc[n++] = one;
             }
-        if ((s = ntt_rows(c, false, base, 0, so, pc, 0, dof, pr, n, tmp, 1, st, nullptr, false, sc))) return s;
+        if ((s = ntt_rows(c, false, base, 0, so, pc, 0, dof, pr, n, tmp, 1, st, nullptr, false, sc, 0, nullptr, nullptr,
+                          nullptr, 0, true)))        // acc's P and last rows, d's last rows: read only here
+            return s;
     } else {
         for (int k2 = 0; k2 < P; ++k2) { so[k2] = Lq + k2; dof[k2] = k2; pr[k2] = c->num_q + k2; }
         if ((s = ntt_rows(c, false, acc, (long long)E * N, so, pc, (long long)P * N, dof, pr, P, tmp, 2 * B, st, nullptr,
-                          false, c->use_tc ? c->moddown_tc[l].qhat_inv : nullptr)))
+                          false, c->use_tc ? c->moddown_tc[l].qhat_inv : nullptr, 0, nullptr, nullptr, nullptr, 0,
+                          true)))                    // acc's P rows: read only here
             return s;
     }
 
@@ -522,7 +530,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         ep.has_post = 1;
         for (int i = 0; i < l; ++i) { ep.pinv[i] = c->pinv[i]; ep.post[i] = c->ql_inv[l][i]; }
         return ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, l, tmp, 2 * B, st,
-                        &ep, c->use_tc, nullptr, 0, fold_fused ? accl : nullptr, F.pmod);
+                        &ep, c->use_tc, nullptr, 0, fold_fused ? accl : nullptr, F.pmod, nullptr, 0, true);
     }
 
     // a9 + a10: NTT of conv, with the ModDown tail (acc - conv) * P^-1 (+ add) fused into the
@@ -538,7 +546,7 @@ static neo_status ks_finish(const neo_ctx* c, const neo_evk* k, const u64* d, lo
         ep.add_galois = add_galois ? galois : 0;   // add0 gathered through sigma_g
         for (int i = 0; i < Lq; ++i) ep.pinv[i] = c->pinv[i];
         if ((s = ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st,
-                          &ep, c->use_tc)))
+                          &ep, c->use_tc, nullptr, 0, nullptr, nullptr, nullptr, 0, true)))   // conv: dead after
             return s;
     }
     return NEO_OK;
@@ -753,7 +761,7 @@ static neo_status klss_core(const neo_ctx* c, const neo_evk* k, const u64* d, lo
     ep.add_galois = 0;
     for (int i = 0; i < Lq; ++i) ep.pinv[i] = c->pinv[i];
     return ntt_rows(c, true, conv, (long long)Lq * N, so, conv, (long long)Lq * N, dof, pr, Lq, tmp, 2 * B, st, &ep,
-                    false, nullptr, 0, nullptr, nullptr, rec, (long long)E * N);
+                    false, nullptr, 0, nullptr, nullptr, rec, (long long)E * N, true);
 }
 
 static neo_status ks_core(const neo_ctx* c, const neo_evk* k, const u64* d, long long d_bs, int l, int B,

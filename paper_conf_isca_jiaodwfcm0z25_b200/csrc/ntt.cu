@@ -210,6 +210,8 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
         u64* dst = rs.dst + b * rs.dst_bstride + (size_t)rs.dst_off[k] * NN;
         double x[R];
         if (FWD) {
+            if (rs.src_dead && tid < N1)                   // a dead source (BConv output): drop its lines
+                discard_line(rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * NN + (size_t)tid * N2 + blk * C);
             if (rs.in_lazy) {                              // lazy doubles (BConv outputs), |x| < 2^40
 #pragma unroll
                 for (int na = 0; na < R; ++na) x[na] = sD[(R * na + r) * C + c];
@@ -245,7 +247,7 @@ k_ntt_col(RowSet rs, NttArgs a, TileMap tm) {
             cyc_dif<R>(x, CYC, q);
             const TWD ta = sA[r * C + c];
             double* dd = reinterpret_cast<double*>(dst);
-            if (rs.l2hint) {
+            if (rs.l2hint == 2) {
                 const uint64_t pol = l2_keep_policy();
 #pragma unroll
                 for (int ib = 0; ib < R; ++ib)
@@ -470,6 +472,9 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
                 }
             }
         } else {
+            if (rs.src_dead)                               // a dead source (KeyIP's P rows): drop its lines
+                for (int i2 = tid; i2 < N2; i2 += NT)
+                    discard_line(rs.src + b * rs.src_bstride + (size_t)rs.src_off[k] * NN + row0 + (size_t)N1 * i2);
             const u64* T = reinterpret_cast<const u64*>(sD);
             int i1o = i1;                                  // row of tmp this thread's row lands in
             if (rs.galois) {
@@ -497,7 +502,7 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
             for (int ia = 0; ia < R; ++ia) x[ia] = S[ia + CF::EP * r];
             cyc_dif<R>(x, CYC, q);
             double* dd = reinterpret_cast<double*>(dst);
-            if (rs.l2hint) {
+            if (rs.l2hint == 2) {
                 const uint64_t pol = l2_keep_policy();
 #pragma unroll
                 for (int na = 0; na < R; ++na) st_keep(dd + (size_t)i1o * N2 + R * na + r, x[BitRev<R>::of(na)], pol);
