@@ -107,7 +107,7 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
                            int batch, cudaStream_t st, const RowEpi* epi = nullptr, bool in_lazy = false,
                            const TWD* scale = nullptr, unsigned galois = 0, const u64* fold = nullptr,
                            const TWD* fold_w = nullptr, const u64* sub = nullptr, long long sub_bs = 0,
-                           bool src_dead = false) {
+                           bool src_dead = false, bool dst_keep = false) {
     if (n <= 0) return NEO_OK;
     if (n > NEO_MAX_ROWS) {               // more rows than one launch's descriptor holds: chunks
         if (epi || fold || sub) FAIL(NEO_EUNSUPPORTED, "too many limb rows for a fused-epilogue transform");
@@ -152,6 +152,8 @@ static neo_status ntt_rows(const neo_ctx* c, bool fwd, const u64* src, long long
     // pin more than the L2 holds: discard only)
     a.l2hint = b.l2hint = l2h ? (((size_t)n * batch * N * 8 <= ((size_t)48 << 20)) ? 2 : 1) : 0;
     a.src_dead = (src_dead && l2h) ? 1 : 0;
+    static const bool keep = [] { const char* e = std::getenv("NEO_UPKEEP"); return !(e && e[0] == '0'); }();
+    b.dst_keep = (keep && dst_keep && fwd && !epi && l2h && (size_t)n * batch * N * 8 <= ((size_t)64 << 20)) ? 1 : 0;
     a.src = src; a.src_bstride = src_bs;
     a.dst = tmp; a.dst_bstride = (long long)n * N;
     b.src = tmp; b.src_bstride = (long long)n * N;
@@ -343,7 +345,8 @@ static neo_status ks_modup(const neo_ctx* c, const u64* d, long long d_bs, int l
         return NEO_OK;
     }
     if ((s = ntt_rows(c, true, up, (long long)beta * E * N, so, up, (long long)beta * E * N, dof, pr, n, tmp, B, st,
-                      nullptr, c->use_tc, nullptr, 0, nullptr, nullptr, nullptr, 0, true)))   // BConv output: dead
+                      nullptr, c->use_tc, nullptr, 0, nullptr, nullptr, nullptr, 0, true,    // BConv output: dead
+                      true)))                                                               // KeyIP reads up next
         return s;
 
     return NEO_OK;

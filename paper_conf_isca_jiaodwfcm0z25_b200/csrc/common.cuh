@@ -154,6 +154,8 @@ struct RowSet {
     int has_scale;                         // inverse column pass: multiply row k by scale[k]
     unsigned galois;                       // inverse row pass: read sigma_g(src) (X -> X^g, NTT domain); 0 = none
     unsigned galois_inv_n1;                //   g^-1 mod N1
+    int dst_keep = 0;                      // second (row) pass, no epilogue: the output is read again soon
+                                           //   (the ModUp rows KeyIP reads next): stored L2 evict_last
     int src_dead = 0;                      // first pass: the source rows are dead once read (a BConv output,
                                            //   KeyIP's P rows): their L2 lines are discarded, no write-back
     int l2hint = 0;                        // the pass's intermediate side (first pass: dst, second: src):

@@ -412,7 +412,16 @@ k_ntt_row(RowSet rs, NttArgs a, TileMap tm, const __grid_constant__ RowEpi ep) {
 #pragma unroll
             for (int ib = 0; ib < R; ++ib) T[swz(r + R * ib, rho)] = d2u(canon(x[BitRev<R>::of(ib)], q, qinv));
             __syncthreads();
-            if (!EPI) {
+            if (!EPI && rs.dst_keep) {
+                const uint64_t pol = l2_keep_policy();
+                for (int e = tid; e < N2 * 8; e += NT) {
+                    const int i2 = e >> 3, p = e & 7;
+                    const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
+                    asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;\n"
+                                 ::"l"(dst + row0 + (size_t)N1 * i2 + 2 * p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w),
+                                   "l"(pol) : "memory");
+                }
+            } else if (!EPI) {
                 for (int e = tid; e < N2 * 8; e += NT) {
                     const int i2 = e >> 3, p = e & 7;
                     const uint4 v = *reinterpret_cast<const uint4*>(T + i2 * 16 + ((p ^ (i2 & 7)) << 1));
