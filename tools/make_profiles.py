@@ -77,7 +77,14 @@ def traffic(rnd, full):
                       "dram_read": r["dram_read"] + c["dram_read"], "dram_write": r["dram_write"] + c["dram_write"],
                       "dur_us_cold": round(r["dur_us_cold"] + c["dur_us_cold"], 3),
                       "source": f"profiles/{rnd}_ncu_full_top_kernels.jsonl (ncu --set full, --clock-control none)"}
-    json.dump(out, open(os.path.join(ROOT, "profiles", "ncu_traffic.json"), "w"), indent=1)
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:                                              # keep entries other tools added (warm-cache captures)
+        old = json.load(open(path))
+        for k, v in old.items():
+            out.setdefault(k, v)
+    except Exception:
+        pass
+    json.dump(out, open(path, "w"), indent=1)
 
 
 def main():
