@@ -207,7 +207,9 @@ neo_status neo_hrot(const neo_ctx* ctx, const neo_evk* rotkey, uint32_t galois_e
  * ciphertext: the automorphism is applied after ModDown instead of before ModUp).
  * keys[r] must come from neo_evk_create_hoisted (which stores sigma_{g^-1}(evk) once).
  * ct_in [batch][2][level+1][N]; ct_out [n_rot][batch][2][level+1][N];
- * ws >= neo_workspace_size(ctx, NEO_OP_HROT_HOISTED, level, batch). */
+ * ws >= neo_workspace_size(ctx, NEO_OP_HROT_HOISTED, level, batch) (two ModDown areas: the odd
+ * rotations run on the context's internal side stream, forked from and joined back into `stream`
+ * by events -- asynchronous and graph-capturable; NEO_TWO_STREAM=0 at process start: one stream). */
 neo_status neo_evk_create_hoisted(const neo_ctx* ctx, const uint64_t* evk, uint32_t galois_elt,
                                   neo_evk** out);
 neo_status neo_hrot_hoisted(const neo_ctx* ctx, const neo_evk* const* keys, int32_t n_rot,
@@ -221,7 +223,9 @@ neo_status neo_hrot_hoisted(const neo_ctx* ctx, const neo_evk* const* keys, int3
  * neo_hrot calls (a different, equally valid ciphertext: ModDown's floor rounding is applied once).
  * keys[k]: neo_evk_create rotation keys (KSGen(s, sigma_{g_k}(s)), L184); galois[k] odd < 2N;
  * cts: host array of n device pointers, each [batch][2][level+1][N]; ct_out likewise, not
- * aliasing any input; 1 <= n <= 64; ws >= neo_workspace_size(ctx, NEO_OP_HROT_SUM, level, batch). */
+ * aliasing any input; 1 <= n <= 64; ws >= neo_workspace_size(ctx, NEO_OP_HROT_SUM, level, batch)
+ * (two ModUp areas: the ModUps of odd k run on the context's internal side stream, joined back
+ * into `stream`; the KeyIP sums stay on `stream` in order). */
 neo_status neo_hrot_sum(const neo_ctx* ctx, const neo_evk* const* keys, const uint32_t* galois, int32_t n,
                         const uint64_t* const* cts, int32_t level, uint64_t* ct_out, int32_t batch, void* ws,
                         size_t ws_bytes, neo_stream_t stream);
