@@ -155,6 +155,46 @@ k_tensor(const u64* __restrict__ cta, const u64* __restrict__ ctb, u64* __restri
     d[ob + 2 * cs] = mul_mod(a1, b1, m);
 }
 
+// Two coefficients per thread with 16-byte accesses; d2 (the key-switch input, read by the INTT
+// that follows) is stored L2 evict_last.
+__global__ void __launch_bounds__(256)
+k_tensor2(const u64* __restrict__ cta, const u64* __restrict__ ctb, u64* __restrict__ d,
+          const ModQ* __restrict__ mods, int limbs, int N) {
+    pdl_wait();
+    const int n = 2 * (blockIdx.x * blockDim.x + threadIdx.x);
+    const int i = blockIdx.y, b = blockIdx.z;
+    if (n >= N) return;
+    const ModQ m = mods[i];
+    const size_t cs = (size_t)limbs * N;
+    const size_t base = (size_t)b * 2 * cs + (size_t)i * N + n;
+    const ulonglong2 A0 = __ldg(reinterpret_cast<const ulonglong2*>(cta + base));
+    const ulonglong2 A1 = __ldg(reinterpret_cast<const ulonglong2*>(cta + base + cs));
+    const ulonglong2 B0 = __ldg(reinterpret_cast<const ulonglong2*>(ctb + base));
+    const ulonglong2 B1 = __ldg(reinterpret_cast<const ulonglong2*>(ctb + base + cs));
+    const size_t ob = (size_t)b * 3 * cs + (size_t)i * N + n;
+    ulonglong2 r0, r1, r2;
+    r0.x = mul_mod(A0.x, B0.x, m);
+    r0.y = mul_mod(A0.y, B0.y, m);
+    {
+        u64 h = 0, l = 0;
+        mac128(h, l, A0.x, B1.x);
+        mac128(h, l, A1.x, B0.x);
+        r1.x = barrett_reduce(h, l, m);
+        h = 0; l = 0;
+        mac128(h, l, A0.y, B1.y);
+        mac128(h, l, A1.y, B0.y);
+        r1.y = barrett_reduce(h, l, m);
+    }
+    r2.x = mul_mod(A1.x, B1.x, m);
+    r2.y = mul_mod(A1.y, B1.y, m);
+    *reinterpret_cast<ulonglong2*>(d + ob) = r0;
+    *reinterpret_cast<ulonglong2*>(d + ob + cs) = r1;
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;\n" : "=l"(pol));
+    asm volatile("st.global.L2::cache_hint.v2.u64 [%0], {%1, %2}, %3;\n" ::"l"(d + ob + 2 * cs), "l"(r2.x), "l"(r2.y),
+                 "l"(pol) : "memory");
+}
+
 // ------------------------------------------------------------------ automorphism (AUTO)
 // out[i] = in[(g i + (g-1)/2) mod N]: X -> X^g in the natural-order NTT domain.
 #ifndef AUTO_ILP
@@ -577,6 +617,9 @@ cudaError_t launch_combine(const CombineArgs& A, int limbs, int batch, cudaStrea
 }
 cudaError_t launch_tensor(const u64* a, const u64* b, u64* d, const ModQ* mods, int limbs, int N, int batch,
                           cudaStream_t st) {
+    static const bool two = [] { const char* e = std::getenv("NEO_TENSOR2"); return !(e && e[0] == '0'); }();
+    if (two && (N % 512) == 0)
+        return launch_k(k_tensor2, dim3(N / 512, limbs, batch), dim3(256), 0, st, a, b, d, mods, limbs, N);
     return launch_k(k_tensor, dim3(g1(N).x, limbs, batch), dim3(256), 0, st, a, b, d, mods, limbs, N);
 }
 cudaError_t launch_automorph(const u64* in, u64* out, unsigned g, int N, int rows, cudaStream_t st, int batch,
